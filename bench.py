@@ -1,0 +1,356 @@
+"""Benchmark of the tiled heat path.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl tiles|reference]
+                    [--config c2|c1|c4] [--T STEPS] [--nstreams S]
+
+One bench "step" = one pass of the whole hot path over one batch of input:
+T heat steps over every tile of the workload (C2 by default: 512^3 fp64,
+8^3 tiles of 64^3, ghost 1, 4 streams, T = 10, periodic, alpha = 0.125).
+
+  value  Gcell-updates/s with the grid already resident in HBM (tile_run of T
+         steps; ghost fill fused into the stencil).
+  e2e    the same metric through the public C API from pinned host memory:
+         tile_invalidate -> tile_run(T) -> tile_sync, i.e. H2D of every tile,
+         T steps, D2H of every tile inside the timed region.
+
+Timing: CUDA events recorded by libtiles on its own streams (tile_timer_*),
+barrier + synchronize on both sides, max over ranks. Inputs (2 x 1.07 GB per
+GPU) are larger than the 126 MB L2. N > 1: weak scaling, each rank owns a
+512^3 z-slab of a 512 x 512 x 512N grid, halos over NCCL.
+"""
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    # name: (per-GPU dims, tile dims, T, nstreams, description)
+    "c1": ((64, 64, 64), (32, 32, 32), 10, 2, "C1 heat fp64 64^3, 2x2x2 tiles, g=1, T=10, 2 streams"),
+    "c2": ((512, 512, 512), (64, 64, 64), 10, 4,
+           "C2 heat fp64 512^3, 8^3 tiles (64^3 cells), g=1, resident in HBM, T=10, 4 streams"),
+}
+ALPHA = 0.125
+METRIC = "Gcell-updates/s incl. H2D/D2H at 1/2/4/8 B200; % transfer time hidden"
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rk = int(os.environ.get("RANK", "0"))
+    lr = int(os.environ.get("LOCAL_RANK", str(rk)))
+    return ws, rk, lr
+
+
+class Clocks:
+    """nvidia-smi sampler for the timed region (B200_PROFILING.md clocks line)."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu):
+        self.gpu, self.rows, self.p = gpu, [], None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.p = None
+        return self
+
+    def _read(self):
+        for line in self.p.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) == 7:
+                self.rows.append(parts)
+
+    def __exit__(self, *a):
+        if self.p:
+            self.p.terminate()
+            try:
+                self.p.wait(2)
+            except Exception:
+                self.p.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = sorted(float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit())
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in self.rows:
+            for n, v in zip(names, r[3:]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": sm[len(sm) // 2] if sm else None,
+                "sm_max_mhz": float(self.rows[0][1]) if self.rows[0][1].replace(".", "").isdigit() else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        j = json.load(open(p))
+        return float(j["hbm_gbs"]), "MEASURED_PEAKS.json hbm_gbs (measured)"
+    return 6650.0, "B200_PROFILING.md fallback 6.65 TB/s"
+
+
+def pcie_bandwidth(torch, nbytes=256 << 20, reps=5):
+    h = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
+    d = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    out = {}
+    for k in ("h2d", "d2h"):
+        best = 0
+        for _ in range(reps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            d.copy_(h, non_blocking=True) if k == "h2d" else h.copy_(d, non_blocking=True)
+            e1.record()
+            torch.cuda.synchronize()
+            best = max(best, nbytes / (e0.elapsed_time(e1) / 1e3) / 1e9)
+        out[k] = best
+    return out
+
+
+def traffic_from_profile(cfg):
+    p = os.path.join(ROOT, "profiles", "heat7_ncu_traffic.json")
+    if os.path.exists(p):
+        j = json.load(open(p))
+        return j.get(cfg)
+    return None
+
+
+def cpu_oracle_time(n, T):
+    import oracle
+    import synth
+    u = np.empty((n, n, n))
+    synth.fill_uniform_native(u.ctypes.data, n, n, n, 0, n, 0, n, 0, n, 42)
+    t0 = time.perf_counter()
+    oracle.heat_c(u, ALPHA, T)
+    return time.perf_counter() - t0
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as it stands, 1 host core."""
+    ws, rk, _ = dist_env()
+    if rk != 0:
+        return 0
+    dims, td, T, ns, desc = CONFIGS[args.config]
+    n = 192 if args.config == "c2" else dims[0]   # bounded sample per step
+    for _ in range(args.warmup):
+        cpu_oracle_time(n, T)
+    t = sum(cpu_oracle_time(n, T) for _ in range(args.steps))
+    val = n ** 3 * T * args.steps / t / 1e9
+    sample = f"{n}^3 grid x T={T} per step (untiled fp64 Jacobi, oracle/heat_oracle.c, 1 thread)"
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "Gcell-updates/s", "n_gpus": ws,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": desc, "sample": sample},
+            "cpu_baseline": {"value": val, "unit": "Gcell-updates/s", "cores": 1, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": val, "unit": "Gcell-updates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="tiles", choices=["tiles", "reference"])
+    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
+    ap.add_argument("--T", type=int, default=None)
+    ap.add_argument("--nstreams", type=int, default=None)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-extras", action="store_true", help="skip sync-baseline / overlap legs")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_icpp_bastemuzas17_b200 import tiles as Tl
+    import synth
+
+    ws, rk, lr = dist_env()
+    torch.cuda.set_device(lr)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", lr))
+    dims, td, T, ns, desc = CONFIGS[args.config]
+    T = args.T if args.T is not None else T
+    ns = args.nstreams or ns
+    nx, ny, nzl = dims
+    gdims = (nx, ny, nzl * ws)
+    cells = nx * ny * nzl  # per rank
+
+    nid = None
+    if ws > 1:
+        obj = [Tl.nccl_unique_id() if rk == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        nid = obj[0]
+
+    def barrier():
+        if ws > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def max_over_ranks(x):
+        if ws == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    u0 = np.empty((nzl, ny, nx))
+    synth.fill_uniform_native(u0.ctypes.data, gdims[0], gdims[1], gdims[2], rk * nzl, nzl, 0, ny, 0, nx, 42)
+    dom = Tl.Domain(gdims, td, ghost=1, device=lr, nranks=ws, rank=rk, nccl_id=nid)
+    dom.load(u0)
+    del u0
+    k = Tl.heat7(ALPHA)
+
+    # ---- device-resident value -------------------------------------------
+    dom.run(k, 1, ns)
+    dom.sync()
+    for _ in range(args.warmup):
+        dom.run(k, T, ns)
+    dom.sync()
+    dom.set_kernel_timing(True)
+    dom.reset_stats()
+    barrier()
+    with Clocks(lr) as clk:
+        dom.timer_start()
+        for _ in range(args.steps):
+            dom.run(k, T, ns)
+        ms = dom.timer_stop()
+    st = dom.stats()
+    dom.set_kernel_timing(False)
+    ms = max_over_ranks(ms)
+    value = ws * cells * T * args.steps / (ms / 1e3) / 1e9
+    launches = st["n_kernels"]
+    avg_kernel_ms = st["kernel_ms"] / max(1, st["kernel_timed"])
+    cells_per_launch = cells * T * args.steps / max(1, st["kernel_timed"])
+    dom.sync()
+
+    # ---- end-to-end from pinned host memory ---------------------------------
+    def e2e_leg(mode=Tl.TILE_MEASURE_NORMAL, steps=args.steps, warm=1):
+        dom.set_measure(mode)
+        for _ in range(warm):
+            dom.invalidate()
+            dom.run(k, T, ns)
+            dom.sync()
+        dom.reset_stats()
+        barrier()
+        tot = 0.0
+        for _ in range(steps):
+            dom.invalidate()
+            dom.timer_start()
+            dom.run(k, T, ns)
+            dom.sync()
+            tot += dom.timer_stop()
+        s = dom.stats()
+        dom.set_measure(Tl.TILE_MEASURE_NORMAL)
+        return max_over_ranks(tot), s
+
+    with Clocks(lr) as clk_e2e:
+        e2e_ms, st_e2e = e2e_leg()
+    e2e_val = ws * cells * T * args.steps / (e2e_ms / 1e3) / 1e9
+    h2d_b = st_e2e["bytes_h2d"] // args.steps
+    d2h_b = st_e2e["bytes_d2h"] // args.steps
+
+    extras = {}
+    if not args.no_extras:
+        xo_ms, _ = e2e_leg(Tl.TILE_MEASURE_XFER_ONLY, steps=2)
+        co_ms, _ = e2e_leg(Tl.TILE_MEASURE_COMP_ONLY, steps=2)
+        wall = e2e_ms / args.steps
+        xo, co = xo_ms / 2, co_ms / 2
+        hidden = max(0.0, min(1.0, (xo + co - wall) / min(xo, co)))
+        bw = pcie_bandwidth(torch)
+        B = cells * 8
+        t_link = B / (bw["h2d"] * 1e9) + B / (bw["d2h"] * 1e9)   # dependency form, SURVEY §8(d)
+        hbm_peak, _ = measured_peaks()
+        t_hbm = T * 16 * cells / (hbm_peak * 1e9)
+        R = max(t_link, t_hbm)
+        extras = {"overlap": {"hidden_frac": hidden, "t_wall_ms": wall, "t_xfer_only_ms": xo,
+                              "t_comp_only_ms": co,
+                              "definition": "(T_xfer_only + T_comp_only - T_wall) / min(...)"},
+                  "e2e_roofline": {"bound": "pcie (dependency form)", "t_link_ms": t_link * 1e3,
+                                   "t_hbm_ms": t_hbm * 1e3, "frac": R / (wall / 1e3),
+                                   "pcie_gbs": bw}}
+        if ws == 1:
+            dom.free()
+            sdom = Tl.Domain(gdims, td, ghost=1, device=lr, sched="sync")
+            u0 = np.empty((nzl, ny, nx))
+            synth.fill_uniform_native(u0.ctypes.data, gdims[0], gdims[1], gdims[2], 0, nzl, 0, ny, 0, nx, 42)
+            sdom.load(u0)
+            del u0
+            sdom.run(k, T, 1)
+            sdom.sync()
+            tot = 0.0
+            for _ in range(2):
+                sdom.invalidate()
+                sdom.timer_start()
+                sdom.run(k, T, 1)
+                sdom.sync()
+                tot += sdom.timer_stop()
+            sdom.free()
+            extras["sync_baseline_e2e"] = {"value": cells * T * 2 / (tot / 1e3) / 1e9,
+                                           "unit": "Gcell-updates/s",
+                                           "schedule": "H2D all, T steps, D2H all, one stream"}
+    try:
+        dom.free()
+    except Exception:
+        pass
+
+    peak, peak_src = measured_peaks()
+    algo_bytes = 16.0 * cells_per_launch
+    achieved = algo_bytes / (avg_kernel_ms / 1e3) / 1e9
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+            "traffic": traffic_from_profile(args.config), "kernel": "heat7_tma",
+            "algorithmic_bytes_per_launch": algo_bytes, "avg_launch_ms": avg_kernel_ms,
+            "peak_source": peak_src}
+
+    cpu = None
+    if rk == 0 and ws == 1 and not args.no_cpu_baseline:
+        n = 384 if args.config == "c2" else dims[0]
+        t = cpu_oracle_time(n, T)
+        cpu = {"value": n ** 3 * T / t / 1e9, "unit": "Gcell-updates/s", "cores": 1, "kind": "oracle",
+               "sample": f"{n}^3 grid x T={T} (untiled Jacobi, oracle/heat_oracle.c, 1 thread)"}
+
+    if rk == 0:
+        clocks = clk.summary()
+        line = {"metric": METRIC, "value": value, "unit": "Gcell-updates/s", "n_gpus": ws,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic",
+                "config": {"workload": desc, "dims_per_gpu": dims, "global_dims": gdims, "tile_dims": td,
+                           "ghost": 1, "T": T, "nstreams": ns, "bc": "periodic", "alpha": ALPHA,
+                           "parallelism": f"z-slab x{ws}" if ws > 1 else "1 GPU",
+                           "l2": "inputs larger than L2 (2 x 1.07 GB per GPU per step)",
+                           "value_def": "grid resident in HBM; T steps of tile_run",
+                           "e2e_def": "tile_invalidate + tile_run(T) + tile_sync from pinned host"},
+                "e2e": {"value": e2e_val, "unit": "Gcell-updates/s", "h2d_bytes_per_step": h2d_b,
+                        "d2h_bytes_per_step": d2h_b, "ms_per_step": e2e_ms / args.steps},
+                "gpu_launches": launches, "roofline": roof, "cpu_baseline": cpu, "clocks": clocks,
+                "clocks_e2e": clk_e2e.summary()}
+        line.update(extras)
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,259 @@
+/* tiles.h — C ABI of libtiles (B200-native tiled, stream-pipelined fp64 heat
+ * stencil and compute-intensive kernel; Bastem et al., "Overlapping Data
+ * Transfers with Computation on GPU with Tiles", ICPP 2017).
+ *
+ * Citations "P:L<n> §<s>" refer to the paper text (PAPER.md line n, section s).
+ *
+ * Model (§III, §IV.A): the grid is decomposed into regions
+ * ("tiles") that are both the transfer unit and the execution unit. Each
+ * tile's data lives in pinned host memory; as many tiles as fit are
+ * placed on the device and the rest are streamed through a
+ * pool of device slots, with transfers queued on CUDA streams so that they
+ * overlap computation on other tiles. Ghost cells of a
+ * tile are refreshed from its neighbours before each step.
+ *
+ * Conventions for every function:
+ *  - Return TILE_OK (0) on success, otherwise a tile_status code; the
+ *    thread-local message is available through tile_last_error().
+ *  - TILE_EINVAL never has side effects.
+ *  - A CUDA or NCCL failure (TILE_ECUDA / TILE_ENCCL) POISONS the domain:
+ *    every later call except tile_free returns TILE_ESTATE.
+ *  - A domain is used from one host thread at a time.
+ *  - Grids are fp64, C order [z][y][x] with x fastest. Sizes are int64.
+ *  - Ownership: the library owns every pinned host buffer and device buffer
+ *    it allocates. Arrays passed to tile_load / tile_store are borrowed for
+ *    the duration of the call only. A caller-provided device pool or stream
+ *    list (e.g. from PyTorch) is borrowed for the domain's lifetime and never
+ *    freed by the library.
+ *  - Multi-GPU (nranks > 1): z-slab decomposition; create / run / sync /
+ *    free are COLLECTIVE (every rank calls them with identical global dims,
+ *    tile_dims, ghost, kernel and steps); load / store move the rank's own
+ *    slab. Halo planes travel between z-neighbour ranks via NCCL.
+ */
+#ifndef TILES_H
+#define TILES_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct tile_domain tile_domain; /* opaque, library-owned */
+
+typedef enum {
+  TILE_OK = 0,
+  TILE_EINVAL = 1,        /* bad argument (no side effects) */
+  TILE_ENOMEM_HOST = 2,   /* pinned host allocation failed */
+  TILE_ENOMEM_DEVICE = 3, /* device budget below the minimum slot count */
+  TILE_ECUDA = 4,         /* CUDA runtime error (domain poisoned) */
+  TILE_ENCCL = 5,         /* NCCL error (domain poisoned) */
+  TILE_ESTATE = 6,        /* poisoned domain, or call not valid in this state */
+  TILE_ENOSYS = 7         /* feature not compiled in (e.g. NCCL) */
+} tile_status;
+
+/* Boundary condition of the global grid (the paper is silent, R3). */
+typedef enum { TILE_BC_PERIODIC = 0, TILE_BC_DIRICHLET = 1 } tile_bc;
+
+typedef enum {
+  /* 7-point Jacobi heat step, "uses its 6 nearest neighbors" (§VI.A):
+   * v = u + alpha*(((xm+xp)+(ym+yp))+(zm+zp) - 6u)   (R1) */
+  TILE_KERNEL_HEAT7 = 1,
+  /* compute-intensive kernel, listing P:L219-L224 §VI.B: per cell,
+   * inner_iters times: s=sin(x); c=cos(x); x=x+sqrt(s*s+c*c) */
+  TILE_KERNEL_SINCOS = 2
+} tile_kernel_kind;
+
+typedef struct {
+  tile_kernel_kind kind;
+  double alpha;        /* HEAT7: dt/dx^2, must be in (0, 1/6] (stability) */
+  int32_t inner_iters; /* SINCOS: kernel_iteration of P:L220 (>= 0) */
+} tile_kernel;
+
+/* Schedules. AUTO picks RESIDENT when every tile fits in the
+ * device budget twice (old/new buffers; once for SINCOS), else STREAM. */
+typedef enum {
+  TILE_SCHED_AUTO = 0,
+  TILE_SCHED_RESIDENT = 1, /* all tiles in HBM, z-layer batches, events */
+  TILE_SCHED_STREAM = 2,   /* out-of-core: per-tile slots, eviction */
+  TILE_SCHED_SYNC = 3      /* synchronous baseline: H2D all, T steps, D2H all,
+                              one stream, no overlap (Fig. 5 comparison) */
+} tile_sched;
+
+/* Measurement-only knobs (SURVEY.md §8(d) overlap efficiency): results of a
+ * run in these modes are NOT valid and must not be checked. */
+typedef enum {
+  TILE_MEASURE_NORMAL = 0,
+  TILE_MEASURE_XFER_ONLY = 1, /* issue every copy/event, launch no kernel */
+  TILE_MEASURE_COMP_ONLY = 2  /* skip every host<->device copy */
+} tile_measure;
+
+typedef struct {
+  int32_t device;               /* CUDA ordinal; -1 = current device */
+  tile_bc bc;                   /* default TILE_BC_PERIODIC */
+  uint64_t device_budget_bytes; /* 0: cudaMemGetInfo free - reserve;
+                                   >0: hard cap, the paper's "limiting GPU
+                                   memory" method */
+  void* device_pool;            /* optional caller-owned device region ... */
+  uint64_t device_pool_bytes;   /* ... and its size; borrowed, never freed */
+  void* const* streams;         /* optional caller-owned cudaStream_t list */
+  int32_t nstreams_provided;    /* number of entries in `streams` */
+  int32_t nranks, rank;         /* z-slab decomposition; 1, 0 = single GPU */
+  const void* nccl_unique_id;   /* 128 bytes, identical on all ranks (the
+                                   caller broadcasts it, e.g. torch.distributed) */
+  tile_sched sched;             /* default TILE_SCHED_AUTO */
+  int32_t dry_run;              /* 1: no CUDA calls at all; the scheduler
+                                   records its op trace (tests on CPU) */
+  int32_t fuse_pointwise_steps; /* SINCOS: 1 (default) = all T steps of a tile
+                                   in one residency pass (tile-major); 0 =
+                                   step-major, every step re-streams (Fig. 8) */
+} tile_options;
+
+typedef struct {
+  uint64_t bytes_h2d, bytes_d2h, bytes_halo; /* payload moved */
+  uint64_t n_h2d, n_d2h, n_kernels, n_halo;  /* operations issued */
+  uint64_t hits, misses, evictions, writebacks;
+  uint64_t steps_done;                       /* cell-update steps completed */
+  double last_run_ms;                        /* host wall time of last tile_run..sync */
+  double kernel_ms;                          /* summed device time of timed kernel launches */
+  uint64_t kernel_timed;                     /* number of timed kernel launches */
+} tile_stats;
+
+typedef struct {
+  int64_t dims[3];        /* global grid (nx, ny, nz) */
+  int64_t local_dims[3];  /* this rank's slab */
+  int64_t tile_dims[3];
+  int64_t tiles[3];       /* tiles per axis on this rank */
+  int64_t ntiles;
+  int64_t z_offset;       /* global z of the slab's first plane */
+  int32_t ghost;
+  int32_t nslots;         /* device interior buffers */
+  int32_t sched;          /* schedule chosen for the last/next run */
+  int32_t resident;       /* 1 if every tile currently has a valid device copy */
+  uint64_t device_bytes;  /* device memory carved by the domain */
+  uint64_t host_bytes;    /* pinned host memory of the tile store */
+} tile_info;
+
+/* One entry of the dry-run trace. */
+typedef enum {
+  TILE_OP_H2D = 1,      /* host tile a -> slot b */
+  TILE_OP_D2H = 2,      /* slot b -> host tile a */
+  TILE_OP_KERNEL = 3,   /* tile a: slot b -> slot c, face parity d (reads d, writes d^1) */
+  TILE_OP_RECORD = 4,   /* event a recorded on stream */
+  TILE_OP_WAIT = 5,     /* stream waits on event a */
+  TILE_OP_FACES_H2D = 6,/* upload all host-extracted faces into parity d */
+  TILE_OP_EXTRACT = 7,  /* tile a in slot b: export its faces into parity d */
+  TILE_OP_HALO = 8,     /* slab halo exchange of parity d */
+  TILE_OP_DROP = 9,     /* tile a leaves slot b without a copy (clean) */
+  TILE_OP_HIT = 10,     /* tile a found in slot b (P:L90 cache hit) */
+  TILE_OP_POINTWISE = 11 /* compute-intensive kernel on tile a in slot b, c iterations */
+} tile_op_kind;
+
+typedef struct {
+  int32_t kind;   /* tile_op_kind */
+  int32_t stream;
+  int64_t a, b, c, d;
+} tile_op;
+
+/* Create a domain: decomposition (tiles = dims / tile_dims per axis), ghost
+ * bookkeeping, pinned host tile store, device budget and slots.
+ *  dims:      global grid (nx, ny, nz), each >= 1
+ *  tile_dims: cells per tile per axis; must divide dims (ragged tiles are
+ *             rejected, R6); tile_dims[0] and [1] must be even
+ *             (128-bit vector access), and for nranks > 1 tile_dims[2] must
+ *             divide nz / nranks.
+ *  ghost:     ghost-cell width g, 1 <= g <= min(tile_dims) (HEAT7 reads the
+ *             innermost layer; g is the width reported by tile_ghost_map).
+ *  opt:       NULL = defaults (periodic, auto budget, 1 rank, own streams).
+ * Errors: EINVAL, ENOMEM_HOST, ENOMEM_DEVICE, ECUDA, ENCCL, ENOSYS. */
+tile_status tile_domain_create(const int64_t dims[3], const int64_t tile_dims[3],
+                               int32_t ghost, const tile_options* opt,
+                               tile_domain** out);
+
+/* Copy the rank's dense slab into the pinned tile-blocked store (regions are
+ * "physically separated"). PERIODIC: src is [nz_local][ny][nx].
+ * DIRICHLET: src is [nz_local+2][ny+2][nx+2] including the fixed 1-deep halo
+ * (the stencil radius), whose values are never updated. Invalidates device
+ * copies. Implies tile_sync first if a run is in flight. */
+tile_status tile_load(tile_domain* dom, const double* src);
+
+/* Pointer to tile `tile_id`'s interior in the pinned host store (contiguous
+ * [tz][ty][tx], x fastest), to fill or read it in place without a dense
+ * staging array. Valid until tile_free. Writing through it requires a
+ * following tile_mark_host_dirty. */
+tile_status tile_host_tile(tile_domain* dom, int64_t tile_id, double** ptr);
+tile_status tile_mark_host_dirty(tile_domain* dom);
+
+/* Enqueue `steps` steps of kernel k over every tile (no sync
+ * after issue). nstreams in [1, 64] streams carry transfers and kernels
+ * (P:L81-L84). Returns once all work is enqueued; may block only for
+ * residency back-pressure. Host data is not valid until tile_sync. */
+tile_status tile_run(tile_domain* dom, const tile_kernel* k, int32_t steps,
+                     int32_t nstreams);
+
+/* Write back every dirty device tile (D2H) and wait for all streams; the host
+ * store is then current (D2H needs synchronization). */
+tile_status tile_sync(tile_domain* dom);
+
+/* tile_sync, then copy the host store into the dense slab dst (same shape as
+ * tile_load's src; DIRICHLET: only the interior of dst is written). */
+tile_status tile_store(tile_domain* dom, double* dst);
+
+/* Drop every device copy without a transfer (host store must be current,
+ * i.e. after tile_sync); the next tile_run re-streams all tiles from host. */
+tile_status tile_invalidate(tile_domain* dom);
+
+/* Ghost-source map of one tile over its full expanded box (tz+2g, ty+2g,
+ * tx+2g), z-major then y, x fastest: the GLOBAL linear index (z*ny+y)*nx+x
+ * of the cell each position holds after periodic wrap, or -1 for a Dirichlet
+ * boundary cell; interior cells map to themselves. out_len
+ * must be >= (tz+2g)(ty+2g)(tx+2g). tile_id is rank-local. */
+tile_status tile_ghost_map(const tile_domain* dom, int64_t tile_id, int64_t* out,
+                           int64_t out_len);
+
+/* Face-source descriptors actually used by the kernels: for tile tile_id and
+ * each face f in (x-, x+, y-, y+, z-, z+), out[2f] = kind (0 = neighbour tile
+ * export on this rank, 1 = Dirichlet fixed face, 2 = slab halo from rank
+ * below, 3 = slab halo from rank above) and out[2f+1] = the neighbour's
+ * rank-local tile id (kind 0) or the tile's position in its z-layer. */
+tile_status tile_face_sources(const tile_domain* dom, int64_t tile_id, int64_t out[12]);
+
+tile_status tile_get_info(const tile_domain* dom, tile_info* out);
+tile_status tile_get_stats(const tile_domain* dom, tile_stats* out);
+tile_status tile_reset_stats(tile_domain* dom);
+
+/* Measurement mode (tile_measure) for subsequent runs. */
+tile_status tile_set_measure(tile_domain* dom, int32_t mode);
+
+/* Device-side timing. tile_timer_start joins every stream of the domain into
+ * its first stream and records a timing event there; tile_timer_stop joins
+ * again, records a second event, synchronizes and returns the elapsed device
+ * milliseconds in *ms. With tile_set_kernel_timing(dom, 1) every kernel
+ * launch is bracketed by events on its own stream and the summed durations
+ * are reported in tile_stats.kernel_ms / kernel_timed after tile_sync or
+ * tile_timer_stop. */
+tile_status tile_timer_start(tile_domain* dom);
+tile_status tile_timer_stop(tile_domain* dom, double* ms);
+tile_status tile_set_kernel_timing(tile_domain* dom, int32_t on);
+
+/* Dry-run trace: number of recorded ops, and copy of up to cap entries. */
+tile_status tile_trace(const tile_domain* dom, tile_op* out, int64_t cap, int64_t* n);
+tile_status tile_trace_clear(tile_domain* dom);
+
+/* Release everything (implies tile_sync unless poisoned). NULL is a no-op. */
+tile_status tile_free(tile_domain* dom);
+
+/* Thread-local description of the last error (never NULL). */
+const char* tile_last_error(void);
+
+/* Fill out[128] with a fresh ncclUniqueId (call on rank 0, then broadcast).
+ * TILE_ENOSYS if built without NCCL. */
+tile_status tile_nccl_unique_id(void* out128);
+
+/* Library version string. */
+const char* tile_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TILES_H */

@@ -1,0 +1,173 @@
+// domain.cpp — tile decomposition, ghost-source bookkeeping and host-side
+// face extraction (CPU only; no CUDA).
+//
+// Regions are "partitions of data ... physically separated in memory"
+// (§IV.A), "expanded to accommodate ghost cells" (§III). The paper
+// computes ghost source/destination indices on the host; here
+// they are computed once per domain as 6 face descriptors per tile, because
+// the decomposition is static (difference D2).
+#include <algorithm>
+#include <thread>
+
+#include "runtime.hpp"
+
+namespace tiles {
+
+Status make_err(tile_status c, const std::string& m) {
+  Status s;
+  s.code = c;
+  s.msg = m;
+  return s;
+}
+
+Status make_geometry(const int64_t dims[3], const int64_t td[3], int ghost, tile_bc bc,
+                     int nranks, int rank, Geometry* out) {
+  Geometry G{};
+  for (int a = 0; a < 3; ++a) {
+    if (dims[a] < 1 || td[a] < 1) return make_err(TILE_EINVAL, "dims and tile_dims must be >= 1");
+    G.g[a] = dims[a];
+    G.t[a] = td[a];
+  }
+  if (nranks < 1 || rank < 0 || rank >= nranks)
+    return make_err(TILE_EINVAL, "need 0 <= rank < nranks");
+  if (dims[2] % nranks) return make_err(TILE_EINVAL, "nz must be divisible by nranks");
+  G.l[0] = dims[0];
+  G.l[1] = dims[1];
+  G.l[2] = dims[2] / nranks;
+  G.zoff = G.l[2] * rank;
+  for (int a = 0; a < 3; ++a) {
+    if (G.l[a] % td[a])
+      return make_err(TILE_EINVAL,
+                      "dims (per rank) must be multiples of tile_dims (ragged tiles rejected)");
+    G.n[a] = G.l[a] / td[a];
+  }
+  if ((td[0] & 1) || (td[1] & 1))
+    return make_err(TILE_EINVAL, "tile_dims x and y must be even (128-bit vector access)");
+  const int64_t tmin = std::min(td[0], std::min(td[1], td[2]));
+  if (ghost < 1 || ghost > tmin) return make_err(TILE_EINVAL, "need 1 <= ghost <= min(tile_dims)");
+  if (bc != TILE_BC_PERIODIC && bc != TILE_BC_DIRICHLET) return make_err(TILE_EINVAL, "bad bc");
+  G.ghost = ghost;
+  G.bc = bc;
+  G.nranks = nranks;
+  G.rank = rank;
+  G.ntiles = G.n[0] * G.n[1] * G.n[2];
+  G.tile_elems = td[0] * td[1] * td[2];
+  G.face_elems[XM] = G.face_elems[XP] = td[2] * td[1];
+  G.face_elems[YM] = G.face_elems[YP] = td[2] * td[0];
+  G.face_elems[ZM] = G.face_elems[ZP] = td[1] * td[0];
+  G.layer_tiles = G.n[0] * G.n[1];
+  *out = G;
+  return Status::ok();
+}
+
+FaceSrc face_source(const Geometry& G, int64_t id, int f) {
+  int64_t c[3];
+  G.tile_coords(id, &c[0], &c[1], &c[2]);
+  const int axis = f / 2;
+  const int dir = (f & 1) ? +1 : -1;
+  int64_t nc[3] = {c[0], c[1], c[2]};
+  nc[axis] += dir;
+  const bool inside = nc[axis] >= 0 && nc[axis] < G.n[axis];
+  if (inside) return {0, G.tile_id(nc[0], nc[1], nc[2])};
+  if (axis < 2 || G.nranks == 1) {
+    // global boundary along x / y, or along z on a single rank
+    if (G.bc == TILE_BC_DIRICHLET) return {1, id};
+    nc[axis] = (nc[axis] + G.n[axis]) % G.n[axis];
+    return {0, G.tile_id(nc[0], nc[1], nc[2])};
+  }
+  // slab seam along z
+  const int64_t pos = c[1] * G.n[0] + c[0];
+  if (dir < 0) {
+    if (G.rank == 0 && G.bc == TILE_BC_DIRICHLET) return {1, id};
+    return {2, pos};
+  }
+  if (G.rank == G.nranks - 1 && G.bc == TILE_BC_DIRICHLET) return {1, id};
+  return {3, pos};
+}
+
+void ghost_map(const Geometry& G, int64_t id, int64_t* out) {
+  int64_t c[3];
+  G.tile_coords(id, &c[0], &c[1], &c[2]);
+  const int64_t g = G.ghost;
+  const int64_t ex = G.t[0] + 2 * g, ey = G.t[1] + 2 * g, ez = G.t[2] + 2 * g;
+  const int64_t ox = c[0] * G.t[0], oy = c[1] * G.t[1], oz = G.zoff + c[2] * G.t[2];
+  int64_t* o = out;
+  for (int64_t k = 0; k < ez; ++k) {
+    const int64_t z = oz + k - g;
+    for (int64_t j = 0; j < ey; ++j) {
+      const int64_t y = oy + j - g;
+      for (int64_t i = 0; i < ex; ++i) {
+        const int64_t x = ox + i - g;
+        const bool out_of = x < 0 || x >= G.g[0] || y < 0 || y >= G.g[1] || z < 0 || z >= G.g[2];
+        if (out_of && G.bc == TILE_BC_DIRICHLET) {
+          *o++ = -1;
+          continue;
+        }
+        const int64_t wx = (x % G.g[0] + G.g[0]) % G.g[0];
+        const int64_t wy = (y % G.g[1] + G.g[1]) % G.g[1];
+        const int64_t wz = (z % G.g[2] + G.g[2]) % G.g[2];
+        *o++ = (wz * G.g[1] + wy) * G.g[0] + wx;
+      }
+    }
+  }
+}
+
+void host_parallel_for(int64_t n, const std::function<void(int64_t, int64_t)>& fn) {
+  unsigned hw = std::thread::hardware_concurrency();
+  int64_t nt = std::max<int64_t>(1, std::min<int64_t>(hw ? hw : 4, n));
+  if (nt == 1) {
+    fn(0, n);
+    return;
+  }
+  std::vector<std::thread> th;
+  for (int64_t i = 0; i < nt; ++i) {
+    int64_t b = n * i / nt, e = n * (i + 1) / nt;
+    th.emplace_back([&fn, b, e] { fn(b, e); });
+  }
+  for (auto& t : th) t.join();
+}
+
+// Export every tile's boundary layers from the host store (layouts as the
+// device faces: x-faces [z][y], y-faces [z][x], z-faces [y][x]).
+void host_extract_faces(const Geometry& G, const double* host, double* const faces[6]) {
+  const int64_t tx = G.t[0], ty = G.t[1], tz = G.t[2];
+  host_parallel_for(G.ntiles, [&](int64_t b, int64_t e) {
+    for (int64_t k = b; k < e; ++k) {
+      const double* u = host + k * G.tile_elems;
+      double* fxm = faces[XM] + k * G.face_elems[XM];
+      double* fxp = faces[XP] + k * G.face_elems[XP];
+      double* fym = faces[YM] + k * G.face_elems[YM];
+      double* fyp = faces[YP] + k * G.face_elems[YP];
+      double* fzm = faces[ZM] + k * G.face_elems[ZM];
+      double* fzp = faces[ZP] + k * G.face_elems[ZP];
+      for (int64_t z = 0; z < tz; ++z)
+        for (int64_t y = 0; y < ty; ++y) {
+          const double* row = u + (z * ty + y) * tx;
+          fxm[z * ty + y] = row[0];
+          fxp[z * ty + y] = row[tx - 1];
+        }
+      for (int64_t z = 0; z < tz; ++z) {
+        std::copy(u + (z * ty) * tx, u + (z * ty) * tx + tx, fym + z * tx);
+        std::copy(u + (z * ty + ty - 1) * tx, u + (z * ty + ty - 1) * tx + tx, fyp + z * tx);
+      }
+      std::copy(u, u + ty * tx, fzm);
+      std::copy(u + (tz - 1) * ty * tx, u + tz * ty * tx, fzp);
+    }
+  });
+}
+
+const double* Domain::face_src_ptr(int64_t id, int f, int parity) const {
+  const FaceSrc s = face_source(G, id, f);
+  switch (s.kind) {
+    case 0:
+      return faces[f ^ 1][parity] + s.val * G.face_elems[f ^ 1];
+    case 1:
+      return dir_faces[f] + id * G.face_elems[f];
+    case 2:
+      return halo[0][parity] + s.val * G.face_elems[ZM];
+    default:
+      return halo[1][parity] + s.val * G.face_elems[ZP];
+  }
+}
+
+}  // namespace tiles

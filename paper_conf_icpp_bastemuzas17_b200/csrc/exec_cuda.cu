@@ -1,0 +1,323 @@
+// exec_cuda.cu — the CUDA executor: maps the scheduler's operations onto
+// CUDA streams, events, cudaMemcpyAsync from pinned memory
+// and the sm_100a kernels of kernels.cu. No CPU fallback exists: every
+// compute operation is a kernel launch.
+#include <cstdio>
+#include <cstring>
+
+#include "runtime.hpp"
+
+namespace tiles {
+namespace {
+
+Status cuda_err(cudaError_t e, const char* what) {
+  char buf[256];
+  std::snprintf(buf, sizeof buf, "%s: %s", what, cudaGetErrorString(e));
+  return make_err(TILE_ECUDA, buf);
+}
+#define CK(call)                                  \
+  do {                                            \
+    cudaError_t e_ = (call);                      \
+    if (e_ != cudaSuccess) return cuda_err(e_, #call); \
+  } while (0)
+
+struct CudaExec final : Exec {
+  int dev = 0;
+  int sms = 148;
+  int heat_occ = 1;
+  std::vector<cudaStream_t> streams;
+  std::vector<char> own_stream;
+  std::vector<cudaEvent_t> events;
+  std::vector<cudaEvent_t> tpool;                 // timing events (free list)
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> tpending;
+  cudaEvent_t t_begin = nullptr, t_end = nullptr;
+
+  Status timing_event(cudaEvent_t* e) {
+    if (!tpool.empty()) {
+      *e = tpool.back();
+      tpool.pop_back();
+      return Status::ok();
+    }
+    CK(cudaEventCreate(e));
+    return Status::ok();
+  }
+  // bracket a kernel launch with timing events on its stream
+  template <class F>
+  Status timed(Domain& d, int st, F&& launch) {
+    if (!d.kernel_timing) {
+      CK(launch());
+      return Status::ok();
+    }
+    cudaEvent_t a, b;
+    Status r = timing_event(&a);
+    if (r.bad()) return r;
+    r = timing_event(&b);
+    if (r.bad()) return r;
+    CK(cudaEventRecord(a, S(st)));
+    CK(launch());
+    CK(cudaEventRecord(b, S(st)));
+    tpending.push_back({a, b});
+    return Status::ok();
+  }
+  Status collect(Domain& d) {  // after a synchronize
+    for (auto& pr : tpending) {
+      float ms = 0;
+      CK(cudaEventElapsedTime(&ms, pr.first, pr.second));
+      d.stats.kernel_ms += ms;
+      d.stats.kernel_timed++;
+      tpool.push_back(pr.first);
+      tpool.push_back(pr.second);
+    }
+    tpending.clear();
+    return Status::ok();
+  }
+  Status join_into0(Domain& d) {
+    for (size_t i = 1; i < streams.size(); ++i) {
+      CK(cudaEventRecord(events[(size_t)(d.ev_misc_base + 4 + i)], streams[i]));
+      CK(cudaStreamWaitEvent(streams[0], events[(size_t)(d.ev_misc_base + 4 + i)], 0));
+    }
+    return Status::ok();
+  }
+  Status timer_start(Domain& d) override {
+    if (!t_begin) CK(cudaEventCreate(&t_begin));
+    if (!t_end) CK(cudaEventCreate(&t_end));
+    Status r = join_into0(d);
+    if (r.bad()) return r;
+    CK(cudaEventRecord(t_begin, streams[0]));
+    // later work on any stream starts after t_begin
+    for (size_t i = 1; i < streams.size(); ++i) CK(cudaStreamWaitEvent(streams[i], t_begin, 0));
+    return Status::ok();
+  }
+  Status timer_stop(Domain& d, double* ms) override {
+    Status r = join_into0(d);
+    if (r.bad()) return r;
+    CK(cudaEventRecord(t_end, streams[0]));
+    CK(cudaEventSynchronize(t_end));
+    float f = 0;
+    CK(cudaEventElapsedTime(&f, t_begin, t_end));
+    *ms = f;
+    r = sync_all(d);
+    if (r.bad()) return r;
+    return Status::ok();
+  }
+
+  cudaStream_t S(int i) { return streams[(size_t)i]; }
+
+  Status h2d(Domain& d, int64_t t0, int64_t n, int s0, int st) override {
+    if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
+    const size_t bytes = (size_t)n * d.G.tile_elems * 8;
+    CK(cudaMemcpyAsync(d.slot_ptr(s0), d.host_tile(t0), bytes, cudaMemcpyHostToDevice, S(st)));
+    d.stats.bytes_h2d += bytes;
+    d.stats.n_h2d++;
+    return Status::ok();
+  }
+  Status d2h(Domain& d, int64_t t0, int64_t n, int s0, int st) override {
+    if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
+    const size_t bytes = (size_t)n * d.G.tile_elems * 8;
+    CK(cudaMemcpyAsync(d.host_tile(t0), d.slot_ptr(s0), bytes, cudaMemcpyDeviceToHost, S(st)));
+    d.stats.bytes_d2h += bytes;
+    d.stats.n_d2h++;
+    return Status::ok();
+  }
+  Status record(Domain&, int ev, int st) override {
+    CK(cudaEventRecord(events[(size_t)ev], S(st)));
+    return Status::ok();
+  }
+  Status wait(Domain&, int ev, int st) override {
+    CK(cudaStreamWaitEvent(S(st), events[(size_t)ev], 0));
+    return Status::ok();
+  }
+  Status heat(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
+              const TileItem* dev_items, int st) override {
+    if (d.measure == TILE_MEASURE_XFER_ONLY || n == 0) return Status::ok();
+    HeatParams p{};
+    p.tx = (int)d.G.t[0];
+    p.ty = (int)d.G.t[1];
+    p.tz = (int)d.G.t[2];
+    p.band = d.band;
+    p.nbands = p.ty / d.band;
+    p.nitems = n;
+    p.alpha = d.kernel_alpha;
+    if (dev_items) {
+      p.items = dev_items;
+    } else {
+      if (n > kMaxInlineItems) return make_err(TILE_ESTATE, "internal: too many inline items");
+      p.items = nullptr;
+      for (int i = 0; i < n; ++i)
+        p.inline_items[i] = {d.slot_ptr(in[i]), d.slot_ptr(out[i]), (int32_t)tiles[i], 0};
+    }
+    p.gsrc = d.gsrc_dev[rp];
+    for (int f = 0; f < 6; ++f) {
+      p.fexp[f] = d.faces[f][rp ^ 1];
+      p.face_elems[f] = d.G.face_elems[f];
+    }
+    // persistent grid: one wave of CTAs, >= 4 planes each
+    const int64_t planes = (int64_t)n * p.nbands * p.tz;
+    int64_t grid = (int64_t)sms * heat_occ;
+    grid = std::max<int64_t>(1, std::min<int64_t>(grid, (planes + 3) / 4));
+    Status r = timed(d, st, [&] { return launch_heat7(p, d.stages, d.heat_smem, (int)grid, S(st)); });
+    if (r.bad()) return r;
+    d.stats.n_kernels++;
+    return Status::ok();
+  }
+  Status sincos(Domain& d, int64_t t, int slot, int64_t iters, int st) override {
+    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
+    SincosParams p{};
+    p.tile_elems = d.G.tile_elems;
+    p.nitems = 1;
+    p.iters = iters;
+    p.items = nullptr;
+    p.inline_items[0] = {d.slot_ptr(slot), d.slot_ptr(slot), (int32_t)t, 0};
+    const int64_t pairs = d.G.tile_elems / 2;
+    int64_t grid = std::min<int64_t>((pairs + 255) / 256, (int64_t)sms * 8);
+    Status r = timed(d, st, [&] { return launch_sincos(p, (int)std::max<int64_t>(1, grid), S(st)); });
+    if (r.bad()) return r;
+    d.stats.n_kernels++;
+    return Status::ok();
+  }
+  Status extract(Domain& d, int64_t t0, int64_t n, int s0, int par, const TileItem* dev_items,
+                 int st) override {
+    if (d.measure == TILE_MEASURE_XFER_ONLY || n == 0) return Status::ok();
+    ExtractParams p{};
+    p.tx = (int)d.G.t[0];
+    p.ty = (int)d.G.t[1];
+    p.tz = (int)d.G.t[2];
+    p.nitems = (int)n;
+    if (dev_items) {
+      p.items = dev_items;
+    } else {
+      if (n > kMaxInlineItems) return make_err(TILE_ESTATE, "internal: too many inline items");
+      for (int64_t i = 0; i < n; ++i)
+        p.inline_items[i] = {d.slot_ptr(s0 + (int)i), nullptr, (int32_t)(t0 + i), 0};
+    }
+    for (int f = 0; f < 6; ++f) {
+      p.fexp[f] = d.faces[f][par];
+      p.face_elems[f] = d.G.face_elems[f];
+    }
+    CK(launch_extract(p, S(st)));
+    d.stats.n_kernels++;
+    return Status::ok();
+  }
+  Status faces_h2d(Domain& d, int par, int st) override {
+    if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
+    for (int f = 0; f < 6; ++f) {
+      const size_t bytes = (size_t)d.G.ntiles * d.G.face_elems[f] * 8;
+      CK(cudaMemcpyAsync(d.faces[f][par], d.host_faces[f], bytes, cudaMemcpyHostToDevice, S(st)));
+      d.stats.bytes_h2d += bytes;
+      d.stats.n_h2d++;
+    }
+    return Status::ok();
+  }
+  Status halo(Domain& d, int par, int st) override {
+    Status r = nccl_halo(d, par, S(st));
+    if (r.bad()) return r;
+    d.stats.n_halo++;
+    return Status::ok();
+  }
+  Status note(Domain&, int, int64_t, int64_t, int) override { return Status::ok(); }
+  Status sync_all(Domain& d) override {
+    for (auto s : streams) CK(cudaStreamSynchronize(s));
+    return collect(d);
+  }
+  Status mem_info(Domain&, uint64_t* fr, uint64_t* tot) override {
+    size_t f = 0, t = 0;
+    CK(cudaMemGetInfo(&f, &t));
+    *fr = f;
+    *tot = t;
+    return Status::ok();
+  }
+  Status alloc_host(Domain&, uint64_t bytes, void** p) override {
+    // pinned (page-locked) host regions, P:L73 (cudaMallocHost)
+    cudaError_t e = cudaHostAlloc(p, bytes ? bytes : 1, cudaHostAllocPortable);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return make_err(TILE_ENOMEM_HOST, std::string("cudaHostAlloc: ") + cudaGetErrorString(e));
+    }
+    return Status::ok();
+  }
+  void free_host(Domain&, void* p) override { cudaFreeHost(p); }
+  Status alloc_device(Domain&, uint64_t bytes, void** p) override {
+    cudaError_t e = cudaMalloc(p, bytes);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return make_err(TILE_ENOMEM_DEVICE, std::string("cudaMalloc: ") + cudaGetErrorString(e));
+    }
+    return Status::ok();
+  }
+  void free_device(Domain&, void* p) override { cudaFree(p); }
+
+  Status setup(Domain& d) override {
+    const int nst = d.halo_stream + 1;
+    streams.assign((size_t)nst, nullptr);
+    own_stream.assign((size_t)nst, 0);
+    for (int i = 0; i < nst; ++i) {
+      if (i < d.opt.nstreams_provided && d.opt.streams && d.opt.streams[i]) {
+        streams[(size_t)i] = static_cast<cudaStream_t>(d.opt.streams[i]);
+      } else {
+        CK(cudaStreamCreateWithFlags(&streams[(size_t)i], cudaStreamNonBlocking));
+        own_stream[(size_t)i] = 1;
+      }
+    }
+    events.assign((size_t)d.nevents, nullptr);
+    for (auto& e : events) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    // events start "completed": record each once on stream 0
+    for (auto& e : events) CK(cudaEventRecord(e, streams[0]));
+    for (int p = 0; p < 2; ++p) {
+      CK(cudaMemcpy(d.gsrc_dev[p], d.gsrc_host[p].data(), d.gsrc_host[p].size() * sizeof(void*),
+                    cudaMemcpyHostToDevice));
+      if (d.mode == MODE_RESIDENT)
+        CK(cudaMemcpy(d.items_dev[p], d.items_host[p].data(),
+                      d.items_host[p].size() * sizeof(TileItem), cudaMemcpyHostToDevice));
+    }
+    CK(heat_configure((int)d.G.t[0], (int)d.G.t[1], d.band, d.stages, d.heat_smem, &heat_occ));
+    if (heat_occ < 1) return make_err(TILE_EINVAL, "heat kernel cannot be resident on an SM");
+    CK(cudaStreamSynchronize(streams[0]));
+    return Status::ok();
+  }
+  Status upload_dir(Domain& d) override {
+    for (int f = 0; f < 6; ++f)
+      CK(cudaMemcpy(d.dir_faces[f], d.host_dir[f], (size_t)d.G.ntiles * d.G.face_elems[f] * 8,
+                    cudaMemcpyHostToDevice));
+    return Status::ok();
+  }
+  void destroy(Domain&) override {
+    for (auto& pr : tpending) {
+      tpool.push_back(pr.first);
+      tpool.push_back(pr.second);
+    }
+    tpending.clear();
+    for (auto e : tpool) cudaEventDestroy(e);
+    tpool.clear();
+    if (t_begin) cudaEventDestroy(t_begin);
+    if (t_end) cudaEventDestroy(t_end);
+    for (auto e : events)
+      if (e) cudaEventDestroy(e);
+    for (size_t i = 0; i < streams.size(); ++i)
+      if (own_stream[i] && streams[i]) cudaStreamDestroy(streams[i]);
+    events.clear();
+    streams.clear();
+  }
+};
+
+}  // namespace
+
+Exec* make_cuda_exec(Domain& d, Status* st) {
+  auto* x = new CudaExec();
+  int dev = d.opt.device;
+  cudaError_t e = cudaSuccess;
+  if (dev < 0) e = cudaGetDevice(&dev);
+  if (e == cudaSuccess) e = cudaSetDevice(dev);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&x->sms, cudaDevAttrMultiProcessorCount, dev);
+  if (e != cudaSuccess) {
+    *st = cuda_err(e, "device setup (is a CUDA device visible?)");
+    delete x;
+    return nullptr;
+  }
+  x->dev = dev;
+  d.device = dev;
+  d.sm_count = x->sms;
+  *st = Status::ok();
+  return x;
+}
+
+}  // namespace tiles

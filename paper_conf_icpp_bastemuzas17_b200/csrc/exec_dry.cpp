@@ -1,0 +1,121 @@
+// exec_dry.cpp — dry-run executor: no CUDA call at all; every operation the
+// scheduler issues is appended to the domain's op trace (tile_trace), so the
+// residency protocol and the dependency structure can be checked on a CPU.
+#include <cstdlib>
+#include <cstring>
+
+#include "runtime.hpp"
+
+namespace tiles {
+namespace {
+
+struct DryExec final : Exec {
+  void put(Domain& d, int kind, int stream, int64_t a, int64_t b, int64_t c, int64_t dd) {
+    tile_op op;
+    op.kind = kind;
+    op.stream = stream;
+    op.a = a;
+    op.b = b;
+    op.c = c;
+    op.d = dd;
+    d.trace.push_back(op);
+  }
+  Status h2d(Domain& d, int64_t t0, int64_t n, int s0, int st) override {
+    d.stats.bytes_h2d += (uint64_t)n * d.G.tile_elems * 8;
+    d.stats.n_h2d++;
+    put(d, TILE_OP_H2D, st, t0, s0, n, 0);
+    return Status::ok();
+  }
+  Status d2h(Domain& d, int64_t t0, int64_t n, int s0, int st) override {
+    d.stats.bytes_d2h += (uint64_t)n * d.G.tile_elems * 8;
+    d.stats.n_d2h++;
+    put(d, TILE_OP_D2H, st, t0, s0, n, 0);
+    return Status::ok();
+  }
+  Status record(Domain& d, int ev, int st) override {
+    put(d, TILE_OP_RECORD, st, ev, 0, 0, 0);
+    return Status::ok();
+  }
+  Status wait(Domain& d, int ev, int st) override {
+    put(d, TILE_OP_WAIT, st, ev, 0, 0, 0);
+    return Status::ok();
+  }
+  Status heat(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
+              const TileItem* dev_items, int st) override {
+    d.stats.n_kernels++;
+    if (dev_items) {  // resident batch: items are a slice of items_host[bit]
+      const int bit = dev_items >= d.items_dev[1] && d.items_dev[1] ? 1 : 0;
+      const int64_t k0 = dev_items - d.items_dev[bit];
+      for (int i = 0; i < n; ++i) {
+        const TileItem& it = d.items_host[bit][(size_t)(k0 + i)];
+        const int is = (int)((it.in - d.slot_base) / d.G.tile_elems);
+        const int os = (int)((it.out - d.slot_base) / d.G.tile_elems);
+        put(d, TILE_OP_KERNEL, st, it.tile, is, os, rp);
+      }
+    } else {
+      for (int i = 0; i < n; ++i) put(d, TILE_OP_KERNEL, st, tiles[i], in[i], out[i], rp);
+    }
+    return Status::ok();
+  }
+  Status sincos(Domain& d, int64_t t, int slot, int64_t iters, int st) override {
+    d.stats.n_kernels++;
+    put(d, TILE_OP_POINTWISE, st, t, slot, iters, 0);
+    return Status::ok();
+  }
+  Status extract(Domain& d, int64_t t0, int64_t n, int s0, int par, const TileItem*,
+                 int st) override {
+    d.stats.n_kernels++;
+    for (int64_t i = 0; i < n; ++i) put(d, TILE_OP_EXTRACT, st, t0 + i, s0 + i, 0, par);
+    return Status::ok();
+  }
+  Status faces_h2d(Domain& d, int par, int st) override {
+    for (int f = 0; f < 6; ++f) d.stats.bytes_h2d += (uint64_t)d.G.ntiles * d.G.face_elems[f] * 8;
+    put(d, TILE_OP_FACES_H2D, st, 0, 0, 0, par);
+    return Status::ok();
+  }
+  Status halo(Domain& d, int par, int st) override {
+    d.stats.n_halo++;
+    d.stats.bytes_halo += 2ull * d.G.layer_tiles * d.G.face_elems[ZM] * 8;
+    put(d, TILE_OP_HALO, st, 0, 0, 0, par);
+    return Status::ok();
+  }
+  Status note(Domain& d, int kind, int64_t a, int64_t b, int st) override {
+    put(d, kind, st, a, b, 0, 0);
+    return Status::ok();
+  }
+  Status sync_all(Domain&) override { return Status::ok(); }
+  Status mem_info(Domain& d, uint64_t* fr, uint64_t* tot) override {
+    // a pretend device: the budget option (or 64 GiB) is all there is
+    *tot = 180ull << 30;
+    *fr = d.opt.device_budget_bytes ? d.opt.device_budget_bytes + (1ull << 30) : (64ull << 30);
+    return Status::ok();
+  }
+  Status alloc_host(Domain&, uint64_t bytes, void** p) override {
+    *p = std::malloc(bytes ? bytes : 1);
+    if (!*p) return make_err(TILE_ENOMEM_HOST, "host allocation failed");
+    return Status::ok();
+  }
+  void free_host(Domain&, void* p) override { std::free(p); }
+  Status alloc_device(Domain&, uint64_t, void** p) override {
+    *p = reinterpret_cast<void*>(uintptr_t(1) << 40);  // never dereferenced
+    return Status::ok();
+  }
+  void free_device(Domain&, void*) override {}
+  Status setup(Domain&) override { return Status::ok(); }
+  Status upload_dir(Domain& d) override {
+    put(d, TILE_OP_FACES_H2D, 0, 1, 0, 0, -1);
+    return Status::ok();
+  }
+  void destroy(Domain&) override {}
+  Status timer_start(Domain&) override { return Status::ok(); }
+  Status timer_stop(Domain&, double* ms) override {
+    *ms = 0;
+    return Status::ok();
+  }
+};
+
+}  // namespace
+
+Exec* make_dry_exec() { return new DryExec(); }
+
+}  // namespace tiles

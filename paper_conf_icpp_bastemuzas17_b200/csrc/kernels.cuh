@@ -1,0 +1,76 @@
+// kernels.cuh — internal interface between the runtime (scheduler.cpp) and
+// the sm_100a kernels (kernels.cu). Not part of the C ABI.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace tiles {
+
+// Face directions of a tile (regions expanded with ghost cells).
+enum Face : int { XM = 0, XP = 1, YM = 2, YP = 3, ZM = 4, ZP = 5 };
+
+// One tile processed by a kernel launch: its interior in (old) and out (new)
+// device buffers, both contiguous [tz][ty][tx].
+struct TileItem {
+  const double* in;
+  double* out;
+  int32_t tile;  // rank-local tile id (indexes the ghost-source table)
+  int32_t pad;
+};
+
+constexpr int kMaxInlineItems = 8;
+
+// Heat7 launch parameters (§VI.A; DESIGN.md §4 "heat7_tma").
+struct HeatParams {
+  int32_t tx, ty, tz;    // tile extents (cells)
+  int32_t band;          // rows of a band (divides ty, even)
+  int32_t nbands;        // ty / band
+  int32_t nitems;
+  double alpha;
+  const TileItem* items; // device array, or nullptr -> inline_items
+  TileItem inline_items[kMaxInlineItems];
+  // Ghost-source planes for the READ parity: gsrc[tile*6 + face] points at the
+  // plane holding the cells just outside `face` of `tile` (the neighbour's
+  // export of the opposite face, a Dirichlet fixed face or a slab halo).
+  const double* const* gsrc;
+  // Export faces for the WRITE parity: face f of tile k starts at
+  // fexp[f] + k * face_elems[f]. Layouts: x-faces [z][y], y-faces [z][x],
+  // z-faces [y][x].
+  double* fexp[6];
+  int64_t face_elems[6];
+};
+
+struct SincosParams {
+  int64_t tile_elems;
+  int32_t nitems;
+  int64_t iters;         // kernel_iteration * fused steps
+  const TileItem* items;
+  TileItem inline_items[kMaxInlineItems];
+};
+
+struct ExtractParams {   // export u's boundary layers into faces (parity p)
+  int32_t tx, ty, tz;
+  int32_t nitems;
+  const TileItem* items; // uses .in and .tile
+  TileItem inline_items[kMaxInlineItems];
+  double* fexp[6];
+  int64_t face_elems[6];
+};
+
+// Launch helpers (return cudaError_t of the launch).
+struct HeatLaunchCfg {
+  int stages;
+  int threads;
+  int grid;
+  size_t smem;
+};
+// Pick the band height and pipeline depth for a tile shape; false if the
+// shape cannot be staged (then tile_domain_create rejects it).
+bool heat_plan(int tx, int ty, int max_smem, int* band, int* stages, size_t* smem);
+cudaError_t heat_configure(int tx, int ty, int band, int stages, size_t smem, int* ctas_per_sm);
+cudaError_t launch_heat7(const HeatParams& p, int stages, size_t smem, int grid,
+                         cudaStream_t s);
+cudaError_t launch_sincos(const SincosParams& p, int grid, cudaStream_t s);
+cudaError_t launch_extract(const ExtractParams& p, cudaStream_t s);
+
+}  // namespace tiles

@@ -1,0 +1,906 @@
+// runtime.cpp — domain lifecycle and the tile scheduler (host C++).
+//
+// Paper mechanisms and where they live here:
+//   allocation policy, "as many regions as fit" -> domain_create
+//   pinned host regions                                 -> host store
+//   one stream per device buffer, async H2D, no sync -> run_*
+//   cache list with -1 = free, D2H(owner) before reuse -> acquire()
+//   ghost update on the device                           -> fused into
+//     heat7 (faces), ordered by per-tile / per-layer events instead of the
+//     paper's global `acc wait` (difference D3)
+//   D2H + synchronize before host access          -> domain_sync
+#include <algorithm>
+#include <cstring>
+#include <set>
+
+#include "runtime.hpp"
+
+namespace tiles {
+
+namespace {
+
+constexpr uint64_t kReserveBytes = 1ull << 30;  // head-room left to the driver/others
+constexpr uint64_t kAlign = 256;
+
+uint64_t align_up(uint64_t v) { return (v + kAlign - 1) / kAlign * kAlign; }
+
+int ev_layer(const Domain& d, int64_t L, int par) { return d.ev_layer_base + (int)(2 * L + par); }
+int ev_tile(const Domain& d, int64_t k, int par) { return d.ev_tile_base + (int)(2 * k + par); }
+int ev_slot(const Domain& d, int s) { return d.ev_slot_base + s; }
+int ev_faces_init(const Domain& d) { return d.ev_misc_base + 0; }
+int ev_halo(const Domain& d, int par) { return d.ev_misc_base + 1 + par; }
+int ev_join(const Domain& d) { return d.ev_misc_base + 3; }
+int ev_stream_tail(const Domain& d, int s) { return d.ev_misc_base + 4 + s; }
+
+bool z_wraps_locally(const Geometry& G) { return G.nranks == 1 && G.bc == TILE_BC_PERIODIC; }
+
+}  // namespace
+
+// ------------------------------------------------------------------ create
+Status domain_create(const int64_t dims[3], const int64_t tdims[3], int ghost,
+                     const tile_options* opt_in, Domain** out) {
+  tile_options opt{};
+  opt.device = -1;
+  opt.bc = TILE_BC_PERIODIC;
+  opt.nranks = 1;
+  opt.rank = 0;
+  opt.sched = TILE_SCHED_AUTO;
+  opt.fuse_pointwise_steps = 1;
+  if (opt_in) opt = *opt_in;
+  if (opt.nranks == 0) opt.nranks = 1;
+  if (opt.sched < TILE_SCHED_AUTO || opt.sched > TILE_SCHED_SYNC)
+    return make_err(TILE_EINVAL, "bad sched");
+  if (opt.nstreams_provided < 0 || opt.nstreams_provided > 64)
+    return make_err(TILE_EINVAL, "nstreams_provided must be in [0, 64]");
+  Geometry G;
+  Status st = make_geometry(dims, tdims, ghost, opt.bc, opt.nranks, opt.rank, &G);
+  if (st.bad()) return st;
+  if (G.nranks > 1 && !opt.nccl_unique_id && !opt.dry_run)
+    return make_err(TILE_EINVAL, "nranks > 1 needs nccl_unique_id");
+
+  int band = 0, stages = 0;
+  size_t smem = 0;
+  if (!heat_plan((int)G.t[0], (int)G.t[1], 200 * 1024, &band, &stages, &smem))
+    return make_err(TILE_EINVAL, "tile x extent too large to stage a 2-row band in shared memory");
+
+  Domain* d = new Domain();
+  d->G = G;
+  d->opt = opt;
+  d->band = band;
+  d->stages = stages;
+  d->heat_smem = smem;
+  if (opt.dry_run) {
+    d->exec = make_dry_exec();
+  } else {
+    d->exec = make_cuda_exec(*d, &st);
+    if (st.bad()) {
+      delete d;
+      return st;
+    }
+  }
+  st = domain_setup(*d);
+  if (st.bad()) {
+    domain_free(d);
+    return st;
+  }
+  *out = d;
+  return Status::ok();
+}
+
+// Memory plan ("calculates how many regions can fit into device
+// memory by checking available memory with cudaMemGetInfo"): persistent
+// face/halo/table storage first, then as many tile slots as the budget holds.
+Status domain_setup(Domain& d) {
+  const Geometry& G = d.G;
+  Exec& X = *d.exec;
+  const uint64_t tile_bytes = (uint64_t)G.tile_elems * 8;
+  const bool dir = G.bc == TILE_BC_DIRICHLET;
+  const bool multi = G.nranks > 1;
+
+  // host: tile store (+ initial faces for streaming, + Dirichlet faces)
+  uint64_t face_bytes_all = 0;
+  for (int f = 0; f < 6; ++f) face_bytes_all += align_up((uint64_t)G.ntiles * G.face_elems[f] * 8);
+  const uint64_t host_store = align_up((uint64_t)G.ntiles * tile_bytes);
+  const uint64_t host_total = host_store + face_bytes_all * (dir ? 2 : 1);
+  void* hp = nullptr;
+  Status st = X.alloc_host(d, host_total, &hp);
+  if (st.bad()) return st;
+  d.host_bytes = host_total;
+  char* hc = static_cast<char*>(hp);
+  d.host = reinterpret_cast<double*>(hc);
+  uint64_t off = host_store;
+  for (int f = 0; f < 6; ++f) {
+    d.host_faces[f] = reinterpret_cast<double*>(hc + off);
+    off += align_up((uint64_t)G.ntiles * G.face_elems[f] * 8);
+  }
+  if (dir)
+    for (int f = 0; f < 6; ++f) {
+      d.host_dir[f] = reinterpret_cast<double*>(hc + off);
+      std::memset(d.host_dir[f], 0, (size_t)G.ntiles * G.face_elems[f] * 8);
+      off += align_up((uint64_t)G.ntiles * G.face_elems[f] * 8);
+    }
+
+  // device: persistent part
+  uint64_t persist = 2 * face_bytes_all;  // export faces, 2 parities
+  if (dir) persist += face_bytes_all;
+  const uint64_t halo_bytes = align_up((uint64_t)G.layer_tiles * G.face_elems[ZM] * 8);
+  if (multi) persist += 4 * halo_bytes;
+  const uint64_t gsrc_bytes = align_up((uint64_t)G.ntiles * 6 * sizeof(double*));
+  const uint64_t items_bytes = align_up((uint64_t)G.ntiles * sizeof(TileItem));
+  persist += 2 * gsrc_bytes + 2 * items_bytes;
+
+  uint64_t budget;
+  if (d.opt.device_pool) {
+    budget = d.opt.device_pool_bytes;
+  } else {
+    uint64_t fr = 0, tot = 0;
+    st = X.mem_info(d, &fr, &tot);
+    if (st.bad()) return st;
+    budget = fr > kReserveBytes ? fr - kReserveBytes : 0;
+  }
+  if (d.opt.device_budget_bytes) budget = std::min<uint64_t>(budget, d.opt.device_budget_bytes);
+  if (budget < persist + 2 * tile_bytes)
+    return make_err(TILE_ENOMEM_DEVICE, "device budget below faces + 2 tile slots");
+  const uint64_t fit = (budget - persist) / tile_bytes;
+  const uint64_t want_res = 2 * (uint64_t)G.ntiles;
+  switch (d.opt.sched) {
+    case TILE_SCHED_RESIDENT:
+    case TILE_SCHED_SYNC:
+      if (fit < want_res) return make_err(TILE_ENOMEM_DEVICE, "resident schedule does not fit");
+      d.mode = MODE_RESIDENT;
+      d.nslots = (int)want_res;
+      break;
+    case TILE_SCHED_STREAM:
+      d.mode = MODE_STREAM;
+      d.nslots = (int)std::min<uint64_t>(fit, want_res);
+      break;
+    default:
+      d.mode = fit >= want_res ? MODE_RESIDENT : MODE_STREAM;
+      d.nslots = (int)std::min<uint64_t>(fit, want_res);
+  }
+  const uint64_t dev_total = persist + (uint64_t)d.nslots * tile_bytes;
+  void* dp = nullptr;
+  if (d.opt.device_pool) {
+    dp = d.opt.device_pool;
+    d.own_pool = false;
+  } else {
+    st = X.alloc_device(d, dev_total, &dp);
+    if (st.bad()) return st;
+    d.own_pool = true;
+  }
+  d.pool = static_cast<char*>(dp);
+  d.pool_bytes = dev_total;
+  d.device_bytes = dev_total;
+  off = 0;
+  auto carve = [&](uint64_t bytes) {
+    char* p = d.pool + off;
+    off += align_up(bytes);
+    return p;
+  };
+  for (int p = 0; p < 2; ++p)
+    for (int f = 0; f < 6; ++f)
+      d.faces[f][p] = reinterpret_cast<double*>(carve((uint64_t)G.ntiles * G.face_elems[f] * 8));
+  if (dir)
+    for (int f = 0; f < 6; ++f)
+      d.dir_faces[f] = reinterpret_cast<double*>(carve((uint64_t)G.ntiles * G.face_elems[f] * 8));
+  if (multi)
+    for (int a = 0; a < 2; ++a)
+      for (int p = 0; p < 2; ++p) d.halo[a][p] = reinterpret_cast<double*>(carve(halo_bytes));
+  for (int p = 0; p < 2; ++p) d.gsrc_dev[p] = reinterpret_cast<const double**>(carve(gsrc_bytes));
+  for (int p = 0; p < 2; ++p) d.items_dev[p] = reinterpret_cast<TileItem*>(carve(items_bytes));
+  d.slot_base = reinterpret_cast<double*>(d.pool + off);
+
+  // ghost-source tables (both parities) and resident item lists
+  for (int p = 0; p < 2; ++p) {
+    d.gsrc_host[p].resize((size_t)G.ntiles * 6);
+    for (int64_t k = 0; k < G.ntiles; ++k)
+      for (int f = 0; f < 6; ++f) d.gsrc_host[p][(size_t)k * 6 + f] = d.face_src_ptr(k, f, p);
+  }
+  if (d.mode == MODE_RESIDENT) {
+    for (int b = 0; b < 2; ++b) {
+      d.items_host[b].resize((size_t)G.ntiles);
+      for (int64_t k = 0; k < G.ntiles; ++k) {
+        const int cur = b == 0 ? (int)k : (int)(G.ntiles + k);
+        const int nxt = b == 0 ? (int)(G.ntiles + k) : (int)k;
+        d.items_host[b][(size_t)k] = {d.slot_ptr(cur), d.slot_ptr(nxt), (int32_t)k, 0};
+      }
+    }
+  } else {
+    d.items_dev[0] = d.items_dev[1] = nullptr;
+  }
+
+  // residency: cache list all -1
+  d.slot_owner.assign((size_t)d.nslots, -1);
+  d.tile_slot.assign((size_t)G.ntiles, -1);
+  d.tile_dirty.assign((size_t)G.ntiles, 0);
+  d.tile_last_use.assign((size_t)G.ntiles, 0);
+  d.free_slots.clear();
+  for (int s = 0; s < d.nslots; ++s) d.free_slots.push_back(s);
+
+  // events
+  d.ev_layer_base = 0;
+  d.ev_tile_base = d.ev_layer_base + (int)(2 * G.n[2]);
+  d.ev_slot_base = d.ev_tile_base + (int)(2 * G.ntiles);
+  d.ev_misc_base = d.ev_slot_base + d.nslots;
+  d.nevents = d.ev_misc_base + 4 + d.halo_stream + 1;
+  st = X.setup(d);
+  if (st.bad()) return st;
+  if (multi && !d.opt.dry_run) {
+    st = nccl_init(d);
+    if (st.bad()) return st;
+  }
+  return Status::ok();
+}
+
+Status domain_free(Domain* d) {
+  if (!d) return Status::ok();
+  Status r;
+  if (d->exec) {
+    if (!d->poisoned && d->in_flight) r = d->exec->sync_all(*d);
+    if (d->nccl_comm) nccl_destroy(*d);
+    d->exec->destroy(*d);
+    if (d->own_pool && d->pool) d->exec->free_device(*d, d->pool);
+    if (d->host) d->exec->free_host(*d, d->host);
+    delete d->exec;
+  }
+  delete d;
+  return r;
+}
+
+// --------------------------------------------------------------- residency
+namespace {
+
+struct Sched {
+  Domain& d;
+  Exec& X;
+  int S;
+  std::set<std::pair<int64_t, int>> lru;  // (last_use, tile) of resident tiles
+
+  explicit Sched(Domain& dd, int s) : d(dd), X(*dd.exec), S(s) {
+    for (int64_t k = 0; k < d.G.ntiles; ++k)
+      if (d.tile_slot[k] >= 0) lru.insert({d.tile_last_use[k], (int)k});
+  }
+  int stream_of(int64_t k) const { return (int)(k % S); }
+
+  void touch(int64_t k) {
+    lru.erase({d.tile_last_use[k], (int)k});
+    d.tile_last_use[k] = ++d.use_clock;
+    lru.insert({d.tile_last_use[k], (int)k});
+  }
+
+  // D2H of tile k from its slot into the pinned host store.
+  Status writeback(int64_t k) {
+    const int s = d.tile_slot[k];
+    const int st = stream_of(k);
+    Status r = X.d2h(d, k, 1, s, st);
+    if (r.bad()) return r;
+    d.tile_dirty[k] = 0;
+    d.stats.writebacks++;
+    return X.record(d, ev_slot(d, s), st);
+  }
+
+  // A free device slot for tile k: a free pointer, else the least
+  // recently used resident tile is evicted — copied back first if dirty
+  // ("queues memory transfers of the region that is currently using
+  // the assigned device memory pointer from device to host"), dropped if
+  // clean. `protect` is never evicted.
+  Status acquire(int64_t k, int stream, int protect, int* out) {
+    int s;
+    if (!d.free_slots.empty()) {
+      s = d.free_slots.front();
+      d.free_slots.pop_front();
+    } else {
+      int victim = -1;
+      for (auto& e : lru) {
+        const int t = e.second;
+        if (t != k && d.tile_slot[t] != protect) {
+          victim = t;
+          break;
+        }
+      }
+      if (victim < 0) return make_err(TILE_ENOMEM_DEVICE, "no evictable slot");
+      s = d.tile_slot[victim];
+      if (d.tile_dirty[victim]) {
+        Status r = writeback(victim);
+        if (r.bad()) return r;
+      } else {
+        Status r = X.note(d, TILE_OP_DROP, victim, s, stream_of(victim));
+        if (r.bad()) return r;
+      }
+      d.stats.evictions++;
+      lru.erase({d.tile_last_use[victim], victim});
+      d.tile_slot[victim] = -1;
+      d.slot_owner[s] = -1;
+    }
+    Status r = X.wait(d, ev_slot(d, s), stream);
+    if (r.bad()) return r;
+    d.slot_owner[s] = (int)k;
+    *out = s;
+    return Status::ok();
+  }
+
+  void release(int s) {
+    d.slot_owner[s] = -1;
+    d.free_slots.push_back(s);
+  }
+};
+
+// Make every stream of this run wait for everything issued before it
+// (previous runs may have used other streams, faces are shared state).
+Status join_streams(Domain& d, int S) {
+  Exec& X = *d.exec;
+  const int nst = d.halo_stream + 1;
+  for (int s = 0; s < nst; ++s) {
+    if (s >= S && s != d.halo_stream) continue;
+    Status r = X.record(d, ev_stream_tail(d, s), s);
+    if (r.bad()) return r;
+  }
+  for (int s = 0; s < nst; ++s) {
+    if (s >= S && s != d.halo_stream) continue;
+    for (int t = 0; t < nst; ++t) {
+      if (t == s || (t >= S && t != d.halo_stream)) continue;
+      Status r = X.wait(d, ev_stream_tail(d, t), s);
+      if (r.bad()) return r;
+    }
+  }
+  return Status::ok();
+}
+
+}  // namespace
+
+// ----------------------------------------------------- resident heat runs
+// Batches are contiguous z-layer ranges; batch i runs on stream i % S. A
+// batch's step s waits for its neighbour batches' step s-1 (their faces are
+// its ghost sources, and it overwrites the face parity they read).
+namespace {
+
+struct Batch {
+  int64_t L0, L1;  // layers [L0, L1)
+  int stream;
+};
+
+struct ResidentRun {
+  Domain& d;
+  Exec& X;
+  const Geometry& G;
+  std::vector<Batch> B;
+  std::vector<std::vector<int>> nbr;  // neighbour batches (excluding self)
+  bool need_load, need_extract, multi;
+  int bit0, fp0, T;
+  double alpha;
+
+  ResidentRun(Domain& dd) : d(dd), X(*dd.exec), G(dd.G) {}
+
+  int64_t tile0(const Batch& b) const { return b.L0 * G.layer_tiles; }
+  int64_t ntl(const Batch& b) const { return (b.L1 - b.L0) * G.layer_tiles; }
+  int cur_slot(int64_t k, int bit) const { return bit == 0 ? (int)k : (int)(G.ntiles + k); }
+
+  void build(int S, bool serial) {
+    const int64_t nL = G.n[2];
+    B.clear();
+    if (serial || (!need_load && !multi)) {
+      B.push_back({0, nL, 0});
+    } else if (!need_load && multi && nL > 2) {
+      B.push_back({0, 1, 0});
+      B.push_back({nL - 1, nL, 1 % S});
+      B.push_back({1, nL - 1, 2 % S});
+    } else {
+      for (int64_t L = 0; L < nL; ++L) B.push_back({L, L + 1, 0});
+      // wrap-aware order: 0, nL-1, 1, nL-2, ... so a periodic layer's
+      // neighbours arrive early
+      std::vector<Batch> o;
+      int64_t lo = 0, hi = nL - 1;
+      bool front = true;
+      while (lo <= hi) {
+        o.push_back(B[front ? lo++ : hi--]);
+        front = !front;
+      }
+      if (!z_wraps_locally(G)) std::sort(o.begin(), o.end(), [](auto& a, auto& b) { return a.L0 < b.L0; });
+      B = o;
+      for (size_t i = 0; i < B.size(); ++i) B[i].stream = (int)(i % S);
+    }
+    // neighbour batches
+    auto batch_of = [&](int64_t L) {
+      for (size_t i = 0; i < B.size(); ++i)
+        if (L >= B[i].L0 && L < B[i].L1) return (int)i;
+      return -1;
+    };
+    nbr.assign(B.size(), {});
+    for (size_t i = 0; i < B.size(); ++i) {
+      std::vector<int64_t> ls = {B[i].L0 - 1, B[i].L1};
+      for (int64_t L : ls) {
+        if (L < 0 || L >= nL) {
+          if (!z_wraps_locally(G)) continue;
+          L = (L + nL) % nL;
+        }
+        int j = batch_of(L);
+        if (j >= 0 && j != (int)i &&
+            std::find(nbr[i].begin(), nbr[i].end(), j) == nbr[i].end())
+          nbr[i].push_back(j);
+      }
+    }
+  }
+  bool boundary(const Batch& b) const { return b.L0 == 0 || b.L1 == G.n[2]; }
+
+  Status issue_load(size_t i) {
+    const Batch& b = B[i];
+    Status r;
+    if (need_load) {
+      r = X.h2d(d, tile0(b), ntl(b), cur_slot(tile0(b), bit0), b.stream);
+      if (r.bad()) return r;
+    }
+    if (need_extract) {
+      r = X.extract(d, tile0(b), ntl(b), cur_slot(tile0(b), bit0), fp0,
+                    d.items_dev[bit0] ? d.items_dev[bit0] + tile0(b) : nullptr, b.stream);
+      if (r.bad()) return r;
+    }
+    return X.record(d, ev_layer(d, (int64_t)i, 1), b.stream);
+  }
+
+  Status issue_kernel(size_t i, int s) {
+    const Batch& b = B[i];
+    Status r;
+    for (int j : nbr[i]) {
+      r = X.wait(d, ev_layer(d, j, (s - 1) & 1), b.stream);
+      if (r.bad()) return r;
+    }
+    if (multi && boundary(b)) {
+      r = X.wait(d, ev_halo(d, (s - 1) & 1), b.stream);
+      if (r.bad()) return r;
+    }
+    const int bit = bit0 ^ (s & 1);
+    const int rp = fp0 ^ (s & 1);
+    r = X.heat(d, nullptr, nullptr, nullptr, (int)ntl(b), rp,
+               d.items_dev[bit] ? d.items_dev[bit] + tile0(b) : nullptr, b.stream);
+    if (r.bad()) return r;
+    (void)alpha;
+    return X.record(d, ev_layer(d, (int64_t)i, s & 1), b.stream);
+  }
+
+  Status issue_halo(int s) {  // exchange the faces written at step s (s = -1: current)
+    const int hs = d.halo_stream;
+    Status r;
+    for (size_t i = 0; i < B.size(); ++i) {
+      if (!boundary(B[i])) continue;
+      r = X.wait(d, ev_layer(d, (int64_t)i, s & 1), hs);
+      if (r.bad()) return r;
+    }
+    r = X.halo(d, fp0 ^ ((s + 1) & 1), hs);
+    if (r.bad()) return r;
+    return X.record(d, ev_halo(d, s & 1), hs);
+  }
+
+  // Greedy list issue of the (load, kernel, halo) DAG in dependency order.
+  Status run() {
+    const size_t nb = B.size();
+    std::vector<int> done(nb, -2);  // last issued: -2 nothing, -1 load, s kernel step s
+    int halo_done = -2;              // last halo step issued (-1 = initial)
+    size_t loads = 0;
+    std::vector<size_t> load_order(nb);
+    for (size_t i = 0; i < nb; ++i) load_order[i] = i;
+    auto kernel_ready = [&](size_t i) {
+      const int s = done[i] + 1;
+      if (s >= T || done[i] < -1) return false;
+      for (int j : nbr[i])
+        if (done[j] < s - 1) return false;
+      if (multi && boundary(B[i]) && halo_done < s - 1) return false;
+      return true;
+    };
+    auto halo_ready = [&]() {
+      if (!multi) return false;
+      const int s = halo_done + 1;  // next halo step to issue
+      if (s > T - 2) return false;  // nobody consumes the last step's halo
+      for (size_t i = 0; i < nb; ++i)
+        if (boundary(B[i]) && done[i] < s) return false;
+      // WAR: the step-s halo overwrites buffers read by step s-1 kernels,
+      // which precede the step-s boundary kernels in stream order.
+      return true;
+    };
+    for (;;) {
+      bool progress = false;
+      // drain everything ready, in (step, batch) order
+      for (bool again = true; again;) {
+        again = false;
+        if (halo_ready()) {
+          Status r = issue_halo(halo_done + 1);
+          if (r.bad()) return r;
+          ++halo_done;
+          again = progress = true;
+        }
+        int best_s = 1 << 30;
+        for (size_t i = 0; i < nb; ++i)
+          if (kernel_ready(i)) best_s = std::min(best_s, done[i] + 1);
+        for (size_t i = 0; i < nb; ++i) {
+          if (kernel_ready(i) && done[i] + 1 == best_s) {
+            Status r = issue_kernel(i, done[i] + 1);
+            if (r.bad()) return r;
+            ++done[i];
+            again = progress = true;
+          }
+        }
+      }
+      if (loads < nb) {
+        Status r = issue_load(load_order[loads]);
+        if (r.bad()) return r;
+        done[load_order[loads]] = -1;
+        ++loads;
+        if (loads == nb && multi && halo_done == -2) {
+          r = issue_halo(-1);
+          if (r.bad()) return r;
+          halo_done = -1;
+        }
+        continue;
+      }
+      if (!progress) break;
+    }
+    for (size_t i = 0; i < nb; ++i)
+      if (done[i] != T - 1) return make_err(TILE_ESTATE, "internal: resident schedule incomplete");
+    return Status::ok();
+  }
+};
+
+}  // namespace
+
+static Status upload_dirichlet_if_needed(Domain& d);
+
+static Status run_heat_resident(Domain& d, double alpha, int T, int S, bool serial) {
+  ResidentRun R(d);
+  R.alpha = alpha;
+  R.T = T;
+  R.need_load = !d.resident_valid;
+  R.need_extract = !d.faces_valid;
+  R.multi = d.G.nranks > 1;
+  R.bit0 = d.res_bit;
+  R.fp0 = d.face_parity;
+  R.build(S, serial);
+  Status r = R.run();
+  if (r.bad()) return r;
+  d.res_bit ^= (T & 1);
+  d.face_parity ^= (T & 1);
+  d.resident_valid = true;
+  d.faces_valid = true;
+  for (int64_t k = 0; k < d.G.ntiles; ++k) {
+    d.tile_slot[k] = R.cur_slot(k, d.res_bit);
+    if (T > 0) d.tile_dirty[k] = 1;
+  }
+  // remember which stream holds each tile's last kernel (for tile_sync)
+  d.trace.reserve(d.trace.size());
+  d.last_batches.clear();
+  for (auto& b : R.B) d.last_batches.push_back({b.L0, b.L1, b.stream});
+  return Status::ok();
+}
+
+// -------------------------------------------------- streaming (out-of-core)
+static Status run_stream(Domain& d, const tile_kernel& k, int T, int S) {
+  Exec& X = *d.exec;
+  const Geometry& G = d.G;
+  Sched sc(d, S);
+  const bool heat = k.kind == TILE_KERNEL_HEAT7;
+  const bool fuse = !heat && d.opt.fuse_pointwise_steps;
+  const int passes = fuse ? (T > 0 ? 1 : 0) : T;
+  const int64_t iters = fuse ? (int64_t)k.inner_iters * T : k.inner_iters;
+  const int64_t N = G.ntiles;
+  const bool multi = G.nranks > 1;
+  Status r;
+
+  if (heat && !d.faces_valid) {
+    if (!d.host_faces_valid) {
+      host_extract_faces(G, d.host, d.host_faces);
+      d.host_faces_valid = true;
+    }
+    r = X.faces_h2d(d, d.face_parity, 0);
+    if (r.bad()) return r;
+    r = X.record(d, ev_faces_init(d), 0);
+    if (r.bad()) return r;
+    d.faces_valid = true;
+  } else if (heat) {
+    r = X.record(d, ev_faces_init(d), 0);
+    if (r.bad()) return r;
+  }
+  const int fp0 = d.face_parity;
+  auto issue_halo = [&](int s) -> Status {  // faces written at pass s (s=-1: current)
+    const int hs = d.halo_stream;
+    for (int64_t t = 0; t < N; ++t) {
+      int64_t ix, iy, iz;
+      G.tile_coords(t, &ix, &iy, &iz);
+      if (iz != 0 && iz != G.n[2] - 1) continue;
+      Status q = X.wait(d, s < 0 ? ev_faces_init(d) : ev_tile(d, t, s & 1), hs);
+      if (q.bad()) return q;
+    }
+    Status q = X.halo(d, fp0 ^ ((s + 1) & 1), hs);
+    if (q.bad()) return q;
+    return X.record(d, ev_halo(d, s & 1), hs);
+  };
+  if (heat && multi && passes > 0) {
+    r = issue_halo(-1);
+    if (r.bad()) return r;
+  }
+
+  // keep window: the last W tiles of a pass stay dirty on the device; the
+  // snake order makes them the first (cache hits) of the next pass.
+  const int64_t W = std::max<int64_t>(0, std::min<int64_t>(N - 1, d.nslots - 4 * (int64_t)S - 2));
+  for (int s = 0; s < passes; ++s) {
+    const int rp = fp0 ^ (s & 1);
+    for (int64_t j = 0; j < N; ++j) {
+      const int64_t t = (s & 1) ? N - 1 - j : j;
+      const int st = sc.stream_of(t);
+      int in = d.tile_slot[t];
+      if (in >= 0) {
+        d.stats.hits++;
+        r = X.note(d, TILE_OP_HIT, t, in, st);
+        if (r.bad()) return r;
+      } else {
+        d.stats.misses++;
+        r = sc.acquire(t, st, -1, &in);
+        if (r.bad()) return r;
+        r = X.h2d(d, t, 1, in, st);
+        if (r.bad()) return r;
+        d.tile_slot[t] = in;
+        d.tile_dirty[t] = 0;
+        sc.touch(t);
+      }
+      if (heat) {
+        int out;
+        r = sc.acquire(t, st, in, &out);
+        if (r.bad()) return r;
+        // ghost sources: neighbours' previous pass (RAW) and their reads of
+        // the parity this kernel overwrites (WAR)
+        bool halo_wait = false;
+        for (int f = 0; f < 6; ++f) {
+          FaceSrc fs = face_source(G, t, f);
+          if (fs.kind == 0 && fs.val != t) {
+            r = X.wait(d, s == 0 ? ev_faces_init(d) : ev_tile(d, fs.val, (s - 1) & 1), st);
+            if (r.bad()) return r;
+          } else if (fs.kind >= 2) {
+            halo_wait = true;
+          }
+        }
+        if (s == 0) {
+          r = X.wait(d, ev_faces_init(d), st);
+          if (r.bad()) return r;
+        }
+        if (halo_wait && multi) {
+          r = X.wait(d, ev_halo(d, (s - 1) & 1), st);
+          if (r.bad()) return r;
+        }
+        const int64_t tl[1] = {t};
+        const int is[1] = {in}, os[1] = {out};
+        r = X.heat(d, tl, is, os, 1, rp, nullptr, st);
+        if (r.bad()) return r;
+        r = X.record(d, ev_tile(d, t, s & 1), st);
+        if (r.bad()) return r;
+        r = X.record(d, ev_slot(d, in), st);
+        if (r.bad()) return r;
+        sc.release(in);
+        d.tile_slot[t] = out;
+        d.slot_owner[out] = (int)t;
+      } else {
+        r = X.sincos(d, t, in, iters, st);
+        if (r.bad()) return r;
+      }
+      d.tile_dirty[t] = 1;
+      sc.touch(t);
+      if (j < N - W) {
+        r = sc.writeback(t);
+        if (r.bad()) return r;
+      } else {
+        r = X.record(d, ev_slot(d, d.tile_slot[t]), st);
+        if (r.bad()) return r;
+      }
+    }
+    if (heat && multi && s < passes - 1) {
+      r = issue_halo(s);
+      if (r.bad()) return r;
+    }
+  }
+  if (heat) d.face_parity ^= (T & 1);
+  return Status::ok();
+}
+
+// ------------------------------------------------------------ public runs
+static Status upload_dirichlet_if_needed(Domain& d) {
+  if (d.G.bc != TILE_BC_DIRICHLET || d.dir_uploaded) return Status::ok();
+  Status r = d.exec->upload_dir(d);
+  if (r.bad()) return r;
+  d.dir_uploaded = true;
+  return Status::ok();
+}
+
+Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
+  if (k.kind == TILE_KERNEL_HEAT7) {
+    if (!(k.alpha > 0.0 && k.alpha <= 1.0 / 6.0))
+      return make_err(TILE_EINVAL, "HEAT7 alpha must be in (0, 1/6]");
+  } else if (k.kind == TILE_KERNEL_SINCOS) {
+    if (k.inner_iters < 0) return make_err(TILE_EINVAL, "SINCOS inner_iters must be >= 0");
+  } else {
+    return make_err(TILE_EINVAL, "unknown kernel kind");
+  }
+  if (steps < 0) return make_err(TILE_EINVAL, "steps must be >= 0");
+  if (nstreams < 1 || nstreams > 64) return make_err(TILE_EINVAL, "nstreams must be in [1, 64]");
+  d.kernel_alpha = k.alpha;
+  Status r = upload_dirichlet_if_needed(d);
+  if (r.bad()) return r;
+  const bool serial = d.opt.sched == TILE_SCHED_SYNC;
+  const int S = serial ? 1 : nstreams;
+  r = join_streams(d, std::max(S, d.streams_used));
+  if (r.bad()) return r;
+  d.streams_used = std::max(d.streams_used, S);
+  d.last_S = S;
+  d.in_flight = true;
+  if (k.kind == TILE_KERNEL_HEAT7 && d.mode == MODE_RESIDENT) {
+    r = run_heat_resident(d, k.alpha, steps, S, serial);
+  } else if (d.mode == MODE_RESIDENT) {
+    // pointwise kernel on resident tiles: per-tile H2D -> kernel, in place
+    Exec& X = *d.exec;
+    const bool fuse = d.opt.fuse_pointwise_steps;
+    const int passes = fuse ? (steps > 0 ? 1 : 0) : steps;
+    const int64_t iters = fuse ? (int64_t)k.inner_iters * steps : k.inner_iters;
+    for (int s = 0; s < passes; ++s)
+      for (int64_t t = 0; t < d.G.ntiles; ++t) {
+        const int st = serial ? 0 : (int)(t % S);
+        const int slot = (int)(d.res_bit == 0 ? t : d.G.ntiles + t);
+        if (!d.resident_valid && s == 0) {
+          r = X.h2d(d, t, 1, slot, st);
+          if (r.bad()) return r;
+        }
+        r = X.sincos(d, t, slot, iters, st);
+        if (r.bad()) return r;
+      }
+    if (passes > 0) {
+      d.resident_valid = true;
+      d.faces_valid = false;  // interiors changed without faces
+      for (int64_t t = 0; t < d.G.ntiles; ++t) {
+        d.tile_slot[t] = (int)(d.res_bit == 0 ? t : d.G.ntiles + t);
+        d.tile_dirty[t] = 1;
+      }
+      d.last_batches.clear();
+      for (int64_t L = 0; L < d.G.n[2]; ++L) d.last_batches.push_back({L, L + 1, -1});
+    }
+  } else {
+    r = run_stream(d, k, steps, S);
+    if (k.kind != TILE_KERNEL_HEAT7 && steps > 0) d.faces_valid = false;
+  }
+  if (r.bad()) return r;
+  if (k.kind == TILE_KERNEL_HEAT7) d.stats.steps_done += (uint64_t)steps;
+  return Status::ok();
+}
+
+// -------------------------------------------------------------- sync/store
+Status domain_sync(Domain& d) {
+  Exec& X = *d.exec;
+  Status r;
+  if (d.mode == MODE_RESIDENT) {
+    for (auto& b : d.last_batches) {
+      const int64_t t0 = b.L0 * d.G.layer_tiles, n = (b.L1 - b.L0) * d.G.layer_tiles;
+      bool any = false;
+      for (int64_t t = t0; t < t0 + n; ++t) any |= d.tile_dirty[t] != 0;
+      if (!any) continue;
+      if (b.stream >= 0) {
+        r = X.d2h(d, t0, n, d.tile_slot[t0], b.stream);
+        if (r.bad()) return r;
+      } else {  // per-tile streams (pointwise kernel)
+        for (int64_t t = t0; t < t0 + n; ++t) {
+          r = X.d2h(d, t, 1, d.tile_slot[t], (int)(t % std::max(1, d.last_S)));
+          if (r.bad()) return r;
+        }
+      }
+      for (int64_t t = t0; t < t0 + n; ++t) d.tile_dirty[t] = 0;
+    }
+  } else {
+    for (int64_t t = 0; t < d.G.ntiles; ++t) {
+      if (!d.tile_dirty[t] || d.tile_slot[t] < 0) continue;
+      const int st = (int)(t % std::max(1, d.last_S));
+      r = X.d2h(d, t, 1, d.tile_slot[t], st);
+      if (r.bad()) return r;
+      d.tile_dirty[t] = 0;
+      r = X.record(d, ev_slot(d, d.tile_slot[t]), st);
+      if (r.bad()) return r;
+    }
+  }
+  r = X.sync_all(d);
+  if (r.bad()) return r;
+  d.in_flight = false;
+  d.host_faces_valid = false;  // host store changed
+  return Status::ok();
+}
+
+Status domain_invalidate(Domain& d) {
+  if (d.in_flight) {
+    Status r = domain_sync(d);
+    if (r.bad()) return r;
+  }
+  for (int64_t t = 0; t < d.G.ntiles; ++t) {
+    if (d.tile_dirty[t]) return make_err(TILE_ESTATE, "dirty tiles; call tile_sync first");
+  }
+  d.resident_valid = false;
+  d.faces_valid = false;
+  if (d.mode == MODE_STREAM) {
+    for (int64_t t = 0; t < d.G.ntiles; ++t) d.tile_slot[t] = -1;
+    d.free_slots.clear();
+    for (int s = 0; s < d.nslots; ++s) {
+      d.slot_owner[s] = -1;
+      d.free_slots.push_back(s);
+    }
+  }
+  return Status::ok();
+}
+
+Status domain_load(Domain& d, const double* src) {
+  if (d.in_flight) {
+    Status r = domain_sync(d);
+    if (r.bad()) return r;
+  }
+  const Geometry& G = d.G;
+  const bool dir = G.bc == TILE_BC_DIRICHLET;
+  const int64_t h = dir ? 1 : 0;
+  const int64_t ex = G.l[0] + 2 * h, ey = G.l[1] + 2 * h;
+  const int64_t tx = G.t[0], ty = G.t[1], tz = G.t[2];
+  host_parallel_for(G.ntiles, [&](int64_t b, int64_t e) {
+    for (int64_t k = b; k < e; ++k) {
+      int64_t ix, iy, iz;
+      G.tile_coords(k, &ix, &iy, &iz);
+      double* dst = d.host_tile(k);
+      for (int64_t z = 0; z < tz; ++z)
+        for (int64_t y = 0; y < ty; ++y) {
+          const double* s =
+              src + ((iz * tz + z + h) * ey + (iy * ty + y + h)) * ex + ix * tx + h;
+          std::memcpy(dst + (z * ty + y) * tx, s, (size_t)tx * 8);
+        }
+    }
+  });
+  if (dir) {  // fixed Dirichlet faces from the halo (only boundary faces used)
+    host_parallel_for(G.ntiles, [&](int64_t b, int64_t e) {
+      for (int64_t k = b; k < e; ++k) {
+        int64_t ix, iy, iz;
+        G.tile_coords(k, &ix, &iy, &iz);
+        const int64_t ox = ix * tx + h, oy = iy * ty + h, oz = iz * tz + h;
+        auto at = [&](int64_t z, int64_t y, int64_t x) { return src[(z * ey + y) * ex + x]; };
+        for (int f = 0; f < 6; ++f) {
+          if (face_source(G, k, f).kind != 1) continue;
+          double* o = d.host_dir[f] + k * G.face_elems[f];
+          if (f <= XP) {
+            const int64_t x = f == XM ? ox - 1 : ox + tx;
+            for (int64_t z = 0; z < tz; ++z)
+              for (int64_t y = 0; y < ty; ++y) o[z * ty + y] = at(oz + z, oy + y, x);
+          } else if (f <= YP) {
+            const int64_t y = f == YM ? oy - 1 : oy + ty;
+            for (int64_t z = 0; z < tz; ++z)
+              for (int64_t x = 0; x < tx; ++x) o[z * tx + x] = at(oz + z, y, ox + x);
+          } else {
+            const int64_t z = f == ZM ? oz - 1 : oz + tz;
+            for (int64_t y = 0; y < ty; ++y)
+              for (int64_t x = 0; x < tx; ++x) o[y * tx + x] = at(z, oy + y, ox + x);
+          }
+        }
+      }
+    });
+    d.dir_uploaded = false;
+  }
+  d.host_faces_valid = false;
+  for (int64_t t = 0; t < G.ntiles; ++t) d.tile_dirty[t] = 0;
+  return domain_invalidate(d);
+}
+
+Status domain_store(Domain& d, double* dst) {
+  Status r = domain_sync(d);
+  if (r.bad()) return r;
+  const Geometry& G = d.G;
+  const int64_t h = G.bc == TILE_BC_DIRICHLET ? 1 : 0;
+  const int64_t ex = G.l[0] + 2 * h, ey = G.l[1] + 2 * h;
+  const int64_t tx = G.t[0], ty = G.t[1], tz = G.t[2];
+  host_parallel_for(G.ntiles, [&](int64_t b, int64_t e) {
+    for (int64_t k = b; k < e; ++k) {
+      int64_t ix, iy, iz;
+      G.tile_coords(k, &ix, &iy, &iz);
+      const double* s = d.host_tile(k);
+      for (int64_t z = 0; z < tz; ++z)
+        for (int64_t y = 0; y < ty; ++y) {
+          double* o = dst + ((iz * tz + z + h) * ey + (iy * ty + y + h)) * ex + ix * tx + h;
+          std::memcpy(o, s + (z * ty + y) * tx, (size_t)tx * 8);
+        }
+    }
+  });
+  return Status::ok();
+}
+
+}  // namespace tiles

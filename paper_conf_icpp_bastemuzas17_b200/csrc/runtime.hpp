@@ -1,0 +1,200 @@
+// runtime.hpp — internal state of a tile domain (not part of the C ABI).
+#pragma once
+#include <cstdint>
+#include <deque>
+#include <functional>
+#include <string>
+#include <vector>
+
+#include "../../include/tiles.h"
+#include "kernels.cuh"
+
+namespace tiles {
+
+struct Status {
+  tile_status code = TILE_OK;
+  std::string msg;
+  static Status ok() { return {}; }
+  bool bad() const { return code != TILE_OK; }
+};
+Status make_err(tile_status c, const std::string& m);
+
+// ------------------------------------------------------------------ geometry
+// Decomposition of a rank's z-slab into tiles (§III, §IV.A).
+struct Geometry {
+  int64_t g[3];   // global nx, ny, nz
+  int64_t l[3];   // local nx, ny, nz (slab)
+  int64_t t[3];   // tile dims
+  int64_t n[3];   // tiles per axis (local)
+  int64_t ntiles;
+  int64_t zoff;   // global z of local z = 0
+  int ghost;
+  tile_bc bc;
+  int nranks, rank;
+  int64_t tile_elems;
+  int64_t face_elems[6];
+  int64_t layer_tiles;  // tiles per z-layer = n[0]*n[1]
+
+  void tile_coords(int64_t id, int64_t* ix, int64_t* iy, int64_t* iz) const {
+    *ix = id % n[0];
+    *iy = (id / n[0]) % n[1];
+    *iz = id / (n[0] * n[1]);
+  }
+  int64_t tile_id(int64_t ix, int64_t iy, int64_t iz) const {
+    return (iz * n[1] + iy) * n[0] + ix;
+  }
+};
+
+Status make_geometry(const int64_t dims[3], const int64_t tdims[3], int ghost, tile_bc bc,
+                     int nranks, int rank, Geometry* out);
+
+// Face source of tile `id`, face f: kind 0 = export of a
+// neighbour tile on this rank (val = its id), 1 = Dirichlet fixed face
+// (val = id), 2 = halo from the rank below (val = position in layer),
+// 3 = halo from the rank above (val = position in layer).
+struct FaceSrc {
+  int kind;
+  int64_t val;
+};
+FaceSrc face_source(const Geometry& G, int64_t id, int f);
+void ghost_map(const Geometry& G, int64_t id, int64_t* out);  // (t+2g)^3 box
+
+// ----------------------------------------------------------------- executor
+// All device work goes through an executor: CudaExec issues CUDA/NCCL calls,
+// DryExec only records the op trace (tests on a CPU-only box).
+struct Domain;
+struct Exec {
+  virtual ~Exec() = default;
+  virtual Status h2d(Domain& d, int64_t tile0, int64_t ntile, int slot0, int stream) = 0;
+  virtual Status d2h(Domain& d, int64_t tile0, int64_t ntile, int slot0, int stream) = 0;
+  virtual Status record(Domain& d, int ev, int stream) = 0;
+  virtual Status wait(Domain& d, int ev, int stream) = 0;
+  // heat over tiles [tile0, tile0+ntile) of one z-layer batch (resident) or
+  // one tile (stream); in/out given by slots
+  virtual Status heat(Domain& d, const int64_t* tiles, const int* in_slots, const int* out_slots,
+                      int nitems, int read_parity, const TileItem* dev_items, int stream) = 0;
+  virtual Status sincos(Domain& d, int64_t tile, int slot, int64_t iters, int stream) = 0;
+  virtual Status extract(Domain& d, int64_t tile0, int64_t ntile, int slot0, int parity,
+                         const TileItem* dev_items, int stream) = 0;
+  virtual Status faces_h2d(Domain& d, int parity, int stream) = 0;
+  virtual Status halo(Domain& d, int parity, int stream) = 0;
+  virtual Status note(Domain& d, int kind, int64_t a, int64_t b, int stream) = 0;  // trace-only ops
+  virtual Status sync_all(Domain& d) = 0;
+  // resources
+  virtual Status mem_info(Domain& d, uint64_t* free_b, uint64_t* total_b) = 0;
+  virtual Status alloc_host(Domain& d, uint64_t bytes, void** p) = 0;
+  virtual void free_host(Domain& d, void* p) = 0;
+  virtual Status alloc_device(Domain& d, uint64_t bytes, void** p) = 0;
+  virtual void free_device(Domain& d, void* p) = 0;
+  virtual Status setup(Domain& d) = 0;       // streams, events, device tables
+  virtual Status upload_dir(Domain& d) = 0;  // Dirichlet fixed faces (sync)
+  virtual void destroy(Domain& d) = 0;
+  virtual Status timer_start(Domain& d) = 0;
+  virtual Status timer_stop(Domain& d, double* ms) = 0;
+};
+
+// -------------------------------------------------------------------- domain
+enum Mode : int { MODE_RESIDENT = 1, MODE_STREAM = 2 };
+
+struct Domain {
+  Geometry G;
+  tile_options opt;
+  bool poisoned = false;
+  int device = 0;
+  int mode = MODE_RESIDENT;
+  int measure = TILE_MEASURE_NORMAL;
+
+  // host (pinned unless dry-run)
+  double* host = nullptr;                  // ntiles * tile_elems, tile-blocked
+  double* host_faces[6] = {};              // initial faces for STREAM mode
+  double* host_dir[6] = {};                // Dirichlet fixed faces
+  bool host_faces_valid = false;
+  bool dir_uploaded = false;
+  uint64_t host_bytes = 0;
+
+  // device (carved from one pool)
+  char* pool = nullptr;
+  uint64_t pool_bytes = 0;
+  bool own_pool = false;
+  double* faces[6][2] = {};                // export faces [face][parity]
+  double* dir_faces[6] = {};               // Dirichlet fixed faces
+  double* halo[2][2] = {};                 // [0 = from below (z-), 1 = from above (z+)][parity]
+  const double** gsrc_dev[2] = {};         // [parity] -> ntiles*6 pointers
+  TileItem* items_dev[2] = {};             // resident mode: [bit] -> ntiles items
+  double* slot_base = nullptr;
+  int nslots = 0;
+  uint64_t device_bytes = 0;
+
+  // residency
+  std::vector<int> slot_owner;             // tile id or -1
+  std::vector<int> tile_slot;              // slot or -1
+  std::vector<char> tile_dirty;
+  std::vector<int64_t> tile_last_use;
+  std::deque<int> free_slots;
+  int res_bit = 0;                         // resident mode: 0 -> A current, 1 -> B
+  bool resident_valid = false;             // resident mode: all tiles on device
+  bool faces_valid = false;                // device faces hold the current state
+  int face_parity = 0;                     // parity of the current state's faces
+  int64_t use_clock = 0;
+
+  // streams / events (ids; CudaExec maps them to CUDA objects)
+  int nstreams_max = 64;
+  int halo_stream = 64;                    // index of the dedicated halo stream
+  int ev_layer_base = 0;                   // 2 per layer
+  int ev_tile_base = 0;                    // 2 per tile (face events)
+  int ev_slot_base = 0;                    // 1 per slot
+  int ev_misc_base = 0;                    // faces init, halo[2], done
+  int nevents = 0;
+
+  // NCCL
+  void* nccl_comm = nullptr;
+
+  // kernel plan
+  int band = 0, stages = 0, heat_grid = 0, sm_count = 148;
+  size_t heat_smem = 0;
+
+  // run bookkeeping
+  struct BatchRec { int64_t L0, L1; int stream; };
+  std::vector<BatchRec> last_batches;      // resident: where each layer's last kernel ran
+  double kernel_alpha = 0.125;
+  int streams_used = 1;                    // streams touched so far (joined at run start)
+  int last_S = 1;
+  std::vector<const double*> gsrc_host[2]; // [parity] -> ntiles*6
+  std::vector<TileItem> items_host[2];
+
+  tile_stats stats{};
+  std::vector<tile_op> trace;
+  Exec* exec = nullptr;
+  bool in_flight = false;
+  double run_t0 = 0;
+  bool kernel_timing = false;
+
+  double* slot_ptr(int s) const { return slot_base + (int64_t)s * G.tile_elems; }
+  double* host_tile(int64_t k) const { return host + k * G.tile_elems; }
+  const double* face_src_ptr(int64_t id, int f, int parity) const;
+};
+
+// runtime.cpp
+Status domain_create(const int64_t dims[3], const int64_t tdims[3], int ghost,
+                     const tile_options* opt, Domain** out);
+Status domain_load(Domain& d, const double* src);
+Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams);
+Status domain_sync(Domain& d);
+Status domain_store(Domain& d, double* dst);
+Status domain_invalidate(Domain& d);
+Status domain_free(Domain* d);
+Status domain_setup(Domain& d);
+void host_extract_faces(const Geometry& G, const double* host, double* const faces[6]);
+void host_parallel_for(int64_t n, const std::function<void(int64_t, int64_t)>& fn);
+
+// executors (exec_cuda.cu / exec_dry.cpp)
+Exec* make_cuda_exec(Domain& d, Status* st);
+Exec* make_dry_exec();
+
+// comm_nccl.cpp
+Status nccl_unique_id(void* out128);
+Status nccl_init(Domain& d);
+Status nccl_halo(Domain& d, int parity, void* stream);
+void nccl_destroy(Domain& d);
+
+}  // namespace tiles

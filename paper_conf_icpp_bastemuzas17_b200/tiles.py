@@ -1,0 +1,294 @@
+"""Thin ctypes binding of libtiles (include/tiles.h): argument marshalling only.
+
+Every step of the hot path runs inside libtiles' CUDA kernels; this module
+only converts Python/NumPy arguments and raises on error codes. The function
+names mirror the C ABI (tile_domain_create, tile_load, tile_run, tile_sync,
+tile_store, tile_free, ...); `Domain` is a convenience wrapper around them.
+
+There is no fallback: if libtiles.so is missing, importing this module
+raises ImportError (build it with `python paper_conf_icpp_bastemuzas17_b200/build.py`).
+"""
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libtiles.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(
+        "libtiles.so not built: run `python paper_conf_icpp_bastemuzas17_b200/build.py` "
+        "(there is no CPU fallback)")
+_lib = ctypes.CDLL(LIB_PATH, mode=ctypes.RTLD_GLOBAL)
+
+# ----------------------------------------------------------------- constants
+TILE_OK, TILE_EINVAL, TILE_ENOMEM_HOST, TILE_ENOMEM_DEVICE, TILE_ECUDA, TILE_ENCCL, \
+    TILE_ESTATE, TILE_ENOSYS = range(8)
+STATUS_NAMES = {0: "OK", 1: "EINVAL", 2: "ENOMEM_HOST", 3: "ENOMEM_DEVICE", 4: "ECUDA",
+                5: "ENCCL", 6: "ESTATE", 7: "ENOSYS"}
+TILE_BC_PERIODIC, TILE_BC_DIRICHLET = 0, 1
+TILE_KERNEL_HEAT7, TILE_KERNEL_SINCOS = 1, 2
+TILE_SCHED_AUTO, TILE_SCHED_RESIDENT, TILE_SCHED_STREAM, TILE_SCHED_SYNC = 0, 1, 2, 3
+TILE_MEASURE_NORMAL, TILE_MEASURE_XFER_ONLY, TILE_MEASURE_COMP_ONLY = 0, 1, 2
+OP_NAMES = {1: "h2d", 2: "d2h", 3: "kernel", 4: "record", 5: "wait", 6: "faces_h2d",
+            7: "extract", 8: "halo", 9: "drop", 10: "hit", 11: "pointwise"}
+SCHEDS = {"auto": 0, "resident": 1, "stream": 2, "sync": 3}
+BCS = {"periodic": 0, "dirichlet": 1}
+
+
+class TileOptions(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int32), ("bc", ctypes.c_int), ("device_budget_bytes", ctypes.c_uint64),
+                ("device_pool", ctypes.c_void_p), ("device_pool_bytes", ctypes.c_uint64),
+                ("streams", ctypes.POINTER(ctypes.c_void_p)), ("nstreams_provided", ctypes.c_int32),
+                ("nranks", ctypes.c_int32), ("rank", ctypes.c_int32),
+                ("nccl_unique_id", ctypes.c_void_p), ("sched", ctypes.c_int),
+                ("dry_run", ctypes.c_int32), ("fuse_pointwise_steps", ctypes.c_int32)]
+
+
+class TileKernel(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int), ("alpha", ctypes.c_double), ("inner_iters", ctypes.c_int32)]
+
+
+class TileStats(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_uint64) for n in ("bytes_h2d", "bytes_d2h", "bytes_halo", "n_h2d", "n_d2h",
+                                               "n_kernels", "n_halo", "hits", "misses", "evictions",
+                                               "writebacks", "steps_done")] + [
+        ("last_run_ms", ctypes.c_double), ("kernel_ms", ctypes.c_double), ("kernel_timed", ctypes.c_uint64)]
+
+    def as_dict(self):
+        return {n: getattr(self, n) for n, _ in self._fields_}
+
+
+class TileInfo(ctypes.Structure):
+    _fields_ = [("dims", ctypes.c_int64 * 3), ("local_dims", ctypes.c_int64 * 3),
+                ("tile_dims", ctypes.c_int64 * 3), ("tiles", ctypes.c_int64 * 3),
+                ("ntiles", ctypes.c_int64), ("z_offset", ctypes.c_int64), ("ghost", ctypes.c_int32),
+                ("nslots", ctypes.c_int32), ("sched", ctypes.c_int32), ("resident", ctypes.c_int32),
+                ("device_bytes", ctypes.c_uint64), ("host_bytes", ctypes.c_uint64)]
+
+    def as_dict(self):
+        out = {}
+        for n, _ in self._fields_:
+            v = getattr(self, n)
+            out[n] = tuple(v) if hasattr(v, "__len__") else v
+        return out
+
+
+class TileOp(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("stream", ctypes.c_int32), ("a", ctypes.c_int64),
+                ("b", ctypes.c_int64), ("c", ctypes.c_int64), ("d", ctypes.c_int64)]
+
+
+_P = ctypes.c_void_p
+_I64P = ctypes.POINTER(ctypes.c_int64)
+_sig = {
+    "tile_domain_create": ([_I64P, _I64P, ctypes.c_int32, ctypes.POINTER(TileOptions), ctypes.POINTER(_P)], ctypes.c_int),
+    "tile_load": ([_P, _P], ctypes.c_int),
+    "tile_host_tile": ([_P, ctypes.c_int64, ctypes.POINTER(_P)], ctypes.c_int),
+    "tile_mark_host_dirty": ([_P], ctypes.c_int),
+    "tile_run": ([_P, ctypes.POINTER(TileKernel), ctypes.c_int32, ctypes.c_int32], ctypes.c_int),
+    "tile_sync": ([_P], ctypes.c_int),
+    "tile_store": ([_P, _P], ctypes.c_int),
+    "tile_invalidate": ([_P], ctypes.c_int),
+    "tile_ghost_map": ([_P, ctypes.c_int64, _I64P, ctypes.c_int64], ctypes.c_int),
+    "tile_face_sources": ([_P, ctypes.c_int64, _I64P], ctypes.c_int),
+    "tile_get_info": ([_P, ctypes.POINTER(TileInfo)], ctypes.c_int),
+    "tile_get_stats": ([_P, ctypes.POINTER(TileStats)], ctypes.c_int),
+    "tile_reset_stats": ([_P], ctypes.c_int),
+    "tile_set_measure": ([_P, ctypes.c_int32], ctypes.c_int),
+    "tile_timer_start": ([_P], ctypes.c_int),
+    "tile_timer_stop": ([_P, ctypes.POINTER(ctypes.c_double)], ctypes.c_int),
+    "tile_set_kernel_timing": ([_P, ctypes.c_int32], ctypes.c_int),
+    "tile_trace": ([_P, ctypes.POINTER(TileOp), ctypes.c_int64, _I64P], ctypes.c_int),
+    "tile_trace_clear": ([_P], ctypes.c_int),
+    "tile_free": ([_P], ctypes.c_int),
+    "tile_last_error": ([], ctypes.c_char_p),
+    "tile_nccl_unique_id": ([_P], ctypes.c_int),
+    "tile_version": ([], ctypes.c_char_p),
+}
+EXPORTED = tuple(_sig)
+for _name, (_args, _res) in _sig.items():
+    _f = getattr(_lib, _name)
+    _f.argtypes = _args
+    _f.restype = _res
+    globals()[_name] = _f
+
+
+class TileError(RuntimeError):
+    def __init__(self, code, where):
+        self.code = code
+        msg = tile_last_error().decode()
+        super().__init__(f"{where}: {STATUS_NAMES.get(code, code)}: {msg}")
+
+
+def _check(code, where):
+    if code != TILE_OK:
+        raise TileError(code, where)
+
+
+def nccl_unique_id():
+    buf = ctypes.create_string_buffer(128)
+    _check(tile_nccl_unique_id(buf), "tile_nccl_unique_id")
+    return buf.raw
+
+
+def heat7(alpha=0.125):
+    """Heat kernel descriptor (reading R1)."""
+    return TileKernel(TILE_KERNEL_HEAT7, alpha, 0)
+
+
+def sincos(inner_iters=32):
+    """Compute-intensive kernel descriptor."""
+    return TileKernel(TILE_KERNEL_SINCOS, 0.0, inner_iters)
+
+
+class Domain:
+    """Tiled domain (tile_domain_create ... tile_free). dims and tile_dims are
+    (nx, ny, nz); arrays are NumPy float64 in [z][y][x] order."""
+
+    def __init__(self, dims, tile_dims, ghost=1, bc="periodic", device=-1, device_budget_bytes=0,
+                 sched="auto", nranks=1, rank=0, nccl_id=None, dry_run=False,
+                 fuse_pointwise_steps=True, device_pool=None, streams=None):
+        self._h = None
+        self.dims = tuple(int(v) for v in dims)
+        self.tile_dims = tuple(int(v) for v in tile_dims)
+        self.bc = BCS[bc] if isinstance(bc, str) else int(bc)
+        o = TileOptions()
+        o.device = device
+        o.bc = self.bc
+        o.device_budget_bytes = int(device_budget_bytes)
+        self._pool = device_pool  # keep the borrowed (torch) pool alive
+        if device_pool is not None:
+            o.device_pool = ctypes.c_void_p(device_pool.data_ptr())
+            o.device_pool_bytes = device_pool.numel() * device_pool.element_size()
+        self._streams = None
+        if streams:
+            arr = (ctypes.c_void_p * len(streams))(*[s.cuda_stream if hasattr(s, "cuda_stream") else s
+                                                     for s in streams])
+            self._streams = (streams, arr)
+            o.streams = ctypes.cast(arr, ctypes.POINTER(ctypes.c_void_p))
+            o.nstreams_provided = len(streams)
+        o.nranks, o.rank = nranks, rank
+        self._nccl_id = None
+        if nccl_id is not None:
+            self._nccl_id = ctypes.create_string_buffer(bytes(nccl_id), 128)
+            o.nccl_unique_id = ctypes.cast(self._nccl_id, ctypes.c_void_p)
+        o.sched = SCHEDS[sched] if isinstance(sched, str) else int(sched)
+        o.dry_run = 1 if dry_run else 0
+        o.fuse_pointwise_steps = 1 if fuse_pointwise_steps else 0
+        d = (ctypes.c_int64 * 3)(*self.dims)
+        t = (ctypes.c_int64 * 3)(*self.tile_dims)
+        h = ctypes.c_void_p()
+        _check(tile_domain_create(d, t, ghost, ctypes.byref(o), ctypes.byref(h)), "tile_domain_create")
+        self._h = h
+        self.info = self.get_info()
+
+    # -- lifecycle --------------------------------------------------------
+    def free(self):
+        if self._h is not None:
+            h, self._h = self._h, None
+            _check(tile_free(h), "tile_free")
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.free()
+
+    # -- data -------------------------------------------------------------
+    def _shape(self):
+        nx, ny, nz = self.info["local_dims"]
+        h = 2 if self.bc == TILE_BC_DIRICHLET else 0
+        return (nz + h, ny + h, nx + h)
+
+    def load(self, arr):
+        a = np.ascontiguousarray(arr, dtype=np.float64)
+        if a.shape != self._shape():
+            raise ValueError(f"expected shape {self._shape()}, got {a.shape}")
+        _check(tile_load(self._h, a.ctypes.data), "tile_load")
+
+    def store(self, out=None):
+        if out is None:
+            out = np.zeros(self._shape(), dtype=np.float64)
+        if out.shape != self._shape() or out.dtype != np.float64 or not out.flags.c_contiguous:
+            raise ValueError("bad output array")
+        _check(tile_store(self._h, out.ctypes.data), "tile_store")
+        return out
+
+    def host_tile(self, tile_id):
+        """Writable NumPy view of a tile in the pinned host store."""
+        p = ctypes.c_void_p()
+        _check(tile_host_tile(self._h, tile_id, ctypes.byref(p)), "tile_host_tile")
+        tx, ty, tz = self.tile_dims
+        buf = (ctypes.c_double * (tx * ty * tz)).from_address(p.value)
+        return np.frombuffer(buf, dtype=np.float64).reshape(tz, ty, tx)
+
+    def mark_host_dirty(self):
+        _check(tile_mark_host_dirty(self._h), "tile_mark_host_dirty")
+
+    # -- execution --------------------------------------------------------
+    def run(self, kernel, steps, nstreams=4):
+        _check(tile_run(self._h, ctypes.byref(kernel), steps, nstreams), "tile_run")
+
+    def sync(self):
+        _check(tile_sync(self._h), "tile_sync")
+
+    def invalidate(self):
+        _check(tile_invalidate(self._h), "tile_invalidate")
+
+    def set_measure(self, mode):
+        _check(tile_set_measure(self._h, mode), "tile_set_measure")
+
+    def timer_start(self):
+        _check(tile_timer_start(self._h), "tile_timer_start")
+
+    def timer_stop(self):
+        ms = ctypes.c_double()
+        _check(tile_timer_stop(self._h, ctypes.byref(ms)), "tile_timer_stop")
+        return ms.value
+
+    def set_kernel_timing(self, on=True):
+        _check(tile_set_kernel_timing(self._h, 1 if on else 0), "tile_set_kernel_timing")
+
+    # -- introspection ----------------------------------------------------
+    def ghost_map(self, tile_id):
+        tx, ty, tz = self.tile_dims
+        g = self.info["ghost"]
+        out = np.empty((tz + 2 * g, ty + 2 * g, tx + 2 * g), dtype=np.int64)
+        _check(tile_ghost_map(self._h, tile_id, out.ctypes.data_as(_I64P), out.size), "tile_ghost_map")
+        return out
+
+    def face_sources(self, tile_id):
+        out = np.empty(12, dtype=np.int64)
+        _check(tile_face_sources(self._h, tile_id, out.ctypes.data_as(_I64P)), "tile_face_sources")
+        return out.reshape(6, 2)
+
+    def get_info(self):
+        i = TileInfo()
+        _check(tile_get_info(self._h, ctypes.byref(i)), "tile_get_info")
+        return i.as_dict()
+
+    def stats(self):
+        s = TileStats()
+        _check(tile_get_stats(self._h, ctypes.byref(s)), "tile_get_stats")
+        return s.as_dict()
+
+    def reset_stats(self):
+        _check(tile_reset_stats(self._h), "tile_reset_stats")
+
+    def trace(self):
+        n = ctypes.c_int64()
+        _check(tile_trace(self._h, None, 0, ctypes.byref(n)), "tile_trace")
+        buf = (TileOp * max(1, n.value))()
+        _check(tile_trace(self._h, buf, n.value, ctypes.byref(n)), "tile_trace")
+        return [(OP_NAMES[o.kind], o.stream, o.a, o.b, o.c, o.d) for o in buf[:n.value]]
+
+    def clear_trace(self):
+        _check(tile_trace_clear(self._h), "tile_trace_clear")

@@ -1,0 +1,198 @@
+"""Replay of libtiles' dry-run op trace on the CPU (test infrastructure).
+
+The scheduler's trace (tile_trace) lists every operation it would issue on
+every stream, plus event records and waits. This replayer executes the ops
+in a RANDOM order that respects exactly the CUDA semantics the real executor
+relies on: each stream is a FIFO, and a wait blocks its stream until the
+most recent record of that event issued BEFORE the wait has executed.
+Data ops move NumPy arrays between a simulated host store, device slots and
+face buffers; kernels apply the ORACLE's arithmetic (oracle.heat_np) to a
+tile expanded with ghost cells taken from the neighbours' exported faces.
+If the scheduler misses a dependency, some random order reads stale or
+future data and the final grid differs from the untiled oracle.
+
+Ghost-source neighbours are derived here from the tile grid (periodic wrap /
+Dirichlet halo), independently of the library's own face tables.
+"""
+import random
+
+import numpy as np
+
+import oracle
+
+XM, XP, YM, YP, ZM, ZP = range(6)
+
+
+class Geometry:
+    def __init__(self, dims, tile_dims, nranks=1, rank=0, bc=0):
+        self.g = tuple(dims)
+        self.t = tuple(tile_dims)
+        self.nranks, self.rank, self.bc = nranks, rank, bc
+        self.l = (dims[0], dims[1], dims[2] // nranks)
+        self.n = tuple(self.l[a] // self.t[a] for a in range(3))
+        self.ntiles = self.n[0] * self.n[1] * self.n[2]
+        self.zoff = self.l[2] * rank
+
+    def coords(self, k):
+        return k % self.n[0], (k // self.n[0]) % self.n[1], k // (self.n[0] * self.n[1])
+
+    def tid(self, ix, iy, iz):
+        return (iz * self.n[1] + iy) * self.n[0] + ix
+
+    def neighbour(self, k, f):
+        """('tile', id) | ('dirichlet', None) | ('halo', 0|1, pos)."""
+        c = list(self.coords(k))
+        axis, step = f // 2, (1 if f & 1 else -1)
+        c[axis] += step
+        if 0 <= c[axis] < self.n[axis]:
+            return ("tile", self.tid(*c))
+        if axis < 2 or self.nranks == 1:
+            if self.bc == 1:
+                return ("dirichlet", None)
+            c[axis] %= self.n[axis]
+            return ("tile", self.tid(*c))
+        pos = c[1] * self.n[0] + c[0]
+        if step < 0:
+            if self.rank == 0 and self.bc == 1:
+                return ("dirichlet", None)
+            return ("halo", 0, pos)
+        if self.rank == self.nranks - 1 and self.bc == 1:
+            return ("dirichlet", None)
+        return ("halo", 1, pos)
+
+
+def faces_of(u):
+    return [u[:, :, 0].copy(), u[:, :, -1].copy(), u[:, 0, :].copy(), u[:, -1, :].copy(),
+            u[0].copy(), u[-1].copy()]
+
+
+class Replayer:
+    def __init__(self, geo, host_tiles, alpha, ext=None, comm=None):
+        """host_tiles: list of (tz,ty,tx) arrays (the pinned store); ext: the
+        Dirichlet extended input of this rank's slab; comm: halo callback."""
+        self.G = geo
+        self.host = [h.copy() for h in host_tiles]
+        self.alpha = alpha
+        self.ext = ext
+        self.slots = {}
+        self.faces = {}
+        self.halo = {}
+        self.comm = comm
+
+    def dirichlet_face(self, k, f):
+        G = self.G
+        ix, iy, iz = G.coords(k)
+        tx, ty, tz = G.t
+        ox, oy, oz = ix * tx + 1, iy * ty + 1, iz * tz + 1
+        e = self.ext
+        if f == XM:
+            return e[oz:oz + tz, oy:oy + ty, ox - 1]
+        if f == XP:
+            return e[oz:oz + tz, oy:oy + ty, ox + tx]
+        if f == YM:
+            return e[oz:oz + tz, oy - 1, ox:ox + tx]
+        if f == YP:
+            return e[oz:oz + tz, oy + ty, ox:ox + tx]
+        if f == ZM:
+            return e[oz - 1, oy:oy + ty, ox:ox + tx]
+        return e[oz + tz, oy:oy + ty, ox:ox + tx]
+
+    def ghost(self, k, f, par):
+        src = self.G.neighbour(k, f)
+        if src[0] == "tile":
+            return self.faces[(src[1], f ^ 1, par)]
+        if src[0] == "dirichlet":
+            return self.dirichlet_face(k, f)
+        return self.halo[(src[1], par)][src[2]]
+
+    def kernel(self, k, sin, sout, par):
+        u = self.slots[sin]
+        tz, ty, tx = u.shape
+        e = np.zeros((tz + 2, ty + 2, tx + 2))
+        e[1:-1, 1:-1, 1:-1] = u
+        e[1:-1, 1:-1, 0] = self.ghost(k, XM, par)
+        e[1:-1, 1:-1, -1] = self.ghost(k, XP, par)
+        e[1:-1, 0, 1:-1] = self.ghost(k, YM, par)
+        e[1:-1, -1, 1:-1] = self.ghost(k, YP, par)
+        e[0, 1:-1, 1:-1] = self.ghost(k, ZM, par)
+        e[-1, 1:-1, 1:-1] = self.ghost(k, ZP, par)
+        v = oracle.heat_np(e, self.alpha, 1, oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+        self.slots[sout] = v
+        for f, plane in enumerate(faces_of(v)):
+            self.faces[(k, f, par ^ 1)] = plane
+
+    def execute(self, op, snapshot_faces):
+        name, st, a, b, c, d = op
+        if name == "h2d":
+            for i in range(c):
+                self.slots[b + i] = self.host[a + i].copy()
+        elif name == "d2h":
+            for i in range(c):
+                self.host[a + i] = self.slots[b + i].copy()
+        elif name == "kernel":
+            self.kernel(a, b, c, d)
+        elif name == "extract":
+            for f, plane in enumerate(faces_of(self.slots[b])):
+                self.faces[(a, f, d)] = plane
+        elif name == "faces_h2d":
+            if d >= 0:
+                for (k, f), plane in snapshot_faces.items():
+                    self.faces[(k, f, d)] = plane.copy()
+        elif name == "pointwise":
+            self.slots[b] = oracle.sincos_c(self.slots[b], c, 1)
+        elif name == "halo":
+            self.comm(self, d)
+        # record / wait / hit / drop: no data movement
+
+    def replay(self, trace, seed):
+        rng = random.Random(seed)
+        snapshot = {(k, f): p for k in range(self.G.ntiles) for f, p in enumerate(faces_of(self.host[k]))}
+        # bind each wait to the latest preceding record of its event
+        last_rec = {}
+        bound = {}
+        for i, op in enumerate(trace):
+            if op[0] == "record":
+                last_rec[op[2]] = i
+            elif op[0] == "wait":
+                bound[i] = last_rec.get(op[2])
+        queues = {}
+        for i, op in enumerate(trace):
+            queues.setdefault(op[1], []).append(i)
+        pos = {s: 0 for s in queues}
+        done = set()
+        remaining = len(trace)
+        while remaining:
+            ready = []
+            for s, q in queues.items():
+                if pos[s] < len(q):
+                    i = q[pos[s]]
+                    op = trace[i]
+                    if op[0] == "wait" and bound[i] is not None and bound[i] not in done:
+                        continue
+                    ready.append(s)
+            if not ready:
+                raise RuntimeError("replay deadlock: no stream can make progress")
+            s = rng.choice(ready)
+            i = queues[s][pos[s]]
+            self.execute(trace[i], snapshot)
+            done.add(i)
+            pos[s] += 1
+            remaining -= 1
+
+    def grid(self):
+        G = self.G
+        tx, ty, tz = G.t
+        out = np.empty((G.l[2], G.l[1], G.l[0]))
+        for k in range(G.ntiles):
+            ix, iy, iz = G.coords(k)
+            out[iz * tz:(iz + 1) * tz, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx] = self.host[k]
+        return out
+
+
+def split_tiles(geo, u):
+    tx, ty, tz = geo.t
+    out = []
+    for k in range(geo.ntiles):
+        ix, iy, iz = geo.coords(k)
+        out.append(u[iz * tz:(iz + 1) * tz, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx].copy())
+    return out

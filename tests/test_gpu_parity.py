@@ -1,0 +1,252 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Heat is compared BIT-EXACTLY (the kernels use explicit round-to-nearest
+intrinsics in the order of reading R1, like the no-FMA oracle), which is
+stricter than the north star's 1e-12 relative max-norm. The compute-intensive
+kernel is compared within 1e-12 relative (CUDA libdevice sin/cos vs glibc,
+DESIGN.md reading R17) plus its closed form x_T ~ x_0 + K*T.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+T = pytest.importorskip("paper_conf_icpp_bastemuzas17_b200.tiles")
+ALPHA = 0.125
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    torch.cuda.init()
+
+
+def _heat(dims, td, steps, ns=2, bc="periodic", seed=42, alpha=ALPHA, runs=None, **kw):
+    nx, ny, nz = dims
+    if bc == "periodic":
+        u0 = synth.uniform_grid(nx, ny, nz, seed)
+        inp = u0
+    else:
+        inp = synth.uniform_grid(nx + 2, ny + 2, nz + 2, seed)
+    with T.Domain(dims, td, bc=bc, **kw) as d:
+        d.load(inp)
+        for s in (runs or [steps]):
+            d.run(T.heat7(alpha), s, ns)
+        out = d.store()
+        info, st = d.info, d.stats()
+    if bc == "periodic":
+        ref = oracle.heat_c(inp, alpha, steps)
+    else:
+        ref = oracle.heat_c(inp, alpha, steps, oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+        out = out[1:-1, 1:-1, 1:-1]
+    return out, ref, info, st
+
+
+def test_c1_bit_exact_and_survey_hash(golden_dir):
+    import hashlib
+    import os
+    out, ref, info, st = _heat((64, 64, 64), (32, 32, 32), 10, ns=2)
+    assert np.array_equal(out, ref)
+    rows = [l.split() for l in open(os.path.join(golden_dir, "c1_survey_values.txt"))
+            if l.strip() and not l.startswith("#")]
+    sha = [r[4] for r in rows if r[0] == "sha_u10"][0]
+    assert hashlib.sha256(out.tobytes()).hexdigest() == sha
+    assert info["sched"] == T.TILE_SCHED_RESIDENT and st["n_kernels"] > 0
+
+
+@pytest.mark.parametrize("dims,td", [((64, 32, 48), (32, 16, 16)), ((128, 64, 32), (64, 32, 8)),
+                                     ((32, 32, 32), (32, 32, 32)), ((48, 40, 20), (24, 20, 5)),
+                                     ((256, 32, 16), (128, 16, 16)), ((64, 64, 64), (16, 64, 64)),
+                                     ((512, 8, 8), (512, 8, 8))])
+def test_tile_shapes_bit_exact(dims, td):
+    out, ref, _, _ = _heat(dims, td, 7, ns=3)
+    assert np.array_equal(out, ref)
+
+
+@pytest.mark.parametrize("ns", [1, 2, 4, 8])
+def test_stream_counts_bit_exact(ns):
+    out, ref, _, _ = _heat((64, 64, 64), (32, 16, 16), 6, ns=ns)
+    assert np.array_equal(out, ref)
+
+
+def test_runs_continue_state():
+    out, ref, _, _ = _heat((64, 64, 64), (32, 32, 16), 9, runs=[4, 1, 0, 4])
+    assert np.array_equal(out, ref)
+
+
+def test_sync_baseline_bit_exact():
+    out, ref, info, _ = _heat((64, 64, 64), (32, 32, 32), 5, sched="sync")
+    assert np.array_equal(out, ref) and info["sched"] == T.TILE_SCHED_SYNC
+
+
+@pytest.mark.parametrize("alpha", [0.1, 1.0 / 6.0])
+def test_other_alphas(alpha):
+    out, ref, _, _ = _heat((64, 32, 32), (32, 16, 16), 5, alpha=alpha)
+    assert np.array_equal(out, ref)
+
+
+def test_dirichlet_random_and_linear():
+    out, ref, _, _ = _heat((64, 32, 32), (32, 16, 16), 6, bc="dirichlet", seed=5)
+    assert np.array_equal(out, ref)
+    ue = synth.linear_grid(32, 32, 32, g=1)
+    with T.Domain((32, 32, 32), (16, 16, 16), bc="dirichlet") as d:
+        d.load(ue)
+        d.run(T.heat7(), 5, 2)
+        out = d.store()
+    assert np.array_equal(out[1:-1, 1:-1, 1:-1], ue[1:-1, 1:-1, 1:-1])
+
+
+def test_sine_mode_decay():
+    import math
+    n = 64
+    u = synth.sine_grid(n, n, n)
+    with T.Domain((n, n, n), (32, 32, 32)) as d:
+        d.load(u)
+        d.run(T.heat7(), 10, 2)
+        out = d.store()
+    lam = 1 - 6 * ALPHA * (1 - math.cos(2 * math.pi / n))
+    assert np.abs(out - lam ** 10 * u).max() / np.abs(u).max() <= 1e-12
+
+
+def _budget(dims, td, nslots, bc="periodic"):
+    # the same plan in dry-run tells the persistent bytes; add nslots tiles
+    lo, hi = 1, 1 << 40
+    while lo < hi:
+        mid = (lo + hi) // 2
+        try:
+            n = T.Domain(dims, td, dry_run=True, sched="stream", bc=bc,
+                         device_budget_bytes=mid).info["nslots"]
+        except T.TileError:
+            n = -1
+        lo, hi = (lo, mid) if n >= nslots else (mid + 1, hi)
+    return lo
+
+
+@pytest.mark.parametrize("nslots,ns", [(2, 1), (3, 2), (6, 4), (17, 3)])
+def test_out_of_core_capped_bit_exact(nslots, ns):
+    dims, td = (64, 64, 64), (32, 16, 16)   # 32 tiles
+    b = _budget(dims, td, nslots)
+    out, ref, info, st = _heat(dims, td, 5, ns=ns, sched="stream", device_budget_bytes=b, runs=[3, 2])
+    assert info["sched"] == T.TILE_SCHED_STREAM and info["nslots"] == nslots
+    assert np.array_equal(out, ref)
+    assert st["misses"] > 0 and st["writebacks"] > 0
+
+
+def test_out_of_core_dirichlet():
+    dims, td = (64, 32, 32), (32, 16, 16)
+    b = _budget(dims, td, 4, bc="dirichlet")
+    out, ref, _, _ = _heat(dims, td, 4, bc="dirichlet", sched="stream", device_budget_bytes=b)
+    assert np.array_equal(out, ref)
+
+
+def test_invalidate_restreams_from_host():
+    u0 = synth.uniform_grid(64, 64, 64, 42)
+    with T.Domain((64, 64, 64), (32, 32, 32)) as d:
+        d.load(u0)
+        d.run(T.heat7(), 3, 2)
+        d.sync()
+        d.invalidate()
+        d.reset_stats()
+        d.run(T.heat7(), 2, 2)
+        out = d.store()
+        st = d.stats()
+    assert np.array_equal(out, oracle.heat_c(u0, ALPHA, 5))
+    assert st["bytes_h2d"] == 64 ** 3 * 8 and st["bytes_d2h"] == 64 ** 3 * 8
+
+
+def test_measure_modes_run():
+    u0 = synth.uniform_grid(64, 64, 64, 1)
+    with T.Domain((64, 64, 64), (32, 32, 32)) as d:
+        d.load(u0)
+        for m in (T.TILE_MEASURE_XFER_ONLY, T.TILE_MEASURE_COMP_ONLY, T.TILE_MEASURE_NORMAL):
+            d.set_measure(m)
+            d.invalidate()
+            d.run(T.heat7(), 2, 2)
+            d.sync()
+
+
+def test_kernel_timing_and_device_timer():
+    u0 = synth.uniform_grid(128, 128, 128, 1)
+    with T.Domain((128, 128, 128), (64, 64, 64)) as d:
+        d.load(u0)
+        d.run(T.heat7(), 1, 1)
+        d.sync()
+        d.set_kernel_timing(True)
+        d.reset_stats()
+        d.timer_start()
+        d.run(T.heat7(), 4, 1)
+        ms = d.timer_stop()
+        st = d.stats()
+    assert ms > 0 and st["kernel_timed"] == 4 and 0 < st["kernel_ms"] <= ms * 1.01
+
+
+# ----------------------------------------------------------- large configs
+def test_c2_full_size_cone_samples():
+    """C2 (512^3, 8^3 tiles of 64^3, resident, 4 streams) at BASELINE size,
+    in the launch configuration bench.py times; sampled blocks vs the cone
+    oracle (bit-exact), including tile seams and the periodic corner."""
+    n, steps = 512, 10
+    u0 = np.empty((n, n, n))
+    synth.fill_uniform_native(u0.ctypes.data, n, n, n, 0, n, 0, n, 0, n, 42)
+    with T.Domain((n, n, n), (64, 64, 64)) as d:
+        d.load(u0)
+        del u0
+        d.run(T.heat7(), steps, 4)
+        out = d.store()
+    rng = np.random.default_rng(1234)
+    blocks = [(0, 0, 0), (n - 2, n - 2, n - 2), (62, 63, 64), (127, 190, 255), (448, 0, 511)]
+    blocks += [tuple(int(v) for v in rng.integers(0, n, 3)) for _ in range(6)]
+    for z0, y0, x0 in blocks:
+        ref = oracle.cone_block(n, n, n, 42, ALPHA, steps, z0, y0, x0, 2, synth.uniform_block)
+        got = out[np.ix_([(z0 + i) % n for i in range(2)], [(y0 + i) % n for i in range(2)],
+                         [(x0 + i) % n for i in range(2)])]
+        assert np.array_equal(got, ref), (z0, y0, x0)
+    # invariant at any size: periodic heat conserves the sum (to rounding)
+    assert out.min() >= 0.0 and out.max() <= 1.0
+
+
+def test_sincos_parity_and_closed_form():
+    x0 = synth.uniform_grid(64, 64, 32, 7)
+    K, steps = 32, 3
+    for sched, fuse in (("auto", True), ("auto", False)):
+        with T.Domain((64, 64, 32), (32, 32, 16), sched=sched, fuse_pointwise_steps=fuse) as d:
+            d.load(x0)
+            d.run(T.sincos(K), steps, 4)
+            out = d.store()
+        ref = oracle.sincos_c(x0, K, steps)
+        assert np.abs(out - ref).max() / np.abs(ref).max() <= 1e-12
+        s = x0.copy()
+        for _ in range(K * steps):
+            s = s + 1.0
+        assert np.all(np.abs(out - s) <= 4 * np.spacing(out))
+
+
+def test_sincos_out_of_core_step_major():
+    dims, td = (64, 64, 32), (32, 32, 16)
+    b = _budget(dims, td, 3)
+    x0 = synth.uniform_grid(*dims, 7)
+    with T.Domain(dims, td, sched="stream", device_budget_bytes=b, fuse_pointwise_steps=False) as d:
+        d.load(x0)
+        d.run(T.sincos(4), 3, 2)
+        out = d.store()
+        st = d.stats()
+    ref = oracle.sincos_c(x0, 4, 3)
+    assert np.abs(out - ref).max() / np.abs(ref).max() <= 1e-12
+    assert st["misses"] >= 8 * 3 - 2 * 3
+
+
+def test_torch_pool_and_streams():
+    import torch
+    u0 = synth.uniform_grid(64, 64, 64, 42)
+    pool = torch.empty(64 << 20, dtype=torch.uint8, device="cuda")
+    streams = [torch.cuda.Stream() for _ in range(2)]
+    with T.Domain((64, 64, 64), (32, 32, 32), device_pool=pool, streams=streams) as d:
+        d.load(u0)
+        d.run(T.heat7(), 4, 2)
+        out = d.store()
+    assert np.array_equal(out, oracle.heat_c(u0, ALPHA, 4))

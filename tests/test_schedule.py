@@ -1,0 +1,257 @@
+"""Host-side logic of libtiles on a CPU (dry-run executor, no GPU).
+
+* The C ABI loads and exports every function include/tiles.h declares.
+* tile_ghost_map / tile_face_sources equal the oracle's brute-force map.
+* The scheduler's op trace, replayed in random valid orders with oracle
+  arithmetic (tests/replay.py), reproduces the untiled oracle bit-exactly for
+  resident, synchronous and out-of-core (streaming) schedules, periodic and
+  Dirichlet boundaries, several stream counts and device budgets.
+* Residency accounting: hits, misses, evictions, bytes.
+"""
+import os
+import re
+import subprocess
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from tests.replay import Geometry, Replayer, split_tiles
+
+T = pytest.importorskip("paper_conf_icpp_bastemuzas17_b200.tiles")
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ALPHA = 0.125
+
+
+def test_cabi_exports_every_declared_symbol():
+    hdr = open(os.path.join(ROOT, "include", "tiles.h")).read()
+    declared = set(re.findall(r"^\s*(?:tile_status|const char\*)\s+(tile_\w+)\s*\(", hdr, re.M))
+    assert len(declared) >= 20
+    out = subprocess.run(["nm", "-D", "--defined-only", T.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r"\bT (tile_\w+)", out))
+    assert declared <= exported, declared - exported
+    assert declared == set(T.EXPORTED)
+
+
+def test_invalid_arguments_have_no_side_effects():
+    bad = [((64, 64, 64), (24, 32, 32), 1),   # ragged
+           ((64, 64, 64), (31, 32, 32), 1),   # odd x
+           ((64, 64, 64), (32, 32, 32), 0),   # ghost < 1
+           ((64, 64, 64), (32, 32, 2), 3),    # ghost > min(tile)
+           ((0, 64, 64), (32, 32, 32), 1)]
+    for dims, td, g in bad:
+        with pytest.raises(T.TileError) as e:
+            T.Domain(dims, td, ghost=g, dry_run=True)
+        assert e.value.code == T.TILE_EINVAL
+    d = T.Domain((16, 16, 16), (8, 8, 8), dry_run=True)
+    for k, steps, ns in [(T.heat7(0.2), 1, 1), (T.heat7(0.0), 1, 1), (T.heat7(), -1, 1),
+                         (T.heat7(), 1, 0), (T.heat7(), 1, 65), (T.sincos(-1), 1, 1)]:
+        with pytest.raises(T.TileError) as e:
+            d.run(k, steps, ns)
+        assert e.value.code == T.TILE_EINVAL
+    assert d.trace() == []
+
+
+@pytest.mark.parametrize("bc", ["periodic", "dirichlet"])
+@pytest.mark.parametrize("dims,td,g", [((8, 4, 4), (2, 2, 2), 1), ((12, 8, 6), (4, 4, 3), 2),
+                                       ((6, 6, 4), (6, 6, 4), 1)])
+def test_ghost_map_matches_oracle(bc, dims, td, g):
+    b = T.BCS[bc]
+    d = T.Domain(dims, td, ghost=g, bc=bc, dry_run=True)
+    for k in range(d.info["ntiles"]):
+        assert np.array_equal(d.ghost_map(k), oracle.ghost_map(dims, td, g, k, b))
+
+
+def test_face_sources_agree_with_ghost_map():
+    # the face descriptor of face f names the tile whose cells fill the
+    # ghost layer just outside f, per the brute-force map
+    dims, td = (8, 12, 8), (4, 4, 4)
+    d = T.Domain(dims, td, dry_run=True)
+    for k in range(d.info["ntiles"]):
+        m = oracle.ghost_map(dims, td, 1, k)
+        fs = d.face_sources(k)
+        probes = {0: m[2, 2, 0], 1: m[2, 2, -1], 2: m[2, 0, 2], 3: m[2, -1, 2], 4: m[0, 2, 2], 5: m[-1, 2, 2]}
+        for f, gidx in probes.items():
+            kind, nb = fs[f]
+            assert kind == 0
+            x, y, z = gidx % 8, (gidx // 8) % 12, gidx // 96
+            assert nb == (z // 4 * 3 + y // 4) * 2 + x // 4
+
+
+def _budget_for(dims, td, nslots, **kw):
+    lo, hi = 1, 1 << 36
+    tile_bytes = td[0] * td[1] * td[2] * 8
+    while lo < hi:
+        mid = (lo + hi) // 2
+        try:
+            n = T.Domain(dims, td, dry_run=True, device_budget_bytes=mid, **kw).info["nslots"]
+        except T.TileError:
+            n = -1
+        if n >= nslots:
+            hi = mid
+        else:
+            lo = mid + 1
+    d = T.Domain(dims, td, dry_run=True, device_budget_bytes=lo, **kw)
+    assert d.info["nslots"] == nslots, (d.info["nslots"], nslots, tile_bytes)
+    return lo
+
+
+def _run_and_replay(dims, td, steps_list, nstreams, seeds=(0, 1, 2), bc="periodic", **kw):
+    nx, ny, nz = dims
+    if bc == "periodic":
+        u0 = synth.uniform_grid(nx, ny, nz, 42)
+        ext = None
+        ref = oracle.heat_c(u0, ALPHA, sum(steps_list))
+    else:
+        ext = synth.uniform_grid(nx + 2, ny + 2, nz + 2, 5)
+        u0 = ext[1:-1, 1:-1, 1:-1].copy()
+        ref = oracle.heat_c(ext, ALPHA, sum(steps_list), oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+    for seed in seeds:
+        d = T.Domain(dims, td, bc=bc, dry_run=True, **kw)
+        d.load(ext if bc == "dirichlet" else u0)
+        G = Geometry(dims, td, bc=T.BCS[bc])
+        rep = Replayer(G, split_tiles(G, u0), ALPHA, ext=ext)
+        for steps in steps_list:
+            d.clear_trace()
+            d.run(T.heat7(ALPHA), steps, nstreams)
+            d.sync()
+            rep.replay(d.trace(), seed)
+        out = rep.grid()
+        assert np.array_equal(out, ref), np.abs(out - ref).max()
+    return d
+
+
+@pytest.mark.parametrize("dims,td,ns", [((16, 16, 16), (8, 8, 8), 2), ((16, 8, 24), (8, 4, 4), 3),
+                                        ((8, 8, 8), (8, 8, 8), 1), ((16, 16, 8), (4, 8, 2), 4)])
+def test_resident_schedule_replays_to_oracle(dims, td, ns):
+    d = _run_and_replay(dims, td, [5], ns)
+    assert d.info["sched"] == T.TILE_SCHED_RESIDENT
+
+
+def test_resident_multiple_runs_and_dirichlet():
+    _run_and_replay((16, 8, 16), (8, 4, 4), [3, 2, 1], 2)
+    _run_and_replay((16, 8, 16), (8, 4, 4), [4], 2, bc="dirichlet")
+
+
+def test_sync_baseline_schedule_is_one_stream():
+    d = _run_and_replay((16, 16, 16), (8, 8, 8), [4], 4, sched="sync")
+    assert {op[1] for op in d.trace() if op[0] in ("h2d", "kernel", "d2h")} == {0}
+
+
+@pytest.mark.parametrize("nslots,ns", [(2, 1), (3, 2), (5, 1), (6, 3), (12, 2), (20, 4)])
+def test_stream_schedule_replays_to_oracle(nslots, ns):
+    dims, td = (16, 16, 16), (8, 8, 4)   # 16 tiles
+    b = _budget_for(dims, td, nslots, sched="stream")
+    d = _run_and_replay(dims, td, [3, 2], ns, seeds=(0, 7), sched="stream", device_budget_bytes=b)
+    st = d.stats()
+    assert d.info["sched"] == T.TILE_SCHED_STREAM and d.info["nslots"] == nslots
+    assert st["misses"] + st["hits"] == 16 * 5  # 3 + 2 passes over 16 tiles
+
+
+def test_stream_schedule_dirichlet():
+    dims, td = (16, 8, 16), (8, 4, 4)
+    b = _budget_for(dims, td, 5, sched="stream", bc="dirichlet")
+    _run_and_replay(dims, td, [4], 2, seeds=(3,), bc="dirichlet", sched="stream", device_budget_bytes=b)
+
+
+def test_stream_residency_accounting():
+    # 16 tiles, few slots: every pass misses every tile (no window), each
+    # tile is copied in and written back once per step
+    dims, td = (16, 16, 16), (8, 8, 4)
+    b = _budget_for(dims, td, 4, sched="stream")
+    d = T.Domain(dims, td, dry_run=True, sched="stream", device_budget_bytes=b)
+    d.load(np.zeros((16, 16, 16)))
+    d.run(T.heat7(), 3, 1)
+    d.sync()
+    st = d.stats()
+    tile_b = 8 * 8 * 4 * 8
+    faces_b = sum(16 * n * 8 for n in (4 * 8, 4 * 8, 4 * 8, 4 * 8, 8 * 8, 8 * 8))
+    # clean tiles left in a slot at the end of a pass are hits at the start
+    # of the next (snake order): at most nslots per pass boundary
+    assert st["misses"] + st["hits"] == 48 and st["hits"] <= 2 * 4
+    assert st["bytes_h2d"] == st["misses"] * tile_b + faces_b
+    assert st["bytes_d2h"] == 48 * tile_b  # write-through: no kept window
+    # generous budget: the snake order turns the kept window into hits
+    b2 = _budget_for(dims, td, 20, sched="stream")
+    d2 = T.Domain(dims, td, dry_run=True, sched="stream", device_budget_bytes=b2)
+    d2.load(np.zeros((16, 16, 16)))
+    d2.run(T.heat7(), 3, 1)
+    d2.sync()
+    s2 = d2.stats()
+    W = 20 - 4 - 2
+    assert s2["hits"] >= 2 * W and s2["misses"] + s2["hits"] == 48
+    assert s2["bytes_d2h"] == 48 * tile_b - 2 * W * tile_b  # kept tiles recomputed before write-back
+
+
+def test_stream_never_evicts_tile_in_use():
+    dims, td = (16, 16, 16), (8, 8, 4)
+    b = _budget_for(dims, td, 2, sched="stream")
+    d = T.Domain(dims, td, dry_run=True, sched="stream", device_budget_bytes=b)
+    d.load(np.zeros((16, 16, 16)))
+    d.run(T.heat7(), 2, 1)
+    d.sync()
+    owner = {}
+    for op in d.trace():
+        if op[0] == "h2d":
+            owner[op[3]] = op[2]
+        if op[0] == "kernel":
+            assert owner[op[3]] == op[2] and op[3] != op[4]
+            owner[op[4]] = op[2]
+
+
+@pytest.mark.parametrize("sched,fuse,nslots", [("auto", True, None), ("stream", True, 3),
+                                               ("stream", False, 3), ("resident", False, None)])
+def test_pointwise_schedule_replays_to_oracle(sched, fuse, nslots):
+    dims, td = (8, 8, 8), (4, 4, 4)
+    K, steps = 3, 2
+    kw = {"sched": sched, "fuse_pointwise_steps": fuse}
+    if nslots:
+        kw["device_budget_bytes"] = _budget_for(dims, td, nslots, sched=sched)
+    x0 = synth.uniform_grid(8, 8, 8, 7)
+    d = T.Domain(dims, td, dry_run=True, **kw)
+    d.load(x0)
+    d.run(T.sincos(K), steps, 2)
+    d.sync()
+    G = Geometry(dims, td)
+    rep = Replayer(G, split_tiles(G, x0), ALPHA)
+    rep.replay(d.trace(), 0)
+    ref = oracle.sincos_c(x0, K, steps)
+    assert np.array_equal(rep.grid(), ref)
+    n_pw = sum(1 for op in d.trace() if op[0] == "pointwise")
+    assert n_pw == (8 if fuse else 16)
+
+
+def test_load_store_roundtrip_and_host_tile_view():
+    dims, td = (16, 8, 8), (8, 4, 4)
+    u = synth.uniform_grid(*dims, 3)
+    d = T.Domain(dims, td, dry_run=True)
+    d.load(u)
+    assert np.array_equal(d.store(), u)
+    v = d.host_tile(3)
+    ix, iy, iz = 3 % 2, (3 // 2) % 2, 3 // 4
+    assert np.array_equal(v, u[iz * 4:(iz + 1) * 4, iy * 4:(iy + 1) * 4, ix * 8:(ix + 1) * 8])
+    v[:] = 1.5
+    d.mark_host_dirty()
+    assert (d.store()[0:4, 4:8, 8:16] == 1.5).all()
+    ue = synth.uniform_grid(18, 10, 10, 4)
+    dd = T.Domain(dims, td, bc="dirichlet", dry_run=True)
+    dd.load(ue)
+    out = np.zeros_like(ue)
+    dd.store(out)
+    assert np.array_equal(out[1:-1, 1:-1, 1:-1], ue[1:-1, 1:-1, 1:-1])
+
+
+def test_trace_ops_are_issue_ordered_per_stream():
+    d = T.Domain((16, 16, 16), (8, 8, 8), dry_run=True)
+    d.load(np.zeros((16, 16, 16)))
+    d.run(T.heat7(), 2, 2)
+    tr = d.trace()
+    # every layer kernel of step 0 follows its own layer's h2d on its stream
+    seen_h2d = set()
+    for op in tr:
+        if op[0] == "h2d":
+            seen_h2d.update(range(op[2], op[2] + op[4]))
+        if op[0] == "kernel":
+            assert op[2] in seen_h2d
