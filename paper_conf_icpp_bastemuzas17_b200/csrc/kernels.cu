@@ -54,6 +54,21 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       "l"(src), "r"(bytes), "r"(smem_u32(bar))
       : "memory");
 }
+__device__ __forceinline__ double2 lds2(uint32_t addr) {
+  double2 v;
+  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "r"(addr));
+  return v;
+}
+__device__ __forceinline__ double lds1(uint32_t addr) {
+  double v;
+  asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(addr));
+  return v;
+}
+// Streaming 128-bit global store (evict-first: the output is re-read only
+// by the next step, far beyond the L2's reach).
+__device__ __forceinline__ void stg2_stream(double* p, double2 v) {
+  asm volatile("st.global.cs.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
+}
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
@@ -66,86 +81,223 @@ __device__ __forceinline__ double heat_update(double c, double xm, double xp, do
   return __dadd_rn(c, __dmul_rn(alpha, __dsub_rn(s, __dmul_rn(6.0, c))));
 }
 
-// ---------------------------------------------------------------- heat7_tma
+// ---------------------------------------------------------------- heat7
+// Producer (one thread): stage plane z of band [y0, y0+BY) of tile `in` into
+// `dst` ((BY+2) rows of tx + 2 x-ghost columns of BY), completion on `bar`.
+// z outside [0, tz) stages the band rows of the z- / z+ ghost-source face.
+__device__ __forceinline__ void stage_plane(double* dst, uint64_t* bar, const double* in,
+                                            const double* const* gs, int z, int tx, int ty,
+                                            int tz, int y0, int BY) {
+  fence_proxy_async();
+  if (z < 0 || z >= tz) {
+    const uint32_t bytes = (uint32_t)BY * tx * 8;
+    mbar_expect_tx(bar, bytes);
+    bulk_g2s(dst + tx, gs[z < 0 ? ZM : ZP] + (size_t)y0 * tx, bytes, bar);
+    return;
+  }
+  const int rows = BY + 2;
+  const uint32_t row_b = (uint32_t)tx * 8;
+  mbar_expect_tx(bar, ((uint32_t)rows * tx + 2u * BY) * 8u);
+  const double* plane = in + (size_t)z * ty * tx;
+  bulk_g2s(dst + tx, plane + (size_t)y0 * tx, row_b * BY, bar);
+  const double* lo = y0 > 0 ? plane + (size_t)(y0 - 1) * tx : gs[YM] + (size_t)z * tx;
+  const double* hi = y0 + BY < ty ? plane + (size_t)(y0 + BY) * tx : gs[YP] + (size_t)z * tx;
+  bulk_g2s(dst, lo, row_b, bar);
+  bulk_g2s(dst + (size_t)(BY + 1) * tx, hi, row_b, bar);
+  bulk_g2s(dst + (size_t)rows * tx, gs[XM] + (size_t)z * ty + y0, (uint32_t)BY * 8, bar);
+  bulk_g2s(dst + (size_t)rows * tx + BY, gs[XP] + (size_t)z * ty + y0, (uint32_t)BY * 8, bar);
+}
+
+// Contiguous range of (tile, band, z) planes owned by this CTA.
+struct PlaneRange {
+  int64_t pb, pe;
+  __device__ PlaneRange(const HeatParams& p) {
+    const int64_t P = (int64_t)p.nitems * p.nbands * p.tz;
+    pb = P * blockIdx.x / gridDim.x;
+    pe = P * (blockIdx.x + 1) / gridDim.x;
+  }
+};
+
+// ---- specialised kernel: compile-time tile width TX, band height BY and
+// ring depth S. Each thread owns column pair c2 and rows r0 + j*RPP
+// (j < NR) of the band in EVERY plane (register z-march: z-1 and z values
+// stay in registers, 5 shared loads per pair and plane). All shared and
+// global offsets are compile-time immediates off two per-thread bases.
+template <int TX, int BY, int S>
+struct Fixed {
+  static constexpr int HALF = TX / 2;
+  static constexpr int RPP = (BY < 512 / HALF) ? BY : 512 / HALF;
+  static constexpr int NT = RPP * HALF;
+  static constexpr int NR = BY / RPP;
+  static constexpr int ROWS = BY + 2;
+  static constexpr int STAGE_ELEMS = ROWS * TX + 2 * BY;
+  static constexpr uint32_t STAGE_BYTES = STAGE_ELEMS * 8;
+  static constexpr size_t SMEM = (size_t)S * STAGE_BYTES + (size_t)S * 8;
+  static_assert(BY % RPP == 0 && NR >= 1 && NR <= 8, "bad fixed config");
+};
+
+template <int TX, int BY, int S>
+__global__ void __launch_bounds__(Fixed<TX, BY, S>::NT)
+    heat7_fixed(const __grid_constant__ HeatParams p) {
+  using C = Fixed<TX, BY, S>;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double* stage_base = reinterpret_cast<double*>(smem_raw);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw + (size_t)S * C::STAGE_BYTES);
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) mbar_init(&bars[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+
+  const int ty = p.ty, tz = p.tz;
+  const PlaneRange R(p);
+  const int c2 = (int)threadIdx.x % C::HALF;
+  const int r0 = (int)threadIdx.x / C::HALF;
+  const int x = c2 * 2;
+  const bool xlo_edge = c2 == 0, xhi_edge = c2 == C::HALF - 1;
+  const double alpha = p.alpha;
+  // per-thread shared byte offsets (stage 0, row j = 0)
+  const char* sm = reinterpret_cast<const char*>(smem_raw);
+  const int coff = ((r0 + 1) * TX + x) * 8;
+  const int xmoff = xlo_edge ? (C::ROWS * TX + r0) * 8 : coff - 8;
+  const int xpoff = xhi_edge ? (C::ROWS * TX + BY + r0) * 8 : coff + 16;
+  const int xmj = xlo_edge ? C::RPP * 8 : C::RPP * TX * 8;  // per-row steps
+  const int xpj = xhi_edge ? C::RPP * 8 : C::RPP * TX * 8;
+  uint32_t seq = 0;
+
+  for (int64_t pp = R.pb; pp < R.pe;) {
+    const int64_t col = pp / tz;
+    const int z0 = (int)(pp - col * tz);
+    const int z1 = (int)(R.pe - pp < (int64_t)(tz - z0) ? z0 + (R.pe - pp) : tz);
+    const int item_i = (int)(col / p.nbands);
+    const int y0 = (int)(col - (int64_t)item_i * p.nbands) * BY;
+    const TileItem it = p.items ? p.items[item_i] : p.inline_items[item_i];
+    const double* const* gs = p.gsrc + (size_t)it.tile * 6;
+    const int nq = z1 - z0 + 2;
+
+    auto issue = [&](int q) {
+      const uint32_t g = seq + q;
+      stage_plane(stage_base + (size_t)(g % S) * C::STAGE_ELEMS, &bars[g % S], it.in, gs,
+                  z0 - 1 + q, TX, ty, tz, y0, BY);
+    };
+    auto wait_q = [&](int q) {
+      const uint32_t g = seq + q;
+      mbar_wait(&bars[g % S], (g / S) & 1u);
+    };
+    if (threadIdx.x == 0)
+      for (int q = 0; q < (S < nq ? S : nq); ++q) issue(q);
+
+    const int64_t tile = it.tile;
+    const int yb = y0 + r0;  // global-in-tile row of j = 0
+    double* fxm = p.fexp[XM] + tile * p.face_elems[XM] + yb;
+    double* fxp = p.fexp[XP] + tile * p.face_elems[XP] + yb;
+    double* fym = p.fexp[YM] + tile * p.face_elems[YM] + x;
+    double* fyp = p.fexp[YP] + tile * p.face_elems[YP] + x;
+    double* fzm = p.fexp[ZM] + tile * p.face_elems[ZM] + (size_t)yb * TX + x;
+    double* fzp = p.fexp[ZP] + tile * p.face_elems[ZP] + (size_t)yb * TX + x;
+    const bool ylo_edge = yb == 0;                              // row j = 0
+    const bool yhi_edge = yb + (C::NR - 1) * C::RPP == ty - 1;  // row j = NR-1
+    double* obase = it.out + (size_t)yb * TX + x;
+    const size_t plane = (size_t)ty * TX;
+
+    double2 zm[C::NR], zc[C::NR];
+    wait_q(0);
+    wait_q(1);
+    {
+      const char* s0 = sm + (size_t)(seq % S) * C::STAGE_BYTES + coff;
+      const char* s1 = sm + (size_t)((seq + 1) % S) * C::STAGE_BYTES + coff;
+#pragma unroll
+      for (int j = 0; j < C::NR; ++j) {
+        zm[j] = *reinterpret_cast<const double2*>(s0 + j * C::RPP * TX * 8);
+        zc[j] = *reinterpret_cast<const double2*>(s1 + j * C::RPP * TX * 8);
+      }
+    }
+    for (int i = 0; i < z1 - z0; ++i) {
+      wait_q(i + 2);
+      const int z = z0 + i;
+      const char* cur = sm + (size_t)((seq + i + 1) % S) * C::STAGE_BYTES;
+      const char* nxt = sm + (size_t)((seq + i + 2) % S) * C::STAGE_BYTES + coff;
+      const char* cc = cur + coff;
+      const char* cxm = cur + xmoff;
+      const char* cxp = cur + xpoff;
+      double* op = obase + (size_t)z * plane;
+      const bool zlo_edge = z == 0, zhi_edge = z == tz - 1;
+#pragma unroll
+      for (int j = 0; j < C::NR; ++j) {
+        const int jo = j * C::RPP * TX * 8;
+        const double2 zp = *reinterpret_cast<const double2*>(nxt + jo);
+        const double2 ym = *reinterpret_cast<const double2*>(cc + jo - TX * 8);
+        const double2 yp = *reinterpret_cast<const double2*>(cc + jo + TX * 8);
+        const double xm = *reinterpret_cast<const double*>(cxm + j * xmj);
+        const double xp = *reinterpret_cast<const double*>(cxp + j * xpj);
+        const double2 c = zc[j];
+        double2 v;
+        v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm[j].x, zp.x, alpha);
+        v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm[j].y, zp.y, alpha);
+        stg2_stream(op + (size_t)j * C::RPP * TX, v);
+        zm[j] = c;
+        zc[j] = zp;
+        // Epilogue: export the new boundary layers (the neighbours' ghost
+        // sources for the next step). Rare, predicated.
+        if (xlo_edge) fxm[(size_t)z * ty + j * C::RPP] = v.x;
+        if (xhi_edge) fxp[(size_t)z * ty + j * C::RPP] = v.y;
+        if (j == 0 && ylo_edge) *reinterpret_cast<double2*>(fym + (size_t)z * TX) = v;
+        if (j == C::NR - 1 && yhi_edge) *reinterpret_cast<double2*>(fyp + (size_t)z * TX) = v;
+        if (zlo_edge) *reinterpret_cast<double2*>(fzm + (size_t)j * C::RPP * TX) = v;
+        if (zhi_edge) *reinterpret_cast<double2*>(fzp + (size_t)j * C::RPP * TX) = v;
+      }
+      __syncthreads();  // stage of plane z (and, at i == 0, of z-1) is free
+      if (threadIdx.x == 0) {
+        if (i == 0 && S < nq) issue(S);
+        if (i + 1 + S < nq) issue(i + 1 + S);
+      }
+    }
+    seq += (uint32_t)nq;
+    pp += z1 - z0;
+  }
+}
+
+// ---- general kernel: any even tile width / band (runtime shape). Every
+// plane is read from shared memory (7 loads per pair). Used when no
+// specialisation matches.
 template <int NT>
-__global__ void __launch_bounds__(NT) heat7_tma(const __grid_constant__ HeatParams p,
-                                                const int stages) {
+__global__ void __launch_bounds__(NT) heat7_generic(const __grid_constant__ HeatParams p,
+                                                    const int stages) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
   const int tx = p.tx, ty = p.ty, tz = p.tz, BY = p.band;
   const int rows = BY + 2;
-  const int stage_elems = rows * tx + 2 * BY;  // rows + x-ghost columns
+  const int stage_elems = rows * tx + 2 * BY;
   double* stage_base = reinterpret_cast<double*>(smem_raw);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw + (size_t)stages * stage_elems * 8);
-
   if (threadIdx.x == 0) {
     for (int s = 0; s < stages; ++s) mbar_init(&bars[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-
-  const int64_t ncols = (int64_t)p.nitems * p.nbands;
-  const int64_t P = ncols * tz;
-  const int64_t pb = P * blockIdx.x / gridDim.x;
-  const int64_t pe = P * (blockIdx.x + 1) / gridDim.x;
+  const PlaneRange R(p);
   const int half = tx >> 1;
-  const bool rowmap = (half <= NT) && (NT % half == 0);
-  const int rpp = rowmap ? NT / half : 0;
-  const int my_c2 = rowmap ? (int)threadIdx.x % half : 0;
-  const int my_r0 = rowmap ? (int)threadIdx.x / half : 0;
   const double alpha = p.alpha;
-  uint32_t seq = 0;  // planes sequenced through the ring by this CTA
-
-  for (int64_t pp = pb; pp < pe;) {
+  uint32_t seq = 0;
+  for (int64_t pp = R.pb; pp < R.pe;) {
     const int64_t col = pp / tz;
     const int z0 = (int)(pp - col * tz);
-    const int z1 = (int)(pe - pp < (int64_t)(tz - z0) ? z0 + (pe - pp) : tz);
+    const int z1 = (int)(R.pe - pp < (int64_t)(tz - z0) ? z0 + (R.pe - pp) : tz);
     const int item_i = (int)(col / p.nbands);
     const int y0 = (int)(col - (int64_t)item_i * p.nbands) * BY;
     const TileItem it = p.items ? p.items[item_i] : p.inline_items[item_i];
     const double* const* gs = p.gsrc + (size_t)it.tile * 6;
-    const int nq = z1 - z0 + 2;  // planes z0-1 .. z1
-
-    // Producer: stage plane q (z = z0-1+q) of this run.
+    const int nq = z1 - z0 + 2;
     auto issue = [&](int q) {
       const uint32_t g = seq + q;
-      const int s = (int)(g % stages);
-      double* dst = stage_base + (size_t)s * stage_elems;
-      uint64_t* bar = &bars[s];
-      const int z = z0 - 1 + q;
-      fence_proxy_async();
-      if (z < 0 || z >= tz) {  // z-ghost plane: band rows of the z- / z+ source face
-        const double* src = gs[z < 0 ? ZM : ZP] + (size_t)y0 * tx;
-        const uint32_t bytes = (uint32_t)BY * tx * 8;
-        mbar_expect_tx(bar, bytes);
-        bulk_g2s(dst + tx, src, bytes, bar);
-      } else {
-        const uint32_t row_b = (uint32_t)tx * 8;
-        const uint32_t total = (uint32_t)stage_elems * 8;
-        mbar_expect_tx(bar, total);
-        const double* plane = it.in + (size_t)z * ty * tx;
-        bulk_g2s(dst + tx, plane + (size_t)y0 * tx, row_b * BY, bar);
-        const double* lo = y0 > 0 ? plane + (size_t)(y0 - 1) * tx : gs[YM] + (size_t)z * tx;
-        const double* hi =
-            y0 + BY < ty ? plane + (size_t)(y0 + BY) * tx : gs[YP] + (size_t)z * tx;
-        bulk_g2s(dst, lo, row_b, bar);
-        bulk_g2s(dst + (size_t)(BY + 1) * tx, hi, row_b, bar);
-        bulk_g2s(dst + (size_t)rows * tx, gs[XM] + (size_t)z * ty + y0, (uint32_t)BY * 8, bar);
-        bulk_g2s(dst + (size_t)rows * tx + BY, gs[XP] + (size_t)z * ty + y0, (uint32_t)BY * 8,
-                 bar);
-      }
+      stage_plane(stage_base + (size_t)(g % stages) * stage_elems, &bars[g % stages], it.in, gs,
+                  z0 - 1 + q, tx, ty, tz, y0, BY);
     };
     auto wait_q = [&](int q) {
       const uint32_t g = seq + q;
       mbar_wait(&bars[g % stages], (g / stages) & 1u);
     };
-
-    if (threadIdx.x == 0) {
-      const int first = min(stages, nq);
-      for (int q = 0; q < first; ++q) issue(q);
-    }
-    wait_q(0);
-    wait_q(1);
-
+    if (threadIdx.x == 0)
+      for (int q = 0; q < min(stages, nq); ++q) issue(q);
     const int64_t tile = it.tile;
     double* fxm = p.fexp[XM] + tile * p.face_elems[XM];
     double* fxp = p.fexp[XP] + tile * p.face_elems[XP];
@@ -153,7 +305,8 @@ __global__ void __launch_bounds__(NT) heat7_tma(const __grid_constant__ HeatPara
     double* fyp = p.fexp[YP] + tile * p.face_elems[YP];
     double* fzm = p.fexp[ZM] + tile * p.face_elems[ZM];
     double* fzp = p.fexp[ZP] + tile * p.face_elems[ZP];
-
+    wait_q(0);
+    wait_q(1);
     for (int i = 0; i < z1 - z0; ++i) {
       wait_q(i + 2);
       const int z = z0 + i;
@@ -163,9 +316,9 @@ __global__ void __launch_bounds__(NT) heat7_tma(const __grid_constant__ HeatPara
       const double* xlo = cur + (size_t)rows * tx;
       const double* xhi = xlo + BY;
       double* out_plane = it.out + (size_t)z * ty * tx;
-
-      auto cell_pair = [&](int r, int c2) {
-        const int x = c2 << 1;
+      const int npairs = BY * half;
+      for (int e = threadIdx.x; e < npairs; e += NT) {
+        const int r = e / half, x = (e % half) << 1;
         const double* crow = cur + (size_t)(r + 1) * tx;
         const double2 c = *reinterpret_cast<const double2*>(crow + x);
         const double2 ym = *reinterpret_cast<const double2*>(cur + (size_t)r * tx + x);
@@ -178,23 +331,15 @@ __global__ void __launch_bounds__(NT) heat7_tma(const __grid_constant__ HeatPara
         v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm.x, zp.x, alpha);
         v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm.y, zp.y, alpha);
         const int y = y0 + r;
-        *reinterpret_cast<double2*>(out_plane + (size_t)y * tx + x) = v;
-        // Epilogue: export the new boundary layers (ghost sources of the
-        // neighbours for the next step).
+        stg2_stream(out_plane + (size_t)y * tx + x, v);
         if (x == 0) fxm[(size_t)z * ty + y] = v.x;
         if (x + 2 == tx) fxp[(size_t)z * ty + y] = v.y;
         if (y == 0) *reinterpret_cast<double2*>(fym + (size_t)z * tx + x) = v;
         if (y == ty - 1) *reinterpret_cast<double2*>(fyp + (size_t)z * tx + x) = v;
         if (z == 0) *reinterpret_cast<double2*>(fzm + (size_t)y * tx + x) = v;
         if (z == tz - 1) *reinterpret_cast<double2*>(fzp + (size_t)y * tx + x) = v;
-      };
-      if (rowmap) {
-        for (int r = my_r0; r < BY; r += rpp) cell_pair(r, my_c2);
-      } else {
-        const int npairs = BY * half;
-        for (int e = threadIdx.x; e < npairs; e += NT) cell_pair(e / half, e % half);
       }
-      __syncthreads();  // stage of plane z-1 is free
+      __syncthreads();
       if (threadIdx.x == 0 && i + stages < nq) issue(i + stages);
     }
     seq += (uint32_t)nq;
@@ -202,13 +347,45 @@ __global__ void __launch_bounds__(NT) heat7_tma(const __grid_constant__ HeatPara
   }
 }
 
-constexpr int kHeatThreads = 256;
+constexpr int kGenericThreads = 256;
+constexpr int kFixedStages = 5;
+
+// Specialisations: (TX, BY) -> kernel. BY is the largest of {64,32,16,8}
+// that divides ty and whose 5-stage ring fits in shared memory.
+struct FixedEntry {
+  int tx, by;
+  void (*fn)(HeatParams);
+  int nt;
+  size_t smem;
+};
+#define FIXED(TX, BY) \
+  {TX, BY, heat7_fixed<TX, BY, kFixedStages>, Fixed<TX, BY, kFixedStages>::NT, Fixed<TX, BY, kFixedStages>::SMEM}
+static const FixedEntry kFixed[] = {
+    FIXED(32, 32), FIXED(32, 16), FIXED(32, 8),  FIXED(64, 64),  FIXED(64, 32),
+    FIXED(64, 16), FIXED(64, 8),  FIXED(128, 32), FIXED(128, 16), FIXED(128, 8),
+    FIXED(256, 16), FIXED(256, 8), FIXED(512, 8)};
+#undef FIXED
+
+static const FixedEntry* find_fixed(int tx, int by) {
+  for (const auto& e : kFixed)
+    if (e.tx == tx && e.by == by) return &e;
+  return nullptr;
+}
 
 bool heat_plan(int tx, int ty, int max_smem, int* band, int* stages, size_t* smem) {
   if (tx < 2 || (tx & 1) || ty < 2 || (ty & 1)) return false;
-  // Largest even divisor of ty (<= 64) whose ring fits; prefer 5 stages
-  // (3 planes in use + 2 in flight), accept 4 or 3.
-  // A band thinner than 16 rows re-reads >12% halo rows; trade a stage for it.
+  for (int by : {64, 32, 16, 8}) {  // specialised kernels first
+    if (ty % by) continue;
+    const FixedEntry* e = find_fixed(tx, by);
+    if (e && e->smem <= (size_t)max_smem) {
+      *band = by;
+      *stages = kFixedStages;
+      *smem = e->smem;
+      return true;
+    }
+  }
+  // general kernel: largest even divisor of ty (<= 64) whose ring fits;
+  // prefer 5 stages, trade stages for bands of >= 16 rows.
   const int want = std::min(ty, 16);
   int best_by = 0, best_s = 0;
   for (int S : {5, 4, 3}) {
@@ -229,17 +406,28 @@ bool heat_plan(int tx, int ty, int max_smem, int* band, int* stages, size_t* sme
 }
 
 cudaError_t heat_configure(int tx, int ty, int band, int stages, size_t smem, int* ctas_per_sm) {
-  (void)tx; (void)ty; (void)band; (void)stages;
-  cudaError_t e = cudaFuncSetAttribute(heat7_tma<kHeatThreads>,
+  (void)ty;
+  const FixedEntry* e = stages == kFixedStages ? find_fixed(tx, band) : nullptr;
+  if (e && e->smem == smem) {
+    cudaError_t r = cudaFuncSetAttribute(e->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (r != cudaSuccess) return r;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, e->fn, e->nt, smem);
+  }
+  cudaError_t r = cudaFuncSetAttribute(heat7_generic<kGenericThreads>,
                                        cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, heat7_tma<kHeatThreads>,
-                                                       kHeatThreads, smem);
+  if (r != cudaSuccess) return r;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, heat7_generic<kGenericThreads>,
+                                                       kGenericThreads, smem);
 }
 
-cudaError_t launch_heat7(const HeatParams& p, int stages, size_t smem, int grid,
-                         cudaStream_t s) {
-  heat7_tma<kHeatThreads><<<grid, kHeatThreads, smem, s>>>(p, stages);
+cudaError_t launch_heat7(const HeatParams& p, int stages, size_t smem, int grid, cudaStream_t s) {
+  const FixedEntry* e = stages == kFixedStages ? find_fixed(p.tx, p.band) : nullptr;
+  if (e && e->smem == smem) {
+    void* args[] = {const_cast<HeatParams*>(&p)};
+    return cudaLaunchKernel(reinterpret_cast<const void*>(e->fn), dim3(grid), dim3(e->nt), args,
+                            smem, s);
+  }
+  heat7_generic<kGenericThreads><<<grid, kGenericThreads, smem, s>>>(p, stages);
   return cudaGetLastError();
 }
 

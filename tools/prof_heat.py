@@ -1,0 +1,13 @@
+"""Profiling driver: C2 resident heat steps (for ncu). Launch order:
+8 layer-batched launches (first run loads the grid), then whole-domain launches."""
+import sys, os
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import synth
+from paper_conf_icpp_bastemuzas17_b200 import tiles as T
+n = int(os.environ.get("N", "512")); t = int(os.environ.get("TILE", "64"))
+u = np.empty((n, n, n)); synth.fill_uniform_native(u.ctypes.data, n, n, n, 0, n, 0, n, 0, n, 42)
+d = T.Domain((n, n, n), (t, t, t))
+d.load(u); d.run(T.heat7(), 1, 4); d.sync()
+d.run(T.heat7(), int(os.environ.get("STEPS", "4")), 4); d.sync()
+print("prof ok")
