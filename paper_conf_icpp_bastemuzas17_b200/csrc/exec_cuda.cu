@@ -138,6 +138,7 @@ struct CudaExec final : Exec {
     p.nbands = p.ty / d.band;
     p.nitems = n;
     p.alpha = d.kernel_alpha;
+    p.cache_flags = d.heat_cache_flags;
     if (dev_items) {
       p.items = dev_items;
     } else {

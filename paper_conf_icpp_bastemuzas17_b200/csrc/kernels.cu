@@ -20,6 +20,7 @@
 #include "kernels.cuh"
 
 #include <algorithm>
+#include <cstdlib>
 
 namespace tiles {
 
@@ -34,6 +35,9 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
                "r"(bytes)
                : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   asm volatile(
@@ -69,6 +73,40 @@ __device__ __forceinline__ double lds1(uint32_t addr) {
 __device__ __forceinline__ void stg2_stream(double* p, double2 v) {
   asm volatile("st.global.cs.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(v.x), "d"(v.y) : "memory");
 }
+// L2 cache policies (createpolicy): interior planes stream through
+// (evict_first); exported faces are re-read by the neighbour in the next
+// step, and one step's faces (~9% of the grid) fit in the 126 MB L2.
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_normal() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policy_evict_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void bulk_g2s_hint(void* dst, const void* src, uint32_t bytes,
+                                              uint64_t* bar, uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint "
+      "[%0], [%1], %2, [%3], %4;" ::"r"(smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+      : "memory");
+}
+__device__ __forceinline__ void st_hint(double* p, double v, uint64_t pol) {
+  asm volatile("st.global.L2::cache_hint.f64 [%0], %1, %2;" ::"l"(p), "d"(v), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void st2_hint(double* p, double2 v, uint64_t pol) {
+  asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(p), "d"(v.x), "d"(v.y),
+               "l"(pol)
+               : "memory");
+}
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
@@ -87,25 +125,28 @@ __device__ __forceinline__ double heat_update(double c, double xm, double xp, do
 // z outside [0, tz) stages the band rows of the z- / z+ ghost-source face.
 __device__ __forceinline__ void stage_plane(double* dst, uint64_t* bar, const double* in,
                                             const double* const* gs, int z, int tx, int ty,
-                                            int tz, int y0, int BY) {
+                                            int tz, int y0, int BY, int flags) {
+  // interior and ghost faces are read once: optionally evict_first
+  const uint64_t pol = (flags & 1) ? policy_evict_first() : policy_evict_normal();
   fence_proxy_async();
   if (z < 0 || z >= tz) {
     const uint32_t bytes = (uint32_t)BY * tx * 8;
     mbar_expect_tx(bar, bytes);
-    bulk_g2s(dst + tx, gs[z < 0 ? ZM : ZP] + (size_t)y0 * tx, bytes, bar);
+    bulk_g2s_hint(dst + tx, gs[z < 0 ? ZM : ZP] + (size_t)y0 * tx, bytes, bar, pol);
     return;
   }
   const int rows = BY + 2;
   const uint32_t row_b = (uint32_t)tx * 8;
   mbar_expect_tx(bar, ((uint32_t)rows * tx + 2u * BY) * 8u);
   const double* plane = in + (size_t)z * ty * tx;
-  bulk_g2s(dst + tx, plane + (size_t)y0 * tx, row_b * BY, bar);
+  bulk_g2s_hint(dst + tx, plane + (size_t)y0 * tx, row_b * BY, bar, pol);
   const double* lo = y0 > 0 ? plane + (size_t)(y0 - 1) * tx : gs[YM] + (size_t)z * tx;
   const double* hi = y0 + BY < ty ? plane + (size_t)(y0 + BY) * tx : gs[YP] + (size_t)z * tx;
-  bulk_g2s(dst, lo, row_b, bar);
-  bulk_g2s(dst + (size_t)(BY + 1) * tx, hi, row_b, bar);
-  bulk_g2s(dst + (size_t)rows * tx, gs[XM] + (size_t)z * ty + y0, (uint32_t)BY * 8, bar);
-  bulk_g2s(dst + (size_t)rows * tx + BY, gs[XP] + (size_t)z * ty + y0, (uint32_t)BY * 8, bar);
+  bulk_g2s_hint(dst, lo, row_b, bar, pol);
+  bulk_g2s_hint(dst + (size_t)(BY + 1) * tx, hi, row_b, bar, pol);
+  bulk_g2s_hint(dst + (size_t)rows * tx, gs[XM] + (size_t)z * ty + y0, (uint32_t)BY * 8, bar, pol);
+  bulk_g2s_hint(dst + (size_t)rows * tx + BY, gs[XP] + (size_t)z * ty + y0, (uint32_t)BY * 8, bar,
+                pol);
 }
 
 // Contiguous range of (tile, band, z) planes owned by this CTA.
@@ -132,37 +173,77 @@ struct Fixed {
   static constexpr int ROWS = BY + 2;
   static constexpr int STAGE_ELEMS = ROWS * TX + 2 * BY;
   static constexpr uint32_t STAGE_BYTES = STAGE_ELEMS * 8;
-  static constexpr size_t SMEM = (size_t)S * STAGE_BYTES + (size_t)S * 8;
+  static constexpr size_t SMEM = (size_t)S * STAGE_BYTES + (size_t)S * 16;  // + full/empty
   static_assert(BY % RPP == 0 && NR >= 1 && NR <= 8, "bad fixed config");
 };
 
 template <int TX, int BY, int S>
-__global__ void __launch_bounds__(Fixed<TX, BY, S>::NT)
+__global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
     heat7_fixed(const __grid_constant__ HeatParams p) {
+  // Warp-specialised: warps 0..NT/32-1 compute, warp NT/32 is the TMA
+  // producer. full[s] completes when stage s has landed (expect_tx bytes);
+  // empty[s] completes when every consumer warp has released it. No
+  // block-wide barrier in the main loop; the producer runs up to S planes
+  // ahead, across column (run) boundaries.
   using C = Fixed<TX, BY, S>;
+  constexpr int NCW = C::NT / 32;  // consumer warps
   extern __shared__ __align__(128) unsigned char smem_raw[];
   double* stage_base = reinterpret_cast<double*>(smem_raw);
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw + (size_t)S * C::STAGE_BYTES);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + (size_t)S * C::STAGE_BYTES);
+  uint64_t* empty = full + S;
   if (threadIdx.x == 0) {
-    for (int s = 0; s < S; ++s) mbar_init(&bars[s], 1);
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], NCW);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
 
   const int ty = p.ty, tz = p.tz;
   const PlaneRange R(p);
+
+  if ((int)threadIdx.x >= C::NT) {  // ---------------- producer warp
+    if (threadIdx.x != C::NT) return;
+    uint32_t g = 0;
+    for (int64_t pp = R.pb; pp < R.pe;) {
+      const int64_t col = pp / tz;
+      const int z0 = (int)(pp - col * tz);
+      const int z1 = (int)(R.pe - pp < (int64_t)(tz - z0) ? z0 + (R.pe - pp) : tz);
+      const int item_i = (int)(col / p.nbands);
+      const int y0 = (int)(col - (int64_t)item_i * p.nbands) * BY;
+      const TileItem it = p.items ? p.items[item_i] : p.inline_items[item_i];
+      const double* const* gs = p.gsrc + (size_t)it.tile * 6;
+      for (int z = z0 - 1; z <= z1; ++z, ++g) {
+        const int s = (int)(g % S);
+        mbar_wait(&empty[s], ((g / S) & 1u) ^ 1u);
+        stage_plane(stage_base + (size_t)s * C::STAGE_ELEMS, &full[s], it.in, gs, z, TX, ty, tz,
+                    y0, BY, p.cache_flags);
+      }
+      pp += z1 - z0;
+    }
+    return;
+  }
+
+  // ------------------------------------------------------- consumer warps
+  const int lane = (int)threadIdx.x & 31;
+  const uint64_t keep = (p.cache_flags & 2) ? policy_evict_last() : policy_evict_normal();
   const int c2 = (int)threadIdx.x % C::HALF;
   const int r0 = (int)threadIdx.x / C::HALF;
   const int x = c2 * 2;
   const bool xlo_edge = c2 == 0, xhi_edge = c2 == C::HALF - 1;
   const double alpha = p.alpha;
-  // per-thread shared byte offsets (stage 0, row j = 0)
   const char* sm = reinterpret_cast<const char*>(smem_raw);
   const int coff = ((r0 + 1) * TX + x) * 8;
   const int xmoff = xlo_edge ? (C::ROWS * TX + r0) * 8 : coff - 8;
   const int xpoff = xhi_edge ? (C::ROWS * TX + BY + r0) * 8 : coff + 16;
-  const int xmj = xlo_edge ? C::RPP * 8 : C::RPP * TX * 8;  // per-row steps
+  const int xmj = xlo_edge ? C::RPP * 8 : C::RPP * TX * 8;
   const int xpj = xhi_edge ? C::RPP * 8 : C::RPP * TX * 8;
+  auto wait_g = [&](uint32_t g) { mbar_wait(&full[g % S], (g / S) & 1u); };
+  auto release_g = [&](uint32_t g) {
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[g % S]);
+  };
   uint32_t seq = 0;
 
   for (int64_t pp = R.pb; pp < R.pe;) {
@@ -172,37 +253,24 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT)
     const int item_i = (int)(col / p.nbands);
     const int y0 = (int)(col - (int64_t)item_i * p.nbands) * BY;
     const TileItem it = p.items ? p.items[item_i] : p.inline_items[item_i];
-    const double* const* gs = p.gsrc + (size_t)it.tile * 6;
     const int nq = z1 - z0 + 2;
 
-    auto issue = [&](int q) {
-      const uint32_t g = seq + q;
-      stage_plane(stage_base + (size_t)(g % S) * C::STAGE_ELEMS, &bars[g % S], it.in, gs,
-                  z0 - 1 + q, TX, ty, tz, y0, BY);
-    };
-    auto wait_q = [&](int q) {
-      const uint32_t g = seq + q;
-      mbar_wait(&bars[g % S], (g / S) & 1u);
-    };
-    if (threadIdx.x == 0)
-      for (int q = 0; q < (S < nq ? S : nq); ++q) issue(q);
-
     const int64_t tile = it.tile;
-    const int yb = y0 + r0;  // global-in-tile row of j = 0
+    const int yb = y0 + r0;
     double* fxm = p.fexp[XM] + tile * p.face_elems[XM] + yb;
     double* fxp = p.fexp[XP] + tile * p.face_elems[XP] + yb;
     double* fym = p.fexp[YM] + tile * p.face_elems[YM] + x;
     double* fyp = p.fexp[YP] + tile * p.face_elems[YP] + x;
     double* fzm = p.fexp[ZM] + tile * p.face_elems[ZM] + (size_t)yb * TX + x;
     double* fzp = p.fexp[ZP] + tile * p.face_elems[ZP] + (size_t)yb * TX + x;
-    const bool ylo_edge = yb == 0;                              // row j = 0
-    const bool yhi_edge = yb + (C::NR - 1) * C::RPP == ty - 1;  // row j = NR-1
+    const bool ylo_edge = yb == 0;
+    const bool yhi_edge = yb + (C::NR - 1) * C::RPP == ty - 1;
     double* obase = it.out + (size_t)yb * TX + x;
     const size_t plane = (size_t)ty * TX;
 
     double2 zm[C::NR], zc[C::NR];
-    wait_q(0);
-    wait_q(1);
+    wait_g(seq);
+    wait_g(seq + 1);
     {
       const char* s0 = sm + (size_t)(seq % S) * C::STAGE_BYTES + coff;
       const char* s1 = sm + (size_t)((seq + 1) % S) * C::STAGE_BYTES + coff;
@@ -212,8 +280,9 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT)
         zc[j] = *reinterpret_cast<const double2*>(s1 + j * C::RPP * TX * 8);
       }
     }
+    release_g(seq);  // plane z0-1 is in registers now
     for (int i = 0; i < z1 - z0; ++i) {
-      wait_q(i + 2);
+      wait_g(seq + i + 2);
       const int z = z0 + i;
       const char* cur = sm + (size_t)((seq + i + 1) % S) * C::STAGE_BYTES;
       const char* nxt = sm + (size_t)((seq + i + 2) % S) * C::STAGE_BYTES + coff;
@@ -239,19 +308,16 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT)
         zc[j] = zp;
         // Epilogue: export the new boundary layers (the neighbours' ghost
         // sources for the next step). Rare, predicated.
-        if (xlo_edge) fxm[(size_t)z * ty + j * C::RPP] = v.x;
-        if (xhi_edge) fxp[(size_t)z * ty + j * C::RPP] = v.y;
-        if (j == 0 && ylo_edge) *reinterpret_cast<double2*>(fym + (size_t)z * TX) = v;
-        if (j == C::NR - 1 && yhi_edge) *reinterpret_cast<double2*>(fyp + (size_t)z * TX) = v;
-        if (zlo_edge) *reinterpret_cast<double2*>(fzm + (size_t)j * C::RPP * TX) = v;
-        if (zhi_edge) *reinterpret_cast<double2*>(fzp + (size_t)j * C::RPP * TX) = v;
+        if (xlo_edge) st_hint(fxm + (size_t)z * ty + j * C::RPP, v.x, keep);
+        if (xhi_edge) st_hint(fxp + (size_t)z * ty + j * C::RPP, v.y, keep);
+        if (j == 0 && ylo_edge) st2_hint(fym + (size_t)z * TX, v, keep);
+        if (j == C::NR - 1 && yhi_edge) st2_hint(fyp + (size_t)z * TX, v, keep);
+        if (zlo_edge) st2_hint(fzm + (size_t)j * C::RPP * TX, v, keep);
+        if (zhi_edge) st2_hint(fzp + (size_t)j * C::RPP * TX, v, keep);
       }
-      __syncthreads();  // stage of plane z (and, at i == 0, of z-1) is free
-      if (threadIdx.x == 0) {
-        if (i == 0 && S < nq) issue(S);
-        if (i + 1 + S < nq) issue(i + 1 + S);
-      }
+      release_g(seq + i + 1);  // plane z no longer read (its centre is in registers)
     }
+    release_g(seq + nq - 1);  // plane z1 (last z+1 neighbour)
     seq += (uint32_t)nq;
     pp += z1 - z0;
   }
@@ -290,7 +356,7 @@ __global__ void __launch_bounds__(NT) heat7_generic(const __grid_constant__ Heat
     auto issue = [&](int q) {
       const uint32_t g = seq + q;
       stage_plane(stage_base + (size_t)(g % stages) * stage_elems, &bars[g % stages], it.in, gs,
-                  z0 - 1 + q, tx, ty, tz, y0, BY);
+                  z0 - 1 + q, tx, ty, tz, y0, BY, p.cache_flags);
     };
     auto wait_q = [&](int q) {
       const uint32_t g = seq + q;
@@ -348,22 +414,23 @@ __global__ void __launch_bounds__(NT) heat7_generic(const __grid_constant__ Heat
 }
 
 constexpr int kGenericThreads = 256;
-constexpr int kFixedStages = 5;
 
 // Specialisations: (TX, BY) -> kernel. BY is the largest of {64,32,16,8}
 // that divides ty and whose 5-stage ring fits in shared memory.
 struct FixedEntry {
-  int tx, by;
+  int tx, by, stages;
   void (*fn)(HeatParams);
   int nt;
   size_t smem;
 };
-#define FIXED(TX, BY) \
-  {TX, BY, heat7_fixed<TX, BY, kFixedStages>, Fixed<TX, BY, kFixedStages>::NT, Fixed<TX, BY, kFixedStages>::SMEM}
+#define FIXED(TX, BY, S) \
+  {TX, BY, S, heat7_fixed<TX, BY, S>, Fixed<TX, BY, S>::NT + 32, Fixed<TX, BY, S>::SMEM}
 static const FixedEntry kFixed[] = {
-    FIXED(32, 32), FIXED(32, 16), FIXED(32, 8),  FIXED(64, 64),  FIXED(64, 32),
-    FIXED(64, 16), FIXED(64, 8),  FIXED(128, 32), FIXED(128, 16), FIXED(128, 8),
-    FIXED(256, 16), FIXED(256, 8), FIXED(512, 8)};
+    FIXED(32, 32, 6),  FIXED(32, 16, 6),  FIXED(32, 8, 6),   FIXED(64, 64, 4),
+    FIXED(64, 64, 6),  FIXED(64, 64, 5),  FIXED(64, 32, 4),  FIXED(64, 32, 3),
+    FIXED(64, 32, 6),  FIXED(64, 16, 6),  FIXED(64, 8, 6),   FIXED(128, 32, 6),
+    FIXED(128, 16, 6), FIXED(128, 8, 6),  FIXED(256, 16, 6), FIXED(256, 8, 6),
+    FIXED(512, 8, 5)};
 #undef FIXED
 
 static const FixedEntry* find_fixed(int tx, int by) {
@@ -372,14 +439,32 @@ static const FixedEntry* find_fixed(int tx, int by) {
   return nullptr;
 }
 
+static const FixedEntry* find_fixed_s(int tx, int by, int st) {
+  for (const auto& e : kFixed)
+    if (e.tx == tx && e.by == by && e.stages == st) return &e;
+  return nullptr;
+}
+
 bool heat_plan(int tx, int ty, int max_smem, int* band, int* stages, size_t* smem) {
   if (tx < 2 || (tx & 1) || ty < 2 || (ty & 1)) return false;
+  // tuning override: TILES_HEAT_BAND / TILES_HEAT_STAGES select a specialisation
+  if (const char* eb = std::getenv("TILES_HEAT_BAND")) {
+    const char* es = std::getenv("TILES_HEAT_STAGES");
+    const int by = std::atoi(eb), st = es ? std::atoi(es) : 0;
+    const FixedEntry* e = st ? find_fixed_s(tx, by, st) : find_fixed(tx, by);
+    if (e && ty % by == 0 && e->smem <= (size_t)max_smem) {
+      *band = by;
+      *stages = e->stages;
+      *smem = e->smem;
+      return true;
+    }
+  }
   for (int by : {64, 32, 16, 8}) {  // specialised kernels first
     if (ty % by) continue;
     const FixedEntry* e = find_fixed(tx, by);
     if (e && e->smem <= (size_t)max_smem) {
       *band = by;
-      *stages = kFixedStages;
+      *stages = e->stages;
       *smem = e->smem;
       return true;
     }
@@ -407,7 +492,7 @@ bool heat_plan(int tx, int ty, int max_smem, int* band, int* stages, size_t* sme
 
 cudaError_t heat_configure(int tx, int ty, int band, int stages, size_t smem, int* ctas_per_sm) {
   (void)ty;
-  const FixedEntry* e = stages == kFixedStages ? find_fixed(tx, band) : nullptr;
+  const FixedEntry* e = find_fixed_s(tx, band, stages);
   if (e && e->smem == smem) {
     cudaError_t r = cudaFuncSetAttribute(e->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (r != cudaSuccess) return r;
@@ -421,7 +506,7 @@ cudaError_t heat_configure(int tx, int ty, int band, int stages, size_t smem, in
 }
 
 cudaError_t launch_heat7(const HeatParams& p, int stages, size_t smem, int grid, cudaStream_t s) {
-  const FixedEntry* e = stages == kFixedStages ? find_fixed(p.tx, p.band) : nullptr;
+  const FixedEntry* e = find_fixed_s(p.tx, p.band, stages);
   if (e && e->smem == smem) {
     void* args[] = {const_cast<HeatParams*>(&p)};
     return cudaLaunchKernel(reinterpret_cast<const void*>(e->fn), dim3(grid), dim3(e->nt), args,

@@ -38,6 +38,8 @@ struct HeatParams {
   // z-faces [y][x].
   double* fexp[6];
   int64_t face_elems[6];
+  // L2 policy bits: 1 = TMA loads evict_first, 2 = face exports evict_last
+  int32_t cache_flags;
 };
 
 struct SincosParams {

@@ -10,6 +10,7 @@
 //     paper's global `acc wait` (difference D3)
 //   D2H + synchronize before host access          -> domain_sync
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <set>
 
@@ -60,7 +61,7 @@ Status domain_create(const int64_t dims[3], const int64_t tdims[3], int ghost,
 
   int band = 0, stages = 0;
   size_t smem = 0;
-  if (!heat_plan((int)G.t[0], (int)G.t[1], 200 * 1024, &band, &stages, &smem))
+  if (!heat_plan((int)G.t[0], (int)G.t[1], 227 * 1024, &band, &stages, &smem))
     return make_err(TILE_EINVAL, "tile x extent too large to stage a 2-row band in shared memory");
 
   Domain* d = new Domain();
@@ -69,6 +70,7 @@ Status domain_create(const int64_t dims[3], const int64_t tdims[3], int ghost,
   d->band = band;
   d->stages = stages;
   d->heat_smem = smem;
+  if (const char* cf = std::getenv("TILES_HEAT_CACHE")) d->heat_cache_flags = std::atoi(cf);
   if (opt.dry_run) {
     d->exec = make_dry_exec();
   } else {

@@ -152,6 +152,7 @@ struct Domain {
   // kernel plan
   int band = 0, stages = 0, heat_grid = 0, sm_count = 148;
   size_t heat_smem = 0;
+  int heat_cache_flags = 2;               // L2 policy bits (kernels.cuh): exports evict_last
 
   // run bookkeeping
   struct BatchRec { int64_t L0, L1; int stream; };
