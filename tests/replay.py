@@ -196,3 +196,82 @@ def split_tiles(geo, u):
         ix, iy, iz = geo.coords(k)
         out.append(u[iz * tz:(iz + 1) * tz, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx].copy())
     return out
+
+
+# ------------------------------------------------------------ multi-rank
+def halo_payload(rep, par):
+    """Faces a rank sends in the halo exchange of parity `par`: its top
+    layer's z+ exports and bottom layer's z- exports (layer-position order)."""
+    G = rep.G
+    lt = G.n[0] * G.n[1]
+    top = [rep.faces[((G.n[2] - 1) * lt + pos, ZP, par)] for pos in range(lt)]
+    bot = [rep.faces[(pos, ZM, par)] for pos in range(lt)]
+    return top, bot
+
+
+def halo_peers(G):
+    R, r = G.nranks, G.rank
+    per = G.bc == 0
+    up = (r + 1) % R if (per or r < R - 1) else None
+    dn = (r - 1) % R if (per or r > 0) else None
+    return up, dn
+
+
+def replay_ranks(reps, traces, seed):
+    """Joint random replay of several ranks' traces; the k-th halo op of
+    every rank executes together (a collective)."""
+    rng = random.Random(seed)
+    state = []
+    for rep, tr in zip(reps, traces):
+        last_rec, bound = {}, {}
+        for i, op in enumerate(tr):
+            if op[0] == "record":
+                last_rec[op[2]] = i
+            elif op[0] == "wait":
+                bound[i] = last_rec.get(op[2])
+        queues = {}
+        for i, op in enumerate(tr):
+            queues.setdefault(op[1], []).append(i)
+        snapshot = {(k, f): p for k in range(rep.G.ntiles) for f, p in enumerate(faces_of(rep.host[k]))}
+        state.append({"bound": bound, "queues": queues, "pos": {s: 0 for s in queues}, "done": set(),
+                      "snap": snapshot})
+    remaining = sum(len(t) for t in traces)
+    while remaining:
+        ready, halo_heads = [], {}
+        for r, (st, tr) in enumerate(zip(state, traces)):
+            for s, q in st["queues"].items():
+                if st["pos"][s] >= len(q):
+                    continue
+                i = q[st["pos"][s]]
+                op = tr[i]
+                if op[0] == "wait" and st["bound"][i] is not None and st["bound"][i] not in st["done"]:
+                    continue
+                if op[0] == "halo":
+                    halo_heads[r] = (s, i)
+                else:
+                    ready.append((r, s, i))
+        if len(halo_heads) == len(reps):
+            ready.append(("halo", None, None))
+        if not ready:
+            raise RuntimeError("multi-rank replay deadlock")
+        pick = rng.choice(ready)
+        if pick[0] == "halo":
+            par = traces[0][halo_heads[0][1]][5]
+            payload = [halo_payload(rep, par) for rep in reps]
+            for r, rep in enumerate(reps):
+                assert traces[r][halo_heads[r][1]][5] == par
+                up, dn = halo_peers(rep.G)
+                if dn is not None:
+                    rep.halo[(0, par)] = payload[dn][0]   # rank below's top layer
+                if up is not None:
+                    rep.halo[(1, par)] = payload[up][1]   # rank above's bottom layer
+                s, i = halo_heads[r]
+                state[r]["done"].add(i)
+                state[r]["pos"][s] += 1
+                remaining -= 1
+            continue
+        r, s, i = pick
+        reps[r].execute(traces[r][i], state[r]["snap"])
+        state[r]["done"].add(i)
+        state[r]["pos"][s] += 1
+        remaining -= 1

@@ -1,0 +1,182 @@
+"""Multi-GPU (z-slab) host logic on CPU, no GPU and no NCCL.
+
+1. In-process: G dry-run ranks' op traces are replayed jointly in random
+   valid orders (tests/replay.py); the k-th halo op of every rank executes as
+   one collective. The assembled slabs must equal the untiled oracle on the
+   global grid, bit-exactly.
+2. world_size 2 over gloo (torch.distributed, 127.0.0.1): each process
+   replays its own rank's trace and performs the halo exchange with gloo
+   send/recv, exactly as libtiles pairs its NCCL sends/receives.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from tests.replay import Geometry, Replayer, halo_payload, halo_peers, replay_ranks, split_tiles
+
+T = pytest.importorskip("paper_conf_icpp_bastemuzas17_b200.tiles")
+ALPHA = 0.125
+
+
+def _global(dims, bc):
+    nx, ny, nz = dims
+    if bc == "periodic":
+        u = synth.uniform_grid(nx, ny, nz, 42)
+        return u, None, oracle.heat_c
+    ext = synth.uniform_grid(nx + 2, ny + 2, nz + 2, 5)
+    return ext[1:-1, 1:-1, 1:-1].copy(), ext, oracle.heat_c
+
+
+def _rank_domain(dims, td, G, r, bc, ext, u, **kw):
+    d = T.Domain(dims, td, bc=bc, nranks=G, rank=r, dry_run=True, **kw)
+    nzl = dims[2] // G
+    if bc == "dirichlet":
+        d.load(ext[r * nzl:(r + 1) * nzl + 2])
+    else:
+        d.load(u[r * nzl:(r + 1) * nzl])
+    return d
+
+
+@pytest.mark.parametrize("G", [2, 3, 4])
+@pytest.mark.parametrize("bc", ["periodic", "dirichlet"])
+@pytest.mark.parametrize("sched", ["resident", "stream"])
+def test_slab_replay_matches_global_oracle(G, bc, sched):
+    dims, td = (16, 8, 8 * G), (8, 4, 4)
+    u, ext, _ = _global(dims, bc)
+    steps = [3, 2]
+    kw = {"sched": sched}
+    if sched == "stream":
+        kw["device_budget_bytes"] = 1  # replaced below by the minimum budget
+    doms, reps = [], []
+    nzl = dims[2] // G
+    for r in range(G):
+        if sched == "stream":
+            # smallest budget giving 3 slots
+            lo, hi = 1, 1 << 32
+            while lo < hi:
+                mid = (lo + hi) // 2
+                try:
+                    n = T.Domain(dims, td, bc=bc, nranks=G, rank=r, dry_run=True, sched="stream",
+                                 device_budget_bytes=mid).info["nslots"]
+                except T.TileError:
+                    n = -1
+                lo, hi = (lo, mid) if n >= 3 else (mid + 1, hi)
+            kw["device_budget_bytes"] = lo
+        d = _rank_domain(dims, td, G, r, bc, ext, u, **kw)
+        doms.append(d)
+        geo = Geometry(dims, td, nranks=G, rank=r, bc=T.BCS[bc])
+        rext = ext[r * nzl:(r + 1) * nzl + 2] if ext is not None else None
+        reps.append(Replayer(geo, split_tiles(geo, u[r * nzl:(r + 1) * nzl]), ALPHA, ext=rext))
+    for s in steps:
+        traces = []
+        for d in doms:
+            d.clear_trace()
+            d.run(T.heat7(ALPHA), s, 2)
+            d.sync()
+            traces.append(d.trace())
+        assert all(sum(op[0] == "halo" for op in tr) == sum(op[0] == "halo" for op in traces[0])
+                   for tr in traces)
+        replay_ranks(reps, traces, seed=s * 7 + G)
+    out = np.concatenate([rep.grid() for rep in reps], axis=0)
+    if bc == "periodic":
+        ref = oracle.heat_c(u, ALPHA, sum(steps))
+    else:
+        ref = oracle.heat_c(ext, ALPHA, sum(steps), oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+    assert np.array_equal(out, ref), np.abs(out - ref).max()
+
+
+def test_slab_geometry_and_face_kinds():
+    d = T.Domain((16, 16, 32), (8, 8, 4), nranks=4, rank=1, dry_run=True)
+    info = d.info
+    assert info["local_dims"] == (16, 16, 8) and info["z_offset"] == 8 and info["tiles"] == (2, 2, 2)
+    fs = d.face_sources(0)           # bottom layer: z- from the rank below
+    assert tuple(fs[4]) == (2, 0)
+    fs = d.face_sources(7)           # top layer, position 3: z+ from the rank above
+    assert tuple(fs[5]) == (3, 3)
+    dd = T.Domain((16, 16, 32), (8, 8, 4), nranks=4, rank=0, bc="dirichlet", dry_run=True)
+    assert tuple(dd.face_sources(0)[4]) == (1, 0)   # global bottom: Dirichlet fixed face
+    m = d.ghost_map(0)
+    assert m[0, 1, 1] == (7 * 16 + 0) * 16 + 0      # z = 8 - 1 = 7 (rank 0's top plane)
+
+
+# ----------------------------------------------------------------- gloo
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _gloo_worker(rank, world, port, bc, sched, out_q):
+    import torch
+    import torch.distributed as dist
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    try:
+        dims, td = (16, 8, 16), (8, 4, 4)
+        u, ext, _ = _global(dims, bc)
+        nzl = dims[2] // world
+        kw = {"sched": sched}
+        if sched == "stream":
+            kw["device_budget_bytes"] = 600_000
+        d = _rank_domain(dims, td, world, rank, bc, ext, u, **kw)
+        geo = Geometry(dims, td, nranks=world, rank=rank, bc=T.BCS[bc])
+        rext = ext[rank * nzl:(rank + 1) * nzl + 2] if ext is not None else None
+
+        def comm(rep, par):
+            top, bot = halo_payload(rep, par)
+            up, dn = halo_peers(rep.G)
+            shape = top[0].shape
+            send_top = torch.from_numpy(np.stack(top))
+            send_bot = torch.from_numpy(np.stack(bot))
+            recv_lo = torch.empty((len(top),) + shape, dtype=torch.float64)
+            recv_hi = torch.empty_like(recv_lo)
+            ops = []
+            # same pairing as comm_nccl.cpp: sends first, then receives
+            if up is not None:
+                ops.append(dist.P2POp(dist.isend, send_top, up))
+            if dn is not None:
+                ops.append(dist.P2POp(dist.isend, send_bot, dn))
+            if dn is not None:
+                ops.append(dist.P2POp(dist.irecv, recv_lo, dn))
+            if up is not None:
+                ops.append(dist.P2POp(dist.irecv, recv_hi, up))
+            for w in dist.batch_isend_irecv(ops):
+                w.wait()
+            if dn is not None:
+                rep.halo[(0, par)] = list(recv_lo.numpy())
+            if up is not None:
+                rep.halo[(1, par)] = list(recv_hi.numpy())
+
+        rep = Replayer(geo, split_tiles(geo, u[rank * nzl:(rank + 1) * nzl]), ALPHA, ext=rext, comm=comm)
+        d.run(T.heat7(ALPHA), 4, 2)
+        d.sync()
+        rep.replay(d.trace(), seed=rank + 11)
+        if bc == "periodic":
+            ref = oracle.heat_c(u, ALPHA, 4)
+        else:
+            ref = oracle.heat_c(ext, ALPHA, 4, oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+        ok = np.array_equal(rep.grid(), ref[rank * nzl:(rank + 1) * nzl])
+        out_q.put((rank, bool(ok)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("bc,sched", [("periodic", "resident"), ("dirichlet", "stream"),
+                                      ("periodic", "stream")])
+def test_gloo_world2_halo_exchange(bc, sched):
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_gloo_worker, args=(r, 2, port, bc, sched, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(180)
+    res = dict(q.get(timeout=5) for _ in range(2))
+    assert res == {0: True, 1: True}
