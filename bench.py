@@ -164,20 +164,229 @@ def run_reference(args):
     return 0
 
 
+def fill_tiles(dom, Tl, synth, gdims, td, z_base, seed):
+    """Write the generator's values straight into the pinned tile store."""
+    info = dom.info
+    ntx, nty, ntz = info["tiles"]
+    for k in range(info["ntiles"]):
+        ix, iy, iz = k % ntx, (k // ntx) % nty, k // (ntx * nty)
+        v = dom.host_tile(k)
+        synth.fill_uniform_native(v.ctypes.data, gdims[0], gdims[1], gdims[2], z_base + iz * td[2], td[2],
+                                  iy * td[1], td[1], ix * td[0], td[0], seed)
+    dom.mark_host_dirty()
+
+
+def run_stream_leg(args):
+    """C3: heat 2048^3 fp64 out-of-core: the device budget is CAPPED (the
+    paper's "limiting GPU memory" method) so only a fraction of the
+    tiles fits; every step streams the tiles through the slot pool.
+    value = e2e: tile_invalidate + tile_run(T) + tile_sync from pinned host."""
+    import torch
+    from paper_conf_icpp_bastemuzas17_b200 import tiles as Tl
+    import synth
+    n = args.n or 2048
+    td = (256, 256, 256) if n % 256 == 0 else (n // 8, n // 8, n // 8)
+    T = args.T if args.T is not None else 2
+    ns = args.nstreams or 4
+    budget = int((args.budget_gb or 12.0) * (1 << 30))
+    gdims = (n, n, n)
+    cells = n ** 3
+    torch.cuda.set_device(0)
+    t0 = time.perf_counter()
+    dom = Tl.Domain(gdims, td, ghost=1, device=0, sched="stream", device_budget_bytes=budget)
+    t_alloc = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    fill_tiles(dom, Tl, synth, gdims, td, 0, 42)
+    t_fill = time.perf_counter() - t0
+    k = Tl.heat7(ALPHA)
+    for _ in range(args.warmup):
+        dom.invalidate()
+        dom.run(k, T, ns)
+        dom.sync()
+    dom.reset_stats()
+    torch.cuda.synchronize()
+    tot = 0.0
+    with Clocks(0) as clk:
+        for _ in range(args.steps):
+            dom.invalidate()
+            dom.timer_start()
+            dom.run(k, T, ns)
+            dom.sync()
+            tot += dom.timer_stop()
+    st = dom.stats()
+    val = cells * T * args.steps / (tot / 1e3) / 1e9
+    info = dom.info
+    # overlap: same schedule, transfers only / kernels only
+    def leg(mode, steps=1):
+        dom.set_measure(mode)
+        t = 0.0
+        for _ in range(steps):
+            dom.invalidate()
+            dom.timer_start()
+            dom.run(k, T, ns)
+            dom.sync()
+            t += dom.timer_stop()
+        dom.set_measure(Tl.TILE_MEASURE_NORMAL)
+        return t / steps
+    xo, co = leg(Tl.TILE_MEASURE_XFER_ONLY), leg(Tl.TILE_MEASURE_COMP_ONLY)
+    wall = tot / args.steps
+    hidden = max(0.0, min(1.0, (xo + co - wall) / min(xo, co)))
+    dom.free()
+    bw = pcie_bandwidth(torch)
+    bidir = pcie_bidir(torch)
+    Bh, Bd = st["bytes_h2d"] / args.steps, st["bytes_d2h"] / args.steps
+    t_link = max(Bh / (bw["h2d"] * 1e9), Bd / (bw["d2h"] * 1e9), (Bh + Bd) / (bidir * 1e9))
+    line = {"metric": METRIC, "value": val, "unit": "Gcell-updates/s", "n_gpus": 1, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": wall, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"C3 heat fp64 {n}^3 out-of-core (device budget capped at "
+                                   f"{budget / 2**30:.1f} GiB, paper method P:L232), T={T}",
+                       "dims": gdims, "tile_dims": td, "T": T, "nstreams": ns, "nslots": info["nslots"],
+                       "ntiles": info["ntiles"], "host_gb": info["host_bytes"] / 1e9,
+                       "device_gb": info["device_bytes"] / 1e9,
+                       "value_def": "e2e streaming: invalidate + tile_run(T) + tile_sync from pinned host",
+                       "setup_s": {"pinned_alloc": t_alloc, "generate": t_fill}},
+            "e2e": {"value": val, "unit": "Gcell-updates/s", "h2d_bytes_per_step": int(Bh),
+                    "d2h_bytes_per_step": int(Bd), "ms_per_step": wall},
+            "gpu_launches": st["n_kernels"] // max(1, args.steps),
+            "residency": {k2: st[k2] // args.steps for k2 in ("hits", "misses", "evictions", "writebacks")},
+            "overlap": {"hidden_frac": hidden, "t_wall_ms": wall, "t_xfer_only_ms": xo, "t_comp_only_ms": co},
+            "roofline": {"bound": "pcie", "form": "streaming: max(Bh/BWh, Bd/BWd, (Bh+Bd)/BWbidir)",
+                         "t_link_ms": t_link * 1e3, "frac": t_link * 1e3 / wall,
+                         "achieved": (Bh + Bd) / (wall / 1e3) / 1e9, "peak": bidir, "unit": "GB/s",
+                         "pcie_gbs": {**bw, "bidir": bidir}},
+            "clocks": clk.summary()}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def pcie_bidir(torch, nbytes=256 << 20, reps=5):
+    h1 = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
+    h2 = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
+    d1 = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    d2 = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    best = 0
+    for _ in range(reps):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        with torch.cuda.stream(s1):
+            d1.copy_(h1, non_blocking=True)
+        with torch.cuda.stream(s2):
+            h2.copy_(d2, non_blocking=True)
+        torch.cuda.synchronize()
+        best = max(best, 2 * nbytes / (time.perf_counter() - t0) / 1e9)
+    return best
+
+
+def run_sincos_leg(args):
+    """C4: the compute-intensive kernel at 1024^3 fp64, 8^3
+    tiles of 128^3, K = 32 inner iterations (reading R12), T = 10 outer steps
+    fused per residency pass; nstreams sweep 1..8 (e2e from pinned host)."""
+    import torch
+    from paper_conf_icpp_bastemuzas17_b200 import tiles as Tl
+    import synth
+    n = args.n or 1024
+    td = (n // 8, n // 8, n // 8)
+    T = args.T if args.T is not None else 10
+    K = args.K
+    gdims = (n, n, n)
+    cells = n ** 3
+    torch.cuda.set_device(0)
+    dom = Tl.Domain(gdims, td, ghost=1, device=0)
+    fill_tiles(dom, Tl, synth, gdims, td, 0, 7)
+    k = Tl.sincos(K)
+    sweep = {}
+    for ns in ([int(v) for v in args.sweep.split(",")] if args.sweep else [1, 2, 4, 8]):
+        for _ in range(max(1, args.warmup)):
+            dom.invalidate()
+            dom.run(k, T, ns)
+            dom.sync()
+        tot = 0.0
+        for _ in range(args.steps):
+            dom.invalidate()
+            dom.timer_start()
+            dom.run(k, T, ns)
+            dom.sync()
+            tot += dom.timer_stop()
+        sweep[ns] = cells * T * args.steps / (tot / 1e3) / 1e9
+    ns_best = max(sweep, key=sweep.get)
+    ns = args.nstreams or 4
+    # resident (compute only) with kernel timing, and the overlap legs
+    dom.invalidate()
+    dom.run(k, T, ns)
+    dom.sync()
+    dom.set_kernel_timing(True)
+    dom.reset_stats()
+    with Clocks(0) as clk:
+        dom.timer_start()
+        for _ in range(args.steps):
+            dom.run(k, T, ns)
+        ms_res = dom.timer_stop()
+    st = dom.stats()
+    dom.set_kernel_timing(False)
+    dom.sync()
+    def leg(mode):
+        dom.set_measure(mode)
+        dom.invalidate()
+        dom.timer_start()
+        dom.run(k, T, ns)
+        dom.sync()
+        t = dom.timer_stop()
+        dom.set_measure(Tl.TILE_MEASURE_NORMAL)
+        return t
+    xo, co = leg(Tl.TILE_MEASURE_XFER_ONLY), leg(Tl.TILE_MEASURE_COMP_ONLY)
+    wall = cells * T / (sweep[ns] * 1e9) * 1e3 if ns in sweep else None
+    hidden = max(0.0, min(1.0, (xo + co - wall) / min(xo, co))) if wall else None
+    dom.free()
+    value = cells * T * args.steps / (ms_res / 1e3) / 1e9
+    # achieved over the resident wall time (per-launch event durations of
+    # concurrent streams overlap, so their sum is not a time)
+    iters_per_s = cells * K * T * args.steps / (ms_res / 1e3)
+    prof = os.path.join(ROOT, "profiles", "sincos_fp64.json")
+    roof = {"bound": "alu", "achieved": iters_per_s / 1e9, "unit": "Gcell-iter/s", "peak": None, "frac": None,
+            "traffic": None, "kernel": "sincos_iter"}
+    if os.path.exists(prof):
+        pj = json.load(open(prof))
+        peak = pj["dp_inst_per_s"] / pj["dp_inst_per_cell_iter"] / 1e9
+        roof.update({"peak": peak, "frac": roof["achieved"] / peak, "peak_source": pj.get("source")})
+    line = {"metric": METRIC, "value": value, "unit": "Gcell-steps/s", "n_gpus": 1, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_res / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"C4 compute-intensive kernel (P:L219-L224) {n}^3 fp64, tiles {td}, "
+                                   f"K={K} inner iterations, T={T} outer steps fused per residency pass",
+                       "nstreams": ns, "value_def": "grid resident; unit = one outer step (K iterations) of one cell"},
+            "e2e": {"value": sweep.get(ns), "unit": "Gcell-steps/s", "h2d_bytes_per_step": cells * 8,
+                    "d2h_bytes_per_step": cells * 8},
+            "stream_sweep_e2e": sweep, "best_nstreams": ns_best,
+            "overlap": {"hidden_frac": hidden, "t_wall_ms": wall, "t_xfer_only_ms": xo, "t_comp_only_ms": co},
+            "gpu_launches": st["n_kernels"], "roofline": roof, "clocks": clk.summary()}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="tiles", choices=["tiles", "reference"])
-    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
+    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS) + ["c3", "c4"])
     ap.add_argument("--T", type=int, default=None)
     ap.add_argument("--nstreams", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-extras", action="store_true", help="skip sync-baseline / overlap legs")
+    ap.add_argument("--n", type=int, default=None, help="c3/c4: grid edge")
+    ap.add_argument("--budget-gb", type=float, default=None, help="c3: device budget cap")
+    ap.add_argument("--K", type=int, default=32, help="c4: kernel_iteration (reading R12)")
+    ap.add_argument("--sweep", default=None, help="c4: comma list of nstreams")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
+    if args.config == "c3":
+        return run_stream_leg(args)
+    if args.config == "c4":
+        return run_sincos_leg(args)
 
     import torch
     import torch.distributed as dist
