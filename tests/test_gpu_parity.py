@@ -250,3 +250,25 @@ def test_torch_pool_and_streams():
         d.run(T.heat7(), 4, 2)
         out = d.store()
     assert np.array_equal(out, oracle.heat_c(u0, ALPHA, 4))
+
+
+def test_sincos_single_iteration_accuracy_wide_range():
+    """One iteration of the listing on arguments spanning small, negative,
+    medium and huge (1e9..1e15, multi-word reduction) values, against the
+    glibc oracle per cell."""
+    rng = np.random.default_rng(3)
+    x = np.concatenate([rng.uniform(0, 2000, 1 << 16), rng.uniform(-400, 0, 1 << 14),
+                        rng.uniform(1e6, 2e6, 1 << 12), rng.uniform(1e9, 1e15, 1 << 12),
+                        np.array([0.0, 1048575.9, 1048576.0, np.pi / 4, np.pi / 2, np.pi, -np.pi / 4])])
+    x = np.concatenate([x, np.full((-x.size) % 4096, 0.5)])
+    n = x.size
+    grid = x.reshape(n // 512, 8, 64)
+    with T.Domain((64, 8, n // 512), (64, 8, 8)) as d:
+        d.load(grid)
+        d.run(T.sincos(1), 1, 1)
+        out = d.store().ravel()
+    ref = oracle.sincos_c(x, 1, 1)
+    # sqrt(s^2+c^2) is 1 within an ulp on both sides, so per cell the
+    # results may differ by ulp(1) (absolute) plus the final rounding
+    err = np.abs(out - ref)
+    assert np.all(err <= np.spacing(1.0) + 2 * np.spacing(np.abs(ref))), x[np.argmax(err)]
