@@ -365,13 +365,84 @@ def run_sincos_leg(args):
     return 0
 
 
+def budget_for_slots(Tl, dims, td, nslots, **kw):
+    """Smallest device budget giving `nslots` tile slots (dry-run plan)."""
+    lo, hi = 1, 1 << 42
+    while lo < hi:
+        mid = (lo + hi) // 2
+        try:
+            n = Tl.Domain(dims, td, dry_run=True, device_budget_bytes=mid, **kw).info["nslots"]
+        except Tl.TileError:
+            n = -1
+        lo, hi = (lo, mid) if n >= nslots else (mid + 1, hi)
+    return lo
+
+
+def run_fig8_leg(args):
+    """NEXT #1 (Fig. 8): the compute-intensive kernel at 512^3,
+    GPU memory limited to two regions vs unlimited vs one region, step-major
+    (every step visits every region, as the paper's time loop does). Also the
+    limited case with tile-major fusion (each region streamed once for all
+    steps) — a schedule the pointwise kernel allows."""
+    import torch
+    from paper_conf_icpp_bastemuzas17_b200 import tiles as Tl
+    import synth
+    n = args.n or 512
+    T = args.T if args.T is not None else 100
+    K = args.K
+    ns = args.nstreams or 2
+    gdims = (n, n, n)
+    cells = n ** 3
+    regions = (n, n, n // 16)  # 16 regions (z-slabs), the paper's region count at 512^3 (P:L210)
+    torch.cuda.set_device(0)
+    variants = {
+        "unlimited_16_regions": dict(td=regions, kw=dict(fuse_pointwise_steps=False)),
+        "limited_2_regions": dict(td=regions, kw=dict(sched="stream", fuse_pointwise_steps=False,
+                                                       device_budget_bytes=budget_for_slots(
+                                                           Tl, gdims, regions, 2, sched="stream"))),
+        "one_region": dict(td=gdims, kw=dict(fuse_pointwise_steps=False)),
+        "limited_2_regions_tile_major": dict(td=regions, kw=dict(sched="stream", fuse_pointwise_steps=True,
+                                                                  device_budget_bytes=budget_for_slots(
+                                                                      Tl, gdims, regions, 2, sched="stream"))),
+    }
+    res = {}
+    for name, v in variants.items():
+        dom = Tl.Domain(gdims, v["td"], ghost=1, device=0, **v["kw"])
+        fill_tiles(dom, Tl, synth, gdims, v["td"], 0, 7)
+        k = Tl.sincos(K)
+        dom.run(k, 1, ns)
+        dom.sync()
+        dom.invalidate()
+        dom.reset_stats()
+        dom.timer_start()
+        dom.run(k, T, ns)
+        dom.sync()
+        ms = dom.timer_stop()
+        st = dom.stats()
+        res[name] = {"ms": ms, "gcell_steps_per_s": cells * T / (ms / 1e3) / 1e9, "nslots": dom.info["nslots"],
+                     "h2d_gb": st["bytes_h2d"] / 1e9, "d2h_gb": st["bytes_d2h"] / 1e9, "launches": st["n_kernels"]}
+        dom.free()
+    base = res["unlimited_16_regions"]["ms"]
+    for r in res.values():
+        r["time_vs_unlimited"] = r["ms"] / base
+    line = {"metric": "time, compute-intensive kernel, limited vs unlimited GPU memory (Fig. 8 analogue)",
+            "value": res["limited_2_regions"]["ms"] / base, "unit": "x unlimited time",
+            "higher_is_better": False, "n_gpus": 1, "steps": 1, "warmup": 1, "dtype": "f64",
+            "data": "synthetic", "vs_baseline": None, "scaling": "weak",
+            "config": {"workload": f"Fig. 8: sincos kernel {n}^3, K={K}, T={T} outer steps, 16 regions, "
+                                   f"{ns} streams", "regions": regions},
+            "variants": res}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="tiles", choices=["tiles", "reference"])
-    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS) + ["c3", "c4"])
+    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS) + ["c3", "c4", "fig8"])
     ap.add_argument("--T", type=int, default=None)
     ap.add_argument("--nstreams", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -387,6 +458,8 @@ def main():
         return run_stream_leg(args)
     if args.config == "c4":
         return run_sincos_leg(args)
+    if args.config == "fig8":
+        return run_fig8_leg(args)
 
     import torch
     import torch.distributed as dist

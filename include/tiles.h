@@ -107,6 +107,8 @@ typedef struct {
   int32_t fuse_pointwise_steps; /* SINCOS: 1 (default) = all T steps of a tile
                                    in one residency pass (tile-major); 0 =
                                    step-major, every step re-streams (Fig. 8) */
+  void* local_group;            /* optional in-process transport (see
+                                   tile_local_group_create); replaces NCCL */
 } tile_options;
 
 typedef struct {
@@ -249,6 +251,15 @@ const char* tile_last_error(void);
 /* Fill out[128] with a fresh ncclUniqueId (call on rank 0, then broadcast).
  * TILE_ENOSYS if built without NCCL. */
 tile_status tile_nccl_unique_id(void* out128);
+
+/* In-process multi-rank transport for testing the slab path on ONE device:
+ * every rank is a domain driven by its own host thread (ranks may share a
+ * GPU); halo exchanges rendezvous on the host and move faces with device
+ * copies ordered by cross-rank CUDA events. Pass the group in
+ * tile_options.local_group (nranks must match). The group must outlive its
+ * domains. */
+tile_status tile_local_group_create(int32_t nranks, void** group);
+tile_status tile_local_group_free(void* group);
 
 /* Library version string. */
 const char* tile_version(void);

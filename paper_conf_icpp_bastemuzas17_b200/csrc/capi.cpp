@@ -213,6 +213,16 @@ tile_status tile_free(tile_domain* h) {
   return s.code;
 }
 
+tile_status tile_local_group_create(int32_t nranks, void** group) {
+  if (!group) return fail(TILE_EINVAL, "null group");
+  return finish(nullptr, tiles::local_group_create(nranks, group));
+}
+
+tile_status tile_local_group_free(void* group) {
+  tiles::local_group_free(group);
+  return TILE_OK;
+}
+
 tile_status tile_nccl_unique_id(void* out128) {
   if (!out128) return fail(TILE_EINVAL, "null out");
   return finish(nullptr, tiles::nccl_unique_id(out128));

@@ -31,6 +31,7 @@ struct CudaExec final : Exec {
   std::vector<cudaEvent_t> tpool;                 // timing events (free list)
   std::vector<std::pair<cudaEvent_t, cudaEvent_t>> tpending;
   cudaEvent_t t_begin = nullptr, t_end = nullptr;
+  cudaEvent_t local_ready = nullptr;  // in-process transport
 
   Status timing_event(cudaEvent_t* e) {
     if (!tpool.empty()) {
@@ -210,6 +211,13 @@ struct CudaExec final : Exec {
     return Status::ok();
   }
   Status halo(Domain& d, int par, int st) override {
+    if (d.opt.local_group) {
+      if (!local_ready) CK(cudaEventCreateWithFlags(&local_ready, cudaEventDisableTiming));
+      Status r = local_halo(d, par, S(st), local_ready);
+      if (r.bad()) return r;
+      d.stats.n_halo++;
+      return Status::ok();
+    }
     Status r = nccl_halo(d, par, S(st));
     if (r.bad()) return r;
     d.stats.n_halo++;
@@ -289,6 +297,7 @@ struct CudaExec final : Exec {
     tpending.clear();
     for (auto e : tpool) cudaEventDestroy(e);
     tpool.clear();
+    if (local_ready) cudaEventDestroy(local_ready);
     if (t_begin) cudaEventDestroy(t_begin);
     if (t_end) cudaEventDestroy(t_end);
     for (auto e : events)

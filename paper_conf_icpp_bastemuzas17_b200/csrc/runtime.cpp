@@ -56,8 +56,8 @@ Status domain_create(const int64_t dims[3], const int64_t tdims[3], int ghost,
   Geometry G;
   Status st = make_geometry(dims, tdims, ghost, opt.bc, opt.nranks, opt.rank, &G);
   if (st.bad()) return st;
-  if (G.nranks > 1 && !opt.nccl_unique_id && !opt.dry_run)
-    return make_err(TILE_EINVAL, "nranks > 1 needs nccl_unique_id");
+  if (G.nranks > 1 && !opt.nccl_unique_id && !opt.dry_run && !opt.local_group)
+    return make_err(TILE_EINVAL, "nranks > 1 needs nccl_unique_id or local_group");
 
   int band = 0, stages = 0;
   size_t smem = 0;
@@ -227,7 +227,7 @@ Status domain_setup(Domain& d) {
   d.nevents = d.ev_misc_base + 4 + d.halo_stream + 1;
   st = X.setup(d);
   if (st.bad()) return st;
-  if (multi && !d.opt.dry_run) {
+  if (multi && !d.opt.dry_run && !d.opt.local_group) {
     st = nccl_init(d);
     if (st.bad()) return st;
   }

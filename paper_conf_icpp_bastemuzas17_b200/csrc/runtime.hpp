@@ -198,4 +198,9 @@ Status nccl_init(Domain& d);
 Status nccl_halo(Domain& d, int parity, void* stream);
 void nccl_destroy(Domain& d);
 
+// comm_local.cu (in-process transport, tests)
+Status local_group_create(int n, void** out);
+void local_group_free(void* g);
+Status local_halo(Domain& d, int parity, void* stream, void* ready_event);
+
 }  // namespace tiles

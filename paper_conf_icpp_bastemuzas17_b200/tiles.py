@@ -43,7 +43,8 @@ class TileOptions(ctypes.Structure):
                 ("streams", ctypes.POINTER(ctypes.c_void_p)), ("nstreams_provided", ctypes.c_int32),
                 ("nranks", ctypes.c_int32), ("rank", ctypes.c_int32),
                 ("nccl_unique_id", ctypes.c_void_p), ("sched", ctypes.c_int),
-                ("dry_run", ctypes.c_int32), ("fuse_pointwise_steps", ctypes.c_int32)]
+                ("dry_run", ctypes.c_int32), ("fuse_pointwise_steps", ctypes.c_int32),
+                ("local_group", ctypes.c_void_p)]
 
 
 class TileKernel(ctypes.Structure):
@@ -105,6 +106,8 @@ _sig = {
     "tile_free": ([_P], ctypes.c_int),
     "tile_last_error": ([], ctypes.c_char_p),
     "tile_nccl_unique_id": ([_P], ctypes.c_int),
+    "tile_local_group_create": ([ctypes.c_int32, ctypes.POINTER(_P)], ctypes.c_int),
+    "tile_local_group_free": ([_P], ctypes.c_int),
     "tile_version": ([], ctypes.c_char_p),
 }
 EXPORTED = tuple(_sig)
@@ -133,6 +136,22 @@ def nccl_unique_id():
     return buf.raw
 
 
+class LocalGroup:
+    """In-process multi-rank transport (tile_local_group_create): one domain
+    per rank, each driven by its own thread, ranks may share one GPU."""
+
+    def __init__(self, nranks):
+        h = ctypes.c_void_p()
+        _check(tile_local_group_create(nranks, ctypes.byref(h)), "tile_local_group_create")
+        self.handle = h
+        self.nranks = nranks
+
+    def free(self):
+        if self.handle is not None:
+            tile_local_group_free(self.handle)
+            self.handle = None
+
+
 def heat7(alpha=0.125):
     """Heat kernel descriptor (reading R1)."""
     return TileKernel(TILE_KERNEL_HEAT7, alpha, 0)
@@ -149,7 +168,7 @@ class Domain:
 
     def __init__(self, dims, tile_dims, ghost=1, bc="periodic", device=-1, device_budget_bytes=0,
                  sched="auto", nranks=1, rank=0, nccl_id=None, dry_run=False,
-                 fuse_pointwise_steps=True, device_pool=None, streams=None):
+                 fuse_pointwise_steps=True, device_pool=None, streams=None, local_group=None):
         self._h = None
         self.dims = tuple(int(v) for v in dims)
         self.tile_dims = tuple(int(v) for v in tile_dims)
@@ -177,6 +196,9 @@ class Domain:
         o.sched = SCHEDS[sched] if isinstance(sched, str) else int(sched)
         o.dry_run = 1 if dry_run else 0
         o.fuse_pointwise_steps = 1 if fuse_pointwise_steps else 0
+        self._group = local_group
+        if local_group is not None:
+            o.local_group = local_group.handle
         d = (ctypes.c_int64 * 3)(*self.dims)
         t = (ctypes.c_int64 * 3)(*self.tile_dims)
         h = ctypes.c_void_p()
