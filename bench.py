@@ -436,13 +436,65 @@ def run_fig8_leg(args):
     return 0
 
 
+def run_fig5_leg(args):
+    """Fig. 5 analogue: C2 heat 512^3, e2e incl. H2D/D2H for
+    T in {1, 10, 100, 1000}: the tiled 4-stream schedule vs the synchronous
+    one-stream schedule (H2D all, T steps, D2H all), same kernels."""
+    import torch
+    from paper_conf_icpp_bastemuzas17_b200 import tiles as Tl
+    import synth
+    n = args.n or 512
+    td = (64, 64, 64)
+    gdims = (n, n, n)
+    cells = n ** 3
+    Ts = [int(v) for v in (args.sweep or "1,10,100,1000").split(",")]
+    torch.cuda.set_device(0)
+    out = {}
+    for sched, ns in (("auto", args.nstreams or 4), ("sync", 1)):
+        dom = Tl.Domain(gdims, td, ghost=1, device=0, sched=sched)
+        fill_tiles(dom, Tl, synth, gdims, td, 0, 42)
+        k = Tl.heat7(ALPHA)
+        for T in Ts:
+            reps = 3 if T <= 10 else 1
+            dom.invalidate()
+            dom.run(k, min(T, 10), ns)
+            dom.sync()
+            best = 1e30
+            for _ in range(reps):
+                dom.invalidate()
+                dom.timer_start()
+                dom.run(k, T, ns)
+                dom.sync()
+                best = min(best, dom.timer_stop())
+            out.setdefault(str(T), {})[sched if sched == "sync" else "tiled"] = {
+                "ms": best, "gcell_per_s": cells * T / (best / 1e3) / 1e9}
+        dom.free()
+    bw = pcie_bandwidth(torch)
+    hbm, _ = measured_peaks()
+    for T, r in out.items():
+        r["speedup_tiled_vs_sync"] = r["sync"]["ms"] / r["tiled"]["ms"]
+        t_link = cells * 8 / (bw["h2d"] * 1e9) + cells * 8 / (bw["d2h"] * 1e9)
+        t_hbm = int(T) * 16 * cells / (hbm * 1e9)
+        r["roofline_ms"] = {"t_link_dependency": t_link * 1e3, "t_hbm": t_hbm * 1e3,
+                            "bound_ms": max(t_link, t_hbm) * 1e3,
+                            "serial_ms": (t_link + t_hbm) * 1e3}
+        r["tiled_frac_of_bound"] = max(t_link, t_hbm) * 1e3 / r["tiled"]["ms"]
+    line = {"metric": "Gcell-updates/s incl. H2D/D2H, tiled vs synchronous (Fig. 5 analogue)",
+            "value": out[str(Ts[0])]["speedup_tiled_vs_sync"], "unit": "x speedup at first T",
+            "higher_is_better": True, "n_gpus": 1, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"C2 heat {n}^3, tiles {td}, T sweep {Ts}"}, "sweep": out,
+            "pcie_gbs": bw}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="tiles", choices=["tiles", "reference"])
-    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS) + ["c3", "c4", "fig8"])
+    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS) + ["c3", "c4", "fig5", "fig8"])
     ap.add_argument("--T", type=int, default=None)
     ap.add_argument("--nstreams", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -460,6 +512,8 @@ def main():
         return run_sincos_leg(args)
     if args.config == "fig8":
         return run_fig8_leg(args)
+    if args.config == "fig5":
+        return run_fig5_leg(args)
 
     import torch
     import torch.distributed as dist

@@ -30,10 +30,26 @@ int ev_tile(const Domain& d, int64_t k, int par) { return d.ev_tile_base + (int)
 int ev_slot(const Domain& d, int s) { return d.ev_slot_base + s; }
 int ev_faces_init(const Domain& d) { return d.ev_misc_base + 0; }
 int ev_halo(const Domain& d, int par) { return d.ev_misc_base + 1 + par; }
-int ev_join(const Domain& d) { return d.ev_misc_base + 3; }
+int ev_phase(const Domain& d) { return d.ev_misc_base + 3; }
+int ev_in(const Domain& d, int64_t i) { return d.ev_in_base + (int)i; }
+int ev_host(const Domain& d, int64_t k) { return d.ev_host_base + (int)k; }
 int ev_stream_tail(const Domain& d, int s) { return d.ev_misc_base + 4 + s; }
 
 bool z_wraps_locally(const Geometry& G) { return G.nranks == 1 && G.bc == TILE_BC_PERIODIC; }
+
+// Stream roles of pipeline i: kernels on comp(i), copies in
+// on in(i), copies out on out(i) — separate streams when 3S <= 64, so a
+// queued copy never holds back an unrelated kernel or copy. Serial (the
+// synchronous baseline) puts everything on stream 0.
+struct Pipes {
+  int S;
+  bool split;
+  Pipes(int s, bool serial) : S(serial ? 1 : s), split(!serial && 3 * s <= 64) {}
+  int comp(int64_t i) const { return (int)(i % S); }
+  int in(int64_t i) const { return split ? S + (int)(i % S) : comp(i); }
+  int out(int64_t i) const { return split ? 2 * S + (int)(i % S) : comp(i); }
+  int used() const { return split ? 3 * S : S; }
+};
 
 }  // namespace
 
@@ -223,7 +239,9 @@ Status domain_setup(Domain& d) {
   d.ev_layer_base = 0;
   d.ev_tile_base = d.ev_layer_base + (int)(2 * G.n[2]);
   d.ev_slot_base = d.ev_tile_base + (int)(2 * G.ntiles);
-  d.ev_misc_base = d.ev_slot_base + d.nslots;
+  d.ev_in_base = d.ev_slot_base + d.nslots;
+  d.ev_host_base = d.ev_in_base + (int)G.ntiles;
+  d.ev_misc_base = d.ev_host_base + (int)G.ntiles;
   d.nevents = d.ev_misc_base + 4 + d.halo_stream + 1;
   st = X.setup(d);
   if (st.bad()) return st;
@@ -252,17 +270,19 @@ Status domain_free(Domain* d) {
 // --------------------------------------------------------------- residency
 namespace {
 
+// Every operation on a device slot waits for the slot's event and records
+// it again afterwards, so the operations on one slot are totally ordered in
+// issue order whatever stream they run on (WAR/WAW/RAW on the slot).
 struct Sched {
   Domain& d;
   Exec& X;
-  int S;
+  Pipes P;
   std::set<std::pair<int64_t, int>> lru;  // (last_use, tile) of resident tiles
 
-  explicit Sched(Domain& dd, int s) : d(dd), X(*dd.exec), S(s) {
+  explicit Sched(Domain& dd, const Pipes& p) : d(dd), X(*dd.exec), P(p) {
     for (int64_t k = 0; k < d.G.ntiles; ++k)
       if (d.tile_slot[k] >= 0) lru.insert({d.tile_last_use[k], (int)k});
   }
-  int stream_of(int64_t k) const { return (int)(k % S); }
 
   void touch(int64_t k) {
     lru.erase({d.tile_last_use[k], (int)k});
@@ -273,12 +293,16 @@ struct Sched {
   // D2H of tile k from its slot into the pinned host store.
   Status writeback(int64_t k) {
     const int s = d.tile_slot[k];
-    const int st = stream_of(k);
-    Status r = X.d2h(d, k, 1, s, st);
+    const int st = P.out(k);
+    Status r = X.wait(d, ev_slot(d, s), st);
+    if (r.bad()) return r;
+    r = X.d2h(d, k, 1, s, st);
     if (r.bad()) return r;
     d.tile_dirty[k] = 0;
     d.stats.writebacks++;
-    return X.record(d, ev_slot(d, s), st);
+    r = X.record(d, ev_slot(d, s), st);
+    if (r.bad()) return r;
+    return X.record(d, ev_host(d, k), st);  // host copy of k written (RAW for its next H2D)
   }
 
   // A free device slot for tile k: a free pointer, else the least
@@ -306,7 +330,7 @@ struct Sched {
         Status r = writeback(victim);
         if (r.bad()) return r;
       } else {
-        Status r = X.note(d, TILE_OP_DROP, victim, s, stream_of(victim));
+        Status r = X.note(d, TILE_OP_DROP, victim, s, P.comp(victim));
         if (r.bad()) return r;
       }
       d.stats.evictions++;
@@ -329,7 +353,7 @@ struct Sched {
 
 // Make every stream of this run wait for everything issued before it
 // (previous runs may have used other streams, faces are shared state).
-Status join_streams(Domain& d, int S) {
+Status join_streams(Domain& d, int S) {  // S = number of low-index streams in use
   Exec& X = *d.exec;
   const int nst = d.halo_stream + 1;
   for (int s = 0; s < nst; ++s) {
@@ -358,7 +382,8 @@ namespace {
 
 struct Batch {
   int64_t L0, L1;  // layers [L0, L1)
-  int stream;
+  int stream;      // compute stream
+  int in, out;     // copy-in / copy-out streams
 };
 
 struct ResidentRun {
@@ -368,6 +393,7 @@ struct ResidentRun {
   std::vector<Batch> B;
   std::vector<std::vector<int>> nbr;  // neighbour batches (excluding self)
   bool need_load, need_extract, multi;
+  bool entry_wait = false;  // first op of every batch waits ev_phase (phase join)
   int bit0, fp0, T;
   double alpha;
 
@@ -377,17 +403,18 @@ struct ResidentRun {
   int64_t ntl(const Batch& b) const { return (b.L1 - b.L0) * G.layer_tiles; }
   int cur_slot(int64_t k, int bit) const { return bit == 0 ? (int)k : (int)(G.ntiles + k); }
 
-  void build(int S, bool serial) {
+  void build(int S, bool serial, bool layered) {
     const int64_t nL = G.n[2];
     B.clear();
-    if (serial || (!need_load && !multi)) {
-      B.push_back({0, nL, 0});
-    } else if (!need_load && multi && nL > 2) {
-      B.push_back({0, 1, 0});
-      B.push_back({nL - 1, nL, 1 % S});
-      B.push_back({1, nL - 1, 2 % S});
+    const Pipes P(S, serial);
+    if (serial || (!layered && !multi)) {
+      B.push_back({0, nL, 0, P.in(0), P.out(0)});
+    } else if (!layered && multi && nL > 2) {
+      B.push_back({0, 1, 0, 0, 0});
+      B.push_back({nL - 1, nL, 0, 0, 0});
+      B.push_back({1, nL - 1, 0, 0, 0});
     } else {
-      for (int64_t L = 0; L < nL; ++L) B.push_back({L, L + 1, 0});
+      for (int64_t L = 0; L < nL; ++L) B.push_back({L, L + 1, 0, 0, 0});
       // wrap-aware order: 0, nL-1, 1, nL-2, ... so a periodic layer's
       // neighbours arrive early
       std::vector<Batch> o;
@@ -399,8 +426,13 @@ struct ResidentRun {
       }
       if (!z_wraps_locally(G)) std::sort(o.begin(), o.end(), [](auto& a, auto& b) { return a.L0 < b.L0; });
       B = o;
-      for (size_t i = 0; i < B.size(); ++i) B[i].stream = (int)(i % S);
     }
+    if (B.size() > 1)
+      for (size_t i = 0; i < B.size(); ++i) {
+        B[i].stream = P.comp((int64_t)i);
+        B[i].in = P.in((int64_t)i);
+        B[i].out = P.out((int64_t)i);
+      }
     // neighbour batches
     auto batch_of = [&](int64_t L) {
       for (size_t i = 0; i < B.size(); ++i)
@@ -427,9 +459,19 @@ struct ResidentRun {
   Status issue_load(size_t i) {
     const Batch& b = B[i];
     Status r;
-    if (need_load) {
-      r = X.h2d(d, tile0(b), ntl(b), cur_slot(tile0(b), bit0), b.stream);
+    if (entry_wait) {
+      r = X.wait(d, ev_phase(d), b.stream);
       if (r.bad()) return r;
+    }
+    if (need_load) {
+      r = X.h2d(d, tile0(b), ntl(b), cur_slot(tile0(b), bit0), b.in);
+      if (r.bad()) return r;
+      if (b.in != b.stream) {
+        r = X.record(d, ev_in(d, (int64_t)i), b.in);
+        if (r.bad()) return r;
+        r = X.wait(d, ev_in(d, (int64_t)i), b.stream);
+        if (r.bad()) return r;
+      }
     }
     if (need_extract) {
       r = X.extract(d, tile0(b), ntl(b), cur_slot(tile0(b), bit0), fp0,
@@ -545,30 +587,71 @@ struct ResidentRun {
 
 static Status upload_dirichlet_if_needed(Domain& d);
 
+// Phases: with a fresh upload, layer batches for the steps
+// the load wavefront can overlap (k1 = nL/2 + 1), whole-domain batches for
+// the middle steps (one launch per step, or bottom/top/interior with slab
+// halos), and layer batches again for the final step so each layer's D2H can
+// start as soon as its last kernel ends. Phases are joined through ev_phase.
 static Status run_heat_resident(Domain& d, double alpha, int T, int S, bool serial) {
-  ResidentRun R(d);
-  R.alpha = alpha;
-  R.T = T;
-  R.need_load = !d.resident_valid;
-  R.need_extract = !d.faces_valid;
-  R.multi = d.G.nranks > 1;
-  R.bit0 = d.res_bit;
-  R.fp0 = d.face_parity;
-  R.build(S, serial);
-  Status r = R.run();
-  if (r.bad()) return r;
-  d.res_bit ^= (T & 1);
-  d.face_parity ^= (T & 1);
+  const bool load = !d.resident_valid;
+  const int64_t nL = d.G.n[2];
+  struct Phase {
+    int steps;
+    bool layered;
+  };
+  std::vector<Phase> ph;
+  if (serial || !load) {
+    ph.push_back({T, false});
+  } else {
+    const int k1 = (int)std::min<int64_t>(T, nL / 2 + 1);
+    if (T <= k1 + 1) {
+      ph.push_back({T, true});
+    } else {
+      ph.push_back({k1, true});
+      ph.push_back({T - k1 - 1, false});
+      ph.push_back({1, true});
+    }
+  }
+  int bit = d.res_bit, fp = d.face_parity;
+  std::vector<std::pair<Batch, int>> last;  // batches of the last phase + final event
+  for (size_t pi = 0; pi < ph.size(); ++pi) {
+    ResidentRun R(d);
+    R.alpha = alpha;
+    R.T = ph[pi].steps;
+    R.need_load = pi == 0 && load;
+    R.need_extract = pi == 0 && !d.faces_valid;
+    R.multi = d.G.nranks > 1;
+    R.entry_wait = pi > 0;
+    R.bit0 = bit;
+    R.fp0 = fp;
+    R.build(S, serial, ph[pi].layered);
+    Status r = R.run();
+    if (r.bad()) return r;
+    bit ^= (R.T & 1);
+    fp ^= (R.T & 1);
+    last.clear();
+    for (size_t i = 0; i < R.B.size(); ++i)
+      last.push_back({R.B[i], ev_layer(d, (int64_t)i, R.T > 0 ? (R.T - 1) & 1 : 1)});
+    if (pi + 1 < ph.size()) {  // join: stream 0 waits for every batch, then ev_phase
+      for (auto& e : last) {
+        r = d.exec->wait(d, e.second, 0);
+        if (r.bad()) return r;
+      }
+      r = d.exec->record(d, ev_phase(d), 0);
+      if (r.bad()) return r;
+    }
+  }
+  d.res_bit = bit;
+  d.face_parity = fp;
   d.resident_valid = true;
   d.faces_valid = true;
   for (int64_t k = 0; k < d.G.ntiles; ++k) {
-    d.tile_slot[k] = R.cur_slot(k, d.res_bit);
+    d.tile_slot[k] = bit == 0 ? (int)k : (int)(d.G.ntiles + k);
     if (T > 0) d.tile_dirty[k] = 1;
   }
-  // remember which stream holds each tile's last kernel (for tile_sync)
-  d.trace.reserve(d.trace.size());
+  // where each layer's last kernel ran and its event (for tile_sync's D2H)
   d.last_batches.clear();
-  for (auto& b : R.B) d.last_batches.push_back({b.L0, b.L1, b.stream});
+  for (auto& e : last) d.last_batches.push_back({e.first.L0, e.first.L1, e.first.stream, e.first.out, e.second});
   return Status::ok();
 }
 
@@ -576,7 +659,8 @@ static Status run_heat_resident(Domain& d, double alpha, int T, int S, bool seri
 static Status run_stream(Domain& d, const tile_kernel& k, int T, int S) {
   Exec& X = *d.exec;
   const Geometry& G = d.G;
-  Sched sc(d, S);
+  const Pipes P(S, false);
+  Sched sc(d, P);
   const bool heat = k.kind == TILE_KERNEL_HEAT7;
   const bool fuse = !heat && d.opt.fuse_pointwise_steps;
   const int passes = fuse ? (T > 0 ? 1 : 0) : T;
@@ -625,7 +709,7 @@ static Status run_stream(Domain& d, const tile_kernel& k, int T, int S) {
     const int rp = fp0 ^ (s & 1);
     for (int64_t j = 0; j < N; ++j) {
       const int64_t t = (s & 1) ? N - 1 - j : j;
-      const int st = sc.stream_of(t);
+      const int st = P.comp(t);
       int in = d.tile_slot[t];
       if (in >= 0) {
         d.stats.hits++;
@@ -633,14 +717,21 @@ static Status run_stream(Domain& d, const tile_kernel& k, int T, int S) {
         if (r.bad()) return r;
       } else {
         d.stats.misses++;
-        r = sc.acquire(t, st, -1, &in);
+        const int is = P.in(t);
+        r = sc.acquire(t, is, -1, &in);
         if (r.bad()) return r;
-        r = X.h2d(d, t, 1, in, st);
+        r = X.wait(d, ev_host(d, t), is);  // host copy of t complete (previous D2H)
+        if (r.bad()) return r;
+        r = X.h2d(d, t, 1, in, is);
+        if (r.bad()) return r;
+        r = X.record(d, ev_slot(d, in), is);
         if (r.bad()) return r;
         d.tile_slot[t] = in;
         d.tile_dirty[t] = 0;
         sc.touch(t);
       }
+      r = X.wait(d, ev_slot(d, in), st);  // after the slot's previous op (H2D or D2H)
+      if (r.bad()) return r;
       if (heat) {
         int out;
         r = sc.acquire(t, st, in, &out);
@@ -673,20 +764,21 @@ static Status run_stream(Domain& d, const tile_kernel& k, int T, int S) {
         if (r.bad()) return r;
         r = X.record(d, ev_slot(d, in), st);
         if (r.bad()) return r;
+        r = X.record(d, ev_slot(d, out), st);
+        if (r.bad()) return r;
         sc.release(in);
         d.tile_slot[t] = out;
         d.slot_owner[out] = (int)t;
       } else {
         r = X.sincos(d, t, in, iters, st);
         if (r.bad()) return r;
+        r = X.record(d, ev_slot(d, in), st);
+        if (r.bad()) return r;
       }
       d.tile_dirty[t] = 1;
       sc.touch(t);
       if (j < N - W) {
         r = sc.writeback(t);
-        if (r.bad()) return r;
-      } else {
-        r = X.record(d, ev_slot(d, d.tile_slot[t]), st);
         if (r.bad()) return r;
       }
     }
@@ -724,10 +816,12 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
   if (r.bad()) return r;
   const bool serial = d.opt.sched == TILE_SCHED_SYNC;
   const int S = serial ? 1 : nstreams;
-  r = join_streams(d, std::max(S, d.streams_used));
+  const Pipes P(S, serial);
+  r = join_streams(d, std::max(P.used(), d.streams_used));
   if (r.bad()) return r;
-  d.streams_used = std::max(d.streams_used, S);
+  d.streams_used = std::max(d.streams_used, P.used());
   d.last_S = S;
+  d.last_serial = serial;
   d.in_flight = true;
   if (k.kind == TILE_KERNEL_HEAT7 && d.mode == MODE_RESIDENT) {
     r = run_heat_resident(d, k.alpha, steps, S, serial);
@@ -739,13 +833,21 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
     const int64_t iters = fuse ? (int64_t)k.inner_iters * steps : k.inner_iters;
     for (int s = 0; s < passes; ++s)
       for (int64_t t = 0; t < d.G.ntiles; ++t) {
-        const int st = serial ? 0 : (int)(t % S);
+        const int st = P.comp(t);
         const int slot = (int)(d.res_bit == 0 ? t : d.G.ntiles + t);
         if (!d.resident_valid && s == 0) {
-          r = X.h2d(d, t, 1, slot, st);
+          r = X.h2d(d, t, 1, slot, P.in(t));
           if (r.bad()) return r;
+          if (P.in(t) != st) {
+            r = X.record(d, ev_in(d, t), P.in(t));
+            if (r.bad()) return r;
+            r = X.wait(d, ev_in(d, t), st);
+            if (r.bad()) return r;
+          }
         }
         r = X.sincos(d, t, slot, iters, st);
+        if (r.bad()) return r;
+        r = X.record(d, ev_tile(d, t, 0), st);
         if (r.bad()) return r;
       }
     if (passes > 0) {
@@ -756,7 +858,7 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
         d.tile_dirty[t] = 1;
       }
       d.last_batches.clear();
-      for (int64_t L = 0; L < d.G.n[2]; ++L) d.last_batches.push_back({L, L + 1, -1});
+      for (int64_t L = 0; L < d.G.n[2]; ++L) d.last_batches.push_back({L, L + 1, -1, -1, -1});
     }
   } else {
     r = run_stream(d, k, steps, S);
@@ -778,24 +880,37 @@ Status domain_sync(Domain& d) {
       for (int64_t t = t0; t < t0 + n; ++t) any |= d.tile_dirty[t] != 0;
       if (!any) continue;
       if (b.stream >= 0) {
-        r = X.d2h(d, t0, n, d.tile_slot[t0], b.stream);
+        if (b.out != b.stream) {
+          r = X.wait(d, b.ev, b.out);  // after the batch's last kernel
+          if (r.bad()) return r;
+        }
+        r = X.d2h(d, t0, n, d.tile_slot[t0], b.out);
         if (r.bad()) return r;
-      } else {  // per-tile streams (pointwise kernel)
+      } else {  // per-tile pipelines (pointwise kernel)
+        const Pipes P(d.last_S, d.last_serial);
         for (int64_t t = t0; t < t0 + n; ++t) {
-          r = X.d2h(d, t, 1, d.tile_slot[t], (int)(t % std::max(1, d.last_S)));
+          r = X.wait(d, ev_tile(d, t, 0), P.out(t));
+          if (r.bad()) return r;
+          r = X.d2h(d, t, 1, d.tile_slot[t], P.out(t));
           if (r.bad()) return r;
         }
       }
       for (int64_t t = t0; t < t0 + n; ++t) d.tile_dirty[t] = 0;
     }
   } else {
+    const Pipes P(d.last_S, false);
     for (int64_t t = 0; t < d.G.ntiles; ++t) {
       if (!d.tile_dirty[t] || d.tile_slot[t] < 0) continue;
-      const int st = (int)(t % std::max(1, d.last_S));
-      r = X.d2h(d, t, 1, d.tile_slot[t], st);
+      const int st = P.out(t);
+      const int sl = d.tile_slot[t];
+      r = X.wait(d, ev_slot(d, sl), st);
+      if (r.bad()) return r;
+      r = X.d2h(d, t, 1, sl, st);
       if (r.bad()) return r;
       d.tile_dirty[t] = 0;
-      r = X.record(d, ev_slot(d, d.tile_slot[t]), st);
+      r = X.record(d, ev_slot(d, sl), st);
+      if (r.bad()) return r;
+      r = X.record(d, ev_host(d, t), st);
       if (r.bad()) return r;
     }
   }

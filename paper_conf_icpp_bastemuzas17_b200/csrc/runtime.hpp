@@ -143,6 +143,8 @@ struct Domain {
   int ev_layer_base = 0;                   // 2 per layer
   int ev_tile_base = 0;                    // 2 per tile (face events)
   int ev_slot_base = 0;                    // 1 per slot
+  int ev_in_base = 0;                      // 1 per tile / batch (H2D done)
+  int ev_host_base = 0;                    // 1 per tile (host copy written)
   int ev_misc_base = 0;                    // faces init, halo[2], done
   int nevents = 0;
 
@@ -155,11 +157,12 @@ struct Domain {
   int heat_cache_flags = 2;               // L2 policy bits (kernels.cuh): exports evict_last
 
   // run bookkeeping
-  struct BatchRec { int64_t L0, L1; int stream; };
+  struct BatchRec { int64_t L0, L1; int stream, out, ev; };  // ev: last kernel's event
   std::vector<BatchRec> last_batches;      // resident: where each layer's last kernel ran
   double kernel_alpha = 0.125;
   int streams_used = 1;                    // streams touched so far (joined at run start)
   int last_S = 1;
+  bool last_serial = false;
   std::vector<const double*> gsrc_host[2]; // [parity] -> ntiles*6
   std::vector<TileItem> items_host[2];
 

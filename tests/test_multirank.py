@@ -45,9 +45,9 @@ def _rank_domain(dims, td, G, r, bc, ext, u, **kw):
 @pytest.mark.parametrize("bc", ["periodic", "dirichlet"])
 @pytest.mark.parametrize("sched", ["resident", "stream"])
 def test_slab_replay_matches_global_oracle(G, bc, sched):
-    dims, td = (16, 8, 8 * G), (8, 4, 4)
+    dims, td = (16, 8, 16 * G), (8, 4, 4)   # 4 tile layers per rank
     u, ext, _ = _global(dims, bc)
-    steps = [3, 2]
+    steps = [6, 2]   # first run: layered / whole-slab / layered phases
     kw = {"sched": sched}
     if sched == "stream":
         kw["device_budget_bytes"] = 1  # replaced below by the minimum budget
