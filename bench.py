@@ -450,8 +450,9 @@ def run_fig5_leg(args):
     Ts = [int(v) for v in (args.sweep or "1,10,100,1000").split(",")]
     torch.cuda.set_device(0)
     out = {}
-    for sched, ns in (("auto", args.nstreams or 4), ("sync", 1)):
-        dom = Tl.Domain(gdims, td, ghost=1, device=0, sched=sched)
+    for sched, ns, pageable in (("auto", args.nstreams or 4, False), ("sync", 1, False),
+                                ("sync_pageable", 1, True)):
+        dom = Tl.Domain(gdims, td, ghost=1, device=0, sched=sched.split("_")[0], pageable_host=pageable)
         fill_tiles(dom, Tl, synth, gdims, td, 0, 42)
         k = Tl.heat7(ALPHA)
         for T in Ts:
@@ -466,13 +467,15 @@ def run_fig5_leg(args):
                 dom.run(k, T, ns)
                 dom.sync()
                 best = min(best, dom.timer_stop())
-            out.setdefault(str(T), {})[sched if sched == "sync" else "tiled"] = {
+            out.setdefault(str(T), {})[sched if sched.startswith("sync") else "tiled"] = {
                 "ms": best, "gcell_per_s": cells * T / (best / 1e3) / 1e9}
         dom.free()
     bw = pcie_bandwidth(torch)
     hbm, _ = measured_peaks()
     for T, r in out.items():
         r["speedup_tiled_vs_sync"] = r["sync"]["ms"] / r["tiled"]["ms"]
+        r["speedup_tiled_vs_sync_pageable"] = r["sync_pageable"]["ms"] / r["tiled"]["ms"]
+        r["speedup_sync_vs_sync_pageable"] = r["sync_pageable"]["ms"] / r["sync"]["ms"]
         t_link = cells * 8 / (bw["h2d"] * 1e9) + cells * 8 / (bw["d2h"] * 1e9)
         t_hbm = int(T) * 16 * cells / (hbm * 1e9)
         r["roofline_ms"] = {"t_link_dependency": t_link * 1e3, "t_hbm": t_hbm * 1e3,

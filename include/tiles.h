@@ -109,6 +109,10 @@ typedef struct {
                                    step-major, every step re-streams (Fig. 8) */
   void* local_group;            /* optional in-process transport (see
                                    tile_local_group_create); replaces NCCL */
+  int32_t pageable_host;        /* 1: host tile store from malloc (pageable),
+                                   the paper's "CUDA pageable" baseline (P:L37,
+                                   Fig. 1/5); copies are staged by the driver
+                                   and do not overlap. 0 (default): pinned. */
 } tile_options;
 
 typedef struct {

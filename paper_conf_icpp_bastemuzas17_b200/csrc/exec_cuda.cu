@@ -3,6 +3,7 @@
 // and the sm_100a kernels of kernels.cu. No CPU fallback exists: every
 // compute operation is a kernel launch.
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 
 #include "runtime.hpp"
@@ -235,7 +236,13 @@ struct CudaExec final : Exec {
     *tot = t;
     return Status::ok();
   }
-  Status alloc_host(Domain&, uint64_t bytes, void** p) override {
+  Status alloc_host(Domain& d, uint64_t bytes, void** p) override {
+    if (d.opt.pageable_host) {  // baseline only: pageable memory
+      *p = std::malloc(bytes ? bytes : 1);
+      if (!*p) return make_err(TILE_ENOMEM_HOST, "malloc failed");
+      std::memset(*p, 0, bytes);
+      return Status::ok();
+    }
     // pinned (page-locked) host regions, P:L73 (cudaMallocHost)
     cudaError_t e = cudaHostAlloc(p, bytes ? bytes : 1, cudaHostAllocPortable);
     if (e != cudaSuccess) {
@@ -244,7 +251,12 @@ struct CudaExec final : Exec {
     }
     return Status::ok();
   }
-  void free_host(Domain&, void* p) override { cudaFreeHost(p); }
+  void free_host(Domain& d, void* p) override {
+    if (d.opt.pageable_host)
+      std::free(p);
+    else
+      cudaFreeHost(p);
+  }
   Status alloc_device(Domain&, uint64_t bytes, void** p) override {
     cudaError_t e = cudaMalloc(p, bytes);
     if (e != cudaSuccess) {

@@ -44,7 +44,7 @@ class TileOptions(ctypes.Structure):
                 ("nranks", ctypes.c_int32), ("rank", ctypes.c_int32),
                 ("nccl_unique_id", ctypes.c_void_p), ("sched", ctypes.c_int),
                 ("dry_run", ctypes.c_int32), ("fuse_pointwise_steps", ctypes.c_int32),
-                ("local_group", ctypes.c_void_p)]
+                ("local_group", ctypes.c_void_p), ("pageable_host", ctypes.c_int32)]
 
 
 class TileKernel(ctypes.Structure):
@@ -168,7 +168,8 @@ class Domain:
 
     def __init__(self, dims, tile_dims, ghost=1, bc="periodic", device=-1, device_budget_bytes=0,
                  sched="auto", nranks=1, rank=0, nccl_id=None, dry_run=False,
-                 fuse_pointwise_steps=True, device_pool=None, streams=None, local_group=None):
+                 fuse_pointwise_steps=True, device_pool=None, streams=None, local_group=None,
+                 pageable_host=False):
         self._h = None
         self.dims = tuple(int(v) for v in dims)
         self.tile_dims = tuple(int(v) for v in tile_dims)
@@ -196,6 +197,7 @@ class Domain:
         o.sched = SCHEDS[sched] if isinstance(sched, str) else int(sched)
         o.dry_run = 1 if dry_run else 0
         o.fuse_pointwise_steps = 1 if fuse_pointwise_steps else 0
+        o.pageable_host = 1 if pageable_host else 0
         self._group = local_group
         if local_group is not None:
             o.local_group = local_group.handle

@@ -272,3 +272,8 @@ def test_sincos_single_iteration_accuracy_wide_range():
     # results may differ by ulp(1) (absolute) plus the final rounding
     err = np.abs(out - ref)
     assert np.all(err <= np.spacing(1.0) + 2 * np.spacing(np.abs(ref))), x[np.argmax(err)]
+
+
+def test_pageable_host_baseline_bit_exact():
+    out, ref, _, _ = _heat((64, 64, 64), (32, 32, 32), 5, sched="sync", pageable_host=True)
+    assert np.array_equal(out, ref)
