@@ -491,13 +491,109 @@ def run_fig5_leg(args):
     return 0
 
 
+def run_c5_leg(args):
+    """C5: heat 4096^3 fp64 slab-decomposed over N GPUs (z-slabs, NCCL halo
+    exchange), each rank streaming its own tiles from pinned host memory.
+    With N = 1 this runs the per-GPU slab of the 8-GPU decomposition
+    (4096 x 4096 x 512) alone (z-periodic), i.e. one rank's work."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_icpp_bastemuzas17_b200 import tiles as Tl
+    import synth
+    ws, rk, lr = dist_env()
+    torch.cuda.set_device(lr)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", lr))
+    n = args.n or 4096
+    nzl = n // 8 if ws == 1 else n // ws
+    gdims = (n, n, nzl * ws)
+    td = (256, 256, 64)
+    T = args.T if args.T is not None else 10
+    ns = args.nstreams or 4
+    cells = n * n * nzl
+    nid = None
+    if ws > 1:
+        obj = [Tl.nccl_unique_id() if rk == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        nid = obj[0]
+
+    def barrier():
+        if ws > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def mx(x):
+        if ws == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    t0 = time.perf_counter()
+    dom = Tl.Domain(gdims, td, ghost=1, device=lr, nranks=ws, rank=rk, nccl_id=nid)
+    fill_tiles(dom, Tl, synth, gdims, td, rk * nzl, 42)
+    t_setup = time.perf_counter() - t0
+    k = Tl.heat7(ALPHA)
+    dom.run(k, 1, ns)
+    dom.sync()
+    barrier()
+    dom.set_kernel_timing(True)
+    dom.reset_stats()
+    with Clocks(lr) as clk:
+        dom.timer_start()
+        for _ in range(args.steps):
+            dom.run(k, T, ns)
+        ms = mx(dom.timer_stop())
+    st = dom.stats()
+    dom.set_kernel_timing(False)
+    dom.sync()
+    value = ws * cells * T * args.steps / (ms / 1e3) / 1e9
+    barrier()
+    tot = 0.0
+    dom.reset_stats()
+    for _ in range(max(1, args.steps // 2)):
+        dom.invalidate()
+        dom.timer_start()
+        dom.run(k, T, ns)
+        dom.sync()
+        tot += dom.timer_stop()
+    tot = mx(tot)
+    reps = max(1, args.steps // 2)
+    st2 = dom.stats()
+    info = dom.info
+    dom.free()
+    e2e = ws * cells * T * reps / (tot / 1e3) / 1e9
+    peak, src = measured_peaks()
+    avg = st["kernel_ms"] / max(1, st["kernel_timed"])
+    per_launch = cells * T * args.steps / max(1, st["kernel_timed"])
+    if rk == 0:
+        line = {"metric": METRIC, "value": value, "unit": "Gcell-updates/s", "n_gpus": ws,
+                "steps": args.steps, "warmup": 1, "ms_per_step": ms / args.steps, "higher_is_better": True,
+                "scaling": "weak" if ws == 1 else "strong", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic",
+                "config": {"workload": f"C5 heat {n}^3 z-slabs" + (" (per-GPU slab of G=8 on 1 GPU)" if ws == 1 else f" over {ws} GPUs"),
+                           "global_dims": gdims, "slab": (n, n, nzl), "tile_dims": td, "T": T, "nstreams": ns,
+                           "sched": info["sched"], "nslots": info["nslots"], "setup_s": t_setup},
+                "e2e": {"value": e2e, "unit": "Gcell-updates/s", "h2d_bytes_per_step": st2["bytes_h2d"] // reps,
+                        "d2h_bytes_per_step": st2["bytes_d2h"] // reps, "ms_per_step": tot / reps},
+                "gpu_launches": st["n_kernels"],
+                "roofline": {"bound": "hbm", "achieved": 16 * per_launch / (avg / 1e3) / 1e9, "peak": peak,
+                             "unit": "GB/s", "frac": 16 * per_launch / (avg / 1e3) / 1e9 / peak, "traffic": None,
+                             "kernel": "heat7_fixed<256,16>", "peak_source": src},
+                "halo_bytes_per_step": st["bytes_halo"] // max(1, args.steps), "clocks": clk.summary()}
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="tiles", choices=["tiles", "reference"])
-    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS) + ["c3", "c4", "fig5", "fig8"])
+    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS) + ["c3", "c4", "c5", "fig5", "fig8"])
     ap.add_argument("--T", type=int, default=None)
     ap.add_argument("--nstreams", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -517,6 +613,8 @@ def main():
         return run_fig8_leg(args)
     if args.config == "fig5":
         return run_fig5_leg(args)
+    if args.config == "c5":
+        return run_c5_leg(args)
 
     import torch
     import torch.distributed as dist

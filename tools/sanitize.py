@@ -1,0 +1,47 @@
+"""Small runs of every schedule for compute-sanitizer (memcheck / racecheck /
+synccheck / initcheck): resident heat (layered + whole-domain phases),
+streaming heat with a tiny budget, Dirichlet, sincos, the generic kernel and
+the in-process multi-rank transport."""
+import os
+import sys
+import threading
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+
+import synth
+from paper_conf_icpp_bastemuzas17_b200 import tiles as T
+
+
+def budget(dims, td, n, **kw):
+    lo, hi = 1, 1 << 36
+    while lo < hi:
+        mid = (lo + hi) // 2
+        try:
+            k = T.Domain(dims, td, dry_run=True, sched="stream", device_budget_bytes=mid, **kw).info["nslots"]
+        except T.TileError:
+            k = -1
+        lo, hi = (lo, mid) if k >= n else (mid + 1, hi)
+    return lo
+
+
+u = synth.uniform_grid(64, 32, 32, 42)
+with T.Domain((64, 32, 32), (32, 16, 8)) as d:          # fixed kernel (32,16), 4 layers -> phases
+    d.load(u); d.run(T.heat7(), 6, 2); d.store()
+with T.Domain((48, 40, 20), (24, 20, 5)) as d:          # generic kernel
+    d.load(synth.uniform_grid(48, 40, 20, 1)); d.run(T.heat7(), 3, 2); d.store()
+with T.Domain((64, 32, 32), (32, 16, 8), sched="stream", device_budget_bytes=budget((64, 32, 32), (32, 16, 8), 3)) as d:
+    d.load(u); d.run(T.heat7(), 3, 2); d.store()
+ext = synth.uniform_grid(66, 34, 34, 5)
+with T.Domain((64, 32, 32), (32, 16, 16), bc="dirichlet") as d:
+    d.load(ext); d.run(T.heat7(), 3, 2); d.store()
+with T.Domain((64, 32, 32), (32, 16, 16)) as d:
+    d.load(u); d.run(T.sincos(2), 2, 2); d.store()
+g = T.LocalGroup(2)
+def rank(r):
+    with T.Domain((64, 32, 64), (32, 16, 16), nranks=2, rank=r, local_group=g) as d:
+        d.load(synth.uniform_grid(64, 32, 64, 42)[r * 32:(r + 1) * 32]); d.run(T.heat7(), 4, 2); d.store()
+th = [threading.Thread(target=rank, args=(r,)) for r in range(2)]
+[t.start() for t in th]; [t.join() for t in th]
+g.free()
+print("sanitize driver ok")
