@@ -52,9 +52,14 @@ Status make_geometry(const int64_t dims[3], const int64_t td[3], int ghost, tile
   G.rank = rank;
   G.ntiles = G.n[0] * G.n[1] * G.n[2];
   G.tile_elems = td[0] * td[1] * td[2];
-  G.face_elems[XM] = G.face_elems[XP] = td[2] * td[1];
-  G.face_elems[YM] = G.face_elems[YP] = td[2] * td[0];
-  G.face_elems[ZM] = G.face_elems[ZP] = td[1] * td[0];
+  // Faces are D = min(ghost, 2) layers deep, layers in increasing
+  // coordinate order: x-faces [z][y][D], y-faces [z][D][x], z-faces [D][y][x].
+  G.depth = ghost < 2 ? 1 : 2;
+  if (G.depth > std::min(td[0], std::min(td[1], td[2])))
+    return make_err(TILE_EINVAL, "ghost 2 needs tiles at least 2 cells deep");
+  G.face_elems[XM] = G.face_elems[XP] = td[2] * td[1] * G.depth;
+  G.face_elems[YM] = G.face_elems[YP] = td[2] * td[0] * G.depth;
+  G.face_elems[ZM] = G.face_elems[ZP] = td[1] * td[0] * G.depth;
   G.layer_tiles = G.n[0] * G.n[1];
   *out = G;
   return Status::ok();
@@ -127,10 +132,11 @@ void host_parallel_for(int64_t n, const std::function<void(int64_t, int64_t)>& f
   for (auto& t : th) t.join();
 }
 
-// Export every tile's boundary layers from the host store (layouts as the
-// device faces: x-faces [z][y], y-faces [z][x], z-faces [y][x]).
+// Export every tile's D boundary layers from the host store (layouts as the
+// device faces: x-faces [z][y][D], y-faces [z][D][x], z-faces [D][y][x], the
+// D layers in increasing coordinate order).
 void host_extract_faces(const Geometry& G, const double* host, double* const faces[6]) {
-  const int64_t tx = G.t[0], ty = G.t[1], tz = G.t[2];
+  const int64_t tx = G.t[0], ty = G.t[1], tz = G.t[2], D = G.depth;
   host_parallel_for(G.ntiles, [&](int64_t b, int64_t e) {
     for (int64_t k = b; k < e; ++k) {
       const double* u = host + k * G.tile_elems;
@@ -143,15 +149,20 @@ void host_extract_faces(const Geometry& G, const double* host, double* const fac
       for (int64_t z = 0; z < tz; ++z)
         for (int64_t y = 0; y < ty; ++y) {
           const double* row = u + (z * ty + y) * tx;
-          fxm[z * ty + y] = row[0];
-          fxp[z * ty + y] = row[tx - 1];
+          for (int64_t l = 0; l < D; ++l) {
+            fxm[(z * ty + y) * D + l] = row[l];
+            fxp[(z * ty + y) * D + l] = row[tx - D + l];
+          }
         }
-      for (int64_t z = 0; z < tz; ++z) {
-        std::copy(u + (z * ty) * tx, u + (z * ty) * tx + tx, fym + z * tx);
-        std::copy(u + (z * ty + ty - 1) * tx, u + (z * ty + ty - 1) * tx + tx, fyp + z * tx);
-      }
-      std::copy(u, u + ty * tx, fzm);
-      std::copy(u + (tz - 1) * ty * tx, u + tz * ty * tx, fzp);
+      for (int64_t z = 0; z < tz; ++z)
+        for (int64_t l = 0; l < D; ++l) {
+          const double* lo = u + (z * ty + l) * tx;
+          const double* hi = u + (z * ty + ty - D + l) * tx;
+          std::copy(lo, lo + tx, fym + (z * D + l) * tx);
+          std::copy(hi, hi + tx, fyp + (z * D + l) * tx);
+        }
+      std::copy(u, u + D * ty * tx, fzm);
+      std::copy(u + (tz - D) * ty * tx, u + tz * ty * tx, fzp);
     }
   });
 }

@@ -141,6 +141,7 @@ struct CudaExec final : Exec {
     p.nitems = n;
     p.alpha = d.kernel_alpha;
     p.cache_flags = d.heat_cache_flags;
+    p.depth = d.G.depth;
     if (dev_items) {
       p.items = dev_items;
     } else {
@@ -182,6 +183,7 @@ struct CudaExec final : Exec {
                  int st) override {
     if (d.measure == TILE_MEASURE_XFER_ONLY || n == 0) return Status::ok();
     ExtractParams p{};
+    p.depth = d.G.depth;
     p.tx = (int)d.G.t[0];
     p.ty = (int)d.G.t[1];
     p.tz = (int)d.G.t[2];

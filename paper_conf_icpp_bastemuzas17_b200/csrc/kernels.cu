@@ -123,30 +123,36 @@ __device__ __forceinline__ double heat_update(double c, double xm, double xp, do
 // Producer (one thread): stage plane z of band [y0, y0+BY) of tile `in` into
 // `dst` ((BY+2) rows of tx + 2 x-ghost columns of BY), completion on `bar`.
 // z outside [0, tz) stages the band rows of the z- / z+ ghost-source face.
+// Stage layout: rows [0, BY+2) of tx (y-halo row, BY band rows, y-halo row),
+// then the x- ghost columns (D per row, 2*BY reserved) and the x+ ghost
+// columns (D per row). Faces are D layers deep; a single step reads the layer
+// nearest the tile (x-: last, x+: first; likewise y and z).
 __device__ __forceinline__ void stage_plane(double* dst, uint64_t* bar, const double* in,
                                             const double* const* gs, int z, int tx, int ty,
-                                            int tz, int y0, int BY, int flags) {
+                                            int tz, int y0, int BY, int flags, int D) {
   // interior and ghost faces are read once: optionally evict_first
   const uint64_t pol = (flags & 1) ? policy_evict_first() : policy_evict_normal();
   fence_proxy_async();
   if (z < 0 || z >= tz) {
     const uint32_t bytes = (uint32_t)BY * tx * 8;
     mbar_expect_tx(bar, bytes);
-    bulk_g2s_hint(dst + tx, gs[z < 0 ? ZM : ZP] + (size_t)y0 * tx, bytes, bar, pol);
+    const double* src = z < 0 ? gs[ZM] + ((size_t)(D - 1) * ty + y0) * tx : gs[ZP] + (size_t)y0 * tx;
+    bulk_g2s_hint(dst + tx, src, bytes, bar, pol);
     return;
   }
   const int rows = BY + 2;
   const uint32_t row_b = (uint32_t)tx * 8;
-  mbar_expect_tx(bar, ((uint32_t)rows * tx + 2u * BY) * 8u);
+  mbar_expect_tx(bar, ((uint32_t)rows * tx + 2u * D * BY) * 8u);
   const double* plane = in + (size_t)z * ty * tx;
   bulk_g2s_hint(dst + tx, plane + (size_t)y0 * tx, row_b * BY, bar, pol);
-  const double* lo = y0 > 0 ? plane + (size_t)(y0 - 1) * tx : gs[YM] + (size_t)z * tx;
-  const double* hi = y0 + BY < ty ? plane + (size_t)(y0 + BY) * tx : gs[YP] + (size_t)z * tx;
+  const double* lo =
+      y0 > 0 ? plane + (size_t)(y0 - 1) * tx : gs[YM] + ((size_t)z * D + D - 1) * tx;
+  const double* hi = y0 + BY < ty ? plane + (size_t)(y0 + BY) * tx : gs[YP] + (size_t)z * D * tx;
   bulk_g2s_hint(dst, lo, row_b, bar, pol);
   bulk_g2s_hint(dst + (size_t)(BY + 1) * tx, hi, row_b, bar, pol);
-  bulk_g2s_hint(dst + (size_t)rows * tx, gs[XM] + (size_t)z * ty + y0, (uint32_t)BY * 8, bar, pol);
-  bulk_g2s_hint(dst + (size_t)rows * tx + BY, gs[XP] + (size_t)z * ty + y0, (uint32_t)BY * 8, bar,
-                pol);
+  const uint32_t xb = (uint32_t)(D * BY) * 8;
+  bulk_g2s_hint(dst + (size_t)rows * tx, gs[XM] + ((size_t)z * ty + y0) * D, xb, bar, pol);
+  bulk_g2s_hint(dst + (size_t)rows * tx + 2 * BY, gs[XP] + ((size_t)z * ty + y0) * D, xb, bar, pol);
 }
 
 // Contiguous range of (tile, band, z) planes owned by this CTA.
@@ -171,13 +177,13 @@ struct Fixed {
   static constexpr int NT = RPP * HALF;
   static constexpr int NR = BY / RPP;
   static constexpr int ROWS = BY + 2;
-  static constexpr int STAGE_ELEMS = ROWS * TX + 2 * BY;
+  static constexpr int STAGE_ELEMS = ROWS * TX + 4 * BY;  // x columns: 2 sides x D <= 2
   static constexpr uint32_t STAGE_BYTES = STAGE_ELEMS * 8;
   static constexpr size_t SMEM = (size_t)S * STAGE_BYTES + (size_t)S * 16;  // + full/empty
   static_assert(BY % RPP == 0 && NR >= 1 && NR <= 8, "bad fixed config");
 };
 
-template <int TX, int BY, int S>
+template <int TX, int BY, int S, int D>
 __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
     heat7_fixed(const __grid_constant__ HeatParams p) {
   // Warp-specialised: warps 0..NT/32-1 compute, warp NT/32 is the TMA
@@ -218,7 +224,7 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
         const int s = (int)(g % S);
         mbar_wait(&empty[s], ((g / S) & 1u) ^ 1u);
         stage_plane(stage_base + (size_t)s * C::STAGE_ELEMS, &full[s], it.in, gs, z, TX, ty, tz,
-                    y0, BY, p.cache_flags);
+                    y0, BY, p.cache_flags, D);
       }
       pp += z1 - z0;
     }
@@ -235,10 +241,10 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
   const double alpha = p.alpha;
   const char* sm = reinterpret_cast<const char*>(smem_raw);
   const int coff = ((r0 + 1) * TX + x) * 8;
-  const int xmoff = xlo_edge ? (C::ROWS * TX + r0) * 8 : coff - 8;
-  const int xpoff = xhi_edge ? (C::ROWS * TX + BY + r0) * 8 : coff + 16;
-  const int xmj = xlo_edge ? C::RPP * 8 : C::RPP * TX * 8;
-  const int xpj = xhi_edge ? C::RPP * 8 : C::RPP * TX * 8;
+  const int xmoff = xlo_edge ? (C::ROWS * TX + r0 * D + D - 1) * 8 : coff - 8;
+  const int xpoff = xhi_edge ? (C::ROWS * TX + 2 * BY + r0 * D) * 8 : coff + 16;
+  const int xmj = xlo_edge ? C::RPP * D * 8 : C::RPP * TX * 8;
+  const int xpj = xhi_edge ? C::RPP * D * 8 : C::RPP * TX * 8;
   auto wait_g = [&](uint32_t g) { mbar_wait(&full[g % S], (g / S) & 1u); };
   auto release_g = [&](uint32_t g) {
     __syncwarp();
@@ -257,16 +263,20 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
 
     const int64_t tile = it.tile;
     const int yb = y0 + r0;
-    double* fxm = p.fexp[XM] + tile * p.face_elems[XM] + yb;
-    double* fxp = p.fexp[XP] + tile * p.face_elems[XP] + yb;
+    double* fxm = p.fexp[XM] + tile * p.face_elems[XM];
+    double* fxp = p.fexp[XP] + tile * p.face_elems[XP];
     double* fym = p.fexp[YM] + tile * p.face_elems[YM] + x;
     double* fyp = p.fexp[YP] + tile * p.face_elems[YP] + x;
     double* fzm = p.fexp[ZM] + tile * p.face_elems[ZM] + (size_t)yb * TX + x;
     double* fzp = p.fexp[ZP] + tile * p.face_elems[ZP] + (size_t)yb * TX + x;
-    const bool ylo_edge = yb == 0;
-    const bool yhi_edge = yb + (C::NR - 1) * C::RPP == ty - 1;
     double* obase = it.out + (size_t)yb * TX + x;
     const size_t plane = (size_t)ty * TX;
+    bool ylo[C::NR], yhi[C::NR];  // rows exported to the y- / y+ faces
+#pragma unroll
+    for (int j = 0; j < C::NR; ++j) {
+      ylo[j] = yb + j * C::RPP < D;
+      yhi[j] = yb + j * C::RPP >= ty - D;
+    }
 
     double2 zm[C::NR], zc[C::NR];
     wait_g(seq);
@@ -290,7 +300,7 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
       const char* cxm = cur + xmoff;
       const char* cxp = cur + xpoff;
       double* op = obase + (size_t)z * plane;
-      const bool zlo_edge = z == 0, zhi_edge = z == tz - 1;
+      const bool zlo = z < D, zhi = z >= tz - D;
 #pragma unroll
       for (int j = 0; j < C::NR; ++j) {
         const int jo = j * C::RPP * TX * 8;
@@ -308,12 +318,19 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
         zc[j] = zp;
         // Epilogue: export the new boundary layers (the neighbours' ghost
         // sources for the next step). Rare, predicated.
-        if (xlo_edge) st_hint(fxm + (size_t)z * ty + j * C::RPP, v.x, keep);
-        if (xhi_edge) st_hint(fxp + (size_t)z * ty + j * C::RPP, v.y, keep);
-        if (j == 0 && ylo_edge) st2_hint(fym + (size_t)z * TX, v, keep);
-        if (j == C::NR - 1 && yhi_edge) st2_hint(fyp + (size_t)z * TX, v, keep);
-        if (zlo_edge) st2_hint(fzm + (size_t)j * C::RPP * TX, v, keep);
-        if (zhi_edge) st2_hint(fzp + (size_t)j * C::RPP * TX, v, keep);
+        const int y = yb + j * C::RPP;
+        if (xlo_edge) {  // x = 0 (and 1): layers of the x- face
+          if (D == 1) st_hint(fxm + (size_t)z * ty + y, v.x, keep);
+          else st2_hint(fxm + ((size_t)z * ty + y) * 2, v, keep);
+        }
+        if (xhi_edge) {  // x = TX-1 (and TX-2)
+          if (D == 1) st_hint(fxp + (size_t)z * ty + y, v.y, keep);
+          else st2_hint(fxp + ((size_t)z * ty + y) * 2, v, keep);
+        }
+        if (ylo[j]) st2_hint(fym + ((size_t)z * D + y) * TX, v, keep);
+        if (yhi[j]) st2_hint(fyp + ((size_t)z * D + y - (ty - D)) * TX, v, keep);
+        if (zlo) st2_hint(fzm + (size_t)z * ty * TX + (size_t)j * C::RPP * TX, v, keep);
+        if (zhi) st2_hint(fzp + (size_t)(z - (tz - D)) * ty * TX + (size_t)j * C::RPP * TX, v, keep);
       }
       release_g(seq + i + 1);  // plane z no longer read (its centre is in registers)
     }
@@ -330,9 +347,9 @@ template <int NT>
 __global__ void __launch_bounds__(NT) heat7_generic(const __grid_constant__ HeatParams p,
                                                     const int stages) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
-  const int tx = p.tx, ty = p.ty, tz = p.tz, BY = p.band;
+  const int tx = p.tx, ty = p.ty, tz = p.tz, BY = p.band, D = p.depth;
   const int rows = BY + 2;
-  const int stage_elems = rows * tx + 2 * BY;
+  const int stage_elems = rows * tx + 4 * BY;
   double* stage_base = reinterpret_cast<double*>(smem_raw);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw + (size_t)stages * stage_elems * 8);
   if (threadIdx.x == 0) {
@@ -356,7 +373,7 @@ __global__ void __launch_bounds__(NT) heat7_generic(const __grid_constant__ Heat
     auto issue = [&](int q) {
       const uint32_t g = seq + q;
       stage_plane(stage_base + (size_t)(g % stages) * stage_elems, &bars[g % stages], it.in, gs,
-                  z0 - 1 + q, tx, ty, tz, y0, BY, p.cache_flags);
+                  z0 - 1 + q, tx, ty, tz, y0, BY, p.cache_flags, D);
     };
     auto wait_q = [&](int q) {
       const uint32_t g = seq + q;
@@ -379,8 +396,8 @@ __global__ void __launch_bounds__(NT) heat7_generic(const __grid_constant__ Heat
       const double* prv = stage_base + (size_t)((seq + i) % stages) * stage_elems;
       const double* cur = stage_base + (size_t)((seq + i + 1) % stages) * stage_elems;
       const double* nxt = stage_base + (size_t)((seq + i + 2) % stages) * stage_elems;
-      const double* xlo = cur + (size_t)rows * tx;
-      const double* xhi = xlo + BY;
+      const double* xlo = cur + (size_t)rows * tx;      // [r][D], nearest layer D-1
+      const double* xhi = xlo + 2 * BY;                  // [r][D], nearest layer 0
       double* out_plane = it.out + (size_t)z * ty * tx;
       const int npairs = BY * half;
       for (int e = threadIdx.x; e < npairs; e += NT) {
@@ -391,19 +408,25 @@ __global__ void __launch_bounds__(NT) heat7_generic(const __grid_constant__ Heat
         const double2 yp = *reinterpret_cast<const double2*>(cur + (size_t)(r + 2) * tx + x);
         const double2 zm = *reinterpret_cast<const double2*>(prv + (size_t)(r + 1) * tx + x);
         const double2 zp = *reinterpret_cast<const double2*>(nxt + (size_t)(r + 1) * tx + x);
-        const double xm = x == 0 ? xlo[r] : crow[x - 1];
-        const double xp = x + 2 == tx ? xhi[r] : crow[x + 2];
+        const double xm = x == 0 ? xlo[r * D + D - 1] : crow[x - 1];
+        const double xp = x + 2 == tx ? xhi[r * D] : crow[x + 2];
         double2 v;
         v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm.x, zp.x, alpha);
         v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm.y, zp.y, alpha);
         const int y = y0 + r;
         stg2_stream(out_plane + (size_t)y * tx + x, v);
-        if (x == 0) fxm[(size_t)z * ty + y] = v.x;
-        if (x + 2 == tx) fxp[(size_t)z * ty + y] = v.y;
-        if (y == 0) *reinterpret_cast<double2*>(fym + (size_t)z * tx + x) = v;
-        if (y == ty - 1) *reinterpret_cast<double2*>(fyp + (size_t)z * tx + x) = v;
-        if (z == 0) *reinterpret_cast<double2*>(fzm + (size_t)y * tx + x) = v;
-        if (z == tz - 1) *reinterpret_cast<double2*>(fzp + (size_t)y * tx + x) = v;
+        if (x == 0) {
+          if (D == 1) fxm[(size_t)z * ty + y] = v.x;
+          else *reinterpret_cast<double2*>(fxm + ((size_t)z * ty + y) * 2) = v;
+        }
+        if (x + 2 == tx) {
+          if (D == 1) fxp[(size_t)z * ty + y] = v.y;
+          else *reinterpret_cast<double2*>(fxp + ((size_t)z * ty + y) * 2) = v;
+        }
+        if (y < D) *reinterpret_cast<double2*>(fym + ((size_t)z * D + y) * tx + x) = v;
+        if (y >= ty - D) *reinterpret_cast<double2*>(fyp + ((size_t)z * D + y - (ty - D)) * tx + x) = v;
+        if (z < D) *reinterpret_cast<double2*>(fzm + ((size_t)z * ty + y) * tx + x) = v;
+        if (z >= tz - D) *reinterpret_cast<double2*>(fzp + ((size_t)(z - (tz - D)) * ty + y) * tx + x) = v;
       }
       __syncthreads();
       if (threadIdx.x == 0 && i + stages < nq) issue(i + stages);
@@ -418,13 +441,14 @@ constexpr int kGenericThreads = 256;
 // Specialisations: (TX, BY) -> kernel. BY is the largest of {64,32,16,8}
 // that divides ty and whose 5-stage ring fits in shared memory.
 struct FixedEntry {
-  int tx, by, stages;
+  int tx, by, stages, depth;
   void (*fn)(HeatParams);
   int nt;
   size_t smem;
 };
-#define FIXED(TX, BY, S) \
-  {TX, BY, S, heat7_fixed<TX, BY, S>, Fixed<TX, BY, S>::NT + 32, Fixed<TX, BY, S>::SMEM}
+#define FIXED1(TX, BY, S, D) \
+  {TX, BY, S, D, heat7_fixed<TX, BY, S, D>, Fixed<TX, BY, S>::NT + 32, Fixed<TX, BY, S>::SMEM}
+#define FIXED(TX, BY, S) FIXED1(TX, BY, S, 1), FIXED1(TX, BY, S, 2)
 static const FixedEntry kFixed[] = {
     FIXED(32, 32, 6),  FIXED(32, 16, 6),  FIXED(32, 8, 6),   FIXED(64, 64, 4),
     FIXED(64, 64, 6),  FIXED(64, 64, 5),  FIXED(64, 32, 4),  FIXED(64, 32, 3),
@@ -439,9 +463,9 @@ static const FixedEntry* find_fixed(int tx, int by) {
   return nullptr;
 }
 
-static const FixedEntry* find_fixed_s(int tx, int by, int st) {
+static const FixedEntry* find_fixed_s(int tx, int by, int st, int depth = 1) {
   for (const auto& e : kFixed)
-    if (e.tx == tx && e.by == by && e.stages == st) return &e;
+    if (e.tx == tx && e.by == by && e.stages == st && e.depth == depth) return &e;
   return nullptr;
 }
 
@@ -476,7 +500,7 @@ bool heat_plan(int tx, int ty, int max_smem, int* band, int* stages, size_t* sme
   for (int S : {5, 4, 3}) {
     for (int by = std::min(ty, 64); by >= 2; --by) {
       if ((by & 1) || ty % by) continue;
-      size_t bytes = (size_t)S * ((size_t)(by + 2) * tx + 2 * by) * 8 + (size_t)S * 8;
+      size_t bytes = (size_t)S * ((size_t)(by + 2) * tx + 4 * by) * 8 + (size_t)S * 8;
       if (bytes > (size_t)max_smem) continue;
       if (by > best_by) { best_by = by; best_s = S; }
       break;
@@ -486,14 +510,19 @@ bool heat_plan(int tx, int ty, int max_smem, int* band, int* stages, size_t* sme
   if (!best_by) return false;
   *band = best_by;
   *stages = best_s;
-  *smem = (size_t)best_s * ((size_t)(best_by + 2) * tx + 2 * best_by) * 8 + (size_t)best_s * 8;
+  *smem = (size_t)best_s * ((size_t)(best_by + 2) * tx + 4 * best_by) * 8 + (size_t)best_s * 8;
   return true;
 }
 
 cudaError_t heat_configure(int tx, int ty, int band, int stages, size_t smem, int* ctas_per_sm) {
   (void)ty;
-  const FixedEntry* e = find_fixed_s(tx, band, stages);
+  const FixedEntry* e = find_fixed_s(tx, band, stages, 1);
   if (e && e->smem == smem) {
+    for (int dd = 1; dd <= 2; ++dd) {  // both face depths share the plan
+      const FixedEntry* f = find_fixed_s(tx, band, stages, dd);
+      cudaError_t r = cudaFuncSetAttribute(f->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      if (r != cudaSuccess) return r;
+    }
     cudaError_t r = cudaFuncSetAttribute(e->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (r != cudaSuccess) return r;
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, e->fn, e->nt, smem);
@@ -506,7 +535,7 @@ cudaError_t heat_configure(int tx, int ty, int band, int stages, size_t smem, in
 }
 
 cudaError_t launch_heat7(const HeatParams& p, int stages, size_t smem, int grid, cudaStream_t s) {
-  const FixedEntry* e = find_fixed_s(p.tx, p.band, stages);
+  const FixedEntry* e = find_fixed_s(p.tx, p.band, stages, p.depth);
   if (e && e->smem == smem) {
     void* args[] = {const_cast<HeatParams*>(&p)};
     return cudaLaunchKernel(reinterpret_cast<const void*>(e->fn), dim3(grid), dim3(e->nt), args,
@@ -552,20 +581,20 @@ __global__ void extract_faces(const __grid_constant__ ExtractParams p) {
   const int item_i = blockIdx.y;
   const int f = blockIdx.z;
   const TileItem it = p.items ? p.items[item_i] : p.inline_items[item_i];
-  const int tx = p.tx, ty = p.ty, tz = p.tz;
+  const int tx = p.tx, ty = p.ty, tz = p.tz, D = p.depth;
   double* dst = p.fexp[f] + (int64_t)it.tile * p.face_elems[f];
   const int64_t n = p.face_elems[f];
   for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n;
        e += (int64_t)gridDim.x * blockDim.x) {
     int64_t src;
-    if (f <= XP) {  // [z][y]
-      const int64_t z = e / ty, y = e % ty;
-      src = (z * ty + y) * tx + (f == XM ? 0 : tx - 1);
-    } else if (f <= YP) {  // [z][x]
-      const int64_t z = e / tx, x = e % tx;
-      src = (z * ty + (f == YM ? 0 : ty - 1)) * tx + x;
-    } else {  // [y][x]
-      src = (int64_t)(f == ZM ? 0 : tz - 1) * ty * tx + e;
+    if (f <= XP) {  // [z][y][D]
+      const int64_t l = e % D, zy = e / D, z = zy / ty, y = zy % ty;
+      src = (z * ty + y) * tx + (f == XM ? l : tx - D + l);
+    } else if (f <= YP) {  // [z][D][x]
+      const int64_t x = e % tx, zl = e / tx, z = zl / D, l = zl % D;
+      src = (z * ty + (f == YM ? l : ty - D + l)) * tx + x;
+    } else {  // [D][y][x]
+      src = (int64_t)(f == ZM ? 0 : tz - D) * ty * tx + e;
     }
     dst[e] = it.in[src];
   }

@@ -40,6 +40,7 @@ struct HeatParams {
   int64_t face_elems[6];
   // L2 policy bits: 1 = TMA loads evict_first, 2 = face exports evict_last
   int32_t cache_flags;
+  int32_t depth;  // face depth D (1 or 2): layers per face, increasing coordinate
 };
 
 struct SincosParams {
@@ -52,6 +53,7 @@ struct SincosParams {
 
 struct ExtractParams {   // export u's boundary layers into faces (parity p)
   int32_t tx, ty, tz;
+  int32_t depth;
   int32_t nitems;
   const TileItem* items; // uses .in and .tile
   TileItem inline_items[kMaxInlineItems];

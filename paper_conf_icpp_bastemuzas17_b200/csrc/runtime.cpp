@@ -972,21 +972,25 @@ Status domain_load(Domain& d, const double* src) {
         G.tile_coords(k, &ix, &iy, &iz);
         const int64_t ox = ix * tx + h, oy = iy * ty + h, oz = iz * tz + h;
         auto at = [&](int64_t z, int64_t y, int64_t x) { return src[(z * ey + y) * ex + x]; };
+        const int64_t D = G.depth;
         for (int f = 0; f < 6; ++f) {
           if (face_source(G, k, f).kind != 1) continue;
+          // the fixed halo value goes to the layer nearest the tile (the
+          // minus faces' last layer, the plus faces' first); others unused
           double* o = d.host_dir[f] + k * G.face_elems[f];
+          const int64_t l = (f & 1) ? 0 : D - 1;
           if (f <= XP) {
             const int64_t x = f == XM ? ox - 1 : ox + tx;
             for (int64_t z = 0; z < tz; ++z)
-              for (int64_t y = 0; y < ty; ++y) o[z * ty + y] = at(oz + z, oy + y, x);
+              for (int64_t y = 0; y < ty; ++y) o[(z * ty + y) * D + l] = at(oz + z, oy + y, x);
           } else if (f <= YP) {
             const int64_t y = f == YM ? oy - 1 : oy + ty;
             for (int64_t z = 0; z < tz; ++z)
-              for (int64_t x = 0; x < tx; ++x) o[z * tx + x] = at(oz + z, y, ox + x);
+              for (int64_t x = 0; x < tx; ++x) o[(z * D + l) * tx + x] = at(oz + z, y, ox + x);
           } else {
             const int64_t z = f == ZM ? oz - 1 : oz + tz;
             for (int64_t y = 0; y < ty; ++y)
-              for (int64_t x = 0; x < tx; ++x) o[y * tx + x] = at(z, oy + y, ox + x);
+              for (int64_t x = 0; x < tx; ++x) o[(l * ty + y) * tx + x] = at(z, oy + y, ox + x);
           }
         }
       }

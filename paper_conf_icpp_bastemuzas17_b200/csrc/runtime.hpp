@@ -29,6 +29,7 @@ struct Geometry {
   int64_t ntiles;
   int64_t zoff;   // global z of local z = 0
   int ghost;
+  int depth;      // face depth D = min(ghost, 2): layers exported per face
   tile_bc bc;
   int nranks, rank;
   int64_t tile_elems;

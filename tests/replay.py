@@ -24,7 +24,8 @@ XM, XP, YM, YP, ZM, ZP = range(6)
 
 
 class Geometry:
-    def __init__(self, dims, tile_dims, nranks=1, rank=0, bc=0):
+    def __init__(self, dims, tile_dims, nranks=1, rank=0, bc=0, ghost=1):
+        self.depth = 1 if ghost < 2 else 2   # face depth D
         self.g = tuple(dims)
         self.t = tuple(tile_dims)
         self.nranks, self.rank, self.bc = nranks, rank, bc
@@ -61,9 +62,23 @@ class Geometry:
         return ("halo", 1, pos)
 
 
-def faces_of(u):
-    return [u[:, :, 0].copy(), u[:, :, -1].copy(), u[:, 0, :].copy(), u[:, -1, :].copy(),
-            u[0].copy(), u[-1].copy()]
+def faces_of(u, D=1):
+    """The D boundary layers of a tile per face, in increasing coordinate
+    order: x-faces (tz,ty,D), y-faces (tz,D,tx), z-faces (D,ty,tx)."""
+    return [u[:, :, :D].copy(), u[:, :, -D:].copy(), u[:, :D, :].copy(), u[:, -D:, :].copy(),
+            u[:D].copy(), u[-D:].copy()]
+
+
+def nearest(plane_stack, f):
+    """Layer of a neighbour's export adjacent to the reading tile's face f
+    (the export is of the opposite face): f = x- reads the last layer of the
+    x+ export, f = x+ the first layer of the x- export, etc."""
+    last = (f & 1) == 0
+    if f <= 1:
+        return plane_stack[:, :, -1] if last else plane_stack[:, :, 0]
+    if f <= 3:
+        return plane_stack[:, -1, :] if last else plane_stack[:, 0, :]
+    return plane_stack[-1] if last else plane_stack[0]
 
 
 class Replayer:
@@ -100,10 +115,10 @@ class Replayer:
     def ghost(self, k, f, par):
         src = self.G.neighbour(k, f)
         if src[0] == "tile":
-            return self.faces[(src[1], f ^ 1, par)]
+            return nearest(self.faces[(src[1], f ^ 1, par)], f)
         if src[0] == "dirichlet":
             return self.dirichlet_face(k, f)
-        return self.halo[(src[1], par)][src[2]]
+        return nearest(self.halo[(src[1], par)][src[2]], f)
 
     def kernel(self, k, sin, sout, par):
         u = self.slots[sin]
@@ -118,7 +133,7 @@ class Replayer:
         e[-1, 1:-1, 1:-1] = self.ghost(k, ZP, par)
         v = oracle.heat_np(e, self.alpha, 1, oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
         self.slots[sout] = v
-        for f, plane in enumerate(faces_of(v)):
+        for f, plane in enumerate(faces_of(v, self.G.depth)):
             self.faces[(k, f, par ^ 1)] = plane
 
     def execute(self, op, snapshot_faces):
@@ -132,7 +147,7 @@ class Replayer:
         elif name == "kernel":
             self.kernel(a, b, c, d)
         elif name == "extract":
-            for f, plane in enumerate(faces_of(self.slots[b])):
+            for f, plane in enumerate(faces_of(self.slots[b], self.G.depth)):
                 self.faces[(a, f, d)] = plane
         elif name == "faces_h2d":
             if d >= 0:
@@ -146,7 +161,8 @@ class Replayer:
 
     def replay(self, trace, seed):
         rng = random.Random(seed)
-        snapshot = {(k, f): p for k in range(self.G.ntiles) for f, p in enumerate(faces_of(self.host[k]))}
+        snapshot = {(k, f): p for k in range(self.G.ntiles)
+                    for f, p in enumerate(faces_of(self.host[k], self.G.depth))}
         # bind each wait to the latest preceding record of its event
         last_rec = {}
         bound = {}
@@ -232,7 +248,8 @@ def replay_ranks(reps, traces, seed):
         queues = {}
         for i, op in enumerate(tr):
             queues.setdefault(op[1], []).append(i)
-        snapshot = {(k, f): p for k in range(rep.G.ntiles) for f, p in enumerate(faces_of(rep.host[k]))}
+        snapshot = {(k, f): p for k in range(rep.G.ntiles)
+                    for f, p in enumerate(faces_of(rep.host[k], rep.G.depth))}
         state.append({"bound": bound, "queues": queues, "pos": {s: 0 for s in queues}, "done": set(),
                       "snap": snapshot})
     remaining = sum(len(t) for t in traces)

@@ -277,3 +277,16 @@ def test_sincos_single_iteration_accuracy_wide_range():
 def test_pageable_host_baseline_bit_exact():
     out, ref, _, _ = _heat((64, 64, 64), (32, 32, 32), 5, sched="sync", pageable_host=True)
     assert np.array_equal(out, ref)
+
+
+@pytest.mark.parametrize("bc,td", [("periodic", (32, 16, 16)), ("dirichlet", (32, 16, 8)),
+                                   ("periodic", (48, 40, 10)), ("periodic", (64, 64, 16))])
+def test_ghost2_faces_bit_exact(bc, td):
+    """ghost = 2: faces are exported 2 layers deep."""
+    dims = (64 if td[0] != 48 else 96, 64 if td[1] != 40 else 80, 32 if td[2] != 10 else 20)
+    out, ref, info, _ = _heat(dims, td, 7, bc=bc, ghost=2, runs=[4, 3])
+    assert info["ghost"] == 2
+    assert np.array_equal(out, ref)
+    b = _budget(dims, td, 3, bc=bc)
+    out, ref, _, _ = _heat(dims, td, 5, bc=bc, ghost=2, sched="stream", device_budget_bytes=b * 2)
+    assert np.array_equal(out, ref)

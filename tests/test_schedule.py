@@ -98,7 +98,7 @@ def _budget_for(dims, td, nslots, **kw):
     return lo
 
 
-def _run_and_replay(dims, td, steps_list, nstreams, seeds=(0, 1, 2), bc="periodic", **kw):
+def _run_and_replay(dims, td, steps_list, nstreams, seeds=(0, 1, 2), bc="periodic", ghost=1, **kw):
     nx, ny, nz = dims
     if bc == "periodic":
         u0 = synth.uniform_grid(nx, ny, nz, 42)
@@ -109,9 +109,9 @@ def _run_and_replay(dims, td, steps_list, nstreams, seeds=(0, 1, 2), bc="periodi
         u0 = ext[1:-1, 1:-1, 1:-1].copy()
         ref = oracle.heat_c(ext, ALPHA, sum(steps_list), oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
     for seed in seeds:
-        d = T.Domain(dims, td, bc=bc, dry_run=True, **kw)
+        d = T.Domain(dims, td, bc=bc, dry_run=True, ghost=ghost, **kw)
         d.load(ext if bc == "dirichlet" else u0)
-        G = Geometry(dims, td, bc=T.BCS[bc])
+        G = Geometry(dims, td, bc=T.BCS[bc], ghost=ghost)
         rep = Replayer(G, split_tiles(G, u0), ALPHA, ext=ext)
         for steps in steps_list:
             d.clear_trace()
@@ -255,3 +255,13 @@ def test_trace_ops_are_issue_ordered_per_stream():
             seen_h2d.update(range(op[2], op[2] + op[4]))
         if op[0] == "kernel":
             assert op[2] in seen_h2d
+
+
+@pytest.mark.parametrize("bc", ["periodic", "dirichlet"])
+@pytest.mark.parametrize("sched", ["resident", "stream"])
+def test_ghost2_schedules_replay_to_oracle(bc, sched):
+    dims, td = (16, 8, 16), (8, 4, 4)
+    kw = {"sched": sched}
+    if sched == "stream":
+        kw["device_budget_bytes"] = _budget_for(dims, td, 5, sched="stream", bc=bc, ghost=2)
+    _run_and_replay(dims, td, [3, 2], 2, seeds=(0, 5), bc=bc, ghost=2, **kw)
