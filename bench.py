@@ -193,7 +193,7 @@ def run_stream_leg(args):
     cells = n ** 3
     torch.cuda.set_device(0)
     t0 = time.perf_counter()
-    dom = Tl.Domain(gdims, td, ghost=1, device=0, sched="stream", device_budget_bytes=budget)
+    dom = Tl.Domain(gdims, td, ghost=args.ghost, device=0, sched="stream", device_budget_bytes=budget)
     t_alloc = time.perf_counter() - t0
     t0 = time.perf_counter()
     fill_tiles(dom, Tl, synth, gdims, td, 0, 42)
@@ -240,7 +240,8 @@ def run_stream_leg(args):
             "warmup": args.warmup, "ms_per_step": wall, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"C3 heat fp64 {n}^3 out-of-core (device budget capped at "
-                                   f"{budget / 2**30:.1f} GiB, paper method P:L232), T={T}",
+                                   f"{budget / 2**30:.1f} GiB, paper method P:L232), T={T}, ghost={args.ghost}",
+                       "ghost": args.ghost, "steps_per_pass": info["steps_per_pass"],
                        "dims": gdims, "tile_dims": td, "T": T, "nstreams": ns, "nslots": info["nslots"],
                        "ntiles": info["ntiles"], "host_gb": info["host_bytes"] / 1e9,
                        "device_gb": info["device_bytes"] / 1e9,
@@ -602,6 +603,9 @@ def main():
     ap.add_argument("--budget-gb", type=float, default=None, help="c3: device budget cap")
     ap.add_argument("--K", type=int, default=32, help="c4: kernel_iteration (reading R12)")
     ap.add_argument("--sweep", default=None, help="c4: comma list of nstreams")
+    ap.add_argument("--ghost", type=int, default=1,
+                    help="c2/c3: ghost width; 2 = two Jacobi steps per pass (temporal blocking)")
+    ap.add_argument("--two-step", type=int, default=0, help="tile_options.two_step (-1, 0, 1)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -653,10 +657,12 @@ def main():
 
     u0 = np.empty((nzl, ny, nx))
     synth.fill_uniform_native(u0.ctypes.data, gdims[0], gdims[1], gdims[2], rk * nzl, nzl, 0, ny, 0, nx, 42)
-    dom = Tl.Domain(gdims, td, ghost=1, device=lr, nranks=ws, rank=rk, nccl_id=nid)
+    dom = Tl.Domain(gdims, td, ghost=args.ghost, device=lr, nranks=ws, rank=rk, nccl_id=nid,
+                    two_step=args.two_step)
     dom.load(u0)
     del u0
     k = Tl.heat7(ALPHA)
+    spp = dom.info["steps_per_pass"]
 
     # ---- device-resident value -------------------------------------------
     dom.run(k, 1, ns)
@@ -678,7 +684,8 @@ def main():
     value = ws * cells * T * args.steps / (ms / 1e3) / 1e9
     launches = st["n_kernels"]
     avg_kernel_ms = st["kernel_ms"] / max(1, st["kernel_timed"])
-    cells_per_launch = cells * T * args.steps / max(1, st["kernel_timed"])
+    # cells swept per launch (a two-step pass sweeps the grid once for 2 steps)
+    cells_per_launch = cells * T * args.steps / spp / max(1, st["kernel_timed"])
     dom.sync()
 
     # ---- end-to-end from pinned host memory ---------------------------------
@@ -728,7 +735,7 @@ def main():
                                    "pcie_gbs": bw}}
         if ws == 1:
             dom.free()
-            sdom = Tl.Domain(gdims, td, ghost=1, device=lr, sched="sync")
+            sdom = Tl.Domain(gdims, td, ghost=args.ghost, device=lr, sched="sync")
             u0 = np.empty((nzl, ny, nx))
             synth.fill_uniform_native(u0.ctypes.data, gdims[0], gdims[1], gdims[2], 0, nzl, 0, ny, 0, nx, 42)
             sdom.load(u0)
@@ -755,7 +762,9 @@ def main():
     algo_bytes = 16.0 * cells_per_launch
     achieved = algo_bytes / (avg_kernel_ms / 1e3) / 1e9
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-            "traffic": traffic_from_profile(args.config), "kernel": "heat7_tma",
+            "traffic": traffic_from_profile(args.config) if spp == 1 else None,
+            "kernel": "heat7_fixed" if spp == 1 else "heat7x2 (2 steps per pass)",
+            "algorithmic_bytes_per_cell_update": 16.0 / spp,
             "algorithmic_bytes_per_launch": algo_bytes, "avg_launch_ms": avg_kernel_ms,
             "peak_source": peak_src}
 
@@ -773,7 +782,8 @@ def main():
                 "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
                 "data": "synthetic",
                 "config": {"workload": desc, "dims_per_gpu": dims, "global_dims": gdims, "tile_dims": td,
-                           "ghost": 1, "T": T, "nstreams": ns, "bc": "periodic", "alpha": ALPHA,
+                           "ghost": args.ghost, "steps_per_pass": spp, "T": T, "nstreams": ns,
+                           "bc": "periodic", "alpha": ALPHA,
                            "parallelism": f"z-slab x{ws}" if ws > 1 else "1 GPU",
                            "l2": "inputs larger than L2 (2 x 1.07 GB per GPU per step)",
                            "value_def": "grid resident in HBM; T steps of tile_run",

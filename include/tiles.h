@@ -113,6 +113,11 @@ typedef struct {
                                    the paper's "CUDA pageable" baseline (P:L37,
                                    Fig. 1/5); copies are staged by the driver
                                    and do not overlap. 0 (default): pinned. */
+  int32_t two_step;             /* HEAT7 with ghost >= 2: 0 (default) = two
+                                   steps per pass in the streaming schedule
+                                   (halves host-link bytes per step), single
+                                   steps when resident; 1 = two steps in every
+                                   schedule; -1 = never */
 } tile_options;
 
 typedef struct {
@@ -138,6 +143,10 @@ typedef struct {
   int32_t resident;       /* 1 if every tile currently has a valid device copy */
   uint64_t device_bytes;  /* device memory carved by the domain */
   uint64_t host_bytes;    /* pinned host memory of the tile store */
+  int32_t steps_per_pass; /* HEAT7 steps per residency pass: 2 with ghost >= 2
+                             (temporal blocking, single rank, supported tile
+                             width), else 1 */
+  int32_t reserved;
 } tile_info;
 
 /* One entry of the dry-run trace. */
@@ -152,7 +161,8 @@ typedef enum {
   TILE_OP_HALO = 8,     /* slab halo exchange of parity d */
   TILE_OP_DROP = 9,     /* tile a leaves slot b without a copy (clean) */
   TILE_OP_HIT = 10,     /* tile a found in slot b (P:L90 cache hit) */
-  TILE_OP_POINTWISE = 11 /* compute-intensive kernel on tile a in slot b, c iterations */
+  TILE_OP_POINTWISE = 11,/* compute-intensive kernel on tile a in slot b, c iterations */
+  TILE_OP_KERNEL2 = 12   /* like KERNEL, two steps in one pass (ghost width 2) */
 } tile_op_kind;
 
 typedef struct {

@@ -167,6 +167,92 @@ void host_extract_faces(const Geometry& G, const double* host, double* const fac
   });
 }
 
+// Global coordinates of the tile-local cell (x, y, z) of tile id.
+static void local_to_tile(const Geometry& G, int64_t c[3], int64_t* tile, bool* inside_all,
+                          int out_axis[3]) {
+  // c is in units of tile-local cells relative to tile `*tile`; wrap
+  // periodically per axis (single rank) and report axes leaving the domain
+  int64_t t[3];
+  G.tile_coords(*tile, &t[0], &t[1], &t[2]);
+  *inside_all = true;
+  for (int a = 0; a < 3; ++a) {
+    out_axis[a] = 0;
+    int64_t off = 0;
+    if (c[a] < 0) off = -1;
+    if (c[a] >= G.t[a]) off = +1;
+    int64_t nt = t[a] + off;
+    if (nt < 0 || nt >= G.n[a]) {
+      if (G.bc == TILE_BC_DIRICHLET || (a == 2 && G.nranks > 1)) {
+        out_axis[a] = off;
+        *inside_all = false;
+        nt = t[a];  // stay on this tile along a (the cell is in its ghost layer)
+        continue;   // keep c[a] as a ghost coordinate
+      }
+      nt = (nt + G.n[a]) % G.n[a];
+    }
+    t[a] = nt;
+    c[a] -= off * G.t[a];
+  }
+  *tile = G.tile_id(t[0], t[1], t[2]);
+}
+
+EdgeSrc edge_source(const Geometry& G, int64_t id, int e) {
+  static const int axes[3][2] = {{0, 1}, {0, 2}, {1, 2}};
+  const int grp = e >> 2, ga = (e >> 1) & 1, gb = e & 1;
+  const int a = axes[grp][0], b = axes[grp][1], line = 3 - a - b;
+  int64_t c[3] = {0, 0, 0};  // tile-local coords of the line's cell 0
+  c[a] = ga ? G.t[a] : -1;
+  c[b] = gb ? G.t[b] : -1;
+  c[line] = 0;
+  int64_t tile = id;
+  bool inside = true;
+  int out[3];
+  local_to_tile(G, c, &tile, &inside, out);
+  if (G.nranks > 1 && (out[2] != 0 || (a == 2 || b == 2))) {
+    // z edges of slab tiles may cross the seam: two-step passes are single-rank only
+    if (out[2] != 0 || G.n[2] == 1) return {-2, 0, 0, 0, 0};
+  }
+  const int nout = (out[a] != 0) + (out[b] != 0);
+  if (nout == 2) return {-1, 0, 0, 0, 0};
+  const int64_t D = G.depth, tx = G.t[0], ty = G.t[1];
+  // the cell is in-domain along the axis that does not leave the domain: it
+  // is an interior cell of `tile` (nout == 0) or a Dirichlet ghost of `tile`
+  // across the leaving axis (nout == 1). Pick a face array that holds it.
+  EdgeSrc s{nout == 0 ? 0 : 1, tile, 0, 0, 1};
+  // the face to read: across the leaving axis if any, else the first axis
+  const int fa = nout == 1 ? (out[a] != 0 ? a : b) : a;
+  const int64_t cf = c[fa];
+  int face;
+  int64_t layer;
+  if (nout == 0) {  // export of the tile's own boundary layers
+    face = 2 * fa + (cf == 0 ? 0 : 1);
+    layer = cf == 0 ? 0 : D - 1;  // cell at coordinate 0 or t-1
+  } else {          // Dirichlet fixed face; the halo value is the nearest layer
+    face = 2 * fa + (cf < 0 ? 0 : 1);
+    layer = cf < 0 ? D - 1 : 0;
+  }
+  s.face = face;
+  // element offset of cell (c) within the face array and stride along `line`
+  auto off_of = [&](int64_t x, int64_t y, int64_t z) -> int64_t {
+    if (face <= XP) return ((z * ty) + y) * D + layer;                // [z][y][D]
+    if (face <= YP) return ((z * D) + layer) * tx + x;                // [z][D][x]
+    return ((layer * ty) + y) * tx + x;                               // [D][y][x]
+  };
+  const int64_t cx = fa == 0 ? 0 : c[0], cy = fa == 1 ? 0 : c[1], cz = fa == 2 ? 0 : c[2];
+  s.offset = off_of(cx, cy, cz);
+  int64_t d1[3] = {cx, cy, cz};
+  d1[line] += 1;
+  s.stride = off_of(d1[0], d1[1], d1[2]) - s.offset;
+  return s;
+}
+
+EdgePtr Domain::edge_src_ptr(int64_t id, int e, int parity) const {
+  const EdgeSrc s = edge_source(G, id, e);
+  if (s.kind < 0) return {nullptr, 0};
+  const double* base = s.kind == 0 ? faces[s.face][parity] : dir_faces[s.face];
+  return {base + s.tile * G.face_elems[s.face] + s.offset, s.stride};
+}
+
 const double* Domain::face_src_ptr(int64_t id, int f, int parity) const {
   const FaceSrc s = face_source(G, id, f);
   switch (s.kind) {

@@ -164,6 +164,43 @@ struct CudaExec final : Exec {
     d.stats.n_kernels++;
     return Status::ok();
   }
+  int heat2_occ = 0;
+  Status heat2(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
+               const TileItem* dev_items, int st) override {
+    if (d.measure == TILE_MEASURE_XFER_ONLY || n == 0) return Status::ok();
+    Heat2Params P{};
+    HeatParams& p = P.h;
+    p.tx = (int)d.G.t[0];
+    p.ty = (int)d.G.t[1];
+    p.tz = (int)d.G.t[2];
+    p.band = d.band2;
+    p.nbands = p.ty / d.band2;
+    p.nitems = n;
+    p.alpha = d.kernel_alpha;
+    p.cache_flags = d.heat_cache_flags;
+    p.depth = 2;
+    if (dev_items) {
+      p.items = dev_items;
+    } else {
+      if (n > kMaxInlineItems) return make_err(TILE_ESTATE, "internal: too many inline items");
+      for (int i = 0; i < n; ++i)
+        p.inline_items[i] = {d.slot_ptr(in[i]), d.slot_ptr(out[i]), (int32_t)tiles[i], 0};
+    }
+    p.gsrc = d.gsrc_dev[rp];
+    for (int f = 0; f < 6; ++f) {
+      p.fexp[f] = d.faces[f][rp ^ 1];
+      p.face_elems[f] = d.G.face_elems[f];
+    }
+    P.esrc = d.esrc_dev[rp];
+    P.fixed_mask = d.fixed_mask_dev;
+    const int64_t planes = (int64_t)n * p.nbands * p.tz;
+    int64_t grid = (int64_t)sms * heat2_occ;
+    grid = std::max<int64_t>(1, std::min<int64_t>(grid, (planes + 3) / 4));
+    Status r = timed(d, st, [&] { return launch_heat7x2(P, d.heat2_smem, (int)grid, S(st)); });
+    if (r.bad()) return r;
+    d.stats.n_kernels++;
+    return Status::ok();
+  }
   Status sincos(Domain& d, int64_t t, int slot, int64_t iters, int st) override {
     if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
     SincosParams p{};
@@ -293,6 +330,19 @@ struct CudaExec final : Exec {
                       d.items_host[p].size() * sizeof(TileItem), cudaMemcpyHostToDevice));
     }
     CK(heat_configure((int)d.G.t[0], (int)d.G.t[1], d.band, d.stages, d.heat_smem, &heat_occ));
+    if (d.x2_ok) {
+      CK(heat2_configure((int)d.G.t[0], d.band2, d.heat2_smem, &heat2_occ));
+      if (heat2_occ < 1) {  // cannot be resident (e.g. profiler-reserved shared memory)
+        std::fprintf(stderr, "libtiles: two-step kernel not resident on an SM; using single steps\n");
+        d.x2_ok = false;
+      }
+      for (int p = 0; p < 2 && d.x2_ok; ++p)
+        CK(cudaMemcpy(d.esrc_dev[p], d.esrc_host[p].data(), d.esrc_host[p].size() * sizeof(EdgePtr),
+                      cudaMemcpyHostToDevice));
+      if (d.x2_ok)
+        CK(cudaMemcpy(d.fixed_mask_dev, d.fixed_mask_host.data(), d.fixed_mask_host.size(),
+                      cudaMemcpyHostToDevice));
+    }
     if (heat_occ < 1) return make_err(TILE_EINVAL, "heat kernel cannot be resident on an SM");
     CK(cudaStreamSynchronize(streams[0]));
     return Status::ok();

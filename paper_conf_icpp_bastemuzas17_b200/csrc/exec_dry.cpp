@@ -57,6 +57,13 @@ struct DryExec final : Exec {
     }
     return Status::ok();
   }
+  Status heat2(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
+               const TileItem* dev_items, int st) override {
+    const size_t mark = d.trace.size();
+    Status r = heat(d, tiles, in, out, n, rp, dev_items, st);
+    for (size_t i = mark; i < d.trace.size(); ++i) d.trace[i].kind = TILE_OP_KERNEL2;
+    return r;
+  }
   Status sincos(Domain& d, int64_t t, int slot, int64_t iters, int st) override {
     d.stats.n_kernels++;
     put(d, TILE_OP_POINTWISE, st, t, slot, iters, 0);

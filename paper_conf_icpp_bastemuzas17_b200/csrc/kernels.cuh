@@ -20,6 +20,13 @@ struct TileItem {
 
 constexpr int kMaxInlineItems = 8;
 
+// An edge line of ghost cells: cell i at ptr[i * stride] (ptr may be null
+// when the edge is never read).
+struct EdgePtr {
+  const double* ptr;
+  int64_t stride;
+};
+
 // Heat7 launch parameters (§VI.A; DESIGN.md §4 "heat7_tma").
 struct HeatParams {
   int32_t tx, ty, tz;    // tile extents (cells)
@@ -41,6 +48,15 @@ struct HeatParams {
   // L2 policy bits: 1 = TMA loads evict_first, 2 = face exports evict_last
   int32_t cache_flags;
   int32_t depth;  // face depth D (1 or 2): layers per face, increasing coordinate
+};
+
+// Two-step pass (temporal blocking, ghost = 2): u^{s+2} from u^s in one
+// launch; ghosts from depth-2 faces and edge lines (runtime.hpp EdgeSrc).
+struct Heat2Params {
+  HeatParams h;          // shape, items, face sources (read parity), exports
+  const EdgePtr* esrc;   // [tile*12 + e] for the read parity
+  // per tile: bit f set if face f is a Dirichlet fixed face (ring fixed)
+  const uint8_t* fixed_mask;
 };
 
 struct SincosParams {
@@ -75,6 +91,10 @@ cudaError_t heat_configure(int tx, int ty, int band, int stages, size_t smem, in
 cudaError_t launch_heat7(const HeatParams& p, int stages, size_t smem, int grid,
                          cudaStream_t s);
 cudaError_t launch_sincos(const SincosParams& p, int grid, cudaStream_t s);
+// Two-step kernel: returns false from heat2_plan if no specialisation fits.
+bool heat2_plan(int tx, int ty, int max_smem, int* band, size_t* smem);
+cudaError_t heat2_configure(int tx, int band, size_t smem, int* ctas_per_sm);
+cudaError_t launch_heat7x2(const Heat2Params& p, size_t smem, int grid, cudaStream_t s);
 cudaError_t launch_extract(const ExtractParams& p, cudaStream_t s);
 
 }  // namespace tiles

@@ -1,0 +1,365 @@
+// kernels_x2.cu — two Jacobi steps per pass (temporal blocking, §8(f) NEXT
+// #2; DESIGN.md §4 "heat7x2"). A tile with a ghost width of 2 can advance two
+// steps per residency pass: u^{s+2} on the tile needs u^{s+1} on the tile plus
+// its face ring (cells one outside in exactly one axis), which needs u^s on
+// the tile, its depth-2 faces and the 12 edge lines (cells one outside in two
+// axes). Faces come from the neighbours' depth-2 exports (or Dirichlet fixed
+// faces); edge lines are read out of the diagonal neighbours' face exports
+// (EdgePtr table), so no extra exports exist. Every cell update uses the same
+// rounded operations as the single step (reading R1), so two single steps and
+// one double step give bit-identical results.
+//
+// Per CTA (persistent over a contiguous range of (tile, band, z) columns, as
+// heat7_fixed): a producer warp stages u^s planes z0-2 .. z1+1 into a ring of
+// S stages (band rows +-2, depth-2 x-ghost columns, edge cells); consumer
+// warps compute u^{s+1} for plane m (band rows +-1, x ring columns) into one
+// of two shared "mid" planes, then u^{s+2} for plane m-1 from the mid planes
+// (register z-march: mid(m-2) of a thread's own cells stays in registers).
+#include "kernels.cuh"
+#include "ptx.cuh"
+
+#include <cstdio>
+#include <cstdlib>
+
+namespace tiles {
+
+template <int TX, int BY, int S_ = 4>
+struct X2 {
+  static constexpr int HALF = TX / 2;
+  static constexpr int RPP = (BY < 512 / HALF) ? BY : 512 / HALF;
+  static constexpr int NT = RPP * HALF;  // consumer threads
+  static constexpr int NR = BY / RPP;    // output rows per consumer thread
+  static constexpr int S = S_;           // input stages
+  static constexpr int IROWS = BY + 4;   // staged rows y0-2 .. y0+BY+1
+  static constexpr int XOFF = IROWS * TX;
+  static constexpr int STAGE_ELEMS = IROWS * TX + 4 * IROWS;  // + x-ghost [2 sides][IROWS][2]
+  static constexpr int MROWS = BY + 2;   // mid rows y0-1 .. y0+BY
+  static constexpr int MPITCH = TX + 4;  // mid col of x is x + 2 (x = -1 .. TX)
+  static constexpr int MID_ELEMS = MROWS * MPITCH;
+  static constexpr size_t SMEM = (size_t)S * STAGE_ELEMS * 8 + 2 * (size_t)MID_ELEMS * 8 + 2 * S * 8;
+  static_assert(BY % RPP == 0 && NR >= 1 && NR <= 8, "bad x2 config");
+};
+
+constexpr int kEdgeXY = 0, kEdgeXZ = 4, kEdgeYZ = 8;
+__host__ __device__ constexpr uint8_t bit(int f) { return (uint8_t)(1u << f); }
+
+// Producer warp: stage u^s plane z of band y0 of tile `in` into dst.
+template <int TX, int BY, int S>
+__device__ __forceinline__ void stage_x2(double* dst, uint64_t* bar, const double* in,
+                                         const double* const* gs, const EdgePtr* es, int z,
+                                         int ty, int tz, int y0, int lane) {
+  using C = X2<TX, BY, S>;
+  const int lo = y0 - 2 < 0 ? 0 : y0 - 2;
+  const int hi = y0 + BY + 2 > ty ? ty : y0 + BY + 2;
+  const int rlo = lo - (y0 - 2);  // staged row of y = lo
+  const bool inplane = z >= 0 && z < tz;
+  const bool near_ghost = z == -1 || z == tz;
+  // 1) edge cells (regular loads by the warp, generic proxy) — written before
+  //    lane 0's arrive, which releases them to the consumers.
+  if (inplane) {
+    if (lane < 4) {
+      const int gx = lane & 1, gy = lane >> 1;
+      const bool need = gy == 0 ? y0 == 0 : y0 + BY == ty;
+      if (need) {
+        const EdgePtr e = es[kEdgeXY + 2 * gx + gy];
+        if (e.ptr) {
+          const int r = (gy == 0 ? -1 : ty) - (y0 - 2);
+          dst[C::XOFF + gx * 2 * C::IROWS + r * 2 + (gx ? 0 : 1)] = e.ptr[(int64_t)z * e.stride];
+        }
+      }
+    }
+  } else if (near_ghost) {
+    const int gz = z < 0 ? 0 : 1;
+    for (int gy = 0; gy < 2; ++gy) {  // rows y = -1 / ty of the ghost plane
+      const bool need = gy == 0 ? y0 == 0 : y0 + BY == ty;
+      const EdgePtr e = es[kEdgeYZ + 2 * gy + gz];
+      if (need && e.ptr) {
+        const int r = (gy == 0 ? -1 : ty) - (y0 - 2);
+        for (int x = lane; x < TX; x += 32) dst[r * TX + x] = e.ptr[(int64_t)x * e.stride];
+      }
+    }
+    for (int gx = 0; gx < 2; ++gx) {  // x = -1 / TX columns of the ghost plane
+      const EdgePtr e = es[kEdgeXZ + 2 * gx + gz];
+      if (!e.ptr) continue;
+      for (int y = y0 + lane; y < y0 + BY; y += 32)
+        dst[C::XOFF + gx * 2 * C::IROWS + (y - (y0 - 2)) * 2 + (gx ? 0 : 1)] =
+            e.ptr[(int64_t)y * e.stride];
+    }
+  }
+  __syncwarp();
+  if (lane != 0) return;
+  // 2) bulk copies (TMA)
+  const uint64_t pol = policy_evict_normal();
+  fence_proxy_async();
+  uint32_t bytes = 0;
+  const uint32_t row_b = TX * 8;
+  if (inplane) {
+    bytes += (uint32_t)(hi - lo) * row_b + 2u * (uint32_t)(hi - lo) * 16u;
+    if (y0 == 0) bytes += 2 * row_b;
+    if (y0 + BY == ty) bytes += 2 * row_b;
+  } else {
+    bytes += (uint32_t)(hi - lo) * row_b;
+  }
+  mbar_expect_tx(bar, bytes);
+  if (inplane) {
+    const double* plane = in + (size_t)z * ty * TX;
+    bulk_g2s_hint(dst + (size_t)rlo * TX, plane + (size_t)lo * TX, (hi - lo) * row_b, bar, pol);
+    if (y0 == 0)  // rows -2, -1: layers 0, 1 of the y- source, plane z ([z][2][x])
+      bulk_g2s_hint(dst, gs[YM] + (size_t)z * 2 * TX, 2 * row_b, bar, pol);
+    if (y0 + BY == ty)  // rows ty, ty+1: layers 0, 1 of the y+ source
+      bulk_g2s_hint(dst + (size_t)(ty - (y0 - 2)) * TX, gs[YP] + (size_t)z * 2 * TX, 2 * row_b, bar,
+                    pol);
+    const uint32_t xb = (uint32_t)(hi - lo) * 16u;  // [y][2] per side
+    bulk_g2s_hint(dst + C::XOFF + rlo * 2, gs[XM] + ((size_t)z * ty + lo) * 2, xb, bar, pol);
+    bulk_g2s_hint(dst + C::XOFF + 2 * C::IROWS + rlo * 2, gs[XP] + ((size_t)z * ty + lo) * 2, xb,
+                  bar, pol);
+  } else {
+    const int l = z < 0 ? z + 2 : z - tz;  // layer of the z source ([2][y][x])
+    const double* src = (z < 0 ? gs[ZM] : gs[ZP]) + ((size_t)l * ty + lo) * TX;
+    bulk_g2s_hint(dst + (size_t)rlo * TX, src, (hi - lo) * row_b, bar, pol);
+  }
+}
+
+template <int TX, int BY, int S>
+__global__ void __launch_bounds__(X2<TX, BY, S>::NT + 32) heat7x2(const __grid_constant__ Heat2Params P) {
+  using C = X2<TX, BY, S>;
+  const HeatParams& p = P.h;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double* stage_base = reinterpret_cast<double*>(smem_raw);
+  double* mid0 = stage_base + (size_t)C::S * C::STAGE_ELEMS;
+  uint64_t* full = reinterpret_cast<uint64_t*>(mid0 + 2 * C::MID_ELEMS);
+  uint64_t* empty = full + C::S;
+  constexpr int NCW = C::NT / 32;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < C::S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], NCW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  const int ty = p.ty, tz = p.tz;
+  const int64_t P_all = (int64_t)p.nitems * p.nbands * tz;
+  const int64_t pb = P_all * blockIdx.x / gridDim.x, pe = P_all * (blockIdx.x + 1) / gridDim.x;
+  const int lane = (int)threadIdx.x & 31;
+
+  if ((int)threadIdx.x >= C::NT) {  // ---------------------- producer warp
+    uint32_t g = 0;
+    for (int64_t pp = pb; pp < pe;) {
+      const int64_t col = pp / tz;
+      const int z0 = (int)(pp - col * tz);
+      const int z1 = (int)(pe - pp < (int64_t)(tz - z0) ? z0 + (pe - pp) : tz);
+      const int item_i = (int)(col / p.nbands);
+      const int y0 = (int)(col - (int64_t)item_i * p.nbands) * BY;
+      const TileItem it = p.items ? p.items[item_i] : p.inline_items[item_i];
+      const double* const* gs = p.gsrc + (size_t)it.tile * 6;
+      const EdgePtr* es = P.esrc + (size_t)it.tile * 12;
+      for (int z = z0 - 2; z <= z1 + 1; ++z, ++g) {
+        const int s = (int)(g % C::S);
+        mbar_wait(&empty[s], ((g / C::S) & 1u) ^ 1u);
+        stage_x2<TX, BY, S>(stage_base + (size_t)s * C::STAGE_ELEMS, &full[s], it.in, gs, es, z, ty, tz,
+                         y0, lane);
+      }
+      pp += z1 - z0;
+    }
+    return;
+  }
+
+  // ------------------------------------------------------- consumer warps
+  const int tid = (int)threadIdx.x;
+  const int c2 = tid % C::HALF, r0 = tid / C::HALF, xo = c2 * 2;
+  const bool xlo_edge = c2 == 0, xhi_edge = c2 == C::HALF - 1;
+  const double alpha = p.alpha;
+  const uint64_t keep = (p.cache_flags & 2) ? policy_evict_last() : policy_evict_normal();
+  auto cbar = [] { asm volatile("bar.sync 1, %0;" ::"n"(C::NT) : "memory"); };
+  auto wait_g = [&](uint32_t g) { mbar_wait(&full[g % C::S], (g / C::S) & 1u); };
+  auto release_g = [&](uint32_t g) {
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[g % C::S]);
+  };
+  uint32_t seq = 0;
+
+  for (int64_t pp = pb; pp < pe;) {
+    const int64_t col = pp / tz;
+    const int z0 = (int)(pp - col * tz);
+    const int z1 = (int)(pe - pp < (int64_t)(tz - z0) ? z0 + (pe - pp) : tz);
+    const int item_i = (int)(col / p.nbands);
+    const int y0 = (int)(col - (int64_t)item_i * p.nbands) * BY;
+    const TileItem it = p.items ? p.items[item_i] : p.inline_items[item_i];
+    const int64_t tile = it.tile;
+    const uint8_t fm = P.fixed_mask[tile];
+    const int nq = z1 - z0 + 4;  // input planes z0-2 .. z1+1
+
+    // input value of plane stage `st` at (x, y), x in [-2, TX+2)
+    auto U = [&](const double* st, int x, int y) -> double {
+      const int r = y - (y0 - 2);
+      if (x < 0) return st[C::XOFF + r * 2 + (x + 2)];
+      if (x >= TX) return st[C::XOFF + 2 * C::IROWS + r * 2 + (x - TX)];
+      return st[r * TX + x];
+    };
+    auto U2 = [&](const double* st, int x, int y) -> double2 {
+      return *reinterpret_cast<const double2*>(st + (y - (y0 - 2)) * TX + x);
+    };
+    auto stage = [&](uint32_t q) { return stage_base + (size_t)((seq + q) % C::S) * C::STAGE_ELEMS; };
+
+    // exports of the output (D = 2 faces)
+    double* fxm = p.fexp[XM] + tile * p.face_elems[XM];
+    double* fxp = p.fexp[XP] + tile * p.face_elems[XP];
+    double* fym = p.fexp[YM] + tile * p.face_elems[YM] + xo;
+    double* fyp = p.fexp[YP] + tile * p.face_elems[YP] + xo;
+    double* fzm = p.fexp[ZM] + tile * p.face_elems[ZM] + xo;
+    double* fzp = p.fexp[ZP] + tile * p.face_elems[ZP] + xo;
+    const int yb = y0 + r0;
+    double* obase = it.out + (size_t)yb * TX + xo;
+    const size_t plane_elems = (size_t)ty * TX;
+
+    double2 zmr[C::NR];  // mid(o-1) at this thread's own output cells
+    wait_g(seq);
+    wait_g(seq + 1);
+    const int nmid = z1 - z0 + 2;  // mid planes z0-1 .. z1
+    for (int mi = 0; mi < nmid; ++mi) {
+      const int m = z0 - 1 + mi;
+      wait_g(seq + mi + 2);
+      const double* prv = stage(mi);
+      const double* cur = stage(mi + 1);
+      const double* nxt = stage(mi + 2);
+      double* mb = mid0 + (size_t)(mi & 1) * C::MID_ELEMS;
+      const bool zring = m < 0 || m >= tz;
+      const bool zfixed = zring && (fm & bit(m < 0 ? ZM : ZP));
+      // --- u^{s+1}: band rows +-1 (band rows only on z-ring planes), x pairs
+      const int ry0 = zring ? 1 : 0, ry1 = zring ? C::MROWS - 1 : C::MROWS;
+      for (int e = tid; e < (ry1 - ry0) * C::HALF; e += C::NT) {
+        const int mr = ry0 + e / C::HALF;
+        const int x = (e % C::HALF) * 2;
+        const int y = y0 - 1 + mr;
+        double2 v;
+        const bool yout = y < 0 || y >= ty;
+        if (zfixed || (yout && (fm & bit(y < 0 ? YM : YP)))) {
+          v = U2(cur, x, y);  // Dirichlet: the ring keeps its fixed value
+        } else {
+          const double2 c = U2(cur, x, y);
+          const double2 ym = U2(cur, x, y - 1), yp = U2(cur, x, y + 1);
+          const double2 zm = U2(prv, x, y), zp = U2(nxt, x, y);
+          const double xm = U(cur, x - 1, y), xp = U(cur, x + 2, y);
+          v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm.x, zp.x, alpha);
+          v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm.y, zp.y, alpha);
+        }
+        *reinterpret_cast<double2*>(mb + mr * C::MPITCH + x + 2) = v;
+      }
+      if (!zring) {  // x ring columns x = -1, TX for band rows
+        for (int e = tid; e < 2 * BY; e += C::NT) {
+          const int side = e / BY;
+          const int y = y0 + e % BY;
+          const int x = side ? TX : -1;
+          double v;
+          if (fm & bit(side ? XP : XM)) {
+            v = U(cur, x, y);
+          } else {
+            v = heat_update(U(cur, x, y), U(cur, x - 1, y), U(cur, x + 1, y), U(cur, x, y - 1),
+                            U(cur, x, y + 1), U(prv, x, y), U(nxt, x, y), alpha);
+          }
+          mb[(y - y0 + 1) * C::MPITCH + x + 2] = v;
+        }
+      }
+      cbar();                // mid plane m complete; input plane m-1 no longer read
+      release_g(seq + mi);
+      if (mi == 0) {
+#pragma unroll
+        for (int j = 0; j < C::NR; ++j)
+          zmr[j] = *reinterpret_cast<const double2*>(mb + (r0 + j * C::RPP + 1) * C::MPITCH + xo + 2);
+      }
+      if (mi >= 2) {  // --- u^{s+2} for plane o = m-1
+        const int o = m - 1;
+        const double* cb = mid0 + (size_t)((mi - 1) & 1) * C::MID_ELEMS;  // mid(o)
+        const double* nb = mb;                                             // mid(o+1)
+        double* op = obase + (size_t)o * plane_elems;
+        const bool zlo = o < 2, zhi = o >= tz - 2;
+#pragma unroll
+        for (int j = 0; j < C::NR; ++j) {
+          const int r = r0 + j * C::RPP;  // band row
+          const double* crow = cb + (r + 1) * C::MPITCH + xo + 2;
+          const double2 c = *reinterpret_cast<const double2*>(crow);
+          const double2 ym = *reinterpret_cast<const double2*>(crow - C::MPITCH);
+          const double2 yp = *reinterpret_cast<const double2*>(crow + C::MPITCH);
+          const double2 zp = *reinterpret_cast<const double2*>(nb + (r + 1) * C::MPITCH + xo + 2);
+          const double xm = crow[-1], xp = crow[2];
+          double2 v;
+          v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zmr[j].x, zp.x, alpha);
+          v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zmr[j].y, zp.y, alpha);
+          stg2_stream(op + (size_t)j * C::RPP * TX, v);
+          zmr[j] = c;
+          const int y = yb + j * C::RPP;
+          if (xlo_edge) st2_hint(fxm + ((size_t)o * ty + y) * 2, v, keep);
+          if (xhi_edge) st2_hint(fxp + ((size_t)o * ty + y) * 2, v, keep);
+          if (y < 2) st2_hint(fym + ((size_t)o * 2 + y) * TX, v, keep);
+          if (y >= ty - 2) st2_hint(fyp + ((size_t)o * 2 + y - (ty - 2)) * TX, v, keep);
+          if (zlo) st2_hint(fzm + ((size_t)o * ty + y) * TX, v, keep);
+          if (zhi) st2_hint(fzp + ((size_t)(o - (tz - 2)) * ty + y) * TX, v, keep);
+        }
+        cbar();  // mid(o) may be overwritten by the next mid plane
+      } else if (mi == 1) {
+        // nothing to output yet; mid(z0-1) is in registers, mid(z0) in buffer 1
+      }
+    }
+    release_g(seq + nq - 2);
+    release_g(seq + nq - 1);
+    seq += (uint32_t)nq;
+    pp += z1 - z0;
+  }
+}
+
+struct X2Entry {
+  int tx, by;
+  void (*fn)(Heat2Params);
+  int nt;
+  size_t smem;
+};
+#define X2E(TX, BY, S) {TX, BY, heat7x2<TX, BY, S>, X2<TX, BY, S>::NT + 32, X2<TX, BY, S>::SMEM}
+static const X2Entry kX2[] = {X2E(64, 64, 4), X2E(64, 32, 3), X2E(32, 32, 4), X2E(32, 16, 4),
+                              X2E(128, 16, 4), X2E(256, 8, 4)};
+#undef X2E
+
+static const X2Entry* find_x2(int tx, int by) {
+  for (const auto& e : kX2)
+    if (e.tx == tx && e.by == by) return &e;
+  return nullptr;
+}
+
+bool heat2_plan(int tx, int ty, int max_smem, int* band, size_t* smem) {
+  if (const char* eb = std::getenv("TILES_X2_BAND")) {  // tuning override
+    const int by = std::atoi(eb);
+    const X2Entry* e = find_x2(tx, by);
+    if (e && ty % by == 0 && e->smem <= (size_t)max_smem) {
+      *band = by;
+      *smem = e->smem;
+      return true;
+    }
+  }
+  for (int by : {64, 32, 16, 8}) {
+    if (ty % by) continue;
+    const X2Entry* e = find_x2(tx, by);
+    if (e && e->smem <= (size_t)max_smem) {
+      *band = by;
+      *smem = e->smem;
+      return true;
+    }
+  }
+  return false;
+}
+
+cudaError_t heat2_configure(int tx, int band, size_t smem, int* ctas_per_sm) {
+  const X2Entry* e = find_x2(tx, band);
+  if (!e || e->smem != smem) return cudaErrorInvalidValue;
+  cudaError_t r = cudaFuncSetAttribute(e->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (r != cudaSuccess) return r;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, e->fn, e->nt, smem);
+}
+
+cudaError_t launch_heat7x2(const Heat2Params& p, size_t smem, int grid, cudaStream_t s) {
+  const X2Entry* e = find_x2(p.h.tx, p.h.band);
+  if (!e || e->smem != smem) return cudaErrorInvalidValue;
+  void* args[] = {const_cast<Heat2Params*>(&p)};
+  return cudaLaunchKernel(reinterpret_cast<const void*>(e->fn), dim3(grid), dim3(e->nt), args, smem, s);
+}
+
+}  // namespace tiles

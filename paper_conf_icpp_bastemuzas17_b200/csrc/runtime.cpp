@@ -82,6 +82,15 @@ Status domain_create(const int64_t dims[3], const int64_t tdims[3], int ghost,
 
   Domain* d = new Domain();
   d->G = G;
+  if (G.depth == 2 && G.nranks == 1 && opt.two_step >= 0) {
+    int b2 = 0;
+    size_t s2 = 0;
+    if (heat2_plan((int)G.t[0], (int)G.t[1], 227 * 1024, &b2, &s2)) {
+      d->x2_ok = true;
+      d->band2 = b2;
+      d->heat2_smem = s2;
+    }
+  }
   d->opt = opt;
   d->band = band;
   d->stages = stages;
@@ -146,6 +155,9 @@ Status domain_setup(Domain& d) {
   const uint64_t gsrc_bytes = align_up((uint64_t)G.ntiles * 6 * sizeof(double*));
   const uint64_t items_bytes = align_up((uint64_t)G.ntiles * sizeof(TileItem));
   persist += 2 * gsrc_bytes + 2 * items_bytes;
+  const uint64_t esrc_bytes = d.x2_ok ? align_up((uint64_t)G.ntiles * 12 * sizeof(EdgePtr)) : 0;
+  const uint64_t mask_bytes = d.x2_ok ? align_up((uint64_t)G.ntiles) : 0;
+  persist += 2 * esrc_bytes + mask_bytes;
 
   uint64_t budget;
   if (d.opt.device_pool) {
@@ -206,6 +218,10 @@ Status domain_setup(Domain& d) {
       for (int p = 0; p < 2; ++p) d.halo[a][p] = reinterpret_cast<double*>(carve(halo_bytes));
   for (int p = 0; p < 2; ++p) d.gsrc_dev[p] = reinterpret_cast<const double**>(carve(gsrc_bytes));
   for (int p = 0; p < 2; ++p) d.items_dev[p] = reinterpret_cast<TileItem*>(carve(items_bytes));
+  if (d.x2_ok) {
+    for (int p = 0; p < 2; ++p) d.esrc_dev[p] = reinterpret_cast<EdgePtr*>(carve(esrc_bytes));
+    d.fixed_mask_dev = reinterpret_cast<uint8_t*>(carve(mask_bytes));
+  }
   d.slot_base = reinterpret_cast<double*>(d.pool + off);
 
   // ghost-source tables (both parities) and resident item lists
@@ -213,6 +229,17 @@ Status domain_setup(Domain& d) {
     d.gsrc_host[p].resize((size_t)G.ntiles * 6);
     for (int64_t k = 0; k < G.ntiles; ++k)
       for (int f = 0; f < 6; ++f) d.gsrc_host[p][(size_t)k * 6 + f] = d.face_src_ptr(k, f, p);
+  }
+  if (d.x2_ok) {
+    for (int p = 0; p < 2; ++p) {
+      d.esrc_host[p].resize((size_t)G.ntiles * 12);
+      for (int64_t k = 0; k < G.ntiles; ++k)
+        for (int e = 0; e < 12; ++e) d.esrc_host[p][(size_t)k * 12 + e] = d.edge_src_ptr(k, e, p);
+    }
+    d.fixed_mask_host.assign((size_t)G.ntiles, 0);
+    for (int64_t k = 0; k < G.ntiles; ++k)
+      for (int f = 0; f < 6; ++f)
+        if (face_source(G, k, f).kind == 1) d.fixed_mask_host[(size_t)k] |= (uint8_t)(1u << f);
   }
   if (d.mode == MODE_RESIDENT) {
     for (int b = 0; b < 2; ++b) {
@@ -394,7 +421,8 @@ struct ResidentRun {
   std::vector<std::vector<int>> nbr;  // neighbour batches (excluding self)
   bool need_load, need_extract, multi;
   bool entry_wait = false;  // first op of every batch waits ev_phase (phase join)
-  int bit0, fp0, T;
+  int bit0, fp0, T;         // T = number of passes (a pass advances 1 or 2 steps)
+  std::vector<int> kpass;   // steps per pass
   double alpha;
 
   ResidentRun(Domain& dd) : d(dd), X(*dd.exec), G(dd.G) {}
@@ -494,8 +522,11 @@ struct ResidentRun {
     }
     const int bit = bit0 ^ (s & 1);
     const int rp = fp0 ^ (s & 1);
-    r = X.heat(d, nullptr, nullptr, nullptr, (int)ntl(b), rp,
-               d.items_dev[bit] ? d.items_dev[bit] + tile0(b) : nullptr, b.stream);
+    const TileItem* items = d.items_dev[bit] ? d.items_dev[bit] + tile0(b) : nullptr;
+    if (kpass[(size_t)s] == 2)
+      r = X.heat2(d, nullptr, nullptr, nullptr, (int)ntl(b), rp, items, b.stream);
+    else
+      r = X.heat(d, nullptr, nullptr, nullptr, (int)ntl(b), rp, items, b.stream);
     if (r.bad()) return r;
     (void)alpha;
     return X.record(d, ev_layer(d, (int64_t)i, s & 1), b.stream);
@@ -592,9 +623,24 @@ static Status upload_dirichlet_if_needed(Domain& d);
 // the middle steps (one launch per step, or bottom/top/interior with slab
 // halos), and layer batches again for the final step so each layer's D2H can
 // start as soon as its last kernel ends. Phases are joined through ev_phase.
-static Status run_heat_resident(Domain& d, double alpha, int T, int S, bool serial) {
+// Steps -> passes: with ghost 2 (and a two-step kernel for the tile shape)
+// a pass advances two steps; an odd remainder is one single-step pass.
+static std::vector<int> plan_passes(const Domain& d, int steps) {
+  std::vector<int> k;
+  if (d.x2_ok && (d.opt.two_step > 0 || d.mode == MODE_STREAM)) {
+    for (int i = 0; i < steps / 2; ++i) k.push_back(2);
+    if (steps & 1) k.push_back(1);
+  } else {
+    k.assign((size_t)steps, 1);
+  }
+  return k;
+}
+
+static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool serial) {
   const bool load = !d.resident_valid;
   const int64_t nL = d.G.n[2];
+  const std::vector<int> kp = plan_passes(d, steps);
+  const int T = (int)kp.size();  // passes
   struct Phase {
     int steps;
     bool layered;
@@ -614,10 +660,13 @@ static Status run_heat_resident(Domain& d, double alpha, int T, int S, bool seri
   }
   int bit = d.res_bit, fp = d.face_parity;
   std::vector<std::pair<Batch, int>> last;  // batches of the last phase + final event
+  size_t pass0 = 0;
   for (size_t pi = 0; pi < ph.size(); ++pi) {
     ResidentRun R(d);
     R.alpha = alpha;
     R.T = ph[pi].steps;
+    R.kpass.assign(kp.begin() + (long)pass0, kp.begin() + (long)(pass0 + (size_t)R.T));
+    pass0 += (size_t)R.T;
     R.need_load = pi == 0 && load;
     R.need_extract = pi == 0 && !d.faces_valid;
     R.multi = d.G.nranks > 1;
@@ -663,7 +712,8 @@ static Status run_stream(Domain& d, const tile_kernel& k, int T, int S) {
   Sched sc(d, P);
   const bool heat = k.kind == TILE_KERNEL_HEAT7;
   const bool fuse = !heat && d.opt.fuse_pointwise_steps;
-  const int passes = fuse ? (T > 0 ? 1 : 0) : T;
+  const std::vector<int> kp = heat ? plan_passes(d, T) : std::vector<int>();
+  const int passes = heat ? (int)kp.size() : fuse ? (T > 0 ? 1 : 0) : T;
   const int64_t iters = fuse ? (int64_t)k.inner_iters * T : k.inner_iters;
   const int64_t N = G.ntiles;
   const bool multi = G.nranks > 1;
@@ -758,7 +808,8 @@ static Status run_stream(Domain& d, const tile_kernel& k, int T, int S) {
         }
         const int64_t tl[1] = {t};
         const int is[1] = {in}, os[1] = {out};
-        r = X.heat(d, tl, is, os, 1, rp, nullptr, st);
+        r = kp[(size_t)s] == 2 ? X.heat2(d, tl, is, os, 1, rp, nullptr, st)
+                               : X.heat(d, tl, is, os, 1, rp, nullptr, st);
         if (r.bad()) return r;
         r = X.record(d, ev_tile(d, t, s & 1), st);
         if (r.bad()) return r;
@@ -787,7 +838,7 @@ static Status run_stream(Domain& d, const tile_kernel& k, int T, int S) {
       if (r.bad()) return r;
     }
   }
-  if (heat) d.face_parity ^= (T & 1);
+  if (heat) d.face_parity ^= (passes & 1);
   return Status::ok();
 }
 

@@ -58,6 +58,24 @@ struct FaceSrc {
   int64_t val;
 };
 FaceSrc face_source(const Geometry& G, int64_t id, int f);
+
+// Edge ghost cells for a two-step pass (D = 2): the 12 lines of cells just
+// outside two faces at once (x,y,z = -1 or t in two axes). Edge e: 0..3 = xy
+// (cells along z), 4..7 = xz (along y), 8..11 = yz (along x); within a group
+// (e & 3) = 2*g_a + g_b with g = 0 for the minus side, 1 for the plus side of
+// the group's first and second axis. Cell i of the line is ptr[i * stride].
+// The value lives in a depth-2 face array: a diagonal neighbour's export, or
+// a Dirichlet fixed face of the tile that borders the out-of-domain axis.
+// kind: 0 export (parity-dependent), 1 Dirichlet face, -1 not needed (both
+// axes leave a Dirichlet domain), -2 unsupported (crosses a slab seam).
+struct EdgeSrc {
+  int kind;
+  int64_t tile;   // owner of the face array
+  int face;       // which face array of that tile
+  int64_t offset; // element offset of cell 0 within that tile's face
+  int64_t stride; // element stride along the line
+};
+EdgeSrc edge_source(const Geometry& G, int64_t id, int e);
 void ghost_map(const Geometry& G, int64_t id, int64_t* out);  // (t+2g)^3 box
 
 // ----------------------------------------------------------------- executor
@@ -75,6 +93,9 @@ struct Exec {
   virtual Status heat(Domain& d, const int64_t* tiles, const int* in_slots, const int* out_slots,
                       int nitems, int read_parity, const TileItem* dev_items, int stream) = 0;
   virtual Status sincos(Domain& d, int64_t tile, int slot, int64_t iters, int stream) = 0;
+  // two-step pass (temporal blocking): same arguments as heat
+  virtual Status heat2(Domain& d, const int64_t* tiles, const int* in_slots, const int* out_slots,
+                       int nitems, int read_parity, const TileItem* dev_items, int stream) = 0;
   virtual Status extract(Domain& d, int64_t tile0, int64_t ntile, int slot0, int parity,
                          const TileItem* dev_items, int stream) = 0;
   virtual Status faces_h2d(Domain& d, int parity, int stream) = 0;
@@ -121,6 +142,13 @@ struct Domain {
   double* dir_faces[6] = {};               // Dirichlet fixed faces
   double* halo[2][2] = {};                 // [0 = from below (z-), 1 = from above (z+)][parity]
   const double** gsrc_dev[2] = {};         // [parity] -> ntiles*6 pointers
+  EdgePtr* esrc_dev[2] = {};               // [parity] -> ntiles*12 (D = 2 only)
+  std::vector<EdgePtr> esrc_host[2];
+  uint8_t* fixed_mask_dev = nullptr;       // per tile: Dirichlet faces (bit f)
+  std::vector<uint8_t> fixed_mask_host;
+  bool x2_ok = false;                      // two-step passes available
+  int band2 = 0, heat2_grid = 0;
+  size_t heat2_smem = 0;
   TileItem* items_dev[2] = {};             // resident mode: [bit] -> ntiles items
   double* slot_base = nullptr;
   int nslots = 0;
@@ -177,6 +205,7 @@ struct Domain {
   double* slot_ptr(int s) const { return slot_base + (int64_t)s * G.tile_elems; }
   double* host_tile(int64_t k) const { return host + k * G.tile_elems; }
   const double* face_src_ptr(int64_t id, int f, int parity) const;
+  EdgePtr edge_src_ptr(int64_t id, int e, int parity) const;
 };
 
 // runtime.cpp

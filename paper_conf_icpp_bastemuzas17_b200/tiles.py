@@ -32,7 +32,7 @@ TILE_KERNEL_HEAT7, TILE_KERNEL_SINCOS = 1, 2
 TILE_SCHED_AUTO, TILE_SCHED_RESIDENT, TILE_SCHED_STREAM, TILE_SCHED_SYNC = 0, 1, 2, 3
 TILE_MEASURE_NORMAL, TILE_MEASURE_XFER_ONLY, TILE_MEASURE_COMP_ONLY = 0, 1, 2
 OP_NAMES = {1: "h2d", 2: "d2h", 3: "kernel", 4: "record", 5: "wait", 6: "faces_h2d",
-            7: "extract", 8: "halo", 9: "drop", 10: "hit", 11: "pointwise"}
+            7: "extract", 8: "halo", 9: "drop", 10: "hit", 11: "pointwise", 12: "kernel2"}
 SCHEDS = {"auto": 0, "resident": 1, "stream": 2, "sync": 3}
 BCS = {"periodic": 0, "dirichlet": 1}
 
@@ -44,7 +44,8 @@ class TileOptions(ctypes.Structure):
                 ("nranks", ctypes.c_int32), ("rank", ctypes.c_int32),
                 ("nccl_unique_id", ctypes.c_void_p), ("sched", ctypes.c_int),
                 ("dry_run", ctypes.c_int32), ("fuse_pointwise_steps", ctypes.c_int32),
-                ("local_group", ctypes.c_void_p), ("pageable_host", ctypes.c_int32)]
+                ("local_group", ctypes.c_void_p), ("pageable_host", ctypes.c_int32),
+                ("two_step", ctypes.c_int32)]
 
 
 class TileKernel(ctypes.Structure):
@@ -66,7 +67,8 @@ class TileInfo(ctypes.Structure):
                 ("tile_dims", ctypes.c_int64 * 3), ("tiles", ctypes.c_int64 * 3),
                 ("ntiles", ctypes.c_int64), ("z_offset", ctypes.c_int64), ("ghost", ctypes.c_int32),
                 ("nslots", ctypes.c_int32), ("sched", ctypes.c_int32), ("resident", ctypes.c_int32),
-                ("device_bytes", ctypes.c_uint64), ("host_bytes", ctypes.c_uint64)]
+                ("device_bytes", ctypes.c_uint64), ("host_bytes", ctypes.c_uint64),
+                ("steps_per_pass", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
     def as_dict(self):
         out = {}
@@ -169,7 +171,7 @@ class Domain:
     def __init__(self, dims, tile_dims, ghost=1, bc="periodic", device=-1, device_budget_bytes=0,
                  sched="auto", nranks=1, rank=0, nccl_id=None, dry_run=False,
                  fuse_pointwise_steps=True, device_pool=None, streams=None, local_group=None,
-                 pageable_host=False):
+                 pageable_host=False, two_step=0):
         self._h = None
         self.dims = tuple(int(v) for v in dims)
         self.tile_dims = tuple(int(v) for v in tile_dims)
@@ -198,6 +200,7 @@ class Domain:
         o.dry_run = 1 if dry_run else 0
         o.fuse_pointwise_steps = 1 if fuse_pointwise_steps else 0
         o.pageable_host = 1 if pageable_host else 0
+        o.two_step = int(two_step)
         self._group = local_group
         if local_group is not None:
             o.local_group = local_group.handle

@@ -290,3 +290,20 @@ def test_ghost2_faces_bit_exact(bc, td):
     b = _budget(dims, td, 3, bc=bc)
     out, ref, _, _ = _heat(dims, td, 5, bc=bc, ghost=2, sched="stream", device_budget_bytes=b * 2)
     assert np.array_equal(out, ref)
+
+
+@pytest.mark.parametrize("bc,dims,td,runs", [("periodic", (128, 64, 64), (64, 64, 16), [6, 3]),
+                                             ("dirichlet", (128, 64, 64), (64, 32, 16), [4, 5]),
+                                             ("periodic", (64, 64, 32), (32, 32, 8), [7]),
+                                             ("periodic", (256, 64, 16), (128, 16, 8), [4]),
+                                             ("dirichlet", (64, 32, 32), (32, 16, 8), [2, 2, 3])])
+def test_two_step_passes_bit_exact(bc, dims, td, runs):
+    """ghost = 2 runs two Jacobi steps per pass (heat7x2): bit-identical to
+    single steps and to the oracle, resident and out-of-core."""
+    out, ref, info, st = _heat(dims, td, sum(runs), bc=bc, ghost=2, runs=runs, two_step=1)
+    assert np.array_equal(out, ref)
+    assert info["steps_per_pass"] == 2
+    b = _budget(dims, td, 4, bc=bc)
+    out, ref, info, _ = _heat(dims, td, sum(runs), bc=bc, ghost=2, runs=runs, sched="stream",
+                              device_budget_bytes=b * 2)
+    assert np.array_equal(out, ref) and info["steps_per_pass"] == 2

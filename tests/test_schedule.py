@@ -265,3 +265,22 @@ def test_ghost2_schedules_replay_to_oracle(bc, sched):
     if sched == "stream":
         kw["device_budget_bytes"] = _budget_for(dims, td, 5, sched="stream", bc=bc, ghost=2)
     _run_and_replay(dims, td, [3, 2], 2, seeds=(0, 5), bc=bc, ghost=2, **kw)
+
+
+@pytest.mark.parametrize("bc", ["periodic", "dirichlet"])
+@pytest.mark.parametrize("sched,td", [("resident", (32, 16, 8)), ("stream", (32, 16, 8)),
+                                      ("resident", (32, 32, 4)), ("resident", (32, 16, 16))])
+def test_two_step_passes_replay_to_oracle(bc, sched, td):
+    """ghost = 2: passes of two steps (temporal blocking). The replay builds
+    each tile's u^s ghost region only from what the schedule made available
+    (depth-2 faces of the neighbours at the read parity, edge cells out of the
+    diagonal neighbours' faces, Dirichlet halo) and NaN elsewhere; two oracle
+    steps must give the untiled oracle bit-exactly with no NaN reaching the
+    tile."""
+    dims = (64, 32, 32)
+    kw = {"sched": sched, "two_step": 1}
+    if sched == "stream":
+        kw["device_budget_bytes"] = _budget_for(dims, td, 3, sched="stream", bc=bc, ghost=2)
+    d = _run_and_replay(dims, td, [5, 2], 2, seeds=(0, 3), bc=bc, ghost=2, **kw)
+    ops = [op[0] for op in d.trace()]
+    assert "kernel2" in ops
