@@ -505,7 +505,23 @@ def run_c5_leg(args):
     torch.cuda.set_device(lr)
     if ws > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", lr))
-    n = args.n or 4096
+    n = args.n
+    if not n:
+        # SURVEY §8(d) fallback ladder: the largest n whose pinned host stores
+        # (all ranks of this node, single array + faces) fit 0.8 x MemAvailable
+        import psutil
+        avail = psutil.virtual_memory().available
+        nloc = int(os.environ.get("LOCAL_WORLD_SIZE", str(ws)))
+        n = 2048
+        for cand in (4096, 3584, 3072, 2560, 2048):
+            per_rank = cand * cand * (cand // (8 if ws == 1 else ws)) * 8 * 1.05
+            if per_rank * (1 if ws == 1 else nloc) <= 0.8 * avail:
+                n = cand
+                break
+        if ws > 1:  # every rank must use the same grid
+            t = torch.tensor([n], dtype=torch.int64, device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MIN)
+            n = int(t.item())
     nzl = n // 8 if ws == 1 else n // ws
     gdims = (n, n, nzl * ws)
     td = (256, 256, 64)
