@@ -247,18 +247,28 @@ __global__ void __launch_bounds__(X2<TX, BY, S>::NT + 32) heat7x2(const __grid_c
         *reinterpret_cast<double2*>(mb + mr * C::MPITCH + x + 2) = v;
       }
       if (!zring) {  // x ring columns x = -1, TX for band rows
-        for (int e = tid; e < 2 * BY; e += C::NT) {
+        // on warps that did not take an extra row above (load balance)
+        constexpr int RB = (C::MROWS * C::HALF) % C::NT == 0 ? 0
+                           : (((C::MROWS * C::HALF) % C::NT + 31) / 32) * 32;
+        constexpr int R0 = (C::NT - RB >= 2 * BY) ? RB : 0;
+        const int e = tid - R0;
+        if (e >= 0 && e < 2 * BY) {
           const int side = e / BY;
           const int y = y0 + e % BY;
-          const int x = side ? TX : -1;
+          const int rr = y - (y0 - 2);
+          const double* xb = cur + C::XOFF + side * 2 * C::IROWS + rr * 2;  // [rr][2]
+          const int own = side ? 0 : 1, far = side ? 1 : 0;   // layer of x = -1/TX, -2/TX+1
           double v;
           if (fm & bit(side ? XP : XM)) {
-            v = U(cur, x, y);
+            v = xb[own];
           } else {
-            v = heat_update(U(cur, x, y), U(cur, x - 1, y), U(cur, x + 1, y), U(cur, x, y - 1),
-                            U(cur, x, y + 1), U(prv, x, y), U(nxt, x, y), alpha);
+            const double inner = cur[rr * TX + (side ? TX - 1 : 0)];
+            const double xm = side ? inner : xb[far], xp = side ? xb[far] : inner;
+            v = heat_update(xb[own], xm, xp, xb[own - 2], xb[own + 2],
+                            prv[C::XOFF + side * 2 * C::IROWS + rr * 2 + own],
+                            nxt[C::XOFF + side * 2 * C::IROWS + rr * 2 + own], alpha);
           }
-          mb[(y - y0 + 1) * C::MPITCH + x + 2] = v;
+          mb[(y - y0 + 1) * C::MPITCH + (side ? TX + 2 : 1)] = v;
         }
       }
       cbar();                // mid plane m complete; input plane m-1 no longer read
@@ -309,19 +319,21 @@ __global__ void __launch_bounds__(X2<TX, BY, S>::NT + 32) heat7x2(const __grid_c
 }
 
 struct X2Entry {
-  int tx, by;
+  int tx, by, stages;
   void (*fn)(Heat2Params);
   int nt;
   size_t smem;
 };
-#define X2E(TX, BY, S) {TX, BY, heat7x2<TX, BY, S>, X2<TX, BY, S>::NT + 32, X2<TX, BY, S>::SMEM}
-static const X2Entry kX2[] = {X2E(64, 64, 4), X2E(64, 32, 3), X2E(32, 32, 4), X2E(32, 16, 4),
-                              X2E(128, 16, 4), X2E(256, 8, 4)};
+#define X2E(TX, BY, S) {TX, BY, S, heat7x2<TX, BY, S>, X2<TX, BY, S>::NT + 32, X2<TX, BY, S>::SMEM}
+static const X2Entry kX2[] = {X2E(64, 64, 4), X2E(64, 32, 6), X2E(64, 32, 5), X2E(64, 32, 4),
+                              X2E(32, 32, 6), X2E(32, 16, 6), X2E(128, 16, 5), X2E(256, 8, 5)};
 #undef X2E
 
-static const X2Entry* find_x2(int tx, int by) {
+static const X2Entry* find_x2(int tx, int by, int st = 0) {
+  if (!st)
+    if (const char* es = std::getenv("TILES_X2_STAGES")) st = std::atoi(es);  // tuning override
   for (const auto& e : kX2)
-    if (e.tx == tx && e.by == by) return &e;
+    if (e.tx == tx && e.by == by && (!st || e.stages == st)) return &e;
   return nullptr;
 }
 
