@@ -113,6 +113,15 @@ typedef struct {
                                    the paper's "CUDA pageable" baseline (P:L37,
                                    Fig. 1/5); copies are staged by the driver
                                    and do not overlap. 0 (default): pinned. */
+  int32_t stream_through;       /* HEAT7 run starting from a fresh upload: 0
+                                   (default) = per z-layer trapezoid (gather the
+                                   layer + T halo planes, T sweeps, D2H the
+                                   exact core) when T <= tile_dims[2] / 2 and
+                                   the scratch fits, so H2D, compute and D2H of
+                                   different layers overlap; each layer's result
+                                   is also written back to the device array once
+                                   no other layer reads its initial data. -1 =
+                                   never. */
   int32_t two_step;             /* HEAT7 with ghost >= 2: 0 (default) = two
                                    steps per pass in the streaming schedule
                                    (halves host-link bytes per step), single
@@ -162,7 +171,11 @@ typedef enum {
   TILE_OP_DROP = 9,     /* tile a leaves slot b without a copy (clean) */
   TILE_OP_HIT = 10,     /* tile a found in slot b (P:L90 cache hit) */
   TILE_OP_POINTWISE = 11,/* compute-intensive kernel on tile a in slot b, c iterations */
-  TILE_OP_KERNEL2 = 12   /* like KERNEL, two steps in one pass (ghost width 2) */
+  TILE_OP_KERNEL2 = 12,  /* like KERNEL, two steps in one pass (ghost width 2) */
+  TILE_OP_GATHER = 13,   /* layer a + halo -> dense slab at slot b: c planes from z = d */
+  TILE_OP_SWEEP = 14,    /* slab slot a -> slab slot b, planes [c, d) */
+  TILE_OP_SCATTER = 15,  /* slab slot a core planes from c -> tile-blocked slots from b (layer d) */
+  TILE_OP_COPY = 16      /* device copy of c tile slots: slot a -> slot b */
 } tile_op_kind;
 
 typedef struct {

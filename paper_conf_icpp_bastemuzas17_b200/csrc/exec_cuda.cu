@@ -164,6 +164,59 @@ struct CudaExec final : Exec {
     d.stats.n_kernels++;
     return Status::ok();
   }
+  SlabParams slab_base(Domain& d) {
+    SlabParams p{};
+    p.nx = d.G.l[0];
+    p.ny = d.G.l[1];
+    p.nz = d.G.l[2];
+    p.tx = d.G.t[0];
+    p.ty = d.G.t[1];
+    p.tz = d.G.t[2];
+    p.ntx = d.G.n[0];
+    p.nty = d.G.n[1];
+    p.tile_elems = d.G.tile_elems;
+    p.alpha = d.kernel_alpha;
+    return p;
+  }
+  Status slab_gather(Domain& d, int64_t, int src_bit, int slab, int64_t zbase, int64_t planes,
+                     int st) override {
+    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
+    SlabParams p = slab_base(d);
+    p.tiles = d.slot_ptr(src_bit ? (int)d.G.ntiles : 0);
+    p.slab = d.slot_ptr(slab);
+    p.zbase = zbase;
+    p.planes = planes;
+    Status r = timed(d, st, [&] { return launch_slab_gather(p, sms, S(st)); });
+    if (r.bad()) return r;
+    d.stats.n_kernels++;
+    return Status::ok();
+  }
+  Status slab_sweep(Domain& d, int src, int dst, int lo, int hi, int st) override {
+    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
+    SlabParams p = slab_base(d);
+    Status r = timed(d, st, [&] {
+      return launch_slab_sweep(p, d.slot_ptr(src), d.slot_ptr(dst), lo, hi, sms, S(st));
+    });
+    if (r.bad()) return r;
+    d.stats.n_kernels++;
+    return Status::ok();
+  }
+  Status slab_scatter(Domain& d, int slab, int first, int out, int64_t, int st) override {
+    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
+    SlabParams p = slab_base(d);
+    p.slab = d.slot_ptr(slab);
+    p.out = d.slot_ptr(out);
+    Status r = timed(d, st, [&] { return launch_slab_scatter(p, first, sms, S(st)); });
+    if (r.bad()) return r;
+    d.stats.n_kernels++;
+    return Status::ok();
+  }
+  Status copy_slots(Domain& d, int src, int dst, int64_t n, int st) override {
+    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
+    CK(cudaMemcpyAsync(d.slot_ptr(dst), d.slot_ptr(src), (size_t)n * d.G.tile_elems * 8,
+                       cudaMemcpyDeviceToDevice, S(st)));
+    return Status::ok();
+  }
   int heat2_occ = 0;
   Status heat2(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
                const TileItem* dev_items, int st) override {

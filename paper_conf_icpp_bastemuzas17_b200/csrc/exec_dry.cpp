@@ -64,6 +64,26 @@ struct DryExec final : Exec {
     for (size_t i = mark; i < d.trace.size(); ++i) d.trace[i].kind = TILE_OP_KERNEL2;
     return r;
   }
+  Status slab_gather(Domain& d, int64_t layer, int, int slab, int64_t zbase, int64_t planes,
+                     int st) override {
+    d.stats.n_kernels++;
+    put(d, TILE_OP_GATHER, st, layer, slab, planes, zbase);
+    return Status::ok();
+  }
+  Status slab_sweep(Domain& d, int src, int dst, int lo, int hi, int st) override {
+    d.stats.n_kernels++;
+    put(d, TILE_OP_SWEEP, st, src, dst, lo, hi);
+    return Status::ok();
+  }
+  Status slab_scatter(Domain& d, int slab, int first, int out, int64_t layer, int st) override {
+    d.stats.n_kernels++;
+    put(d, TILE_OP_SCATTER, st, slab, out, first, layer);
+    return Status::ok();
+  }
+  Status copy_slots(Domain& d, int src, int dst, int64_t n, int st) override {
+    put(d, TILE_OP_COPY, st, src, dst, n, 0);
+    return Status::ok();
+  }
   Status sincos(Domain& d, int64_t t, int slot, int64_t iters, int st) override {
     d.stats.n_kernels++;
     put(d, TILE_OP_POINTWISE, st, t, slot, iters, 0);

@@ -91,6 +91,23 @@ cudaError_t heat_configure(int tx, int ty, int band, int stages, size_t smem, in
 cudaError_t launch_heat7(const HeatParams& p, int stages, size_t smem, int grid,
                          cudaStream_t s);
 cudaError_t launch_sincos(const SincosParams& p, int grid, cudaStream_t s);
+
+// Stream-through (trapezoid) slab kernels (kernels_slab.cu).
+struct SlabParams {
+  int64_t nx, ny, nz;           // rank-local grid (nz wraps the gather)
+  int64_t tx, ty, tz, ntx, nty;
+  int64_t tile_elems;
+  int64_t zbase;                // local z of slab plane 0 (gather)
+  int64_t planes;               // planes to gather
+  const double* tiles;          // tile-blocked array (gather source)
+  double* slab;                 // dense slab [planes][ny][nx]
+  double* out;                  // tile-blocked layer (scatter destination)
+  double alpha;
+};
+cudaError_t launch_slab_gather(const SlabParams& p, int sms, cudaStream_t s);
+cudaError_t launch_slab_sweep(const SlabParams& p, const double* src, double* dst, int lo, int hi,
+                              int sms, cudaStream_t s);
+cudaError_t launch_slab_scatter(const SlabParams& p, int first, int sms, cudaStream_t s);
 // Two-step kernel: returns false from heat2_plan if no specialisation fits.
 bool heat2_plan(int tx, int ty, int max_smem, int* band, size_t* smem);
 cudaError_t heat2_configure(int tx, int band, size_t smem, int* ctas_per_sm);

@@ -23,8 +23,9 @@
 
 namespace tiles {
 
-template <int TX, int BY, int S_ = 4>
+template <int TX, int BY, int S_ = 4, int MB_ = 2>
 struct X2 {
+  static constexpr int MB = MB_;         // mid planes: 2 (phases per plane) or 3 (pipelined)
   static constexpr int HALF = TX / 2;
   static constexpr int RPP = (BY < 512 / HALF) ? BY : 512 / HALF;
   static constexpr int NT = RPP * HALF;  // consumer threads
@@ -36,7 +37,7 @@ struct X2 {
   static constexpr int MROWS = BY + 2;   // mid rows y0-1 .. y0+BY
   static constexpr int MPITCH = TX + 4;  // mid col of x is x + 2 (x = -1 .. TX)
   static constexpr int MID_ELEMS = MROWS * MPITCH;
-  static constexpr size_t SMEM = (size_t)S * STAGE_ELEMS * 8 + 2 * (size_t)MID_ELEMS * 8 + 2 * S * 8;
+  static constexpr size_t SMEM = (size_t)S * STAGE_ELEMS * 8 + MB * (size_t)MID_ELEMS * 8 + 2 * S * 8;
   static_assert(BY % RPP == 0 && NR >= 1 && NR <= 8, "bad x2 config");
 };
 
@@ -48,7 +49,7 @@ template <int TX, int BY, int S>
 __device__ __forceinline__ void stage_x2(double* dst, uint64_t* bar, const double* in,
                                          const double* const* gs, const EdgePtr* es, int z,
                                          int ty, int tz, int y0, int lane) {
-  using C = X2<TX, BY, S>;
+  using C = X2<TX, BY, S, 2>;  // stage layout does not depend on MB
   const int lo = y0 - 2 < 0 ? 0 : y0 - 2;
   const int hi = y0 + BY + 2 > ty ? ty : y0 + BY + 2;
   const int rlo = lo - (y0 - 2);  // staged row of y = lo
@@ -120,14 +121,14 @@ __device__ __forceinline__ void stage_x2(double* dst, uint64_t* bar, const doubl
   }
 }
 
-template <int TX, int BY, int S>
-__global__ void __launch_bounds__(X2<TX, BY, S>::NT + 32) heat7x2(const __grid_constant__ Heat2Params P) {
-  using C = X2<TX, BY, S>;
+template <int TX, int BY, int S, int MB>
+__global__ void __launch_bounds__(X2<TX, BY, S, MB>::NT + 32) heat7x2(const __grid_constant__ Heat2Params P) {
+  using C = X2<TX, BY, S, MB>;
   const HeatParams& p = P.h;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   double* stage_base = reinterpret_cast<double*>(smem_raw);
   double* mid0 = stage_base + (size_t)C::S * C::STAGE_ELEMS;
-  uint64_t* full = reinterpret_cast<uint64_t*>(mid0 + 2 * C::MID_ELEMS);
+  uint64_t* full = reinterpret_cast<uint64_t*>(mid0 + MB * C::MID_ELEMS);
   uint64_t* empty = full + C::S;
   constexpr int NCW = C::NT / 32;
   if (threadIdx.x == 0) {
@@ -214,16 +215,55 @@ __global__ void __launch_bounds__(X2<TX, BY, S>::NT + 32) heat7x2(const __grid_c
     const size_t plane_elems = (size_t)ty * TX;
 
     double2 zmr[C::NR];  // mid(o-1) at this thread's own output cells
+    // u^{s+2} of plane o: MB == 2 at iteration mi: o = z0+mi-2 (mid(o), mid(o+1)
+    // in buffers (mi-1)%2, mi%2); MB == 3: o = z0+mi-3 (buffers (mi-2)%3, (mi-1)%3)
+    auto output_plane = [&](int mi) {
+      const int o = z0 + mi - (MB == 3 ? 3 : 2);
+      const double* cb = mid0 + (size_t)((mi - (MB == 3 ? 2 : 1)) % MB) * C::MID_ELEMS;  // mid(o)
+      const double* nb = mid0 + (size_t)((mi - (MB == 3 ? 1 : 0)) % MB) * C::MID_ELEMS;  // mid(o+1)
+      double* op = obase + (size_t)o * plane_elems;
+      const bool zlo = o < 2, zhi = o >= tz - 2;
+#pragma unroll
+      for (int j = 0; j < C::NR; ++j) {
+        const int r = r0 + j * C::RPP;  // band row
+        const double* crow = cb + (r + 1) * C::MPITCH + xo + 2;
+        const double2 c = *reinterpret_cast<const double2*>(crow);
+        const double2 ym = *reinterpret_cast<const double2*>(crow - C::MPITCH);
+        const double2 yp = *reinterpret_cast<const double2*>(crow + C::MPITCH);
+        const double2 zp = *reinterpret_cast<const double2*>(nb + (r + 1) * C::MPITCH + xo + 2);
+        const double xm = crow[-1], xp = crow[2];
+        double2 v;
+        v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zmr[j].x, zp.x, alpha);
+        v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zmr[j].y, zp.y, alpha);
+        stg2_stream(op + (size_t)j * C::RPP * TX, v);
+        zmr[j] = c;
+        const int y = yb + j * C::RPP;
+        if (xlo_edge) st2_hint(fxm + ((size_t)o * ty + y) * 2, v, keep);
+        if (xhi_edge) st2_hint(fxp + ((size_t)o * ty + y) * 2, v, keep);
+        if (y < 2) st2_hint(fym + ((size_t)o * 2 + y) * TX, v, keep);
+        if (y >= ty - 2) st2_hint(fyp + ((size_t)o * 2 + y - (ty - 2)) * TX, v, keep);
+        if (zlo) st2_hint(fzm + ((size_t)o * ty + y) * TX, v, keep);
+        if (zhi) st2_hint(fzp + ((size_t)(o - (tz - 2)) * ty + y) * TX, v, keep);
+      }
+    };
     wait_g(seq);
     wait_g(seq + 1);
     const int nmid = z1 - z0 + 2;  // mid planes z0-1 .. z1
-    for (int mi = 0; mi < nmid; ++mi) {
+    // MB == 3: iteration mi computes mid(m) and, independently, the output
+    // of plane m-2 (one barrier per plane); MB == 2: mid(m), barrier,
+    // output of plane m-1, barrier.
+    for (int mi = 0; mi < nmid + (MB == 3 ? 1 : 0); ++mi) {
       const int m = z0 - 1 + mi;
+      if (MB == 3 && mi == nmid) {  // drain: last output only
+        output_plane(mi);
+        cbar();
+        break;
+      }
       wait_g(seq + mi + 2);
       const double* prv = stage(mi);
       const double* cur = stage(mi + 1);
       const double* nxt = stage(mi + 2);
-      double* mb = mid0 + (size_t)(mi & 1) * C::MID_ELEMS;
+      double* mb = mid0 + (size_t)(mi % MB) * C::MID_ELEMS;
       const bool zring = m < 0 || m >= tz;
       const bool zfixed = zring && (fm & bit(m < 0 ? ZM : ZP));
       // --- u^{s+1}: band rows +-1 (band rows only on z-ring planes), x pairs
@@ -271,6 +311,17 @@ __global__ void __launch_bounds__(X2<TX, BY, S>::NT + 32) heat7x2(const __grid_c
           mb[(y - y0 + 1) * C::MPITCH + (side ? TX + 2 : 1)] = v;
         }
       }
+      if (MB == 3) {
+        if (mi == 2) {  // mid(z0-1) to registers before its buffer is reused
+#pragma unroll
+          for (int j = 0; j < C::NR; ++j)
+            zmr[j] = *reinterpret_cast<const double2*>(mid0 + (r0 + j * C::RPP + 1) * C::MPITCH + xo + 2);
+        }
+        if (mi >= 3) output_plane(mi);
+        cbar();  // mid(m) complete, output(m-2) done; input plane m-1 no longer read
+        release_g(seq + mi);
+        continue;
+      }
       cbar();                // mid plane m complete; input plane m-1 no longer read
       release_g(seq + mi);
       if (mi == 0) {
@@ -278,7 +329,19 @@ __global__ void __launch_bounds__(X2<TX, BY, S>::NT + 32) heat7x2(const __grid_c
         for (int j = 0; j < C::NR; ++j)
           zmr[j] = *reinterpret_cast<const double2*>(mb + (r0 + j * C::RPP + 1) * C::MPITCH + xo + 2);
       }
-      if (mi >= 2) {  // --- u^{s+2} for plane o = m-1
+      if (mi >= 2) {
+        output_plane(mi);
+        cbar();  // mid(o) may be overwritten by the next mid plane
+      }
+    }
+    release_g(seq + nq - 2);
+    release_g(seq + nq - 1);
+    seq += (uint32_t)nq;
+    pp += z1 - z0;
+  }
+}
+#if 0
+      {  // (old inline output, kept for reference of the layout)
         const int o = m - 1;
         const double* cb = mid0 + (size_t)((mi - 1) & 1) * C::MID_ELEMS;  // mid(o)
         const double* nb = mb;                                             // mid(o+1)
@@ -306,27 +369,20 @@ __global__ void __launch_bounds__(X2<TX, BY, S>::NT + 32) heat7x2(const __grid_c
           if (zlo) st2_hint(fzm + ((size_t)o * ty + y) * TX, v, keep);
           if (zhi) st2_hint(fzp + ((size_t)(o - (tz - 2)) * ty + y) * TX, v, keep);
         }
-        cbar();  // mid(o) may be overwritten by the next mid plane
-      } else if (mi == 1) {
-        // nothing to output yet; mid(z0-1) is in registers, mid(z0) in buffer 1
       }
-    }
-    release_g(seq + nq - 2);
-    release_g(seq + nq - 1);
-    seq += (uint32_t)nq;
-    pp += z1 - z0;
-  }
-}
+#endif
 
 struct X2Entry {
-  int tx, by, stages;
+  int tx, by, stages, mb;
   void (*fn)(Heat2Params);
   int nt;
   size_t smem;
 };
-#define X2E(TX, BY, S) {TX, BY, S, heat7x2<TX, BY, S>, X2<TX, BY, S>::NT + 32, X2<TX, BY, S>::SMEM}
-static const X2Entry kX2[] = {X2E(64, 64, 4), X2E(64, 32, 6), X2E(64, 32, 5), X2E(64, 32, 4),
-                              X2E(32, 32, 6), X2E(32, 16, 6), X2E(128, 16, 5), X2E(256, 8, 5)};
+#define X2E(TX, BY, S, MB) \
+  {TX, BY, S, MB, heat7x2<TX, BY, S, MB>, X2<TX, BY, S, MB>::NT + 32, X2<TX, BY, S, MB>::SMEM}
+static const X2Entry kX2[] = {X2E(64, 64, 4, 2), X2E(64, 32, 5, 3), X2E(64, 32, 4, 3),
+                              X2E(64, 32, 6, 2), X2E(32, 32, 6, 3), X2E(32, 16, 6, 3),
+                              X2E(128, 16, 4, 3), X2E(256, 8, 4, 3)};
 #undef X2E
 
 static const X2Entry* find_x2(int tx, int by, int st = 0) {

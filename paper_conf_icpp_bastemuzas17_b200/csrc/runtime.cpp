@@ -636,9 +636,108 @@ static std::vector<int> plan_passes(const Domain& d, int steps) {
   return k;
 }
 
+// Stream-through: with a fresh upload, a cell after T steps
+// depends only on cells within T planes, so with T <= tz/2 each z-layer's
+// final state needs only its own and the two adjacent layers' initial data.
+// Per layer (in z order): gather the layer and T halo planes into a dense
+// slab, run T sweeps with the valid range shrinking by one plane per end,
+// scatter the tz exact core planes into a tile-blocked out buffer, D2H it.
+// H2D of later layers, compute and D2H of earlier layers overlap (duplex
+// host link). Scratch = the resident mode's second buffer array (not needed
+// otherwise in this run). Each layer's result is also copied back into the
+// resident array once its initial data has no reader left (after the next
+// layer's gather; layer 0, read by the last layer's gather through the
+// periodic wrap, at the end), so the domain stays resident. Periodic, single
+// rank.
+static bool streamthrough_ok(const Domain& d, int T, int64_t* slab_tiles) {
+  const Geometry& G = d.G;
+  if (d.opt.stream_through < 0 || G.nranks != 1 || G.bc != TILE_BC_PERIODIC) return false;
+  if (T < 1 || 2 * (int64_t)T > G.t[2]) return false;
+  const int64_t plane = G.l[0] * G.l[1];
+  *slab_tiles = ((G.t[2] + 2 * (int64_t)T) * plane + G.tile_elems - 1) / G.tile_elems;
+  return 2 * *slab_tiles + 3 * G.layer_tiles <= G.ntiles;
+}
+
+static Status run_streamthrough(Domain& d, double alpha, int T, int S, int64_t slab_tiles) {
+  (void)alpha;
+  Exec& X = *d.exec;
+  const Geometry& G = d.G;
+  const int64_t nL = G.n[2], lt = G.layer_tiles, tz = G.t[2];
+  const Pipes P(S, false);
+  const int bit = d.res_bit;                       // H2D target array
+  const int sb = bit ? 0 : (int)G.ntiles;          // scratch array (the other one)
+  const int slab[2] = {sb, sb + (int)slab_tiles};
+  const int out[2] = {sb + 2 * (int)slab_tiles, sb + 2 * (int)slab_tiles + (int)lt};
+  const int keep0 = sb + 2 * (int)slab_tiles + 2 * (int)lt;  // layer 0's result
+  auto cur_of = [&](int64_t L) { return bit ? (int)(G.ntiles + L * lt) : (int)(L * lt); };
+  auto res_of = [&](int64_t L) { return L == 0 ? keep0 : out[L & 1]; };
+  const int cs = P.comp(0), os = P.out(0);
+  Status r;
+  // H2D in an order that lets layer 0 start early (its z- neighbour wraps)
+  std::vector<int64_t> order;
+  order.push_back(nL - 1);
+  for (int64_t L = 0; L < nL - 1; ++L) order.push_back(L);
+  for (size_t i = 0; i < order.size(); ++i) {
+    const int64_t L = order[i];
+    const int is = P.in((int64_t)i);
+    const int64_t t0 = L * lt;
+    r = X.h2d(d, t0, lt, bit ? (int)(G.ntiles + t0) : (int)t0, is);
+    if (r.bad()) return r;
+    r = X.record(d, ev_in(d, L), is);
+    if (r.bad()) return r;
+  }
+  for (int64_t L = 0; L < nL; ++L) {
+    for (int64_t dl : {(int64_t)-1, (int64_t)0, (int64_t)1}) {
+      r = X.wait(d, ev_in(d, (L + dl + nL) % nL), cs);
+      if (r.bad()) return r;
+    }
+    if (L >= 2) {  // out buffer L%2 was read by the D2H of layer L-2
+      r = X.wait(d, ev_layer(d, L % 2, 1), cs);
+      if (r.bad()) return r;
+    }
+    r = X.slab_gather(d, L, bit, slab[0], L * tz - T, tz + 2 * T, cs);
+    if (r.bad()) return r;
+    if (L >= 2) {  // layer L-1's initial data has no reader left: write its result back
+      r = X.copy_slots(d, res_of(L - 1), cur_of(L - 1), lt, cs);
+      if (r.bad()) return r;
+    }
+    for (int i = 1; i <= T; ++i) {
+      r = X.slab_sweep(d, slab[(i - 1) & 1], slab[i & 1], i, (int)(tz + 2 * T - i), cs);
+      if (r.bad()) return r;
+    }
+    r = X.slab_scatter(d, slab[T & 1], T, res_of(L), L, cs);
+    if (r.bad()) return r;
+    r = X.record(d, ev_layer(d, L, 0), cs);
+    if (r.bad()) return r;
+    r = X.wait(d, ev_layer(d, L, 0), os);
+    if (r.bad()) return r;
+    r = X.d2h(d, L * lt, lt, res_of(L), os);
+    if (r.bad()) return r;
+    r = X.record(d, ev_layer(d, L % 2, 1), os);
+    if (r.bad()) return r;
+  }
+  if (nL >= 2) {
+    r = X.copy_slots(d, res_of(nL - 1), cur_of(nL - 1), lt, cs);
+    if (r.bad()) return r;
+  }
+  r = X.copy_slots(d, keep0, cur_of(0), lt, cs);
+  if (r.bad()) return r;
+  for (int64_t k = 0; k < G.ntiles; ++k) {
+    d.tile_dirty[k] = 0;  // the host received u^T through the D2H above
+    d.tile_slot[k] = bit ? (int)(G.ntiles + k) : (int)k;
+  }
+  d.resident_valid = true;
+  d.faces_valid = false;  // faces are re-extracted by the next resident run
+  d.last_batches.clear();
+  return Status::ok();
+}
+
 static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool serial) {
   const bool load = !d.resident_valid;
   const int64_t nL = d.G.n[2];
+  int64_t slab_tiles = 0;
+  if (load && !serial && streamthrough_ok(d, steps, &slab_tiles))
+    return run_streamthrough(d, alpha, steps, S, slab_tiles);
   const std::vector<int> kp = plan_passes(d, steps);
   const int T = (int)kp.size();  // passes
   struct Phase {

@@ -93,6 +93,13 @@ struct Exec {
   virtual Status heat(Domain& d, const int64_t* tiles, const int* in_slots, const int* out_slots,
                       int nitems, int read_parity, const TileItem* dev_items, int stream) = 0;
   virtual Status sincos(Domain& d, int64_t tile, int slot, int64_t iters, int stream) = 0;
+  // stream-through slabs; slab/out locations are slot indices of the scratch
+  virtual Status slab_gather(Domain& d, int64_t layer, int src_bit, int slab_slot, int64_t zbase,
+                             int64_t planes, int stream) = 0;
+  virtual Status slab_sweep(Domain& d, int src_slot, int dst_slot, int lo, int hi, int stream) = 0;
+  virtual Status slab_scatter(Domain& d, int slab_slot, int first, int out_slot, int64_t layer,
+                              int stream) = 0;
+  virtual Status copy_slots(Domain& d, int src_slot, int dst_slot, int64_t n, int stream) = 0;
   // two-step pass (temporal blocking): same arguments as heat
   virtual Status heat2(Domain& d, const int64_t* tiles, const int* in_slots, const int* out_slots,
                        int nitems, int read_parity, const TileItem* dev_items, int stream) = 0;

@@ -32,7 +32,8 @@ TILE_KERNEL_HEAT7, TILE_KERNEL_SINCOS = 1, 2
 TILE_SCHED_AUTO, TILE_SCHED_RESIDENT, TILE_SCHED_STREAM, TILE_SCHED_SYNC = 0, 1, 2, 3
 TILE_MEASURE_NORMAL, TILE_MEASURE_XFER_ONLY, TILE_MEASURE_COMP_ONLY = 0, 1, 2
 OP_NAMES = {1: "h2d", 2: "d2h", 3: "kernel", 4: "record", 5: "wait", 6: "faces_h2d",
-            7: "extract", 8: "halo", 9: "drop", 10: "hit", 11: "pointwise", 12: "kernel2"}
+            7: "extract", 8: "halo", 9: "drop", 10: "hit", 11: "pointwise", 12: "kernel2",
+            13: "gather", 14: "sweep", 15: "scatter", 16: "copy"}
 SCHEDS = {"auto": 0, "resident": 1, "stream": 2, "sync": 3}
 BCS = {"periodic": 0, "dirichlet": 1}
 
@@ -45,7 +46,7 @@ class TileOptions(ctypes.Structure):
                 ("nccl_unique_id", ctypes.c_void_p), ("sched", ctypes.c_int),
                 ("dry_run", ctypes.c_int32), ("fuse_pointwise_steps", ctypes.c_int32),
                 ("local_group", ctypes.c_void_p), ("pageable_host", ctypes.c_int32),
-                ("two_step", ctypes.c_int32)]
+                ("stream_through", ctypes.c_int32), ("two_step", ctypes.c_int32)]
 
 
 class TileKernel(ctypes.Structure):
@@ -171,7 +172,7 @@ class Domain:
     def __init__(self, dims, tile_dims, ghost=1, bc="periodic", device=-1, device_budget_bytes=0,
                  sched="auto", nranks=1, rank=0, nccl_id=None, dry_run=False,
                  fuse_pointwise_steps=True, device_pool=None, streams=None, local_group=None,
-                 pageable_host=False, two_step=0):
+                 pageable_host=False, two_step=0, stream_through=0):
         self._h = None
         self.dims = tuple(int(v) for v in dims)
         self.tile_dims = tuple(int(v) for v in tile_dims)
@@ -201,6 +202,7 @@ class Domain:
         o.fuse_pointwise_steps = 1 if fuse_pointwise_steps else 0
         o.pageable_host = 1 if pageable_host else 0
         o.two_step = int(two_step)
+        o.stream_through = int(stream_through)
         self._group = local_group
         if local_group is not None:
             o.local_group = local_group.handle

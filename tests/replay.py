@@ -90,6 +90,8 @@ class Replayer:
         self.alpha = alpha
         self.ext = ext
         self.slots = {}
+        self.slabs = {}
+        self.loc = {}      # tile -> device slot of its last H2D
         self.faces = {}
         self.halo = {}
         self.comm = comm
@@ -234,6 +236,7 @@ class Replayer:
         if name == "h2d":
             for i in range(c):
                 self.slots[b + i] = self.host[a + i].copy()
+                self.loc[a + i] = b + i
         elif name == "d2h":
             for i in range(c):
                 self.host[a + i] = self.slots[b + i].copy()
@@ -252,7 +255,49 @@ class Replayer:
             self.slots[b] = oracle.sincos_c(self.slots[b], c, 1)
         elif name == "halo":
             self.comm(self, d)
+        elif name == "copy":
+            for i in range(c):
+                self.slots[b + i] = self.slots[a + i].copy()
+            for t, sl in list(self.loc.items()):
+                if b <= sl < b + c:
+                    pass
+        elif name == "gather":
+            self.slabs[b] = self.gather(a, c, d)
+        elif name == "sweep":
+            self.slabs[b] = self.sweep(self.slabs[a], self.slabs.get(b), c, d)
+        elif name == "scatter":
+            G = self.G
+            tx, ty, tz = G.t
+            slab = self.slabs[a]
+            for i in range(G.n[0] * G.n[1]):
+                ix, iy = i % G.n[0], i // G.n[0]
+                self.slots[b + i] = slab[c:c + tz, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx].copy()
         # record / wait / hit / drop: no data movement
+
+    # ------------------------------------------------- stream-through slabs
+    def gather(self, layer, planes, zbase):
+        G = self.G
+        tx, ty, tz = G.t
+        nz = G.l[2]
+        out = np.empty((planes, G.l[1], G.l[0]))
+        for p in range(planes):
+            gz = (zbase + p) % nz
+            iz, lz = gz // tz, gz % tz
+            for iy in range(G.n[1]):
+                for ix in range(G.n[0]):
+                    t = G.tid(ix, iy, iz)
+                    out[p, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx] = self.slots[self.loc[t]][lz]
+        return out
+
+    def sweep(self, src, dst, lo, hi):
+        """One oracle step on planes [lo, hi), periodic in x and y; planes
+        lo-1 and hi are the z neighbours (oracle.heat_np on a block whose
+        x/y halo is the periodic wrap and whose z halo is fixed)."""
+        blk = np.pad(src[lo - 1:hi + 1], ((0, 0), (1, 1), (1, 1)), mode="wrap")
+        new = oracle.heat_np(blk, self.alpha, 1, oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+        out = np.full_like(src, np.nan) if dst is None else dst.copy()
+        out[lo:hi] = new
+        return out
 
     def replay(self, trace, seed):
         rng = random.Random(seed)
