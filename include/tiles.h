@@ -175,7 +175,11 @@ typedef enum {
   TILE_OP_GATHER = 13,   /* layer a + halo -> dense slab at slot b: c planes from z = d */
   TILE_OP_SWEEP = 14,    /* slab slot a -> slab slot b, planes [c, d) */
   TILE_OP_SCATTER = 15,  /* slab slot a core planes from c -> tile-blocked slots from b (layer d) */
-  TILE_OP_COPY = 16      /* device copy of c tile slots: slot a -> slot b */
+  TILE_OP_COPY = 16,     /* device copy of c tile slots: slot a -> slot b */
+  /* partial (sub-layer) copies of planes [d & 0xffffffff, + d >> 32) of c tiles: */
+  TILE_OP_H2D_PART = 17, /* host tiles a.. -> slots b.. */
+  TILE_OP_D2H_PART = 18, /* packed sub-tiles at slot b -> host tiles a.. */
+  TILE_OP_COPY_PART = 19 /* packed sub-tiles at slot a -> slots b.. */
 } tile_op_kind;
 
 typedef struct {

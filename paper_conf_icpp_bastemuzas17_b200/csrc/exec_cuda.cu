@@ -204,11 +204,39 @@ struct CudaExec final : Exec {
   Status slab_scatter(Domain& d, int slab, int first, int out, int64_t, int st) override {
     if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
     SlabParams p = slab_base(d);
+    p.tz = d.st_unit;  // planes per unit; packed sub-tiles of tz*ty*tx elements
+    p.tile_elems = d.st_unit * d.G.t[0] * d.G.t[1];
     p.slab = d.slot_ptr(slab);
     p.out = d.slot_ptr(out);
     Status r = timed(d, st, [&] { return launch_slab_scatter(p, first, sms, S(st)); });
     if (r.bad()) return r;
     d.stats.n_kernels++;
+    return Status::ok();
+  }
+  Status h2d_part(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int st) override {
+    if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
+    const size_t pl = (size_t)d.G.t[0] * d.G.t[1] * 8, tb = (size_t)d.G.tile_elems * 8;
+    CK(cudaMemcpy2DAsync(reinterpret_cast<char*>(d.slot_ptr(s0)) + p0 * pl, tb,
+                         reinterpret_cast<const char*>(d.host_tile(t0)) + p0 * pl, tb, np * pl,
+                         (size_t)n, cudaMemcpyHostToDevice, S(st)));
+    d.stats.bytes_h2d += (uint64_t)n * np * pl;
+    d.stats.n_h2d++;
+    return Status::ok();
+  }
+  Status d2h_part(Domain& d, int64_t t0, int64_t n, int ps, int64_t p0, int64_t np, int st) override {
+    if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
+    const size_t pl = (size_t)d.G.t[0] * d.G.t[1] * 8, tb = (size_t)d.G.tile_elems * 8;
+    CK(cudaMemcpy2DAsync(reinterpret_cast<char*>(d.host_tile(t0)) + p0 * pl, tb, d.slot_ptr(ps),
+                         np * pl, np * pl, (size_t)n, cudaMemcpyDeviceToHost, S(st)));
+    d.stats.bytes_d2h += (uint64_t)n * np * pl;
+    d.stats.n_d2h++;
+    return Status::ok();
+  }
+  Status copy_part(Domain& d, int ps, int s0, int64_t n, int64_t p0, int64_t np, int st) override {
+    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
+    const size_t pl = (size_t)d.G.t[0] * d.G.t[1] * 8, tb = (size_t)d.G.tile_elems * 8;
+    CK(cudaMemcpy2DAsync(reinterpret_cast<char*>(d.slot_ptr(s0)) + p0 * pl, tb, d.slot_ptr(ps),
+                         np * pl, np * pl, (size_t)n, cudaMemcpyDeviceToDevice, S(st)));
     return Status::ok();
   }
   Status copy_slots(Domain& d, int src, int dst, int64_t n, int st) override {

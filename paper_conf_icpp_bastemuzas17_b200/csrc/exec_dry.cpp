@@ -80,6 +80,22 @@ struct DryExec final : Exec {
     put(d, TILE_OP_SCATTER, st, slab, out, first, layer);
     return Status::ok();
   }
+  Status h2d_part(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int st) override {
+    d.stats.bytes_h2d += (uint64_t)n * np * d.G.t[0] * d.G.t[1] * 8;
+    d.stats.n_h2d++;
+    put(d, TILE_OP_H2D_PART, st, t0, s0, n, p0 | (np << 32));
+    return Status::ok();
+  }
+  Status d2h_part(Domain& d, int64_t t0, int64_t n, int ps, int64_t p0, int64_t np, int st) override {
+    d.stats.bytes_d2h += (uint64_t)n * np * d.G.t[0] * d.G.t[1] * 8;
+    d.stats.n_d2h++;
+    put(d, TILE_OP_D2H_PART, st, t0, ps, n, p0 | (np << 32));
+    return Status::ok();
+  }
+  Status copy_part(Domain& d, int ps, int s0, int64_t n, int64_t p0, int64_t np, int st) override {
+    put(d, TILE_OP_COPY_PART, st, ps, s0, n, p0 | (np << 32));
+    return Status::ok();
+  }
   Status copy_slots(Domain& d, int src, int dst, int64_t n, int st) override {
     put(d, TILE_OP_COPY, st, src, dst, n, 0);
     return Status::ok();

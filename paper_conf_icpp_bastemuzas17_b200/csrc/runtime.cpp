@@ -269,7 +269,7 @@ Status domain_setup(Domain& d) {
   d.ev_in_base = d.ev_slot_base + d.nslots;
   d.ev_host_base = d.ev_in_base + (int)G.ntiles;
   d.ev_misc_base = d.ev_host_base + (int)G.ntiles;
-  d.nevents = d.ev_misc_base + 4 + d.halo_stream + 1;
+  d.nevents = d.ev_misc_base + 4 + d.halo_stream + 1 + 2;  // + 2 stream-through ring events
   st = X.setup(d);
   if (st.bad()) return st;
   if (multi && !d.opt.dry_run && !d.opt.local_group) {
@@ -649,78 +649,114 @@ static std::vector<int> plan_passes(const Domain& d, int steps) {
 // layer's gather; layer 0, read by the last layer's gather through the
 // periodic wrap, at the end), so the domain stays resident. Periodic, single
 // rank.
-static bool streamthrough_ok(const Domain& d, int T, int64_t* slab_tiles) {
+struct StreamPlan {
+  int64_t unit;        // planes per unit (divides tz, >= 2T)
+  int64_t units;       // local nz / unit
+  int64_t slab_tiles;  // one dense slab of unit + 2T planes, in tile slots
+  int64_t sub_tiles;   // one packed unit result (layer_tiles sub-tiles), in tile slots
+};
+
+static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
   const Geometry& G = d.G;
   if (d.opt.stream_through < 0 || G.nranks != 1 || G.bc != TILE_BC_PERIODIC) return false;
   if (T < 1 || 2 * (int64_t)T > G.t[2]) return false;
   const int64_t plane = G.l[0] * G.l[1];
-  *slab_tiles = ((G.t[2] + 2 * (int64_t)T) * plane + G.tile_elems - 1) / G.tile_elems;
-  return 2 * *slab_tiles + 3 * G.layer_tiles <= G.ntiles;
+  // thinnest unit >= max(2T, 16) planes dividing tz (thin units shorten the
+  // pipeline's fill and drain; a unit needs only its two neighbour units)
+  int64_t unit = G.t[2];
+  for (int64_t u = 1; u <= G.t[2]; ++u)
+    if (G.t[2] % u == 0 && u >= 2 * (int64_t)T && u >= std::min<int64_t>(16, G.t[2])) {
+      unit = u;
+      break;
+    }
+  const int64_t units = G.l[2] / unit;
+  if (units > G.ntiles) unit = G.t[2];  // event budget (one per unit)
+  sp->unit = unit;
+  sp->units = G.l[2] / unit;
+  sp->slab_tiles = ((unit + 2 * (int64_t)T) * plane + G.tile_elems - 1) / G.tile_elems;
+  sp->sub_tiles = (G.layer_tiles * unit * G.t[0] * G.t[1] + G.tile_elems - 1) / G.tile_elems;
+  return 2 * sp->slab_tiles + 3 * sp->sub_tiles <= G.ntiles;
 }
 
-static Status run_streamthrough(Domain& d, double alpha, int T, int S, int64_t slab_tiles) {
+// Stream-through over units of `unit` planes (a unit is a slice of one tile
+// layer: planes [p0, p0+unit) of each of its tiles, contiguous per tile, so
+// its H2D/D2H are single strided 2-D copies). Per unit u, in z order:
+// gather u and T halo planes into a dense slab, T sweeps with the valid range
+// shrinking by one plane per end, scatter the exact core into packed
+// sub-tiles, D2H them. Unit u's result is written back into the resident
+// array after unit u+1's gather (unit 0, read by the last unit through the
+// periodic wrap, at the end).
+static Status run_streamthrough(Domain& d, double alpha, int T, int S, const StreamPlan& sp) {
   (void)alpha;
   Exec& X = *d.exec;
   const Geometry& G = d.G;
-  const int64_t nL = G.n[2], lt = G.layer_tiles, tz = G.t[2];
+  const int64_t U = sp.units, lt = G.layer_tiles, tz = G.t[2], un = sp.unit;
   const Pipes P(S, false);
   const int bit = d.res_bit;                       // H2D target array
   const int sb = bit ? 0 : (int)G.ntiles;          // scratch array (the other one)
-  const int slab[2] = {sb, sb + (int)slab_tiles};
-  const int out[2] = {sb + 2 * (int)slab_tiles, sb + 2 * (int)slab_tiles + (int)lt};
-  const int keep0 = sb + 2 * (int)slab_tiles + 2 * (int)lt;  // layer 0's result
-  auto cur_of = [&](int64_t L) { return bit ? (int)(G.ntiles + L * lt) : (int)(L * lt); };
-  auto res_of = [&](int64_t L) { return L == 0 ? keep0 : out[L & 1]; };
-  const int cs = P.comp(0), os = P.out(0);
+  const int slab[2] = {sb, sb + (int)sp.slab_tiles};
+  const int out[2] = {sb + 2 * (int)sp.slab_tiles, sb + 2 * (int)sp.slab_tiles + (int)sp.sub_tiles};
+  const int keep0 = sb + 2 * (int)sp.slab_tiles + 2 * (int)sp.sub_tiles;
+  auto layer_of = [&](int64_t u) { return (u * un) / tz; };
+  auto p0_of = [&](int64_t u) { return (u * un) % tz; };
+  auto cur_slot = [&](int64_t u) {
+    const int64_t t0 = layer_of(u) * lt;
+    return bit ? (int)(G.ntiles + t0) : (int)t0;
+  };
+  auto res_of = [&](int64_t u) { return u == 0 ? keep0 : out[u & 1]; };
+  auto ev_unit_done = [&](int64_t u) { return ev_host(d, u); };  // compute of unit u
+  const int ring_ev[2] = {d.ev_misc_base + 4 + d.halo_stream + 1, d.ev_misc_base + 5 + d.halo_stream + 1};
+  const int cs = P.comp(0), os = P.out(0), is = P.in(0);
+  d.st_unit = un;
   Status r;
-  // H2D in an order that lets layer 0 start early (its z- neighbour wraps)
+  // one copy-in stream, so the copy engine runs the H2Ds in this order (it
+  // may not across streams): the last unit first (unit 0's wrap neighbour)
   std::vector<int64_t> order;
-  order.push_back(nL - 1);
-  for (int64_t L = 0; L < nL - 1; ++L) order.push_back(L);
-  for (size_t i = 0; i < order.size(); ++i) {
-    const int64_t L = order[i];
-    const int is = P.in((int64_t)i);
-    const int64_t t0 = L * lt;
-    r = X.h2d(d, t0, lt, bit ? (int)(G.ntiles + t0) : (int)t0, is);
+  order.push_back(U - 1);
+  for (int64_t u = 0; u < U - 1; ++u) order.push_back(u);
+  for (int64_t u : order) {
+    r = X.h2d_part(d, layer_of(u) * lt, lt, cur_slot(u), p0_of(u), un, is);
     if (r.bad()) return r;
-    r = X.record(d, ev_in(d, L), is);
+    r = X.record(d, ev_in(d, u), is);
     if (r.bad()) return r;
   }
-  for (int64_t L = 0; L < nL; ++L) {
-    for (int64_t dl : {(int64_t)-1, (int64_t)0, (int64_t)1}) {
-      r = X.wait(d, ev_in(d, (L + dl + nL) % nL), cs);
+  for (int64_t u = 0; u < U; ++u) {
+    for (int64_t du : {(int64_t)-1, (int64_t)0, (int64_t)1}) {
+      r = X.wait(d, ev_in(d, (u + du + U) % U), cs);
       if (r.bad()) return r;
     }
-    if (L >= 2) {  // out buffer L%2 was read by the D2H of layer L-2
-      r = X.wait(d, ev_layer(d, L % 2, 1), cs);
+    if (u >= 2) {  // the ring buffer u%2 was last read by unit u-2's D2H
+      r = X.wait(d, ring_ev[u & 1], cs);
       if (r.bad()) return r;
     }
-    r = X.slab_gather(d, L, bit, slab[0], L * tz - T, tz + 2 * T, cs);
+    r = X.slab_gather(d, u, bit, slab[0], u * un - T, un + 2 * T, cs);
     if (r.bad()) return r;
-    if (L >= 2) {  // layer L-1's initial data has no reader left: write its result back
-      r = X.copy_slots(d, res_of(L - 1), cur_of(L - 1), lt, cs);
+    if (u >= 2) {  // unit u-1's initial data has no reader left
+      r = X.copy_part(d, res_of(u - 1), cur_slot(u - 1), lt, p0_of(u - 1), un, cs);
       if (r.bad()) return r;
     }
     for (int i = 1; i <= T; ++i) {
-      r = X.slab_sweep(d, slab[(i - 1) & 1], slab[i & 1], i, (int)(tz + 2 * T - i), cs);
+      r = X.slab_sweep(d, slab[(i - 1) & 1], slab[i & 1], i, (int)(un + 2 * T - i), cs);
       if (r.bad()) return r;
     }
-    r = X.slab_scatter(d, slab[T & 1], T, res_of(L), L, cs);
+    r = X.slab_scatter(d, slab[T & 1], T, res_of(u), u, cs);
     if (r.bad()) return r;
-    r = X.record(d, ev_layer(d, L, 0), cs);
+    r = X.record(d, ev_unit_done(u), cs);
     if (r.bad()) return r;
-    r = X.wait(d, ev_layer(d, L, 0), os);
+    r = X.wait(d, ev_unit_done(u), os);
     if (r.bad()) return r;
-    r = X.d2h(d, L * lt, lt, res_of(L), os);
+    r = X.d2h_part(d, layer_of(u) * lt, lt, res_of(u), p0_of(u), un, os);
     if (r.bad()) return r;
-    r = X.record(d, ev_layer(d, L % 2, 1), os);
+    if (u >= 1) {
+      r = X.record(d, ring_ev[u & 1], os);
+      if (r.bad()) return r;
+    }
+  }
+  if (U >= 2) {
+    r = X.copy_part(d, res_of(U - 1), cur_slot(U - 1), lt, p0_of(U - 1), un, cs);
     if (r.bad()) return r;
   }
-  if (nL >= 2) {
-    r = X.copy_slots(d, res_of(nL - 1), cur_of(nL - 1), lt, cs);
-    if (r.bad()) return r;
-  }
-  r = X.copy_slots(d, keep0, cur_of(0), lt, cs);
+  r = X.copy_part(d, keep0, cur_slot(0), lt, p0_of(0), un, cs);
   if (r.bad()) return r;
   for (int64_t k = 0; k < G.ntiles; ++k) {
     d.tile_dirty[k] = 0;  // the host received u^T through the D2H above
@@ -735,9 +771,8 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, int64_t s
 static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool serial) {
   const bool load = !d.resident_valid;
   const int64_t nL = d.G.n[2];
-  int64_t slab_tiles = 0;
-  if (load && !serial && streamthrough_ok(d, steps, &slab_tiles))
-    return run_streamthrough(d, alpha, steps, S, slab_tiles);
+  StreamPlan sp{};
+  if (load && !serial && streamthrough_ok(d, steps, &sp)) return run_streamthrough(d, alpha, steps, S, sp);
   const std::vector<int> kp = plan_passes(d, steps);
   const int T = (int)kp.size();  // passes
   struct Phase {

@@ -100,6 +100,14 @@ struct Exec {
   virtual Status slab_scatter(Domain& d, int slab_slot, int first, int out_slot, int64_t layer,
                               int stream) = 0;
   virtual Status copy_slots(Domain& d, int src_slot, int dst_slot, int64_t n, int stream) = 0;
+  // planes [p0, p0+np) of n tiles; "packed" = n sub-tiles of np*ty*tx
+  // elements back to back starting at a slot
+  virtual Status h2d_part(Domain& d, int64_t tile0, int64_t n, int slot0, int64_t p0, int64_t np,
+                          int stream) = 0;
+  virtual Status d2h_part(Domain& d, int64_t tile0, int64_t n, int packed_slot, int64_t p0,
+                          int64_t np, int stream) = 0;
+  virtual Status copy_part(Domain& d, int packed_slot, int slot0, int64_t n, int64_t p0, int64_t np,
+                           int stream) = 0;
   // two-step pass (temporal blocking): same arguments as heat
   virtual Status heat2(Domain& d, const int64_t* tiles, const int* in_slots, const int* out_slots,
                        int nitems, int read_parity, const TileItem* dev_items, int stream) = 0;
@@ -153,6 +161,7 @@ struct Domain {
   std::vector<EdgePtr> esrc_host[2];
   uint8_t* fixed_mask_dev = nullptr;       // per tile: Dirichlet faces (bit f)
   std::vector<uint8_t> fixed_mask_host;
+  int64_t st_unit = 0;                     // stream-through unit (planes) of the current run
   bool x2_ok = false;                      // two-step passes available
   int band2 = 0, heat2_grid = 0;
   size_t heat2_smem = 0;

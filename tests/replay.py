@@ -91,6 +91,7 @@ class Replayer:
         self.ext = ext
         self.slots = {}
         self.slabs = {}
+        self.sub = {}      # packed unit results: (base slot, tile-in-layer) -> (np, ty, tx)
         self.loc = {}      # tile -> device slot of its last H2D
         self.faces = {}
         self.halo = {}
@@ -269,9 +270,24 @@ class Replayer:
             G = self.G
             tx, ty, tz = G.t
             slab = self.slabs[a]
+            unit = slab.shape[0] - 2 * c
             for i in range(G.n[0] * G.n[1]):
                 ix, iy = i % G.n[0], i // G.n[0]
-                self.slots[b + i] = slab[c:c + tz, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx].copy()
+                self.sub[(b, i)] = slab[c:c + unit, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx].copy()
+        elif name in ("h2d_part", "d2h_part", "copy_part"):
+            p0, np_ = d & 0xffffffff, d >> 32
+            for i in range(c):
+                if name == "h2d_part":
+                    if b + i not in self.slots:
+                        self.slots[b + i] = np.full(self.host[a + i].shape, np.nan)
+                    self.slots[b + i][p0:p0 + np_] = self.host[a + i][p0:p0 + np_]
+                    self.loc[a + i] = b + i
+                elif name == "d2h_part":
+                    self.host[a + i] = self.host[a + i].copy()
+                    self.host[a + i][p0:p0 + np_] = self.sub[(b, i)]
+                else:
+                    self.slots[b + i] = self.slots[b + i].copy()
+                    self.slots[b + i][p0:p0 + np_] = self.sub[(a, i)]
         # record / wait / hit / drop: no data movement
 
     # ------------------------------------------------- stream-through slabs

@@ -15,6 +15,7 @@ import synth
 pytestmark = pytest.mark.gpu
 
 T = pytest.importorskip("paper_conf_icpp_bastemuzas17_b200.tiles")
+T_ = T
 ALPHA = 0.125
 
 
@@ -307,3 +308,23 @@ def test_two_step_passes_bit_exact(bc, dims, td, runs):
     out, ref, info, _ = _heat(dims, td, sum(runs), bc=bc, ghost=2, runs=runs, sched="stream",
                               device_budget_bytes=b * 2)
     assert np.array_equal(out, ref) and info["steps_per_pass"] == 2
+
+
+@pytest.mark.parametrize("dims,td,T", [((128, 64, 256), (64, 32, 32), 5), ((64, 64, 192), (32, 32, 64), 10),
+                                       ((64, 64, 256), (64, 64, 32), 1)])
+def test_stream_through_bit_exact(dims, td, T):
+    """Fresh-upload runs with T <= tz/2 take the stream-through schedule
+    (units of planes, gather + T sweeps + scatter, D2H, write-back); the host
+    result and the kept device copy (a following resident run) are exact."""
+    nx, ny, nz = dims
+    u0 = synth.uniform_grid(nx, ny, nz, 42)
+    with T_.Domain(dims, td) as d:
+        d.load(u0)
+        d.run(T_.heat7(), T, 2)
+        out1 = d.store()
+        st = d.stats()
+        d.run(T_.heat7(), 3, 2)   # continues from the device copy
+        out2 = d.store()
+    assert np.array_equal(out1, oracle.heat_c(u0, ALPHA, T))
+    assert np.array_equal(out2, oracle.heat_c(u0, ALPHA, T + 3))
+    assert st["bytes_h2d"] == nx * ny * nz * 8 and st["bytes_d2h"] == nx * ny * nz * 8

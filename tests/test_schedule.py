@@ -287,14 +287,15 @@ def test_two_step_passes_replay_to_oracle(bc, sched, td):
 
 
 @pytest.mark.parametrize("dims,td,T,ns", [((16, 16, 64), (8, 8, 8), 3, 2), ((16, 8, 64), (8, 4, 8), 4, 3),
-                                          ((16, 16, 64), (8, 8, 8), 2, 1), ((32, 16, 48), (16, 8, 8), 1, 4)])
+                                          ((16, 16, 64), (8, 8, 8), 2, 1), ((32, 16, 48), (16, 8, 8), 1, 4),
+                                          ((16, 16, 128), (8, 8, 32), 2, 2), ((16, 8, 192), (8, 4, 48), 7, 2)])
 def test_stream_through_schedule_replays_to_oracle(dims, td, T, ns):
     """Fresh-upload heat runs with T <= tz/2 use the stream-through schedule
     (per-layer gather + T shrinking sweeps + scatter + D2H); replayed in random
     valid orders it must give the oracle bit-exactly."""
     d = _run_and_replay(dims, td, [T], ns, seeds=(0, 1, 2))
     ops = [op[0] for op in d.trace()]
-    assert "gather" in ops and "sweep" in ops and "scatter" in ops
+    assert "gather" in ops and "sweep" in ops and "scatter" in ops and "h2d_part" in ops
     assert d.get_info()["resident"]
     # then a resident continuation and a second stream-through
     _run_and_replay(dims, td, [T, T], ns, seeds=(3,))
