@@ -19,6 +19,8 @@ LIB = os.path.join(HERE, "libtiles.so")
 CUDA = os.environ.get("CUDA_HOME", "/usr/local/cuda")
 NVCC = os.path.join(CUDA, "bin", "nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+# experiment hook (e.g. TILES_NVCC_DEFS="-DTILES_ARRIVE_PER_THREAD=1"); use --force when changing it
+EXTRA = os.environ.get("TILES_NVCC_DEFS", "").split()
 
 
 def _nccl_include():
@@ -62,7 +64,7 @@ def build(force=False, verbose=False):
         changed = True
         if src.endswith(".cu"):
             cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
-                   "-Xptxas", "-v", *inc, "-c", src, "-o", obj]
+                   "-Xptxas", "-v", *EXTRA, *inc, "-c", src, "-o", obj]
         else:
             cmd = ["g++", "-O2", "-std=c++17", "-fPIC", "-Wall", "-Wno-unused-function", *inc,
                    "-c", src, "-o", obj]

@@ -106,7 +106,7 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&empty[s], NCW);
+      mbar_init(&empty[s], TILES_ARRIVE_PER_THREAD ? NCW * 32 : NCW);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -153,8 +153,12 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
   const int xpj = xhi_edge ? C::RPP * D * 8 : C::RPP * TX * 8;
   auto wait_g = [&](uint32_t g) { mbar_wait(&full[g % S], (g / S) & 1u); };
   auto release_g = [&](uint32_t g) {
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[g % S]);
+    if (TILES_ARRIVE_PER_THREAD) {
+      mbar_arrive(&empty[g % S]);
+    } else {
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[g % S]);
+    }
   };
   uint32_t seq = 0;
 

@@ -56,7 +56,7 @@ __device__ __forceinline__ void stage_x2(double* dst, uint64_t* bar, const doubl
   const bool inplane = z >= 0 && z < tz;
   const bool near_ghost = z == -1 || z == tz;
   // 1) edge cells (regular loads by the warp, generic proxy) — written before
-  //    lane 0's arrive, which releases them to the consumers.
+  //    the lanes' arrives on `bar`, which release them to the consumers.
   if (inplane) {
     if (lane < 4) {
       const int gx = lane & 1, gy = lane >> 1;
@@ -87,8 +87,15 @@ __device__ __forceinline__ void stage_x2(double* dst, uint64_t* bar, const doubl
             e.ptr[(int64_t)y * e.stride];
     }
   }
-  __syncwarp();
-  if (lane != 0) return;
+  if (TILES_ARRIVE_PER_THREAD) {  // every lane releases its own edge writes
+    if (lane != 0) {
+      mbar_arrive(bar);
+      return;
+    }
+  } else {
+    __syncwarp();
+    if (lane != 0) return;
+  }
   // 2) bulk copies (TMA)
   const uint64_t pol = policy_evict_normal();
   fence_proxy_async();
@@ -133,8 +140,8 @@ __global__ void __launch_bounds__(X2<TX, BY, S, MB>::NT + 32) heat7x2(const __gr
   constexpr int NCW = C::NT / 32;
   if (threadIdx.x == 0) {
     for (int s = 0; s < C::S; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&empty[s], NCW);
+      mbar_init(&full[s], TILES_ARRIVE_PER_THREAD ? 32 : 1);  // producer lanes (edge cells)
+      mbar_init(&empty[s], TILES_ARRIVE_PER_THREAD ? NCW * 32 : NCW);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -175,8 +182,12 @@ __global__ void __launch_bounds__(X2<TX, BY, S, MB>::NT + 32) heat7x2(const __gr
   auto cbar = [] { asm volatile("bar.sync 1, %0;" ::"n"(C::NT) : "memory"); };
   auto wait_g = [&](uint32_t g) { mbar_wait(&full[g % C::S], (g / C::S) & 1u); };
   auto release_g = [&](uint32_t g) {
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[g % C::S]);
+    if (TILES_ARRIVE_PER_THREAD) {
+      mbar_arrive(&empty[g % C::S]);
+    } else {
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[g % C::S]);
+    }
   };
   uint32_t seq = 0;
 

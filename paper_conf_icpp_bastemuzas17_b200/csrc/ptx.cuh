@@ -10,6 +10,14 @@ namespace tiles {
 static __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
+// Pipeline-stage hand-off between warps: one mbarrier arrive per thread (1,
+// default: every thread's shared-memory accesses are ordered by its own
+// release-arrive, which compute-sanitizer racecheck can follow) or one per warp
+// after __syncwarp (0: fewer arrives; racecheck reports the other lanes'
+// accesses as hazards). Throughput is the same within noise (profiles/r01).
+#ifndef TILES_ARRIVE_PER_THREAD
+#define TILES_ARRIVE_PER_THREAD 1
+#endif
 static __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
 }

@@ -1,7 +1,7 @@
 """Small runs of every schedule for compute-sanitizer (memcheck / racecheck /
 synccheck / initcheck): resident heat (layered + whole-domain phases),
 streaming heat with a tiny budget, Dirichlet, sincos, the generic kernel and
-the in-process multi-rank transport."""
+the stream-through schedule and the in-process multi-rank transport."""
 import os
 import sys
 import threading
@@ -37,6 +37,13 @@ with T.Domain((64, 32, 32), (32, 16, 16), bc="dirichlet") as d:
     d.load(ext); d.run(T.heat7(), 3, 2); d.store()
 with T.Domain((64, 32, 32), (32, 16, 16)) as d:
     d.load(u); d.run(T.sincos(2), 2, 2); d.store()
+us = synth.uniform_grid(64, 64, 256, 3)                   # stream-through (units of 16 planes)
+with T.Domain((64, 64, 256), (64, 64, 32)) as d:
+    d.load(us); d.run(T.heat7(), 2, 2); d.store(); d.run(T.heat7(), 1, 2); d.store()
+with T.Domain((64, 64, 256), (32, 32, 32)) as d:          # stream-through, unit = tile layer
+    d.load(us); d.run(T.heat7(), 10, 2); d.store()
+with T.Domain((128, 64, 64), (64, 64, 16), ghost=2, two_step=1) as d:   # heat7x2 (two steps per pass)
+    d.load(synth.uniform_grid(128, 64, 64, 9)); d.run(T.heat7(), 6, 2); d.store()
 g = T.LocalGroup(2)
 def rank(r):
     with T.Domain((64, 32, 64), (32, 16, 16), nranks=2, rank=r, local_group=g) as d:
