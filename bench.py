@@ -453,7 +453,8 @@ def run_fig5_leg(args):
     out = {}
     for sched, ns, pageable in (("auto", args.nstreams or 4, False), ("sync", 1, False),
                                 ("sync_pageable", 1, True)):
-        dom = Tl.Domain(gdims, td, ghost=1, device=0, sched=sched.split("_")[0], pageable_host=pageable)
+        dom = Tl.Domain(gdims, td, ghost=1, device=0, sched=sched.split("_")[0], pageable_host=pageable,
+                        stream_through=args.stream_through if sched == "auto" else 0)
         fill_tiles(dom, Tl, synth, gdims, td, 0, 42)
         k = Tl.heat7(ALPHA)
         for T in Ts:
@@ -488,6 +489,46 @@ def run_fig5_leg(args):
             "higher_is_better": True, "n_gpus": 1, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"C2 heat {n}^3, tiles {td}, T sweep {Ts}"}, "sweep": out,
             "pcie_gbs": bw}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_fig5_tiles_leg(args):
+    """Region-count sweep of the Fig. 5 analogue (the paper's best was
+    16 regions at 512^3): C2 heat e2e (H2D + T steps + D2H) with the default
+    schedule for several tile shapes."""
+    import torch
+    from paper_conf_icpp_bastemuzas17_b200 import tiles as Tl
+    import synth
+    n = args.n or 512
+    gdims = (n, n, n)
+    cells = n ** 3
+    Ts = [int(v) for v in (args.sweep or "1,10,100").split(",")]
+    shapes = [(n, n, n // 16), (n, n // 2, n // 8), (n // 2, n // 2, n // 4), (n // 4, n // 4, n // 4),
+              (n // 8, n // 8, n // 8), (n // 16, n // 16, n // 16)]
+    torch.cuda.set_device(0)
+    out = {}
+    k = Tl.heat7(ALPHA)
+    ns = args.nstreams or 4
+    for td in shapes:
+        dom = Tl.Domain(gdims, td, ghost=1, device=0)
+        fill_tiles(dom, Tl, synth, gdims, td, 0, 42)
+        key = f"{n // td[0] * (n // td[1]) * (n // td[2])} tiles of {td}"
+        for T in Ts:
+            dom.invalidate(); dom.run(k, min(T, 10), ns); dom.sync()
+            best = 1e30
+            for _ in range(3 if T <= 10 else 1):
+                dom.invalidate()
+                dom.timer_start()
+                dom.run(k, T, ns)
+                dom.sync()
+                best = min(best, dom.timer_stop())
+            out.setdefault(key, {})[str(T)] = {"ms": best, "gcell_per_s": cells * T / (best / 1e3) / 1e9}
+        dom.free()
+    line = {"metric": "Gcell-updates/s incl. H2D/D2H vs region count (Fig. 5 analogue)", "value": None,
+            "unit": "Gcell-updates/s", "higher_is_better": True, "n_gpus": 1, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": f"C2 heat {n}^3, T sweep {Ts}, tile sweep"},
+            "sweep": out}
     print(json.dumps(line), flush=True)
     return 0
 
@@ -610,7 +651,7 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="tiles", choices=["tiles", "reference"])
-    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS) + ["c3", "c4", "c5", "fig5", "fig8"])
+    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS) + ["c3", "c4", "c5", "fig5", "fig5tiles", "fig8"])
     ap.add_argument("--T", type=int, default=None)
     ap.add_argument("--nstreams", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -622,6 +663,8 @@ def main():
     ap.add_argument("--ghost", type=int, default=1,
                     help="c2/c3: ghost width; 2 = two Jacobi steps per pass (temporal blocking)")
     ap.add_argument("--two-step", type=int, default=0, help="tile_options.two_step (-1, 0, 1)")
+    ap.add_argument("--stream-through", type=int, default=0,
+                    help="tile_options.stream_through (-1 never, 0 cost model, 1 when feasible)")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -633,6 +676,8 @@ def main():
         return run_fig8_leg(args)
     if args.config == "fig5":
         return run_fig5_leg(args)
+    if args.config == "fig5tiles":
+        return run_fig5_tiles_leg(args)
     if args.config == "c5":
         return run_c5_leg(args)
 

@@ -113,15 +113,19 @@ typedef struct {
                                    the paper's "CUDA pageable" baseline (P:L37,
                                    Fig. 1/5); copies are staged by the driver
                                    and do not overlap. 0 (default): pinned. */
-  int32_t stream_through;       /* HEAT7 run starting from a fresh upload: 0
-                                   (default) = per z-layer trapezoid (gather the
-                                   layer + T halo planes, T sweeps, D2H the
-                                   exact core) when T <= tile_dims[2] / 2 and
-                                   the scratch fits, so H2D, compute and D2H of
-                                   different layers overlap; each layer's result
+  int32_t stream_through;       /* HEAT7 run starting from a fresh upload
+                                   (periodic, single rank, T <= tile_dims[2],
+                                   scratch fits): per unit of planes (a slice
+                                   of a z-layer, >= T planes) trapezoid: gather
+                                   the unit + T halo planes, T sweeps, D2H the
+                                   exact core, so H2D, compute and D2H of
+                                   different units overlap; each unit's result
                                    is also written back to the device array once
-                                   no other layer reads its initial data. -1 =
-                                   never. */
+                                   no other unit reads its initial data.
+                                   0 (default) = when a cost model (runtime.cpp
+                                   streamthrough_ok) rates it faster than the
+                                   batched resident schedule; 1 = whenever
+                                   feasible; -1 = never. */
   int32_t two_step;             /* HEAT7 with ghost >= 2: 0 (default) = two
                                    steps per pass in the streaming schedule
                                    (halves host-link bytes per step), single

@@ -637,7 +637,7 @@ static std::vector<int> plan_passes(const Domain& d, int steps) {
 }
 
 // Stream-through: with a fresh upload, a cell after T steps
-// depends only on cells within T planes, so with T <= tz/2 each z-layer's
+// depends only on cells within T planes, so with T <= tz each z-layer's
 // final state needs only its own and the two adjacent layers' initial data.
 // Per layer (in z order): gather the layer and T halo planes into a dense
 // slab, run T sweeps with the valid range shrinking by one plane per end,
@@ -650,7 +650,7 @@ static std::vector<int> plan_passes(const Domain& d, int steps) {
 // periodic wrap, at the end), so the domain stays resident. Periodic, single
 // rank.
 struct StreamPlan {
-  int64_t unit;        // planes per unit (divides tz, >= 2T)
+  int64_t unit;        // planes per unit (divides tz, >= T)
   int64_t units;       // local nz / unit
   int64_t slab_tiles;  // one dense slab of unit + 2T planes, in tile slots
   int64_t sub_tiles;   // one packed unit result (layer_tiles sub-tiles), in tile slots
@@ -659,16 +659,38 @@ struct StreamPlan {
 static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
   const Geometry& G = d.G;
   if (d.opt.stream_through < 0 || G.nranks != 1 || G.bc != TILE_BC_PERIODIC) return false;
-  if (T < 1 || 2 * (int64_t)T > G.t[2]) return false;
+  if (T < 1 || (int64_t)T > G.t[2]) return false;
   const int64_t plane = G.l[0] * G.l[1];
-  // thinnest unit >= max(2T, 16) planes dividing tz (thin units shorten the
-  // pipeline's fill and drain; a unit needs only its two neighbour units)
+  // unit = a divisor of tz, >= T (after T steps a unit then depends on its
+  // two neighbour units only) and >= min_unit (per-unit overheads). Thin
+  // units shorten the pipeline's fill and drain (~3 units of one-way copies);
+  // thick ones cut the redundant halo sweeps (a unit sweeps T*unit + T^2 - T
+  // planes). Pick the divisor minimising, in per-plane link-copy times,
+  //   max(nz, r * nz * (T + (T^2 - T) / unit)) + 3 * unit,
+  // r = sweep time / duplex link time per plane, 0.03 measured on B200 +
+  // PCIe 5 (slab_sweep ~1.3 us per 512^2 plane, ~48 GB/s per direction).
+  // Fit to the Fig. 5 T sweep (profiles/r01/bench_fig5_st_{never,forced}.json).
+  static const int64_t min_unit = [] {
+    const char* e = getenv("TILES_ST_MINUNIT");
+    return e ? std::max<int64_t>(1, atoll(e)) : (int64_t)16;
+  }();
+  static const double r_sweep = [] {
+    const char* e = getenv("TILES_ST_R");
+    return e ? atof(e) : 0.030;
+  }();
+  const double nz = (double)G.l[2], Td = (double)T;
   int64_t unit = G.t[2];
-  for (int64_t u = 1; u <= G.t[2]; ++u)
-    if (G.t[2] % u == 0 && u >= 2 * (int64_t)T && u >= std::min<int64_t>(16, G.t[2])) {
-      unit = u;
-      break;
-    }
+  double best = 1e300;
+  for (int64_t u = 1; u <= G.t[2]; ++u) {
+    if (G.t[2] % u || u < (int64_t)T || u < std::min<int64_t>(min_unit, G.t[2])) continue;
+    const double est = std::max(nz, r_sweep * nz * (Td + (Td * Td - Td) / (double)u)) + 3.0 * (double)u;
+    if (est < best) best = est, unit = u;
+  }
+  // the batched resident schedule instead: both link directions in sequence
+  // (dependency form, 2 nz) plus T whole-domain steps, partly overlapped
+  // (0.011 per plane-step, same fit); take stream-through only where it is
+  // estimated faster
+  if (d.opt.stream_through == 0 && best > 2.0 * nz + 0.011 * nz * Td) return false;
   const int64_t units = G.l[2] / unit;
   if (units > G.ntiles) unit = G.t[2];  // event budget (one per unit)
   sp->unit = unit;

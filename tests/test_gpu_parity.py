@@ -311,14 +311,15 @@ def test_two_step_passes_bit_exact(bc, dims, td, runs):
 
 
 @pytest.mark.parametrize("dims,td,T", [((128, 64, 256), (64, 32, 32), 5), ((64, 64, 192), (32, 32, 64), 10),
-                                       ((64, 64, 256), (64, 64, 32), 1)])
+                                       ((64, 64, 256), (64, 64, 32), 1), ((64, 64, 512), (64, 64, 32), 20),
+                                       ((64, 32, 1024), (32, 32, 64), 64)])
 def test_stream_through_bit_exact(dims, td, T):
-    """Fresh-upload runs with T <= tz/2 take the stream-through schedule
+    """Fresh-upload runs with T <= tz take the stream-through schedule
     (units of planes, gather + T sweeps + scatter, D2H, write-back); the host
     result and the kept device copy (a following resident run) are exact."""
     nx, ny, nz = dims
     u0 = synth.uniform_grid(nx, ny, nz, 42)
-    with T_.Domain(dims, td) as d:
+    with T_.Domain(dims, td, stream_through=1) as d:   # forced (the default is cost-model driven)
         d.load(u0)
         d.run(T_.heat7(), T, 2)
         out1 = d.store()

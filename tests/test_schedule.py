@@ -288,9 +288,10 @@ def test_two_step_passes_replay_to_oracle(bc, sched, td):
 
 @pytest.mark.parametrize("dims,td,T,ns", [((16, 16, 64), (8, 8, 8), 3, 2), ((16, 8, 64), (8, 4, 8), 4, 3),
                                           ((16, 16, 64), (8, 8, 8), 2, 1), ((32, 16, 48), (16, 8, 8), 1, 4),
-                                          ((16, 16, 128), (8, 8, 32), 2, 2), ((16, 8, 192), (8, 4, 48), 7, 2)])
+                                          ((16, 16, 128), (8, 8, 32), 2, 2), ((16, 8, 192), (8, 4, 48), 7, 2),
+                                          ((16, 16, 64), (8, 8, 8), 6, 2), ((16, 8, 384), (8, 4, 48), 20, 3)])
 def test_stream_through_schedule_replays_to_oracle(dims, td, T, ns):
-    """Fresh-upload heat runs with T <= tz/2 use the stream-through schedule
+    """Fresh-upload heat runs with T <= tz use the stream-through schedule
     (per-layer gather + T shrinking sweeps + scatter + D2H); replayed in random
     valid orders it must give the oracle bit-exactly."""
     d = _run_and_replay(dims, td, [T], ns, seeds=(0, 1, 2))
