@@ -176,9 +176,13 @@ typedef enum {
   TILE_OP_HIT = 10,     /* tile a found in slot b (P:L90 cache hit) */
   TILE_OP_POINTWISE = 11,/* compute-intensive kernel on tile a in slot b, c iterations */
   TILE_OP_KERNEL2 = 12,  /* like KERNEL, two steps in one pass (ghost width 2) */
-  TILE_OP_GATHER = 13,   /* layer a + halo -> dense slab at slot b: c planes from z = d */
-  TILE_OP_SWEEP = 14,    /* slab slot a -> slab slot b, planes [c, d) */
-  TILE_OP_SCATTER = 15,  /* slab slot a core planes from c -> tile-blocked slots from b (layer d) */
+  TILE_OP_GATHER = 13,   /* reserved (no longer emitted: fused into SWEEP) */
+  TILE_OP_SWEEP = 14,    /* one Jacobi sweep of slab planes [c & 0xffffffff, c >> 32),
+                            periodic in x/y. a >= 0: dense slab at slot a; a < 0:
+                            the resident array -1-a with slab plane 0 at local
+                            z = d (wrapped). b >= 0: dense slab at slot b; b < 0:
+                            packed sub-tiles at slot -1-b (sweep plane lo -> 0) */
+  TILE_OP_SCATTER = 15,  /* reserved (no longer emitted: fused into SWEEP) */
   TILE_OP_COPY = 16,     /* device copy of c tile slots: slot a -> slot b */
   /* partial (sub-layer) copies of planes [d & 0xffffffff, + d >> 32) of c tiles: */
   TILE_OP_H2D_PART = 17, /* host tiles a.. -> slots b.. */

@@ -164,51 +164,38 @@ struct CudaExec final : Exec {
     d.stats.n_kernels++;
     return Status::ok();
   }
-  SlabParams slab_base(Domain& d) {
-    SlabParams p{};
-    p.nx = d.G.l[0];
-    p.ny = d.G.l[1];
-    p.nz = d.G.l[2];
-    p.tx = d.G.t[0];
-    p.ty = d.G.t[1];
-    p.tz = d.G.t[2];
-    p.ntx = d.G.n[0];
-    p.nty = d.G.n[1];
-    p.tile_elems = d.G.tile_elems;
-    p.alpha = d.kernel_alpha;
-    return p;
+  SlabView slab_view(Domain& d, const SlabRef& r, int lo) {
+    const Geometry& G = d.G;
+    SlabView v{};
+    v.ntx = (int)G.n[0];
+    v.nty = (int)G.n[1];
+    v.tx = (int)G.t[0];
+    v.ty = (int)G.t[1];
+    v.tz = 1 << 30;
+    if (r.kind == SlabRef::DENSE) {
+      v.base = d.slot_ptr(r.slot);
+      v.tx = (int)G.l[0];
+      v.ty = (int)G.l[1];
+      v.ntx = v.nty = 1;
+    } else if (r.kind == SlabRef::RESIDENT) {
+      v.base = d.slot_ptr(r.slot ? (int)G.ntiles : 0);
+      v.te = G.tile_elems;
+      v.tz = (int)G.t[2];
+      v.zbase = (int)r.zbase;
+      v.nz = (int)G.l[2];
+    } else {  // SUB: packed sub-tiles of st_unit planes; sweep plane lo -> 0
+      v.base = d.slot_ptr(r.slot);
+      v.te = d.st_unit * G.t[0] * G.t[1];
+      v.zbase = -lo;
+    }
+    return v;
   }
-  Status slab_gather(Domain& d, int64_t, int src_bit, int slab, int64_t zbase, int64_t planes,
-                     int st) override {
+  Status slab_sweep(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi, int st) override {
     if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
-    SlabParams p = slab_base(d);
-    p.tiles = d.slot_ptr(src_bit ? (int)d.G.ntiles : 0);
-    p.slab = d.slot_ptr(slab);
-    p.zbase = zbase;
-    p.planes = planes;
-    Status r = timed(d, st, [&] { return launch_slab_gather(p, sms, S(st)); });
-    if (r.bad()) return r;
-    d.stats.n_kernels++;
-    return Status::ok();
-  }
-  Status slab_sweep(Domain& d, int src, int dst, int lo, int hi, int st) override {
-    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
-    SlabParams p = slab_base(d);
+    const SlabView s = slab_view(d, src, lo), t = slab_view(d, dst, lo);
     Status r = timed(d, st, [&] {
-      return launch_slab_sweep(p, d.slot_ptr(src), d.slot_ptr(dst), lo, hi, sms, S(st));
+      return launch_slab_sweep(s, t, (int)d.G.l[0], (int)d.G.l[1], lo, hi, d.kernel_alpha, sms, S(st));
     });
-    if (r.bad()) return r;
-    d.stats.n_kernels++;
-    return Status::ok();
-  }
-  Status slab_scatter(Domain& d, int slab, int first, int out, int64_t, int st) override {
-    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
-    SlabParams p = slab_base(d);
-    p.tz = d.st_unit;  // planes per unit; packed sub-tiles of tz*ty*tx elements
-    p.tile_elems = d.st_unit * d.G.t[0] * d.G.t[1];
-    p.slab = d.slot_ptr(slab);
-    p.out = d.slot_ptr(out);
-    Status r = timed(d, st, [&] { return launch_slab_scatter(p, first, sms, S(st)); });
     if (r.bad()) return r;
     d.stats.n_kernels++;
     return Status::ok();

@@ -64,20 +64,14 @@ struct DryExec final : Exec {
     for (size_t i = mark; i < d.trace.size(); ++i) d.trace[i].kind = TILE_OP_KERNEL2;
     return r;
   }
-  Status slab_gather(Domain& d, int64_t layer, int, int slab, int64_t zbase, int64_t planes,
-                     int st) override {
+  Status slab_sweep(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi, int st) override {
     d.stats.n_kernels++;
-    put(d, TILE_OP_GATHER, st, layer, slab, planes, zbase);
-    return Status::ok();
-  }
-  Status slab_sweep(Domain& d, int src, int dst, int lo, int hi, int st) override {
-    d.stats.n_kernels++;
-    put(d, TILE_OP_SWEEP, st, src, dst, lo, hi);
-    return Status::ok();
-  }
-  Status slab_scatter(Domain& d, int slab, int first, int out, int64_t layer, int st) override {
-    d.stats.n_kernels++;
-    put(d, TILE_OP_SCATTER, st, slab, out, first, layer);
+    // a: slab slot, or -1-bit for the resident array (slab plane 0 at z = d)
+    // b: slab slot, or -1-slot for packed sub-tiles (sweep plane lo -> 0)
+    const int64_t a = src.kind == SlabRef::DENSE ? src.slot : -1 - (int64_t)src.slot;
+    const int64_t b = dst.kind == SlabRef::DENSE ? dst.slot : -1 - (int64_t)dst.slot;
+    put(d, TILE_OP_SWEEP, st, a, b, (int64_t)lo | ((int64_t)hi << 32),
+        src.kind == SlabRef::RESIDENT ? src.zbase : 0);
     return Status::ok();
   }
   Status h2d_part(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int st) override {

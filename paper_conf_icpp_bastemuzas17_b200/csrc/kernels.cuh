@@ -93,21 +93,20 @@ cudaError_t launch_heat7(const HeatParams& p, int stages, size_t smem, int grid,
 cudaError_t launch_sincos(const SincosParams& p, int grid, cudaStream_t s);
 
 // Stream-through (trapezoid) slab kernels (kernels_slab.cu).
-struct SlabParams {
-  int64_t nx, ny, nz;           // rank-local grid (nz wraps the gather)
-  int64_t tx, ty, tz, ntx, nty;
-  int64_t tile_elems;
-  int64_t zbase;                // local z of slab plane 0 (gather)
-  int64_t planes;               // planes to gather
-  const double* tiles;          // tile-blocked array (gather source)
-  double* slab;                 // dense slab [planes][ny][nx]
-  double* out;                  // tile-blocked layer (scatter destination)
-  double alpha;
+// A stream-through slab seen through a (possibly tile-blocked) layout: slab
+// plane p, row y, column x live at
+//   base + [iz*nty*ntx*te + lz*ty*tx] + [iy*ntx*te + ly*tx] + [ix*te + lx]
+// with gz = zbase + p (wrapped mod nz if nz > 0), (iz, lz) = divmod(gz, tz),
+// (iy, ly) = divmod(y, ty), (ix, lx) = divmod(x, tx). A dense slab is the view
+// with tx = nx, ty = ny, one tile.
+struct SlabView {
+  double* base;
+  int64_t te;                   // elements per tile (or per packed sub-tile)
+  int tx, ty, tz, ntx, nty;
+  int zbase, nz;
 };
-cudaError_t launch_slab_gather(const SlabParams& p, int sms, cudaStream_t s);
-cudaError_t launch_slab_sweep(const SlabParams& p, const double* src, double* dst, int lo, int hi,
-                              int sms, cudaStream_t s);
-cudaError_t launch_slab_scatter(const SlabParams& p, int first, int sms, cudaStream_t s);
+cudaError_t launch_slab_sweep(const SlabView& src, const SlabView& dst, int nx, int ny, int lo,
+                              int hi, double alpha, int sms, cudaStream_t s);
 // Two-step kernel: returns false from heat2_plan if no specialisation fits.
 bool heat2_plan(int tx, int ty, int max_smem, int* band, size_t* smem);
 cudaError_t heat2_configure(int tx, int band, size_t smem, int* ctas_per_sm);

@@ -1,104 +1,183 @@
-// kernels_slab.cu — "stream-through" (trapezoid) kernels, DESIGN.md §5.
+// kernels_slab.cu — the stream-through (trapezoid) sweep kernel, DESIGN.md §5.
 //
-// A z-layer of tiles plus T halo planes on each side is gathered into a
-// dense slab ([planes][ny][nx], periodic in x and y within the plane), T
-// Jacobi sweeps run on the slab with the valid z-range shrinking by one plane
-// per sweep at each end, and the layer's tz exact core planes are scattered
-// back into tile-blocked order for the D2H. Every cell update is the same
-// rounded expression as heat7 (reading R1), so results are bit-identical.
-// All three kernels are HBM-streaming (no reuse beyond neighbouring rows and
-// planes, which L1/L2 catch): coalesced 128-bit accesses, grids sized in
-// multiples of the SM count.
+// One Jacobi sweep over planes [lo, hi) of a unit's slab (the unit's planes
+// plus T halo planes on each side, periodic in x and y within the plane).
+// Source and destination are "views" of the same logical slab:
+//   - the dense scratch slab [plane][ny][nx] (middle sweeps),
+//   - the tile-blocked resident array at local z = zbase + plane, wrapped
+//     (first sweep: the gather is fused into it),
+//   - the unit's packed sub-tiles [layer tile][plane - first][ty][tx] (last
+//     sweep: the scatter is fused into it).
+// Every cell update is the same rounded expression as heat7 (reading R1), so
+// results are bit-identical to the untiled oracle.
+//
+// Register z-march: a thread owns one x-pair (double2) of BY rows and walks a
+// chunk of planes keeping planes z-1, z, z+1 in registers;
+// the y neighbours are its own rows (plus two halo rows per plane), the x
+// neighbours come from the adjacent lanes by shuffle (warp-edge lanes load
+// them). Per cell: one 16-B load and one 16-B store of algorithmic traffic.
+#include <cstdlib>
+#include <numeric>
+
 #include "kernels.cuh"
 #include "ptx.cuh"
 
 namespace tiles {
 
-// dense slab plane p (global z = zbase + p, wrapped) <- tile-blocked array
-__global__ void __launch_bounds__(256) slab_gather(const __grid_constant__ SlabParams p) {
-  const int64_t nx = p.nx, ny = p.ny, tx = p.tx, ty = p.ty, tz = p.tz;
-  const int64_t pairs_per_plane = nx * ny / 2;
-  const int64_t total = pairs_per_plane * p.planes;
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total;
-       e += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t pl = e / pairs_per_plane;
-    const int64_t r = e - pl * pairs_per_plane;
-    const int64_t y = (2 * r) / nx, x = (2 * r) % nx;
-    int64_t gz = (p.zbase + pl) % p.nz;
-    if (gz < 0) gz += p.nz;
-    const int64_t iz = gz / tz, lz = gz % tz, ix = x / tx, iy = y / ty;
-    const int64_t tile = (iz * p.nty + iy) * p.ntx + ix;
-    const double* src = p.tiles + tile * p.tile_elems + (lz * ty + (y % ty)) * tx + (x % tx);
-    *reinterpret_cast<double2*>(p.slab + (pl * ny + y) * nx + x) =
-        *reinterpret_cast<const double2*>(src);
+struct ViewDev {
+  double* base;
+  int64_t te;
+  int tx, ty, tz, ntx, nty, zbase, nz;
+  __device__ __forceinline__ int64_t Z(int pl) const {
+    int gz = zbase + pl;
+    if (nz > 0) {
+      gz %= nz;
+      if (gz < 0) gz += nz;
+    }
+    const int iz = gz / tz, lz = gz - iz * tz;
+    return (int64_t)iz * nty * ntx * te + (int64_t)lz * ty * tx;
+  }
+  __device__ __forceinline__ int64_t Y(int y) const {
+    const int iy = y / ty;
+    return (int64_t)iy * ntx * te + (int64_t)(y - iy * ty) * tx;
+  }
+  __device__ __forceinline__ int64_t X(int x) const {
+    const int ix = x / tx;
+    return (int64_t)ix * te + (x - ix * tx);
+  }
+};
+
+static ViewDev to_dev(const SlabView& v) {
+  return ViewDev{v.base, v.te, v.tx, v.ty, v.tz, v.ntx, v.nty, v.zbase, v.nz};
+}
+
+// Work items are (z chunk, column) pairs, column = (x segment of 128 pairs,
+// group of BY rows), enumerated chunk-major; a resident grid of (SMs x
+// blocks per SM) takes them round-robin, so blocks running at the same time
+// work on neighbouring columns of the same z chunk and the halo rows they
+// share come from L2.
+template <int BY>
+__global__ void __launch_bounds__(128, 4) slab_sweep_zm(const ViewDev S, const ViewDev D, const int nx,
+                                                        const int ny, const int lo, const int hi,
+                                                        const int gx, const int zc, const double alpha) {
+  const int npairs = nx >> 1;
+  const int lane = threadIdx.x & 31;
+  const int cols = gx * (ny / BY);
+  const int nch = (hi - lo + zc - 1) / zc;
+  const int64_t items = (int64_t)cols * nch;
+  const double* sb = S.base;
+  const int stx = S.tx, dtx = D.tx;
+
+  for (int64_t it = blockIdx.x; it < items; it += gridDim.x) {
+    const int ch = (int)(it / cols), col = (int)(it - (int64_t)ch * cols);
+    const int zlo = lo + ch * zc, zhi = min(hi, zlo + zc);
+    const int seg = col % gx, y0 = (col / gx) * BY;
+    const int px = seg * 128 + (int)threadIdx.x;
+    const bool valid = px < npairs;
+    const int x = 2 * (valid ? px : npairs - 1);
+    const bool ledge = lane == 0, redge = lane == 31 || px + 1 >= npairs;
+    const int64_t sx = S.X(x), dx = D.X(x);
+    const int64_t exo_m = S.X(x == 0 ? nx - 1 : x - 1) - sx, exo_p = S.X(x + 2 == nx ? 0 : x + 2) - sx;
+    // BY divides ty in every view (the launcher picks it so): the BY rows
+    // are consecutive rows of one tile row, row j at Y(y0) + j * tx
+    const int64_t sy0 = S.Y(y0) + sx, dy0 = D.Y(y0) + dx;
+    const int64_t shm = S.Y(y0 == 0 ? ny - 1 : y0 - 1) + sx;
+    const int64_t shp = S.Y(y0 + BY == ny ? 0 : y0 + BY) + sx;
+
+    double2 zm[BY], zcur[BY];
+    {
+      const int64_t o0 = S.Z(zlo - 1), o1 = S.Z(zlo);
+#pragma unroll
+      for (int j = 0; j < BY; ++j) {
+        zm[j] = *reinterpret_cast<const double2*>(sb + o0 + sy0 + (int64_t)j * stx);
+        zcur[j] = *reinterpret_cast<const double2*>(sb + o1 + sy0 + (int64_t)j * stx);
+      }
+    }
+    for (int z = zlo; z < zhi; ++z) {
+      const int64_t oc = S.Z(z), on = S.Z(z + 1);
+      double2 zp[BY];
+      double em[BY], ep[BY];
+#pragma unroll
+      for (int j = 0; j < BY; ++j) {
+        const int64_t r = sy0 + (int64_t)j * stx;
+        zp[j] = *reinterpret_cast<const double2*>(sb + on + r);
+        em[j] = ledge ? sb[oc + r + exo_m] : 0.0;
+        ep[j] = redge ? sb[oc + r + exo_p] : 0.0;
+      }
+      const double2 hm = *reinterpret_cast<const double2*>(sb + oc + shm);
+      const double2 hp = *reinterpret_cast<const double2*>(sb + oc + shp);
+      const int64_t od = D.Z(z);
+#pragma unroll
+      for (int j = 0; j < BY; ++j) {
+        const double2 c = zcur[j];
+        double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+        double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+        if (ledge) xm = em[j];
+        if (redge) xp = ep[j];
+        const double2 ym = j == 0 ? hm : zcur[j > 0 ? j - 1 : 0];
+        const double2 yp = j == BY - 1 ? hp : zcur[j < BY - 1 ? j + 1 : 0];
+        double2 v;
+        v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm[j].x, zp[j].x, alpha);
+        v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm[j].y, zp[j].y, alpha);
+        if (valid) *reinterpret_cast<double2*>(D.base + od + dy0 + (int64_t)j * dtx) = v;
+      }
+#pragma unroll
+      for (int j = 0; j < BY; ++j) {
+        zm[j] = zcur[j];
+        zcur[j] = zp[j];
+      }
+    }
   }
 }
 
-// one Jacobi sweep on planes [lo, hi) of the slab (src -> dst), periodic in
-// x and y; planes lo-1 and hi must be valid in src
-__global__ void __launch_bounds__(256) slab_sweep(const __grid_constant__ SlabParams p,
-                                                  const double* __restrict__ src,
-                                                  double* __restrict__ dst, int lo, int hi) {
-  const int64_t nx = p.nx, ny = p.ny;
-  const int64_t pairs_per_plane = nx * ny / 2;
-  const int64_t total = pairs_per_plane * (hi - lo);
-  const double alpha = p.alpha;
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total;
-       e += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t pl = lo + e / pairs_per_plane;
-    const int64_t r = e % pairs_per_plane;
-    const int64_t y = (2 * r) / nx, x = (2 * r) % nx;
-    const double* row = src + (pl * ny + y) * nx;
-    const double2 c = *reinterpret_cast<const double2*>(row + x);
-    const double xm = row[x == 0 ? nx - 1 : x - 1];
-    const double xp = row[x + 2 == nx ? 0 : x + 2];
-    const int64_t ym_ = y == 0 ? ny - 1 : y - 1, yp_ = y + 1 == ny ? 0 : y + 1;
-    const double2 ym = *reinterpret_cast<const double2*>(src + (pl * ny + ym_) * nx + x);
-    const double2 yp = *reinterpret_cast<const double2*>(src + (pl * ny + yp_) * nx + x);
-    const double2 zm = *reinterpret_cast<const double2*>(src + ((pl - 1) * ny + y) * nx + x);
-    const double2 zp = *reinterpret_cast<const double2*>(src + ((pl + 1) * ny + y) * nx + x);
-    double2 v;
-    v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm.x, zp.x, alpha);
-    v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm.y, zp.y, alpha);
-    *reinterpret_cast<double2*>(dst + (pl * ny + y) * nx + x) = v;
+static int sweep_occupancy(int BY) {
+  static int occ[3] = {0, 0, 0};
+  const int k = BY == 4 ? 2 : BY == 2 ? 1 : 0;
+  if (!occ[k]) {
+    int o = 1;
+    if (BY == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, slab_sweep_zm<4>, 128, 0);
+    else if (BY == 2) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, slab_sweep_zm<2>, 128, 0);
+    else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, slab_sweep_zm<1>, 128, 0);
+    occ[k] = o < 1 ? 1 : o;
   }
+  return occ[k];
 }
 
-// tile-blocked layer (out) <- slab core planes [first, first+tz)
-__global__ void __launch_bounds__(256) slab_scatter(const __grid_constant__ SlabParams p, int first) {
-  const int64_t nx = p.nx, ny = p.ny, tx = p.tx, ty = p.ty, tz = p.tz;
-  const int64_t pairs_per_plane = nx * ny / 2;
-  const int64_t total = pairs_per_plane * tz;
-  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total;
-       e += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t lz = e / pairs_per_plane;
-    const int64_t r = e - lz * pairs_per_plane;
-    const int64_t y = (2 * r) / nx, x = (2 * r) % nx;
-    const int64_t tile = (y / ty) * p.ntx + (x / tx);  // within the layer
-    double* o = p.out + tile * p.tile_elems + (lz * ty + (y % ty)) * tx + (x % tx);
-    stg2_stream(o, *reinterpret_cast<const double2*>(p.slab + ((first + lz) * ny + y) * nx + x));
+cudaError_t launch_slab_sweep(const SlabView& src, const SlabView& dst, int nx, int ny, int lo,
+                              int hi, double alpha, int sms, cudaStream_t s) {
+  if (hi <= lo) return cudaSuccess;
+  const int npairs = nx / 2;
+  const int gx = (npairs + 127) / 128;
+  // rows per thread: must divide every view's ty (the dense slab's is ny,
+  // the tiled views' the tile's)
+  const int tyg = std::gcd(src.ty, dst.ty);
+  static const int by_max = [] {
+    const char* e = getenv("TILES_SWEEP_BY");
+    return e ? atoi(e) : 4;
+  }();
+  const int BY = tyg % 4 == 0 && by_max >= 4 ? 4 : tyg % 2 == 0 && by_max >= 2 ? 2 : 1;
+  const int64_t cols = (int64_t)gx * (ny / BY);
+  const int planes = hi - lo;
+  const int64_t G = (int64_t)sms * sweep_occupancy(BY);
+  // z chunk: >= 8 planes (a chunk re-reads 2 boundary planes), as many
+  // chunks as balance the resident grid best (items / G rounded up)
+  int zc = planes, best_nch = 1;
+  double best = 1e30;
+  for (int nch = 1; nch <= std::max(1, planes / 8); ++nch) {
+    const int64_t items = cols * nch;
+    const int64_t rounds = (items + G - 1) / G;
+    const int c = (planes + nch - 1) / nch;
+    const double cost = (double)rounds * (c + 2);  // per-block planes incl. prologue
+    if (cost < best) best = cost, best_nch = nch;
   }
-}
-
-static int slab_grid(int64_t work_pairs, int sms) {
-  int64_t g = (work_pairs + 255) / 256;
-  const int64_t cap = (int64_t)sms * 16;
-  return (int)(g < 1 ? 1 : g > cap ? cap : g);
-}
-
-cudaError_t launch_slab_gather(const SlabParams& p, int sms, cudaStream_t s) {
-  slab_gather<<<slab_grid(p.nx * p.ny / 2 * p.planes, sms), 256, 0, s>>>(p);
-  return cudaGetLastError();
-}
-
-cudaError_t launch_slab_sweep(const SlabParams& p, const double* src, double* dst, int lo, int hi,
-                              int sms, cudaStream_t s) {
-  slab_sweep<<<slab_grid(p.nx * p.ny / 2 * (hi - lo), sms), 256, 0, s>>>(p, src, dst, lo, hi);
-  return cudaGetLastError();
-}
-
-cudaError_t launch_slab_scatter(const SlabParams& p, int first, int sms, cudaStream_t s) {
-  slab_scatter<<<slab_grid(p.nx * p.ny / 2 * p.tz, sms), 256, 0, s>>>(p, first);
+  zc = (planes + best_nch - 1) / best_nch;
+  const int64_t grid = std::min<int64_t>(G, cols * ((planes + zc - 1) / zc));
+  const ViewDev S = to_dev(src), D = to_dev(dst);
+  switch (BY) {
+    case 4: slab_sweep_zm<4><<<(unsigned)grid, 128, 0, s>>>(S, D, nx, ny, lo, hi, gx, zc, alpha); break;
+    case 2: slab_sweep_zm<2><<<(unsigned)grid, 128, 0, s>>>(S, D, nx, ny, lo, hi, gx, zc, alpha); break;
+    default: slab_sweep_zm<1><<<(unsigned)grid, 128, 0, s>>>(S, D, nx, ny, lo, hi, gx, zc, alpha); break;
+  }
   return cudaGetLastError();
 }
 

@@ -660,6 +660,7 @@ static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
   const Geometry& G = d.G;
   if (d.opt.stream_through < 0 || G.nranks != 1 || G.bc != TILE_BC_PERIODIC) return false;
   if (T < 1 || (int64_t)T > G.t[2]) return false;
+  if (G.t[0] % 2 || G.l[2] > (1 << 30)) return false;  // x-pairs (double2); int plane index
   const int64_t plane = G.l[0] * G.l[1];
   // unit = a divisor of tz, >= T (after T steps a unit then depends on its
   // two neighbour units only) and >= min_unit (per-unit overheads). Thin
@@ -667,16 +668,16 @@ static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
   // thick ones cut the redundant halo sweeps (a unit sweeps T*unit + T^2 - T
   // planes). Pick the divisor minimising, in per-plane link-copy times,
   //   max(nz, r * nz * (T + (T^2 - T) / unit)) + 3 * unit,
-  // r = sweep time / duplex link time per plane, 0.03 measured on B200 +
-  // PCIe 5 (slab_sweep ~1.3 us per 512^2 plane, ~48 GB/s per direction).
-  // Fit to the Fig. 5 T sweep (profiles/r01/bench_fig5_st_{never,forced}.json).
+  // r = sweep time / duplex link time per plane, 0.024 measured on B200 +
+  // PCIe 5 (slab_sweep_zm ~1.0 us per 512^2 plane, ~48 GB/s per direction;
+  // profiles/r01/ncu_slab_sweep.txt, bench_fig5_st_*.json).
   static const int64_t min_unit = [] {
     const char* e = getenv("TILES_ST_MINUNIT");
     return e ? std::max<int64_t>(1, atoll(e)) : (int64_t)16;
   }();
   static const double r_sweep = [] {
     const char* e = getenv("TILES_ST_R");
-    return e ? atof(e) : 0.030;
+    return e ? atof(e) : 0.024;
   }();
   const double nz = (double)G.l[2], Td = (double)T;
   int64_t unit = G.t[2];
@@ -702,12 +703,13 @@ static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
 
 // Stream-through over units of `unit` planes (a unit is a slice of one tile
 // layer: planes [p0, p0+unit) of each of its tiles, contiguous per tile, so
-// its H2D/D2H are single strided 2-D copies). Per unit u, in z order:
-// gather u and T halo planes into a dense slab, T sweeps with the valid range
-// shrinking by one plane per end, scatter the exact core into packed
-// sub-tiles, D2H them. Unit u's result is written back into the resident
-// array after unit u+1's gather (unit 0, read by the last unit through the
-// periodic wrap, at the end).
+// its H2D/D2H are single strided 2-D copies). Per unit u, in z order: T
+// sweeps over u and T halo planes with the valid range shrinking by one plane
+// per end (the first reads the resident array, the middle ones ping-pong
+// between two dense slabs, the last writes the exact core into packed
+// sub-tiles), then the D2H. Unit u's result is written back into the resident
+// array after unit u+1's first sweep (unit 0, read by the last unit through
+// the periodic wrap, at the end).
 static Status run_streamthrough(Domain& d, double alpha, int T, int S, const StreamPlan& sp) {
   (void)alpha;
   Exec& X = *d.exec;
@@ -751,18 +753,20 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
       r = X.wait(d, ring_ev[u & 1], cs);
       if (r.bad()) return r;
     }
-    r = X.slab_gather(d, u, bit, slab[0], u * un - T, un + 2 * T, cs);
-    if (r.bad()) return r;
-    if (u >= 2) {  // unit u-1's initial data has no reader left
-      r = X.copy_part(d, res_of(u - 1), cur_slot(u - 1), lt, p0_of(u - 1), un, cs);
-      if (r.bad()) return r;
-    }
+    // sweep i reads planes [i-1, un+2T-i+1) and writes [i, un+2T-i); the
+    // first reads the resident array directly (gather fused), the last writes
+    // the unit's packed sub-tiles (scatter fused)
     for (int i = 1; i <= T; ++i) {
-      r = X.slab_sweep(d, slab[(i - 1) & 1], slab[i & 1], i, (int)(un + 2 * T - i), cs);
+      const SlabRef src = i == 1 ? SlabRef{SlabRef::RESIDENT, bit, u * un - T}
+                                 : SlabRef{SlabRef::DENSE, slab[(i - 1) & 1], 0};
+      const SlabRef dst = i == T ? SlabRef{SlabRef::SUB, res_of(u), 0} : SlabRef{SlabRef::DENSE, slab[i & 1], 0};
+      r = X.slab_sweep(d, src, dst, i, (int)(un + 2 * T - i), cs);
       if (r.bad()) return r;
+      if (i == 1 && u >= 2) {  // unit u-1's initial data has no reader left
+        r = X.copy_part(d, res_of(u - 1), cur_slot(u - 1), lt, p0_of(u - 1), un, cs);
+        if (r.bad()) return r;
+      }
     }
-    r = X.slab_scatter(d, slab[T & 1], T, res_of(u), u, cs);
-    if (r.bad()) return r;
     r = X.record(d, ev_unit_done(u), cs);
     if (r.bad()) return r;
     r = X.wait(d, ev_unit_done(u), os);

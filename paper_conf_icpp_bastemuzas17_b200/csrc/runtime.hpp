@@ -82,6 +82,19 @@ void ghost_map(const Geometry& G, int64_t id, int64_t* out);  // (t+2g)^3 box
 // All device work goes through an executor: CudaExec issues CUDA/NCCL calls,
 // DryExec only records the op trace (tests on a CPU-only box).
 struct Domain;
+// Where a stream-through slab lives (runtime.cpp run_streamthrough):
+//   DENSE    - dense [plane][ny][nx] scratch at tile slot `slot`;
+//   RESIDENT - the tile-blocked resident array `slot` (0/1), slab plane 0 at
+//              local z = zbase (wrapped);
+//   SUB      - the unit's packed sub-tiles at slot `slot`; slab plane lo of
+//              the sweep is sub-tile plane 0.
+struct SlabRef {
+  enum Kind { DENSE = 0, RESIDENT = 1, SUB = 2 };
+  int kind;
+  int slot;
+  int64_t zbase;
+};
+
 struct Exec {
   virtual ~Exec() = default;
   virtual Status h2d(Domain& d, int64_t tile0, int64_t ntile, int slot0, int stream) = 0;
@@ -93,12 +106,10 @@ struct Exec {
   virtual Status heat(Domain& d, const int64_t* tiles, const int* in_slots, const int* out_slots,
                       int nitems, int read_parity, const TileItem* dev_items, int stream) = 0;
   virtual Status sincos(Domain& d, int64_t tile, int slot, int64_t iters, int stream) = 0;
-  // stream-through slabs; slab/out locations are slot indices of the scratch
-  virtual Status slab_gather(Domain& d, int64_t layer, int src_bit, int slab_slot, int64_t zbase,
-                             int64_t planes, int stream) = 0;
-  virtual Status slab_sweep(Domain& d, int src_slot, int dst_slot, int lo, int hi, int stream) = 0;
-  virtual Status slab_scatter(Domain& d, int slab_slot, int first, int out_slot, int64_t layer,
-                              int stream) = 0;
+  // stream-through: one Jacobi sweep of slab planes [lo, hi) (periodic in
+  // x and y) from src to dst; see SlabRef
+  virtual Status slab_sweep(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi,
+                            int stream) = 0;
   virtual Status copy_slots(Domain& d, int src_slot, int dst_slot, int64_t n, int stream) = 0;
   // planes [p0, p0+np) of n tiles; "packed" = n sub-tiles of np*ty*tx
   // elements back to back starting at a slot

@@ -262,18 +262,21 @@ class Replayer:
             for t, sl in list(self.loc.items()):
                 if b <= sl < b + c:
                     pass
-        elif name == "gather":
-            self.slabs[b] = self.gather(a, c, d)
         elif name == "sweep":
-            self.slabs[b] = self.sweep(self.slabs[a], self.slabs.get(b), c, d)
-        elif name == "scatter":
-            G = self.G
-            tx, ty, tz = G.t
-            slab = self.slabs[a]
-            unit = slab.shape[0] - 2 * c
-            for i in range(G.n[0] * G.n[1]):
-                ix, iy = i % G.n[0], i // G.n[0]
-                self.sub[(b, i)] = slab[c:c + unit, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx].copy()
+            # a: slab slot, or -1-bit = the resident array with slab plane 0
+            # at local z = d; b: slab slot, or -1-slot = packed sub-tiles
+            # receiving planes [lo, hi)
+            lo, hi = c & 0xffffffff, c >> 32
+            src = self.slabs[a] if a >= 0 else self.gather(hi + 1, d)
+            if b >= 0:
+                self.slabs[b] = self.sweep(src, self.slabs.get(b), lo, hi)
+            else:
+                new = self.sweep(src, None, lo, hi)
+                G = self.G
+                tx, ty, tz = G.t
+                for i in range(G.n[0] * G.n[1]):
+                    ix, iy = i % G.n[0], i // G.n[0]
+                    self.sub[(-b - 1, i)] = new[lo:hi, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx].copy()
         elif name in ("h2d_part", "d2h_part", "copy_part"):
             p0, np_ = d & 0xffffffff, d >> 32
             for i in range(c):
@@ -291,7 +294,7 @@ class Replayer:
         # record / wait / hit / drop: no data movement
 
     # ------------------------------------------------- stream-through slabs
-    def gather(self, layer, planes, zbase):
+    def gather(self, planes, zbase):
         G = self.G
         tx, ty, tz = G.t
         nz = G.l[2]

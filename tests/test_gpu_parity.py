@@ -315,7 +315,8 @@ def test_two_step_passes_bit_exact(bc, dims, td, runs):
                                        ((64, 32, 1024), (32, 32, 64), 64)])
 def test_stream_through_bit_exact(dims, td, T):
     """Fresh-upload runs with T <= tz take the stream-through schedule
-    (units of planes, gather + T sweeps + scatter, D2H, write-back); the host
+    (units of planes, T sweeps reading the resident array first and writing
+    packed sub-tiles last, D2H, write-back); the host
     result and the kept device copy (a following resident run) are exact."""
     nx, ny, nz = dims
     u0 = synth.uniform_grid(nx, ny, nz, 42)

@@ -292,11 +292,13 @@ def test_two_step_passes_replay_to_oracle(bc, sched, td):
                                           ((16, 16, 64), (8, 8, 8), 6, 2), ((16, 8, 384), (8, 4, 48), 20, 3)])
 def test_stream_through_schedule_replays_to_oracle(dims, td, T, ns):
     """Fresh-upload heat runs with T <= tz use the stream-through schedule
-    (per-layer gather + T shrinking sweeps + scatter + D2H); replayed in random
+    (per-unit T shrinking sweeps, resident array -> slabs -> sub-tiles, D2H); replayed in random
     valid orders it must give the oracle bit-exactly."""
     d = _run_and_replay(dims, td, [T], ns, seeds=(0, 1, 2))
     ops = [op[0] for op in d.trace()]
-    assert "gather" in ops and "sweep" in ops and "scatter" in ops and "h2d_part" in ops
+    assert "sweep" in ops and "h2d_part" in ops and "d2h_part" in ops
+    sw = [op for op in d.trace() if op[0] == "sweep"]
+    assert any(op[2] < 0 for op in sw) and any(op[3] < 0 for op in sw)   # fused gather / scatter
     assert d.get_info()["resident"]
     # then a resident continuation and a second stream-through
     _run_and_replay(dims, td, [T, T], ns, seeds=(3,))
