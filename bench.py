@@ -186,14 +186,15 @@ def run_stream_leg(args):
     import synth
     n = args.n or 2048
     td = (256, 256, 256) if n % 256 == 0 else (n // 8, n // 8, n // 8)
-    T = args.T if args.T is not None else 2
+    T = args.T if args.T is not None else 10
     ns = args.nstreams or 4
     budget = int((args.budget_gb or 12.0) * (1 << 30))
     gdims = (n, n, n)
     cells = n ** 3
     torch.cuda.set_device(0)
     t0 = time.perf_counter()
-    dom = Tl.Domain(gdims, td, ghost=args.ghost, device=0, sched="stream", device_budget_bytes=budget)
+    dom = Tl.Domain(gdims, td, ghost=args.ghost, device=0, sched="stream", device_budget_bytes=budget,
+                    stream_through=args.stream_through)
     t_alloc = time.perf_counter() - t0
     t0 = time.perf_counter()
     fill_tiles(dom, Tl, synth, gdims, td, 0, 42)
@@ -216,6 +217,7 @@ def run_stream_leg(args):
     st = dom.stats()
     val = cells * T * args.steps / (tot / 1e3) / 1e9
     info = dom.info
+    Bh_ = st["bytes_h2d"] / args.steps
     # overlap: same schedule, transfers only / kernels only
     def leg(mode, steps=1):
         dom.set_measure(mode)
@@ -242,6 +244,8 @@ def run_stream_leg(args):
             "config": {"workload": f"C3 heat fp64 {n}^3 out-of-core (device budget capped at "
                                    f"{budget / 2**30:.1f} GiB, paper method P:L232), T={T}, ghost={args.ghost}",
                        "ghost": args.ghost, "steps_per_pass": info["steps_per_pass"],
+                       "link_passes_per_run": Bh_ / (cells * 8),
+                       "stream_through": args.stream_through,
                        "dims": gdims, "tile_dims": td, "T": T, "nstreams": ns, "nslots": info["nslots"],
                        "ntiles": info["ntiles"], "host_gb": info["host_bytes"] / 1e9,
                        "device_gb": info["device_bytes"] / 1e9,

@@ -187,7 +187,13 @@ typedef enum {
   /* partial (sub-layer) copies of planes [d & 0xffffffff, + d >> 32) of c tiles: */
   TILE_OP_H2D_PART = 17, /* host tiles a.. -> slots b.. */
   TILE_OP_D2H_PART = 18, /* packed sub-tiles at slot b -> host tiles a.. */
-  TILE_OP_COPY_PART = 19 /* packed sub-tiles at slot a -> slots b.. */
+  TILE_OP_COPY_PART = 19,/* packed sub-tiles at slot a -> slots b.. */
+  TILE_OP_H2D_PACK = 20, /* host tiles a.. (c of them), planes [d & 0xffffffff, +d >> 32)
+                            -> packed sub-tiles at slot b */
+  TILE_OP_SWEEP_U = 21   /* like SWEEP, source = units u-1, u, u+1 (packed sub-tiles at
+                            slots b & 0x1fffff, b >> 21 & 0x1fffff, b >> 42), slab plane 0
+                            at z = u*un - (hi + 1 - un) / 2; a = destination code,
+                            c = lo | hi << 32, d = u | un << 32 */
 } tile_op_kind;
 
 typedef struct {

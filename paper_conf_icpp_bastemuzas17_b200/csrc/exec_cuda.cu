@@ -183,6 +183,15 @@ struct CudaExec final : Exec {
       v.tz = (int)G.t[2];
       v.zbase = (int)r.zbase;
       v.nz = (int)G.l[2];
+    } else if (r.kind == SlabRef::UNITS) {
+      v.ring = 1;
+      v.te = r.un * G.t[0] * G.t[1];
+      v.zbase = (int)r.zbase;
+      v.nz = (int)G.l[2];
+      v.u = (int)r.u;
+      v.un = (int)r.un;
+      v.U = (int)(G.l[2] / r.un);
+      for (int k = 0; k < 3; ++k) v.ubase[k] = d.slot_ptr(r.ring[k]);
     } else {  // SUB: packed sub-tiles of st_unit planes; sweep plane lo -> 0
       v.base = d.slot_ptr(r.slot);
       v.te = d.st_unit * G.t[0] * G.t[1];
@@ -217,6 +226,15 @@ struct CudaExec final : Exec {
                          np * pl, np * pl, (size_t)n, cudaMemcpyDeviceToHost, S(st)));
     d.stats.bytes_d2h += (uint64_t)n * np * pl;
     d.stats.n_d2h++;
+    return Status::ok();
+  }
+  Status h2d_pack(Domain& d, int64_t t0, int64_t n, int ps, int64_t p0, int64_t np, int st) override {
+    if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
+    const size_t pl = (size_t)d.G.t[0] * d.G.t[1] * 8, tb = (size_t)d.G.tile_elems * 8;
+    CK(cudaMemcpy2DAsync(d.slot_ptr(ps), np * pl, reinterpret_cast<const char*>(d.host_tile(t0)) + p0 * pl,
+                         tb, np * pl, (size_t)n, cudaMemcpyHostToDevice, S(st)));
+    d.stats.bytes_h2d += (uint64_t)n * np * pl;
+    d.stats.n_h2d++;
     return Status::ok();
   }
   Status copy_part(Domain& d, int ps, int s0, int64_t n, int64_t p0, int64_t np, int st) override {

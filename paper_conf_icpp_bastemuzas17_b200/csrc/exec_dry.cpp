@@ -66,12 +66,27 @@ struct DryExec final : Exec {
   }
   Status slab_sweep(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi, int st) override {
     d.stats.n_kernels++;
+    if (src.kind == SlabRef::UNITS) {
+      // a: destination code as below; b: unit slots (u-1, u, u+1) packed 21
+      // bits each; c: lo | hi << 32; d: u | un << 32
+      const int64_t b = dst.kind == SlabRef::DENSE ? dst.slot : -1 - (int64_t)dst.slot;
+      put(d, TILE_OP_SWEEP_U, st, b,
+          (int64_t)src.ring[0] | ((int64_t)src.ring[1] << 21) | ((int64_t)src.ring[2] << 42),
+          (int64_t)lo | ((int64_t)hi << 32), src.u | (src.un << 32));
+      return Status::ok();
+    }
     // a: slab slot, or -1-bit for the resident array (slab plane 0 at z = d)
     // b: slab slot, or -1-slot for packed sub-tiles (sweep plane lo -> 0)
     const int64_t a = src.kind == SlabRef::DENSE ? src.slot : -1 - (int64_t)src.slot;
     const int64_t b = dst.kind == SlabRef::DENSE ? dst.slot : -1 - (int64_t)dst.slot;
     put(d, TILE_OP_SWEEP, st, a, b, (int64_t)lo | ((int64_t)hi << 32),
         src.kind == SlabRef::RESIDENT ? src.zbase : 0);
+    return Status::ok();
+  }
+  Status h2d_pack(Domain& d, int64_t t0, int64_t n, int ps, int64_t p0, int64_t np, int st) override {
+    d.stats.bytes_h2d += (uint64_t)n * np * d.G.t[0] * d.G.t[1] * 8;
+    d.stats.n_h2d++;
+    put(d, TILE_OP_H2D_PACK, st, t0, ps, n, p0 | (np << 32));
     return Status::ok();
   }
   Status h2d_part(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int st) override {

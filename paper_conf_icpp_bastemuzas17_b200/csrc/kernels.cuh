@@ -99,11 +99,17 @@ cudaError_t launch_sincos(const SincosParams& p, int grid, cudaStream_t s);
 // with gz = zbase + p (wrapped mod nz if nz > 0), (iz, lz) = divmod(gz, tz),
 // (iy, ly) = divmod(y, ty), (ix, lx) = divmod(x, tx). A dense slab is the view
 // with tx = nx, ty = ny, one tile.
+// Unit-ring variant (out-of-core stream-through): plane gz lies in unit
+// iu = gz / un, held as packed sub-tiles (te = un*ty*tx) in ubase[(iu - u + 1)
+// mod U] (units u-1, u, u+1), local plane gz - iu*un; base is unused.
 struct SlabView {
   double* base;
   int64_t te;                   // elements per tile (or per packed sub-tile)
   int tx, ty, tz, ntx, nty;
   int zbase, nz;
+  int ring;                     // 1: unit-ring view (below)
+  int u, U, un;
+  double* ubase[3];
 };
 cudaError_t launch_slab_sweep(const SlabView& src, const SlabView& dst, int nx, int ny, int lo,
                               int hi, double alpha, int sms, cudaStream_t s);

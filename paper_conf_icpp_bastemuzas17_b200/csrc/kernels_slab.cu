@@ -7,7 +7,9 @@
 //   - the tile-blocked resident array at local z = zbase + plane, wrapped
 //     (first sweep: the gather is fused into it),
 //   - the unit's packed sub-tiles [layer tile][plane - first][ty][tx] (last
-//     sweep: the scatter is fused into it).
+//     sweep: the scatter is fused into it),
+//   - a ring of three units' packed sub-tiles (units u-1, u, u+1: the
+//     out-of-core first sweep).
 // Every cell update is the same rounded expression as heat7 (reading R1), so
 // results are bit-identical to the untiled oracle.
 //
@@ -28,14 +30,24 @@ struct ViewDev {
   double* base;
   int64_t te;
   int tx, ty, tz, ntx, nty, zbase, nz;
-  __device__ __forceinline__ int64_t Z(int pl) const {
+  int ring, u, U, un;
+  double* ub[3];
+  // first element of slab plane pl (x = y = 0 of tile column 0, row 0)
+  __device__ __forceinline__ double* P(int pl) const {
     int gz = zbase + pl;
     if (nz > 0) {
       gz %= nz;
       if (gz < 0) gz += nz;
     }
+    if (ring) {
+      const int iu = gz / un;
+      int k = iu - u + 1;
+      if (k < 0) k += U;
+      if (k >= U) k -= U;
+      return ub[k] + (int64_t)(gz - iu * un) * ty * tx;
+    }
     const int iz = gz / tz, lz = gz - iz * tz;
-    return (int64_t)iz * nty * ntx * te + (int64_t)lz * ty * tx;
+    return base + (int64_t)iz * nty * ntx * te + (int64_t)lz * ty * tx;
   }
   __device__ __forceinline__ int64_t Y(int y) const {
     const int iy = y / ty;
@@ -48,7 +60,8 @@ struct ViewDev {
 };
 
 static ViewDev to_dev(const SlabView& v) {
-  return ViewDev{v.base, v.te, v.tx, v.ty, v.tz, v.ntx, v.nty, v.zbase, v.nz};
+  return ViewDev{v.base, v.te, v.tx, v.ty, v.tz, v.ntx, v.nty, v.zbase, v.nz, v.ring, v.u, v.U, v.un,
+                 {v.ubase[0], v.ubase[1], v.ubase[2]}};
 }
 
 // Work items are (z chunk, column) pairs, column = (x segment of 128 pairs,
@@ -65,7 +78,6 @@ __global__ void __launch_bounds__(128, 4) slab_sweep_zm(const ViewDev S, const V
   const int cols = gx * (ny / BY);
   const int nch = (hi - lo + zc - 1) / zc;
   const int64_t items = (int64_t)cols * nch;
-  const double* sb = S.base;
   const int stx = S.tx, dtx = D.tx;
 
   for (int64_t it = blockIdx.x; it < items; it += gridDim.x) {
@@ -86,27 +98,29 @@ __global__ void __launch_bounds__(128, 4) slab_sweep_zm(const ViewDev S, const V
 
     double2 zm[BY], zcur[BY];
     {
-      const int64_t o0 = S.Z(zlo - 1), o1 = S.Z(zlo);
+      const double* p0 = S.P(zlo - 1);
+      const double* p1 = S.P(zlo);
 #pragma unroll
       for (int j = 0; j < BY; ++j) {
-        zm[j] = *reinterpret_cast<const double2*>(sb + o0 + sy0 + (int64_t)j * stx);
-        zcur[j] = *reinterpret_cast<const double2*>(sb + o1 + sy0 + (int64_t)j * stx);
+        zm[j] = *reinterpret_cast<const double2*>(p0 + sy0 + (int64_t)j * stx);
+        zcur[j] = *reinterpret_cast<const double2*>(p1 + sy0 + (int64_t)j * stx);
       }
     }
     for (int z = zlo; z < zhi; ++z) {
-      const int64_t oc = S.Z(z), on = S.Z(z + 1);
+      const double* pc = S.P(z);
+      const double* pn = S.P(z + 1);
       double2 zp[BY];
       double em[BY], ep[BY];
 #pragma unroll
       for (int j = 0; j < BY; ++j) {
         const int64_t r = sy0 + (int64_t)j * stx;
-        zp[j] = *reinterpret_cast<const double2*>(sb + on + r);
-        em[j] = ledge ? sb[oc + r + exo_m] : 0.0;
-        ep[j] = redge ? sb[oc + r + exo_p] : 0.0;
+        zp[j] = *reinterpret_cast<const double2*>(pn + r);
+        em[j] = ledge ? pc[r + exo_m] : 0.0;
+        ep[j] = redge ? pc[r + exo_p] : 0.0;
       }
-      const double2 hm = *reinterpret_cast<const double2*>(sb + oc + shm);
-      const double2 hp = *reinterpret_cast<const double2*>(sb + oc + shp);
-      const int64_t od = D.Z(z);
+      const double2 hm = *reinterpret_cast<const double2*>(pc + shm);
+      const double2 hp = *reinterpret_cast<const double2*>(pc + shp);
+      double* pd = D.P(z);
 #pragma unroll
       for (int j = 0; j < BY; ++j) {
         const double2 c = zcur[j];
@@ -119,7 +133,7 @@ __global__ void __launch_bounds__(128, 4) slab_sweep_zm(const ViewDev S, const V
         double2 v;
         v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm[j].x, zp[j].x, alpha);
         v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm[j].y, zp[j].y, alpha);
-        if (valid) *reinterpret_cast<double2*>(D.base + od + dy0 + (int64_t)j * dtx) = v;
+        if (valid) *reinterpret_cast<double2*>(pd + dy0 + (int64_t)j * dtx) = v;
       }
 #pragma unroll
       for (int j = 0; j < BY; ++j) {

@@ -794,6 +794,203 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
   return Status::ok();
 }
 
+// ------------------------------------------- out-of-core stream-through
+// The stream (out-of-core) schedule streams every tile through the device
+// once per step. Temporal blocking: a
+// pass of k steps over units of `un` >= k planes needs, per unit, only its
+// own and its two neighbour units' data from the host, so each pass moves
+// every cell across the link once per direction for k steps. Device memory:
+// the input units in a ring (units 0 and U-1 fixed: the periodic wrap reads
+// them at both ends), two dense slabs of un + 2k planes, two packed output
+// units. (k, un) minimise the same estimate as the resident stream-through
+// under the device budget; taken when k >= 2.
+struct OocPlan {
+  int64_t un = 0, U = 0, k = 0, passes = 0, R = 0;
+  int64_t unit_slots = 0, slab_slots = 0;
+};
+
+static bool ooc_streamthrough_ok(const Domain& d, int T, OocPlan* op) {
+  const Geometry& G = d.G;
+  if (d.opt.stream_through < 0 || G.nranks != 1 || G.bc != TILE_BC_PERIODIC || T < 2) return false;
+  if (G.t[0] % 2 || G.l[2] > (1 << 30)) return false;
+  const double nz = (double)G.l[2];
+  const int64_t plane = G.l[0] * G.l[1];
+  static const double r_sweep = [] {
+    const char* e = getenv("TILES_ST_R");
+    return e ? atof(e) : 0.024;
+  }();
+  double best = 1e300;
+  for (int64_t k = 2; k <= std::min<int64_t>(T, G.t[2]); ++k)
+    for (int64_t un = k; un <= G.t[2]; ++un) {
+      if (G.t[2] % un || un < std::min<int64_t>(16, G.t[2])) continue;
+      const int64_t U = G.l[2] / un;
+      if (U > G.ntiles || U < 4) continue;  // one event per unit; ring of >= 2 besides the wrap units
+      const int64_t us = (G.layer_tiles * un * G.t[0] * G.t[1] + G.tile_elems - 1) / G.tile_elems;
+      const int64_t ss = ((un + 2 * k) * plane + G.tile_elems - 1) / G.tile_elems;
+      // 2 fixed input units + R ring units (4, else 3) + 2 output units + 2 slabs
+      const int64_t ring_max = U - 2;
+      int64_t R = std::min<int64_t>(4, ring_max);
+      if ((4 + R) * us + 2 * ss > d.nslots && R > std::min<int64_t>(3, ring_max)) --R;
+      if ((4 + R) * us + 2 * ss > d.nslots) continue;
+      const int64_t P = (T + k - 1) / k;
+      const double kd = (double)(T + P - 1) / P;  // steps per pass (balanced)
+      const double est = (double)P * (std::max(nz, r_sweep * nz * (kd + (kd * kd - kd) / (double)un)) + 3.0 * un);
+      if (est < best) {
+        best = est;
+        op->un = un, op->U = U, op->k = k, op->passes = P, op->R = R, op->unit_slots = us,
+        op->slab_slots = ss;
+      }
+    }
+  if (best >= 1e300) return false;
+  // the per-step stream schedule moves every cell once per direction per
+  // step: T link passes at best
+  if (d.opt.stream_through == 0 && best > (double)T * nz) return false;
+  return true;
+}
+
+static Status run_streamthrough_ooc(Domain& d, int T, int S, const OocPlan& op) {
+  Exec& X = *d.exec;
+  const Geometry& G = d.G;
+  const Pipes P(S, false);
+  const int64_t U = op.U, un = op.un, lt = G.layer_tiles, tz = G.t[2], R = op.R;
+  const int cs = P.comp(0), os = P.out(0), is = P.in(0);
+  Status r;
+  // flush: dirty resident tiles to the host, then nothing is resident
+  {
+    Sched sc(d, P);
+    for (int64_t t = 0; t < G.ntiles; ++t)
+      if (d.tile_slot[t] >= 0 && d.tile_dirty[t]) {
+        r = sc.writeback(t);
+        if (r.bad()) return r;
+      }
+  }
+  for (int s = 0; s < d.nslots; ++s) {  // every slot's previous use before this run
+    r = X.wait(d, ev_slot(d, s), is);
+    if (r.bad()) return r;
+    r = X.wait(d, ev_slot(d, s), cs);
+    if (r.bad()) return r;
+  }
+  for (int64_t t = 0; t < G.ntiles; ++t) {
+    r = X.wait(d, ev_host(d, t), is);  // host copy complete (earlier D2H)
+    if (r.bad()) return r;
+  }
+  // slot layout (unit-sized packed buffers, then slabs)
+  const int us = (int)op.unit_slots, ss = (int)op.slab_slots;
+  const int F0 = 0, F1 = us, ring0 = 2 * us, out0 = ring0 + (int)R * us;
+  const int outb[2] = {out0, out0 + us};
+  const int slab[2] = {out0 + 2 * us, out0 + 2 * us + ss};
+  auto inbuf = [&](int64_t u) {
+    u = (u % U + U) % U;
+    if (u == 0) return F0;
+    if (u == U - 1) return F1;
+    return ring0 + (int)((u - 1) % R) * us;
+  };
+  auto layer_of = [&](int64_t u) { return (u * un) / tz; };
+  auto p0_of = [&](int64_t u) { return (u * un) % tz; };
+  const int ring_ev[2] = {d.ev_misc_base + 4 + d.halo_stream + 1, d.ev_misc_base + 5 + d.halo_stream + 1};
+  auto h2d_unit = [&](int64_t u, int pass) -> Status {
+    if (pass > 0) {
+      Status q = X.wait(d, ev_host(d, u), is);  // previous pass's D2H of u
+      if (q.bad()) return q;
+    }
+    Status q = X.h2d_pack(d, layer_of(u) * lt, lt, inbuf(u), p0_of(u), un, is);
+    if (q.bad()) return q;
+    return X.record(d, ev_in(d, u), is);
+  };
+  for (int pass = 0; pass < (int)op.passes; ++pass) {
+    const int k = (int)(T / op.passes + (pass < T % op.passes ? 1 : 0));
+    if (pass > 0) {  // every buffer of the previous pass is free
+      r = X.wait(d, ev_tile(d, U - 1, 1), is);
+      if (r.bad()) return r;
+    }
+    // H2D order: the wrap neighbour first, then z order; units 1..R fill the
+    // ring, unit u >= R+1 reuses unit u-R's buffer after the first sweep of
+    // unit u-R+1 (its last reader)
+    std::vector<char> issued((size_t)U, 0);
+    auto issue = [&](int64_t u) -> Status {
+      if (u < 0 || u >= U || issued[(size_t)u]) return Status::ok();
+      issued[(size_t)u] = 1;
+      return h2d_unit(u, pass);
+    };
+    r = issue(U - 1);
+    if (r.bad()) return r;
+    for (int64_t u = 0; u <= std::min<int64_t>(R, U - 1); ++u) {
+      r = issue(u);
+      if (r.bad()) return r;
+    }
+    for (int64_t u = 0; u < U; ++u) {
+      for (int64_t du : {(int64_t)-1, (int64_t)0, (int64_t)1}) {
+        r = X.wait(d, ev_in(d, (u + du + U) % U), cs);
+        if (r.bad()) return r;
+      }
+      if (u >= 2 || pass > 0) {  // output buffer u%2 was last read by unit u-2's D2H
+        r = X.wait(d, ring_ev[u & 1], cs);
+        if (r.bad()) return r;
+      }
+      for (int i = 1; i <= k; ++i) {
+        SlabRef src{SlabRef::DENSE, slab[(i - 1) & 1], 0, {0, 0, 0}, 0, 0};
+        if (i == 1) src = SlabRef{SlabRef::UNITS, 0, u * un - k, {inbuf(u - 1), inbuf(u), inbuf(u + 1)}, u, un};
+        const SlabRef dst = i == k ? SlabRef{SlabRef::SUB, outb[u & 1], 0, {0, 0, 0}, 0, 0}
+                                   : SlabRef{SlabRef::DENSE, slab[i & 1], 0, {0, 0, 0}, 0, 0};
+        d.st_unit = un;
+        r = X.slab_sweep(d, src, dst, i, (int)(un + 2 * k - i), cs);
+        if (r.bad()) return r;
+        if (i == 1) {
+          r = X.record(d, ev_tile(d, u, 0), cs);
+          if (r.bad()) return r;
+        }
+      }
+      r = X.record(d, ev_tile(d, u, 1), cs);
+      if (r.bad()) return r;
+      r = X.wait(d, ev_tile(d, u, 1), os);
+      if (r.bad()) return r;
+      r = X.d2h_part(d, layer_of(u) * lt, lt, outb[u & 1], p0_of(u), un, os);
+      if (r.bad()) return r;
+      r = X.record(d, ring_ev[u & 1], os);
+      if (r.bad()) return r;
+      r = X.record(d, ev_host(d, u), os);
+      if (r.bad()) return r;
+      // unit u+R's buffer held unit u; its last reader (unit u+1's first
+      // sweep) is issued next iteration -> issue H2D(u+R) after that
+      if (u >= 2 && u - 1 + R <= U - 2) {
+        r = X.wait(d, ev_tile(d, u, 0), is);
+        if (r.bad()) return r;
+        r = issue(u - 1 + R);
+        if (r.bad()) return r;
+      }
+    }
+    for (int64_t u = 0; u < U; ++u) {  // any left (small U)
+      r = issue(u);
+      if (r.bad()) return r;
+    }
+  }
+  // the host store now holds u^T; nothing is resident. Every slot's and
+  // every tile's host events mark the end of this run for later schedules.
+  r = X.record(d, ev_phase(d), cs);
+  if (r.bad()) return r;
+  r = X.wait(d, ev_phase(d), os);
+  if (r.bad()) return r;
+  for (int s = 0; s < d.nslots; ++s) {
+    r = X.record(d, ev_slot(d, s), os);
+    if (r.bad()) return r;
+  }
+  for (int64_t t = 0; t < G.ntiles; ++t) {
+    r = X.record(d, ev_host(d, t), os);
+    if (r.bad()) return r;
+    d.tile_slot[t] = -1;
+    d.tile_dirty[t] = 0;
+  }
+  d.free_slots.clear();
+  for (int s = 0; s < d.nslots; ++s) {
+    d.slot_owner[s] = -1;
+    d.free_slots.push_back(s);
+  }
+  d.faces_valid = false;
+  d.host_faces_valid = false;
+  d.host_pending = true;
+  return Status::ok();
+}
+
 static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool serial) {
   const bool load = !d.resident_valid;
   const int64_t nL = d.G.n[2];
@@ -879,6 +1076,11 @@ static Status run_stream(Domain& d, const tile_kernel& k, int T, int S) {
   const bool multi = G.nranks > 1;
   Status r;
 
+  if (d.host_pending) {  // host store still being written by an earlier run
+    r = X.sync_all(d);
+    if (r.bad()) return r;
+    d.host_pending = false;
+  }
   if (heat && !d.faces_valid) {
     if (!d.host_faces_valid) {
       host_extract_faces(G, d.host, d.host_faces);
@@ -1072,8 +1274,13 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
       for (int64_t L = 0; L < d.G.n[2]; ++L) d.last_batches.push_back({L, L + 1, -1, -1, -1});
     }
   } else {
-    r = run_stream(d, k, steps, S);
-    if (k.kind != TILE_KERNEL_HEAT7 && steps > 0) d.faces_valid = false;
+    OocPlan op;
+    if (k.kind == TILE_KERNEL_HEAT7 && !serial && ooc_streamthrough_ok(d, steps, &op)) {
+      r = run_streamthrough_ooc(d, steps, S, op);
+    } else {
+      r = run_stream(d, k, steps, S);
+      if (k.kind != TILE_KERNEL_HEAT7 && steps > 0) d.faces_valid = false;
+    }
   }
   if (r.bad()) return r;
   if (k.kind == TILE_KERNEL_HEAT7) d.stats.steps_done += (uint64_t)steps;
@@ -1128,6 +1335,7 @@ Status domain_sync(Domain& d) {
   r = X.sync_all(d);
   if (r.bad()) return r;
   d.in_flight = false;
+  d.host_pending = false;
   d.host_faces_valid = false;  // host store changed
   return Status::ok();
 }

@@ -88,11 +88,16 @@ struct Domain;
 //              local z = zbase (wrapped);
 //   SUB      - the unit's packed sub-tiles at slot `slot`; slab plane lo of
 //              the sweep is sub-tile plane 0.
+//   UNITS    - (source only) units u-1, u, u+1 of `un` planes each as packed
+//              sub-tiles at slots ring[0..2]; slab plane 0 at local z = zbase
+//              (wrapped), z in unit z / un.
 struct SlabRef {
-  enum Kind { DENSE = 0, RESIDENT = 1, SUB = 2 };
+  enum Kind { DENSE = 0, RESIDENT = 1, SUB = 2, UNITS = 3 };
   int kind;
   int slot;
   int64_t zbase;
+  int ring[3];
+  int64_t u, un;
 };
 
 struct Exec {
@@ -119,6 +124,9 @@ struct Exec {
                           int64_t np, int stream) = 0;
   virtual Status copy_part(Domain& d, int packed_slot, int slot0, int64_t n, int64_t p0, int64_t np,
                            int stream) = 0;
+  // host tiles' planes [p0, p0+np) -> packed sub-tiles at a slot
+  virtual Status h2d_pack(Domain& d, int64_t tile0, int64_t n, int packed_slot, int64_t p0, int64_t np,
+                          int stream) = 0;
   // two-step pass (temporal blocking): same arguments as heat
   virtual Status heat2(Domain& d, const int64_t* tiles, const int* in_slots, const int* out_slots,
                        int nitems, int read_parity, const TileItem* dev_items, int stream) = 0;
@@ -226,6 +234,7 @@ struct Domain {
   std::vector<tile_op> trace;
   Exec* exec = nullptr;
   bool in_flight = false;
+  bool host_pending = false;               // async D2H into the host store in flight (ooc stream-through)
   double run_t0 = 0;
   bool kernel_timing = false;
 

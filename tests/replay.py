@@ -277,6 +277,35 @@ class Replayer:
                 for i in range(G.n[0] * G.n[1]):
                     ix, iy = i % G.n[0], i // G.n[0]
                     self.sub[(-b - 1, i)] = new[lo:hi, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx].copy()
+        elif name == "sweep_u":
+            # source: units u-1, u, u+1 as packed sub-tiles (slots in b);
+            # a: destination code as for "sweep"
+            lo, hi = c & 0xffffffff, c >> 32
+            u, un = d & 0xffffffff, d >> 32
+            slots = (b & 0x1fffff, (b >> 21) & 0x1fffff, b >> 42)
+            G = self.G
+            tx, ty, tz = G.t
+            nz, U = G.l[2], G.l[2] // un
+            k = (hi + 1 - un) // 2
+            src = np.empty((hi + 1, G.l[1], G.l[0]))
+            for p in range(hi + 1):
+                gz = (u * un - k + p) % nz
+                iu = gz // un
+                slot = slots[(iu - u + 1) % U if U > 2 else (0 if iu != u else 1)]
+                for i in range(G.n[0] * G.n[1]):
+                    ix, iy = i % G.n[0], i // G.n[0]
+                    src[p, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx] = self.sub[(slot, i)][gz - iu * un]
+            if a >= 0:
+                self.slabs[a] = self.sweep(src, self.slabs.get(a), lo, hi)
+            else:
+                new = self.sweep(src, None, lo, hi)
+                for i in range(G.n[0] * G.n[1]):
+                    ix, iy = i % G.n[0], i // G.n[0]
+                    self.sub[(-a - 1, i)] = new[lo:hi, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx].copy()
+        elif name == "h2d_pack":
+            p0, np_ = d & 0xffffffff, d >> 32
+            for i in range(c):
+                self.sub[(b, i)] = self.host[a + i][p0:p0 + np_].copy()
         elif name in ("h2d_part", "d2h_part", "copy_part"):
             p0, np_ = d & 0xffffffff, d >> 32
             for i in range(c):

@@ -138,6 +138,32 @@ def test_out_of_core_capped_bit_exact(nslots, ns):
     assert st["misses"] > 0 and st["writebacks"] > 0
 
 
+@pytest.mark.parametrize("dims,td,nslots,runs", [((64, 64, 256), (32, 32, 32), 30, [5, 3]),
+                                                 ((64, 64, 256), (32, 32, 32), 30, [13]),
+                                                 ((64, 32, 192), (32, 32, 16), 20, [40]),
+                                                 ((128, 64, 128), (64, 64, 8), 40, [6, 1, 2])])
+def test_out_of_core_stream_through_bit_exact(dims, td, nslots, runs):
+    """Out-of-core heat with temporal blocking: passes of k steps over units
+    of planes (ring of input units, fused first/last sweeps), one H2D and one
+    D2H per cell per pass; bit-identical to the oracle; a following per-step
+    run (stream_through off) continues from the host data."""
+    b = _budget(dims, td, nslots)
+    out, ref, info, st = _heat(dims, td, sum(runs), ns=3, sched="stream", device_budget_bytes=b, runs=runs)
+    assert info["sched"] == T.TILE_SCHED_STREAM and info["nslots"] == nslots
+    assert np.array_equal(out, ref)
+    cells = dims[0] * dims[1] * dims[2]
+    assert st["bytes_h2d"] < sum(runs) * cells * 8   # fewer link passes than steps
+    nx, ny, nz = dims
+    u0 = synth.uniform_grid(nx, ny, nz, 42)
+    with T.Domain(dims, td, sched="stream", device_budget_bytes=b) as d:
+        d.load(u0)
+        d.run(T.heat7(ALPHA), 4, 2)                       # stream-through pass(es)
+        d.run(T.heat7(ALPHA), 1, 2)                       # per-step (T = 1)
+        d.run(T.sincos(2), 1, 2)                          # pointwise after it
+        out2 = d.store()
+    assert np.allclose(out2, oracle.sincos_c(oracle.heat_c(u0, ALPHA, 5), 2, 1), rtol=1e-12, atol=0)
+
+
 def test_out_of_core_dirichlet():
     dims, td = (64, 32, 32), (32, 16, 16)
     b = _budget(dims, td, 4, bc="dirichlet")

@@ -302,3 +302,26 @@ def test_stream_through_schedule_replays_to_oracle(dims, td, T, ns):
     assert d.get_info()["resident"]
     # then a resident continuation and a second stream-through
     _run_and_replay(dims, td, [T, T], ns, seeds=(3,))
+
+
+@pytest.mark.parametrize("dims,td,nslots,runs,ns", [
+    ((16, 16, 128), (8, 8, 32), 30, [5], 2),          # one pass, units of 16 planes
+    ((16, 16, 128), (8, 8, 32), 30, [12, 3], 3),      # two runs
+    ((16, 8, 96), (8, 4, 16), 46, [40], 2),           # several passes (k <= tz = 16)
+    ((8, 8, 64), (8, 8, 8), 14, [7, 2], 1),           # units = tile layers, U = 8
+    ((8, 8, 48), (8, 8, 8), 12, [5], 2),              # U = 6, ring of 3
+])
+def test_ooc_stream_through_replays_to_oracle(dims, td, nslots, runs, ns):
+    """Out-of-core heat runs with a budget below the resident footprint take
+    the temporally blocked stream-through (passes of k >= 2 steps over units
+    of planes with a ring of input units); replayed in random valid orders
+    they give the oracle bit-exactly, and each pass moves every cell across
+    the link once per direction."""
+    b = _budget_for(dims, td, nslots, sched="stream")
+    d = _run_and_replay(dims, td, runs, ns, seeds=(0, 1, 2), sched="stream", device_budget_bytes=b)
+    ops = [op[0] for op in d.trace()]
+    assert "sweep_u" in ops and "h2d_pack" in ops, sorted(set(ops))
+    cells = dims[0] * dims[1] * dims[2]
+    st = d.stats()
+    assert st["bytes_h2d"] % (cells * 8) == 0 and st["bytes_h2d"] == st["bytes_d2h"]
+    assert st["bytes_h2d"] // (cells * 8) < sum(runs)  # fewer link passes than steps
