@@ -90,7 +90,7 @@ if __name__ == "__main__":
             traffic = (g("dram__bytes_read.sum") + g("dram__bytes_write.sum")) * scale
             print(d["kernel"][:80], "dur", g("gpu__time_duration.sum"), d["gpu__time_duration.sum"]["unit"],
                   "dram R+W bytes", traffic, "dram%", g("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed"))
-            if "heat7" in d["kernel"]:
+            if "heat7_fixed" in d["kernel"]:
                 tp = os.path.join(ROOT, "profiles", "heat7_ncu_traffic.json")
                 j = json.load(open(tp)) if os.path.exists(tp) else {}
                 j["c2"] = traffic
