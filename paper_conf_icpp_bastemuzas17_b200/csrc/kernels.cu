@@ -457,8 +457,53 @@ cudaError_t launch_heat7(const HeatParams& p, int stages, size_t smem, int grid,
 
 // -------------------------------------------------------------- sincos_iter
 // Listing P:L219-L224: per cell, `iters` times: s=sin(x); c=cos(x);
-// x = x + sqrt(s*s + c*c). sincos() shares the argument reduction of sin and
-// cos; each thread carries two independent cells (ILP). No FMA contraction.
+// x = x + sqrt(s*s + c*c). Each thread carries two independent cells (ILP);
+// the listing's own operations are rounded one by one (no contraction).
+// sin(x)^2 + cos(x)^2 as the listing evaluates it (s*s + c*c, each product
+// and the sum rounded, no contraction). With x = q*pi/2 + r (|r| <= pi/4),
+// sin x and cos x are +-sin r and +-cos r, swapped when q is odd; the sum of
+// the rounded squares does not depend on signs or order, so the quadrant is
+// never needed. sin r, cos r: fdlibm's minimax polynomials (max 1 ulp /
+// 2 ulp, checked against glibc over 2e7 points), r by a two-constant FMA
+// Cody-Waite reduction (exact to ~1 ulp of r for |q| < 2^20). The fast loop
+// runs while |x| <= 1e6 is guaranteed for all iterations (x grows by at most
+// ~1 per iteration); otherwise libdevice's sincos (Payne-Hanek) is used.
+// Polynomial and reduction constants live in constant memory so the DFMAs
+// take them as c[][] operands (64-bit immediates would cost two uniform
+// moves per use per iteration). TILES_SINCOS_LIBDEVICE=1: libdevice only.
+#ifndef TILES_SINCOS_LIBDEVICE
+#define TILES_SINCOS_LIBDEVICE 0
+#endif
+__constant__ double kSC[16] = {
+    6.36619772367581382433e-01,   // 0: 2/pi
+    1.5707963267948966,           // 1: pi/2 high
+    6.123233995736766e-17,        // 2: pi/2 - high
+    1.58969099521155010221e-10,   // 3..8: sin S6..S1
+    -2.50507602534068634195e-08, 2.75573137070700676789e-06, -1.98412698298579493134e-04,
+    8.33333333332248946124e-03, -1.66666666666666324348e-01,
+    -1.13596475577881948265e-11,  // 9..14: cos C6..C1
+    2.08757232129817482790e-09, -2.75573143513906633035e-07, 2.48015872894767294178e-05,
+    -1.38888888888741095749e-03, 4.16666666666666019037e-02,
+    0.0};
+
+static __device__ __forceinline__ double sin2_plus_cos2_fast(double x) {
+  const double q = rint(__dmul_rn(x, kSC[0]));
+  double r = fma(-q, kSC[1], x);
+  r = fma(-q, kSC[2], r);
+  const double z = __dmul_rn(r, r);
+  const double ps = fma(z, fma(z, fma(z, fma(z, kSC[3], kSC[4]), kSC[5]), kSC[6]), kSC[7]);
+  const double s = fma(__dmul_rn(r, z), fma(z, ps, kSC[8]), r);
+  const double pc = fma(z, fma(z, fma(z, fma(z, fma(z, kSC[9], kSC[10]), kSC[11]), kSC[12]), kSC[13]), kSC[14]);
+  const double c = fma(z, fma(z, pc, -0.5), 1.0);
+  return __dadd_rn(__dmul_rn(s, s), __dmul_rn(c, c));
+}
+
+static __device__ __forceinline__ double sin2_plus_cos2_libdevice(double x) {
+  double s, c;
+  sincos(x, &s, &c);
+  return __dadd_rn(__dmul_rn(s, s), __dmul_rn(c, c));
+}
+
 __global__ void __launch_bounds__(256) sincos_iter(const __grid_constant__ SincosParams p) {
   const int item_i = blockIdx.y;
   const TileItem it = p.items ? p.items[item_i] : p.inline_items[item_i];
@@ -469,12 +514,19 @@ __global__ void __launch_bounds__(256) sincos_iter(const __grid_constant__ Sinco
        j += (int64_t)gridDim.x * blockDim.x) {
     double2 v = src[j];
     double a = v.x, b = v.y;
-    for (int64_t k = 0; k < p.iters; ++k) {
-      double sa, ca, sb, cb;
-      sincos(a, &sa, &ca);
-      sincos(b, &sb, &cb);
-      a = __dadd_rn(a, __dsqrt_rn(__dadd_rn(__dmul_rn(sa, sa), __dmul_rn(ca, ca))));
-      b = __dadd_rn(b, __dsqrt_rn(__dadd_rn(__dmul_rn(sb, sb), __dmul_rn(cb, cb))));
+    const double lim = 1.0e6 - 2.0 * (double)p.iters;  // fast path valid for every iteration
+    if (!TILES_SINCOS_LIBDEVICE && fabs(a) <= lim && fabs(b) <= lim) {
+      for (int64_t k = 0; k < p.iters; ++k) {
+        const double ta = sin2_plus_cos2_fast(a), tb = sin2_plus_cos2_fast(b);
+        a = __dadd_rn(a, __dsqrt_rn(ta));
+        b = __dadd_rn(b, __dsqrt_rn(tb));
+      }
+    } else {
+      for (int64_t k = 0; k < p.iters; ++k) {
+        const double ta = sin2_plus_cos2_libdevice(a), tb = sin2_plus_cos2_libdevice(b);
+        a = __dadd_rn(a, __dsqrt_rn(ta));
+        b = __dadd_rn(b, __dsqrt_rn(tb));
+      }
     }
     data[j] = make_double2(a, b);
   }
