@@ -419,7 +419,8 @@ struct CudaExec final : Exec {
     if (d.x2_ok) {
       CK(heat2_configure((int)d.G.t[0], d.band2, d.heat2_smem, &heat2_occ));
       if (heat2_occ < 1) {  // cannot be resident (e.g. profiler-reserved shared memory)
-        std::fprintf(stderr, "libtiles: two-step kernel not resident on an SM; using single steps\n");
+        std::fprintf(stderr, "libtiles: two-step kernel (band %d, %zu B shared) not resident on an SM; "
+                     "using single steps\n", d.band2, d.heat2_smem);
         d.x2_ok = false;
       }
       for (int p = 0; p < 2 && d.x2_ok; ++p)

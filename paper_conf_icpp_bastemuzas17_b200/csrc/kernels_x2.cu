@@ -383,24 +383,272 @@ __global__ void __launch_bounds__(X2<TX, BY, S, MB>::NT + 32) heat7x2(const __gr
       }
 #endif
 
+// ---- heat7x2r: the same two-step pass with a row-owning thread layout
+// (TX = 64: one warp spans the tile width, lane l owns the x-pair 2l). 16
+// "row warps" own RW = BY/16 consecutive band rows each and keep their mid
+// values u^{s+1} of planes m-2, m-1, m in registers, so the second step reads
+// shared memory only for the two neighbour rows and, on the edge lanes, the
+// x ring; x neighbours come by warp shuffle. A "ring warp" computes the mid
+// halo rows (y0-1, y0+BY) and the x-ring columns (x = -1, TX) of each plane.
+// One named barrier per plane; mid planes in a ring of 3 shared buffers
+// (a buffer is rewritten two barriers after its last read). Same stage
+// layout, producer and rounded operations as heat7x2.
+template <int BY, int S>
+struct X2R {
+  static constexpr int TX = 64;
+  using L = X2<TX, BY, S, 2>;
+  static constexpr int RW = BY / 16;          // band rows per row warp
+  static constexpr int NT = 17 * 32;          // 16 row warps + ring warp
+  static constexpr size_t SMEM = (size_t)S * L::STAGE_ELEMS * 8 + 3 * (size_t)L::MID_ELEMS * 8 + 2 * S * 8;
+  static_assert(BY % 16 == 0 && RW >= 1 && RW <= 4, "bad x2r band");
+};
+
+template <int BY, int S>
+__global__ void __launch_bounds__(X2R<BY, S>::NT + 32) heat7x2r(const __grid_constant__ Heat2Params P) {
+  using R = X2R<BY, S>;
+  using C = typename R::L;
+  constexpr int TX = 64, RW = R::RW;
+  const HeatParams& p = P.h;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double* stage_base = reinterpret_cast<double*>(smem_raw);
+  double* mid0 = stage_base + (size_t)S * C::STAGE_ELEMS;
+  uint64_t* full = reinterpret_cast<uint64_t*>(mid0 + 3 * C::MID_ELEMS);
+  uint64_t* empty = full + S;
+  constexpr int NCW = R::NT / 32;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], TILES_ARRIVE_PER_THREAD ? 32 : 1);
+      mbar_init(&empty[s], TILES_ARRIVE_PER_THREAD ? NCW * 32 : NCW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  const int ty = p.ty, tz = p.tz;
+  const int64_t P_all = (int64_t)p.nitems * p.nbands * tz;
+  const int64_t pb = P_all * blockIdx.x / gridDim.x, pe = P_all * (blockIdx.x + 1) / gridDim.x;
+  const int lane = (int)threadIdx.x & 31, warp = (int)threadIdx.x >> 5;
+
+  if (warp == 17) {  // ---------------------------------------- producer warp
+    uint32_t g = 0;
+    for (int64_t pp = pb; pp < pe;) {
+      const int64_t col = pp / tz;
+      const int z0 = (int)(pp - col * tz);
+      const int z1 = (int)(pe - pp < (int64_t)(tz - z0) ? z0 + (pe - pp) : tz);
+      const int item_i = (int)(col / p.nbands);
+      const int y0 = (int)(col - (int64_t)item_i * p.nbands) * BY;
+      const TileItem it = p.items ? p.items[item_i] : p.inline_items[item_i];
+      const double* const* gs = p.gsrc + (size_t)it.tile * 6;
+      const EdgePtr* es = P.esrc + (size_t)it.tile * 12;
+      for (int z = z0 - 2; z <= z1 + 1; ++z, ++g) {
+        const int s = (int)(g % S);
+        mbar_wait(&empty[s], ((g / S) & 1u) ^ 1u);
+        stage_x2<TX, BY, S>(stage_base + (size_t)s * C::STAGE_ELEMS, &full[s], it.in, gs, es, z, ty, tz, y0,
+                            lane);
+      }
+      pp += z1 - z0;
+    }
+    return;
+  }
+
+  // ---------------------------------------------------------- consumers
+  const bool ring = warp == 16;
+  const int x = 2 * lane;
+  const int rb = RW * warp;  // first band row of a row warp
+  const double alpha = p.alpha;
+  const uint64_t keep = (p.cache_flags & 2) ? policy_evict_last() : policy_evict_normal();
+  auto cbar = [] { asm volatile("bar.sync 1, %0;" ::"n"(R::NT) : "memory"); };
+  auto wait_g = [&](uint32_t g) { mbar_wait(&full[g % S], (g / S) & 1u); };
+  auto release_g = [&](uint32_t g) {
+    if (TILES_ARRIVE_PER_THREAD) {
+      mbar_arrive(&empty[g % S]);
+    } else {
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[g % S]);
+    }
+  };
+  auto row2 = [&](const double* st, int r) {  // band row r (y = y0 + r) of a stage, at x
+    return *reinterpret_cast<const double2*>(st + (r + 2) * TX + x);
+  };
+  auto mid2 = [&](const double* mb, int r) -> double2& {
+    return *reinterpret_cast<double2*>(const_cast<double*>(mb) + (r + 1) * C::MPITCH + x + 2);
+  };
+  uint32_t seq = 0, gm = 0;  // input stage and mid plane counters (across columns)
+
+  for (int64_t pp = pb; pp < pe;) {
+    const int64_t col = pp / tz;
+    const int z0 = (int)(pp - col * tz);
+    const int z1 = (int)(pe - pp < (int64_t)(tz - z0) ? z0 + (pe - pp) : tz);
+    const int item_i = (int)(col / p.nbands);
+    const int y0 = (int)(col - (int64_t)item_i * p.nbands) * BY;
+    const TileItem it = p.items ? p.items[item_i] : p.inline_items[item_i];
+    const int64_t tile = it.tile;
+    const uint8_t fm = P.fixed_mask[tile];
+    const int nq = z1 - z0 + 4;    // input planes z0-2 .. z1+1
+    const int nmid = z1 - z0 + 2;  // mid planes z0-1 .. z1
+    auto stage = [&](int q) { return stage_base + (size_t)((seq + q) % S) * C::STAGE_ELEMS; };
+    auto midb = [&](uint32_t k) { return mid0 + (size_t)(k % 3) * C::MID_ELEMS; };
+
+    double* fxm = p.fexp[XM] + tile * p.face_elems[XM];
+    double* fxp = p.fexp[XP] + tile * p.face_elems[XP];
+    double* fym = p.fexp[YM] + tile * p.face_elems[YM] + x;
+    double* fyp = p.fexp[YP] + tile * p.face_elems[YP] + x;
+    double* fzm = p.fexp[ZM] + tile * p.face_elems[ZM] + x;
+    double* fzp = p.fexp[ZP] + tile * p.face_elems[ZP] + x;
+    double* obase = it.out + (size_t)(y0 + rb) * TX + x;
+    const size_t plane_elems = (size_t)ty * TX;
+
+    double2 mp[RW], mc[RW], mn[RW];  // mid(m-2), mid(m-1), mid(m) at own rows
+    wait_g(seq);
+    wait_g(seq + 1);
+    for (int mi = 0; mi < nmid; ++mi) {
+      const int m = z0 - 1 + mi;
+      wait_g(seq + mi + 2);
+      const double* prv = stage(mi);
+      const double* cur = stage(mi + 1);
+      const double* nxt = stage(mi + 2);
+      double* mb = midb(gm + mi);
+      const bool zring = m < 0 || m >= tz;
+      if (!ring) {
+        // ---- u^{s+1} of plane m at the warp's own rows
+        const bool zfixed = zring && (fm & bit(m < 0 ? ZM : ZP));
+        double2 c[RW];
+#pragma unroll
+        for (int j = 0; j < RW; ++j) c[j] = row2(cur, rb + j);
+        const double2 hm = row2(cur, rb - 1), hp = row2(cur, rb + RW);
+#pragma unroll
+        for (int j = 0; j < RW; ++j) {
+          if (zfixed) {
+            mn[j] = c[j];
+          } else {
+            const int rr = rb + j + 2;  // staged row index
+            double xm = __shfl_up_sync(0xffffffffu, c[j].y, 1);
+            double xp = __shfl_down_sync(0xffffffffu, c[j].x, 1);
+            if (lane == 0) xm = cur[C::XOFF + rr * 2 + 1];
+            if (lane == 31) xp = cur[C::XOFF + 2 * C::IROWS + rr * 2];
+            const double2 ym = j == 0 ? hm : c[j > 0 ? j - 1 : 0];
+            const double2 yp = j == RW - 1 ? hp : c[j < RW - 1 ? j + 1 : 0];
+            const double2 zm = row2(prv, rb + j), zp = row2(nxt, rb + j);
+            mn[j].x = heat_update(c[j].x, xm, c[j].y, ym.x, yp.x, zm.x, zp.x, alpha);
+            mn[j].y = heat_update(c[j].y, c[j].x, xp, ym.y, yp.y, zm.y, zp.y, alpha);
+          }
+          mid2(mb, rb + j) = mn[j];
+        }
+      } else if (!zring) {
+        // ---- ring warp: mid halo rows y0-1, y0+BY (x-pairs) ...
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int r = h ? BY : -1, y = y0 + r;
+          const bool yout = y < 0 || y >= ty;
+          const double2 c = row2(cur, r);
+          double2 v;
+          double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+          double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+          if (yout && (fm & bit(y < 0 ? YM : YP))) {
+            v = c;  // Dirichlet: the ring keeps its fixed value
+          } else {
+            const int rr = r + 2;
+            if (lane == 0) xm = cur[C::XOFF + rr * 2 + 1];
+            if (lane == 31) xp = cur[C::XOFF + 2 * C::IROWS + rr * 2];
+            const double2 ym = row2(cur, r - 1), yp = row2(cur, r + 1);
+            const double2 zm = row2(prv, r), zp = row2(nxt, r);
+            v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm.x, zp.x, alpha);
+            v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm.y, zp.y, alpha);
+          }
+          mid2(mb, r) = v;
+        }
+        // ... and the x-ring columns x = -1, TX of the band rows
+        for (int e = lane; e < 2 * BY; e += 32) {
+          const int side = e / BY;
+          const int y = y0 + e % BY;
+          const int rr = y - (y0 - 2);
+          const double* xb = cur + C::XOFF + side * 2 * C::IROWS + rr * 2;
+          const int own = side ? 0 : 1, far = side ? 1 : 0;
+          double v;
+          if (fm & bit(side ? XP : XM)) {
+            v = xb[own];
+          } else {
+            const double inner = cur[rr * TX + (side ? TX - 1 : 0)];
+            const double xm = side ? inner : xb[far], xp = side ? xb[far] : inner;
+            v = heat_update(xb[own], xm, xp, xb[own - 2], xb[own + 2],
+                            prv[C::XOFF + side * 2 * C::IROWS + rr * 2 + own],
+                            nxt[C::XOFF + side * 2 * C::IROWS + rr * 2 + own], alpha);
+          }
+          mb[(y - y0 + 1) * C::MPITCH + (side ? TX + 2 : 1)] = v;
+        }
+      }
+      cbar();  // mid(m) complete; input plane m-1 no longer read
+      release_g(seq + mi);
+      if (!ring && mi >= 2) {
+        // ---- u^{s+2} of plane o = m-1 at the own rows
+        const int o = m - 1;
+        const double* cb = midb(gm + mi - 1);  // mid(o): neighbour rows, x ring
+        const double2 hm = mid2(cb, rb - 1), hp = mid2(cb, rb + RW);
+        double* op = obase + (size_t)o * plane_elems;
+        const bool zlo = o < 2, zhi = o >= tz - 2;
+#pragma unroll
+        for (int j = 0; j < RW; ++j) {
+          const double2 c = mc[j];
+          double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+          double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+          if (lane == 0) xm = cb[(rb + j + 1) * C::MPITCH + 1];
+          if (lane == 31) xp = cb[(rb + j + 1) * C::MPITCH + TX + 2];
+          const double2 ym = j == 0 ? hm : mc[j > 0 ? j - 1 : 0];
+          const double2 yp = j == RW - 1 ? hp : mc[j < RW - 1 ? j + 1 : 0];
+          double2 v;
+          v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, mp[j].x, mn[j].x, alpha);
+          v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, mp[j].y, mn[j].y, alpha);
+          stg2_stream(op + (size_t)j * TX, v);
+          const int y = y0 + rb + j;
+          if (lane == 0) st2_hint(fxm + ((size_t)o * ty + y) * 2, v, keep);
+          if (lane == 31) st2_hint(fxp + ((size_t)o * ty + y) * 2, v, keep);
+          if (y < 2) st2_hint(fym + ((size_t)o * 2 + y) * TX, v, keep);
+          if (y >= ty - 2) st2_hint(fyp + ((size_t)o * 2 + y - (ty - 2)) * TX, v, keep);
+          if (zlo) st2_hint(fzm + ((size_t)o * ty + y) * TX, v, keep);
+          if (zhi) st2_hint(fzp + ((size_t)(o - (tz - 2)) * ty + y) * TX, v, keep);
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < RW; ++j) {
+        mp[j] = mc[j];
+        mc[j] = mn[j];
+      }
+    }
+    release_g(seq + nq - 2);
+    release_g(seq + nq - 1);
+    seq += (uint32_t)nq;
+    gm += (uint32_t)nmid;
+    pp += z1 - z0;
+  }
+}
+
 struct X2Entry {
-  int tx, by, stages, mb;
+  int tx, by, stages, mb, rows;  // rows = 1: heat7x2r (row-owning layout)
   void (*fn)(Heat2Params);
   int nt;
   size_t smem;
 };
 #define X2E(TX, BY, S, MB) \
-  {TX, BY, S, MB, heat7x2<TX, BY, S, MB>, X2<TX, BY, S, MB>::NT + 32, X2<TX, BY, S, MB>::SMEM}
-static const X2Entry kX2[] = {X2E(64, 64, 4, 2), X2E(64, 32, 5, 3), X2E(64, 32, 4, 3),
+  {TX, BY, S, MB, 0, heat7x2<TX, BY, S, MB>, X2<TX, BY, S, MB>::NT + 32, X2<TX, BY, S, MB>::SMEM}
+#define X2RE(BY, S) {64, BY, S, 3, 1, heat7x2r<BY, S>, X2R<BY, S>::NT + 32, X2R<BY, S>::SMEM}
+// x2r at band 32 / 6 stages: 0.788 ms per C2 pass vs 0.803 for heat7x2<64,64,4,2>
+// (band 64 x2r: 0.997 ms — 18 warps cap it at 96 registers, and it cannot be
+// resident under ncu), profiles/r01/x2_profile/
+static const X2Entry kX2[] = {X2RE(32, 6),
+                              X2E(64, 64, 4, 2), X2E(64, 32, 5, 3), X2E(64, 32, 4, 3),
                               X2E(64, 32, 6, 2), X2E(32, 32, 6, 3), X2E(32, 16, 6, 3),
                               X2E(128, 16, 4, 3), X2E(256, 8, 4, 3)};
 #undef X2E
+#undef X2RE
 
 static const X2Entry* find_x2(int tx, int by, int st = 0) {
   if (!st)
     if (const char* es = std::getenv("TILES_X2_STAGES")) st = std::atoi(es);  // tuning override
+  static const int rows = [] {  // TILES_X2_ROWS=0: the original thread layout only
+    const char* e = std::getenv("TILES_X2_ROWS");
+    return e ? std::atoi(e) : 1;
+  }();
   for (const auto& e : kX2)
-    if (e.tx == tx && e.by == by && (!st || e.stages == st)) return &e;
+    if (e.tx == tx && e.by == by && (!st || e.stages == st) && (rows || !e.rows)) return &e;
   return nullptr;
 }
 
@@ -414,7 +662,7 @@ bool heat2_plan(int tx, int ty, int max_smem, int* band, size_t* smem) {
       return true;
     }
   }
-  for (int by : {64, 32, 16, 8}) {
+  for (int by : {32, 64, 16, 8}) {  // band 32 first: x2r (see kX2)
     if (ty % by) continue;
     const X2Entry* e = find_x2(tx, by);
     if (e && e->smem <= (size_t)max_smem) {
@@ -431,7 +679,15 @@ cudaError_t heat2_configure(int tx, int band, size_t smem, int* ctas_per_sm) {
   if (!e || e->smem != smem) return cudaErrorInvalidValue;
   cudaError_t r = cudaFuncSetAttribute(e->fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (r != cudaSuccess) return r;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, e->fn, e->nt, smem);
+  r = cudaOccupancyMaxActiveBlocksPerMultiprocessor(ctas_per_sm, e->fn, e->nt, smem);
+  if (r == cudaSuccess && *ctas_per_sm < 1) {
+    cudaFuncAttributes fa{};
+    cudaFuncGetAttributes(&fa, e->fn);
+    std::fprintf(stderr, "libtiles: heat7x2 entry (tx %d, band %d, %d threads): regs %d, static smem %zu, "
+                 "max threads %d, max dyn smem %d\n", tx, band, e->nt, fa.numRegs, fa.sharedSizeBytes,
+                 fa.maxThreadsPerBlock, fa.maxDynamicSharedSizeBytes);
+  }
+  return r;
 }
 
 cudaError_t launch_heat7x2(const Heat2Params& p, size_t smem, int grid, cudaStream_t s) {

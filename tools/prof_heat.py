@@ -7,7 +7,8 @@ import synth
 from paper_conf_icpp_bastemuzas17_b200 import tiles as T
 n = int(os.environ.get("N", "512")); t = int(os.environ.get("TILE", "64"))
 u = np.empty((n, n, n)); synth.fill_uniform_native(u.ctypes.data, n, n, n, 0, n, 0, n, 0, n, 42)
-d = T.Domain((n, n, n), (t, t, t), ghost=int(os.environ.get("GHOST", "1")), stream_through=-1)
+d = T.Domain((n, n, n), (t, t, t), ghost=int(os.environ.get("GHOST", "1")), stream_through=-1,
+             two_step=int(os.environ.get("TWO_STEP", "0")))
 d.load(u); d.run(T.heat7(), 1, 4); d.sync()
 d.run(T.heat7(), int(os.environ.get("STEPS", "4")), 4); d.sync()
 print("prof ok")
