@@ -44,6 +44,12 @@ with T.Domain((64, 64, 256), (32, 32, 32)) as d:          # stream-through, unit
     d.load(us); d.run(T.heat7(), 10, 2); d.store()
 with T.Domain((128, 64, 64), (64, 64, 16), ghost=2, two_step=1) as d:   # heat7x2 (two steps per pass)
     d.load(synth.uniform_grid(128, 64, 64, 9)); d.run(T.heat7(), 6, 2); d.store()
+uo = synth.uniform_grid(64, 64, 256, 4)                   # out-of-core stream-through (unit ring)
+bo = budget((64, 64, 256), (32, 32, 32), 30)
+with T.Domain((64, 64, 256), (32, 32, 32), sched="stream", device_budget_bytes=bo) as d:
+    d.load(uo); d.run(T.heat7(), 5, 3); d.store()
+with T.Domain((128, 64, 64), (64, 64, 16), ghost=2, two_step=1) as d:   # heat7x2r (band 32)
+    d.load(synth.uniform_grid(128, 64, 64, 11)); d.run(T.heat7(), 4, 2); d.store()
 g = T.LocalGroup(2)
 def rank(r):
     with T.Domain((64, 32, 64), (32, 16, 16), nranks=2, rank=r, local_group=g) as d:
