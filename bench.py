@@ -41,11 +41,28 @@ ALPHA = 0.125
 METRIC = "Gcell-updates/s incl. H2D/D2H at 1/2/4/8 B200; % transfer time hidden"
 
 
+# Test hook: TILES_BENCH_ONE_GPU=1 runs every rank of a torchrun launch on
+# cuda:0 with a gloo process group (exercises the multi-rank bench path and
+# the peer transport on a one-GPU box; never used for reported numbers).
+ONE_GPU = os.environ.get("TILES_BENCH_ONE_GPU") == "1"
+
+
 def dist_env():
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rk = int(os.environ.get("RANK", "0"))
     lr = int(os.environ.get("LOCAL_RANK", str(rk)))
-    return ws, rk, lr
+    return ws, rk, (0 if ONE_GPU else lr)
+
+
+def init_dist(torch, dist, lr):
+    if ONE_GPU:
+        dist.init_process_group("gloo")
+    else:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", lr))
+
+
+def red_dev():
+    return "cpu" if ONE_GPU else "cuda"
 
 
 class Clocks:
@@ -543,6 +560,22 @@ def run_fig5_tiles_leg(args):
     return 0
 
 
+def multi_domain(Tl, dist, ws, rk, transport, *args, **kw):
+    """Domain for rank rk of ws. transport "peer": halo windows over CUDA IPC
+    (handles all-gathered through torch.distributed); "nccl": NCCL p2p."""
+    if ws == 1:
+        return Tl.Domain(*args, nranks=1, rank=0, **kw)
+    if transport == "peer":
+        dom = Tl.Domain(*args, nranks=ws, rank=rk, peer_transport=True, **kw)
+        hs = [None] * ws
+        dist.all_gather_object(hs, dom.peer_handle())
+        dom.peer_connect(hs)
+        return dom
+    obj = [Tl.nccl_unique_id() if rk == 0 else None]
+    dist.broadcast_object_list(obj, src=0)
+    return Tl.Domain(*args, nranks=ws, rank=rk, nccl_id=obj[0], **kw)
+
+
 def run_c5_leg(args):
     """C5: heat 4096^3 fp64 slab-decomposed over N GPUs (z-slabs, NCCL halo
     exchange), each rank streaming its own tiles from pinned host memory.
@@ -555,7 +588,7 @@ def run_c5_leg(args):
     ws, rk, lr = dist_env()
     torch.cuda.set_device(lr)
     if ws > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", lr))
+        init_dist(torch, dist, lr)
     n = args.n
     if not n:
         # SURVEY §8(d) fallback ladder: the largest n whose pinned host stores
@@ -570,7 +603,7 @@ def run_c5_leg(args):
                 n = cand
                 break
         if ws > 1:  # every rank must use the same grid
-            t = torch.tensor([n], dtype=torch.int64, device="cuda")
+            t = torch.tensor([n], dtype=torch.int64, device=red_dev())
             dist.all_reduce(t, op=dist.ReduceOp.MIN)
             n = int(t.item())
     nzl = n // 8 if ws == 1 else n // ws
@@ -579,11 +612,6 @@ def run_c5_leg(args):
     T = args.T if args.T is not None else 10
     ns = args.nstreams or 4
     cells = n * n * nzl
-    nid = None
-    if ws > 1:
-        obj = [Tl.nccl_unique_id() if rk == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        nid = obj[0]
 
     def barrier():
         if ws > 1:
@@ -593,12 +621,12 @@ def run_c5_leg(args):
     def mx(x):
         if ws == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        t = torch.tensor([x], dtype=torch.float64, device=red_dev())
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
     t0 = time.perf_counter()
-    dom = Tl.Domain(gdims, td, ghost=1, device=lr, nranks=ws, rank=rk, nccl_id=nid)
+    dom = multi_domain(Tl, dist, ws, rk, args.transport, gdims, td, ghost=1, device=lr)
     fill_tiles(dom, Tl, synth, gdims, td, rk * nzl, 42)
     t_setup = time.perf_counter() - t0
     k = Tl.heat7(ALPHA)
@@ -673,6 +701,8 @@ def main():
     ap.add_argument("--ghost", type=int, default=1,
                     help="c2/c3: ghost width; 2 = two Jacobi steps per pass (temporal blocking)")
     ap.add_argument("--two-step", type=int, default=0, help="tile_options.two_step (-1, 0, 1)")
+    ap.add_argument("--transport", default="peer", choices=["peer", "nccl"],
+                    help="N > 1 halo exchange: CUDA IPC windows (default) or NCCL p2p")
     ap.add_argument("--stream-through", type=int, default=0,
                     help="tile_options.stream_through (-1 never, 0 cost model, 1 when feasible)")
     args = ap.parse_args()
@@ -700,19 +730,13 @@ def main():
     ws, rk, lr = dist_env()
     torch.cuda.set_device(lr)
     if ws > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", lr))
+        init_dist(torch, dist, lr)
     dims, td, T, ns, desc = CONFIGS[args.config]
     T = args.T if args.T is not None else T
     ns = args.nstreams or ns
     nx, ny, nzl = dims
     gdims = (nx, ny, nzl * ws)
     cells = nx * ny * nzl  # per rank
-
-    nid = None
-    if ws > 1:
-        obj = [Tl.nccl_unique_id() if rk == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        nid = obj[0]
 
     def barrier():
         if ws > 1:
@@ -722,14 +746,14 @@ def main():
     def max_over_ranks(x):
         if ws == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        t = torch.tensor([x], dtype=torch.float64, device=red_dev())
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
     u0 = np.empty((nzl, ny, nx))
     synth.fill_uniform_native(u0.ctypes.data, gdims[0], gdims[1], gdims[2], rk * nzl, nzl, 0, ny, 0, nx, 42)
-    dom = Tl.Domain(gdims, td, ghost=args.ghost, device=lr, nranks=ws, rank=rk, nccl_id=nid,
-                    two_step=args.two_step)
+    dom = multi_domain(Tl, dist, ws, rk, args.transport, gdims, td, ghost=args.ghost, device=lr,
+                       two_step=args.two_step)
     dom.load(u0)
     del u0
     k = Tl.heat7(ALPHA)
@@ -860,7 +884,7 @@ def main():
                 "config": {"workload": desc, "dims_per_gpu": dims, "global_dims": gdims, "tile_dims": td,
                            "ghost": args.ghost, "steps_per_pass": spp, "T": T, "nstreams": ns,
                            "bc": "periodic", "alpha": ALPHA,
-                           "parallelism": f"z-slab x{ws}" if ws > 1 else "1 GPU",
+                           "parallelism": f"z-slab x{ws}, halo via {args.transport}" if ws > 1 else "1 GPU",
                            "l2": "inputs larger than L2 (2 x 1.07 GB per GPU per step)",
                            "value_def": "grid resident in HBM; T steps of tile_run",
                            "e2e_def": "tile_invalidate + tile_run(T) + tile_sync from pinned host"},

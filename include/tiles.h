@@ -126,6 +126,16 @@ typedef struct {
                                    streamthrough_ok) rates it faster than the
                                    batched resident schedule; 1 = whenever
                                    feasible; -1 = never. */
+  int32_t peer_transport;       /* nranks > 1: 1 = halo exchange by direct
+                                   device-to-device stores into the z-neighbour
+                                   ranks' memory (CUDA IPC; NVLink / NVSwitch
+                                   peer access), synchronised with stream
+                                   memory operations on counters in the
+                                   neighbours' memory — no NCCL. The caller
+                                   gathers every rank's tile_peer_handle and
+                                   passes them to tile_peer_connect before the
+                                   first run. 0 (default) = NCCL (or the
+                                   local_group transport). */
   int32_t two_step;             /* HEAT7 with ghost >= 2: 0 (default) = two
                                    steps per pass in the streaming schedule
                                    (halves host-link bytes per step), single
@@ -296,6 +306,17 @@ const char* tile_last_error(void);
 /* Fill out[128] with a fresh ncclUniqueId (call on rank 0, then broadcast).
  * TILE_ENOSYS if built without NCCL. */
 tile_status tile_nccl_unique_id(void* out128);
+
+/* Peer transport (tile_options.peer_transport = 1). tile_peer_handle writes
+ * the 64-byte CUDA IPC handle of this rank's halo window (receive buffers
+ * and exchange counters) to out64. tile_peer_connect takes every rank's
+ * handle, `nranks` blobs of 64 bytes in rank order (the caller all-gathers
+ * them, e.g. with torch.distributed), and maps the z-neighbours' windows;
+ * it must precede the first tile_run. ESTATE if the domain has no window
+ * (peer_transport off, single rank or dry run); ECUDA if a handle cannot be
+ * opened (no peer access between the devices). */
+tile_status tile_peer_handle(const tile_domain* dom, void* out64);
+tile_status tile_peer_connect(tile_domain* dom, const void* handles, int32_t nranks);
 
 /* In-process multi-rank transport for testing the slab path on ONE device:
  * every rank is a domain driven by its own host thread (ranks may share a

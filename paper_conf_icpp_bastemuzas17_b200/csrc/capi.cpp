@@ -229,4 +229,15 @@ tile_status tile_nccl_unique_id(void* out128) {
   return finish(nullptr, tiles::nccl_unique_id(out128));
 }
 
+tile_status tile_peer_handle(const tile_domain* h, void* out64) {
+  if (!h || !h->d || !out64) return fail(TILE_EINVAL, "null argument");
+  return finish(nullptr, tiles::peer_handle(*h->d, out64));
+}
+
+tile_status tile_peer_connect(tile_domain* h, const void* handles, int32_t nranks) {
+  CHECK_DOM(h);
+  if (!handles) return fail(TILE_EINVAL, "null handles");
+  return finish(h, tiles::peer_connect(*h->d, handles, nranks));
+}
+
 }  // extern "C"

@@ -1,0 +1,176 @@
+// comm_peer.cu — z-slab halo exchange by direct stores into the neighbour
+// ranks' device memory (CUDA IPC; over NVLink 5 / NVSwitch between the GPUs
+// of a node), without NCCL. Not in the paper (single GPU).
+//
+// Each rank owns a "window" (one cudaMalloc, exported with cudaIpcGetMemHandle):
+// its receive buffers halo[2][2] and four 32-bit counters. Exchange k (the
+// k-th halo op, identical on every rank: the op is collective) of parity p,
+// on the rank's halo stream, which is already ordered after the boundary
+// kernels that wrote the exported faces and after the previous readers of
+// halo[.][p]:
+//   1. ready:   write k into the upper neighbour's R_DN and the lower one's
+//               R_UP (my halo[.][p] may now be overwritten);
+//   2. wait:    my R_UP >= k and my R_DN >= k (my receivers are ready);
+//   3. push:    my top z-faces -> upper.halo[0][p], bottom -> lower.halo[1][p]
+//               (peer-to-peer copies);
+//   4. arrived: write k into upper.A_DN and lower.A_UP (after the copies:
+//               cuStreamWriteValue32 fences prior work of the stream);
+//   5. wait:    my A_DN >= k and my A_UP >= k, then the caller records the
+//               halo event its boundary kernels wait for.
+// This is the rendezvous an NCCL send/recv pair provides, without a proxy
+// thread or a staging copy. Counters are stream memory operations
+// (cuStreamWriteValue32 / cuStreamWaitValue32, fetched with
+// cudaGetDriverEntryPoint), so no kernel spins and no SM is held.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdio>
+#include <cstring>
+
+#include "runtime.hpp"
+
+namespace tiles {
+namespace {
+
+enum { R_DN = 0, R_UP = 1, A_DN = 2, A_UP = 3, NFLAGS = 8 };
+
+using WriteFn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+using WaitFn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+WriteFn g_write = nullptr;
+WaitFn g_wait = nullptr;
+
+Status load_memops() {
+  if (g_write && g_wait) return Status::ok();
+  void* w = nullptr;
+  void* v = nullptr;
+  cudaDriverEntryPointQueryResult q1{}, q2{};
+  if (cudaGetDriverEntryPoint("cuStreamWriteValue32", &w, cudaEnableDefault, &q1) != cudaSuccess ||
+      cudaGetDriverEntryPoint("cuStreamWaitValue32", &v, cudaEnableDefault, &q2) != cudaSuccess || !w || !v)
+    return make_err(TILE_ENOSYS, "cuStreamWriteValue32/cuStreamWaitValue32 not available");
+  g_write = reinterpret_cast<WriteFn>(w);
+  g_wait = reinterpret_cast<WaitFn>(v);
+  return Status::ok();
+}
+
+#define PK(call)                                                                         \
+  do {                                                                                   \
+    cudaError_t e_ = (call);                                                             \
+    if (e_ != cudaSuccess) return make_err(TILE_ECUDA, std::string(#call ": ") + cudaGetErrorString(e_)); \
+  } while (0)
+#define DK(call)                                                            \
+  do {                                                                      \
+    CUresult e_ = (call);                                                   \
+    if (e_ != CUDA_SUCCESS) return make_err(TILE_ECUDA, std::string(#call " failed")); \
+  } while (0)
+
+CUdeviceptr flag(void* window_flags, int i) {
+  return reinterpret_cast<CUdeviceptr>(static_cast<uint32_t*>(window_flags) + i);
+}
+
+}  // namespace
+
+// Window: [halo 0/1][parity 0/1] receive buffers, then the counters.
+Status peer_setup(Domain& d, uint64_t halo_bytes) {
+  Status s = load_memops();
+  if (s.bad()) return s;
+  const uint64_t bytes = 4 * halo_bytes + 256;
+  void* w = nullptr;
+  PK(cudaMalloc(&w, bytes));
+  PK(cudaMemset(w, 0, bytes));
+  PK(cudaDeviceSynchronize());
+  d.peer_window = w;
+  char* c = static_cast<char*>(w);
+  for (int a = 0; a < 2; ++a)
+    for (int p = 0; p < 2; ++p) d.halo[a][p] = reinterpret_cast<double*>(c + (2 * a + p) * halo_bytes);
+  d.peer_flags = c + 4 * halo_bytes;
+  d.peer_halo_bytes = halo_bytes;
+  int flush = 0, dev = 0;
+  PK(cudaGetDevice(&dev));
+  // CU_DEVICE_ATTRIBUTE_CAN_FLUSH_REMOTE_WRITES: needed to make the peers'
+  // copies visible to work after a satisfied wait
+  PK(cudaDeviceGetAttribute(&flush, cudaDevAttrCanFlushRemoteWrites, dev));
+  d.peer_wait_flags = CU_STREAM_WAIT_VALUE_GEQ | (flush ? CU_STREAM_WAIT_VALUE_FLUSH : 0);
+  return Status::ok();
+}
+
+Status peer_handle(const Domain& d, void* out64) {
+  if (!d.peer_window) return make_err(TILE_ESTATE, "no peer window (peer_transport off or dry run)");
+  cudaIpcMemHandle_t h;
+  PK(cudaIpcGetMemHandle(&h, d.peer_window));
+  static_assert(sizeof h == 64, "cudaIpcMemHandle_t is 64 bytes");
+  std::memcpy(out64, &h, sizeof h);
+  return Status::ok();
+}
+
+Status peer_connect(Domain& d, const void* handles, int n) {
+  const Geometry& G = d.G;
+  if (n != G.nranks) return make_err(TILE_EINVAL, "peer_connect: handle count != nranks");
+  if (!d.peer_window) return make_err(TILE_ESTATE, "no peer window (peer_transport off or dry run)");
+  const int r = G.rank, R = G.nranks;
+  const bool per = G.bc == TILE_BC_PERIODIC;
+  const int nb[2] = {(r - 1 + R) % R, (r + 1) % R};  // lower, upper
+  const bool has[2] = {per || r > 0, per || r < R - 1};
+  for (int s = 0; s < 2; ++s) {
+    d.peer_base[s] = nullptr;
+    if (!has[s]) continue;
+    const int q = nb[s];
+    if (q == r) return make_err(TILE_EINVAL, "peer_connect: a rank cannot be its own neighbour");
+    if (s == 1 && nb[1] == nb[0] && d.peer_base[0]) {  // G == 2: one peer for both sides
+      d.peer_base[1] = d.peer_base[0];
+      continue;
+    }
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, static_cast<const char*>(handles) + (size_t)q * 64, 64);
+    void* p = nullptr;
+    PK(cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess));
+    d.peer_base[s] = p;
+    d.peer_opened[s] = p;
+  }
+  d.peer_connected = true;
+  return Status::ok();
+}
+
+void peer_destroy(Domain& d) {
+  for (int s = 0; s < 2; ++s) {
+    if (d.peer_opened[s]) cudaIpcCloseMemHandle(d.peer_opened[s]);
+    d.peer_opened[s] = nullptr;
+    d.peer_base[s] = nullptr;
+  }
+  if (d.peer_window) cudaFree(d.peer_window);
+  d.peer_window = nullptr;
+}
+
+Status peer_halo(Domain& d, int par, void* stream_v) {
+  if (!d.peer_connected) return make_err(TILE_ESTATE, "peer transport: call tile_peer_connect first");
+  const Geometry& G = d.G;
+  CUstream st = static_cast<CUstream>(stream_v);
+  const uint32_t k = ++d.peer_k;
+  const uint64_t hb = d.peer_halo_bytes;
+  const size_t cnt = (size_t)G.layer_tiles * G.face_elems[ZM];
+  char* lo = static_cast<char*>(d.peer_base[0]);  // lower neighbour's window
+  char* up = static_cast<char*>(d.peer_base[1]);  // upper neighbour's window
+  void* lo_flags = lo ? lo + 4 * hb : nullptr;
+  void* up_flags = up ? up + 4 * hb : nullptr;
+  // 1. ready to receive exchange k
+  if (up) DK(g_write(st, flag(up_flags, R_DN), k, 0));
+  if (lo) DK(g_write(st, flag(lo_flags, R_UP), k, 0));
+  // 2. receivers ready
+  if (up) DK(g_wait(st, flag(d.peer_flags, R_UP), k, d.peer_wait_flags));
+  if (lo) DK(g_wait(st, flag(d.peer_flags, R_DN), k, d.peer_wait_flags));
+  // 3. push the boundary faces of parity par, 4. signal arrival
+  if (d.measure != TILE_MEASURE_COMP_ONLY) {
+    const double* top = d.faces[ZP][par] + (G.n[2] - 1) * G.layer_tiles * G.face_elems[ZP];
+    const double* bot = d.faces[ZM][par];
+    if (up) PK(cudaMemcpyAsync(up + (0 * 2 + par) * hb, top, cnt * 8, cudaMemcpyDeviceToDevice, (cudaStream_t)st));
+    if (lo) PK(cudaMemcpyAsync(lo + (1 * 2 + par) * hb, bot, cnt * 8, cudaMemcpyDeviceToDevice, (cudaStream_t)st));
+    d.stats.bytes_halo += (uint64_t)((up ? 1 : 0) + (lo ? 1 : 0)) * cnt * 8;
+  }
+  if (up) DK(g_write(st, flag(up_flags, A_DN), k, 0));
+  if (lo) DK(g_write(st, flag(lo_flags, A_UP), k, 0));
+  // 5. my ghosts have arrived
+  if (lo) DK(g_wait(st, flag(d.peer_flags, A_DN), k, d.peer_wait_flags));
+  if (up) DK(g_wait(st, flag(d.peer_flags, A_UP), k, d.peer_wait_flags));
+  return Status::ok();
+}
+
+}  // namespace tiles

@@ -344,7 +344,7 @@ struct CudaExec final : Exec {
       d.stats.n_halo++;
       return Status::ok();
     }
-    Status r = nccl_halo(d, par, S(st));
+    Status r = d.opt.peer_transport ? peer_halo(d, par, S(st)) : nccl_halo(d, par, S(st));
     if (r.bad()) return r;
     d.stats.n_halo++;
     return Status::ok();

@@ -72,8 +72,8 @@ Status domain_create(const int64_t dims[3], const int64_t tdims[3], int ghost,
   Geometry G;
   Status st = make_geometry(dims, tdims, ghost, opt.bc, opt.nranks, opt.rank, &G);
   if (st.bad()) return st;
-  if (G.nranks > 1 && !opt.nccl_unique_id && !opt.dry_run && !opt.local_group)
-    return make_err(TILE_EINVAL, "nranks > 1 needs nccl_unique_id or local_group");
+  if (G.nranks > 1 && !opt.nccl_unique_id && !opt.dry_run && !opt.local_group && !opt.peer_transport)
+    return make_err(TILE_EINVAL, "nranks > 1 needs nccl_unique_id, peer_transport or local_group");
 
   int band = 0, stages = 0;
   size_t smem = 0;
@@ -151,7 +151,8 @@ Status domain_setup(Domain& d) {
   uint64_t persist = 2 * face_bytes_all;  // export faces, 2 parities
   if (dir) persist += face_bytes_all;
   const uint64_t halo_bytes = align_up((uint64_t)G.layer_tiles * G.face_elems[ZM] * 8);
-  if (multi) persist += 4 * halo_bytes;
+  const bool peer = multi && d.opt.peer_transport && !d.opt.dry_run;  // halos live in the IPC window
+  if (multi && !peer) persist += 4 * halo_bytes;
   const uint64_t gsrc_bytes = align_up((uint64_t)G.ntiles * 6 * sizeof(double*));
   const uint64_t items_bytes = align_up((uint64_t)G.ntiles * sizeof(TileItem));
   persist += 2 * gsrc_bytes + 2 * items_bytes;
@@ -213,9 +214,13 @@ Status domain_setup(Domain& d) {
   if (dir)
     for (int f = 0; f < 6; ++f)
       d.dir_faces[f] = reinterpret_cast<double*>(carve((uint64_t)G.ntiles * G.face_elems[f] * 8));
-  if (multi)
+  if (multi && !peer)
     for (int a = 0; a < 2; ++a)
       for (int p = 0; p < 2; ++p) d.halo[a][p] = reinterpret_cast<double*>(carve(halo_bytes));
+  if (peer) {  // before the ghost-source tables, which point into the halos
+    st = peer_setup(d, halo_bytes);
+    if (st.bad()) return st;
+  }
   for (int p = 0; p < 2; ++p) d.gsrc_dev[p] = reinterpret_cast<const double**>(carve(gsrc_bytes));
   for (int p = 0; p < 2; ++p) d.items_dev[p] = reinterpret_cast<TileItem*>(carve(items_bytes));
   if (d.x2_ok) {
@@ -272,7 +277,7 @@ Status domain_setup(Domain& d) {
   d.nevents = d.ev_misc_base + 4 + d.halo_stream + 1 + 2;  // + 2 stream-through ring events
   st = X.setup(d);
   if (st.bad()) return st;
-  if (multi && !d.opt.dry_run && !d.opt.local_group) {
+  if (multi && !d.opt.dry_run && !d.opt.local_group && !d.opt.peer_transport) {
     st = nccl_init(d);
     if (st.bad()) return st;
   }
@@ -285,6 +290,7 @@ Status domain_free(Domain* d) {
   if (d->exec) {
     if (!d->poisoned && d->in_flight) r = d->exec->sync_all(*d);
     if (d->nccl_comm) nccl_destroy(*d);
+    if (d->peer_window) peer_destroy(*d);
     d->exec->destroy(*d);
     if (d->own_pool && d->pool) d->exec->free_device(*d, d->pool);
     if (d->host) d->exec->free_host(*d, d->host);

@@ -214,6 +214,16 @@ struct Domain {
 
   // NCCL
   void* nccl_comm = nullptr;
+  // peer transport (comm_peer.cu): own window (halo buffers + counters),
+  // the neighbours' windows [0 = lower, 1 = upper], exchange counter
+  void* peer_window = nullptr;
+  void* peer_flags = nullptr;
+  uint64_t peer_halo_bytes = 0;
+  void* peer_base[2] = {nullptr, nullptr};
+  void* peer_opened[2] = {nullptr, nullptr};
+  unsigned int peer_wait_flags = 0;
+  uint32_t peer_k = 0;
+  bool peer_connected = false;
 
   // kernel plan
   int band = 0, stages = 0, heat_grid = 0, sm_count = 148;
@@ -271,5 +281,10 @@ void nccl_destroy(Domain& d);
 Status local_group_create(int n, void** out);
 void local_group_free(void* g);
 Status local_halo(Domain& d, int parity, void* stream, void* ready_event);
+Status peer_setup(Domain& d, uint64_t halo_bytes);
+Status peer_handle(const Domain& d, void* out64);
+Status peer_connect(Domain& d, const void* handles, int n);
+Status peer_halo(Domain& d, int parity, void* stream);
+void peer_destroy(Domain& d);
 
 }  // namespace tiles

@@ -47,7 +47,8 @@ class TileOptions(ctypes.Structure):
                 ("nccl_unique_id", ctypes.c_void_p), ("sched", ctypes.c_int),
                 ("dry_run", ctypes.c_int32), ("fuse_pointwise_steps", ctypes.c_int32),
                 ("local_group", ctypes.c_void_p), ("pageable_host", ctypes.c_int32),
-                ("stream_through", ctypes.c_int32), ("two_step", ctypes.c_int32)]
+                ("stream_through", ctypes.c_int32), ("peer_transport", ctypes.c_int32),
+                ("two_step", ctypes.c_int32)]
 
 
 class TileKernel(ctypes.Structure):
@@ -110,6 +111,8 @@ _sig = {
     "tile_free": ([_P], ctypes.c_int),
     "tile_last_error": ([], ctypes.c_char_p),
     "tile_nccl_unique_id": ([_P], ctypes.c_int),
+    "tile_peer_handle": ([_P, _P], ctypes.c_int),
+    "tile_peer_connect": ([_P, _P, ctypes.c_int32], ctypes.c_int),
     "tile_local_group_create": ([ctypes.c_int32, ctypes.POINTER(_P)], ctypes.c_int),
     "tile_local_group_free": ([_P], ctypes.c_int),
     "tile_version": ([], ctypes.c_char_p),
@@ -173,7 +176,7 @@ class Domain:
     def __init__(self, dims, tile_dims, ghost=1, bc="periodic", device=-1, device_budget_bytes=0,
                  sched="auto", nranks=1, rank=0, nccl_id=None, dry_run=False,
                  fuse_pointwise_steps=True, device_pool=None, streams=None, local_group=None,
-                 pageable_host=False, two_step=0, stream_through=0):
+                 pageable_host=False, two_step=0, stream_through=0, peer_transport=False):
         self._h = None
         self.dims = tuple(int(v) for v in dims)
         self.tile_dims = tuple(int(v) for v in tile_dims)
@@ -204,6 +207,7 @@ class Domain:
         o.pageable_host = 1 if pageable_host else 0
         o.two_step = int(two_step)
         o.stream_through = int(stream_through)
+        o.peer_transport = 1 if peer_transport else 0
         self._group = local_group
         if local_group is not None:
             o.local_group = local_group.handle
@@ -312,6 +316,19 @@ class Domain:
 
     def reset_stats(self):
         _check(tile_reset_stats(self._h), "tile_reset_stats")
+
+    def peer_handle(self):
+        """64-byte CUDA IPC handle of this rank's halo window (peer transport)."""
+        buf = ctypes.create_string_buffer(64)
+        _check(tile_peer_handle(self._h, buf), "tile_peer_handle")
+        return buf.raw
+
+    def peer_connect(self, handles):
+        """Map the z-neighbours' windows; `handles` = every rank's peer_handle()
+        in rank order."""
+        blob = b"".join(bytes(h) for h in handles)
+        buf = ctypes.create_string_buffer(blob, len(blob))
+        _check(tile_peer_connect(self._h, buf, len(handles)), "tile_peer_connect")
 
     def trace(self):
         n = ctypes.c_int64()

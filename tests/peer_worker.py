@@ -1,0 +1,36 @@
+"""Worker process for the peer-transport tests (test_gpu_multirank.py): one
+rank of a z-slab domain with tile_options.peer_transport, exchanging its CUDA
+IPC window handle with the parent over a pipe. Test infrastructure only."""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def run(r, G, dims, td, bc, sched, budget, runs, seed, conn):
+    sys.path.insert(0, ROOT)
+    try:
+        import synth
+        from paper_conf_icpp_bastemuzas17_b200 import tiles as T
+        nx, ny, nz = dims
+        nzl = nz // G
+        kw = {"sched": sched}
+        if budget:
+            kw["device_budget_bytes"] = budget
+        with T.Domain(dims, td, bc=bc, nranks=G, rank=r, peer_transport=True, device=0, **kw) as d:
+            conn.send(("handle", d.peer_handle()))
+            kind, handles = conn.recv()
+            d.peer_connect(handles)
+            if bc == "periodic":
+                u = synth.uniform_grid(nx, ny, nz, seed)
+                d.load(u[r * nzl:(r + 1) * nzl])
+            else:
+                ext = synth.uniform_grid(nx + 2, ny + 2, nz + 2, seed)
+                d.load(ext[r * nzl:r * nzl + nzl + 2])
+            for s in runs:
+                d.run(T.heat7(0.125), s, 2)
+            out = d.store()
+            st = d.stats()
+        conn.send(("out", out, st["n_halo"], st["bytes_halo"]))
+    except Exception as e:  # noqa: BLE001
+        conn.send(("error", repr(e)))

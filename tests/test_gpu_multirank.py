@@ -76,3 +76,55 @@ def test_local_group_slabs_bit_exact(G, bc, sched, runs):
     assert not err, err
     got = np.concatenate(out, axis=0)
     assert np.array_equal(got, ref), np.abs(got - ref).max()
+
+
+@pytest.mark.parametrize("G,bc,sched,runs", [(2, "periodic", "resident", [5]), (3, "periodic", "resident", [4, 3]),
+                                             (2, "dirichlet", "resident", [3]), (4, "periodic", "stream", [3]),
+                                             (3, "dirichlet", "stream", [2, 2])])
+def test_peer_transport_processes_bit_exact(G, bc, sched, runs):
+    """Peer transport (tile_options.peer_transport): one PROCESS per rank, all
+    on the one GPU of the pool (CUDA IPC works between processes on a device
+    as between devices); the halo exchange is the IPC window push with
+    stream-memory-op counters, no NCCL. Bit-exact against the oracle."""
+    import multiprocessing as mp
+    from tests import peer_worker
+    dims, td = (64, 32, 16 * G), (32, 16, 8)
+    nx, ny, nz = dims
+    budget = _budget(dims, td, 3, bc=bc, nranks=G, rank=0) if sched == "stream" else 0
+    ctx = mp.get_context("spawn")
+    pipes, procs = [], []
+    for r in range(G):
+        a, b = ctx.Pipe()
+        p = ctx.Process(target=peer_worker.run, args=(r, G, dims, td, bc, sched, budget, runs, 42, b))
+        p.start()
+        pipes.append(a)
+        procs.append(p)
+    try:
+        handles = []
+        for a in pipes:
+            assert a.poll(180), "worker did not report its handle"
+            msg = a.recv()
+            assert msg[0] == "handle", msg
+            handles.append(msg[1])
+        for a in pipes:
+            a.send(("handles", handles))
+        outs = []
+        for a in pipes:
+            assert a.poll(300), "worker did not finish"
+            msg = a.recv()
+            assert msg[0] == "out", msg
+            outs.append(msg)
+    finally:
+        for p in procs:
+            p.join(30)
+            if p.is_alive():
+                p.kill()
+    got = np.concatenate([m[1] for m in outs], axis=0)
+    if bc == "periodic":
+        ref = oracle.heat_c(synth.uniform_grid(nx, ny, nz, 42), ALPHA, sum(runs))
+    else:
+        ext = synth.uniform_grid(nx + 2, ny + 2, nz + 2, 42)
+        ref = oracle.heat_c(ext, ALPHA, sum(runs), oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+        got = np.concatenate([m[1][1:-1, 1:-1, 1:-1] for m in outs], axis=0)
+    assert np.array_equal(got, ref), np.abs(got - ref).max()
+    assert all(m[2] > 0 and m[3] > 0 for m in outs)  # halo exchanges happened through the window
