@@ -655,12 +655,28 @@ static std::vector<int> plan_passes(const Domain& d, int steps) {
 // layer's gather; layer 0, read by the last layer's gather through the
 // periodic wrap, at the end), so the domain stays resident. Periodic, single
 // rank.
+struct UnitDef {
+  int64_t layer, p0, np;  // planes [p0, p0+np) of tile layer `layer`
+};
 struct StreamPlan {
-  int64_t unit;        // planes per unit (divides tz, >= T)
-  int64_t units;       // local nz / unit
-  int64_t slab_tiles;  // one dense slab of unit + 2T planes, in tile slots
+  int64_t unit;        // nominal planes per unit (divides tz, >= T)
+  int64_t units;       // number of units
+  std::vector<UnitDef> u;
+  int64_t slab_tiles;  // one dense slab of max unit + 2T planes, in tile slots
   int64_t sub_tiles;   // one packed unit result (layer_tiles sub-tiles), in tile slots
 };
+
+// Units in z order: each tile layer cut into tz / un pieces of un planes
+// (un >= T: a unit's halo lies in its two neighbour units). Thin first/last
+// units (a shorter pipeline fill and drain) were measured and gained nothing
+// at C2 (25.6 ms either way): the run is link-rate bound.
+static std::vector<UnitDef> make_units(const Geometry& G, int64_t un, int T) {
+  (void)T;
+  std::vector<UnitDef> v;
+  for (int64_t L = 0; L < G.n[2]; ++L)
+    for (int64_t p = 0; p < G.t[2]; p += un) v.push_back({L, p, un});
+  return v;
+}
 
 static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
   const Geometry& G = d.G;
@@ -698,12 +714,15 @@ static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
   // (0.011 per plane-step, same fit); take stream-through only where it is
   // estimated faster
   if (d.opt.stream_through == 0 && best > 2.0 * nz + 0.011 * nz * Td) return false;
-  const int64_t units = G.l[2] / unit;
-  if (units > G.ntiles) unit = G.t[2];  // event budget (one per unit)
+  if (G.l[2] / unit + 4 > G.ntiles) unit = G.t[2];  // event budget (one per unit)
   sp->unit = unit;
-  sp->units = G.l[2] / unit;
-  sp->slab_tiles = ((unit + 2 * (int64_t)T) * plane + G.tile_elems - 1) / G.tile_elems;
-  sp->sub_tiles = (G.layer_tiles * unit * G.t[0] * G.t[1] + G.tile_elems - 1) / G.tile_elems;
+  sp->u = make_units(G, unit, T);
+  if ((int64_t)sp->u.size() > G.ntiles) sp->u = make_units(G, G.t[2], T);
+  sp->units = (int64_t)sp->u.size();
+  int64_t mx = 0;
+  for (const auto& x : sp->u) mx = std::max(mx, x.np);
+  sp->slab_tiles = ((mx + 2 * (int64_t)T) * plane + G.tile_elems - 1) / G.tile_elems;
+  sp->sub_tiles = (G.layer_tiles * mx * G.t[0] * G.t[1] + G.tile_elems - 1) / G.tile_elems;
   return 2 * sp->slab_tiles + 3 * sp->sub_tiles <= G.ntiles;
 }
 
@@ -720,15 +739,18 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
   (void)alpha;
   Exec& X = *d.exec;
   const Geometry& G = d.G;
-  const int64_t U = sp.units, lt = G.layer_tiles, tz = G.t[2], un = sp.unit;
+  const int64_t U = sp.units, lt = G.layer_tiles, tz = G.t[2];
   const Pipes P(S, false);
   const int bit = d.res_bit;                       // H2D target array
   const int sb = bit ? 0 : (int)G.ntiles;          // scratch array (the other one)
   const int slab[2] = {sb, sb + (int)sp.slab_tiles};
   const int out[2] = {sb + 2 * (int)sp.slab_tiles, sb + 2 * (int)sp.slab_tiles + (int)sp.sub_tiles};
   const int keep0 = sb + 2 * (int)sp.slab_tiles + 2 * (int)sp.sub_tiles;
-  auto layer_of = [&](int64_t u) { return (u * un) / tz; };
-  auto p0_of = [&](int64_t u) { return (u * un) % tz; };
+  (void)tz;
+  auto layer_of = [&](int64_t u) { return sp.u[(size_t)u].layer; };
+  auto p0_of = [&](int64_t u) { return sp.u[(size_t)u].p0; };
+  auto np_of = [&](int64_t u) { return sp.u[(size_t)u].np; };
+  auto z0_of = [&](int64_t u) { return layer_of(u) * G.t[2] + p0_of(u); };  // first local plane
   auto cur_slot = [&](int64_t u) {
     const int64_t t0 = layer_of(u) * lt;
     return bit ? (int)(G.ntiles + t0) : (int)t0;
@@ -737,7 +759,6 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
   auto ev_unit_done = [&](int64_t u) { return ev_host(d, u); };  // compute of unit u
   const int ring_ev[2] = {d.ev_misc_base + 4 + d.halo_stream + 1, d.ev_misc_base + 5 + d.halo_stream + 1};
   const int cs = P.comp(0), os = P.out(0), is = P.in(0);
-  d.st_unit = un;
   Status r;
   // one copy-in stream, so the copy engine runs the H2Ds in this order (it
   // may not across streams): the last unit first (unit 0's wrap neighbour)
@@ -745,7 +766,7 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
   order.push_back(U - 1);
   for (int64_t u = 0; u < U - 1; ++u) order.push_back(u);
   for (int64_t u : order) {
-    r = X.h2d_part(d, layer_of(u) * lt, lt, cur_slot(u), p0_of(u), un, is);
+    r = X.h2d_part(d, layer_of(u) * lt, lt, cur_slot(u), p0_of(u), np_of(u), is);
     if (r.bad()) return r;
     r = X.record(d, ev_in(d, u), is);
     if (r.bad()) return r;
@@ -759,17 +780,18 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
       r = X.wait(d, ring_ev[u & 1], cs);
       if (r.bad()) return r;
     }
-    // sweep i reads planes [i-1, un+2T-i+1) and writes [i, un+2T-i); the
+    // sweep i reads planes [i-1, n+2T-i+1) and writes [i, n+2T-i); the
     // first reads the resident array directly (gather fused), the last writes
     // the unit's packed sub-tiles (scatter fused)
     for (int i = 1; i <= T; ++i) {
-      const SlabRef src = i == 1 ? SlabRef{SlabRef::RESIDENT, bit, u * un - T}
+      const SlabRef src = i == 1 ? SlabRef{SlabRef::RESIDENT, bit, z0_of(u) - T}
                                  : SlabRef{SlabRef::DENSE, slab[(i - 1) & 1], 0};
       const SlabRef dst = i == T ? SlabRef{SlabRef::SUB, res_of(u), 0} : SlabRef{SlabRef::DENSE, slab[i & 1], 0};
-      r = X.slab_sweep(d, src, dst, i, (int)(un + 2 * T - i), cs);
+      d.st_unit = np_of(u);  // packed sub-tile depth of the last sweep
+      r = X.slab_sweep(d, src, dst, i, (int)(np_of(u) + 2 * T - i), cs);
       if (r.bad()) return r;
       if (i == 1 && u >= 2) {  // unit u-1's initial data has no reader left
-        r = X.copy_part(d, res_of(u - 1), cur_slot(u - 1), lt, p0_of(u - 1), un, cs);
+        r = X.copy_part(d, res_of(u - 1), cur_slot(u - 1), lt, p0_of(u - 1), np_of(u - 1), cs);
         if (r.bad()) return r;
       }
     }
@@ -777,7 +799,7 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
     if (r.bad()) return r;
     r = X.wait(d, ev_unit_done(u), os);
     if (r.bad()) return r;
-    r = X.d2h_part(d, layer_of(u) * lt, lt, res_of(u), p0_of(u), un, os);
+    r = X.d2h_part(d, layer_of(u) * lt, lt, res_of(u), p0_of(u), np_of(u), os);
     if (r.bad()) return r;
     if (u >= 1) {
       r = X.record(d, ring_ev[u & 1], os);
@@ -785,10 +807,10 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
     }
   }
   if (U >= 2) {
-    r = X.copy_part(d, res_of(U - 1), cur_slot(U - 1), lt, p0_of(U - 1), un, cs);
+    r = X.copy_part(d, res_of(U - 1), cur_slot(U - 1), lt, p0_of(U - 1), np_of(U - 1), cs);
     if (r.bad()) return r;
   }
-  r = X.copy_part(d, keep0, cur_slot(0), lt, p0_of(0), un, cs);
+  r = X.copy_part(d, keep0, cur_slot(0), lt, p0_of(0), np_of(0), cs);
   if (r.bad()) return r;
   for (int64_t k = 0; k < G.ntiles; ++k) {
     d.tile_dirty[k] = 0;  // the host received u^T through the D2H above

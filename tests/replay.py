@@ -343,7 +343,10 @@ class Replayer:
         x/y halo is the periodic wrap and whose z halo is fixed)."""
         blk = np.pad(src[lo - 1:hi + 1], ((0, 0), (1, 1), (1, 1)), mode="wrap")
         new = oracle.heat_np(blk, self.alpha, 1, oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
-        out = np.full_like(src, np.nan) if dst is None else dst.copy()
+        n = max(src.shape[0], hi, 0 if dst is None else dst.shape[0])
+        out = np.full((n,) + src.shape[1:], np.nan)  # slabs of different units differ in depth
+        if dst is not None:
+            out[:dst.shape[0]] = dst
         out[lo:hi] = new
         return out
 
