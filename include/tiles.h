@@ -116,9 +116,9 @@ typedef struct {
   int32_t stream_through;       /* HEAT7 run starting from a fresh upload
                                    (periodic, single rank, T <= tile_dims[2],
                                    scratch fits): per unit of planes (a slice
-                                   of a z-layer, >= T planes) trapezoid: gather
-                                   the unit + T halo planes, T sweeps, D2H the
-                                   exact core, so H2D, compute and D2H of
+                                   of a z-layer, >= T planes) trapezoid: T
+                                   sweeps over the unit + T halo planes, D2H
+                                   of the exact core, so H2D, compute and D2H of
                                    different units overlap; each unit's result
                                    is also written back to the device array once
                                    no other unit reads its initial data.

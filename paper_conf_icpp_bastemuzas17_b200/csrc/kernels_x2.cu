@@ -351,37 +351,6 @@ __global__ void __launch_bounds__(X2<TX, BY, S, MB>::NT + 32) heat7x2(const __gr
     pp += z1 - z0;
   }
 }
-#if 0
-      {  // (old inline output, kept for reference of the layout)
-        const int o = m - 1;
-        const double* cb = mid0 + (size_t)((mi - 1) & 1) * C::MID_ELEMS;  // mid(o)
-        const double* nb = mb;                                             // mid(o+1)
-        double* op = obase + (size_t)o * plane_elems;
-        const bool zlo = o < 2, zhi = o >= tz - 2;
-#pragma unroll
-        for (int j = 0; j < C::NR; ++j) {
-          const int r = r0 + j * C::RPP;  // band row
-          const double* crow = cb + (r + 1) * C::MPITCH + xo + 2;
-          const double2 c = *reinterpret_cast<const double2*>(crow);
-          const double2 ym = *reinterpret_cast<const double2*>(crow - C::MPITCH);
-          const double2 yp = *reinterpret_cast<const double2*>(crow + C::MPITCH);
-          const double2 zp = *reinterpret_cast<const double2*>(nb + (r + 1) * C::MPITCH + xo + 2);
-          const double xm = crow[-1], xp = crow[2];
-          double2 v;
-          v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zmr[j].x, zp.x, alpha);
-          v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zmr[j].y, zp.y, alpha);
-          stg2_stream(op + (size_t)j * C::RPP * TX, v);
-          zmr[j] = c;
-          const int y = yb + j * C::RPP;
-          if (xlo_edge) st2_hint(fxm + ((size_t)o * ty + y) * 2, v, keep);
-          if (xhi_edge) st2_hint(fxp + ((size_t)o * ty + y) * 2, v, keep);
-          if (y < 2) st2_hint(fym + ((size_t)o * 2 + y) * TX, v, keep);
-          if (y >= ty - 2) st2_hint(fyp + ((size_t)o * 2 + y - (ty - 2)) * TX, v, keep);
-          if (zlo) st2_hint(fzm + ((size_t)o * ty + y) * TX, v, keep);
-          if (zhi) st2_hint(fzp + ((size_t)(o - (tz - 2)) * ty + y) * TX, v, keep);
-        }
-      }
-#endif
 
 // ---- heat7x2r: the same two-step pass with a row-owning thread layout
 // (TX = 64: one warp spans the tile width, lane l owns the x-pair 2l). 16

@@ -643,18 +643,17 @@ static std::vector<int> plan_passes(const Domain& d, int steps) {
 }
 
 // Stream-through: with a fresh upload, a cell after T steps
-// depends only on cells within T planes, so with T <= tz each z-layer's
-// final state needs only its own and the two adjacent layers' initial data.
-// Per layer (in z order): gather the layer and T halo planes into a dense
-// slab, run T sweeps with the valid range shrinking by one plane per end,
-// scatter the tz exact core planes into a tile-blocked out buffer, D2H it.
-// H2D of later layers, compute and D2H of earlier layers overlap (duplex
-// host link). Scratch = the resident mode's second buffer array (not needed
-// otherwise in this run). Each layer's result is also copied back into the
-// resident array once its initial data has no reader left (after the next
-// layer's gather; layer 0, read by the last layer's gather through the
-// periodic wrap, at the end), so the domain stays resident. Periodic, single
-// rank.
+// depends only on cells within T planes, so with T <= tz a unit of >= T
+// planes needs only its own and its two neighbour units' initial data. Per
+// unit (in z order): T sweeps over the unit and T halo planes with the valid
+// range shrinking by one plane per end (the first reads the resident array,
+// the last writes the exact core into packed sub-tiles), then its D2H. H2D of
+// later units, compute and D2H of earlier units overlap (duplex host link).
+// Scratch = the resident mode's second buffer array (not needed otherwise in
+// this run). Each unit's result is also copied back into the resident array
+// once its initial data has no reader left (after the next unit's first
+// sweep; unit 0, read by the last unit through the periodic wrap, at the
+// end), so the domain stays resident. Periodic, single rank.
 struct UnitDef {
   int64_t layer, p0, np;  // planes [p0, p0+np) of tile layer `layer`
 };
