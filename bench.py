@@ -66,16 +66,44 @@ def red_dev():
 
 
 class Clocks:
-    """nvidia-smi sampler for the timed region (B200_PROFILING.md clocks line)."""
+    """Clock / throttle-reason sampler for the timed region (B200_PROFILING.md
+    clocks line): NVML polled every ~2 ms from a thread (a C2 value leg lasts
+    ~80 ms, too short for nvidia-smi's 100 ms loop); nvidia-smi if NVML is
+    unavailable."""
 
     Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
 
     def __init__(self, gpu):
-        self.gpu, self.rows, self.p = gpu, [], None
+        self.gpu, self.rows, self.p, self.nv, self.stop = gpu, [], None, None, False
 
     def __enter__(self):
+        try:
+            import pynvml as nv
+            nv.nvmlInit()
+            h = nv.nvmlDeviceGetHandleByIndex(self.gpu)
+            self.nv = nv
+            self.maxc = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
+            bits = [nv.nvmlClocksEventReasonHwSlowdown, nv.nvmlClocksEventReasonHwThermalSlowdown,
+                    nv.nvmlClocksEventReasonSwThermalSlowdown, nv.nvmlClocksEventReasonSwPowerCap]
+
+            def poll():
+                while not self.stop:
+                    try:
+                        sm = nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)
+                        rs = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+                        self.rows.append([str(sm), str(self.maxc), "", *["Active" if rs & b else "Not Active"
+                                                                       for b in bits]])
+                    except Exception:
+                        pass
+                    time.sleep(0.002)
+            self.t = threading.Thread(target=poll, daemon=True)
+            self.t.start()
+            return self
+        except Exception:
+            self.nv = None
         try:
             self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
                                        "--format=csv,noheader,nounits", "-lms", "100"],
@@ -93,6 +121,9 @@ class Clocks:
                 self.rows.append(parts)
 
     def __exit__(self, *a):
+        self.stop = True
+        if self.nv is not None:
+            self.t.join(1)
         if self.p:
             self.p.terminate()
             try:
@@ -105,14 +136,14 @@ class Clocks:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
         sm = sorted(float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit())
         reasons = set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for r in self.rows:
-            for n, v in zip(names, r[3:]):
+            for n, v in zip(self.NAMES, r[3:]):
                 if v.lower().startswith("active"):
                     reasons.add(n)
         return {"sm_mhz": sm[len(sm) // 2] if sm else None,
                 "sm_max_mhz": float(self.rows[0][1]) if self.rows[0][1].replace(".", "").isdigit() else None,
-                "reasons": sorted(reasons), "samples": len(self.rows)}
+                "reasons": sorted(reasons), "samples": len(self.rows),
+                "source": "nvml" if self.nv is not None else "nvidia-smi"}
 
 
 def measured_peaks():
