@@ -75,6 +75,34 @@ def test_stream_counts_bit_exact(ns):
     assert np.array_equal(out, ref)
 
 
+@pytest.mark.parametrize("dims,td,steps,ns", [((8, 8, 8), (2, 2, 2), 4, 2),        # 64 tiny tiles, generic kernel
+                                              ((16, 8, 9), (8, 4, 3), 5, 3),      # odd tile depth
+                                              ((64, 64, 64), (32, 16, 16), 6, 64), # the maximum stream count
+                                              ((16, 16, 8), (16, 16, 8), 3, 1),   # one tile, wraps onto itself
+                                              ((32, 16, 256), (32, 16, 8), 4, 4)]) # 32 thin layers
+def test_edge_shapes_and_counts(dims, td, steps, ns):
+    """Degenerate decompositions: tiles of 2 cells per axis, odd depths, a
+    single tile whose ghosts are its own faces, many thin layers, 64 streams."""
+    out, ref, _, _ = _heat(dims, td, steps, ns=ns)
+    assert np.array_equal(out, ref)
+
+
+def test_zero_work_runs_are_identity():
+    """tile_run with 0 steps, and SINCOS with 0 inner iterations, change nothing."""
+    nx, ny, nz = 64, 32, 32
+    u0 = synth.uniform_grid(nx, ny, nz, 3)
+    with T.Domain((nx, ny, nz), (32, 16, 16)) as d:
+        d.load(u0)
+        d.run(T.heat7(ALPHA), 0, 2)
+        assert np.array_equal(d.store(), u0)
+        d.run(T.sincos(0), 3, 2)
+        assert np.array_equal(d.store(), u0)
+    with T.Domain((nx, ny, nz), (32, 16, 16), sched="stream", device_budget_bytes=_budget((nx, ny, nz), (32, 16, 16), 3)) as d:
+        d.load(u0)
+        d.run(T.heat7(ALPHA), 0, 2)
+        assert np.array_equal(d.store(), u0)
+
+
 def test_runs_continue_state():
     out, ref, _, _ = _heat((64, 64, 64), (32, 32, 16), 9, runs=[4, 1, 0, 4])
     assert np.array_equal(out, ref)
