@@ -44,7 +44,8 @@ struct ViewDev {
       int k = iu - u + 1;
       if (k < 0) k += U;
       if (k >= U) k -= U;
-      return ub[k] + (int64_t)(gz - iu * un) * ty * tx;
+      double* b = k == 0 ? ub[0] : k == 1 ? ub[1] : ub[2];  // selects, not a local-memory array
+      return b + (int64_t)(gz - iu * un) * ty * tx;
     }
     const int iz = gz / tz, lz = gz - iz * tz;
     return base + (int64_t)iz * nty * ntx * te + (int64_t)lz * ty * tx;
@@ -144,6 +145,128 @@ __global__ void __launch_bounds__(128, 4) slab_sweep_zm(const ViewDev S, const V
   }
 }
 
+// cp.async variant: the same z-march and work order, but every plane a
+// thread needs (its BY rows, the two halo rows, the x-edge cells of the warp's
+// edge lanes) is fetched S-1 planes ahead with cp.async into a per-thread
+// shared-memory ring ([stage][row][thread], conflict-free), one commit group
+// per plane. A thread reads only what it fetched itself, so wait_group alone
+// orders it (no block barrier); deep memory-level parallelism at a low
+// register count.
+__device__ __forceinline__ void cp16(void* sdst, const void* gsrc) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"((uint32_t)__cvta_generic_to_shared(sdst)),
+               "l"(gsrc)
+               : "memory");
+}
+__device__ __forceinline__ void cp8(void* sdst, const void* gsrc) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"((uint32_t)__cvta_generic_to_shared(sdst)),
+               "l"(gsrc)
+               : "memory");
+}
+__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+template <int BY, int SG>
+struct CaLayout {
+  static constexpr int ROWS = BY + 2;                      // own rows, then halo y0-1, y0+BY
+  static constexpr int STAGE_V = ROWS * 128;                // double2 per stage (all threads)
+  static constexpr int EDGE_D = 4 * 2 * BY;                 // doubles per stage: [warp][side][row]
+  static constexpr size_t SMEM = (size_t)SG * (STAGE_V * 16 + EDGE_D * 8);
+};
+
+template <int BY, int SG>
+__global__ void __launch_bounds__(128, 4) slab_sweep_ca(const ViewDev S, const ViewDev D, const int nx,
+                                                        const int ny, const int lo, const int hi,
+                                                        const int gx, const int zc, const double alpha) {
+  using L = CaLayout<BY, SG>;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  double2* ring = reinterpret_cast<double2*>(smem_raw);
+  double* edges = reinterpret_cast<double*>(smem_raw + (size_t)SG * L::STAGE_V * 16);
+  const int npairs = nx >> 1;
+  const int tid = (int)threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int cols = gx * (ny / BY);
+  const int nch = (hi - lo + zc - 1) / zc;
+  const int64_t items = (int64_t)cols * nch;
+  const int stx = S.tx, dtx = D.tx;
+  auto slot = [&](int st, int row) -> double2& { return ring[(st * L::ROWS + row) * 128 + tid]; };
+  auto edge = [&](int st, int side, int row) -> double& {
+    return edges[((st * 4 + warp) * 2 + side) * BY + row];
+  };
+
+  for (int64_t it = blockIdx.x; it < items; it += gridDim.x) {
+    const int ch = (int)(it / cols), col = (int)(it - (int64_t)ch * cols);
+    const int zlo = lo + ch * zc, zhi = min(hi, zlo + zc);
+    const int seg = col % gx, y0 = (col / gx) * BY;
+    const int px = seg * 128 + tid;
+    const bool valid = px < npairs;
+    const int x = 2 * (valid ? px : npairs - 1);
+    // one edge lane per side per warp (the smem edge slots have one writer);
+    // invalid (clamped) lanes store nothing and need no edges
+    const bool ledge = valid && lane == 0, redge = valid && (lane == 31 || px + 1 == npairs);
+    const int64_t sx = S.X(x), dx = D.X(x);
+    const int64_t exo_m = S.X(x == 0 ? nx - 1 : x - 1) - sx, exo_p = S.X(x + 2 == nx ? 0 : x + 2) - sx;
+    const int64_t sy0 = S.Y(y0) + sx, dy0 = D.Y(y0) + dx;
+    const int64_t shm = S.Y(y0 == 0 ? ny - 1 : y0 - 1) + sx;
+    const int64_t shp = S.Y(y0 + BY == ny ? 0 : y0 + BY) + sx;
+    // planes zlo-1 .. zhi; plane q = zlo - 1 + i goes to stage i % SG
+    const int nplanes = zhi - zlo + 2;
+    auto fetch = [&](int i) {
+      if (i < nplanes) {
+        const int z = zlo - 1 + i, st = i % SG;
+        const double* pz = S.P(z);
+#pragma unroll
+        for (int j = 0; j < BY; ++j) {
+          const double* g = pz + sy0 + (int64_t)j * stx;
+          cp16(&slot(st, j), g);
+          if (ledge) cp8(&edge(st, 0, j), g + exo_m);
+          if (redge) cp8(&edge(st, 1, j), g + exo_p);
+        }
+        cp16(&slot(st, BY), pz + shm);
+        cp16(&slot(st, BY + 1), pz + shp);
+      }
+      cp_commit();  // (possibly empty) group per plane keeps the count uniform
+    };
+#pragma unroll
+    for (int i = 0; i < SG; ++i) fetch(i);
+    cp_wait<SG - 2>();  // planes zlo-1, zlo landed
+    double2 zm[BY], zcur[BY];
+#pragma unroll
+    for (int j = 0; j < BY; ++j) {
+      zm[j] = slot(0, j);
+      zcur[j] = slot(1 % SG, j);
+    }
+    for (int z = zlo; z < zhi; ++z) {
+      const int i = z - zlo + 1;  // plane z is index i, z+1 is i+1
+      fetch(i + SG - 1);          // into the stage of plane i-1 (its rows are in zm)
+      cp_wait<SG - 2>();          // plane i+1 landed
+      const int sc = i % SG, sn = (i + 1) % SG;
+      const double2 hm = slot(sc, BY), hp = slot(sc, BY + 1);
+      double* pd = D.P(z);
+#pragma unroll
+      for (int j = 0; j < BY; ++j) {
+        const double2 c = zcur[j];
+        const double2 zp = slot(sn, j);
+        double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+        double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+        if (ledge) xm = edge(sc, 0, j);
+        if (redge) xp = edge(sc, 1, j);
+        const double2 ym = j == 0 ? hm : zcur[j > 0 ? j - 1 : 0];
+        const double2 yp = j == BY - 1 ? hp : zcur[j < BY - 1 ? j + 1 : 0];
+        double2 v;
+        v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm[j].x, zp.x, alpha);
+        v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm[j].y, zp.y, alpha);
+        if (valid) *reinterpret_cast<double2*>(pd + dy0 + (int64_t)j * dtx) = v;
+      }
+#pragma unroll
+      for (int j = 0; j < BY; ++j) {  // after the row loop: rows j+-1 read zcur of plane z
+        zm[j] = zcur[j];
+        zcur[j] = slot(sn, j);
+      }
+    }
+    cp_wait<0>();  // drain the (empty) tail groups before the ring is reused
+  }
+}
+
 static int sweep_occupancy(int BY) {
   static int occ[3] = {0, 0, 0};
   const int k = BY == 4 ? 2 : BY == 2 ? 1 : 0;
@@ -187,6 +310,21 @@ cudaError_t launch_slab_sweep(const SlabView& src, const SlabView& dst, int nx, 
   zc = (planes + best_nch - 1) / best_nch;
   const int64_t grid = std::min<int64_t>(G, cols * ((planes + zc - 1) / zc));
   const ViewDev S = to_dev(src), D = to_dev(dst);
+  static const int use_ca = [] {
+    const char* e = getenv("TILES_SWEEP_CA");
+    return e ? atoi(e) : 1;
+  }();
+  if (use_ca && BY == 4) {  // 4 stages: 4 blocks per SM (5 or 6 stages fit 3: slower, 4.0-4.1 TB/s)
+    constexpr size_t sm = CaLayout<4, 4>::SMEM;
+    static bool attr = false;
+    if (!attr) {
+      cudaError_t e = cudaFuncSetAttribute(slab_sweep_ca<4, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+      if (e != cudaSuccess) return e;
+      attr = true;
+    }
+    slab_sweep_ca<4, 4><<<(unsigned)grid, 128, sm, s>>>(S, D, nx, ny, lo, hi, gx, zc, alpha);
+    return cudaGetLastError();
+  }
   switch (BY) {
     case 4: slab_sweep_zm<4><<<(unsigned)grid, 128, 0, s>>>(S, D, nx, ny, lo, hi, gx, zc, alpha); break;
     case 2: slab_sweep_zm<2><<<(unsigned)grid, 128, 0, s>>>(S, D, nx, ny, lo, hi, gx, zc, alpha); break;

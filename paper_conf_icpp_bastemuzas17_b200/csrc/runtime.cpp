@@ -689,8 +689,8 @@ static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
   // thick ones cut the redundant halo sweeps (a unit sweeps T*unit + T^2 - T
   // planes). Pick the divisor minimising, in per-plane link-copy times,
   //   max(nz, r * nz * (T + (T^2 - T) / unit)) + 3 * unit,
-  // r = sweep time / duplex link time per plane, 0.024 measured on B200 +
-  // PCIe 5 (slab_sweep_zm ~1.0 us per 512^2 plane, ~48 GB/s per direction;
+  // r = sweep time / duplex link time per plane, 0.021 measured on B200 +
+  // PCIe 5 (slab_sweep_ca ~0.8 us per 512^2 plane, ~48 GB/s per direction;
   // profiles/r01/ncu_slab_sweep.txt, bench_fig5_st_*.json).
   static const int64_t min_unit = [] {
     const char* e = getenv("TILES_ST_MINUNIT");
@@ -698,7 +698,7 @@ static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
   }();
   static const double r_sweep = [] {
     const char* e = getenv("TILES_ST_R");
-    return e ? atof(e) : 0.024;
+    return e ? atof(e) : 0.021;
   }();
   const double nz = (double)G.l[2], Td = (double)T;
   int64_t unit = G.t[2];
@@ -844,7 +844,7 @@ static bool ooc_streamthrough_ok(const Domain& d, int T, OocPlan* op) {
   const int64_t plane = G.l[0] * G.l[1];
   static const double r_sweep = [] {
     const char* e = getenv("TILES_ST_R");
-    return e ? atof(e) : 0.024;
+    return e ? atof(e) : 0.021;
   }();
   double best = 1e300;
   for (int64_t k = 2; k <= std::min<int64_t>(T, G.t[2]); ++k)
