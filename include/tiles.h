@@ -200,10 +200,15 @@ typedef enum {
   TILE_OP_COPY_PART = 19,/* packed sub-tiles at slot a -> slots b.. */
   TILE_OP_H2D_PACK = 20, /* host tiles a.. (c of them), planes [d & 0xffffffff, +d >> 32)
                             -> packed sub-tiles at slot b */
-  TILE_OP_SWEEP_U = 21   /* like SWEEP, source = units u-1, u, u+1 (packed sub-tiles at
+  TILE_OP_SWEEP_U = 21,  /* like SWEEP, source = units u-1, u, u+1 (packed sub-tiles at
                             slots b & 0x1fffff, b >> 21 & 0x1fffff, b >> 42), slab plane 0
                             at z = u*un - (hi + 1 - un) / 2; a = destination code,
                             c = lo | hi << 32, d = u | un << 32 */
+  TILE_OP_KERNELD = 22,  /* like KERNEL (tile a: slot b -> slot c, face parity d), direct
+                            ghosts: y/z ghosts read from the neighbours' interiors in the
+                            buffer array holding slot b, x ghosts from the parity-d faces;
+                            exports the x faces (and, multi-rank, the slab-end layers'
+                            z faces) only */
 } tile_op_kind;
 
 typedef struct {

@@ -267,4 +267,36 @@ const double* Domain::face_src_ptr(int64_t id, int f, int parity) const {
   }
 }
 
+// Direct ghost sources (HeatParams::gdir): x ghosts from the
+// exported x faces; y and z ghosts from the nearest ghost layer itself — the
+// neighbour tile's boundary row / plane inside its interior in buffer array
+// `bit` when the neighbour is a tile of this rank (resident mode: tile k lives
+// in slot k or ntiles + k), else the nearest layer of the face source.
+const double* Domain::direct_src_ptr(int64_t id, int f, int bit, int parity) const {
+  if (f <= XP) return face_src_ptr(id, f, parity);
+  const int64_t tx = G.t[0], ty = G.t[1], tz = G.t[2], D = G.depth;
+  const FaceSrc s = face_source(G, id, f);
+  if (s.kind == 0) {
+    const double* nb = slot_ptr(bit ? (int)(G.ntiles + s.val) : (int)s.val);
+    switch (f) {
+      case YM: return nb + (ty - 1) * tx;
+      case YP: return nb;
+      case ZM: return nb + (tz - 1) * ty * tx;
+      default: return nb;
+    }
+  }
+  const double* base = face_src_ptr(id, f, parity);
+  switch (f) {
+    case YM: return base + (D - 1) * tx;
+    case YP: return base;
+    case ZM: return base + (D - 1) * ty * tx;
+    default: return base;
+  }
+}
+
+// z-stride of the direct y ghost row of tile `id` (f = YM or YP).
+int64_t Domain::direct_ystride(int64_t id, int f) const {
+  return face_source(G, id, f).kind == 0 ? G.t[1] * G.t[0] : (int64_t)G.depth * G.t[0];
+}
+
 }  // namespace tiles

@@ -2,6 +2,7 @@
 // CUDA streams, events, cudaMemcpyAsync from pinned memory
 // and the sm_100a kernels of kernels.cu. No CPU fallback exists: every
 // compute operation is a kernel launch.
+#include <cstdint>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -130,7 +131,7 @@ struct CudaExec final : Exec {
     return Status::ok();
   }
   Status heat(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
-              const TileItem* dev_items, int st) override {
+              const TileItem* dev_items, int st, int direct_bit, int nstack) override {
     if (d.measure == TILE_MEASURE_XFER_ONLY || n == 0) return Status::ok();
     HeatParams p{};
     p.tx = (int)d.G.t[0];
@@ -154,6 +155,23 @@ struct CudaExec final : Exec {
     for (int f = 0; f < 6; ++f) {
       p.fexp[f] = d.faces[f][rp ^ 1];
       p.face_elems[f] = d.G.face_elems[f];
+    }
+    if (nstack < 1 || n % nstack) return make_err(TILE_ESTATE, "internal: bad tile stack");
+    p.nstack = nstack;
+    p.lt = n / nstack;
+    if (direct_bit >= 0) {  // y/z ghosts from the neighbours' interiors; export x (+ slab-end z)
+      p.gdir = d.gdir_dev[direct_bit][rp];
+      p.ystr = d.ystr_dev;
+      p.exp_y = 0;
+      const bool multi = d.G.nranks > 1;
+      p.exp_zlo_below = multi ? (int32_t)d.G.layer_tiles : 0;
+      p.exp_zhi_from = multi ? (int32_t)(d.G.ntiles - d.G.layer_tiles) : INT32_MAX;
+    } else {
+      p.gdir = nullptr;
+      p.ystr = nullptr;
+      p.exp_y = 1;
+      p.exp_zlo_below = INT32_MAX;
+      p.exp_zhi_from = 0;
     }
     // persistent grid: one wave of CTAs, >= 4 planes each
     const int64_t planes = (int64_t)n * p.nbands * p.tz;
@@ -277,6 +295,10 @@ struct CudaExec final : Exec {
       p.fexp[f] = d.faces[f][rp ^ 1];
       p.face_elems[f] = d.G.face_elems[f];
     }
+    p.nstack = 1;
+    p.lt = n;
+    p.exp_y = 1;
+    p.exp_zlo_below = INT32_MAX;
     P.esrc = d.esrc_dev[rp];
     P.fixed_mask = d.fixed_mask_dev;
     const int64_t planes = (int64_t)n * p.nbands * p.tz;
@@ -414,6 +436,14 @@ struct CudaExec final : Exec {
       if (d.mode == MODE_RESIDENT)
         CK(cudaMemcpy(d.items_dev[p], d.items_host[p].data(),
                       d.items_host[p].size() * sizeof(TileItem), cudaMemcpyHostToDevice));
+    }
+    if (d.direct_ok) {
+      for (int b = 0; b < 2; ++b)
+        for (int p = 0; p < 2; ++p)
+          CK(cudaMemcpy(d.gdir_dev[b][p], d.gdir_host[b][p].data(), d.gdir_host[b][p].size() * sizeof(void*),
+                        cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(d.ystr_dev, d.ystr_host.data(), d.ystr_host.size() * sizeof(int64_t),
+                    cudaMemcpyHostToDevice));
     }
     CK(heat_configure((int)d.G.t[0], (int)d.G.t[1], d.band, d.stages, d.heat_smem, &heat_occ));
     if (d.x2_ok) {

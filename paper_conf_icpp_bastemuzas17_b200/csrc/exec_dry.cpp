@@ -41,8 +41,10 @@ struct DryExec final : Exec {
     return Status::ok();
   }
   Status heat(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
-              const TileItem* dev_items, int st) override {
+              const TileItem* dev_items, int st, int direct_bit, int nstack) override {
     d.stats.n_kernels++;
+    if (nstack < 1 || n % nstack) return make_err(TILE_ESTATE, "internal: bad tile stack");
+    const int kind = direct_bit >= 0 ? TILE_OP_KERNELD : TILE_OP_KERNEL;
     if (dev_items) {  // resident batch: items are a slice of items_host[bit]
       const int bit = dev_items >= d.items_dev[1] && d.items_dev[1] ? 1 : 0;
       const int64_t k0 = dev_items - d.items_dev[bit];
@@ -50,17 +52,17 @@ struct DryExec final : Exec {
         const TileItem& it = d.items_host[bit][(size_t)(k0 + i)];
         const int is = (int)((it.in - d.slot_base) / d.G.tile_elems);
         const int os = (int)((it.out - d.slot_base) / d.G.tile_elems);
-        put(d, TILE_OP_KERNEL, st, it.tile, is, os, rp);
+        put(d, kind, st, it.tile, is, os, rp);
       }
     } else {
-      for (int i = 0; i < n; ++i) put(d, TILE_OP_KERNEL, st, tiles[i], in[i], out[i], rp);
+      for (int i = 0; i < n; ++i) put(d, kind, st, tiles[i], in[i], out[i], rp);
     }
     return Status::ok();
   }
   Status heat2(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
                const TileItem* dev_items, int st) override {
     const size_t mark = d.trace.size();
-    Status r = heat(d, tiles, in, out, n, rp, dev_items, st);
+    Status r = heat(d, tiles, in, out, n, rp, dev_items, st, -1, 1);
     for (size_t i = mark; i < d.trace.size(); ++i) d.trace[i].kind = TILE_OP_KERNEL2;
     return r;
   }

@@ -28,21 +28,30 @@ namespace tiles {
 // ---------------------------------------------------------------- heat7
 // Producer (one thread): stage plane z of band [y0, y0+BY) of tile `in` into
 // `dst` ((BY+2) rows of tx + 2 x-ghost columns of BY), completion on `bar`.
-// z outside [0, tz) stages the band rows of the z- / z+ ghost-source face.
+// z outside [0, tz) stages the band rows of the z- / z+ ghost plane.
 // Stage layout: rows [0, BY+2) of tx (y-halo row, BY band rows, y-halo row),
 // then the x- ghost columns (D per row, 2*BY reserved) and the x+ ghost
 // columns (D per row). Faces are D layers deep; a single step reads the layer
 // nearest the tile (x-: last, x+: first; likewise y and z).
+// Ghost sources gs[f]: with ys == nullptr exported-face bases (layouts of
+// HeatParams::fexp); with ys != nullptr the direct convention of
+// HeatParams::gdir (y/z entries point at the nearest ghost layer, ys[0/1] the
+// z-stride of the y-/y+ source rows).
 __device__ __forceinline__ void stage_plane(double* dst, uint64_t* bar, const double* in,
-                                            const double* const* gs, int z, int tx, int ty,
-                                            int tz, int y0, int BY, int flags, int D) {
+                                            const double* const* gs, const int64_t* ys, int z,
+                                            int tx, int ty, int tz, int y0, int BY, int flags,
+                                            int D) {
   // interior and ghost faces are read once: optionally evict_first
   const uint64_t pol = (flags & 1) ? policy_evict_first() : policy_evict_normal();
   fence_proxy_async();
   if (z < 0 || z >= tz) {
     const uint32_t bytes = (uint32_t)BY * tx * 8;
     mbar_expect_tx(bar, bytes);
-    const double* src = z < 0 ? gs[ZM] + ((size_t)(D - 1) * ty + y0) * tx : gs[ZP] + (size_t)y0 * tx;
+    const double* src;
+    if (ys)
+      src = (z < 0 ? gs[ZM] : gs[ZP]) + (size_t)y0 * tx;
+    else
+      src = z < 0 ? gs[ZM] + ((size_t)(D - 1) * ty + y0) * tx : gs[ZP] + (size_t)y0 * tx;
     bulk_g2s_hint(dst + tx, src, bytes, bar, pol);
     return;
   }
@@ -51,9 +60,16 @@ __device__ __forceinline__ void stage_plane(double* dst, uint64_t* bar, const do
   mbar_expect_tx(bar, ((uint32_t)rows * tx + 2u * D * BY) * 8u);
   const double* plane = in + (size_t)z * ty * tx;
   bulk_g2s_hint(dst + tx, plane + (size_t)y0 * tx, row_b * BY, bar, pol);
-  const double* lo =
-      y0 > 0 ? plane + (size_t)(y0 - 1) * tx : gs[YM] + ((size_t)z * D + D - 1) * tx;
-  const double* hi = y0 + BY < ty ? plane + (size_t)(y0 + BY) * tx : gs[YP] + (size_t)z * D * tx;
+  const double* lo;
+  const double* hi;
+  if (y0 > 0)
+    lo = plane + (size_t)(y0 - 1) * tx;
+  else
+    lo = ys ? gs[YM] + (size_t)z * ys[0] : gs[YM] + ((size_t)z * D + D - 1) * tx;
+  if (y0 + BY < ty)
+    hi = plane + (size_t)(y0 + BY) * tx;
+  else
+    hi = ys ? gs[YP] + (size_t)z * ys[1] : gs[YP] + (size_t)z * D * tx;
   bulk_g2s_hint(dst, lo, row_b, bar, pol);
   bulk_g2s_hint(dst + (size_t)(BY + 1) * tx, hi, row_b, bar, pol);
   const uint32_t xb = (uint32_t)(D * BY) * 8;
@@ -61,13 +77,21 @@ __device__ __forceinline__ void stage_plane(double* dst, uint64_t* bar, const do
   bulk_g2s_hint(dst + (size_t)rows * tx + 2 * BY, gs[XP] + ((size_t)z * ty + y0) * D, xb, bar, pol);
 }
 
-// Contiguous range of (tile, band, z) planes owned by this CTA.
+__device__ __forceinline__ TileItem item_at(const HeatParams& p, int i) {
+  return p.items ? p.items[i] : p.inline_items[i];
+}
+
+// Contiguous range of (column, plane) pairs owned by this CTA. A column is an
+// item column c < lt and a band; its planes g < NZ = nstack*tz run through
+// the stacked tiles items[L*lt + c], L = g / tz (nstack = 1: one tile).
 struct PlaneRange {
   int64_t pb, pe;
+  int NZ;
   __device__ PlaneRange(const HeatParams& p) {
     const int64_t P = (int64_t)p.nitems * p.nbands * p.tz;
     pb = P * blockIdx.x / gridDim.x;
     pe = P * (blockIdx.x + 1) / gridDim.x;
+    NZ = p.nstack * p.tz;
   }
 };
 
@@ -76,6 +100,9 @@ struct PlaneRange {
 // (j < NR) of the band in EVERY plane (register z-march: z-1 and z values
 // stay in registers, 5 shared loads per pair and plane). All shared and
 // global offsets are compile-time immediates off two per-thread bases.
+// The march continues through stacked tiles (HeatParams::nstack): the plane
+// below a tile's first plane is the previous tile's last plane, already in
+// registers, so only the two ends of a CTA's run read a ghost plane.
 template <int TX, int BY, int S>
 struct Fixed {
   static constexpr int HALF = TX / 2;
@@ -114,25 +141,37 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
 
   const int ty = p.ty, tz = p.tz;
   const PlaneRange R(p);
+  const int NZ = R.NZ;
+  const double* const* gtab = p.gdir ? p.gdir : p.gsrc;
 
   if ((int)threadIdx.x >= C::NT) {  // ---------------- producer warp
     if (threadIdx.x != C::NT) return;
     uint32_t g = 0;
     for (int64_t pp = R.pb; pp < R.pe;) {
-      const int64_t col = pp / tz;
-      const int z0 = (int)(pp - col * tz);
-      const int z1 = (int)(R.pe - pp < (int64_t)(tz - z0) ? z0 + (R.pe - pp) : tz);
-      const int item_i = (int)(col / p.nbands);
-      const int y0 = (int)(col - (int64_t)item_i * p.nbands) * BY;
-      const TileItem it = p.items ? p.items[item_i] : p.inline_items[item_i];
-      const double* const* gs = p.gsrc + (size_t)it.tile * 6;
-      for (int z = z0 - 1; z <= z1; ++z, ++g) {
+      const int64_t col = pp / NZ;
+      const int g0 = (int)(pp - col * NZ);
+      const int n = (int)(R.pe - pp < (int64_t)(NZ - g0) ? R.pe - pp : NZ - g0);
+      const int icol = (int)(col / p.nbands);
+      const int y0 = (int)(col - (int64_t)icol * p.nbands) * BY;
+      // planes g0-1 .. g0+n: stacked tile L, local plane z (z = -1 / tz at the
+      // stack ends stage the z ghost planes)
+      int L = g0 / tz, z = g0 - L * tz - 1;
+      if (z < 0 && L > 0) --L, z += tz;
+      TileItem it = item_at(p, L * p.lt + icol);
+      for (int q = 0; q < n + 2; ++q, ++g, ++z) {
+        if (z == tz && L + 1 < p.nstack) {  // next stacked tile
+          ++L;
+          z = 0;
+          it = item_at(p, L * p.lt + icol);
+        }
+        const double* const* gs = gtab + (size_t)it.tile * 6;
+        const int64_t* ys = p.gdir ? p.ystr + (size_t)it.tile * 2 : nullptr;
         const int s = (int)(g % S);
         mbar_wait(&empty[s], ((g / S) & 1u) ^ 1u);
-        stage_plane(stage_base + (size_t)s * C::STAGE_ELEMS, &full[s], it.in, gs, z, TX, ty, tz,
+        stage_plane(stage_base + (size_t)s * C::STAGE_ELEMS, &full[s], it.in, gs, ys, z, TX, ty, tz,
                     y0, BY, p.cache_flags, D);
       }
-      pp += z1 - z0;
+      pp += n;
     }
     return;
   }
@@ -147,10 +186,11 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
   const double alpha = p.alpha;
   const char* sm = reinterpret_cast<const char*>(smem_raw);
   const int coff = ((r0 + 1) * TX + x) * 8;
-  const int xmoff = xlo_edge ? (C::ROWS * TX + r0 * D + D - 1) * 8 : coff - 8;
-  const int xpoff = xhi_edge ? (C::ROWS * TX + 2 * BY + r0 * D) * 8 : coff + 16;
-  const int xmj = xlo_edge ? C::RPP * D * 8 : C::RPP * TX * 8;
-  const int xpj = xhi_edge ? C::RPP * D * 8 : C::RPP * TX * 8;
+  // x ghosts: every thread reads its row neighbours (immediate offsets off
+  // cc); the two edge lanes of a warp then overwrite theirs from the staged
+  // x-ghost columns (a predicated load at an immediate offset off gcol), so
+  // no thread-dependent stride lives in the march
+  const int goff = xlo_edge ? (C::ROWS * TX + r0 * D + D - 1) * 8 : (C::ROWS * TX + 2 * BY + r0 * D) * 8;
   auto wait_g = [&](uint32_t g) { mbar_wait(&full[g % S], (g / S) & 1u); };
   auto release_g = [&](uint32_t g) {
     if (TILES_ARRIVE_PER_THREAD) {
@@ -161,32 +201,16 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
     }
   };
   uint32_t seq = 0;
+  const size_t plane = (size_t)ty * TX;
+  const bool xedge = xlo_edge || xhi_edge;
+  const int xf = xlo_edge ? XM : XP;  // the x face this thread exports, if any
 
   for (int64_t pp = R.pb; pp < R.pe;) {
-    const int64_t col = pp / tz;
-    const int z0 = (int)(pp - col * tz);
-    const int z1 = (int)(R.pe - pp < (int64_t)(tz - z0) ? z0 + (R.pe - pp) : tz);
-    const int item_i = (int)(col / p.nbands);
-    const int y0 = (int)(col - (int64_t)item_i * p.nbands) * BY;
-    const TileItem it = p.items ? p.items[item_i] : p.inline_items[item_i];
-    const int nq = z1 - z0 + 2;
-
-    const int64_t tile = it.tile;
-    const int yb = y0 + r0;
-    double* fxm = p.fexp[XM] + tile * p.face_elems[XM];
-    double* fxp = p.fexp[XP] + tile * p.face_elems[XP];
-    double* fym = p.fexp[YM] + tile * p.face_elems[YM] + x;
-    double* fyp = p.fexp[YP] + tile * p.face_elems[YP] + x;
-    double* fzm = p.fexp[ZM] + tile * p.face_elems[ZM] + (size_t)yb * TX + x;
-    double* fzp = p.fexp[ZP] + tile * p.face_elems[ZP] + (size_t)yb * TX + x;
-    double* obase = it.out + (size_t)yb * TX + x;
-    const size_t plane = (size_t)ty * TX;
-    bool ylo[C::NR], yhi[C::NR];  // rows exported to the y- / y+ faces
-#pragma unroll
-    for (int j = 0; j < C::NR; ++j) {
-      ylo[j] = yb + j * C::RPP < D;
-      yhi[j] = yb + j * C::RPP >= ty - D;
-    }
+    const int64_t col = pp / NZ;
+    const int g0 = (int)(pp - col * NZ);
+    const int n = (int)(R.pe - pp < (int64_t)(NZ - g0) ? R.pe - pp : NZ - g0);
+    const int icol = (int)(col / p.nbands);
+    const int yb = (int)(col - (int64_t)icol * p.nbands) * BY + r0;
 
     double2 zm[C::NR], zc[C::NR];
     wait_g(seq);
@@ -200,53 +224,89 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
         zc[j] = *reinterpret_cast<const double2*>(s1 + j * C::RPP * TX * 8);
       }
     }
-    release_g(seq);  // plane z0-1 is in registers now
-    for (int i = 0; i < z1 - z0; ++i) {
+    release_g(seq);  // plane g0-1 is in registers now
+    int L = g0 / tz, z = g0 - L * tz;
+    int tile = 0;
+    double* op = nullptr;  // output cell pair of row yb, plane z
+    double* fx = nullptr;  // x-face export of row yb, plane z (edge threads)
+    auto enter_tile = [&]() {
+      const TileItem it = item_at(p, L * p.lt + icol);
+      tile = it.tile;
+      op = it.out + ((size_t)z * ty + yb) * TX + x;
+      if (xedge) fx = p.fexp[xf] + (int64_t)tile * p.face_elems[xf] + ((size_t)z * ty + yb) * D;
+    };
+    enter_tile();
+    for (int i = 0; i < n; ++i) {
+      if (z == tz) {  // next stacked tile (cold)
+        ++L;
+        z = 0;
+        enter_tile();
+      }
       wait_g(seq + i + 2);
-      const int z = z0 + i;
       const char* cur = sm + (size_t)((seq + i + 1) % S) * C::STAGE_BYTES;
       const char* nxt = sm + (size_t)((seq + i + 2) % S) * C::STAGE_BYTES + coff;
       const char* cc = cur + coff;
-      const char* cxm = cur + xmoff;
-      const char* cxp = cur + xpoff;
-      double* op = obase + (size_t)z * plane;
-      const bool zlo = z < D, zhi = z >= tz - D;
+      const char* gcol = cur + goff;
+      double2 v[C::NR];
 #pragma unroll
       for (int j = 0; j < C::NR; ++j) {
         const int jo = j * C::RPP * TX * 8;
         const double2 zp = *reinterpret_cast<const double2*>(nxt + jo);
         const double2 ym = *reinterpret_cast<const double2*>(cc + jo - TX * 8);
         const double2 yp = *reinterpret_cast<const double2*>(cc + jo + TX * 8);
-        const double xm = *reinterpret_cast<const double*>(cxm + j * xmj);
-        const double xp = *reinterpret_cast<const double*>(cxp + j * xpj);
+        double xm = *reinterpret_cast<const double*>(cc + jo - 8);
+        double xp = *reinterpret_cast<const double*>(cc + jo + 16);
+        const double xg = *reinterpret_cast<const double*>(gcol + j * C::RPP * D * 8);
+        if (xlo_edge) xm = xg;
+        if (xhi_edge) xp = xg;
         const double2 c = zc[j];
-        double2 v;
-        v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm[j].x, zp.x, alpha);
-        v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm[j].y, zp.y, alpha);
-        stg2_stream(op + (size_t)j * C::RPP * TX, v);
+        v[j].x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm[j].x, zp.x, alpha);
+        v[j].y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm[j].y, zp.y, alpha);
+        stg2_stream(op + (size_t)j * C::RPP * TX, v[j]);
         zm[j] = c;
         zc[j] = zp;
-        // Epilogue: export the new boundary layers (the neighbours' ghost
-        // sources for the next step). Rare, predicated.
-        const int y = yb + j * C::RPP;
-        if (xlo_edge) {  // x = 0 (and 1): layers of the x- face
-          if (D == 1) st_hint(fxm + (size_t)z * ty + y, v.x, keep);
-          else st2_hint(fxm + ((size_t)z * ty + y) * 2, v, keep);
-        }
-        if (xhi_edge) {  // x = TX-1 (and TX-2)
-          if (D == 1) st_hint(fxp + (size_t)z * ty + y, v.y, keep);
-          else st2_hint(fxp + ((size_t)z * ty + y) * 2, v, keep);
-        }
-        if (ylo[j]) st2_hint(fym + ((size_t)z * D + y) * TX, v, keep);
-        if (yhi[j]) st2_hint(fyp + ((size_t)z * D + y - (ty - D)) * TX, v, keep);
-        if (zlo) st2_hint(fzm + (size_t)z * ty * TX + (size_t)j * C::RPP * TX, v, keep);
-        if (zhi) st2_hint(fzp + (size_t)(z - (tz - D)) * ty * TX + (size_t)j * C::RPP * TX, v, keep);
       }
       release_g(seq + i + 1);  // plane z no longer read (its centre is in registers)
+      // Epilogue: export the new boundary layers (the neighbours' ghost
+      // sources for the next step). x: the two edge lanes of every
+      // warp; y (warp-uniform rows) and z (block-uniform planes): rare.
+      if (xedge) {
+#pragma unroll
+        for (int j = 0; j < C::NR; ++j) {
+          double* q = fx + (size_t)j * C::RPP * D;
+          if (D == 1) st_hint(q, xlo_edge ? v[j].x : v[j].y, keep);
+          else st2_hint(q, v[j], keep);
+        }
+      }
+      if (p.exp_y) {
+#pragma unroll
+        for (int j = 0; j < C::NR; ++j) {
+          const int y = yb + j * C::RPP;
+          if (y < D) st2_hint(p.fexp[YM] + (int64_t)tile * p.face_elems[YM] + ((size_t)z * D + y) * TX + x, v[j], keep);
+          if (y >= ty - D)
+            st2_hint(p.fexp[YP] + (int64_t)tile * p.face_elems[YP] + ((size_t)z * D + y - (ty - D)) * TX + x, v[j], keep);
+        }
+      }
+      if (z < D && tile < p.exp_zlo_below) {
+#pragma unroll
+        for (int j = 0; j < C::NR; ++j)
+          st2_hint(p.fexp[ZM] + (int64_t)tile * p.face_elems[ZM] + ((size_t)z * ty + yb + j * C::RPP) * TX + x,
+                   v[j], keep);
+      }
+      if (z >= tz - D && tile >= p.exp_zhi_from) {
+#pragma unroll
+        for (int j = 0; j < C::NR; ++j)
+          st2_hint(p.fexp[ZP] + (int64_t)tile * p.face_elems[ZP] +
+                       ((size_t)(z - (tz - D)) * ty + yb + j * C::RPP) * TX + x,
+                   v[j], keep);
+      }
+      op += plane;
+      fx += (size_t)ty * D;
+      ++z;
     }
-    release_g(seq + nq - 1);  // plane z1 (last z+1 neighbour)
-    seq += (uint32_t)nq;
-    pp += z1 - z0;
+    release_g(seq + n + 1);  // plane g0+n (last z+1 neighbour)
+    seq += (uint32_t)(n + 2);
+    pp += n;
   }
 }
 
@@ -283,7 +343,7 @@ __global__ void __launch_bounds__(NT) heat7_generic(const __grid_constant__ Heat
     auto issue = [&](int q) {
       const uint32_t g = seq + q;
       stage_plane(stage_base + (size_t)(g % stages) * stage_elems, &bars[g % stages], it.in, gs,
-                  z0 - 1 + q, tx, ty, tz, y0, BY, p.cache_flags, D);
+                  nullptr, z0 - 1 + q, tx, ty, tz, y0, BY, p.cache_flags, D);
     };
     auto wait_q = [&](int q) {
       const uint32_t g = seq + q;
@@ -451,8 +511,15 @@ cudaError_t launch_heat7(const HeatParams& p, int stages, size_t smem, int grid,
     return cudaLaunchKernel(reinterpret_cast<const void*>(e->fn), dim3(grid), dim3(e->nt), args,
                             smem, s);
   }
+  // the general kernel takes independent tiles and exported faces only
+  if (p.gdir || p.nstack != 1 || p.lt != p.nitems) return cudaErrorInvalidValue;
   heat7_generic<kGenericThreads><<<grid, kGenericThreads, smem, s>>>(p, stages);
   return cudaGetLastError();
+}
+
+bool heat_is_fixed(int tx, int band, int stages, size_t smem) {
+  const FixedEntry* e = find_fixed_s(tx, band, stages, 1);
+  return e && e->smem == smem;
 }
 
 // -------------------------------------------------------------- sincos_iter

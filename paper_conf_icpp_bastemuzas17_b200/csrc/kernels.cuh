@@ -48,6 +48,28 @@ struct HeatParams {
   // L2 policy bits: 1 = TMA loads evict_first, 2 = face exports evict_last
   int32_t cache_flags;
   int32_t depth;  // face depth D (1 or 2): layers per face, increasing coordinate
+  // Direct ghost sources (resident single-step passes; DESIGN.md §4 "direct
+  // ghosts"): when gdir != nullptr the single-step kernels take the y and z
+  // ghosts from gdir[tile*6 + f] instead of gsrc, where the pointer is the
+  // NEAREST ghost layer itself — a neighbour tile's boundary plane / row inside
+  // its resident interior, or the nearest layer of a face (Dirichlet fixed face,
+  // slab halo) — and ystr[tile*2 + {0,1}] is the distance between consecutive
+  // z of the y- / y+ source row (ty*tx inside a tile, D*tx in a face). x ghosts
+  // always come from the exported x faces (gdir entries 0, 1 = face bases).
+  const double* const* gdir;
+  const int64_t* ystr;
+  // Stacked z-march: the items are nstack tile layers of lt items each
+  // (item (L, c) = items[L*lt + c], consecutive layers z-adjacent), and a
+  // CTA's plane range runs through a column's tiles in z, so the ghost planes
+  // between stacked tiles are the neighbour's own planes already in the ring.
+  // nstack = 1, lt = nitems: independent tiles.
+  int32_t nstack, lt;
+  // Exports: x faces always; y faces iff exp_y; the z- face of tile k iff
+  // k < exp_zlo_below, the z+ face iff k >= exp_zhi_from (direct runs export
+  // only what a face reader still needs: the slab-end layers' z faces for the
+  // halo exchange of a multi-rank domain).
+  int32_t exp_y;
+  int32_t exp_zlo_below, exp_zhi_from;
 };
 
 // Two-step pass (temporal blocking, ghost = 2): u^{s+2} from u^s in one
@@ -90,6 +112,9 @@ bool heat_plan(int tx, int ty, int max_smem, int* band, int* stages, size_t* sme
 cudaError_t heat_configure(int tx, int ty, int band, int stages, size_t smem, int* ctas_per_sm);
 cudaError_t launch_heat7(const HeatParams& p, int stages, size_t smem, int grid,
                          cudaStream_t s);
+// true if launch_heat7 runs a specialised kernel for this plan (the only
+// ones taking direct ghost sources and stacked tiles)
+bool heat_is_fixed(int tx, int band, int stages, size_t smem);
 cudaError_t launch_sincos(const SincosParams& p, int grid, cudaStream_t s);
 
 // Stream-through (trapezoid) slab kernels (kernels_slab.cu).

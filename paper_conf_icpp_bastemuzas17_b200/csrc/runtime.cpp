@@ -156,6 +156,8 @@ Status domain_setup(Domain& d) {
   const uint64_t gsrc_bytes = align_up((uint64_t)G.ntiles * 6 * sizeof(double*));
   const uint64_t items_bytes = align_up((uint64_t)G.ntiles * sizeof(TileItem));
   persist += 2 * gsrc_bytes + 2 * items_bytes;
+  const uint64_t ystr_bytes = align_up((uint64_t)G.ntiles * 2 * sizeof(int64_t));
+  persist += 4 * gsrc_bytes + ystr_bytes;  // direct ghost-source tables (resident mode)
   const uint64_t esrc_bytes = d.x2_ok ? align_up((uint64_t)G.ntiles * 12 * sizeof(EdgePtr)) : 0;
   const uint64_t mask_bytes = d.x2_ok ? align_up((uint64_t)G.ntiles) : 0;
   persist += 2 * esrc_bytes + mask_bytes;
@@ -223,6 +225,9 @@ Status domain_setup(Domain& d) {
   }
   for (int p = 0; p < 2; ++p) d.gsrc_dev[p] = reinterpret_cast<const double**>(carve(gsrc_bytes));
   for (int p = 0; p < 2; ++p) d.items_dev[p] = reinterpret_cast<TileItem*>(carve(items_bytes));
+  for (int b = 0; b < 2; ++b)
+    for (int p = 0; p < 2; ++p) d.gdir_dev[b][p] = reinterpret_cast<const double**>(carve(gsrc_bytes));
+  d.ystr_dev = reinterpret_cast<int64_t*>(carve(ystr_bytes));
   if (d.x2_ok) {
     for (int p = 0; p < 2; ++p) d.esrc_dev[p] = reinterpret_cast<EdgePtr*>(carve(esrc_bytes));
     d.fixed_mask_dev = reinterpret_cast<uint8_t*>(carve(mask_bytes));
@@ -245,6 +250,26 @@ Status domain_setup(Domain& d) {
     for (int64_t k = 0; k < G.ntiles; ++k)
       for (int f = 0; f < 6; ++f)
         if (face_source(G, k, f).kind == 1) d.fixed_mask_host[(size_t)k] |= (uint8_t)(1u << f);
+  }
+  // direct ghost sources: resident mode with a specialised single-step kernel
+  // (TILES_DIRECT=0 keeps every ghost read on the exported faces)
+  {
+    const char* e = std::getenv("TILES_DIRECT");
+    d.direct_ok = d.mode == MODE_RESIDENT && heat_is_fixed((int)G.t[0], d.band, d.stages, d.heat_smem) &&
+                  !(e && std::atoi(e) == 0);
+  }
+  if (d.direct_ok) {
+    for (int b = 0; b < 2; ++b)
+      for (int p = 0; p < 2; ++p) {
+        d.gdir_host[b][p].resize((size_t)G.ntiles * 6);
+        for (int64_t k = 0; k < G.ntiles; ++k)
+          for (int f = 0; f < 6; ++f) d.gdir_host[b][p][(size_t)k * 6 + f] = d.direct_src_ptr(k, f, b, p);
+      }
+    d.ystr_host.resize((size_t)G.ntiles * 2);
+    for (int64_t k = 0; k < G.ntiles; ++k) {
+      d.ystr_host[(size_t)k * 2] = d.direct_ystride(k, YM);
+      d.ystr_host[(size_t)k * 2 + 1] = d.direct_ystride(k, YP);
+    }
   }
   if (d.mode == MODE_RESIDENT) {
     for (int b = 0; b < 2; ++b) {
@@ -531,6 +556,8 @@ struct ResidentRun {
     const TileItem* items = d.items_dev[bit] ? d.items_dev[bit] + tile0(b) : nullptr;
     if (kpass[(size_t)s] == 2)
       r = X.heat2(d, nullptr, nullptr, nullptr, (int)ntl(b), rp, items, b.stream);
+    else if (d.direct_ok && items)  // y/z ghosts from the neighbours' interiors, stacked z-march
+      r = X.heat(d, nullptr, nullptr, nullptr, (int)ntl(b), rp, items, b.stream, bit, (int)(b.L1 - b.L0));
     else
       r = X.heat(d, nullptr, nullptr, nullptr, (int)ntl(b), rp, items, b.stream);
     if (r.bad()) return r;
@@ -816,7 +843,7 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
     d.tile_slot[k] = bit ? (int)(G.ntiles + k) : (int)k;
   }
   d.resident_valid = true;
-  d.faces_valid = false;  // faces are re-extracted by the next resident run
+  d.faces_valid = d.xfaces_valid = false;  // faces are re-extracted by the next resident run
   d.last_batches.clear();
   return Status::ok();
 }
@@ -1012,7 +1039,7 @@ static Status run_streamthrough_ooc(Domain& d, int T, int S, const OocPlan& op) 
     d.slot_owner[s] = -1;
     d.free_slots.push_back(s);
   }
-  d.faces_valid = false;
+  d.faces_valid = d.xfaces_valid = false;
   d.host_faces_valid = false;
   d.host_pending = true;
   return Status::ok();
@@ -1043,6 +1070,8 @@ static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool 
     }
   }
   int bit = d.res_bit, fp = d.face_parity;
+  // passes of two steps read every face; direct single steps only the x faces
+  const bool any_x2 = std::find(kp.begin(), kp.end(), 2) != kp.end();
   std::vector<std::pair<Batch, int>> last;  // batches of the last phase + final event
   size_t pass0 = 0;
   for (size_t pi = 0; pi < ph.size(); ++pi) {
@@ -1052,7 +1081,7 @@ static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool 
     R.kpass.assign(kp.begin() + (long)pass0, kp.begin() + (long)(pass0 + (size_t)R.T));
     pass0 += (size_t)R.T;
     R.need_load = pi == 0 && load;
-    R.need_extract = pi == 0 && !d.faces_valid;
+    R.need_extract = pi == 0 && !(any_x2 || !d.direct_ok ? d.faces_valid : d.xfaces_valid);
     R.multi = d.G.nranks > 1;
     R.entry_wait = pi > 0;
     R.bit0 = bit;
@@ -1077,7 +1106,10 @@ static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool 
   d.res_bit = bit;
   d.face_parity = fp;
   d.resident_valid = true;
-  d.faces_valid = true;
+  if (T > 0) {  // a direct last pass leaves the y/z exports stale
+    d.xfaces_valid = true;
+    d.faces_valid = kp.back() == 2 || !d.direct_ok;
+  }
   for (int64_t k = 0; k < d.G.ntiles; ++k) {
     d.tile_slot[k] = bit == 0 ? (int)k : (int)(d.G.ntiles + k);
     if (T > 0) d.tile_dirty[k] = 1;
@@ -1117,7 +1149,7 @@ static Status run_stream(Domain& d, const tile_kernel& k, int T, int S) {
     if (r.bad()) return r;
     r = X.record(d, ev_faces_init(d), 0);
     if (r.bad()) return r;
-    d.faces_valid = true;
+    d.faces_valid = d.xfaces_valid = true;
   } else if (heat) {
     r = X.record(d, ev_faces_init(d), 0);
     if (r.bad()) return r;
@@ -1292,7 +1324,7 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
       }
     if (passes > 0) {
       d.resident_valid = true;
-      d.faces_valid = false;  // interiors changed without faces
+      d.faces_valid = d.xfaces_valid = false;  // interiors changed without faces
       for (int64_t t = 0; t < d.G.ntiles; ++t) {
         d.tile_slot[t] = (int)(d.res_bit == 0 ? t : d.G.ntiles + t);
         d.tile_dirty[t] = 1;
@@ -1306,7 +1338,7 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
       r = run_streamthrough_ooc(d, steps, S, op);
     } else {
       r = run_stream(d, k, steps, S);
-      if (k.kind != TILE_KERNEL_HEAT7 && steps > 0) d.faces_valid = false;
+      if (k.kind != TILE_KERNEL_HEAT7 && steps > 0) d.faces_valid = d.xfaces_valid = false;
     }
   }
   if (r.bad()) return r;
@@ -1376,7 +1408,7 @@ Status domain_invalidate(Domain& d) {
     if (d.tile_dirty[t]) return make_err(TILE_ESTATE, "dirty tiles; call tile_sync first");
   }
   d.resident_valid = false;
-  d.faces_valid = false;
+  d.faces_valid = d.xfaces_valid = false;
   if (d.mode == MODE_STREAM) {
     for (int64_t t = 0; t < d.G.ntiles; ++t) d.tile_slot[t] = -1;
     d.free_slots.clear();

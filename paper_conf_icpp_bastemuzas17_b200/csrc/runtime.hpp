@@ -108,8 +108,12 @@ struct Exec {
   virtual Status wait(Domain& d, int ev, int stream) = 0;
   // heat over tiles [tile0, tile0+ntile) of one z-layer batch (resident) or
   // one tile (stream); in/out given by slots
+  // direct_bit >= 0: resident pass reading y/z ghosts straight from the
+  // neighbours' interiors in buffer array direct_bit (HeatParams::gdir);
+  // nstack: the items are nstack consecutive tile layers (stacked z-march)
   virtual Status heat(Domain& d, const int64_t* tiles, const int* in_slots, const int* out_slots,
-                      int nitems, int read_parity, const TileItem* dev_items, int stream) = 0;
+                      int nitems, int read_parity, const TileItem* dev_items, int stream,
+                      int direct_bit = -1, int nstack = 1) = 0;
   virtual Status sincos(Domain& d, int64_t tile, int slot, int64_t iters, int stream) = 0;
   // stream-through: one Jacobi sweep of slab planes [lo, hi) (periodic in
   // x and y) from src to dst; see SlabRef
@@ -176,6 +180,13 @@ struct Domain {
   double* dir_faces[6] = {};               // Dirichlet fixed faces
   double* halo[2][2] = {};                 // [0 = from below (z-), 1 = from above (z+)][parity]
   const double** gsrc_dev[2] = {};         // [parity] -> ntiles*6 pointers
+  // direct ghost sources (resident mode, HeatParams::gdir): [bit][parity]
+  // -> ntiles*6 nearest-layer pointers, and ntiles*2 y source z-strides
+  const double** gdir_dev[2][2] = {};
+  int64_t* ystr_dev = nullptr;
+  std::vector<const double*> gdir_host[2][2];
+  std::vector<int64_t> ystr_host;
+  bool direct_ok = false;                  // single-step resident passes read neighbours directly
   EdgePtr* esrc_dev[2] = {};               // [parity] -> ntiles*12 (D = 2 only)
   std::vector<EdgePtr> esrc_host[2];
   uint8_t* fixed_mask_dev = nullptr;       // per tile: Dirichlet faces (bit f)
@@ -198,6 +209,8 @@ struct Domain {
   int res_bit = 0;                         // resident mode: 0 -> A current, 1 -> B
   bool resident_valid = false;             // resident mode: all tiles on device
   bool faces_valid = false;                // device faces hold the current state
+  bool xfaces_valid = false;               // x faces (and, multi-rank, the slab-end z faces) do:
+                                           // what a direct single-step pass reads and leaves
   int face_parity = 0;                     // parity of the current state's faces
   int64_t use_clock = 0;
 
@@ -251,6 +264,8 @@ struct Domain {
   double* slot_ptr(int s) const { return slot_base + (int64_t)s * G.tile_elems; }
   double* host_tile(int64_t k) const { return host + k * G.tile_elems; }
   const double* face_src_ptr(int64_t id, int f, int parity) const;
+  const double* direct_src_ptr(int64_t id, int f, int bit, int parity) const;
+  int64_t direct_ystride(int64_t id, int f) const;
   EdgePtr edge_src_ptr(int64_t id, int e, int parity) const;
 };
 

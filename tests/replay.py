@@ -139,6 +139,45 @@ class Replayer:
         for f, plane in enumerate(faces_of(v, self.G.depth)):
             self.faces[(k, f, par ^ 1)] = plane
 
+    def kernel_direct(self, k, sin, sout, par):
+        """Single step with direct ghosts (TILE_OP_KERNELD): y/z ghosts of a
+        neighbour tile of this rank come from that tile's interior in the
+        same buffer array as `sin` (resident layout: tile j in slot base + j),
+        everything else from faces as in `kernel`. Exports the x faces and,
+        multi-rank, the z- face of layer 0 and the z+ face of the top layer;
+        the other exports of parity par^1 become NaN (stale), so a later read
+        of them poisons the grid."""
+        G = self.G
+        base = sin - k
+        u = self.slots[sin]
+        tz, ty, tx = u.shape
+
+        def g(f):
+            src = G.neighbour(k, f)
+            if f >= YM and src[0] == "tile":
+                nb = self.slots[base + src[1]]
+                return {YM: nb[:, -1, :], YP: nb[:, 0, :], ZM: nb[-1], ZP: nb[0]}[f]
+            return self.ghost(k, f, par)
+        e = np.zeros((tz + 2, ty + 2, tx + 2))
+        e[1:-1, 1:-1, 1:-1] = u
+        e[1:-1, 1:-1, 0] = g(XM)
+        e[1:-1, 1:-1, -1] = g(XP)
+        e[1:-1, 0, 1:-1] = g(YM)
+        e[1:-1, -1, 1:-1] = g(YP)
+        e[0, 1:-1, 1:-1] = g(ZM)
+        e[-1, 1:-1, 1:-1] = g(ZP)
+        v = oracle.heat_np(e, self.alpha, 1, oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+        self.slots[sout] = v
+        lt = G.n[0] * G.n[1]
+        multi = G.nranks > 1
+        keep = {XM, XP}
+        if multi and k < lt:
+            keep.add(ZM)
+        if multi and k >= G.ntiles - lt:
+            keep.add(ZP)
+        for f, plane in enumerate(faces_of(v, G.depth)):
+            self.faces[(k, f, par ^ 1)] = plane if f in keep else np.full(plane.shape, np.nan)
+
     # ------------------------------------------------ two-step pass (ghost 2)
     def edge_value(self, k, x, y, z, par):
         """Value of tile-local cell (x, y, z) of tile k (outside the tile in
@@ -245,6 +284,8 @@ class Replayer:
             self.kernel(a, b, c, d)
         elif name == "kernel2":
             self.kernel2(a, b, c, d)
+        elif name == "kerneld":
+            self.kernel_direct(a, b, c, d)
         elif name == "extract":
             for f, plane in enumerate(faces_of(self.slots[b], self.G.depth)):
                 self.faces[(a, f, d)] = plane

@@ -44,8 +44,12 @@ def _rank_domain(dims, td, G, r, bc, ext, u, **kw):
 @pytest.mark.parametrize("G", [2, 3, 4])
 @pytest.mark.parametrize("bc", ["periodic", "dirichlet"])
 @pytest.mark.parametrize("sched", ["resident", "stream"])
-def test_slab_replay_matches_global_oracle(G, bc, sched):
-    dims, td = (16, 8, 16 * G), (8, 4, 4)   # 4 tile layers per rank
+@pytest.mark.parametrize("td", [(8, 4, 4), (32, 8, 4)])
+def test_slab_replay_matches_global_oracle(G, bc, sched, td):
+    # 4 tile layers per rank; 32-wide tiles take the specialised kernel, so
+    # resident single steps read y/z ghosts directly (KERNELD) and export only
+    # x faces and the slab-end z faces the halo exchange sends
+    dims = (2 * td[0], 2 * td[1], 16 * G)
     u, ext, _ = _global(dims, bc)
     steps = [6, 2]   # first run: layered / whole-slab / layered phases
     kw = {"sched": sched}
@@ -80,6 +84,9 @@ def test_slab_replay_matches_global_oracle(G, bc, sched):
             traces.append(d.trace())
         assert all(sum(op[0] == "halo" for op in tr) == sum(op[0] == "halo" for op in traces[0])
                    for tr in traces)
+        if sched == "resident" and td[0] == 32:
+            assert all(any(op[0] == "kerneld" for op in tr) for tr in traces)
+            assert not any(op[0] == "kernel" for tr in traces for op in tr)
         replay_ranks(reps, traces, seed=s * 7 + G)
     out = np.concatenate([rep.grid() for rep in reps], axis=0)
     if bc == "periodic":

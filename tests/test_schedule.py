@@ -135,6 +135,30 @@ def test_resident_multiple_runs_and_dirichlet():
     _run_and_replay((16, 8, 16), (8, 4, 4), [4], 2, bc="dirichlet")
 
 
+@pytest.mark.parametrize("bc", ["periodic", "dirichlet"])
+@pytest.mark.parametrize("dims,td,ns", [((64, 16, 16), (32, 8, 8), 2), ((64, 32, 24), (32, 16, 4), 3),
+                                        ((32, 8, 8), (32, 8, 8), 1), ((64, 16, 32), (64, 8, 4), 4)])
+def test_direct_ghost_passes_replay_to_oracle(bc, dims, td, ns):
+    """Resident single steps with a specialised kernel read their y/z ghosts
+    straight from the neighbours' interiors (KERNELD) and export
+    only the x faces; the replay takes those ghosts from the neighbour slots
+    of the same buffer array and poisons every stale export, so a schedule
+    that reads a neighbour too early or too late, or a later pass that reads
+    a y/z face a direct pass did not write, breaks bit-exactness."""
+    d = _run_and_replay(dims, td, [3, 2, 1, 4], ns, seeds=(0, 1), bc=bc)
+    ops = [op[0] for op in d.trace()]
+    assert "kerneld" in ops and "kernel" not in ops
+
+
+def test_direct_then_two_step_passes_reextract_faces():
+    # a direct run leaves the y/z exports stale; a following run of two-step
+    # passes (which read every face) must re-extract them first
+    dims, td = (64, 32, 32), (32, 16, 8)
+    d = _run_and_replay(dims, td, [3, 4, 1], 2, seeds=(0, 4), ghost=2, two_step=1)
+    ops = [op[0] for op in d.trace()]
+    assert "kerneld" in ops
+
+
 def test_sync_baseline_schedule_is_one_stream():
     d = _run_and_replay((16, 16, 16), (8, 8, 8), [4], 4, sched="sync")
     assert {op[1] for op in d.trace() if op[0] in ("h2d", "kernel", "d2h")} == {0}
