@@ -593,11 +593,14 @@ def run_fig5_tiles_leg(args):
 
 def multi_domain(Tl, dist, ws, rk, transport, *args, **kw):
     """Domain for rank rk of ws. transport "peer": halo windows over CUDA IPC
-    (handles all-gathered through torch.distributed); "nccl": NCCL p2p."""
+    (handles all-gathered through torch.distributed), the stencil kernel of
+    resident steps storing its slab-end layers straight into the neighbours'
+    windows (fused, tile_options.peer_transport = 2); "peer-copy": the same
+    windows filled by copy-engine pushes after each step (1); "nccl": NCCL p2p."""
     if ws == 1:
         return Tl.Domain(*args, nranks=1, rank=0, **kw)
-    if transport == "peer":
-        dom = Tl.Domain(*args, nranks=ws, rank=rk, peer_transport=True, **kw)
+    if transport in ("peer", "peer-copy"):
+        dom = Tl.Domain(*args, nranks=ws, rank=rk, peer_transport=2 if transport == "peer" else 1, **kw)
         hs = [None] * ws
         dist.all_gather_object(hs, dom.peer_handle())
         dom.peer_connect(hs)
@@ -732,8 +735,9 @@ def main():
     ap.add_argument("--ghost", type=int, default=1,
                     help="c2/c3: ghost width; 2 = two Jacobi steps per pass (temporal blocking)")
     ap.add_argument("--two-step", type=int, default=0, help="tile_options.two_step (-1, 0, 1)")
-    ap.add_argument("--transport", default="peer", choices=["peer", "nccl"],
-                    help="N > 1 halo exchange: CUDA IPC windows (default) or NCCL p2p")
+    ap.add_argument("--transport", default="peer", choices=["peer", "peer-copy", "nccl"],
+                    help="N > 1 halo exchange: CUDA IPC windows written by the stencil kernel "
+                         "(default), the same windows written by copies, or NCCL p2p")
     ap.add_argument("--stream-through", type=int, default=0,
                     help="tile_options.stream_through (-1 never, 0 cost model, 1 when feasible)")
     args = ap.parse_args()

@@ -208,7 +208,11 @@ typedef enum {
                             ghosts: y/z ghosts read from the neighbours' interiors in the
                             buffer array holding slot b, x ghosts from the parity-d faces;
                             exports the x faces (and, multi-rank, the slab-end layers'
-                            z faces) only */
+                            z faces) only; d | 0x100: the launch also stores its slab-end
+                            z layers into the neighbour ranks' receive buffers (fused
+                            halo push, peer_transport = 2) */
+  TILE_OP_HALO_SIGNAL = 23 /* halo exchange of parity d whose data the previous kernels
+                            pushed (fused): synchronisation only */
 } tile_op_kind;
 
 typedef struct {

@@ -18,9 +18,18 @@
 //   5. wait:    my A_DN >= k and my A_UP >= k, then the caller records the
 //               halo event its boundary kernels wait for.
 // This is the rendezvous an NCCL send/recv pair provides, without a proxy
-// thread or a staging copy. Counters are stream memory operations
-// (cuStreamWriteValue32 / cuStreamWaitValue32, fetched with
-// cudaGetDriverEntryPoint), so no kernel spins and no SM is held.
+// thread or a staging copy.
+// Fused mode (tile_options.peer_transport = 2, resident direct passes): the
+// stencil kernel itself stores its slab-end z layers into the neighbours'
+// windows (HeatParams::zpush_*), so the exchange after step s only signals:
+//   mode 2 (op k): A := k at the neighbours (this step's kernels, which the
+//   halo stream follows, have pushed), R := k+1 (my step-s kernels no longer
+//   read the buffers the neighbours' next kernels will push into); wait my
+//   A >= k and R >= k+1. The first exchange of a run (mode 1) is the copy
+//   exchange above plus the R := k+1 arming for the first fused push.
+// Counters are stream memory operations (cuStreamWriteValue32 /
+// cuStreamWaitValue32, fetched with cudaGetDriverEntryPoint), so no kernel
+// spins and no SM is held.
 #include <cuda.h>
 #include <cuda_runtime.h>
 
@@ -140,7 +149,7 @@ void peer_destroy(Domain& d) {
   d.peer_window = nullptr;
 }
 
-Status peer_halo(Domain& d, int par, void* stream_v) {
+Status peer_halo(Domain& d, int par, void* stream_v, int mode) {
   if (!d.peer_connected) return make_err(TILE_ESTATE, "peer transport: call tile_peer_connect first");
   const Geometry& G = d.G;
   CUstream st = static_cast<CUstream>(stream_v);
@@ -151,6 +160,20 @@ Status peer_halo(Domain& d, int par, void* stream_v) {
   char* up = static_cast<char*>(d.peer_base[1]);  // upper neighbour's window
   void* lo_flags = lo ? lo + 4 * hb : nullptr;
   void* up_flags = up ? up + 4 * hb : nullptr;
+  if (mode == 2) {  // signal only: the kernels of this step pushed the data
+    if (up) DK(g_write(st, flag(up_flags, A_DN), k, 0));
+    if (lo) DK(g_write(st, flag(lo_flags, A_UP), k, 0));
+    if (up) DK(g_write(st, flag(up_flags, R_DN), k + 1, 0));
+    if (lo) DK(g_write(st, flag(lo_flags, R_UP), k + 1, 0));
+    if (lo) DK(g_wait(st, flag(d.peer_flags, A_DN), k, d.peer_wait_flags));
+    if (up) DK(g_wait(st, flag(d.peer_flags, A_UP), k, d.peer_wait_flags));
+    if (up) DK(g_wait(st, flag(d.peer_flags, R_UP), k + 1, d.peer_wait_flags));
+    if (lo) DK(g_wait(st, flag(d.peer_flags, R_DN), k + 1, d.peer_wait_flags));
+    const size_t cnt = (size_t)d.G.layer_tiles * d.G.face_elems[ZM];
+    if (d.measure != TILE_MEASURE_COMP_ONLY)
+      d.stats.bytes_halo += (uint64_t)((up ? 1 : 0) + (lo ? 1 : 0)) * cnt * 8;
+    return Status::ok();
+  }
   // 1. ready to receive exchange k
   if (up) DK(g_write(st, flag(up_flags, R_DN), k, 0));
   if (lo) DK(g_write(st, flag(lo_flags, R_UP), k, 0));
@@ -167,9 +190,17 @@ Status peer_halo(Domain& d, int par, void* stream_v) {
   }
   if (up) DK(g_write(st, flag(up_flags, A_DN), k, 0));
   if (lo) DK(g_write(st, flag(lo_flags, A_UP), k, 0));
+  if (mode == 1) {  // arm the first fused push: nothing reads the other parity yet
+    if (up) DK(g_write(st, flag(up_flags, R_DN), k + 1, 0));
+    if (lo) DK(g_write(st, flag(lo_flags, R_UP), k + 1, 0));
+  }
   // 5. my ghosts have arrived
   if (lo) DK(g_wait(st, flag(d.peer_flags, A_DN), k, d.peer_wait_flags));
   if (up) DK(g_wait(st, flag(d.peer_flags, A_UP), k, d.peer_wait_flags));
+  if (mode == 1) {
+    if (up) DK(g_wait(st, flag(d.peer_flags, R_UP), k + 1, d.peer_wait_flags));
+    if (lo) DK(g_wait(st, flag(d.peer_flags, R_DN), k + 1, d.peer_wait_flags));
+  }
   return Status::ok();
 }
 

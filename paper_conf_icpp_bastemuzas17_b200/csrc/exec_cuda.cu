@@ -166,6 +166,16 @@ struct CudaExec final : Exec {
       const bool multi = d.G.nranks > 1;
       p.exp_zlo_below = multi ? (int32_t)d.G.layer_tiles : 0;
       p.exp_zhi_from = multi ? (int32_t)(d.G.ntiles - d.G.layer_tiles) : INT32_MAX;
+      if (multi && d.peer_fused && d.peer_connected && d.measure != TILE_MEASURE_COMP_ONLY) {
+        // write parity rp^1 of the neighbours' receive buffers: the lower
+        // rank's halo[1] (from above) and the upper rank's halo[0]
+        const int wp = rp ^ 1;
+        const uint64_t hb = d.peer_halo_bytes;
+        char* lo = static_cast<char*>(d.peer_base[0]);
+        char* up = static_cast<char*>(d.peer_base[1]);
+        p.zpush_lo = lo ? reinterpret_cast<double*>(lo + (2 + wp) * hb) : nullptr;
+        p.zpush_hi = up ? reinterpret_cast<double*>(up + (0 + wp) * hb) : nullptr;
+      }
     } else {
       p.gdir = nullptr;
       p.ystr = nullptr;
@@ -358,7 +368,7 @@ struct CudaExec final : Exec {
     }
     return Status::ok();
   }
-  Status halo(Domain& d, int par, int st) override {
+  Status halo(Domain& d, int par, int st, int mode) override {
     if (d.opt.local_group) {
       if (!local_ready) CK(cudaEventCreateWithFlags(&local_ready, cudaEventDisableTiming));
       Status r = local_halo(d, par, S(st), local_ready);
@@ -366,7 +376,7 @@ struct CudaExec final : Exec {
       d.stats.n_halo++;
       return Status::ok();
     }
-    Status r = d.opt.peer_transport ? peer_halo(d, par, S(st)) : nccl_halo(d, par, S(st));
+    Status r = d.opt.peer_transport ? peer_halo(d, par, S(st), mode) : nccl_halo(d, par, S(st));
     if (r.bad()) return r;
     d.stats.n_halo++;
     return Status::ok();

@@ -45,6 +45,9 @@ struct DryExec final : Exec {
     d.stats.n_kernels++;
     if (nstack < 1 || n % nstack) return make_err(TILE_ESTATE, "internal: bad tile stack");
     const int kind = direct_bit >= 0 ? TILE_OP_KERNELD : TILE_OP_KERNEL;
+    // d of a direct op: read parity | 0x100 when the launch pushes its slab-end
+    // z exports into the neighbour ranks' receive buffers (fused halo)
+    const int push = direct_bit >= 0 && d.G.nranks > 1 && d.peer_fused ? 0x100 : 0;
     if (dev_items) {  // resident batch: items are a slice of items_host[bit]
       const int bit = dev_items >= d.items_dev[1] && d.items_dev[1] ? 1 : 0;
       const int64_t k0 = dev_items - d.items_dev[bit];
@@ -52,10 +55,10 @@ struct DryExec final : Exec {
         const TileItem& it = d.items_host[bit][(size_t)(k0 + i)];
         const int is = (int)((it.in - d.slot_base) / d.G.tile_elems);
         const int os = (int)((it.out - d.slot_base) / d.G.tile_elems);
-        put(d, kind, st, it.tile, is, os, rp);
+        put(d, kind, st, it.tile, is, os, rp | push);
       }
     } else {
-      for (int i = 0; i < n; ++i) put(d, kind, st, tiles[i], in[i], out[i], rp);
+      for (int i = 0; i < n; ++i) put(d, kind, st, tiles[i], in[i], out[i], rp | push);
     }
     return Status::ok();
   }
@@ -127,10 +130,10 @@ struct DryExec final : Exec {
     put(d, TILE_OP_FACES_H2D, st, 0, 0, 0, par);
     return Status::ok();
   }
-  Status halo(Domain& d, int par, int st) override {
+  Status halo(Domain& d, int par, int st, int mode) override {
     d.stats.n_halo++;
     d.stats.bytes_halo += 2ull * d.G.layer_tiles * d.G.face_elems[ZM] * 8;
-    put(d, TILE_OP_HALO, st, 0, 0, 0, par);
+    put(d, mode == 2 ? TILE_OP_HALO_SIGNAL : TILE_OP_HALO, st, mode, 0, 0, par);
     return Status::ok();
   }
   Status note(Domain& d, int kind, int64_t a, int64_t b, int st) override {

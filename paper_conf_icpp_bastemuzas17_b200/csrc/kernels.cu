@@ -203,6 +203,7 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
   uint32_t seq = 0;
   const size_t plane = (size_t)ty * TX;
   const bool xedge = xlo_edge || xhi_edge;
+  bool pushed = false;  // this thread stored halo layers into a neighbour rank's window
   const int xf = xlo_edge ? XM : XP;  // the x face this thread exports, if any
 
   for (int64_t pp = R.pb; pp < R.pe;) {
@@ -288,17 +289,28 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
         }
       }
       if (z < D && tile < p.exp_zlo_below) {
+        const size_t e = ((size_t)z * ty + yb) * TX + x;
 #pragma unroll
         for (int j = 0; j < C::NR; ++j)
-          st2_hint(p.fexp[ZM] + (int64_t)tile * p.face_elems[ZM] + ((size_t)z * ty + yb + j * C::RPP) * TX + x,
-                   v[j], keep);
+          st2_hint(p.fexp[ZM] + (int64_t)tile * p.face_elems[ZM] + e + (size_t)j * C::RPP * TX, v[j], keep);
+        if (p.zpush_lo) {  // fused halo push into the lower rank's window
+          pushed = true;
+          double* q = p.zpush_lo + (int64_t)tile * p.face_elems[ZM] + e;
+#pragma unroll
+          for (int j = 0; j < C::NR; ++j) *reinterpret_cast<double2*>(q + (size_t)j * C::RPP * TX) = v[j];
+        }
       }
       if (z >= tz - D && tile >= p.exp_zhi_from) {
+        const size_t e = ((size_t)(z - (tz - D)) * ty + yb) * TX + x;
 #pragma unroll
         for (int j = 0; j < C::NR; ++j)
-          st2_hint(p.fexp[ZP] + (int64_t)tile * p.face_elems[ZP] +
-                       ((size_t)(z - (tz - D)) * ty + yb + j * C::RPP) * TX + x,
-                   v[j], keep);
+          st2_hint(p.fexp[ZP] + (int64_t)tile * p.face_elems[ZP] + e + (size_t)j * C::RPP * TX, v[j], keep);
+        if (p.zpush_hi) {  // fused halo push into the upper rank's window
+          pushed = true;
+          double* q = p.zpush_hi + (int64_t)(tile - p.exp_zhi_from) * p.face_elems[ZP] + e;
+#pragma unroll
+          for (int j = 0; j < C::NR; ++j) *reinterpret_cast<double2*>(q + (size_t)j * C::RPP * TX) = v[j];
+        }
       }
       op += plane;
       fx += (size_t)ty * D;
@@ -308,6 +320,9 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
     seq += (uint32_t)(n + 2);
     pp += n;
   }
+  // pushed halo layers visible system-wide (the neighbour ranks' GPUs) before
+  // the halo stream's arrival counter, written after this kernel, is
+  if (pushed) asm volatile("fence.acq_rel.sys;" ::: "memory");
 }
 
 // ---- general kernel: any even tile width / band (runtime shape). Every

@@ -70,6 +70,14 @@ struct HeatParams {
   // halo exchange of a multi-rank domain).
   int32_t exp_y;
   int32_t exp_zlo_below, exp_zhi_from;
+  // Fused halo push (multi-rank peer transport): when non-null,
+  // the z- exports of tiles k < exp_zlo_below are ALSO stored straight into
+  // the lower neighbour rank's receive window at zpush_lo + k*face_elems[ZM],
+  // and the z+ exports of tiles k >= exp_zhi_from into the upper neighbour's
+  // at zpush_hi + (k - exp_zhi_from)*face_elems[ZP] (peer memory over
+  // NVLink / NVSwitch); the halo op then only signals.
+  double* zpush_lo;
+  double* zpush_hi;
 };
 
 // Two-step pass (temporal blocking, ghost = 2): u^{s+2} from u^s in one

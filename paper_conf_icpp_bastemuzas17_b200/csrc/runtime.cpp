@@ -258,6 +258,8 @@ Status domain_setup(Domain& d) {
     d.direct_ok = d.mode == MODE_RESIDENT && heat_is_fixed((int)G.t[0], d.band, d.stages, d.heat_smem) &&
                   !(e && std::atoi(e) == 0);
   }
+  // fused halo push: peer transport mode 2 with direct passes (multi-rank resident)
+  d.peer_fused = multi && d.opt.peer_transport == 2 && d.direct_ok;
   if (d.direct_ok) {
     for (int b = 0; b < 2; ++b)
       for (int p = 0; p < 2; ++p) {
@@ -573,7 +575,9 @@ struct ResidentRun {
       r = X.wait(d, ev_layer(d, (int64_t)i, s & 1), hs);
       if (r.bad()) return r;
     }
-    r = X.halo(d, fp0 ^ ((s + 1) & 1), hs);
+    // fused peer transport: after a step, the kernels have pushed the data
+    const int mode = !d.peer_fused ? 0 : s < 0 ? 1 : 2;
+    r = X.halo(d, fp0 ^ ((s + 1) & 1), hs, mode);
     if (r.bad()) return r;
     return X.record(d, ev_halo(d, s & 1), hs);
   }
@@ -693,14 +697,46 @@ struct StreamPlan {
 };
 
 // Units in z order: each tile layer cut into tz / un pieces of un planes
-// (un >= T: a unit's halo lies in its two neighbour units). Thin first/last
-// units (a shorter pipeline fill and drain) were measured and gained nothing
-// at C2 (25.6 ms either way): the run is link-rate bound.
-static std::vector<UnitDef> make_units(const Geometry& G, int64_t un, int T) {
-  (void)T;
+// (un >= T: a unit's halo lies in its two neighbour units). The H2D order
+// is U-1, 0, 1, ..., U-2: the first D2H waits for the uploads of U-1, 0
+// and 1 (the fill), and the last upload (unit U-2) gates the computes and
+// D2Hs of units U-3, U-2 and U-1, which all follow it (the drain). The last
+// layer's tail is therefore cut into `thin` units of T planes (the smallest
+// a unit may be) and the first layer's head into thin - 1 (<= 2) of them
+// (TILES_ST_THIN, default 3; 0 = uniform units).
+static int st_thin_default() {
+  static const int thin = [] {
+    const char* e = getenv("TILES_ST_THIN");
+    return e ? std::max(0, atoi(e)) : 3;
+  }();
+  return thin;
+}
+
+static std::vector<UnitDef> make_units(const Geometry& G, int64_t un, int T, int thin) {
   std::vector<UnitDef> v;
-  for (int64_t L = 0; L < G.n[2]; ++L)
-    for (int64_t p = 0; p < G.t[2]; p += un) v.push_back({L, p, un});
+  const int64_t tz = G.t[2];
+  const bool cut = thin > 0 && un > T && G.n[2] * (tz / un) >= 4 && G.n[2] >= 2;
+  for (int64_t L = 0; L < G.n[2]; ++L) {
+    const bool last = L == G.n[2] - 1;
+    int64_t tail = 0, head = 0;  // planes of the layer cut into thin units
+    if (cut && last) {
+      tail = (int64_t)thin * T;
+      while (tail > 0 && tz - tail < T) tail -= T;  // the rest stays a unit of >= T planes
+    }
+    if (cut && L == 0) {  // the fill: units 0 and 1 (with U-1) gate the first D2H
+      head = std::min<int64_t>(2, thin - 1) * T;
+      while (head > 0 && tz - head < T) head -= T;
+    }
+    int64_t p = 0;
+    for (; p < head; p += T) v.push_back({L, p, (int64_t)T});
+    for (; p + un <= tz - tail; p += un) v.push_back({L, p, un});
+    if (p < tz - tail) {  // remainder: its own unit if >= T planes, else extends the previous one
+      if (tz - tail - p < T && !v.empty() && v.back().layer == L) v.back().np += tz - tail - p;
+      else v.push_back({L, p, tz - tail - p});
+      p = tz - tail;
+    }
+    for (; p < tz; p += T) v.push_back({L, p, (int64_t)T});
+  }
   return v;
 }
 
@@ -742,14 +778,18 @@ static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
   if (d.opt.stream_through == 0 && best > 2.0 * nz + 0.011 * nz * Td) return false;
   if (G.l[2] / unit + 4 > G.ntiles) unit = G.t[2];  // event budget (one per unit)
   sp->unit = unit;
-  sp->u = make_units(G, unit, T);
-  if ((int64_t)sp->u.size() > G.ntiles) sp->u = make_units(G, G.t[2], T);
-  sp->units = (int64_t)sp->u.size();
-  int64_t mx = 0;
-  for (const auto& x : sp->u) mx = std::max(mx, x.np);
-  sp->slab_tiles = ((mx + 2 * (int64_t)T) * plane + G.tile_elems - 1) / G.tile_elems;
-  sp->sub_tiles = (G.layer_tiles * mx * G.t[0] * G.t[1] + G.tile_elems - 1) / G.tile_elems;
-  return 2 * sp->slab_tiles + 3 * sp->sub_tiles <= G.ntiles;
+  // thin tail units first; uniform units if those do not fit
+  for (int thin : {st_thin_default(), 0}) {
+    sp->u = make_units(G, unit, T, thin);
+    if ((int64_t)sp->u.size() > G.ntiles) sp->u = make_units(G, G.t[2], T, 0);
+    sp->units = (int64_t)sp->u.size();
+    int64_t mx = 0;
+    for (const auto& x : sp->u) mx = std::max(mx, x.np);
+    sp->slab_tiles = ((mx + 2 * (int64_t)T) * plane + G.tile_elems - 1) / G.tile_elems;
+    sp->sub_tiles = (G.layer_tiles * mx * G.t[0] * G.t[1] + G.tile_elems - 1) / G.tile_elems;
+    if (2 * sp->slab_tiles + 3 * sp->sub_tiles <= G.ntiles) return true;
+  }
+  return false;
 }
 
 // Stream-through over units of `unit` planes (a unit is a slice of one tile

@@ -137,7 +137,10 @@ struct Exec {
   virtual Status extract(Domain& d, int64_t tile0, int64_t ntile, int slot0, int parity,
                          const TileItem* dev_items, int stream) = 0;
   virtual Status faces_h2d(Domain& d, int parity, int stream) = 0;
-  virtual Status halo(Domain& d, int parity, int stream) = 0;
+  // mode (peer transport): 0 = push the faces with copies;
+  // 1 = copies, and arm the next exchange, whose data the kernels push
+  // (fused); 2 = signal only: the previous step's kernels pushed the data
+  virtual Status halo(Domain& d, int parity, int stream, int mode = 0) = 0;
   virtual Status note(Domain& d, int kind, int64_t a, int64_t b, int stream) = 0;  // trace-only ops
   virtual Status sync_all(Domain& d) = 0;
   // resources
@@ -237,6 +240,7 @@ struct Domain {
   unsigned int peer_wait_flags = 0;
   uint32_t peer_k = 0;
   bool peer_connected = false;
+  bool peer_fused = false;                 // resident direct passes push z halos from the kernel
 
   // kernel plan
   int band = 0, stages = 0, heat_grid = 0, sm_count = 148;
@@ -299,7 +303,7 @@ Status local_halo(Domain& d, int parity, void* stream, void* ready_event);
 Status peer_setup(Domain& d, uint64_t halo_bytes);
 Status peer_handle(const Domain& d, void* out64);
 Status peer_connect(Domain& d, const void* handles, int n);
-Status peer_halo(Domain& d, int parity, void* stream);
+Status peer_halo(Domain& d, int parity, void* stream, int mode);
 void peer_destroy(Domain& d);
 
 }  // namespace tiles

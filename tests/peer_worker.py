@@ -7,7 +7,7 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def run(r, G, dims, td, bc, sched, budget, runs, seed, conn):
+def run(r, G, dims, td, bc, sched, budget, runs, seed, conn, transport=1):
     sys.path.insert(0, ROOT)
     try:
         import synth
@@ -17,7 +17,7 @@ def run(r, G, dims, td, bc, sched, budget, runs, seed, conn):
         kw = {"sched": sched}
         if budget:
             kw["device_budget_bytes"] = budget
-        with T.Domain(dims, td, bc=bc, nranks=G, rank=r, peer_transport=True, device=0, **kw) as d:
+        with T.Domain(dims, td, bc=bc, nranks=G, rank=r, peer_transport=transport, device=0, **kw) as d:
             conn.send(("handle", d.peer_handle()))
             kind, handles = conn.recv()
             d.peer_connect(handles)

@@ -96,6 +96,7 @@ class Replayer:
         self.faces = {}
         self.halo = {}
         self.comm = comm
+        self.peers = {}    # rank -> Replayer (joint multi-rank replay, fused pushes)
 
     def dirichlet_face(self, k, f):
         G = self.G
@@ -139,7 +140,7 @@ class Replayer:
         for f, plane in enumerate(faces_of(v, self.G.depth)):
             self.faces[(k, f, par ^ 1)] = plane
 
-    def kernel_direct(self, k, sin, sout, par):
+    def kernel_direct(self, k, sin, sout, par, push=False):
         """Single step with direct ghosts (TILE_OP_KERNELD): y/z ghosts of a
         neighbour tile of this rank come from that tile's interior in the
         same buffer array as `sin` (resident layout: tile j in slot base + j),
@@ -177,6 +178,20 @@ class Replayer:
             keep.add(ZP)
         for f, plane in enumerate(faces_of(v, G.depth)):
             self.faces[(k, f, par ^ 1)] = plane if f in keep else np.full(plane.shape, np.nan)
+        if push:  # fused halo push straight into the neighbour ranks' receive buffers
+            up, dn = halo_peers(G)
+            fz = faces_of(v, G.depth)
+            if dn is not None and k < lt:
+                self.peers[dn].push((1, par ^ 1), k, fz[ZM])
+            if up is not None and k >= G.ntiles - lt:
+                self.peers[up].push((0, par ^ 1), k - (G.ntiles - lt), fz[ZP])
+
+    def push(self, key, pos, plane):
+        G = self.G
+        lt = G.n[0] * G.n[1]
+        cur = list(self.halo.get(key, [None] * lt))
+        cur[pos] = plane.copy()
+        self.halo[key] = cur
 
     # ------------------------------------------------ two-step pass (ghost 2)
     def edge_value(self, k, x, y, z, par):
@@ -285,7 +300,7 @@ class Replayer:
         elif name == "kernel2":
             self.kernel2(a, b, c, d)
         elif name == "kerneld":
-            self.kernel_direct(a, b, c, d)
+            self.kernel_direct(a, b, c, d & 0xff, bool(d & 0x100))
         elif name == "extract":
             for f, plane in enumerate(faces_of(self.slots[b], self.G.depth)):
                 self.faces[(a, f, d)] = plane
@@ -469,6 +484,8 @@ def replay_ranks(reps, traces, seed):
     """Joint random replay of several ranks' traces; the k-th halo op of
     every rank executes together (a collective)."""
     rng = random.Random(seed)
+    for rep in reps:
+        rep.peers = {r: x for r, x in enumerate(reps)}
     state = []
     for rep, tr in zip(reps, traces):
         last_rec, bound = {}, {}
@@ -495,7 +512,7 @@ def replay_ranks(reps, traces, seed):
                 op = tr[i]
                 if op[0] == "wait" and st["bound"][i] is not None and st["bound"][i] not in st["done"]:
                     continue
-                if op[0] == "halo":
+                if op[0] in ("halo", "halo_signal"):
                     halo_heads[r] = (s, i)
                 else:
                     ready.append((r, s, i))
@@ -506,13 +523,21 @@ def replay_ranks(reps, traces, seed):
         pick = rng.choice(ready)
         if pick[0] == "halo":
             par = traces[0][halo_heads[0][1]][5]
+            kind = traces[0][halo_heads[0][1]][0]
             payload = [halo_payload(rep, par) for rep in reps]
             for r, rep in enumerate(reps):
                 assert traces[r][halo_heads[r][1]][5] == par
+                assert traces[r][halo_heads[r][1]][0] == kind
                 up, dn = halo_peers(rep.G)
-                if dn is not None:
+                if kind == "halo_signal":
+                    # fused: the kernels pushed the layers; the collective only orders
+                    for key in ((0, par), (1, par)):
+                        if (key == (0, par) and dn is not None) or (key == (1, par) and up is not None):
+                            assert key in rep.halo and all(x is not None for x in rep.halo[key]), \
+                                "fused halo: a boundary layer was not pushed before the signal"
+                elif dn is not None:
                     rep.halo[(0, par)] = payload[dn][0]   # rank below's top layer
-                if up is not None:
+                if kind == "halo" and up is not None:
                     rep.halo[(1, par)] = payload[up][1]   # rank above's bottom layer
                 s, i = halo_heads[r]
                 state[r]["done"].add(i)

@@ -78,14 +78,20 @@ def test_local_group_slabs_bit_exact(G, bc, sched, runs):
     assert np.array_equal(got, ref), np.abs(got - ref).max()
 
 
-@pytest.mark.parametrize("G,bc,sched,runs", [(2, "periodic", "resident", [5]), (3, "periodic", "resident", [4, 3]),
-                                             (2, "dirichlet", "resident", [3]), (4, "periodic", "stream", [3]),
-                                             (3, "dirichlet", "stream", [2, 2])])
-def test_peer_transport_processes_bit_exact(G, bc, sched, runs):
+@pytest.mark.parametrize("G,bc,sched,runs,transport", [
+    (2, "periodic", "resident", [5], 1), (3, "periodic", "resident", [4, 3], 1),
+    (2, "dirichlet", "resident", [3], 1), (4, "periodic", "stream", [3], 1),
+    (3, "dirichlet", "stream", [2, 2], 1),
+    (2, "periodic", "resident", [7, 5], 2), (3, "periodic", "resident", [6, 9], 2),
+    (4, "dirichlet", "resident", [8], 2), (2, "dirichlet", "resident", [4, 4], 2)])
+def test_peer_transport_processes_bit_exact(G, bc, sched, runs, transport):
     """Peer transport (tile_options.peer_transport): one PROCESS per rank, all
     on the one GPU of the pool (CUDA IPC works between processes on a device
     as between devices); the halo exchange is the IPC window push with
-    stream-memory-op counters, no NCCL. Bit-exact against the oracle."""
+    stream-memory-op counters, no NCCL. transport 2 = fused: the stencil
+    kernel of every resident step stores its slab-end layers straight into
+    the neighbours' windows and the exchange only signals. Bit-exact against
+    the oracle."""
     import multiprocessing as mp
     from tests import peer_worker
     dims, td = (64, 32, 16 * G), (32, 16, 8)
@@ -95,7 +101,7 @@ def test_peer_transport_processes_bit_exact(G, bc, sched, runs):
     pipes, procs = [], []
     for r in range(G):
         a, b = ctx.Pipe()
-        p = ctx.Process(target=peer_worker.run, args=(r, G, dims, td, bc, sched, budget, runs, 42, b))
+        p = ctx.Process(target=peer_worker.run, args=(r, G, dims, td, bc, sched, budget, runs, 42, b, transport))
         p.start()
         pipes.append(a)
         procs.append(p)

@@ -44,15 +44,23 @@ def _rank_domain(dims, td, G, r, bc, ext, u, **kw):
 @pytest.mark.parametrize("G", [2, 3, 4])
 @pytest.mark.parametrize("bc", ["periodic", "dirichlet"])
 @pytest.mark.parametrize("sched", ["resident", "stream"])
-@pytest.mark.parametrize("td", [(8, 4, 4), (32, 8, 4)])
-def test_slab_replay_matches_global_oracle(G, bc, sched, td):
+@pytest.mark.parametrize("td,fused", [((8, 4, 4), 0), ((32, 8, 4), 0), ((32, 8, 4), 2)])
+def test_slab_replay_matches_global_oracle(G, bc, sched, td, fused):
     # 4 tile layers per rank; 32-wide tiles take the specialised kernel, so
     # resident single steps read y/z ghosts directly (KERNELD) and export only
-    # x faces and the slab-end z faces the halo exchange sends
+    # x faces and the slab-end z faces the halo exchange sends. fused = 2: the
+    # peer transport's fused mode, where those kernels also store the slab-end
+    # layers straight into the neighbour ranks' receive buffers and the halo
+    # op after a step only synchronises (the replay applies each push when its
+    # kernel executes, so a push racing a reader breaks bit-exactness)
+    if fused and sched != "resident":
+        pytest.skip("fused pushes are a resident direct-pass feature")
     dims = (2 * td[0], 2 * td[1], 16 * G)
     u, ext, _ = _global(dims, bc)
-    steps = [6, 2]   # first run: layered / whole-slab / layered phases
+    steps = [6, 5]   # first run: layered / whole-slab / layered phases; second: one phase
     kw = {"sched": sched}
+    if fused:
+        kw["peer_transport"] = fused
     if sched == "stream":
         kw["device_budget_bytes"] = 1  # replaced below by the minimum budget
     doms, reps = [], []
@@ -87,6 +95,9 @@ def test_slab_replay_matches_global_oracle(G, bc, sched, td):
         if sched == "resident" and td[0] == 32:
             assert all(any(op[0] == "kerneld" for op in tr) for tr in traces)
             assert not any(op[0] == "kernel" for tr in traces for op in tr)
+            pushes = [op for tr in traces for op in tr if op[0] == "kerneld" and op[5] & 0x100]
+            signals = [op for tr in traces for op in tr if op[0] == "halo_signal"]
+            assert bool(pushes) == bool(fused) and bool(signals) == bool(fused)
         replay_ranks(reps, traces, seed=s * 7 + G)
     out = np.concatenate([rep.grid() for rep in reps], axis=0)
     if bc == "periodic":
