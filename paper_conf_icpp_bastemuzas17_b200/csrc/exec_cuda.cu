@@ -131,8 +131,19 @@ struct CudaExec final : Exec {
     return Status::ok();
   }
   Status heat(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
-              const TileItem* dev_items, int st, int direct_bit, int nstack) override {
+              const TileItem* dev_items, int st, int direct_bit, int nstack, int nsteps) override {
     if (d.measure == TILE_MEASURE_XFER_ONLY || n == 0) return Status::ok();
+    if (nsteps > 1 && (!coop || direct_bit < 0 || !dev_items || (int64_t)sms * heat_occ > kMaxProgCtas)) {
+      // no persistent launch possible: one launch per step (buffers and face
+      // parities alternate)
+      const int64_t off = dev_items - d.items_dev[direct_bit];
+      for (int s = 0; s < nsteps; ++s) {
+        const int b = direct_bit ^ (s & 1);
+        Status r = heat(d, tiles, in, out, n, rp ^ (s & 1), d.items_dev[b] + off, st, b, nstack, 1);
+        if (r.bad()) return r;
+      }
+      return Status::ok();
+    }
     HeatParams p{};
     p.tx = (int)d.G.t[0];
     p.ty = (int)d.G.t[1];
@@ -187,11 +198,27 @@ struct CudaExec final : Exec {
     const int64_t planes = (int64_t)n * p.nbands * p.tz;
     int64_t grid = (int64_t)sms * heat_occ;
     grid = std::max<int64_t>(1, std::min<int64_t>(grid, (planes + 3) / 4));
+    p.nsteps = 1;
+    if (nsteps > 1) {  // one persistent launch for all steps (CTA progress counters)
+      const int b1 = direct_bit ^ 1;
+      p.nsteps = nsteps;
+      p.ntx = (int32_t)d.G.n[0];
+      p.nty = (int32_t)d.G.n[1];
+      p.epoch = d.prog_epoch;
+      p.prog = d.prog_dev;
+      p.items_odd = d.items_dev[b1] + (dev_items - d.items_dev[direct_bit]);
+      p.gdir_odd = d.gdir_dev[b1][rp ^ 1];
+      for (int f = 0; f < 6; ++f) p.fexp_odd[f] = d.faces[f][rp];
+      d.prog_epoch += (uint32_t)(nsteps - 1);  // barrier rounds of this launch
+      if (d.prog_grid && d.prog_grid != grid) return make_err(TILE_ESTATE, "internal: persistent grid changed");
+      d.prog_grid = grid;
+    }
     Status r = timed(d, st, [&] { return launch_heat7(p, d.stages, d.heat_smem, (int)grid, S(st)); });
     if (r.bad()) return r;
     d.stats.n_kernels++;
     return Status::ok();
   }
+  int coop = 0;  // cudaDevAttrCooperativeLaunch
   SlabView slab_view(Domain& d, const SlabRef& r, int lo) {
     const Geometry& G = d.G;
     SlabView v{};
@@ -456,6 +483,12 @@ struct CudaExec final : Exec {
                     cudaMemcpyHostToDevice));
     }
     CK(heat_configure((int)d.G.t[0], (int)d.G.t[1], d.band, d.stages, d.heat_smem, &heat_occ));
+    {
+      int dev = 0;
+      CK(cudaGetDevice(&dev));
+      CK(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev));
+    }
+    CK(cudaMemset(d.prog_dev, 0, (size_t)kMaxProgCtas * sizeof(unsigned long long)));
     if (d.x2_ok) {
       CK(heat2_configure((int)d.G.t[0], d.band2, d.heat2_smem, &heat2_occ));
       if (heat2_occ < 1) {  // cannot be resident (e.g. profiler-reserved shared memory)

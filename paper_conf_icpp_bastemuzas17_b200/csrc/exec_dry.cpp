@@ -41,7 +41,17 @@ struct DryExec final : Exec {
     return Status::ok();
   }
   Status heat(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
-              const TileItem* dev_items, int st, int direct_bit, int nstack) override {
+              const TileItem* dev_items, int st, int direct_bit, int nstack, int nsteps) override {
+    if (nsteps > 1) {  // a persistent launch: the same ops as nsteps single steps
+      const int64_t off = dev_items - d.items_dev[direct_bit];
+      for (int s = 0; s < nsteps; ++s) {
+        const int b = direct_bit ^ (s & 1);
+        Status r = heat(d, tiles, in, out, n, rp ^ (s & 1), d.items_dev[b] + off, st, b, nstack, 1);
+        if (r.bad()) return r;
+      }
+      d.stats.n_kernels -= (uint64_t)nsteps - 1;  // one launch
+      return Status::ok();
+    }
     d.stats.n_kernels++;
     if (nstack < 1 || n % nstack) return make_err(TILE_ESTATE, "internal: bad tile stack");
     const int kind = direct_bit >= 0 ? TILE_OP_KERNELD : TILE_OP_KERNEL;
@@ -65,7 +75,7 @@ struct DryExec final : Exec {
   Status heat2(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
                const TileItem* dev_items, int st) override {
     const size_t mark = d.trace.size();
-    Status r = heat(d, tiles, in, out, n, rp, dev_items, st, -1, 1);
+    Status r = heat(d, tiles, in, out, n, rp, dev_items, st, -1, 1, 1);
     for (size_t i = mark; i < d.trace.size(); ++i) d.trace[i].kind = TILE_OP_KERNEL2;
     return r;
   }

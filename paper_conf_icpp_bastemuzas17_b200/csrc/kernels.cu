@@ -85,15 +85,16 @@ __device__ __forceinline__ TileItem item_at(const HeatParams& p, int i) {
 // item column c < lt and a band; its planes g < NZ = nstack*tz run through
 // the stacked tiles items[L*lt + c], L = g / tz (nstack = 1: one tile).
 struct PlaneRange {
-  int64_t pb, pe;
+  int64_t pb, pe, P;
   int NZ;
   __device__ PlaneRange(const HeatParams& p) {
-    const int64_t P = (int64_t)p.nitems * p.nbands * p.tz;
+    P = (int64_t)p.nitems * p.nbands * p.tz;
     pb = P * blockIdx.x / gridDim.x;
     pe = P * (blockIdx.x + 1) / gridDim.x;
     NZ = p.nstack * p.tz;
   }
 };
+
 
 // ---- specialised kernel: compile-time tile width TX, band height BY and
 // ring depth S. Each thread owns column pair c2 and rows r0 + j*RPP
@@ -142,36 +143,56 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
   const int ty = p.ty, tz = p.tz;
   const PlaneRange R(p);
   const int NZ = R.NZ;
-  const double* const* gtab = p.gdir ? p.gdir : p.gsrc;
+  const int nsteps = p.nsteps > 1 ? p.nsteps : 1;
 
   if ((int)threadIdx.x >= C::NT) {  // ---------------- producer warp
     if (threadIdx.x != C::NT) return;
     uint32_t g = 0;
-    for (int64_t pp = R.pb; pp < R.pe;) {
-      const int64_t col = pp / NZ;
-      const int g0 = (int)(pp - col * NZ);
-      const int n = (int)(R.pe - pp < (int64_t)(NZ - g0) ? R.pe - pp : NZ - g0);
-      const int icol = (int)(col / p.nbands);
-      const int y0 = (int)(col - (int64_t)icol * p.nbands) * BY;
-      // planes g0-1 .. g0+n: stacked tile L, local plane z (z = -1 / tz at the
-      // stack ends stage the z ghost planes)
-      int L = g0 / tz, z = g0 - L * tz - 1;
-      if (z < 0 && L > 0) --L, z += tz;
-      TileItem it = item_at(p, L * p.lt + icol);
-      for (int q = 0; q < n + 2; ++q, ++g, ++z) {
-        if (z == tz && L + 1 < p.nstack) {  // next stacked tile
-          ++L;
-          z = 0;
-          it = item_at(p, L * p.lt + icol);
+    for (int s = 0; s < nsteps; ++s) {
+      const bool odd = s & 1;
+      const TileItem* items = odd ? p.items_odd : p.items;
+      const double* const* gtab = odd ? p.gdir_odd : (p.gdir ? p.gdir : p.gsrc);
+      for (int64_t pp = R.pb; pp < R.pe;) {
+        const int64_t col = pp / NZ;
+        const int g0 = (int)(pp - col * NZ);
+        const int n = (int)(R.pe - pp < (int64_t)(NZ - g0) ? R.pe - pp : NZ - g0);
+        const int icol = (int)(col / p.nbands);
+        const int y0 = (int)(col - (int64_t)icol * p.nbands) * BY;
+        // planes g0-1 .. g0+n: stacked tile L, local plane z (z = -1 / tz at the
+        // stack ends stage the z ghost planes)
+        int L = g0 / tz, z = g0 - L * tz - 1;
+        if (z < 0 && L > 0) --L, z += tz;
+        TileItem it = items ? items[L * p.lt + icol] : p.inline_items[L * p.lt + icol];
+        for (int q = 0; q < n + 2; ++q, ++g, ++z) {
+          if (z == tz && L + 1 < p.nstack) {  // next stacked tile
+            ++L;
+            z = 0;
+            it = items ? items[L * p.lt + icol] : p.inline_items[L * p.lt + icol];
+          }
+          const int st = (int)(g % S);
+          mbar_wait(&empty[st], ((g / S) & 1u) ^ 1u);
+          const double* const* gs = gtab + (size_t)it.tile * 6;
+          const int64_t* ys = p.gdir ? p.ystr + (size_t)it.tile * 2 : nullptr;
+          stage_plane(stage_base + (size_t)st * C::STAGE_ELEMS, &full[st], it.in, gs, ys, z, TX, ty, tz,
+                      y0, BY, p.cache_flags, D);
         }
-        const double* const* gs = gtab + (size_t)it.tile * 6;
-        const int64_t* ys = p.gdir ? p.ystr + (size_t)it.tile * 2 : nullptr;
-        const int s = (int)(g % S);
-        mbar_wait(&empty[s], ((g / S) & 1u) ^ 1u);
-        stage_plane(stage_base + (size_t)s * C::STAGE_ELEMS, &full[s], it.in, gs, ys, z, TX, ty, tz,
-                    y0, BY, p.cache_flags, D);
+        pp += n;
       }
-      pp += n;
+      if (s + 1 < nsteps) {
+        // step barrier: every consumer of this CTA done with step s (drain the
+        // ring; mbarrier acquire), their stores released at gpu scope, then
+        // one arrival on the grid counter and a wait for all gridDim.x of them.
+        // Only this thread waits: the consumers block on the ring as usual.
+        for (int i = 0; i < S; ++i) {
+          const uint32_t j = g + (uint32_t)i;
+          mbar_wait(&empty[j % S], ((j / S) & 1u) ^ 1u);
+        }
+        fence_acq_rel_gpu();
+        red_add_release_gpu(p.prog, 1ull);
+        const unsigned long long target = ((unsigned long long)p.epoch + (unsigned long long)s + 1) * gridDim.x;
+        while (ld_acquire_gpu(p.prog) < target) __nanosleep(32);
+        fence_proxy_async_all();  // other CTAs' generic stores -> this thread's TMA reads
+      }
     }
     return;
   }
@@ -203,9 +224,13 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
   uint32_t seq = 0;
   const size_t plane = (size_t)ty * TX;
   const bool xedge = xlo_edge || xhi_edge;
-  bool pushed = false;  // this thread stored halo layers into a neighbour rank's window
   const int xf = xlo_edge ? XM : XP;  // the x face this thread exports, if any
+  bool pushed = false;  // this thread stored halo layers into a neighbour rank's window
 
+  for (int s = 0; s < nsteps; ++s) {
+  const bool odd = s & 1;
+  const TileItem* items = odd ? p.items_odd : p.items;
+  auto fexp = [&](int f) { return odd ? p.fexp_odd[f] : p.fexp[f]; };
   for (int64_t pp = R.pb; pp < R.pe;) {
     const int64_t col = pp / NZ;
     const int g0 = (int)(pp - col * NZ);
@@ -231,10 +256,10 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
     double* op = nullptr;  // output cell pair of row yb, plane z
     double* fx = nullptr;  // x-face export of row yb, plane z (edge threads)
     auto enter_tile = [&]() {
-      const TileItem it = item_at(p, L * p.lt + icol);
+      const TileItem it = items ? items[L * p.lt + icol] : p.inline_items[L * p.lt + icol];
       tile = it.tile;
       op = it.out + ((size_t)z * ty + yb) * TX + x;
-      if (xedge) fx = p.fexp[xf] + (int64_t)tile * p.face_elems[xf] + ((size_t)z * ty + yb) * D;
+      if (xedge) fx = fexp(xf) + (int64_t)tile * p.face_elems[xf] + ((size_t)z * ty + yb) * D;
     };
     enter_tile();
     for (int i = 0; i < n; ++i) {
@@ -283,16 +308,16 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
 #pragma unroll
         for (int j = 0; j < C::NR; ++j) {
           const int y = yb + j * C::RPP;
-          if (y < D) st2_hint(p.fexp[YM] + (int64_t)tile * p.face_elems[YM] + ((size_t)z * D + y) * TX + x, v[j], keep);
+          if (y < D) st2_hint(fexp(YM) + (int64_t)tile * p.face_elems[YM] + ((size_t)z * D + y) * TX + x, v[j], keep);
           if (y >= ty - D)
-            st2_hint(p.fexp[YP] + (int64_t)tile * p.face_elems[YP] + ((size_t)z * D + y - (ty - D)) * TX + x, v[j], keep);
+            st2_hint(fexp(YP) + (int64_t)tile * p.face_elems[YP] + ((size_t)z * D + y - (ty - D)) * TX + x, v[j], keep);
         }
       }
       if (z < D && tile < p.exp_zlo_below) {
         const size_t e = ((size_t)z * ty + yb) * TX + x;
 #pragma unroll
         for (int j = 0; j < C::NR; ++j)
-          st2_hint(p.fexp[ZM] + (int64_t)tile * p.face_elems[ZM] + e + (size_t)j * C::RPP * TX, v[j], keep);
+          st2_hint(fexp(ZM) + (int64_t)tile * p.face_elems[ZM] + e + (size_t)j * C::RPP * TX, v[j], keep);
         if (p.zpush_lo) {  // fused halo push into the lower rank's window
           pushed = true;
           double* q = p.zpush_lo + (int64_t)tile * p.face_elems[ZM] + e;
@@ -304,7 +329,7 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
         const size_t e = ((size_t)(z - (tz - D)) * ty + yb) * TX + x;
 #pragma unroll
         for (int j = 0; j < C::NR; ++j)
-          st2_hint(p.fexp[ZP] + (int64_t)tile * p.face_elems[ZP] + e + (size_t)j * C::RPP * TX, v[j], keep);
+          st2_hint(fexp(ZP) + (int64_t)tile * p.face_elems[ZP] + e + (size_t)j * C::RPP * TX, v[j], keep);
         if (p.zpush_hi) {  // fused halo push into the upper rank's window
           pushed = true;
           double* q = p.zpush_hi + (int64_t)(tile - p.exp_zhi_from) * p.face_elems[ZP] + e;
@@ -319,6 +344,7 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
     release_g(seq + n + 1);  // plane g0+n (last z+1 neighbour)
     seq += (uint32_t)(n + 2);
     pp += n;
+  }
   }
   // pushed halo layers visible system-wide (the neighbour ranks' GPUs) before
   // the halo stream's arrival counter, written after this kernel, is
@@ -523,11 +549,14 @@ cudaError_t launch_heat7(const HeatParams& p, int stages, size_t smem, int grid,
   const FixedEntry* e = find_fixed_s(p.tx, p.band, stages, p.depth);
   if (e && e->smem == smem) {
     void* args[] = {const_cast<HeatParams*>(&p)};
+    if (p.nsteps > 1)  // CTAs wait on each other's progress: all must be co-resident
+      return cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(e->fn), dim3(grid), dim3(e->nt),
+                                         args, smem, s);
     return cudaLaunchKernel(reinterpret_cast<const void*>(e->fn), dim3(grid), dim3(e->nt), args,
                             smem, s);
   }
   // the general kernel takes independent tiles and exported faces only
-  if (p.gdir || p.nstack != 1 || p.lt != p.nitems) return cudaErrorInvalidValue;
+  if (p.gdir || p.nstack != 1 || p.lt != p.nitems || p.nsteps > 1) return cudaErrorInvalidValue;
   heat7_generic<kGenericThreads><<<grid, kGenericThreads, smem, s>>>(p, stages);
   return cudaGetLastError();
 }

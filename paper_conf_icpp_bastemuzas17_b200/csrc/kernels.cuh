@@ -78,6 +78,22 @@ struct HeatParams {
   // NVLink / NVSwitch); the halo op then only signals.
   double* zpush_lo;
   double* zpush_hi;
+  // Persistent multi-step launch (nsteps > 1; DESIGN.md §4 "multi-step"):
+  // single rank, whole domain resident, direct ghosts. Step s uses items /
+  // gdir / fexp for even s and items_odd / gdir_odd / fexp_odd for odd s (the
+  // two buffer arrays and face parities alternate). Between steps each CTA's
+  // producer drains its ring, releases the consumers' stores at gpu scope and
+  // arrives on the grid counter *prog; step s + 1 is staged once the counter
+  // reaches (epoch + s + 1) * gridDim.x (epoch = barrier rounds of earlier
+  // launches, so the counter is never reset). Requires all CTAs co-resident
+  // (cooperative launch).
+  int32_t nsteps;
+  int32_t ntx, nty;
+  uint32_t epoch;
+  unsigned long long* prog;
+  const TileItem* items_odd;
+  const double* const* gdir_odd;
+  double* fexp_odd[6];
 };
 
 // Two-step pass (temporal blocking, ghost = 2): u^{s+2} from u^s in one

@@ -158,6 +158,8 @@ Status domain_setup(Domain& d) {
   persist += 2 * gsrc_bytes + 2 * items_bytes;
   const uint64_t ystr_bytes = align_up((uint64_t)G.ntiles * 2 * sizeof(int64_t));
   persist += 4 * gsrc_bytes + ystr_bytes;  // direct ghost-source tables (resident mode)
+  const uint64_t prog_bytes = align_up(kMaxProgCtas * sizeof(unsigned long long));
+  persist += prog_bytes;                    // multi-step progress counters
   const uint64_t esrc_bytes = d.x2_ok ? align_up((uint64_t)G.ntiles * 12 * sizeof(EdgePtr)) : 0;
   const uint64_t mask_bytes = d.x2_ok ? align_up((uint64_t)G.ntiles) : 0;
   persist += 2 * esrc_bytes + mask_bytes;
@@ -228,6 +230,7 @@ Status domain_setup(Domain& d) {
   for (int b = 0; b < 2; ++b)
     for (int p = 0; p < 2; ++p) d.gdir_dev[b][p] = reinterpret_cast<const double**>(carve(gsrc_bytes));
   d.ystr_dev = reinterpret_cast<int64_t*>(carve(ystr_bytes));
+  d.prog_dev = reinterpret_cast<unsigned long long*>(carve(prog_bytes));
   if (d.x2_ok) {
     for (int p = 0; p < 2; ++p) d.esrc_dev[p] = reinterpret_cast<EdgePtr*>(carve(esrc_bytes));
     d.fixed_mask_dev = reinterpret_cast<uint8_t*>(carve(mask_bytes));
@@ -260,6 +263,11 @@ Status domain_setup(Domain& d) {
   }
   // fused halo push: peer transport mode 2 with direct passes (multi-rank resident)
   d.peer_fused = multi && d.opt.peer_transport == 2 && d.direct_ok;
+  // persistent multi-step launches: single rank, direct passes (TILES_PERSIST=0: off)
+  {
+    const char* e = std::getenv("TILES_PERSIST");
+    d.persist_ok = !multi && d.direct_ok && !(e && std::atoi(e) == 0);
+  }
   if (d.direct_ok) {
     for (int b = 0; b < 2; ++b)
       for (int p = 0; p < 2; ++p) {
@@ -567,6 +575,23 @@ struct ResidentRun {
     return X.record(d, ev_layer(d, (int64_t)i, s & 1), b.stream);
   }
 
+  // every pass of this phase as ONE persistent launch (HeatParams::nsteps):
+  // one whole-domain batch, single rank, direct single steps
+  bool persistent() const {
+    if (!d.persist_ok || multi || B.size() != 1 || T < 2 || !d.items_dev[0]) return false;
+    for (int s = 0; s < T; ++s)
+      if (kpass[(size_t)s] != 1) return false;
+    return true;
+  }
+  Status issue_kernels_persistent() {
+    const Batch& b = B[0];
+    const TileItem* items = d.items_dev[bit0] + tile0(b);
+    Status r = X.heat(d, nullptr, nullptr, nullptr, (int)ntl(b), fp0, items, b.stream, bit0,
+                      (int)(b.L1 - b.L0), T);
+    if (r.bad()) return r;
+    return X.record(d, ev_layer(d, 0, (T - 1) & 1), b.stream);
+  }
+
   Status issue_halo(int s) {  // exchange the faces written at step s (s = -1: current)
     const int hs = d.halo_stream;
     Status r;
@@ -608,6 +633,11 @@ struct ResidentRun {
       // which precede the step-s boundary kernels in stream order.
       return true;
     };
+    if (persistent()) {
+      Status r = issue_load(0);
+      if (r.bad()) return r;
+      return issue_kernels_persistent();
+    }
     for (;;) {
       bool progress = false;
       // drain everything ready, in (step, batch) order

@@ -113,7 +113,7 @@ struct Exec {
   // nstack: the items are nstack consecutive tile layers (stacked z-march)
   virtual Status heat(Domain& d, const int64_t* tiles, const int* in_slots, const int* out_slots,
                       int nitems, int read_parity, const TileItem* dev_items, int stream,
-                      int direct_bit = -1, int nstack = 1) = 0;
+                      int direct_bit = -1, int nstack = 1, int nsteps = 1) = 0;
   virtual Status sincos(Domain& d, int64_t tile, int slot, int64_t iters, int stream) = 0;
   // stream-through: one Jacobi sweep of slab planes [lo, hi) (periodic in
   // x and y) from src to dst; see SlabRef
@@ -158,6 +158,7 @@ struct Exec {
 
 // -------------------------------------------------------------------- domain
 enum Mode : int { MODE_RESIDENT = 1, MODE_STREAM = 2 };
+constexpr int kMaxProgCtas = 2048;  // progress counters of a persistent multi-step launch
 
 struct Domain {
   Geometry G;
@@ -190,6 +191,12 @@ struct Domain {
   std::vector<const double*> gdir_host[2][2];
   std::vector<int64_t> ystr_host;
   bool direct_ok = false;                  // single-step resident passes read neighbours directly
+  // persistent multi-step launches (HeatParams::nsteps): per-CTA progress
+  // counters and the step epoch their values are relative to
+  bool persist_ok = false;
+  unsigned long long* prog_dev = nullptr;  // [0]: grid barrier arrival counter
+  uint32_t prog_epoch = 0;                  // barrier rounds completed by earlier launches
+  int64_t prog_grid = 0;                    // grid of the persistent launches (fixed per domain)
   EdgePtr* esrc_dev[2] = {};               // [parity] -> ntiles*12 (D = 2 only)
   std::vector<EdgePtr> esrc_host[2];
   uint8_t* fixed_mask_dev = nullptr;       // per tile: Dirichlet faces (bit f)

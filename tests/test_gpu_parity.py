@@ -237,7 +237,9 @@ def test_kernel_timing_and_device_timer():
         d.run(T.heat7(), 4, 1)
         ms = d.timer_stop()
         st = d.stats()
-    assert ms > 0 and st["kernel_timed"] == 4 and 0 < st["kernel_ms"] <= ms * 1.01
+    # 4 steps: one persistent multi-step launch (default) or 4 launches (TILES_PERSIST=0)
+    assert st["n_kernels"] in (1, 4) and st["kernel_timed"] == st["n_kernels"]
+    assert ms > 0 and 0 < st["kernel_ms"] <= ms * 1.01
 
 
 # ----------------------------------------------------------- large configs
