@@ -1,6 +1,7 @@
 """Small runs of every schedule for compute-sanitizer (memcheck / racecheck /
 synccheck / initcheck): resident heat (layered + whole-domain phases),
-streaming heat with a tiny budget, Dirichlet, sincos, the generic kernel and
+streaming heat with a tiny budget, Dirichlet, sincos, the generic kernel, the
+persistent multi-step launch (direct ghosts, grid counter) and
 the stream-through schedule and the in-process multi-rank transport."""
 import os
 import sys
@@ -28,6 +29,10 @@ def budget(dims, td, n, **kw):
 u = synth.uniform_grid(64, 32, 32, 42)
 with T.Domain((64, 32, 32), (32, 16, 8)) as d:          # fixed kernel (32,16), 4 layers -> phases
     d.load(u); d.run(T.heat7(), 6, 2); d.store()
+    d.run(T.heat7(), 5, 2); d.store()                    # resident: one persistent multi-step launch
+ext0 = synth.uniform_grid(66, 34, 34, 6)
+with T.Domain((64, 32, 32), (32, 16, 8), bc="dirichlet") as d:   # direct ghosts + Dirichlet, persistent
+    d.load(ext0); d.run(T.heat7(), 2, 2); d.sync(); d.run(T.heat7(), 4, 2); d.store()
 with T.Domain((48, 40, 20), (24, 20, 5)) as d:          # generic kernel
     d.load(synth.uniform_grid(48, 40, 20, 1)); d.run(T.heat7(), 3, 2); d.store()
 with T.Domain((64, 32, 32), (32, 16, 8), sched="stream", device_budget_bytes=budget((64, 32, 32), (32, 16, 8), 3)) as d:
