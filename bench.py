@@ -154,19 +154,23 @@ def measured_peaks():
     return 6650.0, "B200_PROFILING.md fallback 6.65 TB/s"
 
 
-def pcie_bandwidth(torch, nbytes=256 << 20, reps=5):
+def pcie_bandwidth(torch, nbytes=1 << 30, reps=8, warm=2):
+    """Pinned single-direction link rates (GB/s): best of `reps` 1 GiB copies
+    after `warm` untimed ones (a fresh pinned buffer's first DMAs run slower
+    on these VMs), CUDA events on the copy stream."""
     h = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
     d = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
     out = {}
     for k in ("h2d", "d2h"):
         best = 0
-        for _ in range(reps):
+        for i in range(warm + reps):
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
             d.copy_(h, non_blocking=True) if k == "h2d" else h.copy_(d, non_blocking=True)
             e1.record()
             torch.cuda.synchronize()
-            best = max(best, nbytes / (e0.elapsed_time(e1) / 1e3) / 1e9)
+            if i >= warm:
+                best = max(best, nbytes / (e0.elapsed_time(e1) / 1e3) / 1e9)
         out[k] = best
     return out
 
@@ -313,22 +317,32 @@ def run_stream_leg(args):
     return 0
 
 
-def pcie_bidir(torch, nbytes=256 << 20, reps=5):
+def pcie_bidir(torch, nbytes=1 << 30, reps=6, warm=2):
+    """Both directions at once (H2D and D2H of 1 GiB each on two streams):
+    (bytes H2D + bytes D2H) / span, span from CUDA events (start on the
+    current stream, both copy streams wait on it, end = the later stream)."""
     h1 = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
     h2 = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
     d1 = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
     d2 = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
     s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
     best = 0
-    for _ in range(reps):
+    for i in range(warm + reps):
         torch.cuda.synchronize()
-        t0 = time.perf_counter()
-        with torch.cuda.stream(s1):
-            d1.copy_(h1, non_blocking=True)
-        with torch.cuda.stream(s2):
-            h2.copy_(d2, non_blocking=True)
+        e0 = torch.cuda.Event(enable_timing=True)
+        e0.record()
+        ends = []
+        for s_, dst, src in ((s1, d1, h1), (s2, h2, d2)):
+            s_.wait_event(e0)
+            with torch.cuda.stream(s_):
+                dst.copy_(src, non_blocking=True)
+                e = torch.cuda.Event(enable_timing=True)
+                e.record(s_)
+                ends.append(e)
         torch.cuda.synchronize()
-        best = max(best, 2 * nbytes / (time.perf_counter() - t0) / 1e9)
+        if i >= warm:
+            span = max(e0.elapsed_time(e) for e in ends)
+            best = max(best, 2 * nbytes / (span / 1e3) / 1e9)
     return best
 
 
@@ -896,12 +910,17 @@ def main():
     peak, peak_src = measured_peaks()
     algo_bytes = 16.0 * cells_per_launch
     achieved = algo_bytes / (avg_kernel_ms / 1e3) / 1e9
+    # a persistent launch runs every step of a tile_run (steps_per_launch = T);
+    # the ncu capture is of one whole-domain step, so traffic scales by it
+    steps_per_launch = cells_per_launch / cells
+    tps = traffic_from_profile(args.config) if spp == 1 else None
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-            "traffic": traffic_from_profile(args.config) if spp == 1 else None,
+            "traffic": tps * steps_per_launch if tps else None,
+            "traffic_per_step": tps,
             "kernel": "heat7_fixed" if spp == 1 else "heat7x2 (2 steps per pass)",
             "algorithmic_bytes_per_cell_update": 16.0 / spp,
-            "algorithmic_bytes_per_launch": algo_bytes, "avg_launch_ms": avg_kernel_ms,
-            "peak_source": peak_src}
+            "algorithmic_bytes_per_launch": algo_bytes, "steps_per_launch": steps_per_launch,
+            "avg_launch_ms": avg_kernel_ms, "peak_source": peak_src}
 
     cpu = None
     if rk == 0 and ws == 1 and not args.no_cpu_baseline:

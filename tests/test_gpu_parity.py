@@ -108,6 +108,20 @@ def test_runs_continue_state():
     assert np.array_equal(out, ref)
 
 
+@pytest.mark.parametrize("direct,persist", [("1", "1"), ("1", "0"), ("0", "0")])
+@pytest.mark.parametrize("bc", ["periodic", "dirichlet"])
+@pytest.mark.parametrize("dims,td", [((128, 64, 64), (64, 32, 16)), ((64, 96, 48), (32, 32, 8))])
+def test_resident_paths_bit_exact(monkeypatch, direct, persist, bc, dims, td):
+    """The resident single-step variants give the same bits: direct y/z ghosts
+    + persistent multi-step launch (default), direct ghosts with one launch
+    per step, and every ghost from exported faces. Several runs, so a run
+    starts from the state (and the stale y/z exports) a direct run left."""
+    monkeypatch.setenv("TILES_DIRECT", direct)
+    monkeypatch.setenv("TILES_PERSIST", persist)
+    out, ref, _, st = _heat(dims, td, 13, bc=bc, runs=[3, 6, 1, 3])
+    assert np.array_equal(out, ref), np.abs(out - ref).max()
+
+
 def test_sync_baseline_bit_exact():
     out, ref, info, _ = _heat((64, 64, 64), (32, 32, 32), 5, sched="sync")
     assert np.array_equal(out, ref) and info["sched"] == T.TILE_SCHED_SYNC
