@@ -131,11 +131,17 @@ typedef struct {
                                    ranks' memory (CUDA IPC; NVLink / NVSwitch
                                    peer access), synchronised with stream
                                    memory operations on counters in the
-                                   neighbours' memory — no NCCL. The caller
-                                   gathers every rank's tile_peer_handle and
-                                   passes them to tile_peer_connect before the
-                                   first run. 0 (default) = NCCL (or the
-                                   local_group transport). */
+                                   neighbours' memory — no NCCL. 2 = the same
+                                   windows, but in resident single-step runs the
+                                   stencil kernel itself stores each step's
+                                   slab-end z layers into the neighbours'
+                                   windows as it computes them (fused compute +
+                                   exchange); the exchange after a step only
+                                   signals. The caller gathers
+                                   every rank's tile_peer_handle and passes them
+                                   to tile_peer_connect before the first run.
+                                   0 (default) = NCCL (or the local_group
+                                   transport). */
   int32_t two_step;             /* HEAT7 with ghost >= 2: 0 (default) = two
                                    steps per pass in the streaming schedule
                                    (halves host-link bytes per step), single
@@ -316,7 +322,7 @@ const char* tile_last_error(void);
  * TILE_ENOSYS if built without NCCL. */
 tile_status tile_nccl_unique_id(void* out128);
 
-/* Peer transport (tile_options.peer_transport = 1). tile_peer_handle writes
+/* Peer transport (tile_options.peer_transport = 1 or 2). tile_peer_handle writes
  * the 64-byte CUDA IPC handle of this rank's halo window (receive buffers
  * and exchange counters) to out64. tile_peer_connect takes every rank's
  * handle, `nranks` blobs of 64 bytes in rank order (the caller all-gathers

@@ -69,6 +69,8 @@ Status domain_create(const int64_t dims[3], const int64_t tdims[3], int ghost,
     return make_err(TILE_EINVAL, "bad sched");
   if (opt.nstreams_provided < 0 || opt.nstreams_provided > 64)
     return make_err(TILE_EINVAL, "nstreams_provided must be in [0, 64]");
+  if (opt.peer_transport < 0 || opt.peer_transport > 2)
+    return make_err(TILE_EINVAL, "peer_transport must be 0, 1 or 2");
   Geometry G;
   Status st = make_geometry(dims, tdims, ghost, opt.bc, opt.nranks, opt.rank, &G);
   if (st.bad()) return st;

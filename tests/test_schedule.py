@@ -45,6 +45,9 @@ def test_invalid_arguments_have_no_side_effects():
         with pytest.raises(T.TileError) as e:
             T.Domain(dims, td, ghost=g, dry_run=True)
         assert e.value.code == T.TILE_EINVAL
+    with pytest.raises(T.TileError) as e:
+        T.Domain((16, 16, 16), (8, 8, 8), dry_run=True, peer_transport=3)
+    assert e.value.code == T.TILE_EINVAL
     d = T.Domain((16, 16, 16), (8, 8, 8), dry_run=True)
     for k, steps, ns in [(T.heat7(0.2), 1, 1), (T.heat7(0.0), 1, 1), (T.heat7(), -1, 1),
                          (T.heat7(), 1, 0), (T.heat7(), 1, 65), (T.sincos(-1), 1, 1)]:
