@@ -213,8 +213,20 @@ struct CudaExec final : Exec {
       if (d.prog_grid && d.prog_grid != grid) return make_err(TILE_ESTATE, "internal: persistent grid changed");
       d.prog_grid = grid;
     }
-    Status r = timed(d, st, [&] { return launch_heat7(p, d.stages, d.heat_smem, (int)grid, S(st)); });
+    cudaError_t le = cudaSuccess;
+    Status r = timed(d, st, [&] {
+      le = launch_heat7(p, d.stages, d.heat_smem, (int)grid, S(st));
+      return le == cudaErrorCooperativeLaunchTooLarge ? cudaSuccess : le;
+    });
     if (r.bad()) return r;
+    if (le == cudaErrorCooperativeLaunchTooLarge) {
+      // SMs held by another context: no co-residency guarantee, so no
+      // persistent launches on this domain; run the steps one launch each
+      (void)cudaGetLastError();
+      coop = 0;
+      d.prog_epoch -= (uint32_t)(nsteps - 1);
+      return heat(d, tiles, in, out, n, rp, dev_items, st, direct_bit, nstack, nsteps);
+    }
     d.stats.n_kernels++;
     return Status::ok();
   }
