@@ -24,3 +24,13 @@ def cuda_available():
 @pytest.fixture(scope="session")
 def golden_dir():
     return os.path.join(ROOT, "tests", "golden")
+
+
+def import_tiles():
+    """The native binding. On a GPU box a missing or broken libtiles.so is an
+    ERROR (no silent skip: the CUDA path must be the one that runs); on a
+    CPU-only host the GPU-marked modules skip."""
+    if cuda_available():
+        from paper_conf_icpp_bastemuzas17_b200 import tiles
+        return tiles
+    return pytest.importorskip("paper_conf_icpp_bastemuzas17_b200.tiles")

@@ -13,7 +13,9 @@ import oracle
 import synth
 
 pytestmark = pytest.mark.gpu
-T = pytest.importorskip("paper_conf_icpp_bastemuzas17_b200.tiles")
+from tests.conftest import import_tiles
+
+T = import_tiles()
 ALPHA = 0.125
 
 

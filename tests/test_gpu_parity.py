@@ -14,7 +14,9 @@ import synth
 
 pytestmark = pytest.mark.gpu
 
-T = pytest.importorskip("paper_conf_icpp_bastemuzas17_b200.tiles")
+from tests.conftest import import_tiles
+
+T = import_tiles()
 T_ = T
 ALPHA = 0.125
 
