@@ -614,11 +614,27 @@ def multi_domain(Tl, dist, ws, rk, transport, *args, **kw):
     if ws == 1:
         return Tl.Domain(*args, nranks=1, rank=0, **kw)
     if transport in ("peer", "peer-copy"):
-        dom = Tl.Domain(*args, nranks=ws, rank=rk, peer_transport=2 if transport == "peer" else 1, **kw)
-        hs = [None] * ws
-        dist.all_gather_object(hs, dom.peer_handle())
-        dom.peer_connect(hs)
-        return dom
+        # the IPC windows need peer access between every z-neighbour pair; if
+        # any rank cannot set them up (e.g. no P2P between two GPUs of this
+        # box), every rank takes the NCCL transport instead, and says so
+        dom, err = None, ""
+        try:
+            dom = Tl.Domain(*args, nranks=ws, rank=rk, peer_transport=2 if transport == "peer" else 1, **kw)
+            hs = [None] * ws
+            dist.all_gather_object(hs, dom.peer_handle())
+            dom.peer_connect(hs)
+        except Tl.TileError as e:
+            err = str(e)
+        import torch
+        ok = torch.tensor([0 if err else 1], dtype=torch.int32, device=red_dev())
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+        if int(ok.item()) == 1:
+            return dom
+        print(f"rank {rk}: peer transport unavailable ({err or 'on another rank'}); using NCCL",
+              file=sys.stderr, flush=True)
+        if dom is not None:
+            dom.free()
+        multi_domain.fallback = "nccl (peer transport setup failed)"
     obj = [Tl.nccl_unique_id() if rk == 0 else None]
     dist.broadcast_object_list(obj, src=0)
     return Tl.Domain(*args, nranks=ws, rank=rk, nccl_id=obj[0], **kw)
@@ -938,7 +954,7 @@ def main():
                 "config": {"workload": desc, "dims_per_gpu": dims, "global_dims": gdims, "tile_dims": td,
                            "ghost": args.ghost, "steps_per_pass": spp, "T": T, "nstreams": ns,
                            "bc": "periodic", "alpha": ALPHA,
-                           "parallelism": f"z-slab x{ws}, halo via {args.transport}" if ws > 1 else "1 GPU",
+                           "parallelism": f"z-slab x{ws}, halo via {getattr(multi_domain, 'fallback', args.transport)}" if ws > 1 else "1 GPU",
                            "l2": "inputs larger than L2 (2 x 1.07 GB per GPU per step)",
                            "value_def": "grid resident in HBM; T steps of tile_run",
                            "e2e_def": "tile_invalidate + tile_run(T) + tile_sync from pinned host"},

@@ -217,8 +217,12 @@ typedef enum {
                             z faces) only; d | 0x100: the launch also stores its slab-end
                             z layers into the neighbour ranks' receive buffers (fused
                             halo push, peer_transport = 2) */
-  TILE_OP_HALO_SIGNAL = 23 /* halo exchange of parity d whose data the previous kernels
+  TILE_OP_HALO_SIGNAL = 23,/* halo exchange of parity d whose data the previous kernels
                             pushed (fused): synchronisation only */
+  TILE_OP_ST_HALO = 24   /* multi-rank stream-through (peer transport): a = 0 push the
+                            slab-end c planes of initial data (b = 1 top -> upper rank,
+                            0 bottom -> lower rank), 1 wait for side b's halo layer,
+                            2 release side b's halo layer */
 } tile_op_kind;
 
 typedef struct {

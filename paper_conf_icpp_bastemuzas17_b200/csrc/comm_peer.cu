@@ -27,6 +27,17 @@
 //   read the buffers the neighbours' next kernels will push into); wait my
 //   A >= k and R >= k+1. The first exchange of a run (mode 1) is the copy
 //   exchange above plus the R := k+1 arming for the first fused push.
+// Multi-rank stream-through (peer_st_halo): the trapezoid of T
+// steps over a rank's z-slab needs the T planes of INITIAL data beyond each
+// slab end, once per run, and no exchange after that. Run e (d.st_epoch, the
+// same on every rank: runs are collective), on the rank's halo stream once
+// the H2D of its slab-end unit has landed: wait until the receiver released
+// run e-1's layer (CR_UP / CR_DN >= e-1), copy the T planes of every tile of
+// the slab-end layer into the receiver's halo layer (top -> upper.st_lo,
+// bottom -> lower.st_hi), then S_LO / S_HI := e at the receiver. The receiver's
+// compute stream waits S >= e before the first sweep of its unit 0 / U-1,
+// which reads the halo layer in place of the periodic wrap, and writes
+// CR := e at the sender after that sweep.
 // Counters are stream memory operations (cuStreamWriteValue32 /
 // cuStreamWaitValue32, fetched with cudaGetDriverEntryPoint), so no kernel
 // spins and no SM is held.
@@ -41,7 +52,8 @@
 namespace tiles {
 namespace {
 
-enum { R_DN = 0, R_UP = 1, A_DN = 2, A_UP = 3, NFLAGS = 8 };
+enum { R_DN = 0, R_UP = 1, A_DN = 2, A_UP = 3, S_LO = 4, S_HI = 5, CR_UP = 6, CR_DN = 7, NFLAGS = 8 };
+constexpr uint64_t kFlagBytes = 256;
 
 using WriteFn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
 using WaitFn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
@@ -78,11 +90,12 @@ CUdeviceptr flag(void* window_flags, int i) {
 
 }  // namespace
 
-// Window: [halo 0/1][parity 0/1] receive buffers, then the counters.
-Status peer_setup(Domain& d, uint64_t halo_bytes) {
+// Window: [halo 0/1][parity 0/1] receive buffers, the counters, then the two
+// stream-through halo layers (st_bytes each; 0 = none).
+Status peer_setup(Domain& d, uint64_t halo_bytes, uint64_t st_bytes) {
   Status s = load_memops();
   if (s.bad()) return s;
-  const uint64_t bytes = 4 * halo_bytes + 256;
+  const uint64_t bytes = 4 * halo_bytes + kFlagBytes + 2 * st_bytes;
   void* w = nullptr;
   PK(cudaMalloc(&w, bytes));
   PK(cudaMemset(w, 0, bytes));
@@ -93,6 +106,9 @@ Status peer_setup(Domain& d, uint64_t halo_bytes) {
     for (int p = 0; p < 2; ++p) d.halo[a][p] = reinterpret_cast<double*>(c + (2 * a + p) * halo_bytes);
   d.peer_flags = c + 4 * halo_bytes;
   d.peer_halo_bytes = halo_bytes;
+  d.st_halo_bytes = st_bytes;
+  for (int a = 0; a < 2; ++a)
+    d.st_halo[a] = st_bytes ? reinterpret_cast<double*>(c + 4 * halo_bytes + kFlagBytes + a * st_bytes) : nullptr;
   int flush = 0, dev = 0;
   PK(cudaGetDevice(&dev));
   // CU_DEVICE_ATTRIBUTE_CAN_FLUSH_REMOTE_WRITES: needed to make the peers'
@@ -201,6 +217,40 @@ Status peer_halo(Domain& d, int par, void* stream_v, int mode) {
     if (up) DK(g_wait(st, flag(d.peer_flags, R_UP), k + 1, d.peer_wait_flags));
     if (lo) DK(g_wait(st, flag(d.peer_flags, R_DN), k + 1, d.peer_wait_flags));
   }
+  return Status::ok();
+}
+
+Status peer_st_halo(Domain& d, int op, int side, int T, void* stream_v) {
+  if (!d.peer_connected) return make_err(TILE_ESTATE, "peer transport: call tile_peer_connect first");
+  if (!d.st_halo_bytes) return make_err(TILE_ESTATE, "no stream-through halo layers in the window");
+  const Geometry& G = d.G;
+  CUstream st = static_cast<CUstream>(stream_v);
+  const uint32_t e = d.st_epoch;
+  const uint64_t hb = d.peer_halo_bytes;
+  char* nb = static_cast<char*>(d.peer_base[side]);  // side 0: lower, 1: upper neighbour
+  if (!nb) return make_err(TILE_EINVAL, "stream-through halo: no neighbour on that side");
+  void* nb_flags = nb + 4 * hb;
+  if (op == 0) {  // push my slab-end planes to the neighbour on `side`
+    DK(g_wait(st, flag(d.peer_flags, side ? CR_UP : CR_DN), e - 1, d.peer_wait_flags));
+    if (d.measure != TILE_MEASURE_COMP_ONLY) {
+      const size_t plane = (size_t)G.t[0] * G.t[1], te = (size_t)G.tile_elems;
+      const int64_t layer = side ? G.n[2] - 1 : 0;
+      const size_t p0 = side ? (size_t)(G.t[2] - T) : 0;  // first plane within the tiles
+      const double* src = d.slot_ptr(d.res_bit ? (int)G.ntiles : 0) + (size_t)layer * G.layer_tiles * te + p0 * plane;
+      char* dst = nb + 4 * hb + kFlagBytes + (side ? 0 : 1) * d.st_halo_bytes + p0 * plane * 8;
+      PK(cudaMemcpy2DAsync(dst, te * 8, src, te * 8, (size_t)T * plane * 8, (size_t)G.layer_tiles,
+                           cudaMemcpyDeviceToDevice, (cudaStream_t)st));
+      d.stats.bytes_halo += (uint64_t)G.layer_tiles * T * plane * 8;
+    }
+    DK(g_write(st, flag(nb_flags, side ? S_LO : S_HI), e, 0));
+    return Status::ok();
+  }
+  if (op == 1) {  // my halo layer on `side` has arrived
+    DK(g_wait(st, flag(d.peer_flags, side ? S_HI : S_LO), e, d.peer_wait_flags));
+    return Status::ok();
+  }
+  // op 2: my halo layer on `side` has been read: its sender may overwrite it
+  DK(g_write(st, flag(nb_flags, side ? CR_DN : CR_UP), e, 0));
   return Status::ok();
 }
 

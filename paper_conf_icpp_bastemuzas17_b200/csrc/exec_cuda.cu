@@ -250,6 +250,10 @@ struct CudaExec final : Exec {
       v.tz = (int)G.t[2];
       v.zbase = (int)r.zbase;
       v.nz = (int)G.l[2];
+      if (G.nranks > 1) {  // multi-rank stream-through: no wrap inside the slab
+        v.hlo = d.st_halo[0];
+        v.hhi = d.st_halo[1];
+      }
     } else if (r.kind == SlabRef::UNITS) {
       v.ring = 1;
       v.te = r.un * G.t[0] * G.t[1];
@@ -418,6 +422,12 @@ struct CudaExec final : Exec {
     Status r = d.opt.peer_transport ? peer_halo(d, par, S(st), mode) : nccl_halo(d, par, S(st));
     if (r.bad()) return r;
     d.stats.n_halo++;
+    return Status::ok();
+  }
+  Status st_halo(Domain& d, int op, int side, int T, int st) override {
+    Status r = peer_st_halo(d, op, side, T, S(st));
+    if (r.bad()) return r;
+    if (op == 0) d.stats.n_halo++;
     return Status::ok();
   }
   Status note(Domain&, int, int64_t, int64_t, int) override { return Status::ok(); }

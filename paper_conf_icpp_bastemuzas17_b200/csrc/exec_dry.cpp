@@ -146,6 +146,14 @@ struct DryExec final : Exec {
     put(d, mode == 2 ? TILE_OP_HALO_SIGNAL : TILE_OP_HALO, st, mode, 0, 0, par);
     return Status::ok();
   }
+  Status st_halo(Domain& d, int op, int side, int T, int st) override {
+    if (op == 0) {
+      d.stats.n_halo++;
+      d.stats.bytes_halo += (uint64_t)d.G.layer_tiles * T * d.G.t[0] * d.G.t[1] * 8;
+    }
+    put(d, TILE_OP_ST_HALO, st, op, side, T, 0);
+    return Status::ok();
+  }
   Status note(Domain& d, int kind, int64_t a, int64_t b, int st) override {
     put(d, kind, st, a, b, 0, 0);
     return Status::ok();

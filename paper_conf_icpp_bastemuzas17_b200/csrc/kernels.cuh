@@ -159,6 +159,8 @@ struct SlabView {
   int ring;                     // 1: unit-ring view (below)
   int u, U, un;
   double* ubase[3];
+  double* hlo;                  // resident view, multi-rank: planes z < 0 (tile-blocked layer,
+  double* hhi;                  // planes tz+z) and z >= nz (planes z-nz) instead of the wrap
 };
 cudaError_t launch_slab_sweep(const SlabView& src, const SlabView& dst, int nx, int ny, int lo,
                               int hi, double alpha, int sms, cudaStream_t s);

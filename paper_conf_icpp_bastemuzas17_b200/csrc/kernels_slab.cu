@@ -5,7 +5,8 @@
 // Source and destination are "views" of the same logical slab:
 //   - the dense scratch slab [plane][ny][nx] (middle sweeps),
 //   - the tile-blocked resident array at local z = zbase + plane, wrapped
-//     (first sweep: the gather is fused into it),
+//     (first sweep: the gather is fused into it); with z-slab ranks, planes
+//     beyond the slab come from the neighbours' planes in the halo layers,
 //   - the unit's packed sub-tiles [layer tile][plane - first][ty][tx] (last
 //     sweep: the scatter is fused into it),
 //   - a ring of three units' packed sub-tiles (units u-1, u, u+1: the
@@ -32,9 +33,13 @@ struct ViewDev {
   int tx, ty, tz, ntx, nty, zbase, nz;
   int ring, u, U, un;
   double* ub[3];
+  double* hlo;
+  double* hhi;
   // first element of slab plane pl (x = y = 0 of tile column 0, row 0)
   __device__ __forceinline__ double* P(int pl) const {
     int gz = zbase + pl;
+    if (hlo && gz < 0) return hlo + (int64_t)(tz + gz) * ty * tx;   // lower rank's top planes
+    if (hhi && gz >= nz) return hhi + (int64_t)(gz - nz) * ty * tx;  // upper rank's bottom planes
     if (nz > 0) {
       gz %= nz;
       if (gz < 0) gz += nz;
@@ -62,7 +67,7 @@ struct ViewDev {
 
 static ViewDev to_dev(const SlabView& v) {
   return ViewDev{v.base, v.te, v.tx, v.ty, v.tz, v.ntx, v.nty, v.zbase, v.nz, v.ring, v.u, v.U, v.un,
-                 {v.ubase[0], v.ubase[1], v.ubase[2]}};
+                 {v.ubase[0], v.ubase[1], v.ubase[2]}, v.hlo, v.hhi};
 }
 
 // Work items are (z chunk, column) pairs, column = (x segment of 128 pairs,

@@ -21,6 +21,7 @@ namespace tiles {
 namespace {
 
 constexpr uint64_t kReserveBytes = 1ull << 30;  // head-room left to the driver/others
+constexpr uint64_t kStHaloMax = 1ull << 30;     // multi-rank stream-through halo layers, both
 constexpr uint64_t kAlign = 256;
 
 uint64_t align_up(uint64_t v) { return (v + kAlign - 1) / kAlign * kAlign; }
@@ -155,6 +156,13 @@ Status domain_setup(Domain& d) {
   const uint64_t halo_bytes = align_up((uint64_t)G.layer_tiles * G.face_elems[ZM] * 8);
   const bool peer = multi && d.opt.peer_transport && !d.opt.dry_run;  // halos live in the IPC window
   if (multi && !peer) persist += 4 * halo_bytes;
+  // multi-rank stream-through: two tile layers of halo planes in the peer
+  // window (periodic slabs; skipped when they would exceed kStHaloMax)
+  uint64_t st_bytes = 0;
+  if (peer && G.bc == TILE_BC_PERIODIC && d.opt.stream_through >= 0) {
+    const uint64_t layer = align_up((uint64_t)G.layer_tiles * G.tile_elems * 8);
+    if (2 * layer <= kStHaloMax) st_bytes = layer;
+  }
   const uint64_t gsrc_bytes = align_up((uint64_t)G.ntiles * 6 * sizeof(double*));
   const uint64_t items_bytes = align_up((uint64_t)G.ntiles * sizeof(TileItem));
   persist += 2 * gsrc_bytes + 2 * items_bytes;
@@ -174,6 +182,8 @@ Status domain_setup(Domain& d) {
     st = X.mem_info(d, &fr, &tot);
     if (st.bad()) return st;
     budget = fr > kReserveBytes ? fr - kReserveBytes : 0;
+    const uint64_t window = peer ? 4 * halo_bytes + 256 + 2 * st_bytes : 0;  // own cudaMalloc
+    budget = budget > window ? budget - window : 0;
   }
   if (d.opt.device_budget_bytes) budget = std::min<uint64_t>(budget, d.opt.device_budget_bytes);
   if (budget < persist + 2 * tile_bytes)
@@ -224,7 +234,7 @@ Status domain_setup(Domain& d) {
     for (int a = 0; a < 2; ++a)
       for (int p = 0; p < 2; ++p) d.halo[a][p] = reinterpret_cast<double*>(carve(halo_bytes));
   if (peer) {  // before the ghost-source tables, which point into the halos
-    st = peer_setup(d, halo_bytes);
+    st = peer_setup(d, halo_bytes, st_bytes);
     if (st.bad()) return st;
   }
   for (int p = 0; p < 2; ++p) d.gsrc_dev[p] = reinterpret_cast<const double**>(carve(gsrc_bytes));
@@ -311,7 +321,7 @@ Status domain_setup(Domain& d) {
   d.ev_in_base = d.ev_slot_base + d.nslots;
   d.ev_host_base = d.ev_in_base + (int)G.ntiles;
   d.ev_misc_base = d.ev_host_base + (int)G.ntiles;
-  d.nevents = d.ev_misc_base + 4 + d.halo_stream + 1 + 2;  // + 2 stream-through ring events
+  d.nevents = d.ev_misc_base + 4 + d.halo_stream + 1 + 3;  // + 2 stream-through ring events, 1 halo push
   st = X.setup(d);
   if (st.bad()) return st;
   if (multi && !d.opt.dry_run && !d.opt.local_group && !d.opt.peer_transport) {
@@ -744,6 +754,16 @@ static int st_thin_default() {
   return thin;
 }
 
+// Units per H2D copy in the stream-through steady state (TILES_ST_H2D_MERGE,
+// default 2; 1 = one copy per unit).
+static int st_h2d_merge() {
+  static const int m = [] {
+    const char* e = getenv("TILES_ST_H2D_MERGE");
+    return e ? std::max(1, atoi(e)) : 2;
+  }();
+  return m;
+}
+
 static std::vector<UnitDef> make_units(const Geometry& G, int64_t un, int T, int thin) {
   std::vector<UnitDef> v;
   const int64_t tz = G.t[2];
@@ -774,7 +794,10 @@ static std::vector<UnitDef> make_units(const Geometry& G, int64_t un, int T, int
 
 static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
   const Geometry& G = d.G;
-  if (d.opt.stream_through < 0 || G.nranks != 1 || G.bc != TILE_BC_PERIODIC) return false;
+  if (d.opt.stream_through < 0 || G.bc != TILE_BC_PERIODIC) return false;
+  // z-slab ranks: the peer transport's halo layers carry the T planes beyond
+  // each slab end (comm_peer.cu peer_st_halo)
+  if (G.nranks != 1 && !(d.st_halo_bytes && d.peer_connected)) return false;
   if (T < 1 || (int64_t)T > G.t[2]) return false;
   if (G.t[0] % 2 || G.l[2] > (1 << 30)) return false;  // x-pairs (double2); int plane index
   const int64_t plane = G.l[0] * G.l[1];
@@ -857,16 +880,44 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
   auto ev_unit_done = [&](int64_t u) { return ev_host(d, u); };  // compute of unit u
   const int ring_ev[2] = {d.ev_misc_base + 4 + d.halo_stream + 1, d.ev_misc_base + 5 + d.halo_stream + 1};
   const int cs = P.comp(0), os = P.out(0), is = P.in(0);
+  const bool multi = G.nranks > 1;  // z-slab ranks: halo layers replace the periodic wrap
+  const int hs = d.halo_stream;
+  const int ev_push = d.ev_misc_base + 6 + d.halo_stream + 1;
+  if (multi) ++d.st_epoch;
   Status r;
   // one copy-in stream, so the copy engine runs the H2Ds in this order (it
   // may not across streams): the last unit first (unit 0's wrap neighbour)
   std::vector<int64_t> order;
   order.push_back(U - 1);
   for (int64_t u = 0; u < U - 1; ++u) order.push_back(u);
-  for (int64_t u : order) {
-    r = X.h2d_part(d, layer_of(u) * lt, lt, cur_slot(u), p0_of(u), np_of(u), is);
+  // Past the fill, consecutive regular units of one layer share one H2D copy
+  // (up to TILES_ST_H2D_MERGE of them): with D2H running, each copy costs a
+  // ~40 us gap on the H2D side (profiles/r01/pcie_gap.json), and H2D is the
+  // bottleneck of the steady state. The thin end units stay separate.
+  const int merge = st_h2d_merge();
+  for (size_t i = 0; i < order.size();) {
+    const int64_t u = order[i];
+    size_t j = i + 1;
+    int64_t np = np_of(u);
+    if (i >= 3 && np == sp.unit)
+      while (j < order.size() && (int)(j - i) < merge && order[j] == order[j - 1] + 1 &&
+             layer_of(order[j]) == layer_of(u) && np_of(order[j]) == sp.unit)
+        np += np_of(order[j++]);
+    r = X.h2d_part(d, layer_of(u) * lt, lt, cur_slot(u), p0_of(u), np, is);
     if (r.bad()) return r;
-    r = X.record(d, ev_in(d, u), is);
+    for (; i < j; ++i) {
+      r = X.record(d, ev_in(d, order[i]), is);
+      if (r.bad()) return r;
+    }
+  }
+  if (multi) {  // my slab-end planes of initial data to the neighbours, on the halo stream
+    for (int side : {1, 0}) {
+      r = X.wait(d, ev_in(d, side ? U - 1 : 0), hs);
+      if (r.bad()) return r;
+      r = X.st_halo(d, 0, side, T, hs);
+      if (r.bad()) return r;
+    }
+    r = X.record(d, ev_push, hs);
     if (r.bad()) return r;
   }
   for (int64_t u = 0; u < U; ++u) {
@@ -878,6 +929,12 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
       r = X.wait(d, ring_ev[u & 1], cs);
       if (r.bad()) return r;
     }
+    if (multi)  // the slab-end units read the neighbours' planes (halo layers)
+      for (int side : {0, 1})
+        if (u == (side ? U - 1 : 0)) {
+          r = X.st_halo(d, 1, side, T, cs);
+          if (r.bad()) return r;
+        }
     // sweep i reads planes [i-1, n+2T-i+1) and writes [i, n+2T-i); the
     // first reads the resident array directly (gather fused), the last writes
     // the unit's packed sub-tiles (scatter fused)
@@ -892,6 +949,12 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
         r = X.copy_part(d, res_of(u - 1), cur_slot(u - 1), lt, p0_of(u - 1), np_of(u - 1), cs);
         if (r.bad()) return r;
       }
+      if (i == 1 && multi)  // halo layers read: their senders may reuse them
+        for (int side : {0, 1})
+          if (u == (side ? U - 1 : 0)) {
+            r = X.st_halo(d, 2, side, T, cs);
+            if (r.bad()) return r;
+          }
     }
     r = X.record(d, ev_unit_done(u), cs);
     if (r.bad()) return r;
@@ -903,6 +966,10 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
       r = X.record(d, ring_ev[u & 1], os);
       if (r.bad()) return r;
     }
+  }
+  if (multi) {  // the pushes read units 0 and U-1's initial data, overwritten below
+    r = X.wait(d, ev_push, cs);
+    if (r.bad()) return r;
   }
   if (U >= 2) {
     r = X.copy_part(d, res_of(U - 1), cur_slot(U - 1), lt, p0_of(U - 1), np_of(U - 1), cs);

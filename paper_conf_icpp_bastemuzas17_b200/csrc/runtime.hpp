@@ -141,6 +141,11 @@ struct Exec {
   // 1 = copies, and arm the next exchange, whose data the kernels push
   // (fused); 2 = signal only: the previous step's kernels pushed the data
   virtual Status halo(Domain& d, int parity, int stream, int mode = 0) = 0;
+  // multi-rank stream-through (comm_peer.cu): op 0 = push my slab-end T
+  // planes of initial data (side 1: top -> upper, 0: bottom -> lower) once the
+  // receiver has released the previous run's; 1 = wait until side's halo
+  // layer has arrived; 2 = release side's halo layer (read by the first sweep)
+  virtual Status st_halo(Domain& d, int op, int side, int T, int stream) = 0;
   virtual Status note(Domain& d, int kind, int64_t a, int64_t b, int stream) = 0;  // trace-only ops
   virtual Status sync_all(Domain& d) = 0;
   // resources
@@ -248,6 +253,12 @@ struct Domain {
   uint32_t peer_k = 0;
   bool peer_connected = false;
   bool peer_fused = false;                 // resident direct passes push z halos from the kernel
+  // multi-rank stream-through: two tile layers in the window
+  // ([0] lo: the lower neighbour's top T planes of initial data, [1] hi: the
+  // upper neighbour's bottom T planes), tile-blocked like the resident array
+  double* st_halo[2] = {nullptr, nullptr};
+  uint64_t st_halo_bytes = 0;              // one layer (0: no multi-rank stream-through)
+  uint32_t st_epoch = 0;                   // multi-rank stream-through runs so far
 
   // kernel plan
   int band = 0, stages = 0, heat_grid = 0, sm_count = 148;
@@ -307,7 +318,8 @@ void nccl_destroy(Domain& d);
 Status local_group_create(int n, void** out);
 void local_group_free(void* g);
 Status local_halo(Domain& d, int parity, void* stream, void* ready_event);
-Status peer_setup(Domain& d, uint64_t halo_bytes);
+Status peer_setup(Domain& d, uint64_t halo_bytes, uint64_t st_bytes);
+Status peer_st_halo(Domain& d, int op, int side, int T, void* stream);
 Status peer_handle(const Domain& d, void* out64);
 Status peer_connect(Domain& d, const void* handles, int n);
 Status peer_halo(Domain& d, int parity, void* stream, int mode);

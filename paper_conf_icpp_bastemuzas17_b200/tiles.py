@@ -34,7 +34,8 @@ TILE_MEASURE_NORMAL, TILE_MEASURE_XFER_ONLY, TILE_MEASURE_COMP_ONLY = 0, 1, 2
 OP_NAMES = {1: "h2d", 2: "d2h", 3: "kernel", 4: "record", 5: "wait", 6: "faces_h2d",
             7: "extract", 8: "halo", 9: "drop", 10: "hit", 11: "pointwise", 12: "kernel2",
             13: "gather", 14: "sweep", 15: "scatter", 16: "copy", 17: "h2d_part", 18: "d2h_part",
-            19: "copy_part", 20: "h2d_pack", 21: "sweep_u", 22: "kerneld", 23: "halo_signal"}
+            19: "copy_part", 20: "h2d_pack", 21: "sweep_u", 22: "kerneld", 23: "halo_signal",
+            24: "st_halo"}
 SCHEDS = {"auto": 0, "resident": 1, "stream": 2, "sync": 3}
 BCS = {"periodic": 0, "dirichlet": 1}
 

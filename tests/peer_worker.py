@@ -7,14 +7,14 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def run(r, G, dims, td, bc, sched, budget, runs, seed, conn, transport=1):
+def run(r, G, dims, td, bc, sched, budget, runs, seed, conn, transport=1, stream_through=0):
     sys.path.insert(0, ROOT)
     try:
         import synth
         from paper_conf_icpp_bastemuzas17_b200 import tiles as T
         nx, ny, nz = dims
         nzl = nz // G
-        kw = {"sched": sched}
+        kw = {"sched": sched, "stream_through": stream_through}
         if budget:
             kw["device_budget_bytes"] = budget
         with T.Domain(dims, td, bc=bc, nranks=G, rank=r, peer_transport=transport, device=0, **kw) as d:
@@ -27,10 +27,14 @@ def run(r, G, dims, td, bc, sched, budget, runs, seed, conn, transport=1):
             else:
                 ext = synth.uniform_grid(nx + 2, ny + 2, nz + 2, seed)
                 d.load(ext[r * nzl:r * nzl + nzl + 2])
-            for s in runs:
+            firsts = []
+            for i, s in enumerate(runs):
                 d.run(T.heat7(0.125), s, 2)
+                if i == 0:
+                    d.sync()
+                    firsts = [d.stats(), d.store()]
             out = d.store()
             st = d.stats()
-        conn.send(("out", out, st["n_halo"], st["bytes_halo"]))
+        conn.send(("out", out, st["n_halo"], st["bytes_halo"], firsts))
     except Exception as e:  # noqa: BLE001
         conn.send(("error", repr(e)))

@@ -94,16 +94,32 @@ def test_peer_transport_processes_bit_exact(G, bc, sched, runs, transport):
     kernel of every resident step stores its slab-end layers straight into
     the neighbours' windows and the exchange only signals. Bit-exact against
     the oracle."""
-    import multiprocessing as mp
-    from tests import peer_worker
     dims, td = (64, 32, 16 * G), (32, 16, 8)
     nx, ny, nz = dims
     budget = _budget(dims, td, 3, bc=bc, nranks=G, rank=0) if sched == "stream" else 0
+    outs = _peer_procs(G, dims, td, bc, sched, budget, runs, transport)
+    got = np.concatenate([m[1] for m in outs], axis=0)
+    if bc == "periodic":
+        ref = oracle.heat_c(synth.uniform_grid(nx, ny, nz, 42), ALPHA, sum(runs))
+    else:
+        ext = synth.uniform_grid(nx + 2, ny + 2, nz + 2, 42)
+        ref = oracle.heat_c(ext, ALPHA, sum(runs), oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+        got = np.concatenate([m[1][1:-1, 1:-1, 1:-1] for m in outs], axis=0)
+    assert np.array_equal(got, ref), np.abs(got - ref).max()
+    assert all(m[2] > 0 and m[3] > 0 for m in outs)  # halo exchanges happened through the window
+
+
+def _peer_procs(G, dims, td, bc, sched, budget, runs, transport, stream_through=0):
+    """One spawned process per rank (tests/peer_worker.py), IPC handles
+    relayed through pipes; returns every rank's ("out", ...) message."""
+    import multiprocessing as mp
+    from tests import peer_worker
     ctx = mp.get_context("spawn")
     pipes, procs = [], []
     for r in range(G):
         a, b = ctx.Pipe()
-        p = ctx.Process(target=peer_worker.run, args=(r, G, dims, td, bc, sched, budget, runs, 42, b, transport))
+        p = ctx.Process(target=peer_worker.run,
+                        args=(r, G, dims, td, bc, sched, budget, runs, 42, b, transport, stream_through))
         p.start()
         pipes.append(a)
         procs.append(p)
@@ -127,12 +143,31 @@ def test_peer_transport_processes_bit_exact(G, bc, sched, runs, transport):
             p.join(30)
             if p.is_alive():
                 p.kill()
+    return outs
+
+
+@pytest.mark.parametrize("G,T,tz,runs_after", [(2, 4, 8, [3]), (3, 8, 16, []), (4, 1, 8, [2]),
+                                               (2, 8, 16, [5, 4]), (2, 3, 8, [])])
+def test_peer_stream_through_slabs_bit_exact(G, T, tz, runs_after):
+    """Multi-rank stream-through (fresh upload, T <= tz, peer transport): each
+    rank sweeps its slab in units of planes; the T planes of initial data
+    beyond each slab end come once per run from the neighbours' halo layers
+    (comm_peer.cu peer_st_halo) instead of the periodic wrap. One process per
+    rank on the pool's GPU; the first run's result (host) and the resident
+    runs that continue from the device copy are bit-exact against the oracle,
+    and the first run moved each cell across the link exactly once per
+    direction."""
+    dims, td = (64, 32, 8 * tz * G), (32, 16, tz)  # 8 tile layers per rank
+    nx, ny, nz = dims
+    runs = [T] + runs_after
+    outs = _peer_procs(G, dims, td, "periodic", "auto", 0, runs, transport=2, stream_through=1)
+    u0 = synth.uniform_grid(nx, ny, nz, 42)
+    first = np.concatenate([m[4][1] for m in outs], axis=0)
+    assert np.array_equal(first, oracle.heat_c(u0, ALPHA, T)), np.abs(first - oracle.heat_c(u0, ALPHA, T)).max()
     got = np.concatenate([m[1] for m in outs], axis=0)
-    if bc == "periodic":
-        ref = oracle.heat_c(synth.uniform_grid(nx, ny, nz, 42), ALPHA, sum(runs))
-    else:
-        ext = synth.uniform_grid(nx + 2, ny + 2, nz + 2, 42)
-        ref = oracle.heat_c(ext, ALPHA, sum(runs), oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
-        got = np.concatenate([m[1][1:-1, 1:-1, 1:-1] for m in outs], axis=0)
-    assert np.array_equal(got, ref), np.abs(got - ref).max()
-    assert all(m[2] > 0 and m[3] > 0 for m in outs)  # halo exchanges happened through the window
+    assert np.array_equal(got, oracle.heat_c(u0, ALPHA, sum(runs)))
+    nzl = nz // G
+    for m in outs:
+        st = m[4][0]
+        assert st["bytes_h2d"] == nx * ny * nzl * 8 and st["bytes_d2h"] == nx * ny * nzl * 8
+        assert st["bytes_halo"] == 2 * nx * ny * T * 8  # one layer of T planes to each neighbour
