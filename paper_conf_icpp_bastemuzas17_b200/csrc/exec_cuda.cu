@@ -198,6 +198,13 @@ struct CudaExec final : Exec {
     const int64_t planes = (int64_t)n * p.nbands * p.tz;
     int64_t grid = (int64_t)sms * heat_occ;
     grid = std::max<int64_t>(1, std::min<int64_t>(grid, (planes + 3) / 4));
+    // banded tiles: adjacent bands side by side in time (their shared halo
+    // rows from L2); TILES_HEAT_RR=0 keeps contiguous plane ranges
+    static const int rr_on = [] {
+      const char* e = std::getenv("TILES_HEAT_RR");
+      return e ? std::atoi(e) : 1;
+    }();
+    p.rr_rounds = rr_on && p.nbands > 1 ? (int32_t)((int64_t)p.lt * p.nbands / grid) : 0;
     p.nsteps = 1;
     if (nsteps > 1) {  // one persistent launch for all steps (CTA progress counters)
       const int b1 = direct_bit ^ 1;

@@ -96,6 +96,38 @@ struct PlaneRange {
 };
 
 
+// Runs (column, first plane, planes) of this CTA for the specialised kernel:
+// round-robin whole columns first (HeatParams::rr_rounds), then a contiguous
+// share of the remaining columns' planes.
+struct Runs {
+  int64_t c, cend, pp, pe;
+  int NZ;
+  __device__ explicit Runs(const HeatParams& p) {
+    NZ = p.nstack * p.tz;
+    const int64_t ncols = (int64_t)p.lt * p.nbands;
+    cend = (int64_t)p.rr_rounds * gridDim.x;
+    c = blockIdx.x;
+    const int64_t P = (ncols - cend) * NZ;
+    pp = cend * NZ + P * blockIdx.x / gridDim.x;
+    pe = cend * NZ + P * (blockIdx.x + 1) / gridDim.x;
+  }
+  __device__ __forceinline__ bool next(int64_t& col, int& g0, int& n) {
+    if (c < cend) {
+      col = c;
+      g0 = 0;
+      n = NZ;
+      c += gridDim.x;
+      return true;
+    }
+    if (pp >= pe) return false;
+    col = pp / NZ;
+    g0 = (int)(pp - col * NZ);
+    n = (int)(pe - pp < (int64_t)(NZ - g0) ? pe - pp : NZ - g0);
+    pp += n;
+    return true;
+  }
+};
+
 // ---- specialised kernel: compile-time tile width TX, band height BY and
 // ring depth S. Each thread owns column pair c2 and rows r0 + j*RPP
 // (j < NR) of the band in EVERY plane (register z-march: z-1 and z values
@@ -141,8 +173,6 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
   __syncthreads();
 
   const int ty = p.ty, tz = p.tz;
-  const PlaneRange R(p);
-  const int NZ = R.NZ;
   const int nsteps = p.nsteps > 1 ? p.nsteps : 1;
 
   if ((int)threadIdx.x >= C::NT) {  // ---------------- producer warp
@@ -152,10 +182,10 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
       const bool odd = s & 1;
       const TileItem* items = odd ? p.items_odd : p.items;
       const double* const* gtab = odd ? p.gdir_odd : (p.gdir ? p.gdir : p.gsrc);
-      for (int64_t pp = R.pb; pp < R.pe;) {
-        const int64_t col = pp / NZ;
-        const int g0 = (int)(pp - col * NZ);
-        const int n = (int)(R.pe - pp < (int64_t)(NZ - g0) ? R.pe - pp : NZ - g0);
+      Runs W(p);
+      int64_t col;
+      int g0, n;
+      while (W.next(col, g0, n)) {
         const int icol = (int)(col / p.nbands);
         const int y0 = (int)(col - (int64_t)icol * p.nbands) * BY;
         // planes g0-1 .. g0+n: stacked tile L, local plane z (z = -1 / tz at the
@@ -176,7 +206,6 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
           stage_plane(stage_base + (size_t)st * C::STAGE_ELEMS, &full[st], it.in, gs, ys, z, TX, ty, tz,
                       y0, BY, p.cache_flags, D);
         }
-        pp += n;
       }
       if (s + 1 < nsteps) {
         // step barrier: every consumer of this CTA done with step s (drain the
@@ -231,10 +260,10 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
   const bool odd = s & 1;
   const TileItem* items = odd ? p.items_odd : p.items;
   auto fexp = [&](int f) { return odd ? p.fexp_odd[f] : p.fexp[f]; };
-  for (int64_t pp = R.pb; pp < R.pe;) {
-    const int64_t col = pp / NZ;
-    const int g0 = (int)(pp - col * NZ);
-    const int n = (int)(R.pe - pp < (int64_t)(NZ - g0) ? R.pe - pp : NZ - g0);
+  Runs W(p);
+  int64_t col;
+  int g0, n;
+  while (W.next(col, g0, n)) {
     const int icol = (int)(col / p.nbands);
     const int yb = (int)(col - (int64_t)icol * p.nbands) * BY + r0;
 
@@ -343,7 +372,6 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
     }
     release_g(seq + n + 1);  // plane g0+n (last z+1 neighbour)
     seq += (uint32_t)(n + 2);
-    pp += n;
   }
   }
   // pushed halo layers visible system-wide (the neighbour ranks' GPUs) before

@@ -64,6 +64,13 @@ struct HeatParams {
   // between stacked tiles are the neighbour's own planes already in the ring.
   // nstack = 1, lt = nitems: independent tiles.
   int32_t nstack, lt;
+  // Work order of the specialised kernels: the first rr_rounds * gridDim.x
+  // columns (of lt * nbands) go round-robin, whole (CTA b takes columns b,
+  // b + grid, ...: CTAs running side by side march adjacent bands of a tile
+  // through the same planes, so the halo rows one reads are the rows its
+  // neighbour CTA just staged — L2 hits instead of DRAM re-reads); the rest
+  // is split into contiguous plane ranges. rr_rounds = 0: all contiguous.
+  int32_t rr_rounds;
   // Exports: x faces always; y faces iff exp_y; the z- face of tile k iff
   // k < exp_zlo_below, the z+ face iff k >= exp_zhi_from (direct runs export
   // only what a face reader still needs: the slab-end layers' z faces for the

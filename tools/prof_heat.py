@@ -6,8 +6,11 @@ import numpy as np
 import synth
 from paper_conf_icpp_bastemuzas17_b200 import tiles as T
 n = int(os.environ.get("N", "512")); t = int(os.environ.get("TILE", "64"))
-u = np.empty((n, n, n)); synth.fill_uniform_native(u.ctypes.data, n, n, n, 0, n, 0, n, 0, n, 42)
-d = T.Domain((n, n, n), (t, t, t), ghost=int(os.environ.get("GHOST", "1")), stream_through=-1,
+# DIMS="nx,ny,nz" / TD="tx,ty,tz" override the cube (e.g. a C5 slab: 4096,4096,128 / 256,256,64)
+dims = tuple(int(v) for v in os.environ["DIMS"].split(",")) if "DIMS" in os.environ else (n, n, n)
+td = tuple(int(v) for v in os.environ["TD"].split(",")) if "TD" in os.environ else (t, t, t)
+u = np.empty(dims[::-1]); synth.fill_uniform_native(u.ctypes.data, *dims, 0, dims[2], 0, dims[1], 0, dims[0], 42)
+d = T.Domain(dims, td, ghost=int(os.environ.get("GHOST", "1")), stream_through=-1,
              two_step=int(os.environ.get("TWO_STEP", "0")))
 d.load(u); d.run(T.heat7(), 1, 4); d.sync()
 d.run(T.heat7(), int(os.environ.get("STEPS", "4")), 4); d.sync()
