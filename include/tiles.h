@@ -222,7 +222,7 @@ typedef enum {
   TILE_OP_ST_HALO = 24   /* multi-rank stream-through (peer transport): a = 0 push the
                             slab-end c planes of initial data (b = 1 top -> upper rank,
                             0 bottom -> lower rank), 1 wait for side b's halo layer,
-                            2 release side b's halo layer */
+                            2 release side b's halo layer; d = the run's epoch */
 } tile_op_kind;
 
 typedef struct {

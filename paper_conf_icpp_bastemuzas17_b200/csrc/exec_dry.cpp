@@ -151,7 +151,7 @@ struct DryExec final : Exec {
       d.stats.n_halo++;
       d.stats.bytes_halo += (uint64_t)d.G.layer_tiles * T * d.G.t[0] * d.G.t[1] * 8;
     }
-    put(d, TILE_OP_ST_HALO, st, op, side, T, 0);
+    put(d, TILE_OP_ST_HALO, st, op, side, T, d.st_epoch);
     return Status::ok();
   }
   Status note(Domain& d, int kind, int64_t a, int64_t b, int st) override {

@@ -163,6 +163,10 @@ Status domain_setup(Domain& d) {
     const uint64_t layer = align_up((uint64_t)G.layer_tiles * G.tile_elems * 8);
     if (2 * layer <= kStHaloMax) st_bytes = layer;
   }
+  // dry runs (trace replay on CPU) of a peer-transport domain take the same
+  // multi-rank stream-through decisions, with no window behind them
+  if (multi && d.opt.peer_transport && d.opt.dry_run && G.bc == TILE_BC_PERIODIC && d.opt.stream_through >= 0)
+    d.st_halo_bytes = (uint64_t)G.layer_tiles * G.tile_elems * 8;
   const uint64_t gsrc_bytes = align_up((uint64_t)G.ntiles * 6 * sizeof(double*));
   const uint64_t items_bytes = align_up((uint64_t)G.ntiles * sizeof(TileItem));
   persist += 2 * gsrc_bytes + 2 * items_bytes;
@@ -797,7 +801,7 @@ static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
   if (d.opt.stream_through < 0 || G.bc != TILE_BC_PERIODIC) return false;
   // z-slab ranks: the peer transport's halo layers carry the T planes beyond
   // each slab end (comm_peer.cu peer_st_halo)
-  if (G.nranks != 1 && !(d.st_halo_bytes && d.peer_connected)) return false;
+  if (G.nranks != 1 && !(d.st_halo_bytes && (d.peer_connected || d.opt.dry_run))) return false;
   if (T < 1 || (int64_t)T > G.t[2]) return false;
   if (G.t[0] % 2 || G.l[2] > (1 << 30)) return false;  // x-pairs (double2); int plane index
   const int64_t plane = G.l[0] * G.l[1];

@@ -97,6 +97,13 @@ class Replayer:
         self.halo = {}
         self.comm = comm
         self.peers = {}    # rank -> Replayer (joint multi-rank replay, fused pushes)
+        # multi-rank stream-through (comm_peer.cu peer_st_halo): halo layers
+        # [0] lo (the lower rank's top planes), [1] hi (the upper rank's bottom
+        # planes) and their counters: S (arrived epoch) and CR (credit: the
+        # receiver on that side released the epoch's layer I pushed)
+        self.st = {0: None, 1: None}
+        self.st_arrived = {0: 0, 1: 0}
+        self.st_credit = {0: 0, 1: 0}
 
     def dirichlet_face(self, k, f):
         G = self.G
@@ -385,7 +392,14 @@ class Replayer:
         nz = G.l[2]
         out = np.empty((planes, G.l[1], G.l[0]))
         for p in range(planes):
-            gz = (zbase + p) % nz
+            gz = zbase + p
+            if G.nranks > 1 and (gz < 0 or gz >= nz):  # beyond the slab: the neighbours' planes
+                side = 0 if gz < 0 else 1
+                layer = self.st[side]
+                assert layer is not None, "stream-through read a halo layer that never arrived"
+                out[p] = layer[gz + layer.shape[0]] if side == 0 else layer[gz - nz]
+                continue
+            gz %= nz
             iz, lz = gz // tz, gz % tz
             for iy in range(G.n[1]):
                 for ix in range(G.n[0]):
@@ -480,9 +494,11 @@ def halo_peers(G):
     return up, dn
 
 
-def replay_ranks(reps, traces, seed):
+def replay_ranks(reps, traces, seed, lazy=()):
     """Joint random replay of several ranks' traces; the k-th halo op of
-    every rank executes together (a collective)."""
+    every rank executes together (a collective). Ops named in `lazy` run only
+    when nothing else can (adversarial order: e.g. halo pushes as late as
+    their dependencies allow)."""
     rng = random.Random(seed)
     for rep in reps:
         rep.peers = {r: x for r, x in enumerate(reps)}
@@ -514,13 +530,21 @@ def replay_ranks(reps, traces, seed):
                     continue
                 if op[0] in ("halo", "halo_signal"):
                     halo_heads[r] = (s, i)
+                elif op[0] == "st_halo":
+                    # stream-through halo op (a = 0 push, 1 wait, 2 release; b =
+                    # side; c = T; d = epoch): ready when its counter condition holds
+                    _, _, a, side, _, e = op
+                    if (a == 0 and reps[r].st_credit[side] >= e - 1) or \
+                            (a == 1 and reps[r].st_arrived[side] >= e) or a == 2:
+                        ready.append((r, s, i))
                 else:
                     ready.append((r, s, i))
         if len(halo_heads) == len(reps):
             ready.append(("halo", None, None))
         if not ready:
             raise RuntimeError("multi-rank replay deadlock")
-        pick = rng.choice(ready)
+        eager = [x for x in ready if x[0] == "halo" or traces[x[0]][x[2]][0] not in lazy]
+        pick = rng.choice(eager or ready)
         if pick[0] == "halo":
             par = traces[0][halo_heads[0][1]][5]
             kind = traces[0][halo_heads[0][1]][0]
@@ -545,7 +569,20 @@ def replay_ranks(reps, traces, seed):
                 remaining -= 1
             continue
         r, s, i = pick
-        reps[r].execute(traces[r][i], state[r]["snap"])
+        op = traces[r][i]
+        if op[0] == "st_halo":
+            _, _, a, side, T, e = op
+            up, dn = halo_peers(reps[r].G)
+            peer = reps[up if side == 1 else dn]
+            if a == 0:  # my slab-end T planes of the current resident data -> the peer's layer
+                nz = reps[r].G.l[2]
+                peer.st[1 - side] = reps[r].gather(T, nz - T if side == 1 else 0)
+                peer.st_arrived[1 - side] = e
+            elif a == 2:  # released: its sender may overwrite it from now on
+                reps[r].st[side] = np.full_like(reps[r].st[side], np.nan)
+                peer.st_credit[1 - side] = e
+        else:
+            reps[r].execute(op, state[r]["snap"])
         state[r]["done"].add(i)
         state[r]["pos"][s] += 1
         remaining -= 1

@@ -107,6 +107,47 @@ def test_slab_replay_matches_global_oracle(G, bc, sched, td, fused):
     assert np.array_equal(out, ref), np.abs(out - ref).max()
 
 
+@pytest.mark.parametrize("G,T_,tz,ns", [(2, 4, 8, 2), (3, 3, 8, 4), (4, 1, 8, 2), (2, 8, 16, 3)])
+def test_slab_stream_through_replay_matches_global_oracle(G, T_, tz, ns):
+    """Multi-rank stream-through (peer transport, fresh upload, T <= tz): each
+    rank's dry-run trace holds its unit pipeline plus the st_halo ops — push
+    the slab-end T planes of initial data once its H2D landed and the receiver
+    released the previous run's layer; wait for the neighbours' layers before
+    the slab-end units' first sweeps; release after them. The joint random
+    replay moves the planes between ranks only when a push executes, poisons
+    a layer on release, and makes waits / pushes block on the counters, so a
+    missing dependency reads NaN or stale planes. Two stream-through runs
+    (fresh uploads, the second pushing into layers the first released) and a
+    resident run from the device copy must equal the global oracle."""
+    dims, td = (64, 32, 8 * tz * G), (32, 16, tz)
+    u, _, _ = _global(dims, "periodic")
+    nzl = dims[2] // G
+    doms, reps = [], []
+    for r in range(G):
+        doms.append(_rank_domain(dims, td, G, r, "periodic", None, u, peer_transport=2, stream_through=1))
+        geo = Geometry(dims, td, nranks=G, rank=r, bc=0)
+        reps.append(Replayer(geo, split_tiles(geo, u[r * nzl:(r + 1) * nzl]), ALPHA))
+    total = 0
+    for run, (steps, fresh) in enumerate([(T_, True), (T_, True), (3, False)]):
+        traces = []
+        for d in doms:
+            if fresh and run:
+                d.invalidate()  # re-upload from the host store: a fresh stream-through run
+            d.clear_trace()
+            d.run(T.heat7(ALPHA), steps, ns)
+            d.sync()
+            traces.append(d.trace())
+        sth = [op for op in traces[0] if op[0] == "st_halo"]
+        assert (len(sth) == 6) == fresh, sth   # 2 pushes, 2 waits, 2 releases per rank
+        assert all(op[5] == run + 1 for op in sth)
+        # odd runs: halo ops as late as possible (a push that the final
+        # write-back does not wait for would then read results, not u^0)
+        replay_ranks(reps, traces, seed=17 * run + G, lazy=("st_halo",) if run % 2 else ())
+        total += steps
+        out = np.concatenate([rep.grid() for rep in reps], axis=0)
+        assert np.array_equal(out, oracle.heat_c(u, ALPHA, total)), (run, np.abs(out - oracle.heat_c(u, ALPHA, total)).max())
+
+
 def test_slab_geometry_and_face_kinds():
     d = T.Domain((16, 16, 32), (8, 8, 4), nranks=4, rank=1, dry_run=True)
     info = d.info
