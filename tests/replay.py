@@ -420,7 +420,13 @@ class Replayer:
         out[lo:hi] = new
         return out
 
-    def replay(self, trace, seed):
+    def replay(self, trace, seed, st_ready=None, st_exec=None, timeout=120.0):
+        """Random valid order of one rank's trace. st_ready / st_exec: the
+        multi-process transport of stream-through halo ops (an op is runnable
+        when st_ready(self, op); st_exec(self, op) performs it); while only
+        such ops remain blocked the replay polls instead of failing."""
+        import time
+        t_end = time.time() + timeout
         rng = random.Random(seed)
         snapshot = {(k, f): p for k in range(self.G.ntiles)
                     for f, p in enumerate(faces_of(self.host[k], self.G.depth))}
@@ -446,12 +452,20 @@ class Replayer:
                     op = trace[i]
                     if op[0] == "wait" and bound[i] is not None and bound[i] not in done:
                         continue
+                    if op[0] == "st_halo" and st_ready is not None and not st_ready(self, op):
+                        continue
                     ready.append(s)
             if not ready:
+                if st_ready is not None and time.time() < t_end:
+                    time.sleep(0.002)  # a neighbour's halo layer is in flight
+                    continue
                 raise RuntimeError("replay deadlock: no stream can make progress")
             s = rng.choice(ready)
             i = queues[s][pos[s]]
-            self.execute(trace[i], snapshot)
+            if trace[i][0] == "st_halo" and st_exec is not None:
+                st_exec(self, trace[i])
+            else:
+                self.execute(trace[i], snapshot)
             done.add(i)
             pos[s] += 1
             remaining -= 1

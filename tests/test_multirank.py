@@ -225,6 +225,73 @@ def _gloo_worker(rank, world, port, bc, sched, out_q):
         dist.destroy_process_group()
 
 
+def _gloo_st_worker(rank, world, port, out_q):
+    """Multi-rank stream-through over gloo: this process replays its rank's
+    dry-run trace; an st_halo push is a gloo isend of the slab-end T planes
+    (tag = the receiver's side), a wait is runnable once the matching irecv
+    (posted up front) has completed, a release poisons the layer."""
+    import torch
+    import torch.distributed as dist
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    try:
+        Tst, tz = 4, 8
+        dims, td = (64, 32, 8 * tz * world), (32, 16, tz)
+        u, _, _ = _global(dims, "periodic")
+        nzl = dims[2] // world
+        d = _rank_domain(dims, td, world, rank, "periodic", None, u, peer_transport=2, stream_through=1)
+        geo = Geometry(dims, td, nranks=world, rank=rank, bc=0)
+        rep = Replayer(geo, split_tiles(geo, u[rank * nzl:(rank + 1) * nzl]), ALPHA)
+        d.run(T.heat7(ALPHA), Tst, 2)
+        d.sync()
+        tr = d.trace()
+        assert sum(op[0] == "st_halo" for op in tr) == 6
+        up, dn = halo_peers(geo)
+        bufs = {side: torch.empty((Tst, dims[1], dims[0]), dtype=torch.float64) for side in (0, 1)}
+        recv = {0: dist.irecv(bufs[0], src=dn, tag=0), 1: dist.irecv(bufs[1], src=up, tag=1)}
+        # gloo marks an irecv complete only in wait(): wait in helper threads
+        import threading
+        arrived = {side: threading.Event() for side in (0, 1)}
+        for side in (0, 1):
+            threading.Thread(target=lambda sd=side: (recv[sd].wait(), arrived[sd].set()), daemon=True).start()
+        sends = []
+
+        def st_ready(r, op):
+            return op[2] != 1 or arrived[op[3]].is_set()
+
+        def st_exec(r, op):
+            _, _, a, side, T_, _ = op
+            if a == 0:  # top -> upper's lo (tag 0), bottom -> lower's hi (tag 1)
+                planes = r.gather(T_, nzl - T_ if side == 1 else 0)
+                sends.append(dist.isend(torch.from_numpy(np.ascontiguousarray(planes)),
+                                        dst=up if side == 1 else dn, tag=1 - side))
+            elif a == 1:
+                r.st[side] = bufs[side].numpy().copy()
+            else:
+                r.st[side] = np.full_like(r.st[side], np.nan)
+
+        rep.replay(tr, seed=rank + 5, st_ready=st_ready, st_exec=st_exec)
+        for w in sends:
+            w.wait()
+        ok = np.array_equal(rep.grid(), oracle.heat_c(u, ALPHA, Tst)[rank * nzl:(rank + 1) * nzl])
+        out_q.put((rank, bool(ok)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_world2_stream_through():
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_gloo_st_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(180)
+    res = dict(q.get(timeout=5) for _ in range(2))
+    assert res == {0: True, 1: True}
+
+
 @pytest.mark.parametrize("bc,sched", [("periodic", "resident"), ("dirichlet", "stream"),
                                       ("periodic", "stream")])
 def test_gloo_world2_halo_exchange(bc, sched):
