@@ -91,8 +91,11 @@ if __name__ == "__main__":
             print(d["kernel"][:80], "dur", g("gpu__time_duration.sum"), d["gpu__time_duration.sum"]["unit"],
                   "dram R+W bytes", traffic, "dram%", g("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed"))
             if "heat7_fixed" in d["kernel"]:
+                # per STEP: a persistent capture covers NCU_STEPS steps (tools/prof_heat.py STEPS)
+                steps = int(os.environ.get("NCU_STEPS", "4")) if "persistent" in tag else 1
                 tp = os.path.join(ROOT, "profiles", "heat7_ncu_traffic.json")
                 j = json.load(open(tp)) if os.path.exists(tp) else {}
-                j["c2"] = traffic
-                j["c2_source"] = f"profiles/{rnd}/{tag}.json (ncu --set full, whole-domain launch of C2)"
+                j["c2"] = traffic / steps
+                j["c2_source"] = (f"profiles/{rnd}/{tag}.json (ncu --set full, whole-domain launch of C2, "
+                                  f"{steps} step(s) per launch; DRAM read + write per step)")
                 json.dump(j, open(tp, "w"), indent=1)
