@@ -209,6 +209,18 @@ struct CudaExec final : Exec {
     if (nsteps > 1) {  // one persistent launch for all steps (CTA progress counters)
       const int b1 = direct_bit ^ 1;
       p.nsteps = nsteps;
+      // snake order across steps (TILES_SNAKE=0: off; TILES_SNAKE_KEEP: planes
+      // per CTA stored evict_last at the end of a step, default 16)
+      static const int snake = [] {
+        const char* e = std::getenv("TILES_SNAKE");
+        return e ? std::atoi(e) : 1;
+      }();
+      static const int keep_tail = [] {
+        const char* e = std::getenv("TILES_SNAKE_KEEP");
+        return e ? std::atoi(e) : 16;
+      }();
+      p.snake = snake;
+      p.keep_tail = snake ? keep_tail : 0;
       p.ntx = (int32_t)d.G.n[0];
       p.nty = (int32_t)d.G.n[1];
       p.epoch = d.prog_epoch;

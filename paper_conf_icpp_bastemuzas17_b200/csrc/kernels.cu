@@ -100,18 +100,38 @@ struct PlaneRange {
 // round-robin whole columns first (HeatParams::rr_rounds), then a contiguous
 // share of the remaining columns' planes.
 struct Runs {
-  int64_t c, cend, pp, pe;
+  int64_t c, cend, pp, pe, total;
   int NZ;
-  __device__ explicit Runs(const HeatParams& p) {
+  bool rev;  // snake order: the same runs in reverse, each run's planes descending
+  __device__ Runs(const HeatParams& p, bool reverse) {
     NZ = p.nstack * p.tz;
+    rev = reverse;
     const int64_t ncols = (int64_t)p.lt * p.nbands;
     cend = (int64_t)p.rr_rounds * gridDim.x;
-    c = blockIdx.x;
     const int64_t P = (ncols - cend) * NZ;
     pp = cend * NZ + P * blockIdx.x / gridDim.x;
     pe = cend * NZ + P * (blockIdx.x + 1) / gridDim.x;
+    const int64_t mine = cend > (int64_t)blockIdx.x ? (cend - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    total = mine * NZ + (pe - pp);
+    c = !rev ? (int64_t)blockIdx.x : mine ? (int64_t)blockIdx.x + (mine - 1) * gridDim.x : -1;
   }
   __device__ __forceinline__ bool next(int64_t& col, int& g0, int& n) {
+    if (rev) {
+      if (pe > pp) {
+        col = (pe - 1) / NZ;
+        const int64_t start = pp > col * NZ ? pp : col * NZ;
+        g0 = (int)(start - col * NZ);
+        n = (int)(pe - start);
+        pe = start;
+        return true;
+      }
+      if (c < (int64_t)blockIdx.x) return false;
+      col = c;
+      g0 = 0;
+      n = NZ;
+      c -= gridDim.x;
+      return true;
+    }
     if (c < cend) {
       col = c;
       g0 = 0;
@@ -180,24 +200,35 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
     uint32_t g = 0;
     for (int s = 0; s < nsteps; ++s) {
       const bool odd = s & 1;
+      const bool rev = p.snake && odd;
       const TileItem* items = odd ? p.items_odd : p.items;
       const double* const* gtab = odd ? p.gdir_odd : (p.gdir ? p.gdir : p.gsrc);
-      Runs W(p);
+      Runs W(p, rev);
       int64_t col;
       int g0, n;
+      const int NZ = W.NZ;
       while (W.next(col, g0, n)) {
         const int icol = (int)(col / p.nbands);
         const int y0 = (int)(col - (int64_t)icol * p.nbands) * BY;
-        // planes g0-1 .. g0+n: stacked tile L, local plane z (z = -1 / tz at the
-        // stack ends stage the z ghost planes)
-        int L = g0 / tz, z = g0 - L * tz - 1;
-        if (z < 0 && L > 0) --L, z += tz;
+        // planes g0-1 .. g0+n in march order (descending when rev): stacked
+        // tile L, local plane z (z = -1 / tz at the stack ends stage the z
+        // ghost planes)
+        auto locate = [&](int gp, int& L, int& z) {
+          if (gp < 0) L = 0, z = -1;
+          else if (gp >= NZ) L = p.nstack - 1, z = tz;
+          else L = gp / tz, z = gp - L * tz;
+        };
+        int L, z;
+        locate(rev ? g0 + n : g0 - 1, L, z);
         TileItem it = items ? items[L * p.lt + icol] : p.inline_items[L * p.lt + icol];
-        for (int q = 0; q < n + 2; ++q, ++g, ++z) {
-          if (z == tz && L + 1 < p.nstack) {  // next stacked tile
-            ++L;
-            z = 0;
-            it = items ? items[L * p.lt + icol] : p.inline_items[L * p.lt + icol];
+        for (int q = 0; q < n + 2; ++q, ++g) {
+          if (q) {
+            int L2;
+            locate(rev ? g0 + n - q : g0 - 1 + q, L2, z);
+            if (L2 != L) {  // next stacked tile
+              L = L2;
+              it = items ? items[L * p.lt + icol] : p.inline_items[L * p.lt + icol];
+            }
           }
           const int st = (int)(g % S);
           mbar_wait(&empty[st], ((g / S) & 1u) ^ 1u);
@@ -258,9 +289,12 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
 
   for (int s = 0; s < nsteps; ++s) {
   const bool odd = s & 1;
+  const bool rev = p.snake && odd;
   const TileItem* items = odd ? p.items_odd : p.items;
   auto fexp = [&](int f) { return odd ? p.fexp_odd[f] : p.fexp[f]; };
-  Runs W(p);
+  Runs W(p, rev);
+  int64_t left = W.total;  // planes of this step still to store (march order)
+  const int64_t dz = rev ? -1 : 1;
   int64_t col;
   int g0, n;
   while (W.next(col, g0, n)) {
@@ -279,8 +313,9 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
         zc[j] = *reinterpret_cast<const double2*>(s1 + j * C::RPP * TX * 8);
       }
     }
-    release_g(seq);  // plane g0-1 is in registers now
-    int L = g0 / tz, z = g0 - L * tz;
+    release_g(seq);  // plane g0-1 (g0+n when rev) is in registers now
+    const int gfirst = rev ? g0 + n - 1 : g0;
+    int L = gfirst / tz, z = gfirst - L * tz;
     int tile = 0;
     double* op = nullptr;  // output cell pair of row yb, plane z
     double* fx = nullptr;  // x-face export of row yb, plane z (edge threads)
@@ -292,9 +327,9 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
     };
     enter_tile();
     for (int i = 0; i < n; ++i) {
-      if (z == tz) {  // next stacked tile (cold)
-        ++L;
-        z = 0;
+      if (z == tz || z < 0) {  // next stacked tile in march order (cold)
+        L += (int)dz;
+        z = rev ? tz - 1 : 0;
         enter_tile();
       }
       wait_g(seq + i + 2);
@@ -317,10 +352,12 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
         const double2 c = zc[j];
         v[j].x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm[j].x, zp.x, alpha);
         v[j].y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm[j].y, zp.y, alpha);
-        stg2_stream(op + (size_t)j * C::RPP * TX, v[j]);
+        if (left > p.keep_tail) stg2_stream(op + (size_t)j * C::RPP * TX, v[j]);
+        else st2_hint(op + (size_t)j * C::RPP * TX, v[j], keep);  // read first by the next (reversed) step
         zm[j] = c;
         zc[j] = zp;
       }
+      --left;
       release_g(seq + i + 1);  // plane z no longer read (its centre is in registers)
       // Epilogue: export the new boundary layers (the neighbours' ghost
       // sources for the next step). x: the two edge lanes of every
@@ -366,9 +403,9 @@ __global__ void __launch_bounds__(Fixed<TX, BY, S>::NT + 32)
           for (int j = 0; j < C::NR; ++j) *reinterpret_cast<double2*>(q + (size_t)j * C::RPP * TX) = v[j];
         }
       }
-      op += plane;
-      fx += (size_t)ty * D;
-      ++z;
+      op += dz * (int64_t)plane;
+      fx += dz * (int64_t)ty * D;
+      z += (int)dz;
     }
     release_g(seq + n + 1);  // plane g0+n (last z+1 neighbour)
     seq += (uint32_t)(n + 2);

@@ -95,6 +95,12 @@ struct HeatParams {
   // launches, so the counter is never reset). Requires all CTAs co-resident
   // (cooperative launch).
   int32_t nsteps;
+  // Snake order (persistent launches): odd steps run every CTA's runs in
+  // reverse, planes descending, so a step starts on the planes the CTA wrote
+  // last in the previous step; the last keep_tail planes of a CTA's step are
+  // stored with evict_last instead of streaming, so those reads are L2 hits.
+  // (z+1 and z-1 swap roles in the march; their sum is commutative: same bits.)
+  int32_t snake, keep_tail;
   int32_t ntx, nty;
   uint32_t epoch;
   unsigned long long* prog;
