@@ -1,7 +1,7 @@
 """Small runs of every schedule for compute-sanitizer (memcheck / racecheck /
 synccheck / initcheck): resident heat (layered + whole-domain phases),
 streaming heat with a tiny budget, Dirichlet, sincos, the generic kernel, the
-persistent multi-step launch (direct ghosts, grid counter) and
+persistent multi-step launch (direct ghosts, grid counter, snake order; banded tiles in round-robin order) and
 the stream-through schedule and the in-process multi-rank transport."""
 import os
 import sys
@@ -55,6 +55,9 @@ with T.Domain((64, 64, 256), (32, 32, 32), sched="stream", device_budget_bytes=b
     d.load(uo); d.run(T.heat7(), 5, 3); d.store()
 with T.Domain((128, 64, 64), (64, 64, 16), ghost=2, two_step=1) as d:   # heat7x2r (band 32)
     d.load(synth.uniform_grid(128, 64, 64, 11)); d.run(T.heat7(), 4, 2); d.store()
+ub = synth.uniform_grid(512, 512, 16, 12)                 # banded tiles: round-robin columns,
+with T.Domain((512, 512, 16), (32, 64, 8)) as d:          # snake-ordered persistent launch
+    d.load(ub); d.run(T.heat7(), 1, 2); d.sync(); d.run(T.heat7(), 4, 2); d.store()
 g = T.LocalGroup(2)
 def rank(r):
     with T.Domain((64, 32, 64), (32, 16, 16), nranks=2, rank=r, local_group=g) as d:
