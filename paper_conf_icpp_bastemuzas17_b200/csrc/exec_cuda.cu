@@ -197,6 +197,11 @@ struct CudaExec final : Exec {
     // persistent grid: one wave of CTAs, >= 4 planes each
     const int64_t planes = (int64_t)n * p.nbands * p.tz;
     int64_t grid = (int64_t)sms * heat_occ;
+    static const int64_t grid_cap = [] {  // experiment knob: cap the persistent grid
+      const char* e = std::getenv("TILES_HEAT_GRID");
+      return e ? (int64_t)std::atoll(e) : (int64_t)0;
+    }();
+    if (grid_cap > 0) grid = std::min(grid, grid_cap);
     grid = std::max<int64_t>(1, std::min<int64_t>(grid, (planes + 3) / 4));
     // banded tiles: adjacent bands side by side in time (their shared halo
     // rows from L2); TILES_HEAT_RR=0 keeps contiguous plane ranges
