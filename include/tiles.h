@@ -114,8 +114,12 @@ typedef struct {
                                    Fig. 1/5); copies are staged by the driver
                                    and do not overlap. 0 (default): pinned. */
   int32_t stream_through;       /* HEAT7 run starting from a fresh upload
-                                   (periodic, single rank, T <= tile_dims[2],
-                                   scratch fits): per unit of planes (a slice
+                                   (periodic, T <= tile_dims[2], scratch fits;
+                                   single rank, or z-slab ranks over the peer
+                                   transport, whose windows then also hold two
+                                   tile layers that carry the T planes of
+                                   initial data beyond each slab end, once per
+                                   run — DESIGN.md §6): per unit of planes (a slice
                                    of a z-layer, >= T planes) trapezoid: T
                                    sweeps over the unit + T halo planes, D2H
                                    of the exact core, so H2D, compute and D2H of
@@ -327,8 +331,9 @@ const char* tile_last_error(void);
 tile_status tile_nccl_unique_id(void* out128);
 
 /* Peer transport (tile_options.peer_transport = 1 or 2). tile_peer_handle writes
- * the 64-byte CUDA IPC handle of this rank's halo window (receive buffers
- * and exchange counters) to out64. tile_peer_connect takes every rank's
+ * the 64-byte CUDA IPC handle of this rank's halo window (receive buffers,
+ * exchange counters and, for periodic slabs whose two tile layers fit 1 GiB,
+ * the stream-through halo layers) to out64. tile_peer_connect takes every rank's
  * handle, `nranks` blobs of 64 bytes in rank order (the caller all-gathers
  * them, e.g. with torch.distributed), and maps the z-neighbours' windows;
  * it must precede the first tile_run. ESTATE if the domain has no window
