@@ -695,7 +695,9 @@ def run_c5_leg(args):
             n = int(t.item())
     nzl = n // 8 if ws == 1 else n // ws
     gdims = (n, n, nzl * ws)
-    td = (256, 256, 64)
+    # 64^3 tiles (the C2 kernel plan, one band per tile): 372.9 vs 338.3 Gcell/s
+    # with 256^2 x 64 (16-row bands re-read halo rows), profiles/r01/bench_c5_tiles.json
+    td = tuple(int(v) for v in args.tile.split(",")) if args.tile else (64, 64, 64)
     T = args.T if args.T is not None else 10
     ns = args.nstreams or 4
     cells = n * n * nzl
@@ -762,7 +764,7 @@ def run_c5_leg(args):
                 "gpu_launches": st["n_kernels"],
                 "roofline": {"bound": "hbm", "achieved": 16 * per_launch / (avg / 1e3) / 1e9, "peak": peak,
                              "unit": "GB/s", "frac": 16 * per_launch / (avg / 1e3) / 1e9 / peak, "traffic": None,
-                             "kernel": "heat7_fixed<256,16>", "peak_source": src},
+                             "kernel": f"heat7_fixed (tiles {td[0]}x{td[1]}x{td[2]})", "peak_source": src},
                 "halo_bytes_per_step": st["bytes_halo"] // max(1, args.steps), "clocks": clk.summary()}
         print(json.dumps(line), flush=True)
     if ws > 1:
@@ -784,6 +786,7 @@ def main():
     ap.add_argument("--n", type=int, default=None, help="c3/c4: grid edge")
     ap.add_argument("--budget-gb", type=float, default=None, help="c3: device budget cap")
     ap.add_argument("--K", type=int, default=32, help="c4: kernel_iteration (reading R12)")
+    ap.add_argument("--tile", default=None, help="c5: tile dims tx,ty,tz (default 64,64,64)")
     ap.add_argument("--sweep", default=None, help="c4: comma list of nstreams")
     ap.add_argument("--ghost", type=int, default=1,
                     help="c2/c3: ghost width; 2 = two Jacobi steps per pass (temporal blocking)")
