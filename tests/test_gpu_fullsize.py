@@ -155,10 +155,11 @@ def test_c4_sincos_full_size_sampled():
 
 def test_c5_per_gpu_slab_full_size():
     """C5 per-GPU slab of the G = 8 decomposition of 4096^3 (4096 x 4096 x 512,
-    68.7 GB, z-periodic alone), 256^2 x 64 tiles, 4 streams: bench.py
-    --config c5's sequence (one step after the upload, then T = 10 resident)."""
+    68.7 GB, z-periodic alone), 64^3 tiles (32768 of them), 4 streams:
+    bench.py --config c5's sequence (one step after the upload, then T = 10
+    resident in one persistent launch)."""
     n, nzl = 4096, 512
-    gdims, td = (n, n, nzl), (256, 256, 64)
+    gdims, td = (n, n, nzl), (64, 64, 64)
     _need_host(n * n * nzl * 8)
     with T.Domain(gdims, td, ghost=1) as d:
         _fill(d, gdims, td, 42)

@@ -402,3 +402,13 @@ def test_stream_through_bit_exact(dims, td, T):
     assert np.array_equal(out1, oracle.heat_c(u0, ALPHA, T))
     assert np.array_equal(out2, oracle.heat_c(u0, ALPHA, T + 3))
     assert st["bytes_h2d"] == nx * ny * nz * 8 and st["bytes_d2h"] == nx * ny * nz * 8
+
+
+@pytest.mark.parametrize("td,runs", [((32, 64, 8), [1, 4]), ((64, 32, 4), [2, 5])])
+def test_banded_round_robin_snake_bit_exact(td, runs):
+    """Banded tiles (ty > band) with enough columns for the round-robin
+    column order (HeatParams::rr_rounds >= 1 at 148 CTAs), then a persistent
+    multi-step launch in snake order (odd steps reversed): bit-exact."""
+    dims = (512, 512, 16)
+    out, ref, _, _ = _heat(dims, td, sum(runs), runs=runs)
+    assert np.array_equal(out, ref), np.abs(out - ref).max()
