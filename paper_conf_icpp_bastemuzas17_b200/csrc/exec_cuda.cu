@@ -210,6 +210,17 @@ struct CudaExec final : Exec {
       return e ? std::atoi(e) : 1;
     }();
     p.rr_rounds = rr_on && p.nbands > 1 ? (int32_t)((int64_t)p.lt * p.nbands / grid) : 0;
+    {  // z-chunked round-robin items (TILES_HEAT_ZCHUNK planes; experiment)
+      static const int zc = [] {
+        const char* e = std::getenv("TILES_HEAT_ZCHUNK");
+        return e ? std::atoi(e) : 0;
+      }();
+      const int64_t NZ = (int64_t)nstack * p.tz;
+      if (zc > 0 && NZ % zc == 0) {
+        p.zchunk = zc;
+        p.rr_rounds = (int32_t)((int64_t)p.lt * p.nbands * (NZ / zc) / grid);
+      }
+    }
     p.nsteps = 1;
     if (nsteps > 1) {  // one persistent launch for all steps (CTA progress counters)
       const int b1 = direct_bit ^ 1;

@@ -100,49 +100,62 @@ struct PlaneRange {
 // round-robin whole columns first (HeatParams::rr_rounds), then a contiguous
 // share of the remaining columns' planes.
 struct Runs {
-  int64_t c, cend, pp, pe, total;
-  int NZ;
+  // items: (z chunk of ZC planes, column), chunk-major, ZC = HeatParams::zchunk
+  // (0: the whole column depth NZ, one item per column)
+  int64_t c, cend, pp, pe, total, ncols;
+  int NZ, ZC;
   bool rev;  // snake order: the same runs in reverse, each run's planes descending
   __device__ Runs(const HeatParams& p, bool reverse) {
     NZ = p.nstack * p.tz;
+    ZC = p.zchunk > 0 ? p.zchunk : NZ;
     rev = reverse;
-    const int64_t ncols = (int64_t)p.lt * p.nbands;
+    ncols = (int64_t)p.lt * p.nbands;
+    const int64_t nitems = ncols * (NZ / ZC);
     cend = (int64_t)p.rr_rounds * gridDim.x;
-    const int64_t P = (ncols - cend) * NZ;
-    pp = cend * NZ + P * blockIdx.x / gridDim.x;
-    pe = cend * NZ + P * (blockIdx.x + 1) / gridDim.x;
+    const int64_t P = (nitems - cend) * ZC;
+    pp = cend * ZC + P * blockIdx.x / gridDim.x;
+    pe = cend * ZC + P * (blockIdx.x + 1) / gridDim.x;
     const int64_t mine = cend > (int64_t)blockIdx.x ? (cend - 1 - blockIdx.x) / gridDim.x + 1 : 0;
-    total = mine * NZ + (pe - pp);
+    total = mine * ZC + (pe - pp);
     c = !rev ? (int64_t)blockIdx.x : mine ? (int64_t)blockIdx.x + (mine - 1) * gridDim.x : -1;
   }
+  __device__ __forceinline__ void item(int64_t it, int64_t& col, int& gbase) const {
+    const int64_t j = it / ncols;
+    col = it - j * ncols;
+    gbase = (int)(j * ZC);
+  }
   __device__ __forceinline__ bool next(int64_t& col, int& g0, int& n) {
+    int gb;
     if (rev) {
       if (pe > pp) {
-        col = (pe - 1) / NZ;
-        const int64_t start = pp > col * NZ ? pp : col * NZ;
-        g0 = (int)(start - col * NZ);
+        const int64_t it = (pe - 1) / ZC;
+        const int64_t start = pp > it * ZC ? pp : it * ZC;
+        item(it, col, gb);
+        g0 = gb + (int)(start - it * ZC);
         n = (int)(pe - start);
         pe = start;
         return true;
       }
       if (c < (int64_t)blockIdx.x) return false;
-      col = c;
-      g0 = 0;
-      n = NZ;
+      item(c, col, gb);
+      g0 = gb;
+      n = ZC;
       c -= gridDim.x;
       return true;
     }
     if (c < cend) {
-      col = c;
-      g0 = 0;
-      n = NZ;
+      item(c, col, gb);
+      g0 = gb;
+      n = ZC;
       c += gridDim.x;
       return true;
     }
     if (pp >= pe) return false;
-    col = pp / NZ;
-    g0 = (int)(pp - col * NZ);
-    n = (int)(pe - pp < (int64_t)(NZ - g0) ? pe - pp : NZ - g0);
+    const int64_t it = pp / ZC;
+    const int off = (int)(pp - it * ZC);
+    item(it, col, gb);
+    g0 = gb + off;
+    n = (int)(pe - pp < (int64_t)(ZC - off) ? pe - pp : ZC - off);
     pp += n;
     return true;
   }

@@ -71,6 +71,10 @@ struct HeatParams {
   // neighbour CTA just staged — L2 hits instead of DRAM re-reads); the rest
   // is split into contiguous plane ranges. rr_rounds = 0: all contiguous.
   int32_t rr_rounds;
+  // zchunk > 0: work items are z chunks of zchunk planes of a column (chunk-
+  // major), dealt round-robin for rr_rounds rounds, so all CTAs march the same
+  // planes of neighbouring columns at the same time; 0: whole columns.
+  int32_t zchunk;
   // Exports: x faces always; y faces iff exp_y; the z- face of tile k iff
   // k < exp_zlo_below, the z+ face iff k >= exp_zhi_from (direct runs export
   // only what a face reader still needs: the slab-end layers' z faces for the
