@@ -148,6 +148,27 @@ def test_slab_stream_through_replay_matches_global_oracle(G, T_, tz, ns):
         assert np.array_equal(out, oracle.heat_c(u, ALPHA, total)), (run, np.abs(out - oracle.heat_c(u, ALPHA, total)).max())
 
 
+@pytest.mark.parametrize("bc,kw,expect", [("periodic", {"peer_transport": 2}, True),
+                                           ("periodic", {"peer_transport": 2, "stream_through": -1}, False),
+                                           ("periodic", {"peer_transport": 1}, True),
+                                           ("dirichlet", {"peer_transport": 2}, False),
+                                           ("periodic", {}, False)])
+def test_multi_rank_stream_through_eligibility(bc, kw, expect):
+    """Multi-rank stream-through needs the peer transport (its windows carry
+    the halo layers), a periodic slab and stream_through >= 0; everything
+    else keeps the batched schedule (no st_halo ops in the trace)."""
+    G, tz = 2, 8
+    dims, td = (64, 32, 8 * tz * G), (32, 16, tz)
+    u, ext, _ = _global(dims, bc)
+    d = _rank_domain(dims, td, G, 0, bc, ext, u, stream_through=kw.pop("stream_through", 1), **kw)
+    d.clear_trace()
+    d.run(T.heat7(ALPHA), 4, 2)
+    d.sync()
+    tr = d.trace()
+    assert any(op[0] == "st_halo" for op in tr) == expect
+    assert any(op[0] == "sweep" for op in tr) == expect
+
+
 def test_slab_geometry_and_face_kinds():
     d = T.Domain((16, 16, 32), (8, 8, 4), nranks=4, rank=1, dry_run=True)
     info = d.info
