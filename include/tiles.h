@@ -61,13 +61,19 @@ typedef enum {
   TILE_KERNEL_HEAT7 = 1,
   /* compute-intensive kernel, listing P:L219-L224 §VI.B: per cell,
    * inner_iters times: s=sin(x); c=cos(x); x=x+sqrt(s*s+c*c) */
-  TILE_KERNEL_SINCOS = 2
+  TILE_KERNEL_SINCOS = 2,
+  TILE_KERNEL_USER = 3   /* user pointwise function (tile_user_fn_create) */
 } tile_kernel_kind;
+
+typedef struct tile_user_fn tile_user_fn; /* opaque, a compiled user function */
 
 typedef struct {
   tile_kernel_kind kind;
   double alpha;        /* HEAT7: dt/dx^2, must be in (0, 1/6] (stability) */
-  int32_t inner_iters; /* SINCOS: kernel_iteration of P:L220 (>= 0) */
+  int32_t inner_iters; /* SINCOS: kernel_iteration of P:L220 (>= 0); USER:
+                          applications of the function per cell per step */
+  const tile_user_fn* user; /* USER: the function (borrowed for the run;
+                          ignored for the other kinds) */
 } tile_kernel;
 
 /* Schedules. AUTO picks RESIDENT when every tile fits in the
@@ -325,6 +331,24 @@ tile_status tile_free(tile_domain* dom);
 
 /* Thread-local description of the last error (never NULL). */
 const char* tile_last_error(void);
+
+/* User pointwise kernels (general kernels; the paper's
+ * compute(tile) runs user code over a region). `source` is CUDA C
+ * defining
+ *     __device__ double <name>(double u, long long gidx)
+ * (u: the cell's current value; gidx = (z*ny + y)*nx + x, the cell's GLOBAL
+ * linear index). NVRTC compiles it for sm_100a with --fmad=false inside a
+ * wrapper that applies it inner_iters times per step to every cell, in place;
+ * tile_run with {TILE_KERNEL_USER, 0, inner_iters, fn} then schedules tiles
+ * like the compute-intensive kernel (resident, streamed out of core, fused
+ * or step-major per tile_options.fuse_pointwise_steps; no ghosts).
+ * Errors: EINVAL for a null source, a name that is not a C identifier, or a
+ * compile error (the NVRTC log is in tile_last_error); ENOSYS if libnvrtc
+ * cannot be loaded. The compiled cubin is loaded lazily on each device that
+ * runs it. tile_user_fn_free: after the last run using the function has been
+ * synchronised (tile_sync / tile_store / tile_free); NULL is a no-op. */
+tile_status tile_user_fn_create(const char* source, const char* name, tile_user_fn** out);
+tile_status tile_user_fn_free(tile_user_fn* fn);
 
 /* Fill out[128] with a fresh ncclUniqueId (call on rank 0, then broadcast).
  * TILE_ENOSYS if built without NCCL. */

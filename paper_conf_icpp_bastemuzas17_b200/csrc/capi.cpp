@@ -12,6 +12,9 @@ using tiles::Status;
 struct tile_domain {
   Domain* d;
 };
+struct tile_user_fn {
+  tiles::UserFn* f;
+};
 
 namespace {
 thread_local std::string g_err = "no error";
@@ -79,7 +82,10 @@ tile_status tile_run(tile_domain* h, const tile_kernel* k, int32_t steps, int32_
   CHECK_DOM(h);
   if (!k) return fail(TILE_EINVAL, "null kernel");
   auto t0 = std::chrono::steady_clock::now();
+  // USER kernels: the function is read while this call enqueues the launches
+  h->d->user_fn = k->kind == TILE_KERNEL_USER && k->user ? k->user->f : nullptr;
   Status s = tiles::domain_run(*h->d, *k, steps, nstreams);
+  h->d->user_fn = nullptr;
   h->d->run_t0 = std::chrono::duration<double, std::milli>(t0.time_since_epoch()).count();
   return finish(h, s);
 }
@@ -221,6 +227,23 @@ tile_status tile_local_group_create(int32_t nranks, void** group) {
 
 tile_status tile_local_group_free(void* group) {
   tiles::local_group_free(group);
+  return TILE_OK;
+}
+
+tile_status tile_user_fn_create(const char* source, const char* name, tile_user_fn** out) {
+  if (!out) return fail(TILE_EINVAL, "null out");
+  *out = nullptr;
+  tiles::UserFn* f = nullptr;
+  Status s = tiles::userfn_create(source, name, &f);
+  if (s.bad()) return finish(nullptr, s);
+  *out = new tile_user_fn{f};
+  return TILE_OK;
+}
+
+tile_status tile_user_fn_free(tile_user_fn* fn) {
+  if (!fn) return TILE_OK;
+  tiles::userfn_free(fn->f);
+  delete fn;
   return TILE_OK;
 }
 

@@ -399,6 +399,20 @@ struct CudaExec final : Exec {
   }
   Status sincos(Domain& d, int64_t t, int slot, int64_t iters, int st) override {
     if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
+    if (d.user_fn) {  // TILE_KERNEL_USER: the caller's compiled pointwise function
+      int64_t ix, iy, iz;
+      d.G.tile_coords(t, &ix, &iy, &iz);
+      const int64_t td[2] = {d.G.t[0], d.G.t[1]};
+      const int64_t org[3] = {ix * d.G.t[0], iy * d.G.t[1], d.G.zoff + iz * d.G.t[2]};
+      const int64_t gd[2] = {d.G.g[0], d.G.g[1]};
+      Status r = timed(d, st, [&] {
+        Status u = userfn_launch(d.user_fn, d.slot_ptr(slot), d.G.tile_elems, td, org, gd, iters, S(st));
+        return u.bad() ? cudaErrorLaunchFailure : cudaSuccess;
+      });
+      if (r.bad()) return r;
+      d.stats.n_kernels++;
+      return Status::ok();
+    }
     SincosParams p{};
     p.tile_elems = d.G.tile_elems;
     p.nitems = 1;

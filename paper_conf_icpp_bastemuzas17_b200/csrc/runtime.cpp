@@ -1419,8 +1419,9 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
   if (k.kind == TILE_KERNEL_HEAT7) {
     if (!(k.alpha > 0.0 && k.alpha <= 1.0 / 6.0))
       return make_err(TILE_EINVAL, "HEAT7 alpha must be in (0, 1/6]");
-  } else if (k.kind == TILE_KERNEL_SINCOS) {
-    if (k.inner_iters < 0) return make_err(TILE_EINVAL, "SINCOS inner_iters must be >= 0");
+  } else if (k.kind == TILE_KERNEL_SINCOS || k.kind == TILE_KERNEL_USER) {
+    if (k.inner_iters < 0) return make_err(TILE_EINVAL, "inner_iters must be >= 0");
+    if (k.kind == TILE_KERNEL_USER && !d.user_fn) return make_err(TILE_EINVAL, "USER kernel without a function");
   } else {
     return make_err(TILE_EINVAL, "unknown kernel kind");
   }

@@ -1,0 +1,191 @@
+// userfn.cpp — user pointwise kernels ("general
+// kernels"; the paper's compute(tile) runs user code over a region,
+// P:L126-L147). The caller supplies CUDA C source defining
+//     __device__ double <name>(double u, long long gidx)
+// which NVRTC compiles for sm_100a together with a grid-stride wrapper that
+// applies it `iters` times to every cell of a tile in place; tile_run with
+// TILE_KERNEL_USER then moves tiles through the same residency / streaming
+// schedules as the compute-intensive kernel (pointwise, no ghosts). NVRTC is
+// dlopen'ed (ENOSYS without it); the cubin is loaded per device with the
+// driver API fetched through cudaGetDriverEntryPoint (the primary context
+// cudart uses), so no -lcuda / -lnvrtc link dependency exists.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <cctype>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "runtime.hpp"
+
+namespace tiles {
+namespace {
+
+// NVRTC entry points (nvrtc.h signatures, resolved with dlsym)
+using nvrtcResult_t = int;
+using nvrtcProgram_t = void*;
+struct Nvrtc {
+  nvrtcResult_t (*create)(nvrtcProgram_t*, const char*, const char*, int, const char* const*, const char* const*);
+  nvrtcResult_t (*compile)(nvrtcProgram_t, int, const char* const*);
+  nvrtcResult_t (*log_size)(nvrtcProgram_t, size_t*);
+  nvrtcResult_t (*log)(nvrtcProgram_t, char*);
+  nvrtcResult_t (*cubin_size)(nvrtcProgram_t, size_t*);
+  nvrtcResult_t (*cubin)(nvrtcProgram_t, char*);
+  nvrtcResult_t (*destroy)(nvrtcProgram_t*);
+  bool ok = false;
+};
+
+Nvrtc& nvrtc() {
+  static Nvrtc n;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* h = nullptr;
+    for (const char* lib : {"libnvrtc.so.12", "libnvrtc.so", "/usr/local/cuda/lib64/libnvrtc.so.12"})
+      if ((h = dlopen(lib, RTLD_NOW | RTLD_LOCAL))) break;
+    if (!h) return;
+    auto sym = [&](const char* s) { return dlsym(h, s); };
+    n.create = reinterpret_cast<decltype(n.create)>(sym("nvrtcCreateProgram"));
+    n.compile = reinterpret_cast<decltype(n.compile)>(sym("nvrtcCompileProgram"));
+    n.log_size = reinterpret_cast<decltype(n.log_size)>(sym("nvrtcGetProgramLogSize"));
+    n.log = reinterpret_cast<decltype(n.log)>(sym("nvrtcGetProgramLog"));
+    n.cubin_size = reinterpret_cast<decltype(n.cubin_size)>(sym("nvrtcGetCUBINSize"));
+    n.cubin = reinterpret_cast<decltype(n.cubin)>(sym("nvrtcGetCUBIN"));
+    n.destroy = reinterpret_cast<decltype(n.destroy)>(sym("nvrtcDestroyProgram"));
+    n.ok = n.create && n.compile && n.log_size && n.log && n.cubin_size && n.cubin && n.destroy;
+  });
+  return n;
+}
+
+// driver API through the runtime's entry-point query
+struct Drv {
+  CUresult (*load)(CUmodule*, const void*) = nullptr;
+  CUresult (*get)(CUfunction*, CUmodule, const char*) = nullptr;
+  CUresult (*launch)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
+                     CUstream, void**, void**) = nullptr;
+  CUresult (*unload)(CUmodule) = nullptr;
+  bool ok = false;
+};
+
+Drv& drv() {
+  static Drv d;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    cudaDriverEntryPointQueryResult q{};
+    void* p = nullptr;
+    if (cudaGetDriverEntryPoint("cuModuleLoadData", &p, cudaEnableDefault, &q) == cudaSuccess && p)
+      d.load = reinterpret_cast<decltype(d.load)>(p);
+    p = nullptr;
+    if (cudaGetDriverEntryPoint("cuModuleGetFunction", &p, cudaEnableDefault, &q) == cudaSuccess && p)
+      d.get = reinterpret_cast<decltype(d.get)>(p);
+    p = nullptr;
+    if (cudaGetDriverEntryPoint("cuLaunchKernel", &p, cudaEnableDefault, &q) == cudaSuccess && p)
+      d.launch = reinterpret_cast<decltype(d.launch)>(p);
+    p = nullptr;
+    if (cudaGetDriverEntryPoint("cuModuleUnload", &p, cudaEnableDefault, &q) == cudaSuccess && p)
+      d.unload = reinterpret_cast<decltype(d.unload)>(p);
+    d.ok = d.load && d.get && d.launch && d.unload;
+  });
+  return d;
+}
+
+bool valid_identifier(const char* s) {
+  if (!s || !*s || !(std::isalpha((unsigned char)s[0]) || s[0] == '_')) return false;
+  for (const char* c = s; *c; ++c)
+    if (!(std::isalnum((unsigned char)*c) || *c == '_')) return false;
+  return std::strlen(s) < 128;
+}
+
+}  // namespace
+
+struct UserFn {
+  std::string name;
+  std::vector<char> cubin;
+  std::mutex m;
+  std::vector<std::pair<int, CUmodule>> modules;  // per device
+  std::vector<std::pair<int, CUfunction>> fns;
+};
+
+Status userfn_create(const char* source, const char* name, UserFn** out) {
+  if (!source || !out) return make_err(TILE_EINVAL, "null argument");
+  if (!valid_identifier(name)) return make_err(TILE_EINVAL, "user function name must be a C identifier");
+  Nvrtc& n = nvrtc();
+  if (!n.ok) return make_err(TILE_ENOSYS, "libnvrtc not available");
+  const std::string src = std::string(source) +
+                          "\nextern \"C\" __global__ void tile_user_apply(double* __restrict__ u, long long n,"
+                          " long long tx, long long ty, long long x0, long long y0, long long z0,"
+                          " long long nx, long long ny, long long iters) {\n"
+                          "  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;"
+                          " i += (long long)gridDim.x * blockDim.x) {\n"
+                          "    const long long lx = i % tx, r = i / tx, ly = r % ty, lz = r / ty;\n"
+                          "    const long long g = ((z0 + lz) * ny + (y0 + ly)) * nx + (x0 + lx);\n"
+                          "    double v = u[i];\n"
+                          "    for (long long k = 0; k < iters; ++k) v = " + std::string(name) + "(v, g);\n"
+                          "    u[i] = v;\n  }\n}\n";
+  nvrtcProgram_t prog = nullptr;
+  if (n.create(&prog, src.c_str(), "tile_user.cu", 0, nullptr, nullptr) != 0)
+    return make_err(TILE_EINVAL, "nvrtcCreateProgram failed");
+  const char* opts[] = {"--gpu-architecture=sm_100a", "--std=c++17", "-default-device", "--fmad=false"};
+  const int rc = n.compile(prog, 4, opts);
+  size_t ls = 0;
+  n.log_size(prog, &ls);
+  std::string log(ls, '\0');
+  if (ls) n.log(prog, &log[0]);
+  if (rc != 0) {
+    n.destroy(&prog);
+    return make_err(TILE_EINVAL, "user kernel does not compile: " + log);
+  }
+  size_t cs = 0;
+  n.cubin_size(prog, &cs);
+  auto* f = new UserFn;
+  f->name = name;
+  f->cubin.resize(cs);
+  n.cubin(prog, f->cubin.data());
+  n.destroy(&prog);
+  *out = f;
+  return Status::ok();
+}
+
+void userfn_free(UserFn* f) {
+  if (!f) return;
+  Drv& d = drv();
+  if (d.ok)
+    for (auto& m : f->modules) d.unload(m.second);
+  delete f;
+}
+
+Status userfn_launch(UserFn* f, double* data, int64_t n, const int64_t tdims[2], const int64_t org[3],
+                     const int64_t gdims[2], int64_t iters, void* stream) {
+  Drv& d = drv();
+  if (!d.ok) return make_err(TILE_ENOSYS, "driver entry points for module loading unavailable");
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return make_err(TILE_ECUDA, "cudaGetDevice");
+  CUfunction fn = nullptr;
+  {
+    std::lock_guard<std::mutex> lk(f->m);
+    for (auto& p : f->fns)
+      if (p.first == dev) fn = p.second;
+    if (!fn) {
+      CUmodule mod = nullptr;
+      if (d.load(&mod, f->cubin.data()) != CUDA_SUCCESS) return make_err(TILE_ECUDA, "cuModuleLoadData (user kernel)");
+      if (d.get(&fn, mod, "tile_user_apply") != CUDA_SUCCESS) return make_err(TILE_ECUDA, "cuModuleGetFunction");
+      f->modules.push_back({dev, mod});
+      f->fns.push_back({dev, fn});
+    }
+  }
+  long long a_n = n, tx = tdims[0], ty = tdims[1], x0 = org[0], y0 = org[1], z0 = org[2], nx = gdims[0],
+            ny = gdims[1], it = iters;
+  void* args[] = {&data, &a_n, &tx, &ty, &x0, &y0, &z0, &nx, &ny, &it};
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const long long blocks = std::min<long long>((n + 255) / 256, (long long)sms * 8);
+  if (d.launch(fn, (unsigned)std::max<long long>(1, blocks), 1, 1, 256, 1, 1, 0, static_cast<CUstream>(stream),
+               args, nullptr) != CUDA_SUCCESS)
+    return make_err(TILE_ECUDA, "cuLaunchKernel (user kernel)");
+  return Status::ok();
+}
+
+}  // namespace tiles

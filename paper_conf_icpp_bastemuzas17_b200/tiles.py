@@ -28,7 +28,7 @@ TILE_OK, TILE_EINVAL, TILE_ENOMEM_HOST, TILE_ENOMEM_DEVICE, TILE_ECUDA, TILE_ENC
 STATUS_NAMES = {0: "OK", 1: "EINVAL", 2: "ENOMEM_HOST", 3: "ENOMEM_DEVICE", 4: "ECUDA",
                 5: "ENCCL", 6: "ESTATE", 7: "ENOSYS"}
 TILE_BC_PERIODIC, TILE_BC_DIRICHLET = 0, 1
-TILE_KERNEL_HEAT7, TILE_KERNEL_SINCOS = 1, 2
+TILE_KERNEL_HEAT7, TILE_KERNEL_SINCOS, TILE_KERNEL_USER = 1, 2, 3
 TILE_SCHED_AUTO, TILE_SCHED_RESIDENT, TILE_SCHED_STREAM, TILE_SCHED_SYNC = 0, 1, 2, 3
 TILE_MEASURE_NORMAL, TILE_MEASURE_XFER_ONLY, TILE_MEASURE_COMP_ONLY = 0, 1, 2
 OP_NAMES = {1: "h2d", 2: "d2h", 3: "kernel", 4: "record", 5: "wait", 6: "faces_h2d",
@@ -53,7 +53,8 @@ class TileOptions(ctypes.Structure):
 
 
 class TileKernel(ctypes.Structure):
-    _fields_ = [("kind", ctypes.c_int), ("alpha", ctypes.c_double), ("inner_iters", ctypes.c_int32)]
+    _fields_ = [("kind", ctypes.c_int), ("alpha", ctypes.c_double), ("inner_iters", ctypes.c_int32),
+                ("user", ctypes.c_void_p)]
 
 
 class TileStats(ctypes.Structure):
@@ -117,6 +118,8 @@ _sig = {
     "tile_local_group_create": ([ctypes.c_int32, ctypes.POINTER(_P)], ctypes.c_int),
     "tile_local_group_free": ([_P], ctypes.c_int),
     "tile_version": ([], ctypes.c_char_p),
+    "tile_user_fn_create": ([ctypes.c_char_p, ctypes.c_char_p, ctypes.POINTER(_P)], ctypes.c_int),
+    "tile_user_fn_free": ([_P], ctypes.c_int),
 }
 EXPORTED = tuple(_sig)
 for _name, (_args, _res) in _sig.items():
@@ -168,6 +171,35 @@ def heat7(alpha=0.125):
 def sincos(inner_iters=32):
     """Compute-intensive kernel descriptor."""
     return TileKernel(TILE_KERNEL_SINCOS, 0.0, inner_iters)
+
+
+class UserFn:
+    """A user pointwise function compiled by libtiles (tile_user_fn_create):
+    `source` defines ``__device__ double <name>(double u, long long gidx)``."""
+
+    def __init__(self, source, name):
+        h = ctypes.c_void_p()
+        _check(tile_user_fn_create(source.encode(), name.encode(), ctypes.byref(h)), "tile_user_fn_create")
+        self._h = h
+
+    def free(self):
+        if self._h is not None:
+            tile_user_fn_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def user(fn, inner_iters=1):
+    """Kernel descriptor applying UserFn `fn` inner_iters times per step."""
+    k = TileKernel(TILE_KERNEL_USER, 0.0, inner_iters)
+    k.user = fn._h.value
+    k._fn = fn  # keep the function alive as long as the descriptor
+    return k
 
 
 class Domain:
