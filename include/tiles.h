@@ -74,6 +74,12 @@ typedef struct {
                           applications of the function per cell per step */
   const tile_user_fn* user; /* USER: the function (borrowed for the run;
                           ignored for the other kinds) */
+  const int64_t* box;   /* USER, optional: 6 values {x0, y0, z0, x1, y1, z1},
+                          GLOBAL cell coordinates; the function is applied
+                          only to cells with x0 <= x < x1 (etc.) — the
+                          paper's ranged compute(tile, lo, hi), P:L126-L147;
+                          tiles outside the box launch nothing. NULL = every
+                          cell. EINVAL if x0 > x1 (etc.). */
 } tile_kernel;
 
 /* Schedules. AUTO picks RESIDENT when every tile fits in the

@@ -84,6 +84,17 @@ tile_status tile_run(tile_domain* h, const tile_kernel* k, int32_t steps, int32_
   auto t0 = std::chrono::steady_clock::now();
   // USER kernels: the function is read while this call enqueues the launches
   h->d->user_fn = k->kind == TILE_KERNEL_USER && k->user ? k->user->f : nullptr;
+  if (h->d->user_fn) {
+    const tiles::Geometry& G = h->d->G;
+    const int64_t all[6] = {0, 0, 0, G.g[0], G.g[1], G.g[2]};
+    const int64_t* b = k->box ? k->box : all;
+    for (int a = 0; a < 3; ++a)
+      if (b[a] > b[3 + a]) {
+        h->d->user_fn = nullptr;
+        return fail(TILE_EINVAL, "kernel box: lo > hi");
+      }
+    for (int i = 0; i < 6; ++i) h->d->user_box[i] = b[i];
+  }
   Status s = tiles::domain_run(*h->d, *k, steps, nstreams);
   h->d->user_fn = nullptr;
   h->d->run_t0 = std::chrono::duration<double, std::milli>(t0.time_since_epoch()).count();

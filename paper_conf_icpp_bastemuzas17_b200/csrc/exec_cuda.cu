@@ -405,8 +405,11 @@ struct CudaExec final : Exec {
       const int64_t td[2] = {d.G.t[0], d.G.t[1]};
       const int64_t org[3] = {ix * d.G.t[0], iy * d.G.t[1], d.G.zoff + iz * d.G.t[2]};
       const int64_t gd[2] = {d.G.g[0], d.G.g[1]};
+      const int64_t* b = d.user_box;
+      for (int a = 0; a < 3; ++a)  // ranged compute: a tile outside the box launches nothing
+        if (org[a] >= b[3 + a] || org[a] + d.G.t[a] <= b[a]) return Status::ok();
       Status r = timed(d, st, [&] {
-        Status u = userfn_launch(d.user_fn, d.slot_ptr(slot), d.G.tile_elems, td, org, gd, iters, S(st));
+        Status u = userfn_launch(d.user_fn, d.slot_ptr(slot), d.G.tile_elems, td, org, gd, iters, b, S(st));
         return u.bad() ? cudaErrorLaunchFailure : cudaSuccess;
       });
       if (r.bad()) return r;

@@ -260,6 +260,7 @@ struct Domain {
   uint64_t st_halo_bytes = 0;              // one layer (0: no multi-rank stream-through)
   uint32_t st_epoch = 0;                   // multi-rank stream-through runs so far
   struct UserFn* user_fn = nullptr;        // TILE_KERNEL_USER run in progress (borrowed)
+  int64_t user_box[6] = {0, 0, 0, 0, 0, 0}; // its global cell box [x0,y0,z0; x1,y1,z1)
 
   // kernel plan
   int band = 0, stages = 0, heat_grid = 0, sm_count = 148;
@@ -323,7 +324,7 @@ struct UserFn;  // userfn.cpp
 Status userfn_create(const char* source, const char* name, UserFn** out);
 void userfn_free(UserFn* f);
 Status userfn_launch(UserFn* f, double* data, int64_t n, const int64_t tdims[2], const int64_t org[3],
-                     const int64_t gdims[2], int64_t iters, void* stream);
+                     const int64_t gdims[2], int64_t iters, const int64_t box[6], void* stream);
 Status peer_setup(Domain& d, uint64_t halo_bytes, uint64_t st_bytes);
 Status peer_st_halo(Domain& d, int op, int side, int T, void* stream);
 Status peer_handle(const Domain& d, void* out64);

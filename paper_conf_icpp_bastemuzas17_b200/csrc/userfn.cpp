@@ -117,11 +117,14 @@ Status userfn_create(const char* source, const char* name, UserFn** out) {
   const std::string src = std::string(source) +
                           "\nextern \"C\" __global__ void tile_user_apply(double* __restrict__ u, long long n,"
                           " long long tx, long long ty, long long x0, long long y0, long long z0,"
-                          " long long nx, long long ny, long long iters) {\n"
+                          " long long nx, long long ny, long long iters, long long bx0, long long by0,"
+                          " long long bz0, long long bx1, long long by1, long long bz1) {\n"
                           "  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;"
                           " i += (long long)gridDim.x * blockDim.x) {\n"
                           "    const long long lx = i % tx, r = i / tx, ly = r % ty, lz = r / ty;\n"
-                          "    const long long g = ((z0 + lz) * ny + (y0 + ly)) * nx + (x0 + lx);\n"
+                          "    const long long X = x0 + lx, Y = y0 + ly, Z = z0 + lz;\n"
+                          "    if (X < bx0 || X >= bx1 || Y < by0 || Y >= by1 || Z < bz0 || Z >= bz1) continue;\n"
+                          "    const long long g = (Z * ny + Y) * nx + X;\n"
                           "    double v = u[i];\n"
                           "    for (long long k = 0; k < iters; ++k) v = " + std::string(name) + "(v, g);\n"
                           "    u[i] = v;\n  }\n}\n";
@@ -158,7 +161,7 @@ void userfn_free(UserFn* f) {
 }
 
 Status userfn_launch(UserFn* f, double* data, int64_t n, const int64_t tdims[2], const int64_t org[3],
-                     const int64_t gdims[2], int64_t iters, void* stream) {
+                     const int64_t gdims[2], int64_t iters, const int64_t box[6], void* stream) {
   Drv& d = drv();
   if (!d.ok) return make_err(TILE_ENOSYS, "driver entry points for module loading unavailable");
   int dev = 0;
@@ -178,7 +181,9 @@ Status userfn_launch(UserFn* f, double* data, int64_t n, const int64_t tdims[2],
   }
   long long a_n = n, tx = tdims[0], ty = tdims[1], x0 = org[0], y0 = org[1], z0 = org[2], nx = gdims[0],
             ny = gdims[1], it = iters;
-  void* args[] = {&data, &a_n, &tx, &ty, &x0, &y0, &z0, &nx, &ny, &it};
+  long long b[6];
+  for (int i = 0; i < 6; ++i) b[i] = box[i];
+  void* args[] = {&data, &a_n, &tx, &ty, &x0, &y0, &z0, &nx, &ny, &it, &b[0], &b[1], &b[2], &b[3], &b[4], &b[5]};
   int sms = 148;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const long long blocks = std::min<long long>((n + 255) / 256, (long long)sms * 8);

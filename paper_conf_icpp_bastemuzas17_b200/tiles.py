@@ -54,7 +54,7 @@ class TileOptions(ctypes.Structure):
 
 class TileKernel(ctypes.Structure):
     _fields_ = [("kind", ctypes.c_int), ("alpha", ctypes.c_double), ("inner_iters", ctypes.c_int32),
-                ("user", ctypes.c_void_p)]
+                ("user", ctypes.c_void_p), ("box", ctypes.POINTER(ctypes.c_int64))]
 
 
 class TileStats(ctypes.Structure):
@@ -194,11 +194,16 @@ class UserFn:
             pass
 
 
-def user(fn, inner_iters=1):
-    """Kernel descriptor applying UserFn `fn` inner_iters times per step."""
+def user(fn, inner_iters=1, box=None):
+    """Kernel descriptor applying UserFn `fn` inner_iters times per step;
+    box = ((x0, y0, z0), (x1, y1, z1)) restricts it to global cells
+    x0 <= x < x1 etc. (ranged compute)."""
     k = TileKernel(TILE_KERNEL_USER, 0.0, inner_iters)
     k.user = fn._h.value
     k._fn = fn  # keep the function alive as long as the descriptor
+    if box is not None:
+        k._box = (ctypes.c_int64 * 6)(*[int(v) for v in tuple(box[0]) + tuple(box[1])])
+        k.box = ctypes.cast(k._box, ctypes.POINTER(ctypes.c_int64))
     return k
 
 
