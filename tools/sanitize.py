@@ -1,7 +1,7 @@
 """Small runs of every schedule for compute-sanitizer (memcheck / racecheck /
 synccheck / initcheck): resident heat (layered + whole-domain phases),
 streaming heat with a tiny budget, Dirichlet, sincos, the generic kernel, the
-persistent multi-step launch (direct ghosts, grid counter, snake order; banded tiles in round-robin order) and
+persistent multi-step launch (direct ghosts, grid counter, snake order; banded tiles in round-robin order), a ranged NVRTC user kernel and
 the stream-through schedule and the in-process multi-rank transport."""
 import os
 import sys
@@ -58,6 +58,9 @@ with T.Domain((128, 64, 64), (64, 64, 16), ghost=2, two_step=1) as d:   # heat7x
 ub = synth.uniform_grid(512, 512, 16, 12)                 # banded tiles: round-robin columns,
 with T.Domain((512, 512, 16), (32, 64, 8)) as d:          # snake-ordered persistent launch
     d.load(ub); d.run(T.heat7(), 1, 2); d.sync(); d.run(T.heat7(), 4, 2); d.store()
+fu = T.UserFn("__device__ double aff(double u, long long g) { return 2.0 * u + 1.0; }", "aff")
+with T.Domain((64, 32, 32), (32, 16, 16)) as d:           # user pointwise kernel (NVRTC), ranged
+    d.load(u); d.run(T.user(fu, 2, box=((5, 3, 7), (40, 16, 32))), 2, 2); d.store()
 g = T.LocalGroup(2)
 def rank(r):
     with T.Domain((64, 32, 64), (32, 16, 16), nranks=2, rank=r, local_group=g) as d:
