@@ -62,7 +62,8 @@ typedef enum {
   /* compute-intensive kernel, listing P:L219-L224 §VI.B: per cell,
    * inner_iters times: s=sin(x); c=cos(x); x=x+sqrt(s*s+c*c) */
   TILE_KERNEL_SINCOS = 2,
-  TILE_KERNEL_USER = 3   /* user pointwise function (tile_user_fn_create) */
+  TILE_KERNEL_USER = 3,  /* user pointwise function (tile_user_fn_create) */
+  TILE_KERNEL_USER_STENCIL = 4 /* user 7-point stencil (tile_user_stencil_create) */
 } tile_kernel_kind;
 
 typedef struct tile_user_fn tile_user_fn; /* opaque, a compiled user function */
@@ -355,6 +356,18 @@ const char* tile_last_error(void);
  * synchronised (tile_sync / tile_store / tile_free); NULL is a no-op. */
 tile_status tile_user_fn_create(const char* source, const char* name, tile_user_fn** out);
 tile_status tile_user_fn_free(tile_user_fn* fn);
+/* User 7-point stencils (general kernels with ghost exchange): `source` defines
+ *     __device__ double <name>(double c, double xm, double xp, double ym,
+ *                              double yp, double zm, double zp)
+ * (the cell and its six neighbours at the current step, ghosts included).
+ * tile_run with {TILE_KERNEL_USER_STENCIL, 0, 0, fn} advances `steps` Jacobi
+ * steps of u' = f(...) through the tile machinery: ghosts from the neighbour
+ * tiles' exported faces (or Dirichlet fixed faces), each step exporting the new
+ * boundary layers, resident or streamed out of core (the heat kernel's
+ * specialised paths — direct ghosts, persistent and two-step launches,
+ * stream-through — stay HEAT7-only). Single rank, ghost = 1 (EINVAL
+ * otherwise). Free with tile_user_fn_free like a pointwise function. */
+tile_status tile_user_stencil_create(const char* source, const char* name, tile_user_fn** out);
 
 /* Fill out[128] with a fresh ncclUniqueId (call on rank 0, then broadcast).
  * TILE_ENOSYS if built without NCCL. */

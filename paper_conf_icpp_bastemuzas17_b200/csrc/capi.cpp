@@ -83,8 +83,13 @@ tile_status tile_run(tile_domain* h, const tile_kernel* k, int32_t steps, int32_
   if (!k) return fail(TILE_EINVAL, "null kernel");
   auto t0 = std::chrono::steady_clock::now();
   // USER kernels: the function is read while this call enqueues the launches
-  h->d->user_fn = k->kind == TILE_KERNEL_USER && k->user ? k->user->f : nullptr;
-  if (h->d->user_fn) {
+  h->d->user_fn = (k->kind == TILE_KERNEL_USER || k->kind == TILE_KERNEL_USER_STENCIL) && k->user
+                      ? k->user->f : nullptr;
+  if (h->d->user_fn && tiles::userfn_is_stencil(h->d->user_fn) != (k->kind == TILE_KERNEL_USER_STENCIL)) {
+    h->d->user_fn = nullptr;
+    return fail(TILE_EINVAL, "user function kind does not match the kernel kind (pointwise vs stencil)");
+  }
+  if (h->d->user_fn && k->kind == TILE_KERNEL_USER) {
     const tiles::Geometry& G = h->d->G;
     const int64_t all[6] = {0, 0, 0, G.g[0], G.g[1], G.g[2]};
     const int64_t* b = k->box ? k->box : all;
@@ -246,6 +251,16 @@ tile_status tile_user_fn_create(const char* source, const char* name, tile_user_
   *out = nullptr;
   tiles::UserFn* f = nullptr;
   Status s = tiles::userfn_create(source, name, &f);
+  if (s.bad()) return finish(nullptr, s);
+  *out = new tile_user_fn{f};
+  return TILE_OK;
+}
+
+tile_status tile_user_stencil_create(const char* source, const char* name, tile_user_fn** out) {
+  if (!out) return fail(TILE_EINVAL, "null out");
+  *out = nullptr;
+  tiles::UserFn* f = nullptr;
+  Status s = tiles::userfn_create_stencil(source, name, &f);
   if (s.bad()) return finish(nullptr, s);
   *out = new tile_user_fn{f};
   return TILE_OK;

@@ -133,6 +133,32 @@ struct CudaExec final : Exec {
   Status heat(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
               const TileItem* dev_items, int st, int direct_bit, int nstack, int nsteps) override {
     if (d.measure == TILE_MEASURE_XFER_ONLY || n == 0) return Status::ok();
+    if (d.user_fn && userfn_is_stencil(d.user_fn)) {  // TILE_KERNEL_USER_STENCIL (face ghosts)
+      double* fx[6];
+      for (int f = 0; f < 6; ++f) fx[f] = d.faces[f][rp ^ 1];
+      const double* const* gs = d.gsrc_dev[rp];
+      Status r;
+      if (dev_items) {
+        r = timed(d, st, [&] {
+          Status u = userfn_launch_stencil(d.user_fn, dev_items, n, nullptr, nullptr, 0, gs, fx, d.G.face_elems,
+                                           d.G.t, d.G.depth, S(st));
+          return u.bad() ? cudaErrorLaunchFailure : cudaSuccess;
+        });
+        if (r.bad()) return r;
+        d.stats.n_kernels++;
+      } else {
+        for (int i = 0; i < n; ++i) {
+          r = timed(d, st, [&] {
+            Status u = userfn_launch_stencil(d.user_fn, nullptr, 1, d.slot_ptr(in[i]), d.slot_ptr(out[i]),
+                                             (int)tiles[i], gs, fx, d.G.face_elems, d.G.t, d.G.depth, S(st));
+            return u.bad() ? cudaErrorLaunchFailure : cudaSuccess;
+          });
+          if (r.bad()) return r;
+          d.stats.n_kernels++;
+        }
+      }
+      return Status::ok();
+    }
     if (nsteps > 1 && (!coop || direct_bit < 0 || !dev_items || (int64_t)sms * heat_occ > kMaxProgCtas)) {
       // no persistent launch possible: one launch per step (buffers and face
       // parities alternate)

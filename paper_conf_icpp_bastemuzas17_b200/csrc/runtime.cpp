@@ -1269,7 +1269,7 @@ static Status run_stream(Domain& d, const tile_kernel& k, int T, int S) {
   const Geometry& G = d.G;
   const Pipes P(S, false);
   Sched sc(d, P);
-  const bool heat = k.kind == TILE_KERNEL_HEAT7;
+  const bool heat = k.kind == TILE_KERNEL_HEAT7 || k.kind == TILE_KERNEL_USER_STENCIL;
   const bool fuse = !heat && d.opt.fuse_pointwise_steps;
   const std::vector<int> kp = heat ? plan_passes(d, T) : std::vector<int>();
   const int passes = heat ? (int)kp.size() : fuse ? (T > 0 ? 1 : 0) : T;
@@ -1422,6 +1422,10 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
   } else if (k.kind == TILE_KERNEL_SINCOS || k.kind == TILE_KERNEL_USER) {
     if (k.inner_iters < 0) return make_err(TILE_EINVAL, "inner_iters must be >= 0");
     if (k.kind == TILE_KERNEL_USER && !d.user_fn) return make_err(TILE_EINVAL, "USER kernel without a function");
+  } else if (k.kind == TILE_KERNEL_USER_STENCIL) {
+    if (!d.user_fn) return make_err(TILE_EINVAL, "USER_STENCIL kernel without a function");
+    if (d.G.nranks != 1 || d.G.ghost != 1)
+      return make_err(TILE_EINVAL, "USER_STENCIL: single rank and ghost = 1 only");
   } else {
     return make_err(TILE_EINVAL, "unknown kernel kind");
   }
@@ -1439,6 +1443,23 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
   d.last_S = S;
   d.last_serial = serial;
   d.in_flight = true;
+  if (k.kind == TILE_KERNEL_USER_STENCIL) {
+    // the heat kernel's specialised paths (direct ghosts, persistent and
+    // two-step launches, stream-through sweeps) compute HEAT7 itself: a user
+    // stencil runs the face-ghost single-step schedule of the same machinery
+    const bool direct = d.direct_ok, persist = d.persist_ok, x2 = d.x2_ok;
+    const int32_t st_opt = d.opt.stream_through;
+    d.direct_ok = d.persist_ok = d.x2_ok = false;
+    d.opt.stream_through = -1;
+    r = d.mode == MODE_RESIDENT ? run_heat_resident(d, 0.0, steps, S, serial) : run_stream(d, k, steps, S);
+    d.direct_ok = direct;
+    d.persist_ok = persist;
+    d.x2_ok = x2;
+    d.opt.stream_through = st_opt;
+    if (r.bad()) return r;
+    d.stats.steps_done += (uint64_t)steps;
+    return Status::ok();
+  }
   if (k.kind == TILE_KERNEL_HEAT7 && d.mode == MODE_RESIDENT) {
     r = run_heat_resident(d, k.alpha, steps, S, serial);
   } else if (d.mode == MODE_RESIDENT) {

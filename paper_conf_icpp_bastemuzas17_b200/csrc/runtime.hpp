@@ -323,6 +323,11 @@ Status local_halo(Domain& d, int parity, void* stream, void* ready_event);
 struct UserFn;  // userfn.cpp
 Status userfn_create(const char* source, const char* name, UserFn** out);
 void userfn_free(UserFn* f);
+Status userfn_create_stencil(const char* source, const char* name, UserFn** out);
+bool userfn_is_stencil(const UserFn* f);
+Status userfn_launch_stencil(UserFn* f, const void* dev_items, int nitems, const double* in, double* out,
+                             int tile, const double* const* gsrc, double* const fexp[6],
+                             const int64_t face_elems[6], const int64_t t[3], int depth, void* stream);
 Status userfn_launch(UserFn* f, double* data, int64_t n, const int64_t tdims[2], const int64_t org[3],
                      const int64_t gdims[2], int64_t iters, const int64_t box[6], void* stream);
 Status peer_setup(Domain& d, uint64_t halo_bytes, uint64_t st_bytes);

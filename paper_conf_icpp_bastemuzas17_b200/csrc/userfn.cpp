@@ -102,6 +102,7 @@ bool valid_identifier(const char* s) {
 }  // namespace
 
 struct UserFn {
+  bool stencil = false;  // 7-point user stencil (tile_user_stencil_create)
   std::string name;
   std::vector<char> cubin;
   std::mutex m;
@@ -109,11 +110,59 @@ struct UserFn {
   std::vector<std::pair<int, CUfunction>> fns;
 };
 
+static Status compile(const std::string& src, const char* name, bool stencil, UserFn** out);
+
+// 7-point user stencil: the face layouts and ghost conventions of the
+// library's stencil kernels (HeatParams::gsrc / fexp, kernels.cuh), one
+// thread per cell, ghosts from the read-parity faces, the new boundary layers
+// exported to the write-parity faces for the next step's neighbours.
+static const char* kStencilWrapper = R"(
+struct TileItemJ { const double* in; double* out; int tile; int pad; };
+extern "C" __global__ void tile_user_stencil(const TileItemJ* items, const double* in1, double* out1,
+    int tile1, const double* const* gsrc, double* fx0, double* fx1, double* fy0, double* fy1,
+    double* fz0, double* fz1, long long e0, long long e1, long long e2, long long e3, long long e4,
+    long long e5, int tx, int ty, int tz, int D) {
+  TileItemJ it;
+  if (items) it = items[blockIdx.y]; else { it.in = in1; it.out = out1; it.tile = tile1; }
+  const long long n = (long long)tx * ty * tz, pl = (long long)tx * ty, t = it.tile;
+  const double* const* gs = gsrc + t * 6;
+  const double* u = it.in;
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (long long)gridDim.x * blockDim.x) {
+    const int x = (int)(i % tx);
+    const long long r = i / tx;
+    const int y = (int)(r % ty), z = (int)(r / ty);
+    const double c = u[i];
+    const double xm = x > 0 ? u[i - 1] : gs[0][((long long)z * ty + y) * D + (D - 1)];
+    const double xp = x < tx - 1 ? u[i + 1] : gs[1][((long long)z * ty + y) * D];
+    const double ym = y > 0 ? u[i - tx] : gs[2][((long long)z * D + (D - 1)) * tx + x];
+    const double yp = y < ty - 1 ? u[i + tx] : gs[3][((long long)z * D) * tx + x];
+    const double zm = z > 0 ? u[i - pl] : gs[4][((long long)(D - 1) * ty + y) * tx + x];
+    const double zp = z < tz - 1 ? u[i + pl] : gs[5][(long long)y * tx + x];
+    const double v = USER_STENCIL(c, xm, xp, ym, yp, zm, zp);
+    it.out[i] = v;
+    if (x < D) fx0[t * e0 + ((long long)z * ty + y) * D + x] = v;
+    if (x >= tx - D) fx1[t * e1 + ((long long)z * ty + y) * D + (x - (tx - D))] = v;
+    if (y < D) fy0[t * e2 + ((long long)z * D + y) * tx + x] = v;
+    if (y >= ty - D) fy1[t * e3 + ((long long)z * D + (y - (ty - D))) * tx + x] = v;
+    if (z < D) fz0[t * e4 + ((long long)z * ty + y) * tx + x] = v;
+    if (z >= tz - D) fz1[t * e5 + ((long long)(z - (tz - D)) * ty + y) * tx + x] = v;
+  }
+}
+)";
+
+Status userfn_create_stencil(const char* source, const char* name, UserFn** out) {
+  if (!source || !out) return make_err(TILE_EINVAL, "null argument");
+  if (!valid_identifier(name)) return make_err(TILE_EINVAL, "user function name must be a C identifier");
+  std::string w = kStencilWrapper;
+  const std::string key = "USER_STENCIL";
+  w.replace(w.find(key), key.size(), name);
+  return compile(std::string(source) + "\n" + w, name, true, out);
+}
+
 Status userfn_create(const char* source, const char* name, UserFn** out) {
   if (!source || !out) return make_err(TILE_EINVAL, "null argument");
   if (!valid_identifier(name)) return make_err(TILE_EINVAL, "user function name must be a C identifier");
-  Nvrtc& n = nvrtc();
-  if (!n.ok) return make_err(TILE_ENOSYS, "libnvrtc not available");
   const std::string src = std::string(source) +
                           "\nextern \"C\" __global__ void tile_user_apply(double* __restrict__ u, long long n,"
                           " long long tx, long long ty, long long x0, long long y0, long long z0,"
@@ -128,6 +177,12 @@ Status userfn_create(const char* source, const char* name, UserFn** out) {
                           "    double v = u[i];\n"
                           "    for (long long k = 0; k < iters; ++k) v = " + std::string(name) + "(v, g);\n"
                           "    u[i] = v;\n  }\n}\n";
+  return compile(src, name, false, out);
+}
+
+static Status compile(const std::string& src, const char* name, bool stencil, UserFn** out) {
+  Nvrtc& n = nvrtc();
+  if (!n.ok) return make_err(TILE_ENOSYS, "libnvrtc not available");
   nvrtcProgram_t prog = nullptr;
   if (n.create(&prog, src.c_str(), "tile_user.cu", 0, nullptr, nullptr) != 0)
     return make_err(TILE_EINVAL, "nvrtcCreateProgram failed");
@@ -144,6 +199,7 @@ Status userfn_create(const char* source, const char* name, UserFn** out) {
   size_t cs = 0;
   n.cubin_size(prog, &cs);
   auto* f = new UserFn;
+  f->stencil = stencil;
   f->name = name;
   f->cubin.resize(cs);
   n.cubin(prog, f->cubin.data());
@@ -160,25 +216,63 @@ void userfn_free(UserFn* f) {
   delete f;
 }
 
-Status userfn_launch(UserFn* f, double* data, int64_t n, const int64_t tdims[2], const int64_t org[3],
-                     const int64_t gdims[2], int64_t iters, const int64_t box[6], void* stream) {
+static Status function_on_device(UserFn* f, CUfunction* out, int* dev_out) {
   Drv& d = drv();
   if (!d.ok) return make_err(TILE_ENOSYS, "driver entry points for module loading unavailable");
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess) return make_err(TILE_ECUDA, "cudaGetDevice");
-  CUfunction fn = nullptr;
-  {
-    std::lock_guard<std::mutex> lk(f->m);
-    for (auto& p : f->fns)
-      if (p.first == dev) fn = p.second;
-    if (!fn) {
-      CUmodule mod = nullptr;
-      if (d.load(&mod, f->cubin.data()) != CUDA_SUCCESS) return make_err(TILE_ECUDA, "cuModuleLoadData (user kernel)");
-      if (d.get(&fn, mod, "tile_user_apply") != CUDA_SUCCESS) return make_err(TILE_ECUDA, "cuModuleGetFunction");
-      f->modules.push_back({dev, mod});
-      f->fns.push_back({dev, fn});
+  *dev_out = dev;
+  std::lock_guard<std::mutex> lk(f->m);
+  for (auto& p : f->fns)
+    if (p.first == dev) {
+      *out = p.second;
+      return Status::ok();
     }
-  }
+  CUmodule mod = nullptr;
+  CUfunction fn = nullptr;
+  if (d.load(&mod, f->cubin.data()) != CUDA_SUCCESS) return make_err(TILE_ECUDA, "cuModuleLoadData (user kernel)");
+  if (d.get(&fn, mod, f->stencil ? "tile_user_stencil" : "tile_user_apply") != CUDA_SUCCESS)
+    return make_err(TILE_ECUDA, "cuModuleGetFunction");
+  f->modules.push_back({dev, mod});
+  f->fns.push_back({dev, fn});
+  *out = fn;
+  return Status::ok();
+}
+
+bool userfn_is_stencil(const UserFn* f) { return f && f->stencil; }
+
+Status userfn_launch_stencil(UserFn* f, const void* dev_items, int nitems, const double* in, double* out,
+                             int tile, const double* const* gsrc, double* const fexp[6],
+                             const int64_t face_elems[6], const int64_t t[3], int depth, void* stream) {
+  CUfunction fn = nullptr;
+  int dev = 0;
+  Status s = function_on_device(f, &fn, &dev);
+  if (s.bad()) return s;
+  int tx = (int)t[0], ty = (int)t[1], tz = (int)t[2], D = depth, tl = tile;
+  long long e[6];
+  double* fx[6];
+  for (int i = 0; i < 6; ++i) e[i] = face_elems[i], fx[i] = fexp[i];
+  const void* items = dev_items;
+  void* args[] = {&items, &in, &out, &tl, &gsrc, &fx[0], &fx[1], &fx[2], &fx[3], &fx[4], &fx[5],
+                  &e[0], &e[1], &e[2], &e[3], &e[4], &e[5], &tx, &ty, &tz, &D};
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const long long cells = (long long)tx * ty * tz;
+  const long long bx = std::max<long long>(1, std::min<long long>((cells + 255) / 256,
+                                                                  (long long)sms * 8 / std::max(1, nitems) + 1));
+  if (drv().launch(fn, (unsigned)bx, (unsigned)std::max(1, nitems), 1, 256, 1, 1, 0, static_cast<CUstream>(stream),
+                   args, nullptr) != CUDA_SUCCESS)
+    return make_err(TILE_ECUDA, "cuLaunchKernel (user stencil)");
+  return Status::ok();
+}
+
+Status userfn_launch(UserFn* f, double* data, int64_t n, const int64_t tdims[2], const int64_t org[3],
+                     const int64_t gdims[2], int64_t iters, const int64_t box[6], void* stream) {
+  Drv& d = drv();
+  CUfunction fn = nullptr;
+  int dev = 0;
+  Status st = function_on_device(f, &fn, &dev);
+  if (st.bad()) return st;
   long long a_n = n, tx = tdims[0], ty = tdims[1], x0 = org[0], y0 = org[1], z0 = org[2], nx = gdims[0],
             ny = gdims[1], it = iters;
   long long b[6];

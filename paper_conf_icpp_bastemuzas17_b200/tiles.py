@@ -28,7 +28,7 @@ TILE_OK, TILE_EINVAL, TILE_ENOMEM_HOST, TILE_ENOMEM_DEVICE, TILE_ECUDA, TILE_ENC
 STATUS_NAMES = {0: "OK", 1: "EINVAL", 2: "ENOMEM_HOST", 3: "ENOMEM_DEVICE", 4: "ECUDA",
                 5: "ENCCL", 6: "ESTATE", 7: "ENOSYS"}
 TILE_BC_PERIODIC, TILE_BC_DIRICHLET = 0, 1
-TILE_KERNEL_HEAT7, TILE_KERNEL_SINCOS, TILE_KERNEL_USER = 1, 2, 3
+TILE_KERNEL_HEAT7, TILE_KERNEL_SINCOS, TILE_KERNEL_USER, TILE_KERNEL_USER_STENCIL = 1, 2, 3, 4
 TILE_SCHED_AUTO, TILE_SCHED_RESIDENT, TILE_SCHED_STREAM, TILE_SCHED_SYNC = 0, 1, 2, 3
 TILE_MEASURE_NORMAL, TILE_MEASURE_XFER_ONLY, TILE_MEASURE_COMP_ONLY = 0, 1, 2
 OP_NAMES = {1: "h2d", 2: "d2h", 3: "kernel", 4: "record", 5: "wait", 6: "faces_h2d",
@@ -120,6 +120,7 @@ _sig = {
     "tile_version": ([], ctypes.c_char_p),
     "tile_user_fn_create": ([ctypes.c_char_p, ctypes.c_char_p, ctypes.POINTER(_P)], ctypes.c_int),
     "tile_user_fn_free": ([_P], ctypes.c_int),
+    "tile_user_stencil_create": ([ctypes.c_char_p, ctypes.c_char_p, ctypes.POINTER(_P)], ctypes.c_int),
 }
 EXPORTED = tuple(_sig)
 for _name, (_args, _res) in _sig.items():
@@ -177,10 +178,12 @@ class UserFn:
     """A user pointwise function compiled by libtiles (tile_user_fn_create):
     `source` defines ``__device__ double <name>(double u, long long gidx)``."""
 
-    def __init__(self, source, name):
+    def __init__(self, source, name, stencil=False):
         h = ctypes.c_void_p()
-        _check(tile_user_fn_create(source.encode(), name.encode(), ctypes.byref(h)), "tile_user_fn_create")
+        create = tile_user_stencil_create if stencil else tile_user_fn_create
+        _check(create(source.encode(), name.encode(), ctypes.byref(h)), create.__name__)
         self._h = h
+        self.stencil = stencil
 
     def free(self):
         if self._h is not None:
@@ -192,6 +195,14 @@ class UserFn:
             self.free()
         except Exception:
             pass
+
+
+def user_stencil(fn):
+    """Kernel descriptor of a user 7-point stencil (UserFn(..., stencil=True))."""
+    k = TileKernel(TILE_KERNEL_USER_STENCIL, 0.0, 0)
+    k.user = fn._h.value
+    k._fn = fn
+    return k
 
 
 def user(fn, inner_iters=1, box=None):
