@@ -1,7 +1,7 @@
 """Small runs of every schedule for compute-sanitizer (memcheck / racecheck /
 synccheck / initcheck): resident heat (layered + whole-domain phases),
 streaming heat with a tiny budget, Dirichlet, sincos, the generic kernel, the
-persistent multi-step launch (direct ghosts, grid counter, snake order; banded tiles in round-robin order), a ranged NVRTC user kernel and
+persistent multi-step launch (direct ghosts, grid counter, snake order; banded tiles in round-robin order), a ranged NVRTC user kernel, a user stencil and
 the stream-through schedule and the in-process multi-rank transport."""
 import os
 import sys
@@ -61,6 +61,10 @@ with T.Domain((512, 512, 16), (32, 64, 8)) as d:          # snake-ordered persis
 fu = T.UserFn("__device__ double aff(double u, long long g) { return 2.0 * u + 1.0; }", "aff")
 with T.Domain((64, 32, 32), (32, 16, 16)) as d:           # user pointwise kernel (NVRTC), ranged
     d.load(u); d.run(T.user(fu, 2, box=((5, 3, 7), (40, 16, 32))), 2, 2); d.store()
+fs = T.UserFn("__device__ double hu(double c, double xm, double xp, double ym, double yp, double zm, double zp)"
+              " { return c + 0.125 * ((((xm + xp) + (ym + yp)) + (zm + zp)) - 6.0 * c); }", "hu", stencil=True)
+with T.Domain((64, 32, 32), (32, 16, 16)) as d:           # user stencil (NVRTC, face ghosts)
+    d.load(u); d.run(T.user_stencil(fs), 3, 2); d.run(T.heat7(), 2, 2); d.store()
 g = T.LocalGroup(2)
 def rank(r):
     with T.Domain((64, 32, 64), (32, 16, 16), nranks=2, rank=r, local_group=g) as d:
