@@ -114,8 +114,9 @@ static Status compile(const std::string& src, const char* name, bool stencil, Us
 
 // 7-point user stencil: the face layouts and ghost conventions of the
 // library's stencil kernels (HeatParams::gsrc / fexp, kernels.cuh), one
-// thread per cell, ghosts from the read-parity faces, the new boundary layers
-// exported to the write-parity faces for the next step's neighbours.
+// thread per (x, y) column marching z (z-1, z in registers; in-plane
+// neighbours through L1), ghosts from the read-parity faces, the new boundary
+// layers exported to the write-parity faces for the next step's neighbours.
 static const char* kStencilWrapper = R"(
 struct TileItemJ { const double* in; double* out; int tile; int pad; };
 extern "C" __global__ void tile_user_stencil(const TileItemJ* items, const double* in1, double* out1,
@@ -124,29 +125,32 @@ extern "C" __global__ void tile_user_stencil(const TileItemJ* items, const doubl
     long long e5, int tx, int ty, int tz, int D) {
   TileItemJ it;
   if (items) it = items[blockIdx.y]; else { it.in = in1; it.out = out1; it.tile = tile1; }
-  const long long n = (long long)tx * ty * tz, pl = (long long)tx * ty, t = it.tile;
+  const long long pl = (long long)tx * ty, t = it.tile;
   const double* const* gs = gsrc + t * 6;
   const double* u = it.in;
-  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n;
-       i += (long long)gridDim.x * blockDim.x) {
-    const int x = (int)(i % tx);
-    const long long r = i / tx;
-    const int y = (int)(r % ty), z = (int)(r / ty);
-    const double c = u[i];
-    const double xm = x > 0 ? u[i - 1] : gs[0][((long long)z * ty + y) * D + (D - 1)];
-    const double xp = x < tx - 1 ? u[i + 1] : gs[1][((long long)z * ty + y) * D];
-    const double ym = y > 0 ? u[i - tx] : gs[2][((long long)z * D + (D - 1)) * tx + x];
-    const double yp = y < ty - 1 ? u[i + tx] : gs[3][((long long)z * D) * tx + x];
-    const double zm = z > 0 ? u[i - pl] : gs[4][((long long)(D - 1) * ty + y) * tx + x];
-    const double zp = z < tz - 1 ? u[i + pl] : gs[5][(long long)y * tx + x];
-    const double v = USER_STENCIL(c, xm, xp, ym, yp, zm, zp);
-    it.out[i] = v;
-    if (x < D) fx0[t * e0 + ((long long)z * ty + y) * D + x] = v;
-    if (x >= tx - D) fx1[t * e1 + ((long long)z * ty + y) * D + (x - (tx - D))] = v;
-    if (y < D) fy0[t * e2 + ((long long)z * D + y) * tx + x] = v;
-    if (y >= ty - D) fy1[t * e3 + ((long long)z * D + (y - (ty - D))) * tx + x] = v;
-    if (z < D) fz0[t * e4 + ((long long)z * ty + y) * tx + x] = v;
-    if (z >= tz - D) fz1[t * e5 + ((long long)(z - (tz - D)) * ty + y) * tx + x] = v;
+  // one thread per (x, y) column, marching z: z-1 and z stay in registers
+  for (int col = blockIdx.x * blockDim.x + threadIdx.x; col < tx * ty; col += gridDim.x * blockDim.x) {
+    const int x = col % tx, y = col / tx;
+    double zm = gs[4][((long long)(D - 1) * ty + y) * tx + x];
+    double c = u[col];
+    for (int z = 0; z < tz; ++z) {
+      const long long i = (long long)z * pl + col;
+      const double zp = z < tz - 1 ? u[i + pl] : gs[5][(long long)y * tx + x];
+      const double xm = x > 0 ? u[i - 1] : gs[0][((long long)z * ty + y) * D + (D - 1)];
+      const double xp = x < tx - 1 ? u[i + 1] : gs[1][((long long)z * ty + y) * D];
+      const double ym = y > 0 ? u[i - tx] : gs[2][((long long)z * D + (D - 1)) * tx + x];
+      const double yp = y < ty - 1 ? u[i + tx] : gs[3][((long long)z * D) * tx + x];
+      const double v = USER_STENCIL(c, xm, xp, ym, yp, zm, zp);
+      it.out[i] = v;
+      if (x < D) fx0[t * e0 + ((long long)z * ty + y) * D + x] = v;
+      if (x >= tx - D) fx1[t * e1 + ((long long)z * ty + y) * D + (x - (tx - D))] = v;
+      if (y < D) fy0[t * e2 + ((long long)z * D + y) * tx + x] = v;
+      if (y >= ty - D) fy1[t * e3 + ((long long)z * D + (y - (ty - D))) * tx + x] = v;
+      if (z < D) fz0[t * e4 + ((long long)z * ty + y) * tx + x] = v;
+      if (z >= tz - D) fz1[t * e5 + ((long long)(z - (tz - D)) * ty + y) * tx + x] = v;
+      zm = c;
+      c = zp;
+    }
   }
 }
 )";
@@ -255,11 +259,8 @@ Status userfn_launch_stencil(UserFn* f, const void* dev_items, int nitems, const
   const void* items = dev_items;
   void* args[] = {&items, &in, &out, &tl, &gsrc, &fx[0], &fx[1], &fx[2], &fx[3], &fx[4], &fx[5],
                   &e[0], &e[1], &e[2], &e[3], &e[4], &e[5], &tx, &ty, &tz, &D};
-  int sms = 148;
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const long long cells = (long long)tx * ty * tz;
-  const long long bx = std::max<long long>(1, std::min<long long>((cells + 255) / 256,
-                                                                  (long long)sms * 8 / std::max(1, nitems) + 1));
+  const long long cols = (long long)tx * ty;  // one thread per (x, y) column
+  const long long bx = std::max<long long>(1, (cols + 255) / 256);
   if (drv().launch(fn, (unsigned)bx, (unsigned)std::max(1, nitems), 1, 256, 1, 1, 0, static_cast<CUstream>(stream),
                    args, nullptr) != CUDA_SUCCESS)
     return make_err(TILE_ECUDA, "cuLaunchKernel (user stencil)");
