@@ -365,8 +365,9 @@ tile_status tile_user_fn_free(tile_user_fn* fn);
  * tiles' exported faces (or Dirichlet fixed faces), each step exporting the new
  * boundary layers, resident or streamed out of core (the heat kernel's
  * specialised paths — direct ghosts, persistent and two-step launches,
- * stream-through — stay HEAT7-only). Single rank, ghost = 1 (EINVAL
- * otherwise). Free with tile_user_fn_free like a pointwise function. */
+ * stream-through — stay HEAT7-only). z-slab ranks exchange the slab-end
+ * faces with copies (any transport). ghost = 1 (EINVAL otherwise). Free
+ * with tile_user_fn_free like a pointwise function. */
 tile_status tile_user_stencil_create(const char* source, const char* name, tile_user_fn** out);
 
 /* Fill out[128] with a fresh ncclUniqueId (call on rank 0, then broadcast).

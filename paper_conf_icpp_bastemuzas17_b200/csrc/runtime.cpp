@@ -1424,8 +1424,7 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
     if (k.kind == TILE_KERNEL_USER && !d.user_fn) return make_err(TILE_EINVAL, "USER kernel without a function");
   } else if (k.kind == TILE_KERNEL_USER_STENCIL) {
     if (!d.user_fn) return make_err(TILE_EINVAL, "USER_STENCIL kernel without a function");
-    if (d.G.nranks != 1 || d.G.ghost != 1)
-      return make_err(TILE_EINVAL, "USER_STENCIL: single rank and ghost = 1 only");
+    if (d.G.ghost != 1) return make_err(TILE_EINVAL, "USER_STENCIL: ghost = 1 only");
   } else {
     return make_err(TILE_EINVAL, "unknown kernel kind");
   }
@@ -1447,14 +1446,18 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
     // the heat kernel's specialised paths (direct ghosts, persistent and
     // two-step launches, stream-through sweeps) compute HEAT7 itself: a user
     // stencil runs the face-ghost single-step schedule of the same machinery
-    const bool direct = d.direct_ok, persist = d.persist_ok, x2 = d.x2_ok;
+    // z-slab ranks exchange the exported slab-end faces by copies (the fused
+    // transport's in-kernel push is HEAT7's; its exchange counters are
+    // monotonic, so copy and fused exchanges interleave across runs)
+    const bool direct = d.direct_ok, persist = d.persist_ok, x2 = d.x2_ok, fused = d.peer_fused;
     const int32_t st_opt = d.opt.stream_through;
-    d.direct_ok = d.persist_ok = d.x2_ok = false;
+    d.direct_ok = d.persist_ok = d.x2_ok = d.peer_fused = false;
     d.opt.stream_through = -1;
     r = d.mode == MODE_RESIDENT ? run_heat_resident(d, 0.0, steps, S, serial) : run_stream(d, k, steps, S);
     d.direct_ok = direct;
     d.persist_ok = persist;
     d.x2_ok = x2;
+    d.peer_fused = fused;
     d.opt.stream_through = st_opt;
     if (r.bad()) return r;
     d.stats.steps_done += (uint64_t)steps;

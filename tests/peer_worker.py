@@ -7,7 +7,11 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def run(r, G, dims, td, bc, sched, budget, runs, seed, conn, transport=1, stream_through=0):
+HEAT_AS_USER = ("__device__ double hu(double c, double xm, double xp, double ym, double yp, double zm,"
+                " double zp) { return c + 0.125 * ((((xm + xp) + (ym + yp)) + (zm + zp)) - 6.0 * c); }")
+
+
+def run(r, G, dims, td, bc, sched, budget, runs, seed, conn, transport=1, stream_through=0, user_runs=()):
     sys.path.insert(0, ROOT)
     try:
         import synth
@@ -28,8 +32,9 @@ def run(r, G, dims, td, bc, sched, budget, runs, seed, conn, transport=1, stream
                 ext = synth.uniform_grid(nx + 2, ny + 2, nz + 2, seed)
                 d.load(ext[r * nzl:r * nzl + nzl + 2])
             firsts = []
+            fs = T.UserFn(HEAT_AS_USER, "hu", stencil=True) if user_runs else None
             for i, s in enumerate(runs):
-                d.run(T.heat7(0.125), s, 2)
+                d.run(T.user_stencil(fs) if i in user_runs else T.heat7(0.125), s, 2)
                 if i == 0:
                     d.sync()
                     firsts = [d.stats(), d.store()]

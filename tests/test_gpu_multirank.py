@@ -109,7 +109,7 @@ def test_peer_transport_processes_bit_exact(G, bc, sched, runs, transport):
     assert all(m[2] > 0 and m[3] > 0 for m in outs)  # halo exchanges happened through the window
 
 
-def _peer_procs(G, dims, td, bc, sched, budget, runs, transport, stream_through=0):
+def _peer_procs(G, dims, td, bc, sched, budget, runs, transport, stream_through=0, user_runs=()):
     """One spawned process per rank (tests/peer_worker.py), IPC handles
     relayed through pipes; returns every rank's ("out", ...) message."""
     import multiprocessing as mp
@@ -119,7 +119,8 @@ def _peer_procs(G, dims, td, bc, sched, budget, runs, transport, stream_through=
     for r in range(G):
         a, b = ctx.Pipe()
         p = ctx.Process(target=peer_worker.run,
-                        args=(r, G, dims, td, bc, sched, budget, runs, 42, b, transport, stream_through))
+                        args=(r, G, dims, td, bc, sched, budget, runs, 42, b, transport, stream_through,
+                              tuple(user_runs)))
         p.start()
         pipes.append(a)
         procs.append(p)
@@ -171,3 +172,63 @@ def test_peer_stream_through_slabs_bit_exact(G, T, tz, runs_after):
         st = m[4][0]
         assert st["bytes_h2d"] == nx * ny * nzl * 8 and st["bytes_d2h"] == nx * ny * nzl * 8
         assert st["bytes_halo"] == 2 * nx * ny * T * 8  # one layer of T planes to each neighbour
+
+
+@pytest.mark.parametrize("G,bc,sched", [(2, "periodic", "resident"), (3, "dirichlet", "resident"),
+                                        (4, "periodic", "stream")])
+def test_local_group_user_stencil_bit_exact(G, bc, sched):
+    """User 7-point stencil (the heat update as NVRTC source) on z-slab ranks
+    (in-process transport), interleaved with built-in HEAT7 runs: bit-exact."""
+    dims, td = (64, 32, 16 * G), (32, 16, 8)
+    nx, ny, nz = dims
+    nzl = nz // G
+    runs = [("user", 3), ("heat", 2), ("user", 2)]
+    if bc == "periodic":
+        u = synth.uniform_grid(nx, ny, nz, 42)
+        ref = oracle.heat_c(u, ALPHA, 7)
+    else:
+        ext = synth.uniform_grid(nx + 2, ny + 2, nz + 2, 5)
+        ref = oracle.heat_c(ext, ALPHA, 7, oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+    fs = T.UserFn("__device__ double hu(double c, double xm, double xp, double ym, double yp, double zm,"
+                  " double zp) { return c + 0.125 * ((((xm + xp) + (ym + yp)) + (zm + zp)) - 6.0 * c); }",
+                  "hu", stencil=True)
+    group = T.LocalGroup(G)
+    out = [None] * G
+    err = []
+
+    def rank(r):
+        try:
+            kw = {"sched": sched}
+            if sched == "stream":
+                kw["device_budget_bytes"] = _budget(dims, td, 3, bc=bc, nranks=G, rank=r)
+            with T.Domain(dims, td, bc=bc, nranks=G, rank=r, local_group=group, device=0, **kw) as d:
+                d.load(u[r * nzl:(r + 1) * nzl] if bc == "periodic" else ext[r * nzl:r * nzl + nzl + 2])
+                for kind, s in runs:
+                    d.run(T.user_stencil(fs) if kind == "user" else T.heat7(ALPHA), s, 2)
+                o = d.store()
+                out[r] = o if bc == "periodic" else o[1:-1, 1:-1, 1:-1]
+        except Exception as e:  # noqa
+            err.append(e)
+
+    th = [threading.Thread(target=rank, args=(r,)) for r in range(G)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(120)
+    group.free()
+    assert not err, err
+    got = np.concatenate(out, axis=0)
+    assert np.array_equal(got, ref), np.abs(got - ref).max()
+
+
+@pytest.mark.parametrize("G,transport", [(2, 2), (3, 1)])
+def test_peer_user_stencil_interleaved_bit_exact(G, transport):
+    """One process per rank over the peer transport (2 = fused: HEAT7 runs push
+    in-kernel, user-stencil runs exchange by copies, the counters shared):
+    HEAT7 / user stencil / HEAT7 / user stencil runs, bit-exact."""
+    dims, td = (64, 32, 16 * G), (32, 16, 8)
+    nx, ny, nz = dims
+    runs = [4, 3, 5, 2]
+    outs = _peer_procs(G, dims, td, "periodic", "resident", 0, runs, transport, user_runs=(1, 3))
+    got = np.concatenate([m[1] for m in outs], axis=0)
+    assert np.array_equal(got, oracle.heat_c(synth.uniform_grid(nx, ny, nz, 42), ALPHA, sum(runs)))
