@@ -288,6 +288,52 @@ def test_residency_fig7_trace(golden_dir):
     assert ro.trace == exp
 
 
+def _residency_cases(path):
+    cases, cur = [], None
+    for row in _read_rows(path):
+        if row[0] == "case":
+            cur = {"nslots": int(row[2]), "steps": []}
+            cases.append(cur)
+        elif row[0] == ">":
+            cur["steps"].append((row[1:], []))
+        else:
+            cur["steps"][-1][1].append((row[0], int(row[1]), int(row[2])))
+    return cases
+
+
+@pytest.mark.parametrize("track_dirty", [True, False])
+def test_residency_dirty_tracking_golden(golden_dir, track_dirty):
+    """Hand-derived traces (readings R4/R10). Without dirty
+    tracking (the paper's literal rule) every drop becomes a D2H and every
+    GPU-disabled request of a device region copies."""
+    for case in _residency_cases(os.path.join(golden_dir, "residency_dirty.txt")):
+        ro = oracle.ResidencyOracle(case["nslots"], track_dirty=track_dirty)
+        for req, exp in case["steps"]:
+            n0 = len(ro.trace)
+            if req[0] == "gpu":
+                ro.gpu_request(int(req[1]), writes=req[2] == "w")
+            elif req[0] == "cpu":
+                ro.cpu_request(int(req[1]))
+            else:
+                ro.jacobi_request(int(req[1]), int(req[2]), int(req[3]))
+            if not track_dirty:
+                exp = [("d2h",) + e[1:] if e[0] == "drop" else e for e in exp]
+                if req[0] == "cpu" and not exp and int(req[1]) in ro.cache:
+                    exp = [("d2h", int(req[1]), ro.cache.index(int(req[1])))]
+            assert ro.trace[n0:] == exp, (req, ro.trace[n0:], exp)
+
+
+def test_residency_one_pointer_per_region():
+    ro = oracle.ResidencyOracle(3, track_dirty=True)
+    ro.jacobi_request(0, 0, 1)
+    with pytest.raises(ValueError):
+        ro.gpu_request(0, slot=2)      # region 0 lives in pointer 1
+    with pytest.raises(ValueError):
+        ro.jacobi_request(0, 0, 2)
+    with pytest.raises(ValueError):
+        ro.jacobi_request(1, 2, 2)
+
+
 def test_residency_all_fit_only_first_sweep_transfers():
     ro = oracle.ResidencyOracle(4)
     for _ in range(3):

@@ -352,3 +352,102 @@ def test_ooc_stream_through_replays_to_oracle(dims, td, nslots, runs, ns):
     st = d.stats()
     assert st["bytes_h2d"] % (cells * 8) == 0 and st["bytes_h2d"] == st["bytes_d2h"]
     assert st["bytes_h2d"] // (cells * 8) < sum(runs)  # fewer link passes than steps
+
+
+# ----------------------------------------------- residency protocol
+def _trace_through_state_machine(trace, nslots):
+    """Feed libtiles' own requests — (tile, pointer) of every kernel, in issue
+    order — through the cache-list state machine of P:L88-L90
+    (oracle.ResidencyOracle with dirty tracking, reading R10) and require the
+    library's hit / h2d / d2h / drop ops to be exactly the ones the state
+    machine emits for them, op for op. The pointer of a request is the
+    library's choice (P:L79 leaves the region -> pointer map unspecified);
+    a D2H of the tile just computed is a write-through, i.e. a GPU-disabled
+    request; D2Hs issued by tile_sync are GPU-disabled requests too,
+    after which no tile may be left newer on the device than on the host."""
+    ro = oracle.ResidencyOracle(nslots, track_dirty=True)
+    pending, last, nreq = [], None, 0
+    for name, _st, a, b, c, _d in trace:
+        if name in ("hit", "h2d", "d2h", "drop"):
+            if name in ("h2d", "d2h"):
+                assert c == 1, "the cache schedule moves one tile per copy"
+            if name == "d2h" and a == last and not pending:
+                n0 = len(ro.trace)
+                ro.cpu_request(a)
+                assert ro.trace[n0:] == [("d2h", a, b)], ("write-through", a, b, ro.trace[n0:])
+                last = None
+                continue
+            pending.append((name, a, b))
+            last = None
+        elif name in ("kernel", "kernel2", "pointwise"):
+            n0 = len(ro.trace)
+            if name == "pointwise":
+                ro.gpu_request(a, writes=True, slot=b)
+            else:
+                ro.jacobi_request(a, b, c)
+            got = [e for e in ro.trace[n0:] if e[0] != "compute"]
+            assert got == pending, (name, a, b, c, got, pending)
+            pending, last, nreq = [], a, nreq + 1
+        else:
+            assert name in ("record", "wait", "faces_h2d", "halo"), name
+    for name, a, b in pending:  # tile_sync's flush: GPU-disabled requests
+        assert name == "d2h", (name, a, b)
+        n0 = len(ro.trace)
+        ro.cpu_request(a)
+        assert ro.trace[n0:] == [("d2h", a, b)]
+    assert not any(ro.dirty), "tile_sync left device-only data"
+    return ro, nreq
+
+
+def test_fig7_residency_trace_matches_state_machine():
+    """The Fig. 7 scenario: the compute-intensive kernel over
+    4 regions with device memory limited to 2, 2 streams, step-major."""
+    dims, td = (8, 8, 16), (8, 8, 4)
+    kw = dict(sched="stream", fuse_pointwise_steps=False, stream_through=-1)
+    b = _budget_for(dims, td, 2, **kw)
+    d = T.Domain(dims, td, dry_run=True, device_budget_bytes=b, **kw)
+    d.load(np.zeros((16, 8, 8)))
+    d.run(T.sincos(2), 3, 2)
+    d.sync()
+    ro, nreq = _trace_through_state_machine(d.trace(), 2)
+    assert nreq == 12
+    ops = [e[0] for e in ro.trace]
+    assert ops.count("h2d") + ops.count("hit") == 12
+
+
+@pytest.mark.parametrize("kind", ["heat", "pointwise"])
+@pytest.mark.parametrize("nslots,ns,steps", [(2, 1, [3]), (3, 2, [2, 1]), (5, 1, [2]), (6, 3, [1, 2]),
+                                             (12, 2, [3]), (20, 4, [2, 2]), (17, 1, [4])])
+def test_stream_residency_trace_matches_state_machine(kind, nslots, ns, steps):
+    dims, td = (16, 16, 16), (8, 8, 4)   # 16 tiles
+    kw = dict(sched="stream", stream_through=-1)
+    b = _budget_for(dims, td, nslots, **kw)
+    d = T.Domain(dims, td, dry_run=True, device_budget_bytes=b, fuse_pointwise_steps=False, **kw)
+    d.load(np.zeros((16, 16, 16)))
+    for s in steps:
+        d.run(T.heat7() if kind == "heat" else T.sincos(1), s, ns)
+    d.sync()
+    _, nreq = _trace_through_state_machine(d.trace(), nslots)
+    assert nreq == 16 * sum(steps)
+
+
+def test_state_machine_check_catches_a_wrong_trace():
+    """The comparison is not vacuous: dropping a write-back, or turning a
+    drop of a dirty tile into a copy-free eviction, fails it."""
+    dims, td = (16, 16, 16), (8, 8, 4)
+    kw = dict(sched="stream", stream_through=-1)
+    b = _budget_for(dims, td, 3, **kw)
+    d = T.Domain(dims, td, dry_run=True, device_budget_bytes=b, **kw)
+    d.load(np.zeros((16, 16, 16)))
+    d.run(T.heat7(), 2, 1)
+    d.sync()
+    tr = d.trace()
+    _trace_through_state_machine(tr, 3)
+    i = next(i for i, op in enumerate(tr) if op[0] == "d2h")
+    with pytest.raises(AssertionError):
+        _trace_through_state_machine(tr[:i] + tr[i + 1:], 3)
+    j = next(i for i, op in enumerate(tr) if op[0] == "drop")
+    bad = list(tr)
+    bad[j] = ("hit",) + tuple(bad[j][1:])
+    with pytest.raises((AssertionError, ValueError)):
+        _trace_through_state_machine(bad, 3)
