@@ -236,10 +236,13 @@ typedef enum {
                             halo push, peer_transport = 2) */
   TILE_OP_HALO_SIGNAL = 23,/* halo exchange of parity d whose data the previous kernels
                             pushed (fused): synchronisation only */
-  TILE_OP_ST_HALO = 24   /* multi-rank stream-through (peer transport): a = 0 push the
+  TILE_OP_ST_HALO = 24,  /* multi-rank stream-through (peer transport): a = 0 push the
                             slab-end c planes of initial data (b = 1 top -> upper rank,
                             0 bottom -> lower rank), 1 wait for side b's halo layer,
                             2 release side b's halo layer; d = the run's epoch */
+  TILE_OP_SYNC = 25      /* host waits for every stream (stream -1): every op before it
+                            completes before any op after it starts; host-side reads of
+                            the pinned store (face extraction) happen here */
 } tile_op_kind;
 
 typedef struct {

@@ -62,6 +62,27 @@ struct CudaExec final : Exec {
     tpending.push_back({a, b});
     return Status::ok();
   }
+  // the same for a launch that reports a library Status (user kernels: the
+  // real cause — ENOSYS, module load, launch — reaches the caller unchanged)
+  template <class F>
+  Status timed_status(Domain& d, int st, F&& launch) {
+    if (!d.kernel_timing) return launch();
+    cudaEvent_t a, b;
+    Status r = timing_event(&a);
+    if (r.bad()) return r;
+    r = timing_event(&b);
+    if (r.bad()) return r;
+    CK(cudaEventRecord(a, S(st)));
+    r = launch();
+    if (r.bad()) {
+      tpool.push_back(a);
+      tpool.push_back(b);
+      return r;
+    }
+    CK(cudaEventRecord(b, S(st)));
+    tpending.push_back({a, b});
+    return Status::ok();
+  }
   Status collect(Domain& d) {  // after a synchronize
     for (auto& pr : tpending) {
       float ms = 0;
@@ -139,19 +160,17 @@ struct CudaExec final : Exec {
       const double* const* gs = d.gsrc_dev[rp];
       Status r;
       if (dev_items) {
-        r = timed(d, st, [&] {
-          Status u = userfn_launch_stencil(d.user_fn, dev_items, n, nullptr, nullptr, 0, gs, fx, d.G.face_elems,
-                                           d.G.t, d.G.depth, S(st));
-          return u.bad() ? cudaErrorLaunchFailure : cudaSuccess;
+        r = timed_status(d, st, [&] {
+          return userfn_launch_stencil(d.user_fn, dev_items, n, nullptr, nullptr, 0, gs, fx, d.G.face_elems,
+                                       d.G.t, d.G.depth, S(st));
         });
         if (r.bad()) return r;
         d.stats.n_kernels++;
       } else {
         for (int i = 0; i < n; ++i) {
-          r = timed(d, st, [&] {
-            Status u = userfn_launch_stencil(d.user_fn, nullptr, 1, d.slot_ptr(in[i]), d.slot_ptr(out[i]),
-                                             (int)tiles[i], gs, fx, d.G.face_elems, d.G.t, d.G.depth, S(st));
-            return u.bad() ? cudaErrorLaunchFailure : cudaSuccess;
+          r = timed_status(d, st, [&] {
+            return userfn_launch_stencil(d.user_fn, nullptr, 1, d.slot_ptr(in[i]), d.slot_ptr(out[i]),
+                                         (int)tiles[i], gs, fx, d.G.face_elems, d.G.t, d.G.depth, S(st));
           });
           if (r.bad()) return r;
           d.stats.n_kernels++;
@@ -434,9 +453,8 @@ struct CudaExec final : Exec {
       const int64_t* b = d.user_box;
       for (int a = 0; a < 3; ++a)  // ranged compute: a tile outside the box launches nothing
         if (org[a] >= b[3 + a] || org[a] + d.G.t[a] <= b[a]) return Status::ok();
-      Status r = timed(d, st, [&] {
-        Status u = userfn_launch(d.user_fn, d.slot_ptr(slot), d.G.tile_elems, td, org, gd, iters, b, S(st));
-        return u.bad() ? cudaErrorLaunchFailure : cudaSuccess;
+      Status r = timed_status(d, st, [&] {
+        return userfn_launch(d.user_fn, d.slot_ptr(slot), d.G.tile_elems, td, org, gd, iters, b, S(st));
       });
       if (r.bad()) return r;
       d.stats.n_kernels++;

@@ -158,7 +158,10 @@ struct DryExec final : Exec {
     put(d, kind, st, a, b, 0, 0);
     return Status::ok();
   }
-  Status sync_all(Domain&) override { return Status::ok(); }
+  Status sync_all(Domain& d) override {
+    put(d, TILE_OP_SYNC, -1, 0, 0, 0, 0);
+    return Status::ok();
+  }
   Status mem_info(Domain& d, uint64_t* fr, uint64_t* tot) override {
     // a pretend device: the budget option (or 64 GiB) is all there is
     *tot = 180ull << 30;

@@ -1285,6 +1285,18 @@ static Status run_stream(Domain& d, const tile_kernel& k, int T, int S) {
   }
   if (heat && !d.faces_valid) {
     if (!d.host_faces_valid) {
+      // the faces come from the host store, so it must hold every tile's
+      // current values first: tiles still dirty on the device (an earlier
+      // pointwise run's kept window) are written back — GPU-disabled
+      // requests, P:L90 — and every queued D2H completes
+      for (int64_t t = 0; t < N; ++t) {
+        if (!d.tile_dirty[t] || d.tile_slot[t] < 0) continue;
+        r = sc.writeback(t);
+        if (r.bad()) return r;
+      }
+      r = X.sync_all(d);
+      if (r.bad()) return r;
+      d.host_pending = false;
       host_extract_faces(G, d.host, d.host_faces);
       d.host_faces_valid = true;
     }
@@ -1506,7 +1518,11 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
       r = run_streamthrough_ooc(d, steps, S, op);
     } else {
       r = run_stream(d, k, steps, S);
-      if (k.kind != TILE_KERNEL_HEAT7 && steps > 0) d.faces_valid = d.xfaces_valid = false;
+      if (k.kind != TILE_KERNEL_HEAT7 && steps > 0) {
+        // tiles changed without their faces (device or host copies)
+        d.faces_valid = d.xfaces_valid = false;
+        d.host_faces_valid = false;
+      }
     }
   }
   if (r.bad()) return r;

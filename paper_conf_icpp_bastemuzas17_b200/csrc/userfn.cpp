@@ -15,6 +15,7 @@
 
 #include <algorithm>
 #include <cctype>
+#include <cstdio>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -215,8 +216,17 @@ static Status compile(const std::string& src, const char* name, bool stencil, Us
 void userfn_free(UserFn* f) {
   if (!f) return;
   Drv& d = drv();
-  if (d.ok)
-    for (auto& m : f->modules) d.unload(m.second);
+  if (d.ok && !f->modules.empty()) {
+    // each module was loaded in its device's primary context: make that
+    // current for the unload (ranks of one process may use other devices)
+    int cur = -1;
+    const bool have_cur = cudaGetDevice(&cur) == cudaSuccess;
+    for (auto& m : f->modules) {
+      if (cudaSetDevice(m.first) != cudaSuccess || d.unload(m.second) != CUDA_SUCCESS)
+        std::fprintf(stderr, "libtiles: user function module unload failed on device %d\n", m.first);
+    }
+    if (have_cur) cudaSetDevice(cur);
+  }
   delete f;
 }
 
@@ -235,8 +245,10 @@ static Status function_on_device(UserFn* f, CUfunction* out, int* dev_out) {
   CUmodule mod = nullptr;
   CUfunction fn = nullptr;
   if (d.load(&mod, f->cubin.data()) != CUDA_SUCCESS) return make_err(TILE_ECUDA, "cuModuleLoadData (user kernel)");
-  if (d.get(&fn, mod, f->stencil ? "tile_user_stencil" : "tile_user_apply") != CUDA_SUCCESS)
+  if (d.get(&fn, mod, f->stencil ? "tile_user_stencil" : "tile_user_apply") != CUDA_SUCCESS) {
+    d.unload(mod);
     return make_err(TILE_ECUDA, "cuModuleGetFunction");
+  }
   f->modules.push_back({dev, mod});
   f->fns.push_back({dev, fn});
   *out = fn;
@@ -261,9 +273,18 @@ Status userfn_launch_stencil(UserFn* f, const void* dev_items, int nitems, const
                   &e[0], &e[1], &e[2], &e[3], &e[4], &e[5], &tx, &ty, &tz, &D};
   const long long cols = (long long)tx * ty;  // one thread per (x, y) column
   const long long bx = std::max<long long>(1, (cols + 255) / 256);
-  if (drv().launch(fn, (unsigned)bx, (unsigned)std::max(1, nitems), 1, 256, 1, 1, 0, static_cast<CUstream>(stream),
-                   args, nullptr) != CUDA_SUCCESS)
-    return make_err(TILE_ECUDA, "cuLaunchKernel (user stencil)");
+  // blockIdx.y = item: launch at most 65535 items at a time (gridDim.y limit;
+  // the wrapper's TileItemJ has TileItem's layout)
+  static_assert(sizeof(TileItem) == 24, "TileItemJ layout");
+  constexpr int kMaxY = 65535;
+  const int total = dev_items ? std::max(1, nitems) : 1;
+  for (int i0 = 0; i0 < total; i0 += kMaxY) {
+    const int ny = std::min(kMaxY, total - i0);
+    items = dev_items ? static_cast<const void*>(static_cast<const TileItem*>(dev_items) + i0) : nullptr;
+    if (drv().launch(fn, (unsigned)bx, (unsigned)ny, 1, 256, 1, 1, 0, static_cast<CUstream>(stream), args,
+                     nullptr) != CUDA_SUCCESS)
+      return make_err(TILE_ECUDA, "cuLaunchKernel (user stencil)");
+  }
   return Status::ok();
 }
 

@@ -35,7 +35,7 @@ OP_NAMES = {1: "h2d", 2: "d2h", 3: "kernel", 4: "record", 5: "wait", 6: "faces_h
             7: "extract", 8: "halo", 9: "drop", 10: "hit", 11: "pointwise", 12: "kernel2",
             13: "gather", 14: "sweep", 15: "scatter", 16: "copy", 17: "h2d_part", 18: "d2h_part",
             19: "copy_part", 20: "h2d_pack", 21: "sweep_u", 22: "kerneld", 23: "halo_signal",
-            24: "st_halo"}
+            24: "st_halo", 25: "sync"}
 SCHEDS = {"auto": 0, "resident": 1, "stream": 2, "sync": 3}
 BCS = {"periodic": 0, "dirichlet": 1}
 
@@ -227,6 +227,7 @@ class Domain:
                  fuse_pointwise_steps=True, device_pool=None, streams=None, local_group=None,
                  pageable_host=False, two_step=0, stream_through=0, peer_transport=False):
         self._h = None
+        self._inflight = []  # kernel descriptors (user functions) of unsynchronised runs
         self.dims = tuple(int(v) for v in dims)
         self.tile_dims = tuple(int(v) for v in tile_dims)
         self.bc = BCS[bc] if isinstance(bc, str) else int(bc)
@@ -272,6 +273,7 @@ class Domain:
         if self._h is not None:
             h, self._h = self._h, None
             _check(tile_free(h), "tile_free")
+            self._inflight.clear()
 
     def __del__(self):
         try:
@@ -296,6 +298,7 @@ class Domain:
         if a.shape != self._shape():
             raise ValueError(f"expected shape {self._shape()}, got {a.shape}")
         _check(tile_load(self._h, a.ctypes.data), "tile_load")
+        self._inflight.clear()
 
     def store(self, out=None):
         if out is None:
@@ -303,6 +306,7 @@ class Domain:
         if out.shape != self._shape() or out.dtype != np.float64 or not out.flags.c_contiguous:
             raise ValueError("bad output array")
         _check(tile_store(self._h, out.ctypes.data), "tile_store")
+        self._inflight.clear()
         return out
 
     def host_tile(self, tile_id):
@@ -319,12 +323,19 @@ class Domain:
     # -- execution --------------------------------------------------------
     def run(self, kernel, steps, nstreams=4):
         _check(tile_run(self._h, ctypes.byref(kernel), steps, nstreams), "tile_run")
+        # a user function's module must outlive the launches queued with it
+        # (tiles.h: free it only after tile_sync): keep the descriptor until
+        # the next call that synchronises
+        if getattr(kernel, "_fn", None) is not None:
+            self._inflight.append(kernel)
 
     def sync(self):
         _check(tile_sync(self._h), "tile_sync")
+        self._inflight.clear()
 
     def invalidate(self):
         _check(tile_invalidate(self._h), "tile_invalidate")
+        self._inflight.clear()
 
     def set_measure(self, mode):
         _check(tile_set_measure(self._h, mode), "tile_set_measure")

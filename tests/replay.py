@@ -444,12 +444,17 @@ class Replayer:
         pos = {s: 0 for s in queues}
         done = set()
         remaining = len(trace)
+        syncs = [i for i, op in enumerate(trace) if op[0] == "sync"]
         while remaining:
             ready = []
+            # host sync (TILE_OP_SYNC): a barrier over every stream
+            barrier = next((i for i in syncs if i not in done), len(trace))
             for s, q in queues.items():
                 if pos[s] < len(q):
                     i = q[pos[s]]
                     op = trace[i]
+                    if i > barrier or (i == barrier and len(done) < barrier):
+                        continue
                     if op[0] == "wait" and bound[i] is not None and bound[i] not in done:
                         continue
                     if op[0] == "st_halo" and st_ready is not None and not st_ready(self, op):
@@ -464,6 +469,9 @@ class Replayer:
             i = queues[s][pos[s]]
             if trace[i][0] == "st_halo" and st_exec is not None:
                 st_exec(self, trace[i])
+            elif trace[i][0] == "sync":  # host-side face extraction reads the store now
+                snapshot = {(k, f): p for k in range(self.G.ntiles)
+                            for f, p in enumerate(faces_of(self.host[k], self.G.depth))}
             else:
                 self.execute(trace[i], snapshot)
             done.add(i)
@@ -530,16 +538,19 @@ def replay_ranks(reps, traces, seed, lazy=()):
         snapshot = {(k, f): p for k in range(rep.G.ntiles)
                     for f, p in enumerate(faces_of(rep.host[k], rep.G.depth))}
         state.append({"bound": bound, "queues": queues, "pos": {s: 0 for s in queues}, "done": set(),
-                      "snap": snapshot})
+                      "snap": snapshot, "syncs": [i for i, op in enumerate(tr) if op[0] == "sync"]})
     remaining = sum(len(t) for t in traces)
     while remaining:
         ready, halo_heads = [], {}
         for r, (st, tr) in enumerate(zip(state, traces)):
+            barrier = next((i for i in st["syncs"] if i not in st["done"]), len(tr))
             for s, q in st["queues"].items():
                 if st["pos"][s] >= len(q):
                     continue
                 i = q[st["pos"][s]]
                 op = tr[i]
+                if i > barrier or (i == barrier and len(st["done"]) < barrier):
+                    continue
                 if op[0] == "wait" and st["bound"][i] is not None and st["bound"][i] not in st["done"]:
                     continue
                 if op[0] in ("halo", "halo_signal"):
@@ -595,6 +606,10 @@ def replay_ranks(reps, traces, seed, lazy=()):
             elif a == 2:  # released: its sender may overwrite it from now on
                 reps[r].st[side] = np.full_like(reps[r].st[side], np.nan)
                 peer.st_credit[1 - side] = e
+        elif op[0] == "sync":
+            rp = reps[r]
+            state[r]["snap"] = {(k, f): p for k in range(rp.G.ntiles)
+                                for f, p in enumerate(faces_of(rp.host[k], rp.G.depth))}
         else:
             reps[r].execute(op, state[r]["snap"])
         state[r]["done"].add(i)

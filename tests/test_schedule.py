@@ -388,13 +388,16 @@ def _trace_through_state_machine(trace, nslots):
             got = [e for e in ro.trace[n0:] if e[0] != "compute"]
             assert got == pending, (name, a, b, c, got, pending)
             pending, last, nreq = [], a, nreq + 1
+        elif name == "sync":  # host sync: D2Hs queued since the last kernel were host requests
+            for pn, pa, pb in pending:
+                assert pn == "d2h", (pn, pa, pb)
+                n0 = len(ro.trace)
+                ro.cpu_request(pa)
+                assert ro.trace[n0:] == [("d2h", pa, pb)]
+            pending, last = [], None
         else:
             assert name in ("record", "wait", "faces_h2d", "halo"), name
-    for name, a, b in pending:  # tile_sync's flush: GPU-disabled requests
-        assert name == "d2h", (name, a, b)
-        n0 = len(ro.trace)
-        ro.cpu_request(a)
-        assert ro.trace[n0:] == [("d2h", a, b)]
+    assert not pending, pending
     assert not any(ro.dirty), "tile_sync left device-only data"
     return ro, nreq
 
@@ -451,3 +454,33 @@ def test_state_machine_check_catches_a_wrong_trace():
     bad[j] = ("hit",) + tuple(bad[j][1:])
     with pytest.raises((AssertionError, ValueError)):
         _trace_through_state_machine(bad, 3)
+
+
+@pytest.mark.parametrize("first", ["sincos", "heat"])
+@pytest.mark.parametrize("nslots", [3, 24])
+def test_stream_pointwise_then_heat_without_sync(first, nslots):
+    """Out-of-core runs of different kernels back to back with no tile_sync
+    between them: a heat run after a pointwise run needs its ghost faces from
+    the pointwise run's results — including the tiles still dirty on the
+    device and the write-backs still in flight — and a heat -> sincos ->
+    heat sequence must not reuse faces extracted before the sincos run."""
+    dims, td = (32, 16, 24), (8, 8, 4)
+    kw = dict(sched="stream", stream_through=-1, fuse_pointwise_steps=False)
+    b = _budget_for(dims, td, nslots, **kw)
+    u0 = synth.uniform_grid(*dims, 42)
+    runs = [("sincos", 1, 1), ("heat", 2, 0)] if first == "sincos" else \
+        [("heat", 1, 0), ("sincos", 1, 1), ("heat", 2, 0)]
+    ref = u0.copy()
+    for kind, steps, K in runs:
+        ref = oracle.sincos_c(ref, K, steps) if kind == "sincos" else oracle.heat_c(ref, ALPHA, steps)
+    for seed in (0, 1, 2):
+        d = T.Domain(dims, td, dry_run=True, device_budget_bytes=b, **kw)
+        d.load(u0)
+        for kind, steps, K in runs:
+            d.run(T.sincos(K) if kind == "sincos" else T.heat7(ALPHA), steps, 2)
+        d.sync()
+        G = Geometry(dims, td)
+        rep = Replayer(G, split_tiles(G, u0), ALPHA)
+        rep.replay(d.trace(), seed)
+        assert np.array_equal(rep.grid(), ref), np.abs(rep.grid() - ref).max()
+        _trace_through_state_machine(d.trace(), nslots)
