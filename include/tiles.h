@@ -18,6 +18,11 @@
  *  - TILE_EINVAL never has side effects.
  *  - A CUDA or NCCL failure (TILE_ECUDA / TILE_ENCCL) POISONS the domain:
  *    every later call except tile_free returns TILE_ESTATE.
+ *  - Tests force these paths with TILES_FAULT=<kind>:<n> (kind = h2d, d2h,
+ *    kernel, sync or host_alloc): the n-th such operation of a domain fails
+ *    through the executor's real error path (on a GPU an invalid copy is
+ *    queued, so the CUDA runtime reports the error; host_alloc requests an
+ *    impossible pinned size). Unset, it costs one integer compare.
  *  - A domain is used from one host thread at a time.
  *  - Grids are fp64, C order [z][y][x] with x fastest. Sizes are int64.
  *  - Ownership: the library owns every pinned host buffer and device buffer

@@ -131,7 +131,7 @@ tile_status tile_invalidate(tile_domain* h) {
 }
 
 tile_status tile_ghost_map(const tile_domain* h, int64_t tile_id, int64_t* out, int64_t out_len) {
-  if (!h || !h->d) return fail(TILE_EINVAL, "null domain");
+  CHECK_DOM(h);
   const tiles::Geometry& G = h->d->G;
   if (!out || tile_id < 0 || tile_id >= G.ntiles) return fail(TILE_EINVAL, "bad tile id or out");
   const int64_t need = (G.t[0] + 2 * G.ghost) * (G.t[1] + 2 * G.ghost) * (G.t[2] + 2 * G.ghost);
@@ -141,7 +141,7 @@ tile_status tile_ghost_map(const tile_domain* h, int64_t tile_id, int64_t* out, 
 }
 
 tile_status tile_face_sources(const tile_domain* h, int64_t tile_id, int64_t out[12]) {
-  if (!h || !h->d) return fail(TILE_EINVAL, "null domain");
+  CHECK_DOM(h);
   if (!out || tile_id < 0 || tile_id >= h->d->G.ntiles) return fail(TILE_EINVAL, "bad tile id");
   for (int f = 0; f < 6; ++f) {
     tiles::FaceSrc s = tiles::face_source(h->d->G, tile_id, f);
@@ -152,7 +152,8 @@ tile_status tile_face_sources(const tile_domain* h, int64_t tile_id, int64_t out
 }
 
 tile_status tile_get_info(const tile_domain* h, tile_info* o) {
-  if (!h || !h->d || !o) return fail(TILE_EINVAL, "null argument");
+  CHECK_DOM(h);
+  if (!o) return fail(TILE_EINVAL, "null argument");
   const Domain& d = *h->d;
   std::memset(o, 0, sizeof *o);
   for (int a = 0; a < 3; ++a) {
@@ -176,13 +177,14 @@ tile_status tile_get_info(const tile_domain* h, tile_info* o) {
 }
 
 tile_status tile_get_stats(const tile_domain* h, tile_stats* o) {
-  if (!h || !h->d || !o) return fail(TILE_EINVAL, "null argument");
+  CHECK_DOM(h);
+  if (!o) return fail(TILE_EINVAL, "null argument");
   *o = h->d->stats;
   return TILE_OK;
 }
 
 tile_status tile_reset_stats(tile_domain* h) {
-  if (!h || !h->d) return fail(TILE_EINVAL, "null domain");
+  CHECK_DOM(h);
   h->d->stats = tile_stats{};
   return TILE_OK;
 }
@@ -215,7 +217,8 @@ tile_status tile_set_kernel_timing(tile_domain* h, int32_t on) {
 }
 
 tile_status tile_trace(const tile_domain* h, tile_op* out, int64_t cap, int64_t* n) {
-  if (!h || !h->d || !n) return fail(TILE_EINVAL, "null argument");
+  CHECK_DOM(h);
+  if (!n) return fail(TILE_EINVAL, "null argument");
   const auto& t = h->d->trace;
   *n = (int64_t)t.size();
   if (out && cap > 0) std::memcpy(out, t.data(), sizeof(tile_op) * (size_t)std::min<int64_t>(cap, *n));
@@ -223,7 +226,7 @@ tile_status tile_trace(const tile_domain* h, tile_op* out, int64_t cap, int64_t*
 }
 
 tile_status tile_trace_clear(tile_domain* h) {
-  if (!h || !h->d) return fail(TILE_EINVAL, "null domain");
+  CHECK_DOM(h);
   h->d->trace.clear();
   return TILE_OK;
 }
@@ -279,7 +282,8 @@ tile_status tile_nccl_unique_id(void* out128) {
 }
 
 tile_status tile_peer_handle(const tile_domain* h, void* out64) {
-  if (!h || !h->d || !out64) return fail(TILE_EINVAL, "null argument");
+  CHECK_DOM(h);
+  if (!out64) return fail(TILE_EINVAL, "null argument");
   return finish(nullptr, tiles::peer_handle(*h->d, out64));
 }
 

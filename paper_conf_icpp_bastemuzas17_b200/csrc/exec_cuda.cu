@@ -127,7 +127,21 @@ struct CudaExec final : Exec {
 
   cudaStream_t S(int i) { return streams[(size_t)i]; }
 
+  // TILES_FAULT: the n-th operation of a kind fails with a real CUDA error
+  // (an invalid copy queued on the same stream), reported through CK.
+  Status inject(Domain& d, int kind, int st) {
+    if (!fault_fires(d, kind)) return Status::ok();
+    CK(cudaMemcpyAsync(nullptr, nullptr, 8, cudaMemcpyDeviceToDevice, S(st < 0 ? 0 : st)));
+    return make_err(TILE_ECUDA, "injected fault did not fail");
+  }
+#define INJECT(kind, st)                 \
+  do {                                   \
+    Status f_ = inject(d, kind, st);     \
+    if (f_.bad()) return f_;             \
+  } while (0)
+
   Status h2d(Domain& d, int64_t t0, int64_t n, int s0, int st) override {
+    INJECT(FAULT_H2D, st);
     if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
     const size_t bytes = (size_t)n * d.G.tile_elems * 8;
     CK(cudaMemcpyAsync(d.slot_ptr(s0), d.host_tile(t0), bytes, cudaMemcpyHostToDevice, S(st)));
@@ -136,6 +150,7 @@ struct CudaExec final : Exec {
     return Status::ok();
   }
   Status d2h(Domain& d, int64_t t0, int64_t n, int s0, int st) override {
+    INJECT(FAULT_D2H, st);
     if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
     const size_t bytes = (size_t)n * d.G.tile_elems * 8;
     CK(cudaMemcpyAsync(d.host_tile(t0), d.slot_ptr(s0), bytes, cudaMemcpyDeviceToHost, S(st)));
@@ -153,6 +168,7 @@ struct CudaExec final : Exec {
   }
   Status heat(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
               const TileItem* dev_items, int st, int direct_bit, int nstack, int nsteps) override {
+    INJECT(FAULT_KERNEL, st);
     if (d.measure == TILE_MEASURE_XFER_ONLY || n == 0) return Status::ok();
     if (d.user_fn && userfn_is_stencil(d.user_fn)) {  // TILE_KERNEL_USER_STENCIL (face ghosts)
       double* fx[6];
@@ -351,6 +367,7 @@ struct CudaExec final : Exec {
     return v;
   }
   Status slab_sweep(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi, int st) override {
+    INJECT(FAULT_KERNEL, st);
     if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
     const SlabView s = slab_view(d, src, lo), t = slab_view(d, dst, lo);
     Status r = timed(d, st, [&] {
@@ -361,6 +378,7 @@ struct CudaExec final : Exec {
     return Status::ok();
   }
   Status h2d_part(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int st) override {
+    INJECT(FAULT_H2D, st);
     if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
     const size_t pl = (size_t)d.G.t[0] * d.G.t[1] * 8, tb = (size_t)d.G.tile_elems * 8;
     CK(cudaMemcpy2DAsync(reinterpret_cast<char*>(d.slot_ptr(s0)) + p0 * pl, tb,
@@ -371,6 +389,7 @@ struct CudaExec final : Exec {
     return Status::ok();
   }
   Status d2h_part(Domain& d, int64_t t0, int64_t n, int ps, int64_t p0, int64_t np, int st) override {
+    INJECT(FAULT_D2H, st);
     if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
     const size_t pl = (size_t)d.G.t[0] * d.G.t[1] * 8, tb = (size_t)d.G.tile_elems * 8;
     CK(cudaMemcpy2DAsync(reinterpret_cast<char*>(d.host_tile(t0)) + p0 * pl, tb, d.slot_ptr(ps),
@@ -380,6 +399,7 @@ struct CudaExec final : Exec {
     return Status::ok();
   }
   Status h2d_pack(Domain& d, int64_t t0, int64_t n, int ps, int64_t p0, int64_t np, int st) override {
+    INJECT(FAULT_H2D, st);
     if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
     const size_t pl = (size_t)d.G.t[0] * d.G.t[1] * 8, tb = (size_t)d.G.tile_elems * 8;
     CK(cudaMemcpy2DAsync(d.slot_ptr(ps), np * pl, reinterpret_cast<const char*>(d.host_tile(t0)) + p0 * pl,
@@ -404,6 +424,7 @@ struct CudaExec final : Exec {
   int heat2_occ = 0;
   Status heat2(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
                const TileItem* dev_items, int st) override {
+    INJECT(FAULT_KERNEL, st);
     if (d.measure == TILE_MEASURE_XFER_ONLY || n == 0) return Status::ok();
     Heat2Params P{};
     HeatParams& p = P.h;
@@ -443,6 +464,7 @@ struct CudaExec final : Exec {
     return Status::ok();
   }
   Status sincos(Domain& d, int64_t t, int slot, int64_t iters, int st) override {
+    INJECT(FAULT_KERNEL, st);
     if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
     if (d.user_fn) {  // TILE_KERNEL_USER: the caller's compiled pointwise function
       int64_t ix, iy, iz;
@@ -528,6 +550,7 @@ struct CudaExec final : Exec {
   }
   Status note(Domain&, int, int64_t, int64_t, int) override { return Status::ok(); }
   Status sync_all(Domain& d) override {
+    INJECT(FAULT_SYNC, 0);
     for (auto s : streams) CK(cudaStreamSynchronize(s));
     return collect(d);
   }
@@ -545,8 +568,10 @@ struct CudaExec final : Exec {
       std::memset(*p, 0, bytes);
       return Status::ok();
     }
-    // pinned (page-locked) host regions, P:L73 (cudaMallocHost)
-    cudaError_t e = cudaHostAlloc(p, bytes ? bytes : 1, cudaHostAllocPortable);
+    // pinned (page-locked) host regions, P:L73 (cudaMallocHost); an injected
+    // fault asks for more than any host has
+    const uint64_t req = fault_fires(d, FAULT_HOST_ALLOC) ? (1ull << 62) : (bytes ? bytes : 1);
+    cudaError_t e = cudaHostAlloc(p, req, cudaHostAllocPortable);
     if (e != cudaSuccess) {
       cudaGetLastError();
       return make_err(TILE_ENOMEM_HOST, std::string("cudaHostAlloc: ") + cudaGetErrorString(e));

@@ -10,6 +10,11 @@ namespace tiles {
 namespace {
 
 struct DryExec final : Exec {
+  // TILES_FAULT in a dry run: the failing operation reports TILE_ECUDA as
+  // the CUDA executor's would (nothing is recorded for it)
+  static Status inject(Domain& d, int kind) {
+    return fault_fires(d, kind) ? make_err(TILE_ECUDA, "injected fault (TILES_FAULT, dry run)") : Status::ok();
+  }
   void put(Domain& d, int kind, int stream, int64_t a, int64_t b, int64_t c, int64_t dd) {
     tile_op op;
     op.kind = kind;
@@ -21,12 +26,14 @@ struct DryExec final : Exec {
     d.trace.push_back(op);
   }
   Status h2d(Domain& d, int64_t t0, int64_t n, int s0, int st) override {
+    if (Status f_ = inject(d, FAULT_H2D); f_.bad()) return f_;
     d.stats.bytes_h2d += (uint64_t)n * d.G.tile_elems * 8;
     d.stats.n_h2d++;
     put(d, TILE_OP_H2D, st, t0, s0, n, 0);
     return Status::ok();
   }
   Status d2h(Domain& d, int64_t t0, int64_t n, int s0, int st) override {
+    if (Status f_ = inject(d, FAULT_D2H); f_.bad()) return f_;
     d.stats.bytes_d2h += (uint64_t)n * d.G.tile_elems * 8;
     d.stats.n_d2h++;
     put(d, TILE_OP_D2H, st, t0, s0, n, 0);
@@ -42,6 +49,7 @@ struct DryExec final : Exec {
   }
   Status heat(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
               const TileItem* dev_items, int st, int direct_bit, int nstack, int nsteps) override {
+    if (Status f_ = inject(d, FAULT_KERNEL); f_.bad()) return f_;
     if (nsteps > 1) {  // a persistent launch: the same ops as nsteps single steps
       const int64_t off = dev_items - d.items_dev[direct_bit];
       for (int s = 0; s < nsteps; ++s) {
@@ -74,12 +82,14 @@ struct DryExec final : Exec {
   }
   Status heat2(Domain& d, const int64_t* tiles, const int* in, const int* out, int n, int rp,
                const TileItem* dev_items, int st) override {
+    if (Status f_ = inject(d, FAULT_KERNEL); f_.bad()) return f_;
     const size_t mark = d.trace.size();
     Status r = heat(d, tiles, in, out, n, rp, dev_items, st, -1, 1, 1);
     for (size_t i = mark; i < d.trace.size(); ++i) d.trace[i].kind = TILE_OP_KERNEL2;
     return r;
   }
   Status slab_sweep(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi, int st) override {
+    if (Status f_ = inject(d, FAULT_KERNEL); f_.bad()) return f_;
     d.stats.n_kernels++;
     if (src.kind == SlabRef::UNITS) {
       // a: destination code as below; b: unit slots (u-1, u, u+1) packed 21
@@ -99,18 +109,21 @@ struct DryExec final : Exec {
     return Status::ok();
   }
   Status h2d_pack(Domain& d, int64_t t0, int64_t n, int ps, int64_t p0, int64_t np, int st) override {
+    if (Status f_ = inject(d, FAULT_H2D); f_.bad()) return f_;
     d.stats.bytes_h2d += (uint64_t)n * np * d.G.t[0] * d.G.t[1] * 8;
     d.stats.n_h2d++;
     put(d, TILE_OP_H2D_PACK, st, t0, ps, n, p0 | (np << 32));
     return Status::ok();
   }
   Status h2d_part(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int st) override {
+    if (Status f_ = inject(d, FAULT_H2D); f_.bad()) return f_;
     d.stats.bytes_h2d += (uint64_t)n * np * d.G.t[0] * d.G.t[1] * 8;
     d.stats.n_h2d++;
     put(d, TILE_OP_H2D_PART, st, t0, s0, n, p0 | (np << 32));
     return Status::ok();
   }
   Status d2h_part(Domain& d, int64_t t0, int64_t n, int ps, int64_t p0, int64_t np, int st) override {
+    if (Status f_ = inject(d, FAULT_D2H); f_.bad()) return f_;
     d.stats.bytes_d2h += (uint64_t)n * np * d.G.t[0] * d.G.t[1] * 8;
     d.stats.n_d2h++;
     put(d, TILE_OP_D2H_PART, st, t0, ps, n, p0 | (np << 32));
@@ -125,6 +138,7 @@ struct DryExec final : Exec {
     return Status::ok();
   }
   Status sincos(Domain& d, int64_t t, int slot, int64_t iters, int st) override {
+    if (Status f_ = inject(d, FAULT_KERNEL); f_.bad()) return f_;
     d.stats.n_kernels++;
     put(d, TILE_OP_POINTWISE, st, t, slot, iters, 0);
     return Status::ok();
@@ -159,6 +173,7 @@ struct DryExec final : Exec {
     return Status::ok();
   }
   Status sync_all(Domain& d) override {
+    if (Status f_ = inject(d, FAULT_SYNC); f_.bad()) return f_;
     put(d, TILE_OP_SYNC, -1, 0, 0, 0, 0);
     return Status::ok();
   }
@@ -168,7 +183,8 @@ struct DryExec final : Exec {
     *fr = d.opt.device_budget_bytes ? d.opt.device_budget_bytes + (1ull << 30) : (64ull << 30);
     return Status::ok();
   }
-  Status alloc_host(Domain&, uint64_t bytes, void** p) override {
+  Status alloc_host(Domain& d, uint64_t bytes, void** p) override {
+    if (fault_fires(d, FAULT_HOST_ALLOC)) return make_err(TILE_ENOMEM_HOST, "host allocation failed (injected)");
     *p = std::malloc(bytes ? bytes : 1);
     if (!*p) return make_err(TILE_ENOMEM_HOST, "host allocation failed");
     return Status::ok();

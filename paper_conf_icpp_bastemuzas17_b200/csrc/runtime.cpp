@@ -99,6 +99,7 @@ Status domain_create(const int64_t dims[3], const int64_t tdims[3], int ghost,
   d->stages = stages;
   d->heat_smem = smem;
   if (const char* cf = std::getenv("TILES_HEAT_CACHE")) d->heat_cache_flags = std::atoi(cf);
+  d->fault = parse_fault_env();
   if (opt.dry_run) {
     d->exec = make_dry_exec();
   } else {
@@ -115,6 +116,30 @@ Status domain_create(const int64_t dims[3], const int64_t tdims[3], int ghost,
   }
   *out = d;
   return Status::ok();
+}
+
+Fault parse_fault_env() {
+  Fault f;
+  const char* e = std::getenv("TILES_FAULT");
+  if (!e || !*e) return f;
+  static const struct { const char* name; int kind; } kinds[] = {
+      {"h2d", FAULT_H2D}, {"d2h", FAULT_D2H}, {"kernel", FAULT_KERNEL}, {"sync", FAULT_SYNC},
+      {"host_alloc", FAULT_HOST_ALLOC}};
+  const char* colon = std::strchr(e, ':');
+  const size_t len = colon ? (size_t)(colon - e) : std::strlen(e);
+  for (auto& k : kinds)
+    if (std::strlen(k.name) == len && std::strncmp(e, k.name, len) == 0) {
+      f.kind = k.kind;
+      f.left = colon ? std::max<int64_t>(1, std::atoll(colon + 1)) - 1 : 0;
+    }
+  return f;
+}
+
+bool fault_fires(Domain& d, int kind) {
+  if (d.fault.kind != kind) return false;
+  if (d.fault.left-- > 0) return false;
+  d.fault.kind = FAULT_NONE;  // fires once
+  return true;
 }
 
 // Memory plan ("calculates how many regions can fit into device

@@ -165,9 +165,21 @@ struct Exec {
 enum Mode : int { MODE_RESIDENT = 1, MODE_STREAM = 2 };
 constexpr int kMaxProgCtas = 2048;  // progress counters of a persistent multi-step launch
 
+// Fault injection for tests of the error contract (tiles.h conventions):
+// TILES_FAULT=<kind>:<n> makes the n-th operation of that kind (counted
+// from tile_domain_create) fail through the executor's real error path.
+enum FaultKind { FAULT_NONE = 0, FAULT_H2D, FAULT_D2H, FAULT_KERNEL, FAULT_SYNC, FAULT_HOST_ALLOC };
+struct Fault {
+  int kind = FAULT_NONE;
+  int64_t left = 0;  // operations of `kind` still to pass before the failing one
+};
+Fault parse_fault_env();
+bool fault_fires(Domain& d, int kind);  // true once, at the n-th call of `kind`
+
 struct Domain {
   Geometry G;
   tile_options opt;
+  Fault fault;
   bool poisoned = false;
   int device = 0;
   int mode = MODE_RESIDENT;
