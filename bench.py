@@ -1,22 +1,30 @@
 """Benchmark of the tiled heat path.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl tiles|reference]
-                    [--config c2|c1|c4] [--T STEPS] [--nstreams S]
+                    [--config c2|c1|c3|c4|c5|fig5|fig5tiles|fig8] [--T STEPS] [--nstreams S]
 
 One bench "step" = one pass of the whole hot path over one batch of input:
 T heat steps over every tile of the workload (C2 by default: 512^3 fp64,
-8^3 tiles of 64^3, ghost 1, 4 streams, T = 10, periodic, alpha = 0.125).
+8^3 tiles of 64^3, ghost 1, 4 streams, T = 10, periodic, alpha = 0.125),
+with every cell's H2D and D2H inside the step.
 
-  value  Gcell-updates/s with the grid already resident in HBM (tile_run of T
-         steps; ghost fill fused into the stencil).
-  e2e    the same metric through the public C API from pinned host memory:
-         tile_invalidate -> tile_run(T) -> tile_sync, i.e. H2D of every tile,
-         T steps, D2H of every tile inside the timed region.
+  value  the metric as BASELINE.json defines it: Gcell-updates/s INCLUDING
+         H2D/D2H, through the public C API from the library's pinned host
+         store: tile_invalidate -> tile_run(T) -> tile_sync (H2D of every
+         tile, T steps, D2H of every tile inside the timed region). `e2e`
+         repeats this measurement with its byte counts.
+  resident  the same T steps with the grid already resident in HBM (the
+         kernel-level rate; its roofline is the heat7 kernel's).
+  roofline  the dominant kernel of the timed step (the stream-through sweep
+         at T <= 16; heat7 when the batched schedule runs), achieved HBM
+         bytes from per-launch CUDA events on the launching streams.
 
 Timing: CUDA events recorded by libtiles on its own streams (tile_timer_*),
 barrier + synchronize on both sides, max over ranks. Inputs (2 x 1.07 GB per
-GPU) are larger than the 126 MB L2. N > 1: weak scaling, each rank owns a
-512^3 z-slab of a 512 x 512 x 512N grid, halos over NCCL.
+GPU) are larger than the 126 MB L2. N > 1: one process per GPU (bench.py
+re-launches itself under torch.distributed.run when WORLD_SIZE is unset),
+weak scaling, each rank owns a 512^3 z-slab of a 512 x 512 x 512N grid,
+halos over CUDA IPC peer memory (default) or NCCL.
 """
 import argparse
 import json
@@ -205,37 +213,143 @@ def traffic_from_profile(cfg):
     return None
 
 
-def cpu_oracle_time(n, T):
+def traffic_per_cell(kernel):
+    """ncu DRAM bytes per swept cell of `kernel` from a committed capture
+    (profiles/<kernel>_ncu_traffic.json), with its source; None if absent."""
+    p = os.path.join(ROOT, "profiles", f"{kernel}_ncu_traffic.json")
+    if os.path.exists(p):
+        j = json.load(open(p))
+        return j["dram_bytes_per_cell"], j.get("source", p)
+    return None
+
+
+def host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+def cpu_oracle_time(n, T, threads=1):
+    """Seconds for T untiled oracle steps on an n^3 sample (the C oracle;
+    threads > 1: its bit-identical OpenMP twin)."""
     import oracle
     import synth
     u = np.empty((n, n, n))
     synth.fill_uniform_native(u.ctypes.data, n, n, n, 0, n, 0, n, 0, n, 42)
     t0 = time.perf_counter()
-    oracle.heat_c(u, ALPHA, T)
+    oracle.heat_c(u, ALPHA, T, threads=threads)
     return time.perf_counter() - t0
 
 
+def cpu_baseline(T, n1=384, nall=512):
+    """The oracle on the host cores: 1 thread on an n1^3 sample and all cores
+    (OpenMP twin) on an nall^3 sample, T steps each (~10-20 s together)."""
+    cores = host_cores()
+    t1 = cpu_oracle_time(n1, T, 1)
+    ta = cpu_oracle_time(nall, T, cores)
+    v1, va = n1 ** 3 * T / t1 / 1e9, nall ** 3 * T / ta / 1e9
+    return {"value": va, "unit": "Gcell-updates/s", "cores": cores, "kind": "oracle",
+            "sample": f"{nall}^3 grid x T={T} on {cores} threads (oracle/heat_oracle.c OpenMP twin, "
+                      f"bit-identical); 1 thread: {n1}^3 x T={T}",
+            "by_cores": {"1": v1, str(cores): va}}
+
+
 def run_reference(args):
-    """--impl reference: the CPU oracle as it stands, 1 host core."""
+    """--impl reference: the CPU oracle as it stands on the host's cores (the
+    OpenMP twin of the untiled C oracle, bit-identical to it), one bounded
+    sample of the workload per step. Under torchrun only rank 0 runs."""
     ws, rk, _ = dist_env()
     if rk != 0:
         return 0
-    dims, td, T, ns, desc = CONFIGS[args.config]
-    n = 192 if args.config == "c2" else dims[0]   # bounded sample per step
+    dims, td, T, ns, desc = CONFIGS.get(args.config, CONFIGS["c2"])
+    cores = host_cores()
+    n = 320 if args.config != "c1" else dims[0]   # bounded sample per step
     for _ in range(args.warmup):
-        cpu_oracle_time(n, T)
-    t = sum(cpu_oracle_time(n, T) for _ in range(args.steps))
+        cpu_oracle_time(n, T, cores)
+    t = sum(cpu_oracle_time(n, T, cores) for _ in range(args.steps))
     val = n ** 3 * T * args.steps / t / 1e9
-    sample = f"{n}^3 grid x T={T} per step (untiled fp64 Jacobi, oracle/heat_oracle.c, 1 thread)"
+    sample = f"{n}^3 grid x T={T} per step (untiled fp64 Jacobi, oracle/heat_oracle.c OpenMP twin, {cores} threads)"
     line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "Gcell-updates/s", "n_gpus": ws,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": t / args.steps * 1e3,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic", "config": {"workload": desc, "sample": sample},
-            "cpu_baseline": {"value": val, "unit": "Gcell-updates/s", "cores": 1, "kind": "oracle",
+            "cpu_baseline": {"value": val, "unit": "Gcell-updates/s", "cores": cores, "kind": "oracle",
                              "sample": sample},
             "e2e": {"value": val, "unit": "Gcell-updates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
+
+
+# ---------------------------------------------------------------- CUPTI
+def _union(iv):
+    out = []
+    for a, b in sorted(iv):
+        if out and a <= out[-1][1]:
+            out[-1][1] = max(out[-1][1], b)
+        else:
+            out.append([a, b])
+    return out
+
+
+def _inter(a, b):
+    i = j = 0
+    tot = 0.0
+    while i < len(a) and j < len(b):
+        lo, hi = max(a[i][0], b[j][0]), min(a[i][1], b[j][1])
+        if hi > lo:
+            tot += hi - lo
+        if a[i][1] < b[j][1]:
+            i += 1
+        else:
+            j += 1
+    return tot
+
+
+def cupti_overlap(torch, fn):
+    """Run fn() once under torch.profiler (CUPTI activity records of every
+    kernel and memcpy in the process, libtiles' included) and return the
+    interval statistics: busy times, Σ(copy ∩ kernel) / min(Σcopy, Σkernel)
+    (SURVEY §8(d) cross-check of the overlap metric) and H2D ∥ D2H."""
+    import tempfile
+    from torch.profiler import ProfilerActivity, profile
+    torch.cuda.synchronize()
+    with profile(activities=[ProfilerActivity.CUDA]) as prof:
+        fn()
+        torch.cuda.synchronize()
+    with tempfile.NamedTemporaryFile(suffix=".json", delete=False) as f:
+        path = f.name
+    try:
+        prof.export_chrome_trace(path)
+        ev = json.load(open(path))["traceEvents"]
+    finally:
+        os.unlink(path)
+    ker, h2d, d2h = [], [], []
+    for e in ev:
+        if e.get("ph") != "X" or "dur" not in e:
+            continue
+        iv = (e["ts"], e["ts"] + e["dur"])
+        cat, name = e.get("cat", ""), e.get("name", "")
+        if cat == "kernel":
+            ker.append(iv)
+        elif cat in ("gpu_memcpy", "memcpy") or "Memcpy" in name:
+            if "HtoD" in name:
+                h2d.append(iv)
+            elif "DtoH" in name:
+                d2h.append(iv)
+    if not ker or not (h2d or d2h):
+        return None
+    K, H, D = _union(ker), _union(h2d), _union(d2h)
+    X = _union(h2d + d2h)
+    busy = lambda s_: sum(b - a for a, b in s_)
+    allv = ker + h2d + d2h
+    span = max(x[1] for x in allv) - min(x[0] for x in allv)
+    return {"span_ms": span / 1e3, "kernel_busy_ms": busy(K) / 1e3, "h2d_busy_ms": busy(H) / 1e3,
+            "d2h_busy_ms": busy(D) / 1e3, "copy_busy_ms": busy(X) / 1e3,
+            "copy_and_kernel_ms": _inter(X, K) / 1e3, "h2d_and_d2h_ms": _inter(H, D) / 1e3,
+            "hidden_frac": _inter(X, K) / max(1e-9, min(busy(X), busy(K))),
+            "n_kernels": len(ker), "n_h2d": len(h2d), "n_d2h": len(d2h),
+            "definition": "CUPTI activity intervals: sum(copy ∩ kernel) / min(sum copy, sum kernel)"}
 
 
 def fill_tiles(dom, Tl, synth, gdims, td, z_base, seed):
@@ -250,7 +364,7 @@ def fill_tiles(dom, Tl, synth, gdims, td, z_base, seed):
     dom.mark_host_dirty()
 
 
-def run_stream_leg(args):
+def c3_line(args):
     """C3: heat 2048^3 fp64 out-of-core: the device budget is CAPPED (the
     paper's "limiting GPU memory" method) so only a fraction of the
     tiles fits; every step streams the tiles through the slot pool.
@@ -304,9 +418,9 @@ def run_stream_leg(args):
             t += dom.timer_stop()
         dom.set_measure(Tl.TILE_MEASURE_NORMAL)
         return t / steps
-    xo, co = leg(Tl.TILE_MEASURE_XFER_ONLY), leg(Tl.TILE_MEASURE_COMP_ONLY)
+    xo, co = leg(Tl.TILE_MEASURE_XFER_ONLY, args.steps), leg(Tl.TILE_MEASURE_COMP_ONLY, args.steps)
     wall = tot / args.steps
-    hidden = max(0.0, min(1.0, (xo + co - wall) / min(xo, co)))
+    hidden = (xo + co - wall) / min(xo, co)   # unclamped; same repetitions as the wall time
     dom.free()
     bw = pcie_bandwidth(torch)
     bidir = pcie_bidir(torch)
@@ -329,14 +443,14 @@ def run_stream_leg(args):
                     "d2h_bytes_per_step": int(Bd), "ms_per_step": wall},
             "gpu_launches": st["n_kernels"] // max(1, args.steps),
             "residency": {k2: st[k2] // args.steps for k2 in ("hits", "misses", "evictions", "writebacks")},
-            "overlap": {"hidden_frac": hidden, "t_wall_ms": wall, "t_xfer_only_ms": xo, "t_comp_only_ms": co},
+            "overlap": {"hidden_frac": hidden, "t_wall_ms": wall, "t_xfer_only_ms": xo, "t_comp_only_ms": co,
+                        "reps": args.steps},
             "roofline": {"bound": "pcie", "form": "streaming: max(Bh/BWh, Bd/BWd, (Bh+Bd)/BWbidir)",
                          "t_link_ms": t_link * 1e3, "frac": t_link * 1e3 / wall,
                          "achieved": (Bh + Bd) / (wall / 1e3) / 1e9, "peak": bidir, "unit": "GB/s",
                          "pcie_gbs": {**bw, "bidir": bidir}},
             "clocks": clk.summary()}
-    print(json.dumps(line), flush=True)
-    return 0
+    return line
 
 
 def pcie_bidir(torch, nbytes=1 << 30, reps=6, warm=2):
@@ -368,7 +482,7 @@ def pcie_bidir(torch, nbytes=1 << 30, reps=6, warm=2):
     return best
 
 
-def run_sincos_leg(args):
+def c4_line(args):
     """C4: the compute-intensive kernel at 1024^3 fp64, 8^3
     tiles of 128^3, K = 32 inner iterations (reading R12), T = 10 outer steps
     fused per residency pass; nstreams sweep 1..8 (e2e from pinned host)."""
@@ -415,18 +529,20 @@ def run_sincos_leg(args):
     st = dom.stats()
     dom.set_kernel_timing(False)
     dom.sync()
-    def leg(mode):
+    def leg(mode, reps):
         dom.set_measure(mode)
-        dom.invalidate()
-        dom.timer_start()
-        dom.run(k, T, ns)
-        dom.sync()
-        t = dom.timer_stop()
+        t = 0.0
+        for _ in range(reps):
+            dom.invalidate()
+            dom.timer_start()
+            dom.run(k, T, ns)
+            dom.sync()
+            t += dom.timer_stop()
         dom.set_measure(Tl.TILE_MEASURE_NORMAL)
-        return t
-    xo, co = leg(Tl.TILE_MEASURE_XFER_ONLY), leg(Tl.TILE_MEASURE_COMP_ONLY)
-    wall = cells * T / (sweep[ns] * 1e9) * 1e3 if ns in sweep else None
-    hidden = max(0.0, min(1.0, (xo + co - wall) / min(xo, co))) if wall else None
+        return t / reps
+    wall = leg(Tl.TILE_MEASURE_NORMAL, args.steps)
+    xo, co = leg(Tl.TILE_MEASURE_XFER_ONLY, args.steps), leg(Tl.TILE_MEASURE_COMP_ONLY, args.steps)
+    hidden = (xo + co - wall) / min(xo, co)   # unclamped, equal repetitions
     dom.free()
     value = cells * T * args.steps / (ms_res / 1e3) / 1e9
     # achieved over the resident wall time (per-launch event durations of
@@ -448,10 +564,10 @@ def run_sincos_leg(args):
             "e2e": {"value": sweep.get(ns), "unit": "Gcell-steps/s", "h2d_bytes_per_step": cells * 8,
                     "d2h_bytes_per_step": cells * 8},
             "stream_sweep_e2e": sweep, "best_nstreams": ns_best,
-            "overlap": {"hidden_frac": hidden, "t_wall_ms": wall, "t_xfer_only_ms": xo, "t_comp_only_ms": co},
+            "overlap": {"hidden_frac": hidden, "t_wall_ms": wall, "t_xfer_only_ms": xo, "t_comp_only_ms": co,
+                        "reps": args.steps},
             "gpu_launches": st["n_kernels"], "roofline": roof, "clocks": clk.summary()}
-    print(json.dumps(line), flush=True)
-    return 0
+    return line
 
 
 def budget_for_slots(Tl, dims, td, nslots, **kw):
@@ -772,6 +888,59 @@ def run_c5_leg(args):
     return 0
 
 
+
+# ------------------------------------------------------------ multi-process
+def free_port():
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        return so.getsockname()[1]
+
+
+def spawn_cmd(argv, n, port):
+    """One process per GPU on this node, the driver's own launch line."""
+    return [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+            "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *argv]
+
+
+def maybe_spawn(args, argv):
+    """--gpus N > 1 with no torchrun environment: re-launch this script under
+    torch.distributed.run (N ranks, 127.0.0.1) and return its exit code;
+    None when this process is already a rank (or N = 1)."""
+    if args.gpus <= 1 or "WORLD_SIZE" in os.environ:
+        return None
+    if not args.spawn_probe and not ONE_GPU:
+        import torch
+        have = torch.cuda.device_count()
+        if have < args.gpus:
+            print(f"bench.py: --gpus {args.gpus} but only {have} CUDA device(s) visible", file=sys.stderr)
+            return 2
+    return subprocess.call(spawn_cmd(argv, args.gpus, free_port()))
+
+
+def check_world(args):
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    if ws != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={ws}")
+    return ws
+
+
+def run_spawn_probe(args):
+    """--spawn-probe: the multi-process launch alone (CPU, gloo): every rank
+    reports itself, rank 0 prints the world it sees."""
+    import torch.distributed as dist
+    ws, rk, lr = dist_env()
+    got = [{"rank": rk, "local_rank": lr, "pid": os.getpid()}]
+    if ws > 1:
+        dist.init_process_group("gloo")
+        got = [None] * ws
+        dist.all_gather_object(got, {"rank": rk, "local_rank": lr, "pid": os.getpid()})
+        dist.destroy_process_group()
+    if rk == 0:
+        print(json.dumps({"spawn_probe": True, "world_size": ws, "ranks": got}), flush=True)
+    return 0
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -782,7 +951,8 @@ def main():
     ap.add_argument("--T", type=int, default=None)
     ap.add_argument("--nstreams", type=int, default=None)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--no-extras", action="store_true", help="skip sync-baseline / overlap legs")
+    ap.add_argument("--no-extras", action="store_true",
+                    help="skip the overlap / sync-baseline / CUPTI / C3 / C4 extras")
     ap.add_argument("--n", type=int, default=None, help="c3/c4: grid edge")
     ap.add_argument("--budget-gb", type=float, default=None, help="c3: device budget cap")
     ap.add_argument("--K", type=int, default=32, help="c4: kernel_iteration (reading R12)")
@@ -796,13 +966,23 @@ def main():
                          "(default), the same windows written by copies, or NCCL p2p")
     ap.add_argument("--stream-through", type=int, default=0,
                     help="tile_options.stream_through (-1 never, 0 cost model, 1 when feasible)")
-    args = ap.parse_args()
+    ap.add_argument("--spawn-probe", action="store_true", help="test hook: the N-process launch only")
+    argv = sys.argv[1:]
+    args = ap.parse_args(argv)
+    rc = maybe_spawn(args, argv)
+    if rc is not None:
+        return rc
+    check_world(args)
+    if args.spawn_probe:
+        return run_spawn_probe(args)
     if args.impl == "reference":
         return run_reference(args)
     if args.config == "c3":
-        return run_stream_leg(args)
+        print(json.dumps(c3_line(args)), flush=True)
+        return 0
     if args.config == "c4":
-        return run_sincos_leg(args)
+        print(json.dumps(c4_line(args)), flush=True)
+        return 0
     if args.config == "fig8":
         return run_fig8_leg(args)
     if args.config == "fig5":
@@ -811,6 +991,18 @@ def main():
         return run_fig5_tiles_leg(args)
     if args.config == "c5":
         return run_c5_leg(args)
+    return run_main_leg(args)
+
+
+SCHED_NAMES = {0: "none", 1: "resident batched (layer batches + whole-domain steps)",
+               2: "stream-through (fresh upload, T <= tz)", 3: "out-of-core per-tile stream",
+               4: "out-of-core stream-through", 5: "synchronous (one stream)", 6: "wavefront (fresh upload)"}
+SWEEP_KERNEL = {1: "heat7_fixed", 2: "slab_sweep_ca", 4: "slab_sweep_ca", 5: "heat7_fixed",
+                6: "wave_sweep"}
+
+
+def run_main_leg(args):
+    import argparse as _ap
 
     import torch
     import torch.distributed as dist
@@ -829,6 +1021,7 @@ def main():
     nx, ny, nzl = dims
     gdims = (nx, ny, nzl * ws)
     cells = nx * ny * nzl  # per rank
+    NORMAL = Tl.TILE_MEASURE_NORMAL
 
     def barrier():
         if ws > 1:
@@ -845,13 +1038,64 @@ def main():
     u0 = np.empty((nzl, ny, nx))
     synth.fill_uniform_native(u0.ctypes.data, gdims[0], gdims[1], gdims[2], rk * nzl, nzl, 0, ny, 0, nx, 42)
     dom = multi_domain(Tl, dist, ws, rk, args.transport, gdims, td, ghost=args.ghost, device=lr,
-                       two_step=args.two_step)
-    dom.load(u0)
+                       two_step=args.two_step, stream_through=args.stream_through)
+    t0 = time.perf_counter()
+    dom.load(u0)   # tile_load: dense slab -> tile-blocked pinned store (outside the timed region)
+    t_load_ms = (time.perf_counter() - t0) * 1e3
     del u0
     k = Tl.heat7(ALPHA)
     spp = dom.info["steps_per_pass"]
 
-    # ---- device-resident value -------------------------------------------
+    def e2e_steps(mode, reps, timing=False):
+        """reps bench steps: tile_invalidate (host store is the source) ->
+        tile_run(T) -> tile_sync (every tile back in the pinned store)."""
+        dom.set_measure(mode)
+        dom.set_kernel_timing(timing)
+        dom.reset_stats()
+        barrier()
+        tot = 0.0
+        for _ in range(reps):
+            dom.invalidate()
+            dom.timer_start()
+            dom.run(k, T, ns)
+            dom.sync()
+            tot += dom.timer_stop()
+        st_ = dom.stats()
+        dom.set_kernel_timing(False)
+        dom.set_measure(NORMAL)
+        return max_over_ranks(tot), st_
+
+    # ---- value: the metric, H2D and D2H of every cell inside the step --------
+    for _ in range(args.warmup):
+        dom.invalidate()
+        dom.run(k, T, ns)
+        dom.sync()
+    with Clocks(lr) as clk:
+        ms, st = e2e_steps(NORMAL, args.steps, timing=True)
+    value = ws * cells * T * args.steps / (ms / 1e3) / 1e9
+    sched = dom.get_info().get("last_schedule", 0)
+    h2d_b = st["bytes_h2d"] // args.steps
+    d2h_b = st["bytes_d2h"] // args.steps
+    peak, peak_src = measured_peaks()
+    sw_ms, sw_cells, sw_n = st["sweep_ms"], st["sweep_cells"], max(1, st["sweep_timed"])
+    achieved = 16.0 * sw_cells / (sw_ms / 1e3) / 1e9 if sw_ms > 0 else None
+    kname = SWEEP_KERNEL.get(sched, "stencil sweeps")
+    prof = traffic_per_cell(kname)
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+            "frac": achieved / peak if achieved else None,
+            "traffic": prof[0] * sw_cells / sw_n if prof else None,
+            "traffic_source": prof[1] if prof else None,
+            "kernel": kname, "schedule": SCHED_NAMES.get(sched, str(sched)),
+            "algorithmic_bytes_per_cell_sweep": 16.0,
+            "algorithmic_bytes_per_launch": 16.0 * sw_cells / sw_n,
+            "launches_per_step": sw_n / args.steps, "avg_launch_ms": sw_ms / sw_n,
+            "kernel_share_of_step": sw_ms / ms if ms > 0 else None,
+            "note": "achieved = 16 B x cells swept by the timed launches / their summed CUDA-event "
+                    "durations on the launching streams (concurrent launches overlap, so the share can "
+                    "exceed 1 only if they do); the e2e step itself is host-link-bound: see roofline_link",
+            "peak_source": peak_src}
+
+    # ---- the kernel-level rate: grid resident in HBM ------------------------
     dom.run(k, 1, ns)
     dom.sync()
     for _ in range(args.warmup):
@@ -860,54 +1104,54 @@ def main():
     dom.set_kernel_timing(True)
     dom.reset_stats()
     barrier()
-    with Clocks(lr) as clk:
+    with Clocks(lr) as clk_res:
         dom.timer_start()
         for _ in range(args.steps):
             dom.run(k, T, ns)
-        ms = dom.timer_stop()
-    st = dom.stats()
+        ms_res = dom.timer_stop()
+    st_res = dom.stats()
     dom.set_kernel_timing(False)
-    ms = max_over_ranks(ms)
-    value = ws * cells * T * args.steps / (ms / 1e3) / 1e9
-    launches = st["n_kernels"]
-    avg_kernel_ms = st["kernel_ms"] / max(1, st["kernel_timed"])
-    # cells swept per launch (a two-step pass sweeps the grid once for 2 steps)
-    cells_per_launch = cells * T * args.steps / spp / max(1, st["kernel_timed"])
+    ms_res = max_over_ranks(ms_res)
     dom.sync()
-
-    # ---- end-to-end from pinned host memory ---------------------------------
-    def e2e_leg(mode=Tl.TILE_MEASURE_NORMAL, steps=args.steps, warm=1):
-        dom.set_measure(mode)
-        for _ in range(warm):
-            dom.invalidate()
-            dom.run(k, T, ns)
-            dom.sync()
-        dom.reset_stats()
-        barrier()
-        tot = 0.0
-        for _ in range(steps):
-            dom.invalidate()
-            dom.timer_start()
-            dom.run(k, T, ns)
-            dom.sync()
-            tot += dom.timer_stop()
-        s = dom.stats()
-        dom.set_measure(Tl.TILE_MEASURE_NORMAL)
-        return max_over_ranks(tot), s
-
-    with Clocks(lr) as clk_e2e:
-        e2e_ms, st_e2e = e2e_leg()
-    e2e_val = ws * cells * T * args.steps / (e2e_ms / 1e3) / 1e9
-    h2d_b = st_e2e["bytes_h2d"] // args.steps
-    d2h_b = st_e2e["bytes_d2h"] // args.steps
+    res_value = ws * cells * T * args.steps / (ms_res / 1e3) / 1e9
+    rs_ms, rs_cells, rs_n = st_res["sweep_ms"], st_res["sweep_cells"], max(1, st_res["sweep_timed"])
+    r_ach = 16.0 * rs_cells / (rs_ms / 1e3) / 1e9 if rs_ms > 0 else None
+    tps = traffic_from_profile(args.config) if spp == 1 else None
+    steps_per_launch = rs_cells / rs_n / cells
+    resident = {"value": res_value, "unit": "Gcell-updates/s", "ms_per_step": ms_res / args.steps,
+                "def": "grid resident in HBM; tile_run(T) per step, no host transfers",
+                "gpu_launches": st_res["n_kernels"],
+                "roofline": {"bound": "hbm", "achieved": r_ach, "peak": peak, "unit": "GB/s",
+                             "frac": r_ach / peak if r_ach else None,
+                             "traffic": tps * steps_per_launch if tps else None, "traffic_per_step": tps,
+                             "kernel": "heat7_fixed" if spp == 1 else "heat7x2 (2 steps per pass)",
+                             "algorithmic_bytes_per_cell_update": 16.0 / spp,
+                             "algorithmic_bytes_per_launch": 16.0 * rs_cells / rs_n,
+                             "steps_per_launch": steps_per_launch * spp, "avg_launch_ms": rs_ms / rs_n,
+                             "peak_source": peak_src},
+                "clocks": clk_res.summary()}
 
     extras = {}
     if not args.no_extras:
-        xo_ms, _ = e2e_leg(Tl.TILE_MEASURE_XFER_ONLY, steps=2)
-        co_ms, _ = e2e_leg(Tl.TILE_MEASURE_COMP_ONLY, steps=2)
-        wall = e2e_ms / args.steps
-        xo, co = xo_ms / 2, co_ms / 2
-        hidden = max(0.0, min(1.0, (xo + co - wall) / min(xo, co)))
+        # overlap: the same schedule with kernels skipped / copies skipped,
+        # as many repetitions as the timed value leg, unclamped
+        xo_ms, _ = e2e_steps(Tl.TILE_MEASURE_XFER_ONLY, args.steps)
+        co_ms, _ = e2e_steps(Tl.TILE_MEASURE_COMP_ONLY, args.steps)
+        wall, xo, co = ms / args.steps, xo_ms / args.steps, co_ms / args.steps
+        hidden = (xo + co - wall) / min(xo, co)
+        ov = {"hidden_frac": hidden, "t_wall_ms": wall, "t_xfer_only_ms": xo, "t_comp_only_ms": co,
+              "reps": args.steps, "definition": "(T_xfer_only + T_comp_only - T_wall) / min(...), unclamped",
+              "note": "compute << transfer here, so this is the fraction of the kernel time hidden "
+                      "under transfers; > 1 means T_wall < T_xfer_only (the xfer-only schedule "
+                      "issues the same copies without the kernels' events, so it is not a strict bound)"}
+        try:
+            def one():
+                dom.invalidate()
+                dom.run(k, T, ns)
+                dom.sync()
+            ov["cupti"] = cupti_overlap(torch, one)
+        except Exception as e:  # profiler unavailable: say so
+            ov["cupti"] = {"error": str(e)[:200]}
         bw = pcie_bandwidth(torch)
         bidir = pcie_bidir(torch)
         B = cells * 8
@@ -915,16 +1159,14 @@ def main():
         # once each way; no schedule beats max(B/h2d, B/d2h, 2B/bidir)
         t_link = max(B / (bw["h2d"] * 1e9), B / (bw["d2h"] * 1e9), 2 * B / (bidir * 1e9))
         t_dep = B / (bw["h2d"] * 1e9) + B / (bw["d2h"] * 1e9)     # tile-granular dependency form
-        hbm_peak, _ = measured_peaks()
-        t_hbm = T * 16 * cells / (hbm_peak * 1e9)
+        t_hbm = T * 16 * cells / (peak * 1e9)
         R = max(t_link, t_hbm)
-        extras = {"overlap": {"hidden_frac": hidden, "t_wall_ms": wall, "t_xfer_only_ms": xo,
-                              "t_comp_only_ms": co,
-                              "definition": "(T_xfer_only + T_comp_only - T_wall) / min(...)"},
-                  "e2e_roofline": {"bound": "pcie (streaming/duplex form)", "t_link_ms": t_link * 1e3,
-                                   "t_link_dependency_form_ms": t_dep * 1e3,
-                                   "t_hbm_ms": t_hbm * 1e3, "frac": R / (wall / 1e3),
-                                   "pcie_gbs": {**bw, "bidir": bidir}}}
+        extras["overlap"] = ov
+        extras["roofline_link"] = {"bound": "pcie (streaming/duplex form: max(B/h2d, B/d2h, 2B/bidir))",
+                                   "t_bound_ms": R * 1e3, "t_link_ms": t_link * 1e3,
+                                   "t_link_dependency_form_ms": t_dep * 1e3, "t_hbm_ms": t_hbm * 1e3,
+                                   "frac": R / (wall / 1e3), "achieved_gbs": (h2d_b + d2h_b) / (wall / 1e3) / 1e9,
+                                   "peak_gbs": bidir, "pcie_gbs": {**bw, "bidir": bidir}}
         if ws == 1:
             dom.free()
             sdom = Tl.Domain(gdims, td, ghost=args.ghost, device=lr, sched="sync")
@@ -935,45 +1177,42 @@ def main():
             sdom.run(k, T, 1)
             sdom.sync()
             tot = 0.0
-            for _ in range(2):
+            reps = max(2, args.steps // 4)
+            for _ in range(reps):
                 sdom.invalidate()
                 sdom.timer_start()
                 sdom.run(k, T, 1)
                 sdom.sync()
                 tot += sdom.timer_stop()
             sdom.free()
-            extras["sync_baseline_e2e"] = {"value": cells * T * 2 / (tot / 1e3) / 1e9,
-                                           "unit": "Gcell-updates/s",
-                                           "schedule": "H2D all, T steps, D2H all, one stream"}
+            extras["sync_baseline_e2e"] = {"value": cells * T * reps / (tot / 1e3) / 1e9,
+                                           "unit": "Gcell-updates/s", "ms_per_step": tot / reps,
+                                           "schedule": "H2D all, T steps, D2H all, one stream (pinned)"}
     try:
         dom.free()
     except Exception:
         pass
 
-    peak, peak_src = measured_peaks()
-    algo_bytes = 16.0 * cells_per_launch
-    achieved = algo_bytes / (avg_kernel_ms / 1e3) / 1e9
-    # a persistent launch runs every step of a tile_run (steps_per_launch = T);
-    # the ncu capture is of one whole-domain step, so traffic scales by it
-    steps_per_launch = cells_per_launch / cells
-    tps = traffic_from_profile(args.config) if spp == 1 else None
-    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-            "traffic": tps * steps_per_launch if tps else None,
-            "traffic_per_step": tps,
-            "kernel": "heat7_fixed" if spp == 1 else "heat7x2 (2 steps per pass)",
-            "algorithmic_bytes_per_cell_update": 16.0 / spp,
-            "algorithmic_bytes_per_launch": algo_bytes, "steps_per_launch": steps_per_launch,
-            "avg_launch_ms": avg_kernel_ms, "peak_source": peak_src}
-
     cpu = None
     if rk == 0 and ws == 1 and not args.no_cpu_baseline:
-        n = 384 if args.config == "c2" else dims[0]
-        t = cpu_oracle_time(n, T)
-        cpu = {"value": n ** 3 * T / t / 1e9, "unit": "Gcell-updates/s", "cores": 1, "kind": "oracle",
-               "sample": f"{n}^3 grid x T={T} (untiled Jacobi, oracle/heat_oracle.c, 1 thread)"}
+        cpu = cpu_baseline(T, 384 if args.config == "c2" else dims[0], 512 if args.config == "c2" else dims[0])
+
+    if ws == 1 and not args.no_extras and args.config == "c2":
+        # the other BASELINE.json configs, driver-observed: C3 out of core
+        # (2048^3, capped budget) and C4 (the compute-intensive kernel)
+        for key, fn, kw in (("c3", c3_line, dict(n=None, T=None, nstreams=None, budget_gb=None, ghost=1,
+                                                  stream_through=0, steps=2, warmup=1)),
+                            ("c4", c4_line, dict(n=None, T=None, nstreams=None, K=args.K, sweep="1,2,4,8",
+                                                  steps=2, warmup=1))):
+            try:
+                ln = fn(_ap.Namespace(**kw))
+                extras[key] = {kk: ln[kk] for kk in ("value", "unit", "ms_per_step", "config", "e2e", "overlap",
+                                                      "roofline", "clocks", "stream_sweep_e2e")
+                               if kk in ln}
+            except Exception as e:  # e.g. not enough host RAM for C3's pinned store
+                extras[key] = {"error": str(e)[:300]}
 
     if rk == 0:
-        clocks = clk.summary()
         line = {"metric": METRIC, "value": value, "unit": "Gcell-updates/s", "n_gpus": ws,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
                 "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
@@ -981,15 +1220,19 @@ def main():
                 "config": {"workload": desc, "dims_per_gpu": dims, "global_dims": gdims, "tile_dims": td,
                            "ghost": args.ghost, "steps_per_pass": spp, "T": T, "nstreams": ns,
                            "bc": "periodic", "alpha": ALPHA,
-                           "parallelism": f"z-slab x{ws}, halo via {getattr(multi_domain, 'fallback', args.transport)}" if ws > 1 else "1 GPU",
-                           "host_cpus": numa,
+                           "parallelism": f"z-slab x{ws}, one process per GPU" if ws > 1 else "1 GPU",
+                           "transport": getattr(multi_domain, "fallback", args.transport) if ws > 1 else None,
+                           "comm_ranks": ws,
+                           "schedule": SCHED_NAMES.get(sched, str(sched)),
+                           "host_cpus": numa, "tile_load_ms": t_load_ms,
                            "l2": "inputs larger than L2 (2 x 1.07 GB per GPU per step)",
-                           "value_def": "grid resident in HBM; T steps of tile_run",
-                           "e2e_def": "tile_invalidate + tile_run(T) + tile_sync from pinned host"},
-                "e2e": {"value": e2e_val, "unit": "Gcell-updates/s", "h2d_bytes_per_step": h2d_b,
-                        "d2h_bytes_per_step": d2h_b, "ms_per_step": e2e_ms / args.steps},
-                "gpu_launches": launches, "roofline": roof, "cpu_baseline": cpu, "clocks": clocks,
-                "clocks_e2e": clk_e2e.summary()}
+                           "value_def": "the metric: tile_invalidate + tile_run(T) + tile_sync from the "
+                                        "pinned host store, H2D and D2H of every cell inside the timed step",
+                           "e2e_def": "same measurement as value (the metric includes H2D/D2H)"},
+                "e2e": {"value": value, "unit": "Gcell-updates/s", "h2d_bytes_per_step": h2d_b,
+                        "d2h_bytes_per_step": d2h_b, "ms_per_step": ms / args.steps},
+                "gpu_launches": st["n_kernels"], "roofline": roof, "resident": resident,
+                "cpu_baseline": cpu, "clocks": clk.summary()}
         line.update(extras)
         print(json.dumps(line), flush=True)
     if ws > 1:

@@ -179,6 +179,12 @@ typedef struct {
   double last_run_ms;                        /* host wall time of last tile_run..sync */
   double kernel_ms;                          /* summed device time of timed kernel launches */
   uint64_t kernel_timed;                     /* number of timed kernel launches */
+  double sweep_ms;                           /* the part of kernel_ms spent in stencil
+                                                sweeps (heat7, heat7x2, stream-through) */
+  uint64_t sweep_cells;                      /* cells those timed sweeps read and wrote
+                                                once each (16 B of algorithmic HBM traffic
+                                                per cell; a two-step pass counts once) */
+  uint64_t sweep_timed;                      /* number of timed sweep launches */
 } tile_stats;
 
 typedef struct {
@@ -197,7 +203,12 @@ typedef struct {
   int32_t steps_per_pass; /* HEAT7 steps per residency pass: 2 with ghost >= 2
                              (temporal blocking, single rank, supported tile
                              width), else 1 */
-  int32_t reserved;
+  int32_t last_schedule;  /* schedule the last tile_run took:
+                             0 none yet, 1 resident batched (layer batches /
+                             whole-domain steps), 2 stream-through (fresh
+                             upload), 3 out-of-core per-tile stream, 4
+                             out-of-core stream-through, 5 synchronous (one
+                             stream), 6 wavefront (fresh upload) */
 } tile_info;
 
 /* One entry of the dry-run trace. */

@@ -31,7 +31,12 @@ struct CudaExec final : Exec {
   std::vector<char> own_stream;
   std::vector<cudaEvent_t> events;
   std::vector<cudaEvent_t> tpool;                 // timing events (free list)
-  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> tpending;
+  struct Timed {
+    cudaEvent_t a, b;
+    uint64_t cells;  // cells read + written once by the launch (stencil sweeps), else 0
+  };
+  std::vector<Timed> tpending;
+  uint64_t next_cells = 0;  // cells of the next timed launch (set just before it)
   cudaEvent_t t_begin = nullptr, t_end = nullptr;
   cudaEvent_t local_ready = nullptr;  // in-process transport
 
@@ -59,7 +64,8 @@ struct CudaExec final : Exec {
     CK(cudaEventRecord(a, S(st)));
     CK(launch());
     CK(cudaEventRecord(b, S(st)));
-    tpending.push_back({a, b});
+    tpending.push_back({a, b, next_cells});
+    next_cells = 0;
     return Status::ok();
   }
   // the same for a launch that reports a library Status (user kernels: the
@@ -80,17 +86,23 @@ struct CudaExec final : Exec {
       return r;
     }
     CK(cudaEventRecord(b, S(st)));
-    tpending.push_back({a, b});
+    tpending.push_back({a, b, next_cells});
+    next_cells = 0;
     return Status::ok();
   }
   Status collect(Domain& d) {  // after a synchronize
     for (auto& pr : tpending) {
       float ms = 0;
-      CK(cudaEventElapsedTime(&ms, pr.first, pr.second));
+      CK(cudaEventElapsedTime(&ms, pr.a, pr.b));
       d.stats.kernel_ms += ms;
       d.stats.kernel_timed++;
-      tpool.push_back(pr.first);
-      tpool.push_back(pr.second);
+      if (pr.cells) {
+        d.stats.sweep_ms += ms;
+        d.stats.sweep_cells += pr.cells;
+        d.stats.sweep_timed++;
+      }
+      tpool.push_back(pr.a);
+      tpool.push_back(pr.b);
     }
     tpending.clear();
     return Status::ok();
@@ -310,6 +322,7 @@ struct CudaExec final : Exec {
       d.prog_grid = grid;
     }
     cudaError_t le = cudaSuccess;
+    next_cells = d.kernel_timing ? (uint64_t)n * d.G.tile_elems * (uint64_t)p.nsteps : 0;
     Status r = timed(d, st, [&] {
       le = launch_heat7(p, d.stages, d.heat_smem, (int)grid, S(st));
       return le == cudaErrorCooperativeLaunchTooLarge ? cudaSuccess : le;
@@ -370,6 +383,7 @@ struct CudaExec final : Exec {
     INJECT(FAULT_KERNEL, st);
     if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
     const SlabView s = slab_view(d, src, lo), t = slab_view(d, dst, lo);
+    next_cells = d.kernel_timing ? (uint64_t)(hi - lo) * d.G.l[0] * d.G.l[1] : 0;
     Status r = timed(d, st, [&] {
       return launch_slab_sweep(s, t, (int)d.G.l[0], (int)d.G.l[1], lo, hi, d.kernel_alpha, sms, S(st));
     });
@@ -458,6 +472,7 @@ struct CudaExec final : Exec {
     const int64_t planes = (int64_t)n * p.nbands * p.tz;
     int64_t grid = (int64_t)sms * heat2_occ;
     grid = std::max<int64_t>(1, std::min<int64_t>(grid, (planes + 3) / 4));
+    next_cells = d.kernel_timing ? (uint64_t)n * d.G.tile_elems : 0;  // one pass for two steps
     Status r = timed(d, st, [&] { return launch_heat7x2(P, d.heat2_smem, (int)grid, S(st)); });
     if (r.bad()) return r;
     d.stats.n_kernels++;
@@ -658,8 +673,8 @@ struct CudaExec final : Exec {
   }
   void destroy(Domain&) override {
     for (auto& pr : tpending) {
-      tpool.push_back(pr.first);
-      tpool.push_back(pr.second);
+      tpool.push_back(pr.a);
+      tpool.push_back(pr.b);
     }
     tpending.clear();
     for (auto e : tpool) cudaEventDestroy(e);

@@ -1217,7 +1217,11 @@ static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool 
   const bool load = !d.resident_valid;
   const int64_t nL = d.G.n[2];
   StreamPlan sp{};
-  if (load && !serial && streamthrough_ok(d, steps, &sp)) return run_streamthrough(d, alpha, steps, S, sp);
+  if (load && !serial && streamthrough_ok(d, steps, &sp)) {
+    d.last_schedule = 2;
+    return run_streamthrough(d, alpha, steps, S, sp);
+  }
+  d.last_schedule = serial ? 5 : 1;
   const std::vector<int> kp = plan_passes(d, steps);
   const int T = (int)kp.size();  // passes
   struct Phase {
@@ -1540,8 +1544,10 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
   } else {
     OocPlan op;
     if (k.kind == TILE_KERNEL_HEAT7 && !serial && ooc_streamthrough_ok(d, steps, &op)) {
+      d.last_schedule = 4;
       r = run_streamthrough_ooc(d, steps, S, op);
     } else {
+      d.last_schedule = serial ? 5 : 3;
       r = run_stream(d, k, steps, S);
       if (k.kind != TILE_KERNEL_HEAT7 && steps > 0) {
         // tiles changed without their faces (device or host copies)

@@ -181,6 +181,7 @@ struct Domain {
   tile_options opt;
   Fault fault;
   bool poisoned = false;
+  int last_schedule = 0;  // tile_info.last_schedule
   int device = 0;
   int mode = MODE_RESIDENT;
   int measure = TILE_MEASURE_NORMAL;

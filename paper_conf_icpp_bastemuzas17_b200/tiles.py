@@ -61,7 +61,8 @@ class TileStats(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint64) for n in ("bytes_h2d", "bytes_d2h", "bytes_halo", "n_h2d", "n_d2h",
                                                "n_kernels", "n_halo", "hits", "misses", "evictions",
                                                "writebacks", "steps_done")] + [
-        ("last_run_ms", ctypes.c_double), ("kernel_ms", ctypes.c_double), ("kernel_timed", ctypes.c_uint64)]
+        ("last_run_ms", ctypes.c_double), ("kernel_ms", ctypes.c_double), ("kernel_timed", ctypes.c_uint64),
+        ("sweep_ms", ctypes.c_double), ("sweep_cells", ctypes.c_uint64), ("sweep_timed", ctypes.c_uint64)]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}
@@ -73,7 +74,7 @@ class TileInfo(ctypes.Structure):
                 ("ntiles", ctypes.c_int64), ("z_offset", ctypes.c_int64), ("ghost", ctypes.c_int32),
                 ("nslots", ctypes.c_int32), ("sched", ctypes.c_int32), ("resident", ctypes.c_int32),
                 ("device_bytes", ctypes.c_uint64), ("host_bytes", ctypes.c_uint64),
-                ("steps_per_pass", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("steps_per_pass", ctypes.c_int32), ("last_schedule", ctypes.c_int32)]
 
     def as_dict(self):
         out = {}

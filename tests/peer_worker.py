@@ -11,7 +11,10 @@ HEAT_AS_USER = ("__device__ double hu(double c, double xm, double xp, double ym,
                 " double zp) { return c + 0.125 * ((((xm + xp) + (ym + yp)) + (zm + zp)) - 6.0 * c); }")
 
 
-def run(r, G, dims, td, bc, sched, budget, runs, seed, conn, transport=1, stream_through=0, user_runs=()):
+def run(r, G, dims, td, bc, sched, budget, runs, seed, conn, transport=1, stream_through=0, user_runs=(),
+        device=0, nccl_id=None):
+    """transport 1/2: peer windows (copies / fused); 0: NCCL (nccl_id given,
+    each rank on its own device). device: this rank's CUDA ordinal."""
     sys.path.insert(0, ROOT)
     try:
         import synth
@@ -21,10 +24,15 @@ def run(r, G, dims, td, bc, sched, budget, runs, seed, conn, transport=1, stream
         kw = {"sched": sched, "stream_through": stream_through}
         if budget:
             kw["device_budget_bytes"] = budget
-        with T.Domain(dims, td, bc=bc, nranks=G, rank=r, peer_transport=transport, device=0, **kw) as d:
-            conn.send(("handle", d.peer_handle()))
+        if transport == 0:
+            kw["nccl_id"] = nccl_id
+        else:
+            kw["peer_transport"] = transport
+        with T.Domain(dims, td, bc=bc, nranks=G, rank=r, device=device, **kw) as d:
+            conn.send(("handle", d.peer_handle() if transport else b""))
             kind, handles = conn.recv()
-            d.peer_connect(handles)
+            if transport:
+                d.peer_connect(handles)
             if bc == "periodic":
                 u = synth.uniform_grid(nx, ny, nz, seed)
                 d.load(u[r * nzl:(r + 1) * nzl])

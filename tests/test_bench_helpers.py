@@ -111,3 +111,39 @@ def test_multi_domain_transport_fallback(monkeypatch, fail_rank, other_ok, expec
     assert (getattr(bench.multi_domain, "fallback", None) is not None) == expect_nccl
     if expect_nccl and fail_rank is None:   # this rank's peer domain was built, then released
         assert made[0].freed
+
+
+def test_bench_spawns_one_process_per_gpu():
+    """`python bench.py --gpus 2` with no torchrun environment re-launches
+    itself under torch.distributed.run (127.0.0.1), one process per GPU:
+    the probe mode stops right after the launch and has rank 0 report the
+    world it sees (gloo on CPU)."""
+    import json
+    import subprocess
+    import sys
+    env = {k: v for k, v in os.environ.items()
+           if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK", "MASTER_ADDR", "MASTER_PORT")}
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--spawn-probe"],
+                       capture_output=True, text=True, env=env, timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [json.loads(x) for x in r.stdout.splitlines() if x.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    ln = lines[0]
+    assert ln["world_size"] == 2 and sorted(x["rank"] for x in ln["ranks"]) == [0, 1]
+    assert len({x["pid"] for x in ln["ranks"]}) == 2
+
+
+def test_bench_rejects_world_size_mismatch():
+    import subprocess
+    import sys
+    env = dict(os.environ, WORLD_SIZE="3", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--spawn-probe"],
+                       capture_output=True, text=True, env=env, timeout=120)
+    assert r.returncode != 0 and "WORLD_SIZE=3" in r.stderr
+
+
+def test_spawn_command_is_the_drivers_launch_line():
+    cmd = bench.spawn_cmd(["--gpus", "4", "--steps", "5"], 4, 29511)
+    assert cmd[1:4] == ["-m", "torch.distributed.run", "--nnodes=1"]
+    assert "--nproc-per-node=4" in cmd and "127.0.0.1" in cmd and "--master-port=29511" in cmd
+    assert cmd[-4:] == ["--gpus", "4", "--steps", "5"]

@@ -109,18 +109,21 @@ def test_peer_transport_processes_bit_exact(G, bc, sched, runs, transport):
     assert all(m[2] > 0 and m[3] > 0 for m in outs)  # halo exchanges happened through the window
 
 
-def _peer_procs(G, dims, td, bc, sched, budget, runs, transport, stream_through=0, user_runs=()):
+def _peer_procs(G, dims, td, bc, sched, budget, runs, transport, stream_through=0, user_runs=(),
+                multi_device=False):
     """One spawned process per rank (tests/peer_worker.py), IPC handles
-    relayed through pipes; returns every rank's ("out", ...) message."""
+    relayed through pipes; returns every rank's ("out", ...) message.
+    multi_device: rank r on CUDA device r (transport 0 = NCCL needs it)."""
     import multiprocessing as mp
     from tests import peer_worker
     ctx = mp.get_context("spawn")
     pipes, procs = [], []
+    nid = T.nccl_unique_id() if transport == 0 else None
     for r in range(G):
         a, b = ctx.Pipe()
         p = ctx.Process(target=peer_worker.run,
                         args=(r, G, dims, td, bc, sched, budget, runs, 42, b, transport, stream_through,
-                              tuple(user_runs)))
+                              tuple(user_runs), r if multi_device else 0, nid))
         p.start()
         pipes.append(a)
         procs.append(p)
@@ -232,3 +235,94 @@ def test_peer_user_stencil_interleaved_bit_exact(G, transport):
     outs = _peer_procs(G, dims, td, "periodic", "resident", 0, runs, transport, user_runs=(1, 3))
     got = np.concatenate([m[1] for m in outs], axis=0)
     assert np.array_equal(got, oracle.heat_c(synth.uniform_grid(nx, ny, nz, 42), ALPHA, sum(runs)))
+
+
+
+# ------------------------------------------------ several physical devices
+def _need_devices(G):
+    import torch
+    if torch.cuda.device_count() < G:
+        pytest.skip(f"needs {G} CUDA devices (this box has {torch.cuda.device_count()})")
+
+
+def _oracle_ref(dims, bc, steps):
+    nx, ny, nz = dims
+    if bc == "periodic":
+        return oracle.heat_c(synth.uniform_grid(nx, ny, nz, 42), ALPHA, steps)
+    ext = synth.uniform_grid(nx + 2, ny + 2, nz + 2, 42)
+    return oracle.heat_c(ext, ALPHA, steps, oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+
+
+@pytest.mark.parametrize("G,transport,bc,sched,runs", [
+    (2, 0, "periodic", "resident", [5, 3]), (2, 0, "dirichlet", "resident", [4]),
+    (2, 0, "periodic", "stream", [3]), (4, 0, "periodic", "resident", [6]),
+    (2, 1, "periodic", "resident", [5]), (2, 2, "periodic", "resident", [7, 4]),
+    (4, 2, "dirichlet", "resident", [6]), (8, 2, "periodic", "resident", [5]),
+    (8, 0, "periodic", "resident", [5])])
+def test_multi_device_halo_transports_bit_exact(G, transport, bc, sched, runs):
+    """One process per rank, rank r on CUDA device r: the NCCL send/recv
+    exchange (transport 0), the peer-window copies over NVLink (1) and the
+    fused in-kernel push into the neighbour GPU's window (2), bit-exact
+    against the oracle on the global grid. Skips with fewer devices."""
+    _need_devices(G)
+    dims, td = (64, 32, 16 * G), (32, 16, 8)
+    budget = _budget(dims, td, 3, bc=bc, nranks=G, rank=0) if sched == "stream" else 0
+    outs = _peer_procs(G, dims, td, bc, sched, budget, runs, transport, multi_device=True)
+    got = np.concatenate([m[1] if bc == "periodic" else m[1][1:-1, 1:-1, 1:-1] for m in outs], axis=0)
+    ref = _oracle_ref(dims, bc, sum(runs))
+    assert np.array_equal(got, ref), np.abs(got - ref).max()
+    assert all(m[2] > 0 for m in outs)
+
+
+@pytest.mark.parametrize("G,T,runs_after", [(2, 8, [3]), (4, 4, [2])])
+def test_multi_device_stream_through_bit_exact(G, T, runs_after):
+    """Multi-rank stream-through across physical devices (halo layers of
+    initial data pushed once per run into the neighbour GPU's window)."""
+    _need_devices(G)
+    tz = 16
+    dims, td = (64, 32, 8 * tz * G), (32, 16, tz)
+    runs = [T] + runs_after
+    outs = _peer_procs(G, dims, td, "periodic", "auto", 0, runs, transport=2, stream_through=1,
+                       multi_device=True)
+    u0 = synth.uniform_grid(*dims, 42)
+    first = np.concatenate([m[4][1] for m in outs], axis=0)
+    assert np.array_equal(first, oracle.heat_c(u0, ALPHA, T))
+    got = np.concatenate([m[1] for m in outs], axis=0)
+    assert np.array_equal(got, oracle.heat_c(u0, ALPHA, sum(runs)))
+
+
+def _bench_line(args, env_extra):
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = {k: v for k, v in os.environ.items()
+           if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK", "MASTER_ADDR", "MASTER_PORT")}
+    env.update(env_extra)
+    r = subprocess.run([sys.executable, os.path.join(root, "bench.py"), *args], capture_output=True,
+                       text=True, env=env, timeout=900)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [json.loads(x) for x in r.stdout.splitlines() if x.startswith("{")]
+    assert len(lines) == 1, r.stdout[-3000:]
+    return lines[0]
+
+
+def test_bench_two_ranks_spawned_on_one_gpu():
+    """`bench.py --gpus 2` spawns its own two ranks (TILES_BENCH_ONE_GPU=1:
+    both on the pool's one GPU, gloo; a functional check, not a number)."""
+    ln = _bench_line(["--gpus", "2", "--steps", "2", "--warmup", "1", "--no-extras", "--no-cpu-baseline"],
+                     {"TILES_BENCH_ONE_GPU": "1"})
+    assert ln["n_gpus"] == 2 and ln["config"]["comm_ranks"] == 2
+    assert ln["config"]["transport"] == "peer" and ln["value"] > 0
+    assert ln["e2e"]["h2d_bytes_per_step"] == 512 ** 3 * 8
+
+
+def test_bench_multi_device_spawn():
+    """`bench.py --gpus 2` over two physical devices (peer transport, then
+    NCCL): one line, n_gpus 2, the transport named."""
+    _need_devices(2)
+    for tr in ("peer", "nccl"):
+        ln = _bench_line(["--gpus", "2", "--steps", "2", "--warmup", "1", "--no-extras", "--no-cpu-baseline",
+                          "--transport", tr], {})
+        assert ln["n_gpus"] == 2 and ln["config"]["transport"].startswith(tr)

@@ -343,3 +343,13 @@ def test_residency_all_fit_only_first_sweep_transfers():
     assert ops.count("h2d") == 4 and ops.count("d2h") == 0 and ops.count("hit") == 8
     ro.cpu_request(2)
     assert ro.trace[-1] == ("d2h", 2, 2)
+
+
+def test_all_core_twin_is_bit_identical():
+    """The OpenMP twin (all-core CPU baseline) equals the
+    single-threaded oracle bit for bit, and both equal the NumPy twin."""
+    u = synth.uniform_grid(24, 20, 18, 42)
+    one = oracle.heat_c(u, ALPHA, 4)
+    for th in (2, 3, 8):
+        assert np.array_equal(oracle.heat_c(u, ALPHA, 4, threads=th), one)
+    assert np.array_equal(one, oracle.heat_np(u, ALPHA, 4))
