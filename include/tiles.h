@@ -169,6 +169,19 @@ typedef struct {
                                    (halves host-link bytes per step), single
                                    steps when resident; 1 = two steps in every
                                    schedule; -1 = never */
+  int32_t wavefront;            /* HEAT7 run starting from a fresh upload
+                                   (periodic, single rank, resident, 2T planes
+                                   of scratch fit): time-skewed march over
+                                   chunks of planes — level s of chunk i
+                                   covers planes [c*i - s, c*i + c - s), so a
+                                   chunk needs only its own upload and the
+                                   previous chunk, and its final planes go
+                                   back to the host as soon as it ends; no
+                                   redundant sweeps besides a T^2 bootstrap at
+                                   the periodic seam. -1 =
+                                   never, 0 (default) = when the cost model
+                                   prefers it to stream-through and the
+                                   batched schedule, 1 = whenever feasible */
 } tile_options;
 
 typedef struct {
@@ -256,9 +269,19 @@ typedef enum {
                             slab-end c planes of initial data (b = 1 top -> upper rank,
                             0 bottom -> lower rank), 1 wait for side b's halo layer,
                             2 release side b's halo layer; d = the run's epoch */
-  TILE_OP_SYNC = 25      /* host waits for every stream (stream -1): every op before it
+  TILE_OP_SYNC = 25,     /* host waits for every stream (stream -1): every op before it
                             completes before any op after it starts; host-side reads of
                             the pinned store (face extraction) happen here */
+  TILE_OP_WSWEEP = 26,   /* wavefront sweep of planes [lo, hi) (c = lo | hi << 32, two
+                            signed 32-bit halves), periodic in x/y; a = source view, b =
+                            destination view: bit 0 = 1: planes z >= 0 in resident array
+                            (bit 1), z < 0 in the d tile layers of scratch starting at
+                            slot (code >> 2); bit 0 = 0: resident array (bit 1), z
+                            wrapped (no scratch) */
+  TILE_OP_D2H_PLANES = 27,/* planes [d & 0xffffffff, + d >> 32) of c tile slots b.. ->
+                            the same planes of host tiles a.. */
+  TILE_OP_COPY_PLANES = 28/* planes [d & 0xffffffff, + d >> 32) of c tile slots a.. ->
+                            the same planes of slots b.. */
 } tile_op_kind;
 
 typedef struct {

@@ -363,6 +363,14 @@ struct CudaExec final : Exec {
         v.hlo = d.st_halo[0];
         v.hhi = d.st_halo[1];
       }
+    } else if (r.kind == SlabRef::WAVE) {
+      v.base = d.slot_ptr(r.slot ? (int)G.ntiles : 0);
+      v.te = G.tile_elems;
+      v.tz = (int)G.t[2];
+      v.zbase = 0;
+      v.nz = (int)G.l[2];
+      v.hlo = d.slot_ptr(r.ring[0]);
+      v.nlo = (int)r.un;
     } else if (r.kind == SlabRef::UNITS) {
       v.ring = 1;
       v.te = r.un * G.t[0] * G.t[1];
@@ -427,6 +435,25 @@ struct CudaExec final : Exec {
     const size_t pl = (size_t)d.G.t[0] * d.G.t[1] * 8, tb = (size_t)d.G.tile_elems * 8;
     CK(cudaMemcpy2DAsync(reinterpret_cast<char*>(d.slot_ptr(s0)) + p0 * pl, tb, d.slot_ptr(ps),
                          np * pl, np * pl, (size_t)n, cudaMemcpyDeviceToDevice, S(st)));
+    return Status::ok();
+  }
+  Status d2h_planes(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int st) override {
+    INJECT(FAULT_D2H, st);
+    if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
+    const size_t pl = (size_t)d.G.t[0] * d.G.t[1] * 8, tb = (size_t)d.G.tile_elems * 8;
+    CK(cudaMemcpy2DAsync(reinterpret_cast<char*>(d.host_tile(t0)) + p0 * pl, tb,
+                         reinterpret_cast<const char*>(d.slot_ptr(s0)) + p0 * pl, tb, np * pl, (size_t)n,
+                         cudaMemcpyDeviceToHost, S(st)));
+    d.stats.bytes_d2h += (uint64_t)n * np * pl;
+    d.stats.n_d2h++;
+    return Status::ok();
+  }
+  Status copy_planes(Domain& d, int src0, int dst0, int64_t n, int64_t p0, int64_t np, int st) override {
+    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
+    const size_t pl = (size_t)d.G.t[0] * d.G.t[1] * 8, tb = (size_t)d.G.tile_elems * 8;
+    CK(cudaMemcpy2DAsync(reinterpret_cast<char*>(d.slot_ptr(dst0)) + p0 * pl, tb,
+                         reinterpret_cast<const char*>(d.slot_ptr(src0)) + p0 * pl, tb, np * pl, (size_t)n,
+                         cudaMemcpyDeviceToDevice, S(st)));
     return Status::ok();
   }
   Status copy_slots(Domain& d, int src, int dst, int64_t n, int st) override {

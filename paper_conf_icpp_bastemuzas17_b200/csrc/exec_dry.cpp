@@ -100,6 +100,18 @@ struct DryExec final : Exec {
           (int64_t)lo | ((int64_t)hi << 32), src.u | (src.un << 32));
       return Status::ok();
     }
+    if (src.kind == SlabRef::WAVE || dst.kind == SlabRef::WAVE) {
+      // wavefront sweep: view codes (bit 0: 1 = WAVE, 0 = RESIDENT wrapped at
+      // zbase 0; bit 1: the resident array; bits 2..: WAVE scratch slot);
+      // c: lo, hi as two signed 32-bit halves; d: scratch layers (nlo)
+      auto code = [](const SlabRef& r) {
+        return r.kind == SlabRef::WAVE ? 1 | ((int64_t)r.slot << 1) | ((int64_t)r.ring[0] << 2)
+                                       : ((int64_t)r.slot << 1);
+      };
+      put(d, TILE_OP_WSWEEP, st, code(src), code(dst),
+          (int64_t)(uint32_t)lo | ((int64_t)(uint32_t)hi << 32), dst.kind == SlabRef::WAVE ? dst.un : src.un);
+      return Status::ok();
+    }
     // a: slab slot, or -1-bit for the resident array (slab plane 0 at z = d)
     // b: slab slot, or -1-slot for packed sub-tiles (sweep plane lo -> 0)
     const int64_t a = src.kind == SlabRef::DENSE ? src.slot : -1 - (int64_t)src.slot;
@@ -131,6 +143,17 @@ struct DryExec final : Exec {
   }
   Status copy_part(Domain& d, int ps, int s0, int64_t n, int64_t p0, int64_t np, int st) override {
     put(d, TILE_OP_COPY_PART, st, ps, s0, n, p0 | (np << 32));
+    return Status::ok();
+  }
+  Status d2h_planes(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int st) override {
+    if (Status f_ = inject(d, FAULT_D2H); f_.bad()) return f_;
+    d.stats.bytes_d2h += (uint64_t)n * np * d.G.t[0] * d.G.t[1] * 8;
+    d.stats.n_d2h++;
+    put(d, TILE_OP_D2H_PLANES, st, t0, s0, n, p0 | (np << 32));
+    return Status::ok();
+  }
+  Status copy_planes(Domain& d, int src0, int dst0, int64_t n, int64_t p0, int64_t np, int st) override {
+    put(d, TILE_OP_COPY_PLANES, st, src0, dst0, n, p0 | (np << 32));
     return Status::ok();
   }
   Status copy_slots(Domain& d, int src, int dst, int64_t n, int st) override {

@@ -176,8 +176,9 @@ struct SlabView {
   int ring;                     // 1: unit-ring view (below)
   int u, U, un;
   double* ubase[3];
-  double* hlo;                  // resident view, multi-rank: planes z < 0 (tile-blocked layer,
-  double* hhi;                  // planes tz+z) and z >= nz (planes z-nz) instead of the wrap
+  double* hlo;                  // resident view: planes z < 0 from nlo tile-blocked layers here
+  double* hhi;                  // (multi-rank halo layer, nlo = 1; wavefront scratch), planes
+  int nlo;                      // z >= nz (planes z-nz) from hhi, instead of the periodic wrap
 };
 cudaError_t launch_slab_sweep(const SlabView& src, const SlabView& dst, int nx, int ny, int lo,
                               int hi, double alpha, int sms, cudaStream_t s);

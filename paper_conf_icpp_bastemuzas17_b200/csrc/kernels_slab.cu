@@ -35,10 +35,14 @@ struct ViewDev {
   double* ub[3];
   double* hlo;
   double* hhi;
+  int nlo;
   // first element of slab plane pl (x = y = 0 of tile column 0, row 0)
   __device__ __forceinline__ double* P(int pl) const {
     int gz = zbase + pl;
-    if (hlo && gz < 0) return hlo + (int64_t)(tz + gz) * ty * tx;   // lower rank's top planes
+    if (hlo && gz < 0) {  // lower rank's top planes / wavefront scratch: nlo tile layers
+      const int q = gz + nlo * tz, L = q / tz;
+      return hlo + (int64_t)L * nty * ntx * te + (int64_t)(q - L * tz) * ty * tx;
+    }
     if (hhi && gz >= nz) return hhi + (int64_t)(gz - nz) * ty * tx;  // upper rank's bottom planes
     if (nz > 0) {
       gz %= nz;
@@ -67,7 +71,7 @@ struct ViewDev {
 
 static ViewDev to_dev(const SlabView& v) {
   return ViewDev{v.base, v.te, v.tx, v.ty, v.tz, v.ntx, v.nty, v.zbase, v.nz, v.ring, v.u, v.U, v.un,
-                 {v.ubase[0], v.ubase[1], v.ubase[2]}, v.hlo, v.hhi};
+                 {v.ubase[0], v.ubase[1], v.ubase[2]}, v.hlo, v.hhi, v.nlo > 0 ? v.nlo : 1};
 }
 
 // Work items are (z chunk, column) pairs, column = (x segment of 128 pairs,

@@ -247,6 +247,7 @@ Status domain_setup(Domain& d) {
   d.pool = static_cast<char*>(dp);
   d.pool_bytes = dev_total;
   d.device_bytes = dev_total;
+  d.budget_left = budget > dev_total ? budget - dev_total : 0;
   off = 0;
   auto carve = [&](uint64_t bytes) {
     char* p = d.pool + off;
@@ -369,6 +370,7 @@ Status domain_free(Domain* d) {
     if (d->peer_window) peer_destroy(*d);
     d->exec->destroy(*d);
     if (d->own_pool && d->pool) d->exec->free_device(*d, d->pool);
+    if (d->own_wave && d->wave_base) d->exec->free_device(*d, d->wave_base);
     if (d->host) d->exec->free_host(*d, d->host);
     delete d->exec;
   }
@@ -821,7 +823,7 @@ static std::vector<UnitDef> make_units(const Geometry& G, int64_t un, int T, int
   return v;
 }
 
-static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
+static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp, double* est_out) {
   const Geometry& G = d.G;
   if (d.opt.stream_through < 0 || G.bc != TILE_BC_PERIODIC) return false;
   // z-slab ranks: the peer transport's halo layers carry the T planes beyond
@@ -855,11 +857,10 @@ static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp) {
     const double est = std::max(nz, r_sweep * nz * (Td + (Td * Td - Td) / (double)u)) + 3.0 * (double)u;
     if (est < best) best = est, unit = u;
   }
-  // the batched resident schedule instead: both link directions in sequence
-  // (dependency form, 2 nz) plus T whole-domain steps, partly overlapped
-  // (0.011 per plane-step, same fit); take stream-through only where it is
-  // estimated faster
-  if (d.opt.stream_through == 0 && best > 2.0 * nz + 0.011 * nz * Td) return false;
+  // the caller compares with the batched resident schedule (both link
+  // directions in sequence, 2 nz, plus T whole-domain steps partly
+  // overlapped, 0.011 per plane-step, same fit) and the wavefront
+  *est_out = best;
   if (G.l[2] / unit + 4 > G.ntiles) unit = G.t[2];  // event budget (one per unit)
   sp->unit = unit;
   // thin tail units first; uniform units if those do not fit
@@ -1213,13 +1214,224 @@ static Status run_streamthrough_ooc(Domain& d, int T, int S, const OocPlan& op) 
   return Status::ok();
 }
 
+// ---------------------------------------------------------------- wavefront
+// Fresh-upload heat runs beyond the stream-through's reach (T > tz, or where
+// its redundant halo sweeps cost more than they save): a
+// time-skewed march over chunks of c planes. Level s (the grid after s
+// steps) of iteration i covers planes [c*i - s, c*i + c - s), in unwrapped
+// coordinates: a plane z < 0 is the ring's top plane nz + z, kept in a
+// scratch of whole tile layers. Computing it reads level s-1 on
+// [c*i - s - 1, c*i + c - s + 1): level s-1 of the same iteration plus the
+// top two planes of iteration i-1. So iteration i depends only on its own
+// chunk's upload and on iteration i-1, every cell is updated once per level
+// (no redundant halo sweeps), and iteration i's level-T chunk is final when
+// the iteration ends: its D2H starts then, while later chunks are still
+// uploading. Iteration 0 reads level s-1 at planes -s-1, -s, which the ring
+// computes last: a bootstrap trapezoid computes them first from the initial
+// data of the top 2T planes (uploaded first) — T sweeps over [-2T + t, -t),
+// t = 1..T-1, about T^2 plane updates (the dependency cone of the seam).
+// Buffers: level s in resident array bit ^ (s & 1) for z >= 0, in scratch
+// parity s & 1 (nlo = ceil(2T / tz) tile layers) for z < 0; level 0 is read
+// through the wrapped resident view. Level s+2 overwrites level s only where
+// no reader of level s remains (level s+1 of the same iteration runs before
+// it; the two planes iteration i+1 reads lie above level s+2's chunk of
+// iteration i) — checked on CPU by the random-order replay of the trace.
+struct WavePlan {
+  int64_t c = 0;    // chunk planes (divides tz)
+  int64_t B = 0;    // bootstrap region: the top B planes, uploaded first (multiple of c, >= 2T)
+  int64_t nlo = 0;  // scratch tile layers per parity
+  double est = 0;   // estimated time in link-plane units (streamthrough_ok's scale)
+};
+
+static int64_t wave_chunk() {
+  static const int64_t c = [] {
+    const char* e = getenv("TILES_WAVE_C");
+    return e ? std::max<int64_t>(1, atoll(e)) : (int64_t)16;
+  }();
+  return c;
+}
+
+static double sweep_ratio() {  // sweep time / duplex link time per plane (see streamthrough_ok)
+  static const double r = [] {
+    const char* e = getenv("TILES_ST_R");
+    return e ? atof(e) : 0.021;
+  }();
+  return r;
+}
+
+static bool wavefront_ok(const Domain& d, int T, WavePlan* wp) {
+  const Geometry& G = d.G;
+  if (d.opt.wavefront < 0 || G.nranks != 1 || G.bc != TILE_BC_PERIODIC || d.mode != MODE_RESIDENT) return false;
+  if (T < 1 || G.t[0] % 2 || G.l[2] > (1 << 28)) return false;
+  const int64_t nz = G.l[2], tz = G.t[2];
+  int64_t c = std::min<int64_t>(wave_chunk(), tz);
+  while (tz % c) --c;
+  while (nz / c > G.ntiles) c *= 2;  // one event per chunk (ev_in / ev_host)
+  if (tz % c || nz / c > G.ntiles) return false;
+  const int64_t B = (2 * (int64_t)T + c - 1) / c * c;
+  if (B + c > nz) return false;  // the seam's cone would cover the ring
+  const int64_t nlo = (2 * (int64_t)T + tz - 1) / tz;
+  const uint64_t need = (uint64_t)(2 * nlo * G.layer_tiles) * (uint64_t)G.tile_elems * 8;
+  if ((int64_t)d.wave_slots < 2 * nlo * G.layer_tiles && need > d.budget_left + (uint64_t)d.wave_slots * G.tile_elems * 8)
+    return false;
+  const double r = sweep_ratio(), Td = (double)T, n = (double)nz;
+  wp->c = c;
+  wp->B = B;
+  wp->nlo = nlo;
+  // the bootstrap waits for the top B planes and sweeps ~T^2 planes; then
+  // the march is bound by the link (every plane down once, the rest up) or
+  // by its T sweeps per plane; one chunk of fill/drain
+  wp->est = (double)B + r * Td * Td + std::max(n, r * n * Td) + (double)c * (1.0 + r * Td);
+  return true;
+}
+
+static Status ensure_wave_scratch(Domain& d, int64_t slots) {
+  if (d.wave_slots >= slots) return Status::ok();
+  const uint64_t bytes = (uint64_t)slots * d.G.tile_elems * 8;
+  if (d.own_wave && d.wave_base) {
+    Status r = d.exec->sync_all(d);  // the old scratch may still be read
+    if (r.bad()) return r;
+    d.exec->free_device(d, d.wave_base);
+    d.budget_left += (uint64_t)d.wave_slots * d.G.tile_elems * 8;
+    d.wave_base = nullptr;
+    d.wave_slots = 0;
+  }
+  if (bytes > d.budget_left) return make_err(TILE_ENOMEM_DEVICE, "wavefront scratch exceeds the device budget");
+  if (d.opt.device_pool) {  // the caller's pool: its tail past the domain's carve
+    d.wave_base = reinterpret_cast<double*>(d.pool + d.pool_bytes);
+    d.own_wave = false;
+  } else {
+    void* p = nullptr;
+    Status r = d.exec->alloc_device(d, bytes, &p);
+    if (r.bad()) return r;
+    d.wave_base = static_cast<double*>(p);
+    d.own_wave = true;
+  }
+  d.budget_left -= bytes;
+  d.wave_slots = (int)slots;
+  return Status::ok();
+}
+
+static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
+  Exec& X = *d.exec;
+  const Geometry& G = d.G;
+  const int64_t nz = G.l[2], tz = G.t[2], lt = G.layer_tiles, c = wp.c, B = wp.B, nlo = wp.nlo;
+  const int64_t U = nz / c, iB = (nz - B) / c;  // iterations; first chunk inside the bootstrap region
+  Status r = ensure_wave_scratch(d, 2 * nlo * lt);
+  if (r.bad()) return r;
+  const Pipes P(S, false);
+  const int cs = P.comp(0), os = P.out(0), is = P.in(0);
+  const int bit = d.res_bit;
+  const int scr[2] = {d.nslots, d.nslots + (int)(nlo * lt)};
+  const int fin = bit ^ (T & 1);  // array holding level T (z >= 0)
+  auto arr0 = [&](int a, int64_t L) { return (int)((a ? G.ntiles : 0) + L * lt); };
+  // planes [z0, z1) of the ring (physical, 0 <= z0 < z1 <= nz) in tile-layer pieces
+  auto pieces = [&](int64_t z0, int64_t z1, auto&& f) -> Status {
+    for (int64_t z = z0; z < z1;) {
+      const int64_t L = z / tz, lz = z - L * tz, np = std::min(z1 - z, tz - lz);
+      Status q = f(L, lz, np);
+      if (q.bad()) return q;
+      z += np;
+    }
+    return Status::ok();
+  };
+  auto upload = [&](int64_t z0, int64_t z1) {
+    return pieces(z0, z1, [&](int64_t L, int64_t lz, int64_t np) {
+      return X.h2d_part(d, L * lt, lt, arr0(bit, L), lz, np, is);
+    });
+  };
+  // uploads on one copy-in stream, in march order: the seam's cone first
+  r = upload(nz - B, nz);
+  if (r.bad()) return r;
+  r = X.record(d, ev_in(d, iB), is);
+  if (r.bad()) return r;
+  for (int64_t i = 0; i < iB; ++i) {
+    r = upload(i * c, (i + 1) * c);
+    if (r.bad()) return r;
+    r = X.record(d, ev_in(d, i), is);
+    if (r.bad()) return r;
+  }
+  auto lvl = [&](int s) {  // view of level s (s = 0: the initial data, wrapped)
+    return s == 0 ? SlabRef{SlabRef::RESIDENT, bit, 0, {0, 0, 0}, 0, 0}
+                  : SlabRef{SlabRef::WAVE, bit ^ (s & 1), 0, {scr[s & 1], 0, 0}, 0, nlo};
+  };
+  // bootstrap: level t on [-2T + t, -t) from the top 2T planes
+  r = X.wait(d, ev_in(d, iB), cs);
+  if (r.bad()) return r;
+  for (int t = 1; t < T; ++t) {
+    r = X.slab_sweep(d, lvl(t - 1), lvl(t), -2 * T + t, -t, cs);
+    if (r.bad()) return r;
+  }
+  // the march
+  for (int64_t i = 0; i < U; ++i) {
+    if (i < iB) {
+      r = X.wait(d, ev_in(d, i), cs);
+      if (r.bad()) return r;
+    }
+    for (int s = 1; s <= T; ++s) {
+      r = X.slab_sweep(d, lvl(s - 1), lvl(s), (int)(c * i - s), (int)(c * i + c - s), cs);
+      if (r.bad()) return r;
+    }
+    r = X.record(d, ev_host(d, i), cs);
+    if (r.bad()) return r;
+    r = X.wait(d, ev_host(d, i), os);
+    if (r.bad()) return r;
+    // level-T planes [c*i - T, c*i + c - T): z < 0 from the scratch (the
+    // ring's top planes), z >= 0 from the resident array
+    const int64_t a = c * i - T, b = c * i + c - T;
+    if (a < 0) {
+      r = pieces(nz + a, nz + std::min<int64_t>(b, 0), [&](int64_t L, int64_t lz, int64_t np) {
+        const int64_t Ls = L - (nz / tz - nlo);  // scratch layer of physical layer L
+        return X.d2h_planes(d, L * lt, lt, scr[T & 1] + (int)(Ls * lt), lz, np, os);
+      });
+      if (r.bad()) return r;
+    }
+    if (b > 0) {
+      r = pieces(std::max<int64_t>(a, 0), b, [&](int64_t L, int64_t lz, int64_t np) {
+        return X.d2h_planes(d, L * lt, lt, arr0(fin, L), lz, np, os);
+      });
+      if (r.bad()) return r;
+    }
+  }
+  // leave the domain resident at level T: the ring's top T planes from the scratch
+  r = pieces(nz - T, nz, [&](int64_t L, int64_t lz, int64_t np) {
+    const int64_t Ls = L - (nz / tz - nlo);
+    return X.copy_planes(d, scr[T & 1] + (int)(Ls * lt), arr0(fin, L), lt, lz, np, cs);
+  });
+  if (r.bad()) return r;
+  d.res_bit = fin;
+  for (int64_t k = 0; k < G.ntiles; ++k) {
+    d.tile_dirty[k] = 0;  // the host received u^T through the D2H above
+    d.tile_slot[k] = fin ? (int)(G.ntiles + k) : (int)k;
+  }
+  d.resident_valid = true;
+  d.faces_valid = d.xfaces_valid = false;  // faces are re-extracted by the next resident run
+  d.last_batches.clear();
+  return Status::ok();
+}
+
 static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool serial) {
   const bool load = !d.resident_valid;
   const int64_t nL = d.G.n[2];
   StreamPlan sp{};
-  if (load && !serial && streamthrough_ok(d, steps, &sp)) {
-    d.last_schedule = 2;
-    return run_streamthrough(d, alpha, steps, S, sp);
+  if (load && !serial) {  // fresh upload: stream-through, wavefront or the batched schedule
+    double est_st = 0;
+    WavePlan wp;
+    const bool st = streamthrough_ok(d, steps, &sp, &est_st);
+    const bool wf = wavefront_ok(d, steps, &wp);
+    const double nz = (double)d.G.l[2];
+    const double est_batched = 2.0 * nz + 0.011 * nz * steps;  // same fit as streamthrough_ok
+    bool take_wf = wf && (d.opt.wavefront > 0 || (d.opt.stream_through <= 0 && wp.est < est_batched &&
+                                                  (!st || wp.est < est_st)));
+    bool take_st = !take_wf && st && (d.opt.stream_through > 0 || est_st < est_batched);
+    if (take_wf) {
+      d.last_schedule = 6;
+      return run_wavefront(d, steps, S, wp);
+    }
+    if (take_st) {
+      d.last_schedule = 2;
+      return run_streamthrough(d, alpha, steps, S, sp);
+    }
   }
   d.last_schedule = serial ? 5 : 1;
   const std::vector<int> kp = plan_passes(d, steps);
@@ -1491,15 +1703,16 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams) {
     // transport's in-kernel push is HEAT7's; its exchange counters are
     // monotonic, so copy and fused exchanges interleave across runs)
     const bool direct = d.direct_ok, persist = d.persist_ok, x2 = d.x2_ok, fused = d.peer_fused;
-    const int32_t st_opt = d.opt.stream_through;
+    const int32_t st_opt = d.opt.stream_through, wf_opt = d.opt.wavefront;
     d.direct_ok = d.persist_ok = d.x2_ok = d.peer_fused = false;
-    d.opt.stream_through = -1;
+    d.opt.stream_through = d.opt.wavefront = -1;
     r = d.mode == MODE_RESIDENT ? run_heat_resident(d, 0.0, steps, S, serial) : run_stream(d, k, steps, S);
     d.direct_ok = direct;
     d.persist_ok = persist;
     d.x2_ok = x2;
     d.peer_fused = fused;
     d.opt.stream_through = st_opt;
+    d.opt.wavefront = wf_opt;
     if (r.bad()) return r;
     d.stats.steps_done += (uint64_t)steps;
     return Status::ok();

@@ -91,8 +91,12 @@ struct Domain;
 //   UNITS    - (source only) units u-1, u, u+1 of `un` planes each as packed
 //              sub-tiles at slots ring[0..2]; slab plane 0 at local z = zbase
 //              (wrapped), z in unit z / un.
+//   WAVE     - wavefront (runtime.cpp run_wavefront): the tile-blocked
+//              resident array `slot` (0/1) for planes z >= 0 (no wrap) and,
+//              for z < 0, ring[0] = first slot of un tile layers of scratch
+//              holding planes [-un*tz, 0).
 struct SlabRef {
-  enum Kind { DENSE = 0, RESIDENT = 1, SUB = 2, UNITS = 3 };
+  enum Kind { DENSE = 0, RESIDENT = 1, SUB = 2, UNITS = 3, WAVE = 4 };
   int kind;
   int slot;
   int64_t zbase;
@@ -120,6 +124,10 @@ struct Exec {
   virtual Status slab_sweep(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi,
                             int stream) = 0;
   virtual Status copy_slots(Domain& d, int src_slot, int dst_slot, int64_t n, int stream) = 0;
+  // planes [p0, p0+np) of n tile slots: slots s0.. -> host tiles t0.. (the
+  // same planes), and slots -> slots (wavefront)
+  virtual Status d2h_planes(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int stream) = 0;
+  virtual Status copy_planes(Domain& d, int src0, int dst0, int64_t n, int64_t p0, int64_t np, int stream) = 0;
   // planes [p0, p0+np) of n tiles; "packed" = n sub-tiles of np*ty*tx
   // elements back to back starting at a slot
   virtual Status h2d_part(Domain& d, int64_t tile0, int64_t n, int slot0, int64_t p0, int64_t np,
@@ -182,6 +190,12 @@ struct Domain {
   Fault fault;
   bool poisoned = false;
   int last_schedule = 0;  // tile_info.last_schedule
+  // wavefront scratch (allocated at its first use, within the budget):
+  // slots [nslots, nslots + wave_slots), whole tile layers
+  int wave_slots = 0;
+  double* wave_base = nullptr;
+  bool own_wave = false;
+  uint64_t budget_left = 0;  // device budget not carved by domain_setup
   int device = 0;
   int mode = MODE_RESIDENT;
   int measure = TILE_MEASURE_NORMAL;
@@ -298,7 +312,9 @@ struct Domain {
   double run_t0 = 0;
   bool kernel_timing = false;
 
-  double* slot_ptr(int s) const { return slot_base + (int64_t)s * G.tile_elems; }
+  double* slot_ptr(int s) const {
+    return s < nslots ? slot_base + (int64_t)s * G.tile_elems : wave_base + (int64_t)(s - nslots) * G.tile_elems;
+  }
   double* host_tile(int64_t k) const { return host + k * G.tile_elems; }
   const double* face_src_ptr(int64_t id, int f, int parity) const;
   const double* direct_src_ptr(int64_t id, int f, int bit, int parity) const;

@@ -35,7 +35,7 @@ OP_NAMES = {1: "h2d", 2: "d2h", 3: "kernel", 4: "record", 5: "wait", 6: "faces_h
             7: "extract", 8: "halo", 9: "drop", 10: "hit", 11: "pointwise", 12: "kernel2",
             13: "gather", 14: "sweep", 15: "scatter", 16: "copy", 17: "h2d_part", 18: "d2h_part",
             19: "copy_part", 20: "h2d_pack", 21: "sweep_u", 22: "kerneld", 23: "halo_signal",
-            24: "st_halo", 25: "sync"}
+            24: "st_halo", 25: "sync", 26: "wsweep", 27: "d2h_planes", 28: "copy_planes"}
 SCHEDS = {"auto": 0, "resident": 1, "stream": 2, "sync": 3}
 BCS = {"periodic": 0, "dirichlet": 1}
 
@@ -49,7 +49,7 @@ class TileOptions(ctypes.Structure):
                 ("dry_run", ctypes.c_int32), ("fuse_pointwise_steps", ctypes.c_int32),
                 ("local_group", ctypes.c_void_p), ("pageable_host", ctypes.c_int32),
                 ("stream_through", ctypes.c_int32), ("peer_transport", ctypes.c_int32),
-                ("two_step", ctypes.c_int32)]
+                ("two_step", ctypes.c_int32), ("wavefront", ctypes.c_int32)]
 
 
 class TileKernel(ctypes.Structure):
@@ -226,7 +226,7 @@ class Domain:
     def __init__(self, dims, tile_dims, ghost=1, bc="periodic", device=-1, device_budget_bytes=0,
                  sched="auto", nranks=1, rank=0, nccl_id=None, dry_run=False,
                  fuse_pointwise_steps=True, device_pool=None, streams=None, local_group=None,
-                 pageable_host=False, two_step=0, stream_through=0, peer_transport=False):
+                 pageable_host=False, two_step=0, stream_through=0, peer_transport=False, wavefront=0):
         self._h = None
         self._inflight = []  # kernel descriptors (user functions) of unsynchronised runs
         self.dims = tuple(int(v) for v in dims)
@@ -258,6 +258,7 @@ class Domain:
         o.pageable_host = 1 if pageable_host else 0
         o.two_step = int(two_step)
         o.stream_through = int(stream_through)
+        o.wavefront = int(wavefront)
         o.peer_transport = int(peer_transport)  # True/1: copy pushes; 2: fused kernel pushes
         self._group = local_group
         if local_group is not None:

@@ -62,6 +62,13 @@ class Geometry:
         return ("halo", 1, pos)
 
 
+def wsweep_range(c):
+    """lo, hi of a TILE_OP_WSWEEP (two signed 32-bit halves of c)."""
+    cu = c & 0xFFFFFFFFFFFFFFFF
+    s32 = lambda v: v - (1 << 32) if v & 0x80000000 else v
+    return s32(cu & 0xFFFFFFFF), s32(cu >> 32)
+
+
 def faces_of(u, D=1):
     """The D boundary layers of a tile per face, in increasing coordinate
     order: x-faces (tz,ty,D), y-faces (tz,D,tx), z-faces (D,ty,tx)."""
@@ -365,6 +372,27 @@ class Replayer:
                 for i in range(G.n[0] * G.n[1]):
                     ix, iy = i % G.n[0], i // G.n[0]
                     self.sub[(-a - 1, i)] = new[lo:hi, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx].copy()
+        elif name == "wsweep":
+            lo, hi = wsweep_range(c)
+            G = self.G
+            blk = np.stack([self.wave_get(a, p, d) for p in range(lo - 1, hi + 1)])
+            new = self.sweep(blk, None, 1, hi - lo + 1)
+            for p in range(lo, hi):
+                self.wave_set(b, p, d, new[p - lo + 1])
+        elif name == "d2h_planes":
+            p0, np_ = d & 0xffffffff, d >> 32
+            for i in range(c):
+                self.host[a + i] = self.host[a + i].copy()
+                self.host[a + i][p0:p0 + np_] = self.slots[b + i][p0:p0 + np_]
+        elif name == "copy_planes":
+            p0, np_ = d & 0xffffffff, d >> 32
+            for i in range(c):
+                src = self.slots[a + i][p0:p0 + np_].copy()
+                if b + i not in self.slots:
+                    self.slots[b + i] = np.full(self.host[0].shape, np.nan)
+                else:
+                    self.slots[b + i] = self.slots[b + i].copy()
+                self.slots[b + i][p0:p0 + np_] = src
         elif name == "h2d_pack":
             p0, np_ = d & 0xffffffff, d >> 32
             for i in range(c):
@@ -407,6 +435,46 @@ class Replayer:
                     out[p, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx] = self.slots[self.loc[t]][lz]
         return out
 
+    # ------------------------------------------------------------ wavefront
+    def _wave_loc(self, code, p, nlo):
+        """(first slot of the tile layer, plane in the tiles) of unwrapped
+        plane p in a TILE_OP_WSWEEP view: bit 0 set and p < 0: the scratch
+        tile layers at slot code >> 2 (nlo of them, planes [-nlo*tz, 0));
+        otherwise resident array (code >> 1) & 1, wrapped only for bit 0 = 0."""
+        G = self.G
+        tz, lt, nz = G.t[2], G.n[0] * G.n[1], G.l[2]
+        if code & 1 and p < 0:
+            q = p + nlo * tz
+            assert q >= 0, "wavefront read below its scratch"
+            return (code >> 2) + (q // tz) * lt, q % tz
+        if code & 1:
+            assert p < nz, "wavefront view read past the ring"
+        gz = p % nz
+        return ((code >> 1) & 1) * G.ntiles + (gz // tz) * lt, gz % tz
+
+    def wave_get(self, code, p, nlo):
+        G = self.G
+        tx, ty = G.t[0], G.t[1]
+        base, lz = self._wave_loc(code, p, nlo)
+        plane = np.full((G.l[1], G.l[0]), np.nan)
+        for i in range(G.n[0] * G.n[1]):
+            t = self.slots.get(base + i)
+            if t is not None:
+                ix, iy = i % G.n[0], i // G.n[0]
+                plane[iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx] = t[lz]
+        return plane
+
+    def wave_set(self, code, p, nlo, plane):
+        G = self.G
+        tx, ty = G.t[0], G.t[1]
+        base, lz = self._wave_loc(code, p, nlo)
+        for i in range(G.n[0] * G.n[1]):
+            s = base + i
+            t = self.slots[s].copy() if s in self.slots else np.full(self.host[0].shape, np.nan)
+            ix, iy = i % G.n[0], i // G.n[0]
+            t[lz] = plane[iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx]
+            self.slots[s] = t
+
     def sweep(self, src, dst, lo, hi):
         """One oracle step on planes [lo, hi), periodic in x and y; planes
         lo-1 and hi are the z neighbours (oracle.heat_np on a block whose
@@ -420,8 +488,9 @@ class Replayer:
         out[lo:hi] = new
         return out
 
-    def replay(self, trace, seed, st_ready=None, st_exec=None, timeout=120.0):
-        """Random valid order of one rank's trace. st_ready / st_exec: the
+    def replay(self, trace, seed, st_ready=None, st_exec=None, timeout=120.0, lazy=()):
+        """Random valid order of one rank's trace; ops named in `lazy` run
+        only when nothing else can (adversarial orders). st_ready / st_exec: the
         multi-process transport of stream-through halo ops (an op is runnable
         when st_ready(self, op); st_exec(self, op) performs it); while only
         such ops remain blocked the replay polls instead of failing."""
@@ -465,7 +534,8 @@ class Replayer:
                     time.sleep(0.002)  # a neighbour's halo layer is in flight
                     continue
                 raise RuntimeError("replay deadlock: no stream can make progress")
-            s = rng.choice(ready)
+            eager = [x for x in ready if trace[queues[x][pos[x]]][0] not in lazy]
+            s = rng.choice(eager or ready)
             i = queues[s][pos[s]]
             if trace[i][0] == "st_halo" and st_exec is not None:
                 st_exec(self, trace[i])

@@ -94,6 +94,22 @@ def _check_cone(dom, gdims, td, steps, blocks, b=2):
         assert np.array_equal(got, ref), (z0, y0, x0, np.abs(got - ref).max())
 
 
+def test_c2_wavefront_fig5_path():
+    """C2 512^3, 64^3 tiles, 4 streams, a fresh upload with T = 64 (the
+    Fig. 5 sweep's mid range, bench.py --config fig5): the cost model takes
+    the wavefront; sampled blocks at the tile, chunk and periodic seams vs
+    the cone oracle, bit-exact."""
+    n, td = 512, (64, 64, 64)
+    gdims = (n, n, n)
+    with T.Domain(gdims, td) as d:
+        _fill(d, gdims, td, 42)
+        d.run(T.heat7(ALPHA), 64, 4)
+        d.sync()
+        assert d.get_info()["last_schedule"] == 6
+        blocks = _seam_blocks(gdims, td, 2)[:5] + [(n - 64, 7, 300), (n - 1, n - 1, n - 1), (n - 130, 0, 0)]
+        _check_cone(d, gdims, td, 64, blocks)
+
+
 def test_c2_value_path_persistent_resident():
     """C2 512^3, 64^3 tiles, 4 streams: the first run after the upload is the
     e2e (stream-through) path, the next two are bench.py's `value` path

@@ -404,6 +404,36 @@ def test_stream_through_bit_exact(dims, td, T):
     assert st["bytes_h2d"] == nx * ny * nz * 8 and st["bytes_d2h"] == nx * ny * nz * 8
 
 
+@pytest.mark.parametrize("dims,td,T", [((64, 32, 128), (32, 16, 16), 20), ((128, 64, 256), (64, 64, 32), 48),
+                                       ((64, 64, 64), (32, 32, 8), 7), ((96, 64, 160), (32, 32, 32), 1),
+                                       ((64, 32, 512), (32, 32, 64), 100), ((512, 64, 128), (64, 64, 64), 16)])
+def test_wavefront_bit_exact(dims, td, T):
+    """Fresh-upload runs on the time-skewed wavefront (forced): chunks of
+    planes, level s of chunk i on planes [c*i - s, c*i + c - s), the seam's
+    bootstrap trapezoid in the scratch layers, each chunk's final planes
+    back to the host as soon as it ends; the host result, the kept device
+    copy (a following resident run) and a second wavefront run are exact,
+    and every cell crossed the link once per direction."""
+    nx, ny, nz = dims
+    u0 = synth.uniform_grid(nx, ny, nz, 42)
+    with T_.Domain(dims, td, wavefront=1) as d:
+        d.load(u0)
+        d.run(T_.heat7(), T, 2)
+        out1 = d.store()
+        st = d.stats()
+        sched = d.get_info()["last_schedule"]
+        d.run(T_.heat7(), 3, 2)   # continues from the device copy
+        out2 = d.store()
+        d.invalidate()
+        d.run(T_.heat7(), T, 4)   # a second fresh upload of u^{T+3}
+        out3 = d.store()
+    assert sched == 6
+    assert np.array_equal(out1, oracle.heat_c(u0, ALPHA, T))
+    assert np.array_equal(out2, oracle.heat_c(u0, ALPHA, T + 3))
+    assert np.array_equal(out3, oracle.heat_c(u0, ALPHA, 2 * T + 3))
+    assert st["bytes_h2d"] == nx * ny * nz * 8 and st["bytes_d2h"] == nx * ny * nz * 8
+
+
 @pytest.mark.parametrize("td,runs", [((32, 64, 8), [1, 4]), ((32, 128, 8), [2, 5])])
 def test_banded_round_robin_snake_bit_exact(td, runs):
     """Banded tiles (ty > band) with enough columns for the round-robin

@@ -17,7 +17,7 @@ import pytest
 
 import oracle
 import synth
-from tests.replay import Geometry, Replayer, split_tiles
+from tests.replay import Geometry, Replayer, split_tiles, wsweep_range
 
 T = pytest.importorskip("paper_conf_icpp_bastemuzas17_b200.tiles")
 
@@ -101,7 +101,7 @@ def _budget_for(dims, td, nslots, **kw):
     return lo
 
 
-def _run_and_replay(dims, td, steps_list, nstreams, seeds=(0, 1, 2), bc="periodic", ghost=1, **kw):
+def _run_and_replay(dims, td, steps_list, nstreams, seeds=(0, 1, 2), bc="periodic", ghost=1, lazy=(), **kw):
     nx, ny, nz = dims
     if bc == "periodic":
         u0 = synth.uniform_grid(nx, ny, nz, 42)
@@ -120,7 +120,7 @@ def _run_and_replay(dims, td, steps_list, nstreams, seeds=(0, 1, 2), bc="periodi
             d.clear_trace()
             d.run(T.heat7(ALPHA), steps, nstreams)
             d.sync()
-            rep.replay(d.trace(), seed)
+            rep.replay(d.trace(), seed, lazy=lazy)
         out = rep.grid()
         assert np.array_equal(out, ref), np.abs(out - ref).max()
     return d
@@ -321,14 +321,14 @@ def test_stream_through_schedule_replays_to_oracle(dims, td, T, ns):
     """Fresh-upload heat runs with T <= tz use the stream-through schedule
     (per-unit T shrinking sweeps, resident array -> slabs -> sub-tiles, D2H); replayed in random
     valid orders it must give the oracle bit-exactly."""
-    d = _run_and_replay(dims, td, [T], ns, seeds=(0, 1, 2))
+    d = _run_and_replay(dims, td, [T], ns, seeds=(0, 1, 2), wavefront=-1)
     ops = [op[0] for op in d.trace()]
     assert "sweep" in ops and "h2d_part" in ops and "d2h_part" in ops
     sw = [op for op in d.trace() if op[0] == "sweep"]
     assert any(op[2] < 0 for op in sw) and any(op[3] < 0 for op in sw)   # fused gather / scatter
     assert d.get_info()["resident"]
     # then a resident continuation and a second stream-through
-    _run_and_replay(dims, td, [T, T], ns, seeds=(3,))
+    _run_and_replay(dims, td, [T, T], ns, seeds=(3,), wavefront=-1)
 
 
 @pytest.mark.parametrize("dims,td,nslots,runs,ns", [
@@ -484,3 +484,64 @@ def test_stream_pointwise_then_heat_without_sync(first, nslots):
         rep.replay(d.trace(), seed)
         assert np.array_equal(rep.grid(), ref), np.abs(rep.grid() - ref).max()
         _trace_through_state_machine(d.trace(), nslots)
+
+
+@pytest.mark.parametrize("dims,td,T,ns,runs_after", [
+    ((16, 8, 64), (8, 4, 16), 3, 2, []),          # chunk 16 = tz / 1, bootstrap 16 planes
+    ((16, 8, 128), (8, 4, 16), 20, 3, [2]),       # T > tz: nlo = 3 scratch layers
+    ((16, 16, 96), (8, 8, 32), 17, 1, [5]),       # B = 48 (not a layer multiple)
+    ((8, 8, 64), (8, 8, 8), 7, 2, [3, 1]),        # tz = 8 < chunk: c = 8
+    ((16, 8, 80), (8, 8, 16), 1, 2, []),          # T = 1: no bootstrap sweep
+    ((16, 8, 160), (8, 4, 32), 40, 4, [])])       # long run, 3 layers of scratch
+def test_wavefront_schedule_replays_to_oracle(dims, td, T, ns, runs_after):
+    """Fresh-upload heat runs on the time-skewed wavefront (run_wavefront):
+    replayed in random valid orders the trace gives the untiled oracle
+    bit-exactly — a missing dependency, a WAR on a level buffer or a wrong
+    scratch mapping reads NaN or stale planes — moves every cell across the
+    link exactly once per direction, leaves the domain resident for the
+    following runs, and sweeps each cell once per step plus the ~T^2 bootstrap."""
+    d = _run_and_replay(dims, td, [T] + runs_after, ns, seeds=(0, 1, 2), wavefront=1)
+    assert d.get_info()["resident"]
+    # adversarial orders: uploads as late as their waits allow (a sweep that
+    # does not wait for its chunk reads NaN), then sweeps as late as possible
+    # (a D2H or copy that does not wait for its iteration moves stale planes)
+    for lazy in (("h2d_part",), ("wsweep",)):
+        _run_and_replay(dims, td, [T], ns, seeds=(5,), wavefront=1, lazy=lazy)
+    # the wavefront run on its own: ops, link bytes and swept cells
+    d2 = T_run_dry(dims, td, T, ns, wavefront=1)
+    ops = [op[0] for op in d2.trace()]
+    assert "wsweep" in ops and "d2h_planes" in ops and "sweep" not in ops
+    st = d2.stats()
+    cells = dims[0] * dims[1] * dims[2]
+    assert st["bytes_h2d"] == cells * 8 and st["bytes_d2h"] == cells * 8
+    assert d2.get_info()["last_schedule"] == 6
+    planes = 0
+    for op in d2.trace():
+        if op[0] == "wsweep":
+            lo, hi = wsweep_range(op[4])
+            planes += hi - lo
+    assert planes == dims[2] * T + sum(max(0, 2 * T - 2 * t) for t in range(1, T))
+
+
+def T_run_dry(dims, td, steps, ns, **kw):
+    d = T.Domain(dims, td, dry_run=True, **kw)
+    d.load(np.zeros(dims[::-1]))
+    d.run(T.heat7(ALPHA), steps, ns)
+    d.sync()
+    return d
+
+
+def test_wavefront_cost_model_choice():
+    """The fresh-upload schedule choice (cost model, link-plane units): at
+    C2 shape, stream-through at T = 10, the wavefront at T = 32..100, the
+    batched schedule where the seam's cone covers the ring."""
+    dims, td = (512, 512, 512), (64, 64, 64)
+    sched = {}
+    for steps in (10, 32, 64, 100, 300):
+        d = T.Domain(dims, td, dry_run=True)
+        d.invalidate()
+        d.run(T.heat7(ALPHA), steps, 4)
+        sched[steps] = d.get_info()["last_schedule"]
+        d.free()
+    assert sched[10] == 2 and sched[32] == 6 and sched[64] == 6 and sched[100] == 6
+    assert sched[300] == 1
