@@ -182,6 +182,14 @@ typedef struct {
                                    never, 0 (default) = when the cost model
                                    prefers it to stream-through and the
                                    batched schedule, 1 = whenever feasible */
+  double sweep_link_ratio;      /* cost model of the fresh-upload schedules
+                                   (DESIGN.md §5): time of one stencil sweep
+                                   per plane over one plane's duplex host-link
+                                   time. 0 (default) = measured on the device
+                                   at tile_domain_create (a few ms: up to
+                                   64 MiB of H2D and a 16-plane sweep, resident
+                                   single-rank domains), else env TILES_ST_R,
+                                   else 0.021 */
 } tile_options;
 
 typedef struct {
@@ -222,6 +230,7 @@ typedef struct {
                              upload), 3 out-of-core per-tile stream, 4
                              out-of-core stream-through, 5 synchronous (one
                              stream), 6 wavefront (fresh upload) */
+  double sweep_link_ratio; /* the cost model's ratio in use (see tile_options) */
 } tile_info;
 
 /* One entry of the dry-run trace. */

@@ -174,6 +174,7 @@ tile_status tile_get_info(const tile_domain* h, tile_info* o) {
   o->host_bytes = d.host_bytes;
   o->steps_per_pass = d.x2_ok && (d.opt.two_step > 0 || d.mode == tiles::MODE_STREAM) ? 2 : 1;
   o->last_schedule = d.last_schedule;
+  o->sweep_link_ratio = d.r_sweep;
   return TILE_OK;
 }
 

@@ -340,6 +340,23 @@ struct CudaExec final : Exec {
     return Status::ok();
   }
   int coop = 0;  // cudaDevAttrCooperativeLaunch
+  SweepMaps maps{};
+  bool maps_tried = false;
+  const double* maps_wave = nullptr;
+  // tensor maps of the slot pool and the wavefront scratch (x halos of the
+  // tile-column sweep), encoded once per allocation
+  void ensure_maps(Domain& d) {
+    if (!maps_tried) {
+      maps_tried = true;
+      sweep_map_encode(&maps, 0, d.slot_base, (uint64_t)d.nslots * d.G.tile_elems * 8, (int)d.G.t[0],
+                       sweep_tile_band());
+    }
+    if (d.wave_base && maps_wave != d.wave_base) {
+      maps_wave = d.wave_base;
+      sweep_map_encode(&maps, 1, d.wave_base, (uint64_t)d.wave_slots * d.G.tile_elems * 8, (int)d.G.t[0],
+                       sweep_tile_band());
+    }
+  }
   SlabView slab_view(Domain& d, const SlabRef& r, int lo) {
     const Geometry& G = d.G;
     SlabView v{};
@@ -349,10 +366,11 @@ struct CudaExec final : Exec {
     v.ty = (int)G.t[1];
     v.tz = 1 << 30;
     if (r.kind == SlabRef::DENSE) {
+      // scratch slab, tile-blocked like the packed sub-tiles: [tile (x, y)]
+      // [plane < slab_depth][ty][tx], so the sweep kernels stage bands of
+      // rows as single contiguous ranges
       v.base = d.slot_ptr(r.slot);
-      v.tx = (int)G.l[0];
-      v.ty = (int)G.l[1];
-      v.ntx = v.nty = 1;
+      v.te = d.slab_depth * G.t[0] * G.t[1];
     } else if (r.kind == SlabRef::RESIDENT) {
       v.base = d.slot_ptr(r.slot ? (int)G.ntiles : 0);
       v.te = G.tile_elems;
@@ -392,8 +410,9 @@ struct CudaExec final : Exec {
     if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
     const SlabView s = slab_view(d, src, lo), t = slab_view(d, dst, lo);
     next_cells = d.kernel_timing ? (uint64_t)(hi - lo) * d.G.l[0] * d.G.l[1] : 0;
+    ensure_maps(d);
     Status r = timed(d, st, [&] {
-      return launch_slab_sweep(s, t, (int)d.G.l[0], (int)d.G.l[1], lo, hi, d.kernel_alpha, sms, S(st));
+      return launch_slab_sweep(s, t, (int)d.G.l[0], (int)d.G.l[1], lo, hi, d.kernel_alpha, sms, S(st), &maps);
     });
     if (r.bad()) return r;
     d.stats.n_kernels++;
@@ -595,6 +614,70 @@ struct CudaExec final : Exec {
     INJECT(FAULT_SYNC, 0);
     for (auto s : streams) CK(cudaStreamSynchronize(s));
     return collect(d);
+  }
+  // Link: best of 3 H2D copies of up to 64 MiB from the pinned tile store
+  // (duplex H2D runs at ~0.87 of the solo rate on PCIe 5, pcie_gap.json).
+  // Sweep: best of 3 sweeps of 16 planes between the two resident arrays
+  // (zeroed first: no uninitialised reads). Both timed with events on
+  // stream 0, before any user data exists.
+  Status calibrate(Domain& d, double* r) override {
+    *r = 0;
+    const Geometry& G = d.G;
+    const uint64_t plane_b = (uint64_t)G.l[0] * G.l[1] * 8;
+    const uint64_t nb = std::min<uint64_t>(64ull << 20, (uint64_t)G.ntiles * G.tile_elems * 8);
+    const int planes = 16;
+    cudaStream_t s0 = S(0);
+    cudaEvent_t a, b;
+    CK(cudaEventCreate(&a));
+    CK(cudaEventCreate(&b));
+    float best_l = 1e30f, best_s = 1e30f;
+    Status res = Status::ok();
+    ensure_maps(d);
+    auto run = [&]() -> cudaError_t {
+      cudaError_t e = cudaMemsetAsync(d.slot_ptr(0), 0, (size_t)planes * plane_b + plane_b, s0);
+      if (e != cudaSuccess) return e;
+      for (int i = 0; i < 4; ++i) {  // first rep warms the pinned pages
+        if ((e = cudaEventRecord(a, s0)) != cudaSuccess) return e;
+        if ((e = cudaMemcpyAsync(d.slot_ptr(0), d.host, nb, cudaMemcpyHostToDevice, s0)) != cudaSuccess) return e;
+        if ((e = cudaEventRecord(b, s0)) != cudaSuccess) return e;
+        if ((e = cudaEventSynchronize(b)) != cudaSuccess) return e;
+        float ms = 0;
+        cudaEventElapsedTime(&ms, a, b);
+        if (i) best_l = std::min(best_l, ms);
+      }
+      SlabView v{};
+      v.base = d.slot_ptr(0);
+      v.te = G.tile_elems;
+      v.tx = (int)G.t[0];
+      v.ty = (int)G.t[1];
+      v.tz = (int)G.t[2];
+      v.ntx = (int)G.n[0];
+      v.nty = (int)G.n[1];
+      v.nz = (int)G.l[2];
+      SlabView w = v;
+      w.base = d.slot_ptr((int)G.ntiles);
+      if ((e = cudaMemsetAsync(d.slot_ptr(0), 0, (size_t)G.ntiles * G.tile_elems * 8, s0)) != cudaSuccess) return e;
+      for (int i = 0; i < 4; ++i) {
+        if ((e = cudaEventRecord(a, s0)) != cudaSuccess) return e;
+        if ((e = launch_slab_sweep(v, w, (int)G.l[0], (int)G.l[1], 1, 1 + planes, 0.125, sms, s0, &maps)) !=
+            cudaSuccess)
+          return e;
+        if ((e = cudaEventRecord(b, s0)) != cudaSuccess) return e;
+        if ((e = cudaEventSynchronize(b)) != cudaSuccess) return e;
+        float ms = 0;
+        cudaEventElapsedTime(&ms, a, b);
+        if (i) best_s = std::min(best_s, ms);
+      }
+      return cudaSuccess;
+    };
+    const cudaError_t e = run();
+    cudaEventDestroy(a);
+    cudaEventDestroy(b);
+    if (e != cudaSuccess) return cuda_err(e, "calibration");
+    const double link_plane = (double)best_l / ((double)nb / (double)plane_b) / 0.87;  // ms per plane, duplex
+    const double sweep_plane = (double)best_s / planes;
+    if (link_plane > 0 && sweep_plane > 0) *r = sweep_plane / link_plane;
+    return res;
   }
   Status mem_info(Domain&, uint64_t* fr, uint64_t* tot) override {
     size_t f = 0, t = 0;

@@ -180,8 +180,25 @@ struct SlabView {
   double* hhi;                  // (multi-rank halo layer, nlo = 1; wavefront scratch), planes
   int nlo;                      // z >= nz (planes z-nz) from hhi, instead of the periodic wrap
 };
+// TMA tensor maps over the tile slots for the sweep kernel's x-halo columns
+// (2 x band cells per side, a strided column): [k] views memory [base[k],
+// end[k]) as rows of tx doubles (k = 0 the slot pool, 1 the wavefront
+// scratch); valid[k] = 0 when absent. Opaque 128-byte CUtensorMap blobs.
+struct alignas(64) TensorMapBlob {
+  unsigned char b[128];
+};
+struct SweepMaps {
+  TensorMapBlob xmap[2];
+  const double* base[2];
+  const double* end[2];
+  int valid[2];
+  int band;  // box rows the maps were encoded for
+};
+// encode map k over [base, base + bytes) as rows of tx doubles, box {2, band}
+bool sweep_map_encode(SweepMaps* m, int k, const double* base, uint64_t bytes, int tx, int band);
+int sweep_tile_band();  // box rows (band) of the tile-column sweep kernel
 cudaError_t launch_slab_sweep(const SlabView& src, const SlabView& dst, int nx, int ny, int lo,
-                              int hi, double alpha, int sms, cudaStream_t s);
+                              int hi, double alpha, int sms, cudaStream_t s, const SweepMaps* maps = nullptr);
 // Two-step kernel: returns false from heat2_plan if no specialisation fits.
 bool heat2_plan(int tx, int ty, int max_smem, int* band, size_t* smem);
 cudaError_t heat2_configure(int tx, int band, size_t smem, int* ctas_per_sm);

@@ -354,6 +354,21 @@ Status domain_setup(Domain& d) {
   d.nevents = d.ev_misc_base + 4 + d.halo_stream + 1 + 3;  // + 2 stream-through ring events, 1 halo push
   st = X.setup(d);
   if (st.bad()) return st;
+  // cost-model calibration: r = sweep time / duplex link time
+  // per plane. Explicit (tile_options.sweep_link_ratio, env TILES_ST_R), else
+  // measured here on the box when a fresh-upload schedule can use it, else
+  // the B200 + PCIe 5 fit (0.021)
+  d.r_sweep = 0.021;
+  if (d.opt.sweep_link_ratio > 0) {
+    d.r_sweep = d.opt.sweep_link_ratio;
+  } else if (const char* e = getenv("TILES_ST_R")) {
+    d.r_sweep = atof(e);
+  } else if (d.mode == MODE_RESIDENT && !multi && G.t[0] % 2 == 0 && G.l[2] >= 32) {
+    double r = 0;
+    st = X.calibrate(d, &r);
+    if (st.bad()) return st;
+    if (r > 0) d.r_sweep = r;
+  }
   if (multi && !d.opt.dry_run && !d.opt.local_group && !d.opt.peer_transport) {
     st = nccl_init(d);
     if (st.bad()) return st;
@@ -845,10 +860,7 @@ static bool streamthrough_ok(const Domain& d, int T, StreamPlan* sp, double* est
     const char* e = getenv("TILES_ST_MINUNIT");
     return e ? std::max<int64_t>(1, atoll(e)) : (int64_t)16;
   }();
-  static const double r_sweep = [] {
-    const char* e = getenv("TILES_ST_R");
-    return e ? atof(e) : 0.021;
-  }();
+  const double r_sweep = d.r_sweep;  // calibrated per box (domain_setup)
   const double nz = (double)G.l[2], Td = (double)T;
   int64_t unit = G.t[2];
   double best = 1e300;
@@ -894,6 +906,7 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
   const Pipes P(S, false);
   const int bit = d.res_bit;                       // H2D target array
   const int sb = bit ? 0 : (int)G.ntiles;          // scratch array (the other one)
+  d.slab_depth = sp.slab_tiles * G.tile_elems / (G.l[0] * G.l[1]);  // planes a slab holds
   const int slab[2] = {sb, sb + (int)sp.slab_tiles};
   const int out[2] = {sb + 2 * (int)sp.slab_tiles, sb + 2 * (int)sp.slab_tiles + (int)sp.sub_tiles};
   const int keep0 = sb + 2 * (int)sp.slab_tiles + 2 * (int)sp.sub_tiles;
@@ -1038,10 +1051,7 @@ static bool ooc_streamthrough_ok(const Domain& d, int T, OocPlan* op) {
   if (G.t[0] % 2 || G.l[2] > (1 << 30)) return false;
   const double nz = (double)G.l[2];
   const int64_t plane = G.l[0] * G.l[1];
-  static const double r_sweep = [] {
-    const char* e = getenv("TILES_ST_R");
-    return e ? atof(e) : 0.021;
-  }();
+  const double r_sweep = d.r_sweep;
   double best = 1e300;
   for (int64_t k = 2; k <= std::min<int64_t>(T, G.t[2]); ++k)
     for (int64_t un = k; un <= G.t[2]; ++un) {
@@ -1077,6 +1087,7 @@ static Status run_streamthrough_ooc(Domain& d, int T, int S, const OocPlan& op) 
   const Pipes P(S, false);
   const int64_t U = op.U, un = op.un, lt = G.layer_tiles, tz = G.t[2], R = op.R;
   const int cs = P.comp(0), os = P.out(0), is = P.in(0);
+  d.slab_depth = op.slab_slots * G.tile_elems / (G.l[0] * G.l[1]);  // planes a slab holds
   Status r;
   // flush: dirty resident tiles to the host, then nothing is resident
   {
@@ -1246,18 +1257,11 @@ struct WavePlan {
 static int64_t wave_chunk() {
   static const int64_t c = [] {
     const char* e = getenv("TILES_WAVE_C");
-    return e ? std::max<int64_t>(1, atoll(e)) : (int64_t)16;
+    return e ? std::max<int64_t>(1, atoll(e)) : (int64_t)32;  // C2 Fig. 5: 32 > 64 > 16 planes
   }();
   return c;
 }
 
-static double sweep_ratio() {  // sweep time / duplex link time per plane (see streamthrough_ok)
-  static const double r = [] {
-    const char* e = getenv("TILES_ST_R");
-    return e ? atof(e) : 0.021;
-  }();
-  return r;
-}
 
 static bool wavefront_ok(const Domain& d, int T, WavePlan* wp) {
   const Geometry& G = d.G;
@@ -1274,7 +1278,7 @@ static bool wavefront_ok(const Domain& d, int T, WavePlan* wp) {
   const uint64_t need = (uint64_t)(2 * nlo * G.layer_tiles) * (uint64_t)G.tile_elems * 8;
   if ((int64_t)d.wave_slots < 2 * nlo * G.layer_tiles && need > d.budget_left + (uint64_t)d.wave_slots * G.tile_elems * 8)
     return false;
-  const double r = sweep_ratio(), Td = (double)T, n = (double)nz;
+  const double r = d.r_sweep, Td = (double)T, n = (double)nz;
   wp->c = c;
   wp->B = B;
   wp->nlo = nlo;
@@ -1287,6 +1291,11 @@ static bool wavefront_ok(const Domain& d, int T, WavePlan* wp) {
 
 static Status ensure_wave_scratch(Domain& d, int64_t slots) {
   if (d.wave_slots >= slots) return Status::ok();
+  // room for up to 4 tile layers per parity when the budget allows, so runs
+  // with growing T do not reallocate (a reallocation synchronises)
+  const int64_t roomy = 2 * std::min<int64_t>(4, d.G.n[2] / 2) * d.G.layer_tiles;
+  const uint64_t avail = d.budget_left + (uint64_t)d.wave_slots * d.G.tile_elems * 8;
+  if (roomy > slots && (uint64_t)roomy * d.G.tile_elems * 8 <= avail / 2) slots = roomy;
   const uint64_t bytes = (uint64_t)slots * d.G.tile_elems * 8;
   if (d.own_wave && d.wave_base) {
     Status r = d.exec->sync_all(d);  // the old scratch may still be read
@@ -1420,7 +1429,11 @@ static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool 
     const bool st = streamthrough_ok(d, steps, &sp, &est_st);
     const bool wf = wavefront_ok(d, steps, &wp);
     const double nz = (double)d.G.l[2];
-    const double est_batched = 2.0 * nz + 0.011 * nz * steps;  // same fit as streamthrough_ok
+    // the batched schedule: both link directions in sequence plus T
+    // whole-domain steps partly overlapped (0.52 r per plane-step: the
+    // persistent heat7 step per plane over the duplex link-plane time, fitted
+    // with r on the Fig. 5 sweep)
+    const double est_batched = 2.0 * nz + 0.52 * d.r_sweep * nz * steps;
     bool take_wf = wf && (d.opt.wavefront > 0 || (d.opt.stream_through <= 0 && wp.est < est_batched &&
                                                   (!st || wp.est < est_st)));
     bool take_st = !take_wf && st && (d.opt.stream_through > 0 || est_st < est_batched);

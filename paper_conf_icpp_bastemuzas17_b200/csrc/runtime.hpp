@@ -156,6 +156,9 @@ struct Exec {
   virtual Status st_halo(Domain& d, int op, int side, int T, int stream) = 0;
   virtual Status note(Domain& d, int kind, int64_t a, int64_t b, int stream) = 0;  // trace-only ops
   virtual Status sync_all(Domain& d) = 0;
+  // cost-model calibration: *r = one sweep's time per plane / one plane's
+  // duplex host-link time, measured on this device (0: not measured)
+  virtual Status calibrate(Domain& d, double* r) = 0;
   // resources
   virtual Status mem_info(Domain& d, uint64_t* free_b, uint64_t* total_b) = 0;
   virtual Status alloc_host(Domain& d, uint64_t bytes, void** p) = 0;
@@ -190,6 +193,7 @@ struct Domain {
   Fault fault;
   bool poisoned = false;
   int last_schedule = 0;  // tile_info.last_schedule
+  double r_sweep = 0.021;  // cost model: sweep / duplex link time per plane (calibrated at setup)
   // wavefront scratch (allocated at its first use, within the budget):
   // slots [nslots, nslots + wave_slots), whole tile layers
   int wave_slots = 0;
@@ -234,6 +238,7 @@ struct Domain {
   uint8_t* fixed_mask_dev = nullptr;       // per tile: Dirichlet faces (bit f)
   std::vector<uint8_t> fixed_mask_host;
   int64_t st_unit = 0;                     // stream-through unit (planes) of the current run
+  int64_t slab_depth = 0;                  // planes per stream-through scratch slab (tile-blocked)
   bool x2_ok = false;                      // two-step passes available
   int band2 = 0, heat2_grid = 0;
   size_t heat2_smem = 0;

@@ -49,7 +49,8 @@ class TileOptions(ctypes.Structure):
                 ("dry_run", ctypes.c_int32), ("fuse_pointwise_steps", ctypes.c_int32),
                 ("local_group", ctypes.c_void_p), ("pageable_host", ctypes.c_int32),
                 ("stream_through", ctypes.c_int32), ("peer_transport", ctypes.c_int32),
-                ("two_step", ctypes.c_int32), ("wavefront", ctypes.c_int32)]
+                ("two_step", ctypes.c_int32), ("wavefront", ctypes.c_int32),
+                ("sweep_link_ratio", ctypes.c_double)]
 
 
 class TileKernel(ctypes.Structure):
@@ -74,7 +75,8 @@ class TileInfo(ctypes.Structure):
                 ("ntiles", ctypes.c_int64), ("z_offset", ctypes.c_int64), ("ghost", ctypes.c_int32),
                 ("nslots", ctypes.c_int32), ("sched", ctypes.c_int32), ("resident", ctypes.c_int32),
                 ("device_bytes", ctypes.c_uint64), ("host_bytes", ctypes.c_uint64),
-                ("steps_per_pass", ctypes.c_int32), ("last_schedule", ctypes.c_int32)]
+                ("steps_per_pass", ctypes.c_int32), ("last_schedule", ctypes.c_int32),
+                ("sweep_link_ratio", ctypes.c_double)]
 
     def as_dict(self):
         out = {}
@@ -226,7 +228,8 @@ class Domain:
     def __init__(self, dims, tile_dims, ghost=1, bc="periodic", device=-1, device_budget_bytes=0,
                  sched="auto", nranks=1, rank=0, nccl_id=None, dry_run=False,
                  fuse_pointwise_steps=True, device_pool=None, streams=None, local_group=None,
-                 pageable_host=False, two_step=0, stream_through=0, peer_transport=False, wavefront=0):
+                 pageable_host=False, two_step=0, stream_through=0, peer_transport=False, wavefront=0,
+                 sweep_link_ratio=0.0):
         self._h = None
         self._inflight = []  # kernel descriptors (user functions) of unsynchronised runs
         self.dims = tuple(int(v) for v in dims)
@@ -259,6 +262,7 @@ class Domain:
         o.two_step = int(two_step)
         o.stream_through = int(stream_through)
         o.wavefront = int(wavefront)
+        o.sweep_link_ratio = float(sweep_link_ratio)
         o.peer_transport = int(peer_transport)  # True/1: copy pushes; 2: fused kernel pushes
         self._group = local_group
         if local_group is not None:

@@ -442,3 +442,16 @@ def test_banded_round_robin_snake_bit_exact(td, runs):
     dims = (512, 512, 16)
     out, ref, _, _ = _heat(dims, td, sum(runs), runs=runs)
     assert np.array_equal(out, ref), np.abs(out - ref).max()
+
+
+def test_cost_model_calibrated_on_device():
+    """tile_domain_create measures the fresh-upload cost model's ratio (one
+    sweep's time per plane / one plane's duplex host-link time) on the box;
+    an explicit tile_options value overrides it."""
+    d = T_.Domain((512, 512, 512), (64, 64, 64))
+    r = d.get_info()["sweep_link_ratio"]
+    d.free()
+    assert 0.003 < r < 0.2, r
+    d = T_.Domain((512, 512, 512), (64, 64, 64), sweep_link_ratio=0.05)
+    assert d.get_info()["sweep_link_ratio"] == 0.05
+    d.free()

@@ -545,3 +545,21 @@ def test_wavefront_cost_model_choice():
         d.free()
     assert sched[10] == 2 and sched[32] == 6 and sched[64] == 6 and sched[100] == 6
     assert sched[300] == 1
+
+
+def test_cost_model_ratio_option_and_report():
+    """tile_options.sweep_link_ratio sets the fresh-upload cost model's
+    sweep / link time ratio (dry runs: else the 0.021 fit); tile_info
+    reports it, and it moves the schedule choice: a slow sweep (large ratio)
+    sends a T = 32 run to the batched schedule, a fast one to the wavefront."""
+    dims, td = (512, 512, 512), (64, 64, 64)
+    d = T.Domain(dims, td, dry_run=True)
+    assert abs(d.get_info()["sweep_link_ratio"] - 0.021) < 1e-12
+    got = {}
+    for r in (0.005, 0.021, 0.2):
+        d = T.Domain(dims, td, dry_run=True, sweep_link_ratio=r)
+        assert d.get_info()["sweep_link_ratio"] == r
+        d.invalidate()
+        d.run(T.heat7(ALPHA), 32, 4)
+        got[r] = d.get_info()["last_schedule"]
+    assert got[0.005] == 6 and got[0.021] == 6 and got[0.2] == 1
