@@ -187,7 +187,7 @@ typedef struct {
                                    per plane over one plane's duplex host-link
                                    time. 0 (default) = measured on the device
                                    at tile_domain_create (a few ms: up to
-                                   64 MiB of H2D and a 16-plane sweep, resident
+                                   64 MiB of H2D and a 32-plane sweep, resident
                                    single-rank domains), else env TILES_ST_R,
                                    else 0.021 */
 } tile_options;

@@ -617,7 +617,7 @@ struct CudaExec final : Exec {
   }
   // Link: best of 3 H2D copies of up to 64 MiB from the pinned tile store
   // (duplex H2D runs at ~0.87 of the solo rate on PCIe 5, pcie_gap.json).
-  // Sweep: best of 3 sweeps of 16 planes between the two resident arrays
+  // Sweep: best of 3 sweeps of 32 planes between the two resident arrays
   // (zeroed first: no uninitialised reads). Both timed with events on
   // stream 0, before any user data exists.
   Status calibrate(Domain& d, double* r) override {
@@ -625,7 +625,7 @@ struct CudaExec final : Exec {
     const Geometry& G = d.G;
     const uint64_t plane_b = (uint64_t)G.l[0] * G.l[1] * 8;
     const uint64_t nb = std::min<uint64_t>(64ull << 20, (uint64_t)G.ntiles * G.tile_elems * 8);
-    const int planes = 16;
+    const int planes = (int)std::min<int64_t>(32, G.l[2] - 2);  // a wavefront chunk
     cudaStream_t s0 = S(0);
     cudaEvent_t a, b;
     CK(cudaEventCreate(&a));

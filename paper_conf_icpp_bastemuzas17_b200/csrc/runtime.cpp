@@ -1285,7 +1285,9 @@ static bool wavefront_ok(const Domain& d, int T, WavePlan* wp) {
   // the bootstrap waits for the top B planes and sweeps ~T^2 planes; then
   // the march is bound by the link (every plane down once, the rest up) or
   // by its T sweeps per plane; one chunk of fill/drain
-  wp->est = (double)B + r * Td * Td + std::max(n, r * n * Td) + (double)c * (1.0 + r * Td);
+  // (the bootstrap's sweeps are thick, about 0.7 of a chunk sweep's cost per
+  // plane, fitted on the Fig. 5 sweep at T = 64 and 100)
+  wp->est = (double)B + 0.7 * r * Td * Td + std::max(n, r * n * Td) + (double)c * (1.0 + r * Td);
   return true;
 }
 
