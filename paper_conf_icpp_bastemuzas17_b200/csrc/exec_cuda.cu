@@ -576,7 +576,8 @@ struct CudaExec final : Exec {
       p.fexp[f] = d.faces[f][par];
       p.face_elems[f] = d.G.face_elems[f];
     }
-    CK(launch_extract(p, S(st)));
+    Status r = timed(d, st, [&] { return launch_extract(p, S(st)); });
+    if (r.bad()) return r;
     d.stats.n_kernels++;
     return Status::ok();
   }

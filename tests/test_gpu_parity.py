@@ -253,8 +253,10 @@ def test_kernel_timing_and_device_timer():
         d.run(T.heat7(), 4, 1)
         ms = d.timer_stop()
         st = d.stats()
-    # 4 steps: one persistent multi-step launch (default) or 4 launches (TILES_PERSIST=0)
-    assert st["n_kernels"] in (1, 4) and st["kernel_timed"] == st["n_kernels"]
+    # 4 steps: one persistent multi-step launch (default) or 4 launches
+    # (TILES_PERSIST=0), plus one face extraction when the first run took a
+    # fresh-upload schedule that leaves the faces to the next resident run
+    assert st["n_kernels"] in (1, 2, 4, 5) and st["kernel_timed"] == st["n_kernels"]
     assert ms > 0 and 0 < st["kernel_ms"] <= ms * 1.01
 
 
