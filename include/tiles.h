@@ -328,6 +328,27 @@ tile_status tile_load(tile_domain* dom, const double* src);
 tile_status tile_host_tile(tile_domain* dom, int64_t tile_id, double** ptr);
 tile_status tile_mark_host_dirty(tile_domain* dom);
 
+/* GPU-disabled request of one region (§IV.B.4): if the tile's newest
+ * data is on the device it is copied back on its stream and waited for
+ * (P:L86), then *ptr = the tile's interior in the pinned host store
+ * (contiguous [tz][ty][tx]). TILE_HOST_READ keeps the device copy (clean);
+ * TILE_HOST_WRITE also drops it because CPU code will change the host data:
+ * in the streaming schedule the tile's slot is freed, in the resident one
+ * every device-newer tile is written back and the next run re-uploads the
+ * domain. Valid until the next tile_run / tile_load / tile_free. */
+typedef enum { TILE_HOST_READ = 0, TILE_HOST_WRITE = 1 } tile_host_mode;
+tile_status tile_host_region(tile_domain* dom, int64_t tile_id, int32_t mode, double** ptr);
+
+/* Host-side ghost update (§III, §IV.B.6: the ghost cells of a
+ * region on the host are updated on the host): fills out (out_len >=
+ * (tx+2g)(ty+2g)(tz+2g), layout of tile_ghost_map) with tile `tile_id` and
+ * its g-deep shell from the host store — periodic wrap, Dirichlet fixed
+ * faces (shell cells outside the domain in two or three axes are NaN: the
+ * 7-point stencil never reads them). Device-newer tiles are written back
+ * first (implicit tile_sync). z-slab ranks: TILE_EINVAL for tiles whose
+ * shell reaches another rank. */
+tile_status tile_host_ghosts(tile_domain* dom, int64_t tile_id, double* out, int64_t out_len);
+
 /* Enqueue `steps` steps of kernel k over every tile (no sync
  * after issue). nstreams in [1, 64] streams carry transfers and kernels
  * (P:L81-L84). Returns once all work is enqueued; may block only for

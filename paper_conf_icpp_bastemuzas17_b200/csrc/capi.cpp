@@ -66,6 +66,22 @@ tile_status tile_host_tile(tile_domain* h, int64_t tile_id, double** ptr) {
   return TILE_OK;
 }
 
+tile_status tile_host_region(tile_domain* h, int64_t tile_id, int32_t mode, double** ptr) {
+  CHECK_DOM(h);
+  if (!ptr || tile_id < 0 || tile_id >= h->d->G.ntiles) return fail(TILE_EINVAL, "bad tile id");
+  if (mode != TILE_HOST_READ && mode != TILE_HOST_WRITE) return fail(TILE_EINVAL, "bad host mode");
+  return finish(h, tiles::domain_host_region(*h->d, tile_id, mode, ptr));
+}
+
+tile_status tile_host_ghosts(tile_domain* h, int64_t tile_id, double* out, int64_t out_len) {
+  CHECK_DOM(h);
+  const tiles::Geometry& G = h->d->G;
+  if (!out || tile_id < 0 || tile_id >= G.ntiles) return fail(TILE_EINVAL, "bad tile id or out");
+  const int64_t need = (G.t[0] + 2 * G.ghost) * (G.t[1] + 2 * G.ghost) * (G.t[2] + 2 * G.ghost);
+  if (out_len < need) return fail(TILE_EINVAL, "out_len too small");
+  return finish(h, tiles::domain_host_ghosts(*h->d, tile_id, out));
+}
+
 tile_status tile_mark_host_dirty(tile_domain* h) {
   CHECK_DOM(h);
   Domain& d = *h->d;

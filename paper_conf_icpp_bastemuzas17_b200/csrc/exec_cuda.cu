@@ -429,10 +429,36 @@ struct CudaExec final : Exec {
     d.stats.n_h2d++;
     return Status::ok();
   }
+  // TILES_D2H_KERNEL=N (N > 0 CTAs): partial D2H copies by the SMs into the
+  // mapped host store instead of the copy engine (experiment)
+  int push_ctas() {
+    static const int n = [] {
+      const char* e = getenv("TILES_D2H_KERNEL");
+      return e ? atoi(e) : 0;
+    }();
+    return n;
+  }
+  double* host_dev(Domain& d, int64_t t) {
+    if (!host_dptr) {
+      void* p = nullptr;
+      if (cudaHostGetDevicePointer(&p, d.host, 0) != cudaSuccess) return nullptr;
+      host_dptr = static_cast<double*>(p);
+    }
+    return host_dptr + t * d.G.tile_elems;
+  }
+  double* host_dptr = nullptr;
   Status d2h_part(Domain& d, int64_t t0, int64_t n, int ps, int64_t p0, int64_t np, int st) override {
     INJECT(FAULT_D2H, st);
     if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
     const size_t pl = (size_t)d.G.t[0] * d.G.t[1] * 8, tb = (size_t)d.G.tile_elems * 8;
+    if (push_ctas() > 0 && !d.opt.pageable_host && host_dev(d, t0)) {
+      const int64_t pe = (int64_t)(pl / 8);
+      CK(launch_push_rows(d.slot_ptr(ps), np * pe, host_dev(d, t0) + p0 * pe, d.G.tile_elems, n, np * pe,
+                          push_ctas(), S(st)));
+      d.stats.bytes_d2h += (uint64_t)n * np * pl;
+      d.stats.n_d2h++;
+      return Status::ok();
+    }
     CK(cudaMemcpy2DAsync(reinterpret_cast<char*>(d.host_tile(t0)) + p0 * pl, tb, d.slot_ptr(ps),
                          np * pl, np * pl, (size_t)n, cudaMemcpyDeviceToHost, S(st)));
     d.stats.bytes_d2h += (uint64_t)n * np * pl;
@@ -460,6 +486,14 @@ struct CudaExec final : Exec {
     INJECT(FAULT_D2H, st);
     if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();
     const size_t pl = (size_t)d.G.t[0] * d.G.t[1] * 8, tb = (size_t)d.G.tile_elems * 8;
+    if (push_ctas() > 0 && !d.opt.pageable_host && host_dev(d, t0)) {
+      const int64_t pe = (int64_t)(pl / 8);
+      CK(launch_push_rows(d.slot_ptr(s0) + p0 * pe, d.G.tile_elems, host_dev(d, t0) + p0 * pe, d.G.tile_elems, n,
+                          np * pe, push_ctas(), S(st)));
+      d.stats.bytes_d2h += (uint64_t)n * np * pl;
+      d.stats.n_d2h++;
+      return Status::ok();
+    }
     CK(cudaMemcpy2DAsync(reinterpret_cast<char*>(d.host_tile(t0)) + p0 * pl, tb,
                          reinterpret_cast<const char*>(d.slot_ptr(s0)) + p0 * pl, tb, np * pl, (size_t)n,
                          cudaMemcpyDeviceToHost, S(st)));
@@ -697,7 +731,7 @@ struct CudaExec final : Exec {
     // pinned (page-locked) host regions, P:L73 (cudaMallocHost); an injected
     // fault asks for more than any host has
     const uint64_t req = fault_fires(d, FAULT_HOST_ALLOC) ? (1ull << 62) : (bytes ? bytes : 1);
-    cudaError_t e = cudaHostAlloc(p, req, cudaHostAllocPortable);
+    cudaError_t e = cudaHostAlloc(p, req, cudaHostAllocPortable | cudaHostAllocMapped);
     if (e != cudaSuccess) {
       cudaGetLastError();
       return make_err(TILE_ENOMEM_HOST, std::string("cudaHostAlloc: ") + cudaGetErrorString(e));

@@ -758,3 +758,29 @@ cudaError_t launch_extract(const ExtractParams& p, cudaStream_t s) {
 }
 
 }  // namespace tiles
+
+namespace tiles {
+
+// ---------------------------------------------------------------- push_rows
+// Device -> pinned host copy done by the SMs (the host store is mapped): n
+// rows of len double2, row r from src + r * sp to dst + r * dp (in double2
+// units). The copy engine then carries only host -> device traffic, and the
+// writes leave as posted PCIe writes from a few CTAs.
+__global__ void __launch_bounds__(256) push_rows(const double2* __restrict__ src, int64_t sp, double2* dst,
+                                                 int64_t dp, int64_t len) {
+  const double2* s = src + (int64_t)blockIdx.y * sp;
+  double2* d = dst + (int64_t)blockIdx.y * dp;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < len; i += (int64_t)gridDim.x * blockDim.x)
+    d[i] = __ldcs(s + i);
+}
+
+cudaError_t launch_push_rows(const double* src, int64_t src_pitch, double* dst, int64_t dst_pitch, int64_t rows,
+                             int64_t len, int ctas, cudaStream_t st) {
+  if (rows <= 0 || len <= 0) return cudaSuccess;
+  const int64_t gx = std::max<int64_t>(1, ctas / std::max<int64_t>(1, rows));
+  push_rows<<<dim3((unsigned)gx, (unsigned)rows), 256, 0, st>>>(
+      reinterpret_cast<const double2*>(src), src_pitch / 2, reinterpret_cast<double2*>(dst), dst_pitch / 2, len / 2);
+  return cudaGetLastError();
+}
+
+}  // namespace tiles

@@ -197,6 +197,10 @@ struct SweepMaps {
 // encode map k over [base, base + bytes) as rows of tx doubles, box {2, band}
 bool sweep_map_encode(SweepMaps* m, int k, const double* base, uint64_t bytes, int tx, int band);
 int sweep_tile_band();  // box rows (band) of the tile-column sweep kernel
+// device -> mapped pinned host rows copied by the SMs (pitches, len in doubles;
+// len and pitches even)
+cudaError_t launch_push_rows(const double* src, int64_t src_pitch, double* dst, int64_t dst_pitch, int64_t rows,
+                             int64_t len, int ctas, cudaStream_t st);
 cudaError_t launch_slab_sweep(const SlabView& src, const SlabView& dst, int nx, int ny, int lo,
                               int hi, double alpha, int sms, cudaStream_t s, const SweepMaps* maps = nullptr);
 // Two-step kernel: returns false from heat2_plan if no specialisation fits.

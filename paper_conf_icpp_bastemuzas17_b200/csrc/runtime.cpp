@@ -10,6 +10,7 @@
 //     paper's global `acc wait` (difference D3)
 //   D2H + synchronize before host access          -> domain_sync
 #include <algorithm>
+#include <cmath>
 #include <cstdlib>
 #include <cstring>
 #include <set>
@@ -1860,6 +1861,144 @@ Status domain_invalidate(Domain& d) {
       d.free_slots.push_back(s);
     }
   }
+  return Status::ok();
+}
+
+// GPU-disabled request of one region (§IV.B.4: "If programmer
+// requests a region on CPU ... TileAcc performs a check on cache list to see
+// if the region is on device", and if so copies it back first; the
+// D2H is waited for before the host pointer is returned). READ keeps the
+// device copy (now clean); WRITE also drops it, since the caller's CPU code
+// will change the host data (stream mode: the tile's slot is freed; resident
+// mode: every other device-newer tile is written back too and the next run
+// re-uploads the domain).
+Status domain_host_region(Domain& d, int64_t t, int mode, double** ptr) {
+  Exec& X = *d.exec;
+  Status r;
+  if (d.tile_dirty[t] && d.tile_slot[t] >= 0) {
+    const int sl = d.tile_slot[t];
+    int st = 0;
+    if (d.mode == MODE_STREAM) {
+      const Pipes P(d.last_S, false);
+      st = P.out(t);
+      r = X.wait(d, ev_slot(d, sl), st);
+      if (r.bad()) return r;
+    } else {
+      // after the kernel of the tile's layer that wrote it last
+      int64_t ix, iy, iz;
+      d.G.tile_coords(t, &ix, &iy, &iz);
+      bool found = false;
+      for (auto& b : d.last_batches)
+        if (iz >= b.L0 && iz < b.L1 && b.stream >= 0) {
+          st = b.out;
+          r = X.wait(d, b.ev, st);
+          if (r.bad()) return r;
+          found = true;
+        }
+      if (!found) {  // per-tile pipelines (pointwise kernels)
+        const Pipes P(d.last_S, d.last_serial);
+        st = P.out(t);
+        r = X.wait(d, ev_tile(d, t, 0), st);
+        if (r.bad()) return r;
+      }
+    }
+    r = X.d2h(d, t, 1, sl, st);
+    if (r.bad()) return r;
+    if (d.mode == MODE_STREAM) {
+      r = X.record(d, ev_slot(d, sl), st);
+      if (r.bad()) return r;
+      r = X.record(d, ev_host(d, t), st);
+      if (r.bad()) return r;
+    }
+    d.tile_dirty[t] = 0;
+    d.stats.writebacks++;
+  }
+  r = X.sync_all(d);  // the D2H above and any write-back still in flight
+  if (r.bad()) return r;
+  d.host_pending = false;
+  if (mode == TILE_HOST_WRITE) {
+    d.host_faces_valid = false;
+    if (d.mode == MODE_STREAM) {
+      const int sl = d.tile_slot[t];
+      if (sl >= 0) {
+        d.tile_slot[t] = -1;
+        d.slot_owner[sl] = -1;
+        d.free_slots.push_back(sl);
+      }
+      d.faces_valid = d.xfaces_valid = false;  // the tile's exported faces are stale too
+    } else if (d.resident_valid) {
+      r = domain_sync(d);  // the other device-newer tiles reach the host first
+      if (r.bad()) return r;
+      d.resident_valid = false;
+      d.faces_valid = d.xfaces_valid = false;
+      for (int64_t k = 0; k < d.G.ntiles; ++k) d.tile_slot[k] = -1;
+    }
+  }
+  if (d.in_flight) {
+    bool any = false;
+    for (int64_t k = 0; k < d.G.ntiles; ++k) any |= d.tile_dirty[k] != 0;
+    d.in_flight = any;
+  }
+  *ptr = d.host_tile(t);
+  return Status::ok();
+}
+
+// Host-side ghost update (§III, §IV.B.6: regions on the host get
+// their ghost cells updated on the host): tile t with its g-deep shell,
+// gathered from the host store through the ghost map — the periodic wrap, the
+// Dirichlet fixed faces (edge and corner cells outside the domain in two or
+// three axes are not stored: NaN), or, with z-slab ranks, only shells inside
+// the rank's slab (others: EINVAL). Device-newer tiles are written back first.
+Status domain_host_ghosts(Domain& d, int64_t t, double* out) {
+  const Geometry& G = d.G;
+  int64_t c[3];
+  G.tile_coords(t, &c[0], &c[1], &c[2]);
+  const int64_t g = G.ghost;
+  if (G.nranks > 1 && G.bc == TILE_BC_PERIODIC && (c[2] == 0 || c[2] == G.n[2] - 1))
+    return make_err(TILE_EINVAL, "ghost cells of this tile live on another rank");
+  if (G.nranks > 1 && G.bc == TILE_BC_DIRICHLET && ((c[2] == 0 && G.rank > 0) || (c[2] == G.n[2] - 1 && G.rank < G.nranks - 1)))
+    return make_err(TILE_EINVAL, "ghost cells of this tile live on another rank");
+  bool dirty = d.host_pending;
+  for (int64_t k = 0; k < G.ntiles && !dirty; ++k) dirty = d.tile_dirty[k] && d.tile_slot[k] >= 0;
+  if (dirty || d.in_flight) {
+    Status r = domain_sync(d);
+    if (r.bad()) return r;
+  }
+  const int64_t ex = G.t[0] + 2 * g, ey = G.t[1] + 2 * g, ez = G.t[2] + 2 * g;
+  std::vector<int64_t> map((size_t)(ex * ey * ez));
+  ghost_map(G, t, map.data());
+  const int64_t tx = G.t[0], ty = G.t[1], tz = G.t[2], nx = G.g[0], ny = G.g[1];
+  const int64_t D = G.depth;
+  for (int64_t k = 0; k < ez; ++k)
+    for (int64_t j = 0; j < ey; ++j)
+      for (int64_t i = 0; i < ex; ++i) {
+        const int64_t m = map[(size_t)((k * ey + j) * ex + i)];
+        double v;
+        if (m >= 0) {
+          const int64_t x = m % nx, y = (m / nx) % ny, z = m / (nx * ny) - G.zoff;  // local z
+          const int64_t k2 = ((z / tz) * G.n[1] + y / ty) * G.n[0] + x / tx;
+          v = d.host_tile(k2)[((z % tz) * ty + y % ty) * tx + x % tx];
+        } else {  // Dirichlet: the fixed face of the domain boundary (nearest layer)
+          int64_t p[3] = {c[0] * tx + i - g, c[1] * ty + j - g, c[2] * tz + k - g};  // local coords
+          const int64_t lim[3] = {G.l[0], G.l[1], G.l[2]};
+          int axis = -1, nout = 0;
+          for (int a = 0; a < 3; ++a)
+            if (p[a] < 0 || p[a] >= lim[a]) ++nout, axis = a;
+          v = std::nan("");  // outside in two or three axes: not stored
+          if (nout == 1) {
+            const int f = 2 * axis + (p[axis] < 0 ? 0 : 1);
+            p[axis] = p[axis] < 0 ? 0 : lim[axis] - 1;  // the adjacent interior cell
+            const int64_t k2 = ((p[2] / tz) * G.n[1] + p[1] / ty) * G.n[0] + p[0] / tx;
+            const int64_t lx = p[0] % tx, ly = p[1] % ty, lz = p[2] % tz;
+            const double* fc = d.host_dir[f] + k2 * G.face_elems[f];
+            const int64_t l = (f & 1) ? 0 : D - 1;  // the layer nearest the tile
+            if (f <= XP) v = fc[(lz * ty + ly) * D + l];
+            else if (f <= YP) v = fc[(lz * D + l) * tx + lx];
+            else v = fc[(l * ty + ly) * tx + lx];
+          }
+        }
+        out[(k * ey + j) * ex + i] = v;
+      }
   return Status::ok();
 }
 

@@ -335,6 +335,8 @@ Status domain_run(Domain& d, const tile_kernel& k, int steps, int nstreams);
 Status domain_sync(Domain& d);
 Status domain_store(Domain& d, double* dst);
 Status domain_invalidate(Domain& d);
+Status domain_host_region(Domain& d, int64_t tile, int mode, double** ptr);
+Status domain_host_ghosts(Domain& d, int64_t tile, double* out);
 Status domain_free(Domain* d);
 Status domain_setup(Domain& d);
 void host_extract_faces(const Geometry& G, const double* host, double* const faces[6]);

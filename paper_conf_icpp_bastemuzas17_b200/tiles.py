@@ -98,6 +98,8 @@ _sig = {
     "tile_load": ([_P, _P], ctypes.c_int),
     "tile_host_tile": ([_P, ctypes.c_int64, ctypes.POINTER(_P)], ctypes.c_int),
     "tile_mark_host_dirty": ([_P], ctypes.c_int),
+    "tile_host_region": ([_P, ctypes.c_int64, ctypes.c_int32, ctypes.POINTER(_P)], ctypes.c_int),
+    "tile_host_ghosts": ([_P, ctypes.c_int64, _P, ctypes.c_int64], ctypes.c_int),
     "tile_run": ([_P, ctypes.POINTER(TileKernel), ctypes.c_int32, ctypes.c_int32], ctypes.c_int),
     "tile_sync": ([_P], ctypes.c_int),
     "tile_store": ([_P, _P], ctypes.c_int),
@@ -327,6 +329,24 @@ class Domain:
         _check(tile_mark_host_dirty(self._h), "tile_mark_host_dirty")
 
     # -- execution --------------------------------------------------------
+    def host_region(self, tile_id, write=False):
+        """GPU-disabled request of one region: the tile's current data
+        as a writable NumPy view of the pinned store; write=True drops the
+        device copy (CPU code will change it)."""
+        p = ctypes.c_void_p()
+        _check(tile_host_region(self._h, tile_id, 1 if write else 0, ctypes.byref(p)), "tile_host_region")
+        tx, ty, tz = self.tile_dims
+        buf = (ctypes.c_double * (tx * ty * tz)).from_address(p.value)
+        return np.frombuffer(buf, dtype=np.float64).reshape(tz, ty, tx)
+
+    def host_ghosts(self, tile_id):
+        """Tile with its ghost shell gathered on the host (P:L96 host update)."""
+        g = self.info["ghost"]
+        tx, ty, tz = self.tile_dims
+        out = np.empty((tz + 2 * g, ty + 2 * g, tx + 2 * g))
+        _check(tile_host_ghosts(self._h, tile_id, out.ctypes.data, out.size), "tile_host_ghosts")
+        return out
+
     def run(self, kernel, steps, nstreams=4):
         _check(tile_run(self._h, ctypes.byref(kernel), steps, nstreams), "tile_run")
         # a user function's module must outlive the launches queued with it

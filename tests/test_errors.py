@@ -30,7 +30,7 @@ def _every_call_is_estate(d):
     arr = np.zeros((16, 16, 32))
     k = T.heat7()
     info, stats = T.TileInfo(), T.TileStats()
-    gm = (ctypes.c_int64 * (18 * 10 * 10))()
+    gm = (ctypes.c_int64 * (18 * 10 * 10))()  # also a large-enough double buffer
     fs = (ctypes.c_int64 * 12)()
     p = ctypes.c_void_p()
     ms = ctypes.c_double()
@@ -40,6 +40,8 @@ def _every_call_is_estate(d):
         "tile_load": lambda: T.tile_load(h, arr.ctypes.data),
         "tile_host_tile": lambda: T.tile_host_tile(h, 0, ctypes.byref(p)),
         "tile_mark_host_dirty": lambda: T.tile_mark_host_dirty(h),
+        "tile_host_region": lambda: T.tile_host_region(h, 0, 0, ctypes.byref(p)),
+        "tile_host_ghosts": lambda: T.tile_host_ghosts(h, 0, gm, len(gm)),
         "tile_run": lambda: T.tile_run(h, ctypes.byref(k), 1, 2),
         "tile_sync": lambda: T.tile_sync(h),
         "tile_store": lambda: T.tile_store(h, arr.ctypes.data),

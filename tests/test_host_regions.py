@@ -1,0 +1,126 @@
+"""The paper's CPU side of the uniform API (CPU half):
+a GPU-disabled request of one region (§IV.B.4: the region is copied
+back if its newest data is on the device, then the host pointer is returned,
+P:L86) and the host-side ghost update (§III, §IV.B.6: ghost cells
+of a region on the host are filled on the host). CPU tests use dry runs (the
+host logic and the op trace); GPU tests check the data against the oracle."""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from tests.conftest import cuda_available, import_tiles
+from tests.test_schedule import _budget_for
+
+T = import_tiles()
+ALPHA = 0.125
+
+
+def _gather(u, m):
+    flat = u.ravel()
+    out = np.full(m.shape, np.nan)
+    ok = m >= 0
+    out[ok] = flat[m[ok]]
+    return out
+
+
+@pytest.mark.parametrize("dims,td,g", [((16, 8, 12), (8, 4, 4), 1), ((12, 8, 8), (4, 4, 4), 2)])
+def test_host_ghosts_equal_the_ghost_map_gather_dry(dims, td, g):
+    u = synth.uniform_grid(*dims, 21)
+    d = T.Domain(dims, td, ghost=g, dry_run=True)
+    d.load(u)
+    for k in range(d.info["ntiles"]):
+        m = oracle.ghost_map(dims, td, g, k)
+        assert np.array_equal(d.host_ghosts(k), _gather(u, m))
+
+
+def test_host_ghosts_dirichlet_faces_dry():
+    dims, td = (16, 8, 8), (8, 4, 4)
+    ext = synth.uniform_grid(18, 10, 10, 3)
+    d = T.Domain(dims, td, bc="dirichlet", dry_run=True)
+    d.load(ext)
+    for k in range(d.info["ntiles"]):
+        got = d.host_ghosts(k)
+        ix, iy, iz = k % 2, (k // 2) % 2, k // 4
+        exp = ext[iz * 4:iz * 4 + 6, iy * 4:iy * 4 + 6, ix * 8:ix * 8 + 10].copy()
+        # shell cells outside the domain in two or three axes are not stored
+        zz, yy, xx = np.meshgrid(np.arange(6) + iz * 4 - 1, np.arange(6) + iy * 4 - 1, np.arange(10) + ix * 8 - 1,
+                                 indexing="ij")
+        outside = (xx < 0) | (xx >= 16)
+        nout = outside.astype(int) + ((yy < 0) | (yy >= 8)).astype(int) + ((zz < 0) | (zz >= 8)).astype(int)
+        exp[nout >= 2] = np.nan
+        assert np.array_equal(got, exp, equal_nan=True), k
+
+
+def test_host_region_read_copies_back_only_that_tile_dry():
+    """Resident dry run: a READ of one device-newer tile issues one D2H of
+    that tile and a host sync; the device copy stays (the next run is
+    resident, no H2D)."""
+    dims, td = (16, 16, 16), (8, 8, 8)
+    d = T.Domain(dims, td, dry_run=True, wavefront=-1, stream_through=-1)
+    d.load(np.zeros((16, 16, 16)))
+    d.run(T.heat7(ALPHA), 2, 2)
+    d.clear_trace()
+    d.host_region(5)
+    ops = [(op[0], op[2]) for op in d.trace() if op[0] in ("d2h", "sync", "h2d")]
+    assert ops == [("d2h", 5), ("sync", 0)]
+    d.clear_trace()
+    d.run(T.heat7(ALPHA), 1, 2)
+    assert not [op for op in d.trace() if op[0] == "h2d"]
+
+
+def test_host_region_write_drops_the_device_copy_dry():
+    """WRITE: stream mode frees the tile's slot (its next visit is a miss with
+    an H2D); resident mode writes every device-newer tile back and the next
+    run re-uploads the domain."""
+    dims, td = (16, 16, 16), (8, 8, 4)
+    b = _budget_for(dims, td, 20, sched="stream", stream_through=-1)
+    d = T.Domain(dims, td, dry_run=True, sched="stream", device_budget_bytes=b, stream_through=-1)
+    d.load(np.zeros((16, 16, 16)))
+    d.run(T.heat7(ALPHA), 1, 2)
+    d.sync()
+    d.host_region(15, write=True)
+    d.clear_trace()
+    d.run(T.heat7(ALPHA), 1, 2)
+    h2d = {op[2] for op in d.trace() if op[0] == "h2d"}
+    assert 15 in h2d
+    r = T.Domain(dims, td, dry_run=True, wavefront=-1, stream_through=-1)
+    r.load(np.zeros((16, 16, 16)))
+    r.run(T.heat7(ALPHA), 2, 2)
+    r.host_region(3, write=True)
+    assert not r.get_info()["resident"]
+    r.clear_trace()
+    r.run(T.heat7(ALPHA), 1, 2)
+    assert sum(op[4] for op in r.trace() if op[0] == "h2d") == r.info["ntiles"]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("sched", ["resident", "stream"])
+def test_host_region_and_ghosts_gpu(sched):
+    """After device runs, one region read on the host equals the oracle's
+    tile (no full tile_sync), its host ghost shell equals the oracle grid's
+    shell, and a region changed on the host (WRITE) is what the next device
+    steps start from."""
+    if not cuda_available():
+        pytest.skip("no CUDA device")
+    dims, td = (64, 32, 48), (32, 16, 16)
+    u = synth.uniform_grid(*dims, 42)
+    kw = {"stream_through": -1}
+    if sched == "stream":
+        kw.update(sched="stream", device_budget_bytes=_budget_for(dims, td, 5, sched="stream", stream_through=-1))
+    with T.Domain(dims, td, **kw) as d:
+        d.load(u)
+        d.run(T.heat7(ALPHA), 3, 2)
+        ref = oracle.heat_c(u, ALPHA, 3)
+        k = 7
+        ix, iy, iz = k % 2, (k // 2) % 2, k // 4
+        sl = np.s_[iz * 16:(iz + 1) * 16, iy * 16:(iy + 1) * 16, ix * 32:(ix + 1) * 32]
+        assert np.array_equal(d.host_region(k), ref[sl])
+        assert np.array_equal(d.host_ghosts(k), _gather(ref, oracle.ghost_map(dims, td, 1, k)))
+        v = d.host_region(k, write=True)
+        v[:] = 0.25                      # CPU code changes the region
+        mod = ref.copy()
+        mod[sl] = 0.25
+        d.run(T.heat7(ALPHA), 2, 2)
+        out = d.store()
+    assert np.array_equal(out, oracle.heat_c(mod, ALPHA, 2))

@@ -2,7 +2,8 @@
 synccheck / initcheck): resident heat (layered + whole-domain phases),
 streaming heat with a tiny budget, Dirichlet, sincos, the generic kernel, the
 persistent multi-step launch (direct ghosts, grid counter, snake order; banded tiles in round-robin order), a ranged NVRTC user kernel, a user stencil and
-the stream-through schedule and the in-process multi-rank transport."""
+the stream-through schedule, the wavefront (tile-column TMA sweeps with
+tensor-map x halos) and the in-process multi-rank transport."""
 import os
 import sys
 import threading
@@ -65,6 +66,12 @@ fs = T.UserFn("__device__ double hu(double c, double xm, double xp, double ym, d
               " { return c + 0.125 * ((((xm + xp) + (ym + yp)) + (zm + zp)) - 6.0 * c); }", "hu", stencil=True)
 with T.Domain((64, 32, 32), (32, 16, 16)) as d:           # user stencil (NVRTC, face ghosts)
     d.load(u); d.run(T.user_stencil(fs), 3, 2); d.run(T.heat7(), 2, 2); d.store()
+uw = synth.uniform_grid(128, 64, 256, 13)                 # wavefront (T > tz: scratch layers, bootstrap),
+with T.Domain((128, 64, 256), (64, 64, 32), wavefront=1) as d:   # tile-column TMA sweeps
+    d.load(uw); d.run(T.heat7(), 40, 2); d.store(); d.run(T.heat7(), 2, 2); d.store()
+    d.invalidate(); d.run(T.heat7(), 7, 3); d.store()
+with T.Domain((128, 64, 256), (64, 64, 32), stream_through=1, wavefront=-1) as d:  # stream-through, tile kernel
+    d.load(uw); d.run(T.heat7(), 12, 2); d.store()
 g = T.LocalGroup(2)
 def rank(r):
     with T.Domain((64, 32, 64), (32, 16, 16), nranks=2, rank=r, local_group=g) as d:
