@@ -654,6 +654,9 @@ __global__ void __launch_bounds__(TileCfg<BY, RPP, S>::NT + 32, MB)
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
+  // programmatic dependent launch: the next sweep on this stream may be
+  // scheduled now (it waits for this grid before touching memory, below)
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   const int ntx = Sv.ntx * Sv.tx / TX;  // 64-wide columns per row (views share nx)
   const int np = hi - lo;
   const int64_t ncols = (int64_t)ntx * (ny / BY);
@@ -662,6 +665,10 @@ __global__ void __launch_bounds__(TileCfg<BY, RPP, S>::NT + 32, MB)
 
   if ((int)threadIdx.x >= C::NT) {  // ---------------- producer (one thread)
     if (threadIdx.x != C::NT) return;
+    // the previous kernel on the stream complete and its writes visible
+    // before the first load (consumers write only after consuming a stage,
+    // so this also orders their stores after the previous grid's reads)
+    asm volatile("griddepcontrol.wait;" ::: "memory");
     uint32_t g = 0;
     for (int64_t pp = pb; pp < pe;) {
       const int64_t col = pp / np;
@@ -791,8 +798,21 @@ static cudaError_t launch_tile_cfg(const ViewDev& Sv, const ViewDev& Dv, const S
     const char* e = getenv("TILES_SWEEP_ST");
     return e ? atoi(e) : 0;
   }();
-  slab_sweep_tile<BY, RPP, S, MB><<<(unsigned)grid, C::NT + 32, C::SMEM, s>>>(Sv, Dv, m, ny, lo, hi, alpha, st_mode);
-  return cudaGetLastError();
+  static const int pdl = [] {
+    const char* e = getenv("TILES_SWEEP_PDL");
+    return e ? atoi(e) : 1;
+  }();
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(C::NT + 32);
+  cfg.dynamicSmemBytes = C::SMEM;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, slab_sweep_tile<BY, RPP, S, MB>, Sv, Dv, m, ny, lo, hi, alpha, st_mode);
 }
 
 // driver entry point for cuTensorMapEncodeTiled (no -lcuda link dependency)
