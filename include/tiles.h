@@ -289,13 +289,8 @@ typedef enum {
                             wrapped (no scratch) */
   TILE_OP_D2H_PLANES = 27,/* planes [d & 0xffffffff, + d >> 32) of c tile slots b.. ->
                             the same planes of host tiles a.. */
-  TILE_OP_COPY_PLANES = 28,/* planes [d & 0xffffffff, + d >> 32) of c tile slots a.. ->
+  TILE_OP_COPY_PLANES = 28/* planes [d & 0xffffffff, + d >> 32) of c tile slots a.. ->
                             the same planes of slots b.. */
-  TILE_OP_WSWEEP2 = 29   /* wavefront, two levels in one pass: level s on planes [lo, hi)
-                            (c = lo | hi << 32, signed halves) from view a, written to view
-                            (b & 0xffffffff) only at planes hi-2, hi-1 (planes lo-2, lo-1 of
-                            level s are read from it); level s+1 on [lo-1, hi-1) into view
-                            b >> 32. Views coded as for TILE_OP_WSWEEP, d = scratch layers */
 } tile_op_kind;
 
 typedef struct {

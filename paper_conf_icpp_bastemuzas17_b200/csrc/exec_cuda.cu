@@ -418,33 +418,6 @@ struct CudaExec final : Exec {
     d.stats.n_kernels++;
     return Status::ok();
   }
-  Status slab_sweep2(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, int a, int b,
-                     int st) override {
-    INJECT(FAULT_KERNEL, st);
-    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
-    ensure_maps(d);
-    const SlabView s = slab_view(d, src, a), m = slab_view(d, mid, a), t = slab_view(d, dst, a);
-    bool fused = true;
-    next_cells = d.kernel_timing ? (uint64_t)(b - a) * d.G.l[0] * d.G.l[1] : 0;  // one pass, two levels
-    Status r = timed(d, st, [&] {
-      cudaError_t e = launch_slab_sweep2(s, m, t, (int)d.G.l[0], (int)d.G.l[1], a, b, d.kernel_alpha, sms, S(st),
-                                         &maps);
-      if (e == cudaErrorNotSupported) {
-        fused = false;
-        cudaGetLastError();
-        return cudaSuccess;
-      }
-      return e;
-    });
-    if (r.bad()) return r;
-    if (!fused) {  // shapes the fused kernel does not cover: the two levels one after the other
-      r = slab_sweep(d, src, mid, a, b, st);
-      if (r.bad()) return r;
-      return slab_sweep(d, mid, dst, a - 1, b - 1, st);
-    }
-    d.stats.n_kernels++;
-    return Status::ok();
-  }
   Status h2d_part(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int st) override {
     INJECT(FAULT_H2D, st);
     if (d.measure == TILE_MEASURE_COMP_ONLY) return Status::ok();

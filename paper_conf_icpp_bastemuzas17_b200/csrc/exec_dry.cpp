@@ -120,17 +120,6 @@ struct DryExec final : Exec {
         src.kind == SlabRef::RESIDENT ? src.zbase : 0);
     return Status::ok();
   }
-  Status slab_sweep2(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, int a, int b,
-                     int st) override {
-    if (Status f_ = inject(d, FAULT_KERNEL); f_.bad()) return f_;
-    d.stats.n_kernels++;
-    auto code = [](const SlabRef& r) {
-      return r.kind == SlabRef::WAVE ? 1 | ((int64_t)r.slot << 1) | ((int64_t)r.ring[0] << 2) : ((int64_t)r.slot << 1);
-    };
-    put(d, TILE_OP_WSWEEP2, st, code(src), code(mid) | (code(dst) << 32),
-        (int64_t)(uint32_t)a | ((int64_t)(uint32_t)b << 32), dst.un);
-    return Status::ok();
-  }
   Status h2d_pack(Domain& d, int64_t t0, int64_t n, int ps, int64_t p0, int64_t np, int st) override {
     if (Status f_ = inject(d, FAULT_H2D); f_.bad()) return f_;
     d.stats.bytes_h2d += (uint64_t)n * np * d.G.t[0] * d.G.t[1] * 8;

@@ -189,7 +189,6 @@ struct alignas(64) TensorMapBlob {
 };
 struct SweepMaps {
   TensorMapBlob xmap[2];
-  TensorMapBlob xmap2[2];  // the same memory, box {2, 2} (the fused sweep's extra halo rows)
   const double* base[2];
   const double* end[2];
   int valid[2];
@@ -204,12 +203,6 @@ cudaError_t launch_push_rows(const double* src, int64_t src_pitch, double* dst, 
                              int64_t len, int ctas, cudaStream_t st);
 cudaError_t launch_slab_sweep(const SlabView& src, const SlabView& dst, int nx, int ny, int lo,
                               int hi, double alpha, int sms, cudaStream_t s, const SweepMaps* maps = nullptr);
-// Two levels per sweep (wavefront): level s on planes [a, b)
-// from src (level s-1), level s+1 on [a-1, b-1) into dst; level s itself
-// stays on chip except its top two planes (and the two below a are read),
-// through view mid. Returns cudaErrorNotSupported when the shapes do not fit.
-cudaError_t launch_slab_sweep2(const SlabView& src, const SlabView& mid, const SlabView& dst, int nx, int ny, int a,
-                               int b, double alpha, int sms, cudaStream_t s, const SweepMaps* maps);
 // Two-step kernel: returns false from heat2_plan if no specialisation fits.
 bool heat2_plan(int tx, int ty, int max_smem, int* band, size_t* smem);
 cudaError_t heat2_configure(int tx, int band, size_t smem, int* ctas_per_sm);

@@ -856,258 +856,11 @@ bool sweep_map_encode(SweepMaps* m, int k, const double* base, uint64_t bytes, i
         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
     return false;
-  const cuuint32_t box2[2] = {2, 2};
-  if (f(reinterpret_cast<CUtensorMap*>(&m->xmap2[k]), CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double*>(base),
-        dims, strides, box2, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-        CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
-    return false;
   m->base[k] = base;
   m->end[k] = base + rows * tx;
   m->valid[k] = 1;
   m->band = band;
   return true;
-}
-
-// ---- two levels per sweep (wavefront): slab_sweep2_tile. A CTA owns runs
-// of (column, plane) pairs of level s+1 like slab_sweep_tile; for a run of
-// level-s+1 planes [p0, p1) it needs level s on [p0-1, p1+1): planes below a
-// (at most two, a-2 and a-1, written by the previous chunk) come from HBM
-// through view mid, the others are computed on chip from level s-1 over the
-// band extended by one row and one column per side (BY+2 rows x 66 cells;
-// level s-1 staged as BY+4 rows x 64 + x halos of 2 columns, nine TMA
-// operations per plane) into a ring of four level-s planes in shared memory
-// ([BY+2][68], x offset 2: 16-byte aligned pairs); level s+1 on the band is
-// computed from that ring one plane behind. Level s goes to HBM only at its
-// chunk's top two planes (b-2, b-1), which the next chunk reads. One named
-// barrier per plane orders the ring (level s written -> level s+1 read).
-namespace w2 {
-constexpr int BY = 32, TX = 64, NT = 512, S = 4;
-constexpr int SROWS = BY + 4;                       // staged rows: y0-2 .. y0+BY+1
-constexpr int XH = SROWS * TX;                      // x halos: per side three boxes, each at a
-                                                    // 128-byte boundary: rows 0-1, 2..BY+1, BY+2..BY+3
-constexpr int HS = 96;                              // doubles per side (16 + 64 + 16)
-constexpr int STAGE = XH + 2 * HS;                  // doubles (multiple of 16)
-constexpr uint32_t BYTES = (uint32_t)(SROWS * TX + 4 * SROWS) * 8;  // bytes landed per plane
-__device__ __forceinline__ int hoff(int side, int sr) {  // x-halo pair of staged row sr
-  const int o = side * HS;
-  return sr < 2 ? o + 2 * sr : sr < BY + 2 ? o + 16 + 2 * (sr - 2) : o + 80 + 2 * (sr - BY - 2);
-}
-constexpr int MROWS = BY + 2, MW = 68;              // level-s plane: rows y0-1 .. y0+BY, x -2 .. 65
-constexpr int MID = MROWS * MW;                     // doubles per ring slot
-constexpr size_t SMEM = (size_t)S * STAGE * 8 + (size_t)4 * MID * 8 + (size_t)2 * S * 8;
-static_assert(STAGE % 16 == 0 && MID % 2 == 0, "layout");
-}  // namespace w2
-
-static __device__ __forceinline__ void bar_consumers() {
-  asm volatile("bar.sync 1, %0;" ::"n"(w2::NT) : "memory");
-}
-
-__global__ void __launch_bounds__(w2::NT + 32, 1)
-    slab_sweep2_tile(const ViewDev Sv, const ViewDev Mv, const ViewDev Dv, const __grid_constant__ SweepMaps maps,
-                     const int ny, const int a, const int b, const double alpha) {
-  using namespace w2;
-  extern __shared__ __align__(128) unsigned char smem_raw[];
-  double* stage = reinterpret_cast<double*>(smem_raw);
-  double* mid = stage + (size_t)S * STAGE;
-  uint64_t* full = reinterpret_cast<uint64_t*>(mid + (size_t)4 * MID);
-  uint64_t* empty = full + S;
-  if (threadIdx.x == 0) {
-    for (int s = 0; s < S; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&empty[s], NT);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-  const int ntx = Sv.ntx * Sv.tx / TX;
-  const int np = b - a;                              // level s+1 planes [a-1, b-1)
-  const int64_t ncols = (int64_t)ntx * (ny / BY);
-  const int64_t P = ncols * np;
-  const int64_t pb = P * blockIdx.x / gridDim.x, pe = P * (blockIdx.x + 1) / gridDim.x;
-  // a run: column col, level-s+1 planes [p0, p1) (within [a-1, b-1))
-  auto run_at = [&](int64_t pp, int64_t& col, int& p0, int& p1) {
-    col = pp / np;
-    p0 = a - 1 + (int)(pp - col * np);
-    const int64_t left = pe - pp, inrun = (int64_t)(b - 1 - p0);
-    p1 = p0 + (int)(left < inrun ? left : inrun);
-  };
-
-  if ((int)threadIdx.x >= NT) {  // ---------------- producer (one thread)
-    if (threadIdx.x != NT) return;
-    asm volatile("griddepcontrol.wait;" ::: "memory");
-    uint32_t g = 0;
-    for (int64_t pp = pb; pp < pe;) {
-      int64_t col;
-      int p0, p1;
-      run_at(pp, col, p0, p1);
-      pp += p1 - p0;
-      const int cx = (int)(col % ntx), y0 = (int)(col / ntx) * BY;
-      const int x0 = cx * TX, xl = (cx == 0 ? ntx - 1 : cx - 1) * TX, xr = (cx == ntx - 1 ? 0 : cx + 1) * TX;
-      const int ya = y0 < 2 ? y0 - 2 + ny : y0 - 2;             // rows y0-2, y0-1 (one tile)
-      const int yb = y0 + BY + 2 > ny ? y0 + BY - ny : y0 + BY;  // rows y0+BY, y0+BY+1
-      const int zc0 = p0 - 1 > a ? p0 - 1 : a;                  // first computed level-s plane
-      const int nl_ = (a < p1 + 1 ? a : p1 + 1) - (p0 - 1);
-      const int nload = nl_ > 0 ? nl_ : 0;                      // level-s planes read (p0-1 .. a-1)
-      const int nstg = (p1 + 1) - zc0 + 2;                      // level s-1 planes zc0-1 .. p1+1
-      for (int q = 0; q < nload + nstg; ++q, ++g) {
-        const bool ld = q < nload;
-        const ViewDev& V = ld ? Mv : Sv;
-        const int z = ld ? p0 - 1 + q : zc0 - 1 + (q - nload);
-        const int st = (int)(g % S);
-        mbar_wait(&empty[st], ((g / S) & 1u) ^ 1u);
-        double* dst = stage + (size_t)st * STAGE;
-        const double* pz = V.P(z);
-        fence_proxy_async();
-        mbar_expect_tx(&full[st], BYTES);
-        bulk_g2s(dst + 2 * TX, pz + V.Y(y0) + V.X(x0), (uint32_t)BY * TX * 8, &full[st]);
-        bulk_g2s(dst, pz + V.Y(ya) + V.X(x0), 2 * TX * 8, &full[st]);
-        bulk_g2s(dst + (BY + 2) * TX, pz + V.Y(yb) + V.X(x0), 2 * TX * 8, &full[st]);
-        const double* cl[3] = {pz + V.Y(ya) + V.X(xl), pz + V.Y(y0) + V.X(xl), pz + V.Y(yb) + V.X(xl)};
-        const double* cr[3] = {pz + V.Y(ya) + V.X(xr), pz + V.Y(y0) + V.X(xr), pz + V.Y(yb) + V.X(xr)};
-        const int boff[3] = {0, 16, 80};  // the three boxes of a side (128-byte aligned)
-#pragma unroll
-        for (int h = 0; h < 3; ++h) {
-          const int kl = (cl[h] >= maps.base[1] && cl[h] < maps.end[1]) ? 1 : 0;
-          const int kr = (cr[h] >= maps.base[1] && cr[h] < maps.end[1]) ? 1 : 0;
-          const TensorMapBlob* ml = h == 1 ? &maps.xmap[kl] : &maps.xmap2[kl];
-          const TensorMapBlob* mr = h == 1 ? &maps.xmap[kr] : &maps.xmap2[kr];
-          tma_2d(dst + XH + boff[h], ml, TX - 2, (int)((cl[h] - maps.base[kl]) / TX), &full[st]);
-          tma_2d(dst + XH + HS + boff[h], mr, 0, (int)((cr[h] - maps.base[kr]) / TX), &full[st]);
-        }
-      }
-    }
-    return;
-  }
-
-  // ------------------------------------------------------- consumer warps
-  const int t = (int)threadIdx.x;
-  uint32_t seq = 0;
-  auto wait_g = [&](uint32_t g) { mbar_wait(&full[g % S], (g / S) & 1u); };
-  auto release_g = [&](uint32_t g) { mbar_arrive(&empty[g % S]); };
-  // staged level s-1 value at stage row sr (0 <=> y0-2), x in [-2, 66)
-  auto sval = [&](const double* st, int sr, int x) -> double {
-    return x < 0 ? st[XH + hoff(0, sr) + (x + 2)] : x >= TX ? st[XH + hoff(1, sr) + (x - TX)] : st[sr * TX + x];
-  };
-  for (int64_t pp = pb; pp < pe;) {
-    int64_t col;
-    int p0, p1;
-    run_at(pp, col, p0, p1);
-    pp += p1 - p0;
-    const int cx = (int)(col % ntx), y0 = (int)(col / ntx) * BY;
-    const int zc0 = p0 - 1 > a ? p0 - 1 : a;
-    const int nl_ = (a < p1 + 1 ? a : p1 + 1) - (p0 - 1);
-    const int nload = nl_ > 0 ? nl_ : 0;
-    const int base = p0 - 1;  // mid slot of level-s plane z: (z - base) & 3
-    // loaded level-s planes -> mid slots ([MROWS][MW], x offset 2)
-    for (int q = 0; q < nload; ++q) {
-      wait_g(seq + q);
-      const double* st = stage + (size_t)((seq + q) % S) * STAGE;
-      double* m = mid + (size_t)(((p0 - 1 + q) - base) & 3) * MID;
-      for (int i = t; i < MROWS * 66; i += NT) {
-        const int r = i / 66, x = i - r * 66 - 1;  // x in [-1, 65)
-        m[r * MW + x + 2] = sval(st, r + 1, x);
-      }
-      release_g(seq + q);
-    }
-    const uint32_t s0 = seq + nload;  // stage of level s-1 plane zc0-1
-    // output offsets (band pairs): level s+1 rows y0 + r, x = 2 * c2
-    for (int z = zc0; z < p1 + 1; ++z) {
-      const uint32_t gz = s0 + (uint32_t)(z - (zc0 - 1));  // stage of level s-1 plane z
-      if (z == zc0) wait_g(gz - 1);
-      wait_g(gz);
-      wait_g(gz + 1);
-      const double* sm1 = stage + (size_t)((gz - 1) % S) * STAGE;
-      const double* s00 = stage + (size_t)(gz % S) * STAGE;
-      const double* sp1 = stage + (size_t)((gz + 1) % S) * STAGE;
-      double* m = mid + (size_t)((z - base) & 3) * MID;
-      const bool top = z >= b - 2;  // level s to HBM (the next chunk reads it)
-      double* mo = top ? Mv.P(z) : nullptr;
-      // inner pairs: rows r in [0, MROWS) (y0-1+r), x = 2*pc
-      for (int q = t; q < MROWS * 32; q += NT) {
-        const int r = q >> 5, x = (q & 31) * 2, sr = r + 1;
-        const double2 c = *reinterpret_cast<const double2*>(s00 + sr * TX + x);
-        const double2 ym = *reinterpret_cast<const double2*>(s00 + (sr - 1) * TX + x);
-        const double2 yp = *reinterpret_cast<const double2*>(s00 + (sr + 1) * TX + x);
-        const double2 zm = *reinterpret_cast<const double2*>(sm1 + sr * TX + x);
-        const double2 zp = *reinterpret_cast<const double2*>(sp1 + sr * TX + x);
-        const double xm = x == 0 ? s00[XH + hoff(0, sr) + 1] : s00[sr * TX + x - 1];
-        const double xp = x == TX - 2 ? s00[XH + hoff(1, sr)] : s00[sr * TX + x + 2];
-        double2 v;
-        v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm.x, zp.x, alpha);
-        v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm.y, zp.y, alpha);
-        *reinterpret_cast<double2*>(m + r * MW + x + 2) = v;
-        if (top && r >= 1 && r <= BY)
-          *reinterpret_cast<double2*>(mo + Mv.Y(y0 + r - 1) + Mv.X(cx * TX + x)) = v;
-      }
-      // edge cells x = -1 and x = 64 of every extended row
-      if (t < 2 * MROWS) {
-        const int side = t / MROWS, r = t - side * MROWS, sr = r + 1, x = side ? TX : -1;
-        const double c = sval(s00, sr, x);
-        const double v = heat_update(c, sval(s00, sr, x - 1), sval(s00, sr, x + 1), sval(s00, sr - 1, x),
-                                     sval(s00, sr + 1, x), sval(sm1, sr, x), sval(sp1, sr, x), alpha);
-        m[r * MW + x + 2] = v;
-      }
-      release_g(gz - 1);  // level s-1 plane z-1: no reader left
-      bar_consumers();    // level s plane z complete in the ring
-      const int w = z - 1;  // level s+1 plane
-      if (w >= p0) {
-        const double* mm = mid + (size_t)((w - 1 - base) & 3) * MID;
-        const double* mc = mid + (size_t)((w - base) & 3) * MID;
-        const double* mp = m;
-        double* od = Dv.P(w);
-        for (int q = t; q < BY * 32; q += NT) {
-          const int r = q >> 5, x = (q & 31) * 2, mr = r + 1;
-          const double* cc = mc + mr * MW + x + 2;
-          const double2 c = *reinterpret_cast<const double2*>(cc);
-          const double2 ym = *reinterpret_cast<const double2*>(cc - MW);
-          const double2 yp = *reinterpret_cast<const double2*>(cc + MW);
-          const double2 zm = *reinterpret_cast<const double2*>(mm + mr * MW + x + 2);
-          const double2 zp = *reinterpret_cast<const double2*>(mp + mr * MW + x + 2);
-          double2 v;
-          v.x = heat_update(c.x, cc[-1], c.y, ym.x, yp.x, zm.x, zp.x, alpha);
-          v.y = heat_update(c.y, c.x, cc[2], ym.y, yp.y, zm.y, zp.y, alpha);
-          stg2_stream(od + Dv.Y(y0 + r) + Dv.X(cx * TX + x), v);
-        }
-      }
-    }
-    // the last two staged planes (p1, p1+1 of level s-1) are released here
-    release_g(s0 + (uint32_t)(p1 + 1 - (zc0 - 1)));
-    release_g(s0 + (uint32_t)(p1 + 1 - (zc0 - 1)) - 1);
-    seq = s0 + (uint32_t)(p1 + 1 - (zc0 - 1)) + 1;
-    bar_consumers();  // the ring is reused by the next run
-  }
-}
-
-cudaError_t launch_slab_sweep2(const SlabView& src, const SlabView& mid, const SlabView& dst, int nx, int ny, int a,
-                               int b, double alpha, int sms, cudaStream_t s, const SweepMaps* maps) {
-  using namespace w2;
-  if (b <= a) return cudaSuccess;
-  if (!maps || !maps->valid[0] || maps->band != BY || src.ring || src.hhi || mid.hhi || src.tx != TX ||
-      mid.tx != TX || dst.tx != TX || src.ty % 64 || mid.ty % 64 || dst.ty % BY || nx % TX || ny % 64)
-    return cudaErrorNotSupported;
-  for (const SlabView* v : {&src, &mid})
-    if (v->hlo && !(maps->valid[1] && v->hlo >= maps->base[1] && v->hlo < maps->end[1]))
-      return cudaErrorNotSupported;
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(slab_sweep2_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
-    if (e != cudaSuccess) return e;
-    attr = true;
-  }
-  const int64_t P = (int64_t)(nx / TX) * (ny / BY) * (b - a);
-  const int64_t grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)sms, P / 8));
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((unsigned)grid);
-  cfg.blockDim = dim3(NT + 32);
-  cfg.dynamicSmemBytes = SMEM;
-  cfg.stream = s;
-  cudaLaunchAttribute attr1[1];
-  attr1[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  attr1[0].val.programmaticStreamSerializationAllowed = 1;
-  cfg.attrs = attr1;
-  cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, slab_sweep2_tile, to_dev(src), to_dev(mid), to_dev(dst), *maps, ny, a, b, alpha);
 }
 
 template <int TX, int BY, int RPP, int S>

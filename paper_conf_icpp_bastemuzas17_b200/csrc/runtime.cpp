@@ -1374,26 +1374,14 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
     r = X.slab_sweep(d, lvl(t - 1), lvl(t), -2 * T + t, -t, cs);
     if (r.bad()) return r;
   }
-  // the march: levels in pairs (s, s+1) per pass when fused (the level-s
-  // chunk stays on chip but for its top two planes), a single sweep for an
-  // odd last level
-  static const int fuse = [] {
-    const char* e = getenv("TILES_WAVE_FUSE");
-    return e ? atoi(e) : 1;
-  }();
+  // the march
   for (int64_t i = 0; i < U; ++i) {
     if (i < iB) {
       r = X.wait(d, ev_in(d, i), cs);
       if (r.bad()) return r;
     }
-    for (int s = 1; s <= T;) {
-      if (fuse && s + 1 <= T) {
-        r = X.slab_sweep2(d, lvl(s - 1), lvl(s), lvl(s + 1), (int)(c * i - s), (int)(c * i + c - s), cs);
-        s += 2;
-      } else {
-        r = X.slab_sweep(d, lvl(s - 1), lvl(s), (int)(c * i - s), (int)(c * i + c - s), cs);
-        s += 1;
-      }
+    for (int s = 1; s <= T; ++s) {
+      r = X.slab_sweep(d, lvl(s - 1), lvl(s), (int)(c * i - s), (int)(c * i + c - s), cs);
       if (r.bad()) return r;
     }
     r = X.record(d, ev_host(d, i), cs);

@@ -124,11 +124,6 @@ struct Exec {
   virtual Status slab_sweep(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi,
                             int stream) = 0;
   virtual Status copy_slots(Domain& d, int src_slot, int dst_slot, int64_t n, int stream) = 0;
-  // wavefront: levels s (planes [a, b), kept on chip but its top two planes,
-  // written to mid, whose planes a-2, a-1 it also reads) and s+1 (planes
-  // [a-1, b-1) into dst) of one chunk in one pass
-  virtual Status slab_sweep2(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, int a, int b,
-                             int stream) = 0;
   // planes [p0, p0+np) of n tile slots: slots s0.. -> host tiles t0.. (the
   // same planes), and slots -> slots (wavefront)
   virtual Status d2h_planes(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int stream) = 0;

@@ -379,19 +379,6 @@ class Replayer:
             new = self.sweep(blk, None, 1, hi - lo + 1)
             for p in range(lo, hi):
                 self.wave_set(b, p, d, new[p - lo + 1])
-        elif name == "wsweep2":
-            # levels s on [lo, hi) (only hi-2, hi-1 reach view mid; lo-2, lo-1
-            # come from it) and s+1 on [lo-1, hi-1) into view dst
-            lo, hi = wsweep_range(c)
-            mid, dst = b & 0xFFFFFFFF, (b >> 32) & 0xFFFFFFFF
-            blk = np.stack([self.wave_get(a, p, d) for p in range(lo - 1, hi + 1)])
-            lev = self.sweep(blk, None, 1, hi - lo + 1)[1:hi - lo + 1]      # level s, planes lo..hi-1
-            for p in (hi - 2, hi - 1):
-                self.wave_set(mid, p, d, lev[p - lo])
-            blk2 = np.concatenate([np.stack([self.wave_get(mid, lo - 2, d), self.wave_get(mid, lo - 1, d)]), lev])
-            lev2 = self.sweep(blk2, None, 1, hi - lo + 1)[1:hi - lo + 1]    # level s+1, planes lo-1..hi-2
-            for p in range(lo - 1, hi - 1):
-                self.wave_set(dst, p, d, lev2[p - lo + 1])
         elif name == "d2h_planes":
             p0, np_ = d & 0xffffffff, d >> 32
             for i in range(c):

@@ -510,18 +510,17 @@ def test_wavefront_schedule_replays_to_oracle(dims, td, T, ns, runs_after):
     # the wavefront run on its own: ops, link bytes and swept cells
     d2 = T_run_dry(dims, td, T, ns, wavefront=1)
     ops = [op[0] for op in d2.trace()]
-    assert ("wsweep" in ops or "wsweep2" in ops) and "d2h_planes" in ops and "sweep" not in ops
+    assert "wsweep" in ops and "d2h_planes" in ops and "sweep" not in ops
     st = d2.stats()
     cells = dims[0] * dims[1] * dims[2]
     assert st["bytes_h2d"] == cells * 8 and st["bytes_d2h"] == cells * 8
     assert d2.get_info()["last_schedule"] == 6
     planes = 0
     for op in d2.trace():
-        if op[0] in ("wsweep", "wsweep2"):
+        if op[0] == "wsweep":
             lo, hi = wsweep_range(op[4])
-            planes += (hi - lo) * (2 if op[0] == "wsweep2" else 1)
+            planes += hi - lo
     assert planes == dims[2] * T + sum(max(0, 2 * T - 2 * t) for t in range(1, T))
-    assert ("wsweep2" in ops) == (T >= 2)
 
 
 def T_run_dry(dims, td, steps, ns, **kw):
