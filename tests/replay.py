@@ -375,6 +375,12 @@ class Replayer:
         elif name == "wsweep":
             lo, hi = wsweep_range(c)
             G = self.G
+            # one kernel reads [lo-1, hi+1) and writes [lo, hi) with all its CTAs
+            # at once: the two must not share memory (an in-kernel WAR race the
+            # op-level replay could not otherwise see)
+            rd = {self._wave_loc(a, p, d) for p in range(lo - 1, hi + 1)}
+            wr = {self._wave_loc(b, p, d) for p in range(lo, hi)}
+            assert not rd & wr, "sweep writes planes it reads (in-kernel race)"
             blk = np.stack([self.wave_get(a, p, d) for p in range(lo - 1, hi + 1)])
             new = self.sweep(blk, None, 1, hi - lo + 1)
             for p in range(lo, hi):
