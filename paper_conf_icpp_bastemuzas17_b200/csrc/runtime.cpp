@@ -1352,12 +1352,30 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
       return X.h2d_part(d, L * lt, lt, arr0(bit, L), lz, np, is);
     });
   };
-  // uploads on one copy-in stream, in march order: the seam's cone first
-  r = upload(nz - B, nz);
-  if (r.bad()) return r;
-  r = X.record(d, ev_in(d, iB), is);
-  if (r.bad()) return r;
-  for (int64_t i = 0; i < iB; ++i) {
+  // Uploads on one copy-in stream: the seam's cone [-B, 0) in chunks going
+  // down from the seam (region chunk k = planes [-(k+1)c, -kc) = ring chunk
+  // U-1-k), chunk 0 right after the first of them, then chunks 1.. in march
+  // order. The bootstrap runs in rounds as the region chunks land (a
+  // downward skewed march: round k extends level t to [-(k+1)c + t, ...)),
+  // and iteration 0's level s runs as soon as its seam strip (level s-1 at
+  // planes -s-1, -s, complete once (k+1)c >= 2s) exists, so the bootstrap's
+  // compute overlaps the cone's upload instead of following it.
+  const int64_t nB = B / c;
+  auto region_chunk = [&](int64_t k) { return U - 1 - k; };
+  for (int64_t k = 0; k < nB; ++k) {
+    const int64_t ch = region_chunk(k);
+    r = upload(ch * c, (ch + 1) * c);
+    if (r.bad()) return r;
+    r = X.record(d, ev_in(d, ch), is);
+    if (r.bad()) return r;
+    if (k == 0 && iB > 0) {
+      r = upload(0, c);
+      if (r.bad()) return r;
+      r = X.record(d, ev_in(d, 0), is);
+      if (r.bad()) return r;
+    }
+  }
+  for (int64_t i = 1; i < iB; ++i) {
     r = upload(i * c, (i + 1) * c);
     if (r.bad()) return r;
     r = X.record(d, ev_in(d, i), is);
@@ -1367,22 +1385,50 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
     return s == 0 ? SlabRef{SlabRef::RESIDENT, bit, 0, {0, 0, 0}, 0, 0}
                   : SlabRef{SlabRef::WAVE, bit ^ (s & 1), 0, {scr[s & 1], 0, 0}, 0, nlo};
   };
-  // bootstrap: level t on [-2T + t, -t) from the top 2T planes
-  r = X.wait(d, ev_in(d, iB), cs);
-  if (r.bad()) return r;
-  for (int t = 1; t < T; ++t) {
-    r = X.slab_sweep(d, lvl(t - 1), lvl(t), -2 * T + t, -t, cs);
+  auto level_of_iteration = [&](int64_t i, int s) {
+    return X.slab_sweep(d, lvl(s - 1), lvl(s), (int)(c * i - s), (int)(c * i + c - s), cs);
+  };
+  // bootstrap rounds, with iteration 0's levels interleaved
+  int s0 = 1;  // next level of iteration 0
+  for (int64_t k = 0; k < nB; ++k) {
+    r = X.wait(d, ev_in(d, region_chunk(k)), cs);
+    if (r.bad()) return r;
+    for (int t = 1; t < T; ++t) {  // level t over [-2T + t, -t), the part this chunk makes computable
+      const int64_t lo = std::max<int64_t>(-2 * (int64_t)T + t, -(k + 1) * c + t);
+      const int64_t hi = std::min<int64_t>(-t, -k * c + t);
+      const int64_t lo_prev = std::max<int64_t>(-2 * (int64_t)T + t, -k * c + t);  // computed before
+      const int64_t h = k == 0 ? hi : std::min(hi, lo_prev);
+      if (lo < h) {
+        r = X.slab_sweep(d, lvl(t - 1), lvl(t), (int)lo, (int)h, cs);
+        if (r.bad()) return r;
+      }
+    }
+    if (k == 0 && iB > 0) {
+      r = X.wait(d, ev_in(d, 0), cs);
+      if (r.bad()) return r;
+    }
+    // iteration 0's levels whose seam strip is complete: level s needs level
+    // s-1 at -s-1, -s, i.e. (k+1)c >= 2(s-1) + 2 (level 0: region chunk 0)
+    for (; s0 <= T && (k + 1) * c >= 2 * (int64_t)s0; ++s0) {
+      r = level_of_iteration(0, s0);
+      if (r.bad()) return r;
+    }
+  }
+  for (; s0 <= T; ++s0) {
+    r = level_of_iteration(0, s0);
     if (r.bad()) return r;
   }
   // the march
   for (int64_t i = 0; i < U; ++i) {
-    if (i < iB) {
-      r = X.wait(d, ev_in(d, i), cs);
-      if (r.bad()) return r;
-    }
-    for (int s = 1; s <= T; ++s) {
-      r = X.slab_sweep(d, lvl(s - 1), lvl(s), (int)(c * i - s), (int)(c * i + c - s), cs);
-      if (r.bad()) return r;
+    if (i > 0) {
+      if (i < iB) {
+        r = X.wait(d, ev_in(d, i), cs);
+        if (r.bad()) return r;
+      }
+      for (int s = 1; s <= T; ++s) {
+        r = level_of_iteration(i, s);
+        if (r.bad()) return r;
+      }
     }
     r = X.record(d, ev_host(d, i), cs);
     if (r.bad()) return r;
