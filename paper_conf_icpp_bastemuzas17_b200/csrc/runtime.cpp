@@ -1328,28 +1328,7 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
   Exec& X = *d.exec;
   const Geometry& G = d.G;
   const int64_t nz = G.l[2], tz = G.t[2], lt = G.layer_tiles, c = wp.c, B = wp.B, nlo = wp.nlo;
-  // Chunk boundaries zb[0] = 0 < zb[1] < ... < zb[U] = nz. Thin chunks (c)
-  // where the pipeline fills (the first two) and drains (the seam's region,
-  // iterations iB.. in chunks of c), thick ones (TILES_WAVE_BIG x c, default
-  // 4) in between: the march is compute-bound there, and a thick chunk's
-  // level sweeps amortise each launch's ramp and drain over more planes.
-  static const int64_t big = [] {
-    const char* e = getenv("TILES_WAVE_BIG");
-    return e ? std::max<int64_t>(1, atoll(e)) : (int64_t)4;
-  }();
-  std::vector<int64_t> zb{0};
-  {
-    const int64_t zr = nz - B;  // the region starts here
-    while (zb.back() < zr) {
-      const int64_t z = zb.back(), left = zr - z;
-      const int64_t n = (zb.size() <= 2 || left < (big + 2) * c) ? c : big * c;
-      zb.push_back(z + std::min(n, left));
-    }
-    for (int64_t z = zr + c; z <= nz; z += c) zb.push_back(z);
-  }
-  const int64_t U = (int64_t)zb.size() - 1;  // iterations
-  int64_t iB = 0;                             // first iteration inside the bootstrap region
-  while (zb[(size_t)iB] < nz - B) ++iB;
+  const int64_t U = nz / c, iB = (nz - B) / c;  // iterations; first chunk inside the bootstrap region
   Status r = ensure_wave_scratch(d, 2 * nlo * lt);
   if (r.bad()) return r;
   const Pipes P(S, false);
@@ -1385,19 +1364,19 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
   auto region_chunk = [&](int64_t k) { return U - 1 - k; };
   for (int64_t k = 0; k < nB; ++k) {
     const int64_t ch = region_chunk(k);
-    r = upload(zb[(size_t)ch], zb[(size_t)ch + 1]);
+    r = upload(ch * c, (ch + 1) * c);
     if (r.bad()) return r;
     r = X.record(d, ev_in(d, ch), is);
     if (r.bad()) return r;
     if (k == 0 && iB > 0) {
-      r = upload(zb[0], zb[1]);
+      r = upload(0, c);
       if (r.bad()) return r;
       r = X.record(d, ev_in(d, 0), is);
       if (r.bad()) return r;
     }
   }
   for (int64_t i = 1; i < iB; ++i) {
-    r = upload(zb[(size_t)i], zb[(size_t)i + 1]);
+    r = upload(i * c, (i + 1) * c);
     if (r.bad()) return r;
     r = X.record(d, ev_in(d, i), is);
     if (r.bad()) return r;
@@ -1407,7 +1386,7 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
                   : SlabRef{SlabRef::WAVE, bit ^ (s & 1), 0, {scr[s & 1], 0, 0}, 0, nlo};
   };
   auto level_of_iteration = [&](int64_t i, int s) {
-    return X.slab_sweep(d, lvl(s - 1), lvl(s), (int)(zb[(size_t)i] - s), (int)(zb[(size_t)i + 1] - s), cs);
+    return X.slab_sweep(d, lvl(s - 1), lvl(s), (int)(c * i - s), (int)(c * i + c - s), cs);
   };
   // bootstrap rounds, with iteration 0's levels interleaved
   int s0 = 1;  // next level of iteration 0
@@ -1457,7 +1436,7 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
     if (r.bad()) return r;
     // level-T planes [c*i - T, c*i + c - T): z < 0 from the scratch (the
     // ring's top planes), z >= 0 from the resident array
-    const int64_t a = zb[(size_t)i] - T, b = zb[(size_t)i + 1] - T;
+    const int64_t a = c * i - T, b = c * i + c - T;
     if (a < 0) {
       r = pieces(nz + a, nz + std::min<int64_t>(b, 0), [&](int64_t L, int64_t lz, int64_t np) {
         const int64_t Ls = L - (nz / tz - nlo);  // scratch layer of physical layer L
