@@ -289,323 +289,6 @@ __global__ void __launch_bounds__(128, 4) slab_sweep_ca(const ViewDev S, const V
   }
 }
 
-// ---- TMA variant (the default where the shapes allow): warp-specialised
-// like heat7_fixed. A column is an x segment of TX cells (TX divides both
-// views' tile widths) and a band of BY rows (BY divides both views' tile
-// heights); every CTA owns a contiguous range of (column, plane) pairs, so
-// the work is balanced to the plane and a CTA restarts its march only at
-// column boundaries. Producer warp, per plane: lane 0 arms the stage's
-// mbarrier with the byte count of the BY + 2 rows (band + y halo, periodic
-// in y), the lanes issue one 1-D bulk copy (TMA) per row, and the 2*BY
-// x-halo cells (periodic in x; a strided column, no bulk copy) come by 8-byte
-// cp.async whose completion each lane signals on the same mbarrier
-// (cp.async.mbarrier.arrive.noinc). Consumers: a register z-march (planes
-// z-1, z in registers), 5 shared loads per cell pair and plane, one streaming
-// 128-bit store. Any view: P(z) + Y(y) + X(x) addressing per row.
-template <int TX, int BY, int RPP, int S>
-struct TmaCfg {
-  static constexpr int HALF = TX / 2;
-  static constexpr int NT = RPP * HALF;  // consumer threads
-  static constexpr int NR = BY / RPP;    // rows per consumer thread
-  static constexpr int ROWS = BY + 2;
-  static constexpr int STAGE = ROWS * TX + 2 * BY;  // doubles
-  static constexpr size_t SMEM = (size_t)S * STAGE * 8 + (size_t)2 * S * 8;
-  static_assert(BY % RPP == 0 && NT % 32 == 0 && 2 * BY <= 32 * 8, "bad sweep config");
-};
-
-static __device__ __forceinline__ void cp_async_bar_arrive_noinc(uint64_t* bar) {
-  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
-
-template <int TX, int BY, int RPP, int S>
-__global__ void __launch_bounds__(TmaCfg<TX, BY, RPP, S>::NT + 32)
-    slab_sweep_tma(const ViewDev Sv, const ViewDev Dv, const int nx, const int ny, const int lo, const int hi,
-                   const double alpha) {
-  using C = TmaCfg<TX, BY, RPP, S>;
-  extern __shared__ __align__(128) unsigned char smem_raw[];
-  double* stage = reinterpret_cast<double*>(smem_raw);
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + (size_t)S * C::STAGE * 8);
-  uint64_t* empty = full + S;
-  if (threadIdx.x == 0) {
-    for (int s = 0; s < S; ++s) {
-      mbar_init(&full[s], 1 + 32);  // expect_tx arrive + 32 cp.async (noinc) arrivals
-      mbar_init(&empty[s], C::NT);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  const int cx = nx / TX;
-  const int np = hi - lo;
-  const int64_t ncols = (int64_t)cx * (ny / BY);
-  const int64_t P = ncols * np;
-  const int64_t pb = P * blockIdx.x / gridDim.x, pe = P * (blockIdx.x + 1) / gridDim.x;
-
-  if ((int)threadIdx.x >= C::NT) {  // ---------------- producer warp
-    const int lane = (int)threadIdx.x - C::NT;
-    uint32_t g = 0;
-    for (int64_t pp = pb; pp < pe;) {
-      const int64_t col = pp / np;
-      const int z0 = lo + (int)(pp - col * np);
-      const int64_t left_ = pe - pp, inrun_ = (int64_t)(lo + np - z0);
-      const int n = (int)(left_ < inrun_ ? left_ : inrun_);
-      pp += n;
-      const int x0 = (int)(col % cx) * TX, y0 = (int)(col / cx) * BY;
-      const int64_t xo = Sv.X(x0);
-      const int xl = x0 == 0 ? nx - 1 : x0 - 1, xr = x0 + TX == nx ? 0 : x0 + TX;
-      for (int q = 0; q < n + 2; ++q, ++g) {
-        const int z = z0 - 1 + q;
-        const int st = (int)(g % S);
-        mbar_wait(&empty[st], ((g / S) & 1u) ^ 1u);
-        double* dst = stage + (size_t)st * C::STAGE;
-        const double* pz = Sv.P(z);
-        if (lane == 0) {
-          fence_proxy_async();
-          mbar_expect_tx(&full[st], (uint32_t)C::ROWS * TX * 8);
-        }
-        __syncwarp();
-        for (int r = lane; r < C::ROWS; r += 32) {
-          int y = y0 - 1 + r;
-          y = y < 0 ? y + ny : (y >= ny ? y - ny : y);
-          bulk_g2s(dst + r * TX, pz + Sv.Y(y) + xo, TX * 8, &full[st]);
-        }
-        for (int k = lane; k < 2 * BY; k += 32) {
-          const int side = k / BY, j = k - side * BY;
-          const double* src = pz + Sv.Y(y0 + j) + Sv.X(side ? xr : xl);
-          asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst + C::ROWS * TX + k)),
-                       "l"(src)
-                       : "memory");
-        }
-        cp_async_bar_arrive_noinc(&full[st]);
-      }
-    }
-    return;
-  }
-
-  // ------------------------------------------------------- consumer warps
-  const int c2 = (int)threadIdx.x % C::HALF, r0 = (int)threadIdx.x / C::HALF;
-  const int x = 2 * c2;
-  const bool xl_edge = c2 == 0, xr_edge = c2 == C::HALF - 1;
-  uint32_t seq = 0;
-  auto wait_g = [&](uint32_t g) { mbar_wait(&full[g % S], (g / S) & 1u); };
-  auto release_g = [&](uint32_t g) { mbar_arrive(&empty[g % S]); };
-  for (int64_t pp = pb; pp < pe;) {
-    const int64_t col = pp / np;
-    const int z0 = lo + (int)(pp - col * np);
-    const int64_t left_ = pe - pp, inrun_ = (int64_t)(lo + np - z0);
-      const int n = (int)(left_ < inrun_ ? left_ : inrun_);
-    pp += n;
-    const int x0 = (int)(col % cx) * TX, y0 = (int)(col / cx) * BY;
-    int64_t orow[C::NR];
-#pragma unroll
-    for (int j = 0; j < C::NR; ++j) orow[j] = Dv.Y(y0 + r0 + j * RPP) + Dv.X(x0 + x);
-    double2 zm[C::NR], zc[C::NR];
-    wait_g(seq);
-    wait_g(seq + 1);
-    {
-      const double* s0 = stage + (size_t)(seq % S) * C::STAGE + (r0 + 1) * TX + x;
-      const double* s1 = stage + (size_t)((seq + 1) % S) * C::STAGE + (r0 + 1) * TX + x;
-#pragma unroll
-      for (int j = 0; j < C::NR; ++j) {
-        zm[j] = *reinterpret_cast<const double2*>(s0 + j * RPP * TX);
-        zc[j] = *reinterpret_cast<const double2*>(s1 + j * RPP * TX);
-      }
-    }
-    release_g(seq);
-    for (int i = 0; i < n; ++i) {
-      wait_g(seq + i + 2);
-      const double* cur = stage + (size_t)((seq + i + 1) % S) * C::STAGE;
-      const double* nxt = stage + (size_t)((seq + i + 2) % S) * C::STAGE + (r0 + 1) * TX + x;
-      const double* cc = cur + (r0 + 1) * TX + x;
-      const double* hx = cur + C::ROWS * TX;
-      double* od = Dv.P(z0 + i);
-#pragma unroll
-      for (int j = 0; j < C::NR; ++j) {
-        const int jo = j * RPP * TX;
-        const double2 zp = *reinterpret_cast<const double2*>(nxt + jo);
-        const double2 ym = *reinterpret_cast<const double2*>(cc + jo - TX);
-        const double2 yp = *reinterpret_cast<const double2*>(cc + jo + TX);
-        double xm = xl_edge ? hx[r0 + j * RPP] : cc[jo - 1];
-        double xp = xr_edge ? hx[BY + r0 + j * RPP] : cc[jo + 2];
-        const double2 c = zc[j];
-        double2 v;
-        v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm[j].x, zp.x, alpha);
-        v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm[j].y, zp.y, alpha);
-        stg2_stream(od + orow[j], v);
-        zm[j] = c;
-        zc[j] = zp;
-      }
-      release_g(seq + i + 1);
-    }
-    release_g(seq + n + 1);
-    seq += (uint32_t)(n + 2);
-  }
-}
-
-// ---- full-width band variant (the default where NX fits): a CTA's column is
-// a band of BY rows spanning the whole plane width NX, so the x neighbours,
-// periodic wrap included, are all in the staged rows: no x-halo loads. Per
-// plane the producer warp arms the stage's mbarrier with (BY + 2) rows of NX
-// doubles and its lanes issue one 1-D bulk copy per row segment (a whole row
-// for a dense view, one tile row of tx cells for tile-blocked views). 512
-// consumer threads own K = NX*BY/1024 cell pairs of every plane (same pairs
-// in every plane: register z-march); x neighbours by warp shuffle (the warp's
-// edge lanes read theirs from the stage), y neighbours from the staged rows.
-// One CTA per SM (the ring holds S planes of (BY+2) * NX * 8 bytes), each
-// owning a contiguous range of (band, plane) pairs.
-template <int NX, int BY, int S>
-struct RowCfg {
-  static constexpr int NT = 512;
-  static constexpr int HALF = NX / 2;
-  static constexpr int K = HALF * BY / NT;    // pairs per thread
-  static constexpr int ROWS = BY + 2;
-  static constexpr int STAGE = ROWS * NX;      // doubles
-  static constexpr size_t SMEM = (size_t)S * STAGE * 8 + (size_t)2 * S * 8;
-  static_assert(K >= 1 && HALF * BY == K * NT && HALF % 32 == 0, "bad row-sweep config");
-};
-
-template <int NX, int BY, int S>
-__global__ void __launch_bounds__(RowCfg<NX, BY, S>::NT + 32, 1)
-    slab_sweep_row(const ViewDev Sv, const ViewDev Dv, const int ny, const int lo, const int hi,
-                   const double alpha) {
-  using C = RowCfg<NX, BY, S>;
-  extern __shared__ __align__(128) unsigned char smem_raw[];
-  double* stage = reinterpret_cast<double*>(smem_raw);
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + (size_t)S * C::STAGE * 8);
-  uint64_t* empty = full + S;
-  if (threadIdx.x == 0) {
-    for (int s = 0; s < S; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&empty[s], C::NT);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  const int np = hi - lo;
-  const int64_t P = (int64_t)(ny / BY) * np;
-  const int64_t pb = P * blockIdx.x / gridDim.x, pe = P * (blockIdx.x + 1) / gridDim.x;
-
-  if ((int)threadIdx.x >= C::NT) {  // ---------------- producer warp
-    const int lane = (int)threadIdx.x - C::NT;
-    const int seg = Sv.tx < NX ? Sv.tx : NX;  // contiguous cells per row segment
-    const int nseg = NX / seg;
-    uint32_t g = 0;
-    for (int64_t pp = pb; pp < pe;) {
-      const int64_t band = pp / np;
-      const int z0 = lo + (int)(pp - band * np);
-      const int64_t left = pe - pp, inrun = lo + np - z0;
-      const int n = (int)(left < inrun ? left : inrun);
-      pp += n;
-      const int y0 = (int)band * BY;
-      for (int q = 0; q < n + 2; ++q, ++g) {
-        const int z = z0 - 1 + q;
-        const int st = (int)(g % S);
-        mbar_wait(&empty[st], ((g / S) & 1u) ^ 1u);
-        double* dst = stage + (size_t)st * C::STAGE;
-        const double* pz = Sv.P(z);
-        if (lane == 0) {
-          fence_proxy_async();
-          mbar_expect_tx(&full[st], (uint32_t)C::STAGE * 8);
-        }
-        __syncwarp();
-        for (int k = lane; k < C::ROWS * nseg; k += 32) {
-          const int r = k / nseg, sg = k - r * nseg;
-          int y = y0 - 1 + r;
-          y = y < 0 ? y + ny : (y >= ny ? y - ny : y);
-          bulk_g2s(dst + r * NX + sg * seg, pz + Sv.Y(y) + Sv.X(sg * seg), (uint32_t)seg * 8, &full[st]);
-        }
-      }
-    }
-    return;
-  }
-
-  // ------------------------------------------------------- consumer warps
-  const int tid = (int)threadIdx.x, lane = tid & 31;
-  // pair q = tid + k*NT of the band plane: row q / HALF, pair column q % HALF
-  // (NT is a multiple of HALF or HALF of NT/K... both compile-time: the row
-  // offset of pair k is tid's row plus a constant)
-  const int r0 = tid / C::HALF, c20 = tid - r0 * C::HALF;
-  constexpr int RSTEP = C::NT / C::HALF;  // rows between a thread's pairs (NT % HALF == 0)
-  static_assert(C::NT % C::HALF == 0, "row-sweep: NT must be a multiple of NX/2");
-  const int sbase = (r0 + 1) * NX + 2 * c20;  // stage offset of pair 0 (row + 1: the y halo)
-  const bool lft = lane == 0, rgt = lane == 31;  // warp edges (HALF % 32 == 0: rows start at lane 0)
-  const int xl = c20 == 0 ? NX - 1 : -1, xr = c20 == C::HALF - 1 ? 2 - NX : 2;  // periodic wrap
-  uint32_t seq = 0;
-  auto wait_g = [&](uint32_t g) { mbar_wait(&full[g % S], (g / S) & 1u); };
-  auto release_g = [&](uint32_t g) { mbar_arrive(&empty[g % S]); };
-  for (int64_t pp = pb; pp < pe;) {
-    const int64_t band = pp / np;
-    const int z0 = lo + (int)(pp - band * np);
-    const int64_t left = pe - pp, inrun = lo + np - z0;
-    const int n = (int)(left < inrun ? left : inrun);
-    pp += n;
-    const int y0 = (int)band * BY;
-    int orow[C::K];  // output offsets within the plane (host checks they fit int32)
-    const int64_t ox = Dv.X(2 * c20);
-#pragma unroll
-    for (int k = 0; k < C::K; ++k) orow[k] = (int)(Dv.Y(y0 + r0 + k * RSTEP) + ox);
-    double2 zm[C::K], zc[C::K];
-    wait_g(seq);
-    wait_g(seq + 1);
-    {
-      const double* s0 = stage + (size_t)(seq % S) * C::STAGE;
-      const double* s1 = stage + (size_t)((seq + 1) % S) * C::STAGE;
-#pragma unroll
-      for (int k = 0; k < C::K; ++k) {
-        zm[k] = *reinterpret_cast<const double2*>(s0 + sbase + k * RSTEP * NX);
-        zc[k] = *reinterpret_cast<const double2*>(s1 + sbase + k * RSTEP * NX);
-      }
-    }
-    release_g(seq);
-    for (int i = 0; i < n; ++i) {
-      wait_g(seq + i + 2);
-      const double* cur = stage + (size_t)((seq + i + 1) % S) * C::STAGE;
-      const double* nxt = stage + (size_t)((seq + i + 2) % S) * C::STAGE;
-      double* od = Dv.P(z0 + i);
-#pragma unroll
-      for (int k = 0; k < C::K; ++k) {
-        const double* cc = cur + sbase + k * RSTEP * NX;
-        const double2 c = zc[k];
-        const double2 zp = *reinterpret_cast<const double2*>(nxt + sbase + k * RSTEP * NX);
-        const double2 ym = *reinterpret_cast<const double2*>(cc - NX);
-        const double2 yp = *reinterpret_cast<const double2*>(cc + NX);
-        double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
-        double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
-        // warp edges and the periodic wrap: from the staged row
-        if (lft) xm = cc[xl];
-        if (rgt) xp = cc[xr];
-        double2 v;
-        v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm[k].x, zp.x, alpha);
-        v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm[k].y, zp.y, alpha);
-        stg2_stream(od + orow[k], v);
-        zm[k] = c;
-        zc[k] = zp;
-      }
-      release_g(seq + i + 1);
-    }
-    release_g(seq + n + 1);
-    seq += (uint32_t)(n + 2);
-  }
-}
-
-template <int NX, int BY, int S>
-static cudaError_t launch_row_cfg(const ViewDev& Sv, const ViewDev& Dv, int ny, int lo, int hi, double alpha,
-                                  int sms, cudaStream_t s) {
-  using C = RowCfg<NX, BY, S>;
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(slab_sweep_row<NX, BY, S>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)C::SMEM);
-    if (e != cudaSuccess) return e;
-    attr = true;
-  }
-  const int64_t P = (int64_t)(ny / BY) * (hi - lo);
-  const int64_t grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)sms, P / 4));
-  if ((int64_t)Dv.te * Dv.ntx * Dv.nty >= (1ll << 31) || (int64_t)Dv.tx * ny >= (1ll << 31))
-    return cudaErrorInvalidValue;  // plane offsets are int32 in the consumers
-  slab_sweep_row<NX, BY, S><<<(unsigned)grid, C::NT + 32, C::SMEM, s>>>(Sv, Dv, ny, lo, hi, alpha);
-  return cudaGetLastError();
-}
-
 // ---- tile-column TMA variant (the default for tile-blocked views of 64-wide
 // tiles): a CTA's column is a band of BY rows of one 64-wide tile column, so
 // per plane the producer issues five TMA operations, as heat7_fixed does —
@@ -830,15 +513,7 @@ static EncodeTiledFn encode_fn() {
   return f;
 }
 
-static int sweep_cfg() {  // TILES_SWEEP_CFG: tile-column kernel configuration (experiments)
-  static const int cfg = [] {
-    const char* e = getenv("TILES_SWEEP_CFG");
-    return e ? atoi(e) : 1;
-  }();
-  return cfg;
-}
-
-int sweep_tile_band() { return sweep_cfg() == 3 ? 64 : 32; }
+int sweep_tile_band() { return 32; }
 
 bool sweep_map_encode(SweepMaps* m, int k, const double* base, uint64_t bytes, int tx, int band) {
   static_assert(sizeof(CUtensorMap) == sizeof(TensorMapBlob), "CUtensorMap size");
@@ -863,29 +538,6 @@ bool sweep_map_encode(SweepMaps* m, int k, const double* base, uint64_t bytes, i
   return true;
 }
 
-template <int TX, int BY, int RPP, int S>
-static cudaError_t launch_tma_cfg(const ViewDev& Sv, const ViewDev& Dv, int nx, int ny, int lo, int hi,
-                                  double alpha, int sms, cudaStream_t s) {
-  using C = TmaCfg<TX, BY, RPP, S>;
-  static int occ = 0;
-  if (!occ) {
-    cudaError_t e = cudaFuncSetAttribute(slab_sweep_tma<TX, BY, RPP, S>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::SMEM);
-    if (e != cudaSuccess) return e;
-    int o = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, slab_sweep_tma<TX, BY, RPP, S>, C::NT + 32, C::SMEM);
-    occ = o < 1 ? 1 : o;
-  }
-  const int64_t P = (int64_t)(nx / TX) * (ny / BY) * (hi - lo);
-  // every CTA >= ~6 planes (each run stages 2 extra), at most the resident grid
-  const int64_t grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * occ, P / 6));
-  slab_sweep_tma<TX, BY, RPP, S><<<(unsigned)grid, C::NT + 32, C::SMEM, s>>>(Sv, Dv, nx, ny, lo, hi, alpha);
-  return cudaGetLastError();
-}
-
-static bool view_fits(const SlabView& v, int TX, int BY) {
-  return v.tx % TX == 0 && v.ty % BY == 0;
-}
 
 static int sweep_occupancy(int BY) {
   static int occ[3] = {0, 0, 0};
@@ -903,33 +555,20 @@ static int sweep_occupancy(int BY) {
 cudaError_t launch_slab_sweep(const SlabView& src, const SlabView& dst, int nx, int ny, int lo,
                               int hi, double alpha, int sms, cudaStream_t s, const SweepMaps* maps) {
   if (hi <= lo) return cudaSuccess;
+  // TILES_SWEEP_TMA=0: the cp.async kernel everywhere (A/B runs)
   static const int use_tma = [] {
     const char* e = getenv("TILES_SWEEP_TMA");
-    return e ? atoi(e) : 3;
+    return e ? atoi(e) : 1;
   }();
-  // 3 (default): tile columns with tensor-map x halos, for 64-wide tiled
-  // views whose memory the maps cover (every plane of the source)
+  // tile columns with tensor-map x halos, for 64-wide tiled views whose
+  // memory the maps cover (every plane of the source)
   const int tb = sweep_tile_band();
-  if (use_tma == 3 && maps && maps->valid[0] && maps->band == tb && !src.ring && src.tx == 64 && dst.tx == 64 &&
+  if (use_tma && maps && maps->valid[0] && maps->band == tb && !src.ring && src.tx == 64 && dst.tx == 64 &&
       src.ty % tb == 0 && dst.ty % tb == 0 && nx % 64 == 0 && ny % tb == 0 && !src.hhi &&
       (!src.hlo || (maps->valid[1] && src.hlo >= maps->base[1] && src.hlo < maps->end[1])))
-  {
-    const int cfg = sweep_cfg();
-    const ViewDev a = to_dev(src), b = to_dev(dst);
-    if (cfg == 0) return launch_tile_cfg<32, 16, 4, 2>(a, b, *maps, nx, ny, lo, hi, alpha, sms, s);
-    if (cfg == 2) return launch_tile_cfg<32, 8, 4, 3>(a, b, *maps, nx, ny, lo, hi, alpha, sms, s);
-    if (cfg == 3) return launch_tile_cfg<64, 16, 4, 1>(a, b, *maps, nx, ny, lo, hi, alpha, sms, s);
-    return launch_tile_cfg<32, 8, 4, 2>(a, b, *maps, nx, ny, lo, hi, alpha, sms, s);
-  }
-  // 1 (default): full-width bands; 2: 64-wide columns with cp.async x halos; 0: the cp.async kernel
-  if (use_tma == 1 && nx == 512 && ny % 8 == 0 && (src.tx == 512 || 512 % src.tx == 0) && src.ty % 8 == 0 &&
-      dst.ty % 8 == 0 && src.tx % 2 == 0 && dst.tx % 2 == 0)
-    return launch_row_cfg<512, 8, 4>(to_dev(src), to_dev(dst), ny, lo, hi, alpha, sms, s);
-  if (use_tma == 1 && nx == 256 && ny % 8 == 0 && (src.tx == 256 || 256 % src.tx == 0) && src.ty % 8 == 0 &&
-      dst.ty % 8 == 0 && src.tx % 2 == 0 && dst.tx % 2 == 0)
-    return launch_row_cfg<256, 8, 4>(to_dev(src), to_dev(dst), ny, lo, hi, alpha, sms, s);
-  if (use_tma == 2 && nx % 64 == 0 && ny % 16 == 0 && view_fits(src, 64, 16) && view_fits(dst, 64, 16))
-    return launch_tma_cfg<64, 16, 8, 4>(to_dev(src), to_dev(dst), nx, ny, lo, hi, alpha, sms, s);
+    // band 32, 4 rows per consumer thread, 4 stages, 2 CTAs per SM (band 16 or 64, 3 CTAs per SM
+    // and 6 stages measured slower: profiles/r02/bench_sweep_cfg*.json)
+    return launch_tile_cfg<32, 8, 4, 2>(to_dev(src), to_dev(dst), *maps, nx, ny, lo, hi, alpha, sms, s);
   const int npairs = nx / 2;
   const int gx = (npairs + 127) / 128;
   // rows per thread: must divide every view's ty (the dense slab's is ny,

@@ -1,4 +1,3 @@
 python -c "import __graft_entry__ as g; g.build()" || exit 1
-timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_fullsize.py -m gpu -x -q -k "wavefront" 2>&1 | tail -2
-for bg in 4 1 2 8; do TILES_WAVE_BIG=$bg timeout 600 python bench.py --config fig5 --steps 1 --sweep 32,48,64,100 --wavefront 1 > gpurun_out/fig5_big$bg.json 2>/dev/null
-python -c "import json;j=json.loads(open('gpurun_out/fig5_big$bg.json').read().strip().splitlines()[-1]);print($bg, {T:(round(r['tiled']['ms'],1), round(r['tiled_frac_of_bound'],3)) for T,r in j['sweep'].items()})"; done
+for mu in 16 32 64 16 32; do TILES_ST_MINUNIT=$mu timeout 600 python bench.py --no-cpu-baseline --no-extras --steps 20 > gpurun_out/bench_mu$mu.json 2>/dev/null
+python -c "import json;j=json.loads(open('gpurun_out/bench_mu$mu.json').read().strip().splitlines()[-1]);print($mu, round(j['value'],2), round(j['ms_per_step'],2), 'sweep', round(j['roofline']['achieved']), round(j['roofline']['frac'],3), round(j['roofline']['avg_launch_ms']*1e3,1), j['roofline']['launches_per_step'])"; done
