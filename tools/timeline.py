@@ -2,7 +2,7 @@
 (nsys is not in the image). Writes a chrome trace and an overlap summary:
 busy time of kernels, H2D and D2H and their pairwise overlaps.
 
-  python tools/timeline.py {c4|c3|c2} out_prefix
+  python tools/timeline.py {c4|c3|c2|wave} out_prefix
 """
 import json
 import os
@@ -48,6 +48,8 @@ def main():
         n, td, kern, steps, kw = 512, (64, 64, 64), T.sincos(32), 10, {}
     elif cfg == "c2":
         n, td, kern, steps, kw = 512, (64, 64, 64), T.heat7(), 10, {}
+    elif cfg == "wave":   # C2 shape, fresh upload at T = 64: the wavefront schedule
+        n, td, kern, steps, kw = 512, (64, 64, 64), T.heat7(), 64, {}
     else:  # small out-of-core heat, budget for 8 tiles
         n, td, kern, steps, kw = 512, (128, 128, 128), T.heat7(), 2, {"sched": "stream",
                                                                         "device_budget_bytes": 1200 << 20}
@@ -55,7 +57,7 @@ def main():
     u = np.empty((n, n, n))
     synth.fill_uniform_native(u.ctypes.data, n, n, n, 0, n, 0, n, 0, n, 7)
     d.load(u)
-    d.run(kern, 1, 4)
+    d.run(kern, steps, 4)  # warm-up at the same T (schedule, scratch)
     d.sync()
     d.invalidate()
     torch.cuda.synchronize()
