@@ -1173,6 +1173,16 @@ def run_main_leg(args):
                 dom.run(k, T, ns)
                 dom.sync()
             ov["cupti"] = cupti_overlap(torch, one)
+            kb = ov["cupti"]["kernel_busy_ms"] if ov["cupti"] else 0
+            if kb and sw_cells:
+                # the same step's kernels as the GPU ran them inside the
+                # pipeline (CUPTI activity records: with programmatic dependent
+                # launch the sweeps overlap their neighbours' ramp and drain,
+                # which per-launch CUDA events cannot show)
+                ach = 16.0 * (sw_cells / args.steps) / (kb / 1e3) / 1e9
+                roof.update({"achieved_in_pipeline": ach, "frac_in_pipeline": ach / peak,
+                             "in_pipeline_def": "16 B x cells swept per step / the step's CUPTI kernel-busy "
+                                                "time (union of kernel intervals; only sweeps run in it)"})
         except Exception as e:  # profiler unavailable: say so
             ov["cupti"] = {"error": str(e)[:200]}
         bw = pcie_bandwidth(torch)

@@ -1,3 +1,8 @@
 python -c "import __graft_entry__ as g; g.build()" || exit 1
-for mu in 16 32 64 16 32; do TILES_ST_MINUNIT=$mu timeout 600 python bench.py --no-cpu-baseline --no-extras --steps 20 > gpurun_out/bench_mu$mu.json 2>/dev/null
-python -c "import json;j=json.loads(open('gpurun_out/bench_mu$mu.json').read().strip().splitlines()[-1]);print($mu, round(j['value'],2), round(j['ms_per_step'],2), 'sweep', round(j['roofline']['achieved']), round(j['roofline']['frac'],3), round(j['roofline']['avg_launch_ms']*1e3,1), j['roofline']['launches_per_step'])"; done
+timeout 600 python -m pytest tests/test_gpu_parity.py -m gpu -x -q -k "wavefront or stream_through" 2>&1 | tail -1
+timeout 900 python bench.py --config fig5 --steps 1 > gpurun_out/fig5_final2.json 2>/dev/null
+python -c "import json;j=json.loads(open('gpurun_out/fig5_final2.json').read().strip().splitlines()[-1]);print({T:(round(r['tiled']['ms'],1), round(r['tiled_frac_of_bound'],3), round(r['tiled_frac_of_causal_bound'],3), round(r['speedup_tiled_vs_sync'],2)) for T,r in j['sweep'].items()})"
+mkdir -p gpurun_out/tl
+timeout 600 python tools/timeline.py wave gpurun_out/tl/timeline_wave64 > /dev/null 2>&1; cat gpurun_out/tl/timeline_wave64.summary.json
+timeout 600 python tools/timeline.py c2 gpurun_out/tl/timeline_c2 > /dev/null 2>&1; cat gpurun_out/tl/timeline_c2.summary.json
+rm -f gpurun_out/tl/*.trace.json
