@@ -43,7 +43,8 @@ CONFIGS = {
     # name: (per-GPU dims, tile dims, T, nstreams, description)
     "c1": ((64, 64, 64), (32, 32, 32), 10, 2, "C1 heat fp64 64^3, 2x2x2 tiles, g=1, T=10, 2 streams"),
     "c2": ((512, 512, 512), (64, 64, 64), 10, 4,
-           "C2 heat fp64 512^3, 8^3 tiles (64^3 cells), g=1, resident in HBM, T=10, 4 streams"),
+           "C2 heat fp64 512^3, 8^3 tiles (64^3 cells), g=1, T=10, 4 streams; every cell's H2D and D2H "
+           "inside the step (fresh upload from the pinned host store)"),
 }
 ALPHA = 0.125
 METRIC = "Gcell-updates/s incl. H2D/D2H at 1/2/4/8 B200; % transfer time hidden"
