@@ -181,7 +181,10 @@ typedef struct {
                                    the periodic seam. -1 =
                                    never, 0 (default) = when the cost model
                                    prefers it to stream-through and the
-                                   batched schedule, 1 = whenever feasible */
+                                   batched schedule, 1 = whenever feasible
+                                   (two levels per pass through a third level
+                                   buffer when the budget holds it), 2 =
+                                   whenever feasible, one level per pass */
   double sweep_link_ratio;      /* cost model of the fresh-upload schedules
                                    (DESIGN.md §5): time of one stencil sweep
                                    per plane over one plane's duplex host-link
@@ -283,14 +286,20 @@ typedef enum {
                             the pinned store (face extraction) happen here */
   TILE_OP_WSWEEP = 26,   /* wavefront sweep of planes [lo, hi) (c = lo | hi << 32, two
                             signed 32-bit halves), periodic in x/y; a = source view, b =
-                            destination view: bit 0 = 1: planes z >= 0 in resident array
-                            (bit 1), z < 0 in the d tile layers of scratch starting at
-                            slot (code >> 2); bit 0 = 0: resident array (bit 1), z
-                            wrapped (no scratch) */
+                            destination view: bit 0 = 1: planes z >= 0 in the tile-blocked
+                            array starting at slot (code >> 1) & 0x7fffffff, z < 0 in the d
+                            tile layers of scratch starting at slot code >> 32; bit 0 = 0:
+                            resident array (bit 1), z wrapped (no scratch) */
   TILE_OP_D2H_PLANES = 27,/* planes [d & 0xffffffff, + d >> 32) of c tile slots b.. ->
                             the same planes of host tiles a.. */
-  TILE_OP_COPY_PLANES = 28/* planes [d & 0xffffffff, + d >> 32) of c tile slots a.. ->
+  TILE_OP_COPY_PLANES = 28,/* planes [d & 0xffffffff, + d >> 32) of c tile slots a.. ->
                             the same planes of slots b.. */
+  TILE_OP_WSWEEP2 = 29,  /* wavefront, two levels in one kernel (recorded as this op and the
+                            next, TILE_OP_WSWEEP2_DST, on the same stream): level s on planes
+                            [lo, hi) (c = lo | hi << 32, signed halves) from view a, written to
+                            view b only at planes hi-2, hi-1 (its planes lo-2, lo-1 are read
+                            from b); d = scratch layers. Views coded as for TILE_OP_WSWEEP */
+  TILE_OP_WSWEEP2_DST = 30/* the same kernel: level s+1 on [lo-1, hi-1) into view a */
 } tile_op_kind;
 
 typedef struct {

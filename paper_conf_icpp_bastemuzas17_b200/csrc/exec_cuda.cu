@@ -382,7 +382,7 @@ struct CudaExec final : Exec {
         v.hhi = d.st_halo[1];
       }
     } else if (r.kind == SlabRef::WAVE) {
-      v.base = d.slot_ptr(r.slot ? (int)G.ntiles : 0);
+      v.base = d.slot_ptr(r.slot);  // the level's tile-blocked array (its first slot)
       v.te = G.tile_elems;
       v.tz = (int)G.t[2];
       v.zbase = 0;
@@ -415,6 +415,33 @@ struct CudaExec final : Exec {
       return launch_slab_sweep(s, t, (int)d.G.l[0], (int)d.G.l[1], lo, hi, d.kernel_alpha, sms, S(st), &maps);
     });
     if (r.bad()) return r;
+    d.stats.n_kernels++;
+    return Status::ok();
+  }
+  Status slab_sweep2(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, int a, int b,
+                     int st) override {
+    INJECT(FAULT_KERNEL, st);
+    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
+    ensure_maps(d);
+    const SlabView s = slab_view(d, src, a), m = slab_view(d, mid, a), t = slab_view(d, dst, a);
+    bool fused = true;
+    next_cells = d.kernel_timing ? (uint64_t)(b - a) * d.G.l[0] * d.G.l[1] : 0;  // one pass over the cells
+    Status r = timed(d, st, [&] {
+      const cudaError_t e = launch_slab_sweep2(s, m, t, (int)d.G.l[0], (int)d.G.l[1], a, b, d.kernel_alpha, sms,
+                                               S(st), &maps);
+      if (e == cudaErrorNotSupported) {
+        fused = false;
+        cudaGetLastError();
+        return cudaSuccess;
+      }
+      return e;
+    });
+    if (r.bad()) return r;
+    if (!fused) {  // shapes the fused kernel does not cover: both levels in full, one after the other
+      r = slab_sweep(d, src, mid, a, b, st);
+      if (r.bad()) return r;
+      return slab_sweep(d, mid, dst, a - 1, b - 1, st);
+    }
     d.stats.n_kernels++;
     return Status::ok();
   }

@@ -105,7 +105,7 @@ struct DryExec final : Exec {
       // zbase 0; bit 1: the resident array; bits 2..: WAVE scratch slot);
       // c: lo, hi as two signed 32-bit halves; d: scratch layers (nlo)
       auto code = [](const SlabRef& r) {
-        return r.kind == SlabRef::WAVE ? 1 | ((int64_t)r.slot << 1) | ((int64_t)r.ring[0] << 2)
+        return r.kind == SlabRef::WAVE ? 1 | ((int64_t)r.slot << 1) | ((int64_t)r.ring[0] << 32)
                                        : ((int64_t)r.slot << 1);
       };
       put(d, TILE_OP_WSWEEP, st, code(src), code(dst),
@@ -118,6 +118,19 @@ struct DryExec final : Exec {
     const int64_t b = dst.kind == SlabRef::DENSE ? dst.slot : -1 - (int64_t)dst.slot;
     put(d, TILE_OP_SWEEP, st, a, b, (int64_t)lo | ((int64_t)hi << 32),
         src.kind == SlabRef::RESIDENT ? src.zbase : 0);
+    return Status::ok();
+  }
+  Status slab_sweep2(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, int a, int b,
+                     int st) override {
+    if (Status f_ = inject(d, FAULT_KERNEL); f_.bad()) return f_;
+    d.stats.n_kernels++;
+    auto code = [](const SlabRef& r) {
+      return r.kind == SlabRef::WAVE ? 1 | ((int64_t)r.slot << 1) | ((int64_t)r.ring[0] << 32) : ((int64_t)r.slot << 1);
+    };
+    // one kernel, two records (a trace entry has four operands): the
+    // parameters, then the destination view (the replay executes at the second)
+    put(d, TILE_OP_WSWEEP2, st, code(src), code(mid), (int64_t)(uint32_t)a | ((int64_t)(uint32_t)b << 32), dst.un);
+    put(d, TILE_OP_WSWEEP2_DST, st, code(dst), 0, 0, 0);
     return Status::ok();
   }
   Status h2d_pack(Domain& d, int64_t t0, int64_t n, int ps, int64_t p0, int64_t np, int st) override {

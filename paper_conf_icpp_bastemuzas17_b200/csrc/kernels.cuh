@@ -189,6 +189,7 @@ struct alignas(64) TensorMapBlob {
 };
 struct SweepMaps {
   TensorMapBlob xmap[2];
+  TensorMapBlob xmap2[2];  // the same memory, box {2, 2} (the two-level sweep's extra halo rows)
   const double* base[2];
   const double* end[2];
   int valid[2];
@@ -197,6 +198,13 @@ struct SweepMaps {
 // encode map k over [base, base + bytes) as rows of tx doubles, box {2, band}
 bool sweep_map_encode(SweepMaps* m, int k, const double* base, uint64_t bytes, int tx, int band);
 int sweep_tile_band();  // box rows (band) of the tile-column sweep kernel
+// Two levels per pass (wavefront with three level buffers):
+// level s on planes [a, b) from src (level s-1) stays on chip except its top
+// two planes, written to mid (whose planes a-2, a-1 it reads); level s+1 on
+// [a-1, b-1) into dst. src and dst must not share memory. Returns
+// cudaErrorNotSupported when the shapes do not fit.
+cudaError_t launch_slab_sweep2(const SlabView& src, const SlabView& mid, const SlabView& dst, int nx, int ny, int a,
+                               int b, double alpha, int sms, cudaStream_t s, const SweepMaps* maps);
 // device -> mapped pinned host rows copied by the SMs (pitches, len in doubles;
 // len and pitches even)
 cudaError_t launch_push_rows(const double* src, int64_t src_pitch, double* dst, int64_t dst_pitch, int64_t rows,

@@ -513,6 +513,294 @@ static EncodeTiledFn encode_fn() {
   return f;
 }
 
+// ---- two levels per pass: slab_sweep2_tile (the wavefront with three level
+// buffers). A CTA owns runs of (band column, level-s+1 plane) pairs, as
+// slab_sweep_tile does; a run of level-s+1 planes [p0, p1) needs level s on
+// [p0-1, p1+1): planes below a (a-2, a-1: the previous chunk's top) are read
+// through view mid, the others computed here from level s-1 on the band plus
+// one row and one column on each side. Staging (one producer thread, nine
+// TMA operations per plane): level s-1 rows y0-2 .. y0+BY+1 of the tile
+// column (band; two contiguous row pairs, each inside one tile) and the x
+// halos x0-2, x0-1 / x0+64, x0+65 of those rows (tensor-map boxes {2, BY} and
+// {2, 2}). Consumers: warp w owns band rows w and w+16 (one pair per lane:
+// x neighbours by shuffle) and, warps 0/1, the extended rows y0-1 / y0+BY;
+// warps 2..4 compute the 68 extended-column cells (x = -1, 64). Both levels
+// march z in registers (level s-1 at z-1, z; level s at z-2, z-1, z), so per
+// cell pair and level only the y neighbours and the next plane come from
+// shared memory; level s goes through a 3-plane shared ring for the other
+// threads' y neighbours and the x edges, one named barrier per plane.
+namespace w2 {
+constexpr int BY = 32, TX = 64, NT = 512, S = 4;
+constexpr int SROWS = BY + 4;                     // staged rows: y0-2 .. y0+BY+1
+constexpr int XH = SROWS * TX;                    // x halos: per side boxes at 128-byte boundaries
+constexpr int HS = 96;                            // doubles per side: rows 0-1 | 2..BY+1 | BY+2..BY+3
+constexpr int STAGE = XH + 2 * HS;                // doubles (multiple of 16)
+constexpr uint32_t BYTES = (uint32_t)(SROWS * TX + 4 * SROWS) * 8;
+constexpr int MROWS = BY + 2, MW = 68;            // level-s plane: rows y0-1 .. y0+BY, x -2 .. 65
+constexpr int MID = MROWS * MW;
+constexpr size_t SMEM = (size_t)S * STAGE * 8 + (size_t)3 * MID * 8 + (size_t)2 * S * 8;
+static_assert(STAGE % 16 == 0 && MID % 2 == 0 && NT == 16 * 32, "layout");
+__device__ __forceinline__ int hoff(int side, int sr) {  // x-halo pair of staged row sr
+  const int o = side * HS;
+  return sr < 2 ? o + 2 * sr : sr < BY + 2 ? o + 16 + 2 * (sr - 2) : o + 80 + 2 * (sr - BY - 2);
+}
+}  // namespace w2
+
+static __device__ __forceinline__ void bar_consumers512() { asm volatile("bar.sync 1, 512;" ::: "memory"); }
+
+__global__ void __launch_bounds__(w2::NT + 32, 1)
+    slab_sweep2_tile(const ViewDev Sv, const ViewDev Mv, const ViewDev Dv, const __grid_constant__ SweepMaps maps,
+                     const int ny, const int a, const int b, const double alpha) {
+  using namespace w2;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double* stage = reinterpret_cast<double*>(smem_raw);
+  double* mid = stage + (size_t)S * STAGE;
+  uint64_t* full = reinterpret_cast<uint64_t*>(mid + (size_t)3 * MID);
+  uint64_t* empty = full + S;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], NT);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  const int ntx = Sv.ntx * Sv.tx / TX;
+  const int np = b - a;  // level s+1 planes [a-1, b-1)
+  const int64_t ncols = (int64_t)ntx * (ny / BY);
+  const int64_t P = ncols * np;
+  const int64_t pb = P * blockIdx.x / gridDim.x, pe = P * (blockIdx.x + 1) / gridDim.x;
+  auto run_at = [&](int64_t pp, int64_t& col, int& p0, int& p1) {
+    col = pp / np;
+    p0 = a - 1 + (int)(pp - col * np);
+    const int64_t left = pe - pp, inrun = (int64_t)(b - 1 - p0);
+    p1 = p0 + (int)(left < inrun ? left : inrun);
+  };
+  auto plan = [&](int p0, int p1, int& zc0, int& nload) {
+    zc0 = p0 - 1 > a ? p0 - 1 : a;  // first computed level-s plane
+    const int nl = (a < p1 + 1 ? a : p1 + 1) - (p0 - 1);
+    nload = nl > 0 ? nl : 0;        // level-s planes read: p0-1 .. p0-2+nload
+  };
+
+  if ((int)threadIdx.x >= NT) {  // ---------------- producer (one thread)
+    if (threadIdx.x != NT) return;
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    uint32_t g = 0;
+    for (int64_t pp = pb; pp < pe;) {
+      int64_t col;
+      int p0, p1, zc0, nload;
+      run_at(pp, col, p0, p1);
+      pp += p1 - p0;
+      plan(p0, p1, zc0, nload);
+      const int cx = (int)(col % ntx), y0 = (int)(col / ntx) * BY;
+      const int x0 = cx * TX, xl = (cx == 0 ? ntx - 1 : cx - 1) * TX, xr = (cx == ntx - 1 ? 0 : cx + 1) * TX;
+      const int ya = y0 < 2 ? y0 - 2 + ny : y0 - 2;
+      const int yb = y0 + BY + 2 > ny ? y0 + BY - ny : y0 + BY;
+      const int nstg = (p1 + 1) - zc0 + 2;  // level s-1 planes zc0-1 .. p1+1
+      for (int q = 0; q < nload + nstg; ++q, ++g) {
+        const bool ld = q < nload;
+        const ViewDev& V = ld ? Mv : Sv;
+        const int z = ld ? p0 - 1 + q : zc0 - 1 + (q - nload);
+        const int st = (int)(g % S);
+        mbar_wait(&empty[st], ((g / S) & 1u) ^ 1u);
+        double* dst = stage + (size_t)st * STAGE;
+        const double* pz = V.P(z);
+        fence_proxy_async();
+        mbar_expect_tx(&full[st], BYTES);
+        bulk_g2s(dst + 2 * TX, pz + V.Y(y0) + V.X(x0), (uint32_t)BY * TX * 8, &full[st]);
+        bulk_g2s(dst, pz + V.Y(ya) + V.X(x0), 2 * TX * 8, &full[st]);
+        bulk_g2s(dst + (BY + 2) * TX, pz + V.Y(yb) + V.X(x0), 2 * TX * 8, &full[st]);
+        const int yy[3] = {ya, y0, yb};
+        const int boff[3] = {0, 16, 80};
+#pragma unroll
+        for (int h = 0; h < 3; ++h) {
+          const double* cl = pz + V.Y(yy[h]) + V.X(xl);
+          const double* cr = pz + V.Y(yy[h]) + V.X(xr);
+          const int kl = (cl >= maps.base[1] && cl < maps.end[1]) ? 1 : 0;
+          const int kr = (cr >= maps.base[1] && cr < maps.end[1]) ? 1 : 0;
+          tma_2d(dst + XH + boff[h], h == 1 ? &maps.xmap[kl] : &maps.xmap2[kl], TX - 2,
+                 (int)((cl - maps.base[kl]) / TX), &full[st]);
+          tma_2d(dst + XH + HS + boff[h], h == 1 ? &maps.xmap[kr] : &maps.xmap2[kr], 0,
+                 (int)((cr - maps.base[kr]) / TX), &full[st]);
+        }
+      }
+    }
+    return;
+  }
+
+  // ------------------------------------------------------- consumer warps
+  const int t = (int)threadIdx.x, lane = t & 31, warp = t >> 5;
+  const int x = 2 * lane;
+  // pairs: k = 0, 1 band rows warp, warp + 16 (stage row +2, mid row +1);
+  // k = 2 (warps 0, 1): the extended rows y0-1 (mid row 0) / y0+BY (mid row 33)
+  const bool ext = warp < 2;
+  const int srow[3] = {warp + 2, warp + 18, warp == 0 ? 1 : BY + 2};
+  const int mrow[3] = {warp + 1, warp + 17, warp == 0 ? 0 : BY + 1};
+  const bool edge = t >= 64 && t < 64 + 2 * MROWS;  // an extended-column cell x = -1 / 64
+  const int eside = (t - 64) / MROWS, er = (t - 64) - eside * MROWS, ex = eside ? TX : -1;
+  uint32_t seq = 0;
+  auto wait_g = [&](uint32_t g) { mbar_wait(&full[g % S], (g / S) & 1u); };
+  auto release_g = [&](uint32_t g) { mbar_arrive(&empty[g % S]); };
+  auto sv = [&](const double* st, int sr, int xx) -> double {  // staged cell, xx in [-2, 66)
+    return xx < 0 ? st[XH + hoff(0, sr) + (xx + 2)] : xx >= TX ? st[XH + hoff(1, sr) + (xx - TX)] : st[sr * TX + xx];
+  };
+  for (int64_t pp = pb; pp < pe;) {
+    int64_t col;
+    int p0, p1, zc0, nload;
+    run_at(pp, col, p0, p1);
+    pp += p1 - p0;
+    plan(p0, p1, zc0, nload);
+    const int cx = (int)(col % ntx), y0 = (int)(col / ntx) * BY;
+    const int base = p0 - 1;  // ring slot of level-s plane z: (z - base) % 3
+    int64_t od[2], om[2];
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+      od[k] = Dv.Y(y0 + mrow[k] - 1) + Dv.X(cx * TX + x);
+      om[k] = Mv.Y(y0 + mrow[k] - 1) + Mv.X(cx * TX + x);
+    }
+    // level s of the own band pairs at planes z-2, z-1 (l2, l1): filled by the
+    // loaded planes or by the first computed ones
+    double2 l1[2], l2[2];
+    for (int q = 0; q < nload; ++q) {
+      wait_g(seq + q);
+      const double* st = stage + (size_t)((seq + q) % S) * STAGE;
+      double* m = mid + (size_t)((p0 - 1 + q - base) % 3) * MID;
+      for (int i = t; i < MROWS * 66; i += NT) {
+        const int r = i / 66, xx = i - r * 66 - 1;
+        m[r * MW + xx + 2] = sv(st, r + 1, xx);
+      }
+#pragma unroll
+      for (int k = 0; k < 2; ++k) {
+        l2[k] = l1[k];
+        l1[k] = *reinterpret_cast<const double2*>(st + srow[k] * TX + x);
+      }
+      release_g(seq + q);
+    }
+    const uint32_t s0 = seq + nload;  // stage of level s-1 plane zc0-1
+    // level s-1 of the own pairs at planes z-1, z (register march)
+    double2 cm[3], cc[3];
+    wait_g(s0);
+    wait_g(s0 + 1);
+    {
+      const double* a0 = stage + (size_t)(s0 % S) * STAGE;
+      const double* a1 = stage + (size_t)((s0 + 1) % S) * STAGE;
+#pragma unroll
+      for (int k = 0; k < 3; ++k) {
+        if (k == 2 && !ext) break;
+        cm[k] = *reinterpret_cast<const double2*>(a0 + srow[k] * TX + x);
+        cc[k] = *reinterpret_cast<const double2*>(a1 + srow[k] * TX + x);
+      }
+    }
+    for (int z = zc0; z <= p1; ++z) {
+      const uint32_t gz = s0 + (uint32_t)(z - (zc0 - 1));  // stage of level s-1 plane z
+      wait_g(gz + 1);
+      const double* s00 = stage + (size_t)(gz % S) * STAGE;
+      const double* sp1 = stage + (size_t)((gz + 1) % S) * STAGE;
+      double* m = mid + (size_t)((z - base) % 3) * MID;
+      const bool top = z >= b - 2;
+      double* mo = top ? Mv.P(z) : nullptr;
+      double2 lv[2];
+      // level s at z, own pairs
+#pragma unroll
+      for (int k = 0; k < 3; ++k) {
+        if (k == 2 && !ext) break;
+        const int sr = srow[k];
+        const double2 c = cc[k];
+        const double2 zp = *reinterpret_cast<const double2*>(sp1 + sr * TX + x);
+        const double2 ym = *reinterpret_cast<const double2*>(s00 + (sr - 1) * TX + x);
+        const double2 yp = *reinterpret_cast<const double2*>(s00 + (sr + 1) * TX + x);
+        double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+        double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+        if (lane == 0) xm = s00[XH + hoff(0, sr) + 1];
+        if (lane == 31) xp = s00[XH + hoff(1, sr)];
+        double2 v;
+        v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, cm[k].x, zp.x, alpha);
+        v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, cm[k].y, zp.y, alpha);
+        *reinterpret_cast<double2*>(m + mrow[k] * MW + x + 2) = v;
+        if (k < 2) {
+          lv[k] = v;
+          if (top) *reinterpret_cast<double2*>(mo + om[k]) = v;
+        }
+        cm[k] = c;
+        cc[k] = zp;
+      }
+      if (edge) {  // the extended columns x = -1 / 64 (stage z-1 still held: released below)
+        const double* sm1 = stage + (size_t)((gz - 1) % S) * STAGE;
+        const int sr = er + 1;
+        const double c = sv(s00, sr, ex);
+        m[er * MW + ex + 2] = heat_update(c, sv(s00, sr, ex - 1), sv(s00, sr, ex + 1), sv(s00, sr - 1, ex),
+                                          sv(s00, sr + 1, ex), sv(sm1, sr, ex), sv(sp1, sr, ex), alpha);
+      }
+      release_g(gz - 1);  // level s-1 plane z-1: no reader left
+      bar_consumers512();  // level s plane z-1 (written last step) complete in the ring
+      const int w = z - 1;
+      if (w >= p0) {  // level s+1 at w: z-march in registers, y / x neighbours of plane w from the ring
+        const double* mw = mid + (size_t)((w - base) % 3) * MID;
+        double* dw = Dv.P(w);
+#pragma unroll
+        for (int k = 0; k < 2; ++k) {
+          const double* p = mw + mrow[k] * MW + x + 2;
+          const double2 c = l1[k];
+          const double2 ym = *reinterpret_cast<const double2*>(p - MW);
+          const double2 yp = *reinterpret_cast<const double2*>(p + MW);
+          double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+          double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+          if (lane == 0) xm = p[-1];
+          if (lane == 31) xp = p[2];
+          double2 v;
+          v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, l2[k].x, lv[k].x, alpha);
+          v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, l2[k].y, lv[k].y, alpha);
+          stg2_stream(dw + od[k], v);
+        }
+      }
+#pragma unroll
+      for (int k = 0; k < 2; ++k) {
+        l2[k] = l1[k];
+        l1[k] = lv[k];
+      }
+    }
+    // the last two staged planes (p1, p1+1 of level s-1)
+    const uint32_t glast = s0 + (uint32_t)(p1 + 1 - (zc0 - 1));
+    release_g(glast - 1);
+    release_g(glast);
+    seq = glast + 1;
+    bar_consumers512();  // the ring is reused by the next run
+  }
+}
+
+cudaError_t launch_slab_sweep2(const SlabView& src, const SlabView& mid, const SlabView& dst, int nx, int ny, int a,
+                               int b, double alpha, int sms, cudaStream_t s, const SweepMaps* maps) {
+  using namespace w2;
+  if (b <= a) return cudaSuccess;
+  if (b - a < 2 || !maps || !maps->valid[0] || maps->band != BY || src.ring || mid.ring || src.hhi || mid.hhi ||
+      src.tx != TX || mid.tx != TX || dst.tx != TX || src.ty % 64 || mid.ty % 64 || dst.ty % BY || nx % TX ||
+      ny % 64 || nx / TX < 2)
+    return cudaErrorNotSupported;
+  for (const SlabView* v : {&src, &mid})
+    if (v->hlo && !(maps->valid[1] && v->hlo >= maps->base[1] && v->hlo < maps->end[1]))
+      return cudaErrorNotSupported;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(slab_sweep2_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  const int64_t P = (int64_t)(nx / TX) * (ny / BY) * (b - a);
+  const int64_t grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)sms, P / 8));
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(NT + 32);
+  cfg.dynamicSmemBytes = SMEM;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, slab_sweep2_tile, to_dev(src), to_dev(mid), to_dev(dst), *maps, ny, a, b, alpha);
+}
+
 int sweep_tile_band() { return 32; }
 
 bool sweep_map_encode(SweepMaps* m, int k, const double* base, uint64_t bytes, int tx, int band) {
@@ -530,6 +818,11 @@ bool sweep_map_encode(SweepMaps* m, int k, const double* base, uint64_t bytes, i
   if (f(tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double*>(base), dims, strides, box, estr,
         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    return false;
+  const cuuint32_t box2[2] = {2, 2};
+  if (f(reinterpret_cast<CUtensorMap*>(&m->xmap2[k]), CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<double*>(base),
+        dims, strides, box2, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+        CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
     return false;
   m->base[k] = base;
   m->end[k] = base + rows * tx;

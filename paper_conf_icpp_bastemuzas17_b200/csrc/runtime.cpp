@@ -1249,6 +1249,7 @@ static Status run_streamthrough_ooc(Domain& d, int T, int S, const OocPlan& op) 
 // it; the two planes iteration i+1 reads lie above level s+2's chunk of
 // iteration i) — checked on CPU by the random-order replay of the trace.
 struct WavePlan {
+  bool fused = false;  // two levels per pass (three level buffers)
   int64_t c = 0;    // chunk planes (divides tz)
   int64_t B = 0;    // bootstrap region: the top B planes, uploaded first (multiple of c, >= 2T)
   int64_t nlo = 0;  // scratch tile layers per parity
@@ -1276,9 +1277,18 @@ static bool wavefront_ok(const Domain& d, int T, WavePlan* wp) {
   const int64_t B = (2 * (int64_t)T + c - 1) / c * c;
   if (B + c > nz) return false;  // the seam's cone would cover the ring
   const int64_t nlo = (2 * (int64_t)T + tz - 1) / tz;
-  const uint64_t need = (uint64_t)(2 * nlo * G.layer_tiles) * (uint64_t)G.tile_elems * 8;
-  if ((int64_t)d.wave_slots < 2 * nlo * G.layer_tiles && need > d.budget_left + (uint64_t)d.wave_slots * G.tile_elems * 8)
-    return false;
+  // two levels per pass (TILES_WAVE_FUSE, default on) take a third level
+  // array (ntiles slots) and three scratch parities, when the budget has them
+  static const int fuse = [] {
+    const char* e = getenv("TILES_WAVE_FUSE");
+    return e ? atoi(e) : 1;
+  }();
+  const uint64_t avail = d.budget_left + (uint64_t)d.wave_slots * G.tile_elems * 8;
+  const int64_t slots3 = G.ntiles + 3 * nlo * G.layer_tiles, slots2 = 2 * nlo * G.layer_tiles;
+  wp->fused = fuse && d.opt.wavefront != 2 && T >= 2 &&
+              (d.wave_slots >= slots3 || (uint64_t)slots3 * G.tile_elems * 8 <= avail);
+  const int64_t need_slots = wp->fused ? slots3 : slots2;
+  if (d.wave_slots < need_slots && (uint64_t)need_slots * G.tile_elems * 8 > avail) return false;
   const double r = d.r_sweep, Td = (double)T, n = (double)nz;
   wp->c = c;
   wp->B = B;
@@ -1288,7 +1298,8 @@ static bool wavefront_ok(const Domain& d, int T, WavePlan* wp) {
   // by its T sweeps per plane; one chunk of fill/drain
   // (the bootstrap's sweeps are thick, about 0.7 of a chunk sweep's cost per
   // plane, fitted on the Fig. 5 sweep at T = 64 and 100)
-  wp->est = (double)B + 0.7 * r * Td * Td + std::max(n, r * n * Td) + (double)c * (1.0 + r * Td);
+  const double rm = wp->fused ? 0.6 * r : r;  // two levels per pass: ~0.6 of the sweep time per level
+  wp->est = (double)B + 0.7 * r * Td * Td + std::max(n, rm * n * Td) + (double)c * (1.0 + rm * Td);
   return true;
 }
 
@@ -1329,13 +1340,23 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
   const Geometry& G = d.G;
   const int64_t nz = G.l[2], tz = G.t[2], lt = G.layer_tiles, c = wp.c, B = wp.B, nlo = wp.nlo;
   const int64_t U = nz / c, iB = (nz - B) / c;  // iterations; first chunk inside the bootstrap region
-  Status r = ensure_wave_scratch(d, 2 * nlo * lt);
+  // level buffers: two (level s in array bit ^ (s & 1)) or, with two levels
+  // per pass, three (s % 3: the arrays bit, bit ^ 1 and a third one in the
+  // wave scratch) — a fused pass writes level s+1 while its other CTAs still
+  // read level s-1, so the two may not share memory. Scratch parities for
+  // planes z < 0 likewise.
+  const int nbuf = wp.fused ? 3 : 2;
+  Status r = ensure_wave_scratch(d, wp.fused ? G.ntiles + 3 * nlo * lt : 2 * nlo * lt);
   if (r.bad()) return r;
   const Pipes P(S, false);
   const int cs = P.comp(0), os = P.out(0), is = P.in(0);
   const int bit = d.res_bit;
-  const int scr[2] = {d.nslots, d.nslots + (int)(nlo * lt)};
-  const int fin = bit ^ (T & 1);  // array holding level T (z >= 0)
+  const int arrA = bit ? (int)G.ntiles : 0, arrB = bit ? 0 : (int)G.ntiles;
+  const int sc0 = d.nslots + (wp.fused ? (int)G.ntiles : 0);
+  const int arr[3] = {arrA, arrB, d.nslots};
+  const int scr[3] = {sc0, sc0 + (int)(nlo * lt), sc0 + 2 * (int)(nlo * lt)};
+  const int ib = T % nbuf;                  // buffer holding level T
+  const int fin = ib == 1 ? bit ^ 1 : bit;  // resident array that ends up holding it
   auto arr0 = [&](int a, int64_t L) { return (int)((a ? G.ntiles : 0) + L * lt); };
   // planes [z0, z1) of the ring (physical, 0 <= z0 < z1 <= nz) in tile-layer pieces
   auto pieces = [&](int64_t z0, int64_t z1, auto&& f) -> Status {
@@ -1382,11 +1403,25 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
     if (r.bad()) return r;
   }
   auto lvl = [&](int s) {  // view of level s (s = 0: the initial data, wrapped)
+    const int k = s % nbuf;
     return s == 0 ? SlabRef{SlabRef::RESIDENT, bit, 0, {0, 0, 0}, 0, 0}
-                  : SlabRef{SlabRef::WAVE, bit ^ (s & 1), 0, {scr[s & 1], 0, 0}, 0, nlo};
+                  : SlabRef{SlabRef::WAVE, arr[k], 0, {scr[k], 0, 0}, 0, nlo};
   };
   auto level_of_iteration = [&](int64_t i, int s) {
     return X.slab_sweep(d, lvl(s - 1), lvl(s), (int)(c * i - s), (int)(c * i + c - s), cs);
+  };
+  // levels s, s+1 of iteration i in one pass
+  auto levels_of_iteration = [&](int64_t i, int s) {
+    return X.slab_sweep2(d, lvl(s - 1), lvl(s), lvl(s + 1), (int)(c * i - s), (int)(c * i + c - s), cs);
+  };
+  // the next pass of an iteration from level s: two levels when fused; returns the levels done
+  auto pass_of_iteration = [&](int64_t i, int s, int* done) {
+    if (wp.fused && s + 1 <= T) {
+      *done = 2;
+      return levels_of_iteration(i, s);
+    }
+    *done = 1;
+    return level_of_iteration(i, s);
   };
   // bootstrap rounds, with iteration 0's levels interleaved
   int s0 = 1;  // next level of iteration 0
@@ -1407,16 +1442,23 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
       r = X.wait(d, ev_in(d, 0), cs);
       if (r.bad()) return r;
     }
-    // iteration 0's levels whose seam strip is complete: level s needs level
-    // s-1 at -s-1, -s, i.e. (k+1)c >= 2(s-1) + 2 (level 0: region chunk 0)
-    for (; s0 <= T && (k + 1) * c >= 2 * (int64_t)s0; ++s0) {
-      r = level_of_iteration(0, s0);
+    // iteration 0's levels whose seam strips are complete: level s needs
+    // level s-1 at -s-1, -s, i.e. (k+1)c >= 2s (level 0: region chunk 0); a
+    // fused pass (s, s+1) also level s at -s-2, -s-1: (k+1)c >= 2(s+1)
+    while (s0 <= T) {
+      const int last = (wp.fused && s0 + 1 <= T) ? s0 + 1 : s0;
+      if ((k + 1) * c < 2 * (int64_t)last) break;
+      int done = 0;
+      r = pass_of_iteration(0, s0, &done);
       if (r.bad()) return r;
+      s0 += done;
     }
   }
-  for (; s0 <= T; ++s0) {
-    r = level_of_iteration(0, s0);
+  while (s0 <= T) {
+    int done = 0;
+    r = pass_of_iteration(0, s0, &done);
     if (r.bad()) return r;
+    s0 += done;
   }
   // the march
   for (int64_t i = 0; i < U; ++i) {
@@ -1425,9 +1467,11 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
         r = X.wait(d, ev_in(d, i), cs);
         if (r.bad()) return r;
       }
-      for (int s = 1; s <= T; ++s) {
-        r = level_of_iteration(i, s);
+      for (int s = 1; s <= T;) {
+        int done = 0;
+        r = pass_of_iteration(i, s, &done);
         if (r.bad()) return r;
+        s += done;
       }
     }
     r = X.record(d, ev_host(d, i), cs);
@@ -1440,23 +1484,30 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
     if (a < 0) {
       r = pieces(nz + a, nz + std::min<int64_t>(b, 0), [&](int64_t L, int64_t lz, int64_t np) {
         const int64_t Ls = L - (nz / tz - nlo);  // scratch layer of physical layer L
-        return X.d2h_planes(d, L * lt, lt, scr[T & 1] + (int)(Ls * lt), lz, np, os);
+        return X.d2h_planes(d, L * lt, lt, scr[ib] + (int)(Ls * lt), lz, np, os);
       });
       if (r.bad()) return r;
     }
     if (b > 0) {
       r = pieces(std::max<int64_t>(a, 0), b, [&](int64_t L, int64_t lz, int64_t np) {
-        return X.d2h_planes(d, L * lt, lt, arr0(fin, L), lz, np, os);
+        return X.d2h_planes(d, L * lt, lt, arr[ib] + (int)(L * lt), lz, np, os);
       });
       if (r.bad()) return r;
     }
   }
-  // leave the domain resident at level T: the ring's top T planes from the scratch
+  // leave the domain resident at level T: the ring's top T planes from the
+  // scratch (and, when level T is in the third array, the rest from it)
   r = pieces(nz - T, nz, [&](int64_t L, int64_t lz, int64_t np) {
     const int64_t Ls = L - (nz / tz - nlo);
-    return X.copy_planes(d, scr[T & 1] + (int)(Ls * lt), arr0(fin, L), lt, lz, np, cs);
+    return X.copy_planes(d, scr[ib] + (int)(Ls * lt), arr0(fin, L), lt, lz, np, cs);
   });
   if (r.bad()) return r;
+  if (ib == 2) {
+    r = pieces(0, nz - T, [&](int64_t L, int64_t lz, int64_t np) {
+      return X.copy_planes(d, arr[2] + (int)(L * lt), arr0(fin, L), lt, lz, np, cs);
+    });
+    if (r.bad()) return r;
+  }
   d.res_bit = fin;
   for (int64_t k = 0; k < G.ntiles; ++k) {
     d.tile_dirty[k] = 0;  // the host received u^T through the D2H above

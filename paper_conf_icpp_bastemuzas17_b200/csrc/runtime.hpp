@@ -92,7 +92,7 @@ struct Domain;
 //              sub-tiles at slots ring[0..2]; slab plane 0 at local z = zbase
 //              (wrapped), z in unit z / un.
 //   WAVE     - wavefront (runtime.cpp run_wavefront): the tile-blocked
-//              resident array `slot` (0/1) for planes z >= 0 (no wrap) and,
+//              array starting at slot `slot` for planes z >= 0 (no wrap) and,
 //              for z < 0, ring[0] = first slot of un tile layers of scratch
 //              holding planes [-un*tz, 0).
 struct SlabRef {
@@ -124,6 +124,11 @@ struct Exec {
   virtual Status slab_sweep(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi,
                             int stream) = 0;
   virtual Status copy_slots(Domain& d, int src_slot, int dst_slot, int64_t n, int stream) = 0;
+  // wavefront, two levels per pass (three level buffers): level s on planes
+  // [a, b) from src, only its top two planes written to mid (whose planes a-2,
+  // a-1 are read), level s+1 on [a-1, b-1) into dst
+  virtual Status slab_sweep2(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, int a, int b,
+                             int stream) = 0;
   // planes [p0, p0+np) of n tile slots: slots s0.. -> host tiles t0.. (the
   // same planes), and slots -> slots (wavefront)
   virtual Status d2h_planes(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int stream) = 0;

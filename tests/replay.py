@@ -108,6 +108,7 @@ class Replayer:
         # [0] lo (the lower rank's top planes), [1] hi (the upper rank's bottom
         # planes) and their counters: S (arrived epoch) and CR (credit: the
         # receiver on that side released the epoch's layer I pushed)
+        self.pending2 = {}  # stream -> parameters of a two-level sweep (TILE_OP_WSWEEP2)
         self.st = {0: None, 1: None}
         self.st_arrived = {0: 0, 1: 0}
         self.st_credit = {0: 0, 1: 0}
@@ -385,6 +386,27 @@ class Replayer:
             new = self.sweep(blk, None, 1, hi - lo + 1)
             for p in range(lo, hi):
                 self.wave_set(b, p, d, new[p - lo + 1])
+        elif name == "wsweep2":  # parameters of a two-level pass; executed at its _dst record
+            self.pending2[st] = (a, b, c, d)
+        elif name == "wsweep2_dst":
+            # level s on [lo, hi) from view src, written to view mid only at
+            # hi-2, hi-1 (mid's planes lo-2, lo-1 are read); level s+1 on
+            # [lo-1, hi-1) into view a
+            src, mid, cc, nlo = self.pending2.pop(st)
+            lo, hi = wsweep_range(cc)
+            rd = {self._wave_loc(src, p, nlo) for p in range(lo - 1, hi + 1)} | \
+                 {self._wave_loc(mid, p, nlo) for p in (lo - 2, lo - 1)}
+            wr = {self._wave_loc(a, p, nlo) for p in range(lo - 1, hi - 1)} | \
+                 {self._wave_loc(mid, p, nlo) for p in (hi - 2, hi - 1)}
+            assert not rd & wr, "two-level sweep writes memory it reads (in-kernel race)"
+            blk = np.stack([self.wave_get(src, p, nlo) for p in range(lo - 1, hi + 1)])
+            lev = self.sweep(blk, None, 1, hi - lo + 1)[1:hi - lo + 1]  # level s, planes lo..hi-1
+            blk2 = np.concatenate([np.stack([self.wave_get(mid, lo - 2, nlo), self.wave_get(mid, lo - 1, nlo)]), lev])
+            lev2 = self.sweep(blk2, None, 1, hi - lo + 1)[1:hi - lo + 1]  # level s+1, planes lo-1..hi-2
+            for p in (hi - 2, hi - 1):
+                self.wave_set(mid, p, nlo, lev[p - lo])
+            for p in range(lo - 1, hi - 1):
+                self.wave_set(a, p, nlo, lev2[p - lo + 1])
         elif name == "d2h_planes":
             p0, np_ = d & 0xffffffff, d >> 32
             for i in range(c):
@@ -445,16 +467,18 @@ class Replayer:
     def _wave_loc(self, code, p, nlo):
         """(first slot of the tile layer, plane in the tiles) of unwrapped
         plane p in a TILE_OP_WSWEEP view: bit 0 set and p < 0: the scratch
-        tile layers at slot code >> 2 (nlo of them, planes [-nlo*tz, 0));
-        otherwise resident array (code >> 1) & 1, wrapped only for bit 0 = 0."""
+        tile layers at slot code >> 32 (nlo of them, planes [-nlo*tz, 0));
+        bit 0 set, p >= 0: the array starting at slot (code >> 1) & 0x7fffffff;
+        bit 0 clear: resident array (code >> 1) & 1, wrapped."""
         G = self.G
         tz, lt, nz = G.t[2], G.n[0] * G.n[1], G.l[2]
         if code & 1 and p < 0:
             q = p + nlo * tz
             assert q >= 0, "wavefront read below its scratch"
-            return (code >> 2) + (q // tz) * lt, q % tz
+            return (code >> 32) + (q // tz) * lt, q % tz
         if code & 1:
             assert p < nz, "wavefront view read past the ring"
+            return ((code >> 1) & 0x7FFFFFFF) + (p // tz) * lt, p % tz
         gz = p % nz
         return ((code >> 1) & 1) * G.ntiles + (gz // tz) * lt, gz % tz
 

@@ -94,7 +94,7 @@ def _run_to_fault(d, u):
                                                ("sync:1", "resident", "tile_sync")])
 def test_cuda_error_poisons_domain_dry(monkeypatch, fault, sched, where):
     monkeypatch.setenv("TILES_FAULT", fault)
-    kw = {"sched": sched, "stream_through": -1}
+    kw = {"sched": sched, "stream_through": -1, "wavefront": -1}
     if sched == "stream":
         kw["device_budget_bytes"] = _budget_for(DIMS, TD, 4, sched="stream", stream_through=-1)
     d = T.Domain(DIMS, TD, dry_run=True, **kw)
@@ -154,7 +154,7 @@ def test_cuda_error_poisons_domain_gpu(monkeypatch, fault, sched, where):
     if not cuda_available():
         pytest.skip("no CUDA device")
     monkeypatch.setenv("TILES_FAULT", fault)
-    kw = {"sched": sched, "stream_through": -1, "device": 0}
+    kw = {"sched": sched, "stream_through": -1, "wavefront": -1, "device": 0}
     if sched == "stream":
         kw["device_budget_bytes"] = _budget_for(DIMS, TD, 4, sched="stream", stream_through=-1)
     d = T.Domain(DIMS, TD, **kw)

@@ -510,17 +510,21 @@ def test_wavefront_schedule_replays_to_oracle(dims, td, T, ns, runs_after):
     # the wavefront run on its own: ops, link bytes and swept cells
     d2 = T_run_dry(dims, td, T, ns, wavefront=1)
     ops = [op[0] for op in d2.trace()]
-    assert "wsweep" in ops and "d2h_planes" in ops and "sweep" not in ops
+    assert "d2h_planes" in ops and "sweep" not in ops
+    assert ("wsweep2" in ops) == (T >= 2)   # two levels per pass (three level buffers)
     st = d2.stats()
     cells = dims[0] * dims[1] * dims[2]
     assert st["bytes_h2d"] == cells * 8 and st["bytes_d2h"] == cells * 8
     assert d2.get_info()["last_schedule"] == 6
     planes = 0
     for op in d2.trace():
-        if op[0] == "wsweep":
+        if op[0] in ("wsweep", "wsweep2"):
             lo, hi = wsweep_range(op[4])
-            planes += hi - lo
+            planes += (hi - lo) * (2 if op[0] == "wsweep2" else 1)
     assert planes == dims[2] * T + sum(max(0, 2 * T - 2 * t) for t in range(1, T))
+    # one level per pass (two level buffers, wavefront = 2) replays exactly too
+    d3 = _run_and_replay(dims, td, [T], ns, seeds=(7,), wavefront=2)
+    assert "wsweep2" not in [op[0] for op in d3.trace()]
 
 
 def T_run_dry(dims, td, steps, ns, **kw):
@@ -556,10 +560,10 @@ def test_cost_model_ratio_option_and_report():
     d = T.Domain(dims, td, dry_run=True)
     assert abs(d.get_info()["sweep_link_ratio"] - 0.021) < 1e-12
     got = {}
-    for r in (0.005, 0.021, 0.2):
+    for r in (0.005, 0.021, 0.5):
         d = T.Domain(dims, td, dry_run=True, sweep_link_ratio=r)
         assert d.get_info()["sweep_link_ratio"] == r
         d.invalidate()
         d.run(T.heat7(ALPHA), 32, 4)
         got[r] = d.get_info()["last_schedule"]
-    assert got[0.005] in (2, 6) and got[0.021] == 6 and got[0.2] == 1
+    assert got[0.005] in (2, 6) and got[0.021] == 6 and got[0.5] == 1
