@@ -181,10 +181,12 @@ typedef struct {
                                    the periodic seam. -1 =
                                    never, 0 (default) = when the cost model
                                    prefers it to stream-through and the
-                                   batched schedule, 1 = whenever feasible
-                                   (two levels per pass through a third level
-                                   buffer when the budget holds it), 2 =
-                                   whenever feasible, one level per pass */
+                                   batched schedule, 1 = whenever feasible,
+                                   2 = whenever feasible, two levels per pass
+                                   through a third level buffer when the
+                                   budget holds it (one kernel per pass,
+                                   slab_sweep2_tile; measured slower than two
+                                   single-level passes on B200) */
   double sweep_link_ratio;      /* cost model of the fresh-upload schedules
                                    (DESIGN.md §5): time of one stencil sweep
                                    per plane over one plane's duplex host-link

@@ -530,7 +530,7 @@ static EncodeTiledFn encode_fn() {
 // shared memory; level s goes through a 3-plane shared ring for the other
 // threads' y neighbours and the x edges, one named barrier per plane.
 namespace w2 {
-constexpr int BY = 32, TX = 64, NT = 512, S = 4;
+constexpr int BY = 32, TX = 64, NT = 512, S = 6;
 constexpr int SROWS = BY + 4;                     // staged rows: y0-2 .. y0+BY+1
 constexpr int XH = SROWS * TX;                    // x halos: per side boxes at 128-byte boundaries
 constexpr int HS = 96;                            // doubles per side: rows 0-1 | 2..BY+1 | BY+2..BY+3
@@ -598,9 +598,20 @@ __global__ void __launch_bounds__(w2::NT + 32, 1)
       const int ya = y0 < 2 ? y0 - 2 + ny : y0 - 2;
       const int yb = y0 + BY + 2 > ny ? y0 + BY - ny : y0 + BY;
       const int nstg = (p1 + 1) - zc0 + 2;  // level s-1 planes zc0-1 .. p1+1
+      // in-plane offsets of the nine copies, per view (0: level s-1, 1: level s), once per run
+      int64_t off[2][9];
+#pragma unroll
+      for (int v = 0; v < 2; ++v) {
+        const ViewDev& V = v ? Mv : Sv;
+        const int64_t oa = V.Y(ya), o0 = V.Y(y0), ob = V.Y(yb), xc = V.X(x0), xL = V.X(xl), xR = V.X(xr);
+        off[v][0] = o0 + xc, off[v][1] = oa + xc, off[v][2] = ob + xc;
+        off[v][3] = oa + xL, off[v][4] = o0 + xL, off[v][5] = ob + xL;
+        off[v][6] = oa + xR, off[v][7] = o0 + xR, off[v][8] = ob + xR;
+      }
       for (int q = 0; q < nload + nstg; ++q, ++g) {
         const bool ld = q < nload;
         const ViewDev& V = ld ? Mv : Sv;
+        const int64_t* o = off[ld ? 1 : 0];
         const int z = ld ? p0 - 1 + q : zc0 - 1 + (q - nload);
         const int st = (int)(g % S);
         mbar_wait(&empty[st], ((g / S) & 1u) ^ 1u);
@@ -608,15 +619,14 @@ __global__ void __launch_bounds__(w2::NT + 32, 1)
         const double* pz = V.P(z);
         fence_proxy_async();
         mbar_expect_tx(&full[st], BYTES);
-        bulk_g2s(dst + 2 * TX, pz + V.Y(y0) + V.X(x0), (uint32_t)BY * TX * 8, &full[st]);
-        bulk_g2s(dst, pz + V.Y(ya) + V.X(x0), 2 * TX * 8, &full[st]);
-        bulk_g2s(dst + (BY + 2) * TX, pz + V.Y(yb) + V.X(x0), 2 * TX * 8, &full[st]);
-        const int yy[3] = {ya, y0, yb};
+        bulk_g2s(dst + 2 * TX, pz + o[0], (uint32_t)BY * TX * 8, &full[st]);
+        bulk_g2s(dst, pz + o[1], 2 * TX * 8, &full[st]);
+        bulk_g2s(dst + (BY + 2) * TX, pz + o[2], 2 * TX * 8, &full[st]);
         const int boff[3] = {0, 16, 80};
 #pragma unroll
         for (int h = 0; h < 3; ++h) {
-          const double* cl = pz + V.Y(yy[h]) + V.X(xl);
-          const double* cr = pz + V.Y(yy[h]) + V.X(xr);
+          const double* cl = pz + o[3 + h];
+          const double* cr = pz + o[6 + h];
           const int kl = (cl >= maps.base[1] && cl < maps.end[1]) ? 1 : 0;
           const int kr = (cr >= maps.base[1] && cr < maps.end[1]) ? 1 : 0;
           tma_2d(dst + XH + boff[h], h == 1 ? &maps.xmap[kl] : &maps.xmap2[kl], TX - 2,
@@ -635,8 +645,9 @@ __global__ void __launch_bounds__(w2::NT + 32, 1)
   // pairs: k = 0, 1 band rows warp, warp + 16 (stage row +2, mid row +1);
   // k = 2 (warps 0, 1): the extended rows y0-1 (mid row 0) / y0+BY (mid row 33)
   const bool ext = warp < 2;
-  const int srow[3] = {warp + 2, warp + 18, warp == 0 ? 1 : BY + 2};
-  const int mrow[3] = {warp + 1, warp + 17, warp == 0 ? 0 : BY + 1};
+  // stage / ring rows of pair k (band rows: stage r+2, ring r+1)
+  auto srow = [&](int k) { return k == 0 ? warp + 2 : k == 1 ? warp + 18 : (warp == 0 ? 1 : BY + 2); };
+  auto mrow = [&](int k) { return k == 0 ? warp + 1 : k == 1 ? warp + 17 : (warp == 0 ? 0 : BY + 1); };
   const bool edge = t >= 64 && t < 64 + 2 * MROWS;  // an extended-column cell x = -1 / 64
   const int eside = (t - 64) / MROWS, er = (t - 64) - eside * MROWS, ex = eside ? TX : -1;
   uint32_t seq = 0;
@@ -653,12 +664,9 @@ __global__ void __launch_bounds__(w2::NT + 32, 1)
     plan(p0, p1, zc0, nload);
     const int cx = (int)(col % ntx), y0 = (int)(col / ntx) * BY;
     const int base = p0 - 1;  // ring slot of level-s plane z: (z - base) % 3
-    int64_t od[2], om[2];
-#pragma unroll
-    for (int k = 0; k < 2; ++k) {
-      od[k] = Dv.Y(y0 + mrow[k] - 1) + Dv.X(cx * TX + x);
-      om[k] = Mv.Y(y0 + mrow[k] - 1) + Mv.X(cx * TX + x);
-    }
+    // output offsets of the two band pairs (rows warp, warp + 16: one tile row apart by 16)
+    const int64_t od0 = Dv.Y(y0 + warp) + Dv.X(cx * TX + x), odd = Dv.Y(y0 + warp + 16) - Dv.Y(y0 + warp);
+    const int64_t om0 = Mv.Y(y0 + warp) + Mv.X(cx * TX + x), omd = Mv.Y(y0 + warp + 16) - Mv.Y(y0 + warp);
     // level s of the own band pairs at planes z-2, z-1 (l2, l1): filled by the
     // loaded planes or by the first computed ones
     double2 l1[2], l2[2];
@@ -673,23 +681,23 @@ __global__ void __launch_bounds__(w2::NT + 32, 1)
 #pragma unroll
       for (int k = 0; k < 2; ++k) {
         l2[k] = l1[k];
-        l1[k] = *reinterpret_cast<const double2*>(st + srow[k] * TX + x);
+        l1[k] = *reinterpret_cast<const double2*>(st + srow(k) * TX + x);
       }
       release_g(seq + q);
     }
     const uint32_t s0 = seq + nload;  // stage of level s-1 plane zc0-1
-    // level s-1 of the own pairs at planes z-1, z (register march)
-    double2 cm[3], cc[3];
+    // level s-1 of the own band pairs at planes z-1, z (register march; the
+    // extended rows of warps 0/1 read theirs from the stages)
+    double2 cm[2], cc[2];
     wait_g(s0);
     wait_g(s0 + 1);
     {
       const double* a0 = stage + (size_t)(s0 % S) * STAGE;
       const double* a1 = stage + (size_t)((s0 + 1) % S) * STAGE;
 #pragma unroll
-      for (int k = 0; k < 3; ++k) {
-        if (k == 2 && !ext) break;
-        cm[k] = *reinterpret_cast<const double2*>(a0 + srow[k] * TX + x);
-        cc[k] = *reinterpret_cast<const double2*>(a1 + srow[k] * TX + x);
+      for (int k = 0; k < 2; ++k) {
+        cm[k] = *reinterpret_cast<const double2*>(a0 + srow(k) * TX + x);
+        cc[k] = *reinterpret_cast<const double2*>(a1 + srow(k) * TX + x);
       }
     }
     for (int z = zc0; z <= p1; ++z) {
@@ -702,11 +710,13 @@ __global__ void __launch_bounds__(w2::NT + 32, 1)
       double* mo = top ? Mv.P(z) : nullptr;
       double2 lv[2];
       // level s at z, own pairs
+      const double* sm1 = stage + (size_t)((gz - 1) % S) * STAGE;
 #pragma unroll
       for (int k = 0; k < 3; ++k) {
         if (k == 2 && !ext) break;
-        const int sr = srow[k];
-        const double2 c = cc[k];
+        const int sr = srow(k);
+        const double2 c = k < 2 ? cc[k] : *reinterpret_cast<const double2*>(s00 + sr * TX + x);
+        const double2 zmv = k < 2 ? cm[k] : *reinterpret_cast<const double2*>(sm1 + sr * TX + x);
         const double2 zp = *reinterpret_cast<const double2*>(sp1 + sr * TX + x);
         const double2 ym = *reinterpret_cast<const double2*>(s00 + (sr - 1) * TX + x);
         const double2 yp = *reinterpret_cast<const double2*>(s00 + (sr + 1) * TX + x);
@@ -715,18 +725,17 @@ __global__ void __launch_bounds__(w2::NT + 32, 1)
         if (lane == 0) xm = s00[XH + hoff(0, sr) + 1];
         if (lane == 31) xp = s00[XH + hoff(1, sr)];
         double2 v;
-        v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, cm[k].x, zp.x, alpha);
-        v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, cm[k].y, zp.y, alpha);
-        *reinterpret_cast<double2*>(m + mrow[k] * MW + x + 2) = v;
+        v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zmv.x, zp.x, alpha);
+        v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zmv.y, zp.y, alpha);
+        *reinterpret_cast<double2*>(m + mrow(k) * MW + x + 2) = v;
         if (k < 2) {
           lv[k] = v;
-          if (top) *reinterpret_cast<double2*>(mo + om[k]) = v;
+          if (top) *reinterpret_cast<double2*>(mo + om0 + k * omd) = v;
+          cm[k] = c;
+          cc[k] = zp;
         }
-        cm[k] = c;
-        cc[k] = zp;
       }
       if (edge) {  // the extended columns x = -1 / 64 (stage z-1 still held: released below)
-        const double* sm1 = stage + (size_t)((gz - 1) % S) * STAGE;
         const int sr = er + 1;
         const double c = sv(s00, sr, ex);
         m[er * MW + ex + 2] = heat_update(c, sv(s00, sr, ex - 1), sv(s00, sr, ex + 1), sv(s00, sr - 1, ex),
@@ -740,7 +749,7 @@ __global__ void __launch_bounds__(w2::NT + 32, 1)
         double* dw = Dv.P(w);
 #pragma unroll
         for (int k = 0; k < 2; ++k) {
-          const double* p = mw + mrow[k] * MW + x + 2;
+          const double* p = mw + mrow(k) * MW + x + 2;
           const double2 c = l1[k];
           const double2 ym = *reinterpret_cast<const double2*>(p - MW);
           const double2 yp = *reinterpret_cast<const double2*>(p + MW);
@@ -751,7 +760,7 @@ __global__ void __launch_bounds__(w2::NT + 32, 1)
           double2 v;
           v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, l2[k].x, lv[k].x, alpha);
           v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, l2[k].y, lv[k].y, alpha);
-          stg2_stream(dw + od[k], v);
+          stg2_stream(dw + od0 + k * odd, v);
         }
       }
 #pragma unroll

@@ -1277,15 +1277,11 @@ static bool wavefront_ok(const Domain& d, int T, WavePlan* wp) {
   const int64_t B = (2 * (int64_t)T + c - 1) / c * c;
   if (B + c > nz) return false;  // the seam's cone would cover the ring
   const int64_t nlo = (2 * (int64_t)T + tz - 1) / tz;
-  // two levels per pass (TILES_WAVE_FUSE, default on) take a third level
-  // array (ntiles slots) and three scratch parities, when the budget has them
-  static const int fuse = [] {
-    const char* e = getenv("TILES_WAVE_FUSE");
-    return e ? atoi(e) : 1;
-  }();
+  // two levels per pass (wavefront = 2) take a third level array (ntiles
+  // slots) and three scratch parities, when the budget has them
   const uint64_t avail = d.budget_left + (uint64_t)d.wave_slots * G.tile_elems * 8;
   const int64_t slots3 = G.ntiles + 3 * nlo * G.layer_tiles, slots2 = 2 * nlo * G.layer_tiles;
-  wp->fused = fuse && d.opt.wavefront != 2 && T >= 2 &&
+  wp->fused = d.opt.wavefront == 2 && T >= 2 &&
               (d.wave_slots >= slots3 || (uint64_t)slots3 * G.tile_elems * 8 <= avail);
   const int64_t need_slots = wp->fused ? slots3 : slots2;
   if (d.wave_slots < need_slots && (uint64_t)need_slots * G.tile_elems * 8 > avail) return false;

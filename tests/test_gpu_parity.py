@@ -409,16 +409,18 @@ def test_stream_through_bit_exact(dims, td, T):
 @pytest.mark.parametrize("dims,td,T", [((64, 32, 128), (32, 16, 16), 20), ((128, 64, 256), (64, 64, 32), 48),
                                        ((64, 64, 64), (32, 32, 8), 7), ((96, 64, 160), (32, 32, 32), 1),
                                        ((64, 32, 512), (32, 32, 64), 100), ((512, 64, 128), (64, 64, 64), 16)])
-def test_wavefront_bit_exact(dims, td, T):
+@pytest.mark.parametrize("wave", [1, 2])
+def test_wavefront_bit_exact(dims, td, T, wave):
     """Fresh-upload runs on the time-skewed wavefront (forced): chunks of
     planes, level s of chunk i on planes [c*i - s, c*i + c - s), the seam's
     bootstrap trapezoid in the scratch layers, each chunk's final planes
     back to the host as soon as it ends; the host result, the kept device
     copy (a following resident run) and a second wavefront run are exact,
-    and every cell crossed the link once per direction."""
+    and every cell crossed the link once per direction. wave = 1: one level
+    per pass (slab_sweep_tile); 2: two levels per pass (slab_sweep2_tile)."""
     nx, ny, nz = dims
     u0 = synth.uniform_grid(nx, ny, nz, 42)
-    with T_.Domain(dims, td, wavefront=1) as d:
+    with T_.Domain(dims, td, wavefront=wave) as d:
         d.load(u0)
         d.run(T_.heat7(), T, 2)
         out1 = d.store()

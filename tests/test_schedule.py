@@ -511,7 +511,7 @@ def test_wavefront_schedule_replays_to_oracle(dims, td, T, ns, runs_after):
     d2 = T_run_dry(dims, td, T, ns, wavefront=1)
     ops = [op[0] for op in d2.trace()]
     assert "d2h_planes" in ops and "sweep" not in ops
-    assert ("wsweep2" in ops) == (T >= 2)   # two levels per pass (three level buffers)
+    assert "wsweep2" not in ops   # one level per pass (two level buffers)
     st = d2.stats()
     cells = dims[0] * dims[1] * dims[2]
     assert st["bytes_h2d"] == cells * 8 and st["bytes_d2h"] == cells * 8
@@ -522,9 +522,18 @@ def test_wavefront_schedule_replays_to_oracle(dims, td, T, ns, runs_after):
             lo, hi = wsweep_range(op[4])
             planes += (hi - lo) * (2 if op[0] == "wsweep2" else 1)
     assert planes == dims[2] * T + sum(max(0, 2 * T - 2 * t) for t in range(1, T))
-    # one level per pass (two level buffers, wavefront = 2) replays exactly too
-    d3 = _run_and_replay(dims, td, [T], ns, seeds=(7,), wavefront=2)
-    assert "wsweep2" not in [op[0] for op in d3.trace()]
+    # two levels per pass (three level buffers, wavefront = 2) replays exactly
+    # too, in random and adversarial orders, with the same swept planes
+    d3 = _run_and_replay(dims, td, [T], ns, seeds=(7, 8), wavefront=2)
+    _run_and_replay(dims, td, [T], ns, seeds=(9,), wavefront=2, lazy=("wsweep",))
+    ops3 = [op[0] for op in d3.trace()]
+    assert ("wsweep2" in ops3) == (T >= 2)
+    planes3 = 0
+    for op in d3.trace():
+        if op[0] in ("wsweep", "wsweep2"):
+            lo, hi = wsweep_range(op[4])
+            planes3 += (hi - lo) * (2 if op[0] == "wsweep2" else 1)
+    assert planes3 == planes
 
 
 def T_run_dry(dims, td, steps, ns, **kw):
