@@ -1093,7 +1093,7 @@ def run_main_leg(args):
     h2d_b = st["bytes_h2d"] // args.steps
     d2h_b = st["bytes_d2h"] // args.steps
     peak, peak_src = measured_peaks()
-    # the step's kernels with per-launch CUDA events: the same schedule with
+    # the step's kernels with CUDA events: the same schedule with
     # the copies skipped (TILE_MEASURE_COMP_ONLY), so the launches run back to
     # back and each event pair brackets its kernel (timed inside the e2e leg,
     # the events would also bracket the host's enqueue gaps while the stream
@@ -1114,9 +1114,10 @@ def run_main_leg(args):
             "kernel_ms_per_step": sw_ms / args.steps,
             "kernel_share_of_step": sw_ms / ms if ms > 0 else None,
             "note": "achieved = 16 B x cells swept by the step's sweep launches / their summed CUDA-event "
-                    "durations on the launching stream, measured on the same schedule with the copies "
-                    "skipped (comp-only) so that launches run back to back; the e2e step itself is "
-                    "host-link-bound: see roofline_link",
+                    "durations on the launching stream (one event pair per run of consecutive sweeps on a "
+                    "stream, so programmatic dependent launch keeps overlapping them), measured on the same "
+                    "schedule with the copies skipped (comp-only) so that launches run back to back; the "
+                    "e2e step itself is host-link-bound: see roofline_link",
             "peak_source": peak_src}
 
     # ---- the kernel-level rate: grid resident in HBM ------------------------

@@ -405,9 +405,11 @@ tile_status tile_set_measure(tile_domain* dom, int32_t mode);
  * its first stream and records a timing event there; tile_timer_stop joins
  * again, records a second event, synchronizes and returns the elapsed device
  * milliseconds in *ms. With tile_set_kernel_timing(dom, 1) every kernel
- * launch is bracketed by events on its own stream and the summed durations
- * are reported in tile_stats.kernel_ms / kernel_timed after tile_sync or
- * tile_timer_stop. */
+ * launch is bracketed by events on its own stream — a run of consecutive
+ * stencil sweeps on one stream by one pair around the run, so programmatic
+ * dependent launch still overlaps them — and the summed durations are
+ * reported in tile_stats.kernel_ms / kernel_timed (launches) after tile_sync
+ * or tile_timer_stop. */
 tile_status tile_timer_start(tile_domain* dom);
 tile_status tile_timer_stop(tile_domain* dom, double* ms);
 tile_status tile_set_kernel_timing(tile_domain* dom, int32_t on);

@@ -33,10 +33,19 @@ struct CudaExec final : Exec {
   std::vector<cudaEvent_t> tpool;                 // timing events (free list)
   struct Timed {
     cudaEvent_t a, b;
-    uint64_t cells;  // cells read + written once by the launch (stencil sweeps), else 0
+    uint64_t cells;  // cells read + written once by the launches (stencil sweeps), else 0
+    uint32_t n;      // launches inside [a, b]
   };
   std::vector<Timed> tpending;
-  uint64_t next_cells = 0;  // cells of the next timed launch (set just before it)
+  // a run of consecutive sweep launches on one stream shares one event pair:
+  // an event between two launches would end programmatic dependent launch
+  // (the next sweep's ramp overlapping the previous one's drain), so a
+  // per-launch pair times each sweep alone. The interval is closed (its end
+  // event recorded) by the next other operation on that stream (S() below),
+  // a join or a synchronize.
+  std::vector<int> open_iv;  // per stream: index into tpending, or -1
+  bool in_launch = false;    // S() inside a timed launch does not close
+  uint64_t next_cells = 0;   // cells of the next timed launch (set just before it)
   cudaEvent_t t_begin = nullptr, t_end = nullptr;
   cudaEvent_t local_ready = nullptr;  // in-process transport
 
@@ -49,65 +58,86 @@ struct CudaExec final : Exec {
     CK(cudaEventCreate(e));
     return Status::ok();
   }
-  // bracket a kernel launch with timing events on its stream
+  Status close_iv(int st) {
+    if (open_iv.size() <= (size_t)st || open_iv[(size_t)st] < 0) return Status::ok();
+    Timed& t = tpending[(size_t)open_iv[(size_t)st]];
+    open_iv[(size_t)st] = -1;
+    Status r = timing_event(&t.b);
+    if (r.bad()) return r;
+    CK(cudaEventRecord(t.b, streams[(size_t)st]));
+    return Status::ok();
+  }
+  Status close_all() {
+    for (size_t i = 0; i < open_iv.size(); ++i) {
+      Status r = close_iv((int)i);
+      if (r.bad()) return r;
+    }
+    return Status::ok();
+  }
+  // bracket a kernel launch with timing events on its stream (a sweep joins
+  // the stream's open interval)
   template <class F>
   Status timed(Domain& d, int st, F&& launch) {
-    if (!d.kernel_timing) {
+    return timed_status(d, st, [&]() -> Status {
       CK(launch());
       return Status::ok();
-    }
-    cudaEvent_t a, b;
-    Status r = timing_event(&a);
-    if (r.bad()) return r;
-    r = timing_event(&b);
-    if (r.bad()) return r;
-    CK(cudaEventRecord(a, S(st)));
-    CK(launch());
-    CK(cudaEventRecord(b, S(st)));
-    tpending.push_back({a, b, next_cells});
-    next_cells = 0;
-    return Status::ok();
+    });
   }
   // the same for a launch that reports a library Status (user kernels: the
   // real cause — ENOSYS, module load, launch — reaches the caller unchanged)
   template <class F>
   Status timed_status(Domain& d, int st, F&& launch) {
-    if (!d.kernel_timing) return launch();
-    cudaEvent_t a, b;
-    Status r = timing_event(&a);
-    if (r.bad()) return r;
-    r = timing_event(&b);
-    if (r.bad()) return r;
-    CK(cudaEventRecord(a, S(st)));
-    r = launch();
-    if (r.bad()) {
-      tpool.push_back(a);
-      tpool.push_back(b);
+    const uint64_t cells = next_cells;
+    next_cells = 0;
+    if (!d.kernel_timing) {
+      Status r = close_iv(st);
+      if (r.bad()) return r;
+      in_launch = true;
+      r = launch();
+      in_launch = false;
       return r;
     }
-    CK(cudaEventRecord(b, S(st)));
-    tpending.push_back({a, b, next_cells});
-    next_cells = 0;
+    if (open_iv.size() < streams.size()) open_iv.resize(streams.size(), -1);
+    if (!cells || open_iv[(size_t)st] < 0) {
+      Status r = close_iv(st);
+      if (r.bad()) return r;
+      cudaEvent_t a;
+      r = timing_event(&a);
+      if (r.bad()) return r;
+      CK(cudaEventRecord(a, streams[(size_t)st]));
+      tpending.push_back({a, nullptr, 0, 0});
+      open_iv[(size_t)st] = (int)tpending.size() - 1;
+    }
+    in_launch = true;
+    Status r = launch();
+    in_launch = false;
+    if (r.bad()) return r;  // the open interval is closed by the sync that reports it
+    Timed& t = tpending[(size_t)open_iv[(size_t)st]];
+    t.cells += cells;
+    t.n++;
+    if (!cells) return close_iv(st);
     return Status::ok();
   }
   Status collect(Domain& d) {  // after a synchronize
     for (auto& pr : tpending) {
       float ms = 0;
-      CK(cudaEventElapsedTime(&ms, pr.a, pr.b));
+      if (pr.b) CK(cudaEventElapsedTime(&ms, pr.a, pr.b));
       d.stats.kernel_ms += ms;
-      d.stats.kernel_timed++;
+      d.stats.kernel_timed += pr.n;
       if (pr.cells) {
         d.stats.sweep_ms += ms;
         d.stats.sweep_cells += pr.cells;
-        d.stats.sweep_timed++;
+        d.stats.sweep_timed += pr.n;
       }
       tpool.push_back(pr.a);
-      tpool.push_back(pr.b);
+      if (pr.b) tpool.push_back(pr.b);
     }
     tpending.clear();
     return Status::ok();
   }
   Status join_into0(Domain& d) {
+    Status r0 = close_all();
+    if (r0.bad()) return r0;
     for (size_t i = 1; i < streams.size(); ++i) {
       CK(cudaEventRecord(events[(size_t)(d.ev_misc_base + 4 + i)], streams[i]));
       CK(cudaStreamWaitEvent(streams[0], events[(size_t)(d.ev_misc_base + 4 + i)], 0));
@@ -137,7 +167,12 @@ struct CudaExec final : Exec {
     return Status::ok();
   }
 
-  cudaStream_t S(int i) { return streams[(size_t)i]; }
+  // the stream of an operation; any operation but a timed sweep ends the
+  // stream's open timing interval first
+  cudaStream_t S(int i) {
+    if (!in_launch && (size_t)i < open_iv.size() && open_iv[(size_t)i] >= 0) (void)close_iv(i);
+    return streams[(size_t)i];
+  }
 
   // TILES_FAULT: the n-th operation of a kind fails with a real CUDA error
   // (an invalid copy queued on the same stream), reported through CK.
@@ -674,6 +709,8 @@ struct CudaExec final : Exec {
   Status note(Domain&, int, int64_t, int64_t, int) override { return Status::ok(); }
   Status sync_all(Domain& d) override {
     INJECT(FAULT_SYNC, 0);
+    Status r = close_all();
+    if (r.bad()) return r;
     for (auto s : streams) CK(cudaStreamSynchronize(s));
     return collect(d);
   }
