@@ -86,6 +86,9 @@ def main():
     xfer = union(h2d + d2h)
     summ["transfer_busy_us"] = busy(xfer)
     summ["transfer_hidden_under_kernels"] = inter(xfer, K) / max(1e-9, busy(xfer))
+    t0 = min(x[0] for x in ker + h2d + d2h)
+    rel = lambda L: [[round(a - t0, 1), round(b - t0, 1)] for a, b in sorted(L)]
+    json.dump({"h2d": rel(h2d), "d2h": rel(d2h), "kernels": rel(ker)}, open(prefix + ".intervals.json", "w"))
     json.dump(summ, open(prefix + ".summary.json", "w"), indent=1)
     print(json.dumps(summ))
 
