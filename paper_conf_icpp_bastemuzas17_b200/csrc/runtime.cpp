@@ -923,40 +923,80 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
   auto res_of = [&](int64_t u) { return u == 0 ? keep0 : out[u & 1]; };
   auto ev_unit_done = [&](int64_t u) { return ev_host(d, u); };  // compute of unit u
   const int ring_ev[2] = {d.ev_misc_base + 4 + d.halo_stream + 1, d.ev_misc_base + 5 + d.halo_stream + 1};
-  const int cs = P.comp(0), os = P.out(0), is = P.in(0);
+  const int cs = P.comp(0), os = P.out(0);
   const bool multi = G.nranks > 1;  // z-slab ranks: halo layers replace the periodic wrap
   const int hs = d.halo_stream;
   const int ev_push = d.ev_misc_base + 6 + d.halo_stream + 1;
   if (multi) ++d.st_epoch;
   Status r;
   // one copy-in stream, so the copy engine runs the H2Ds in this order (it
-  // may not across streams): the last unit first (unit 0's wrap neighbour)
-  std::vector<int64_t> order;
-  order.push_back(U - 1);
-  for (int64_t u = 0; u < U - 1; ++u) order.push_back(u);
-  // Past the fill, consecutive regular units of one layer share one H2D copy
-  // (up to TILES_ST_H2D_MERGE of them): with D2H running, each copy costs a
-  // ~40 us gap on the H2D side (profiles/r01/pcie_gap.json), and H2D is the
-  // bottleneck of the steady state. The thin end units stay separate.
+  // may not across streams): the last unit first (unit 0's wrap neighbour),
+  // then the planes below it in z order. Past the fill, the copies are cut
+  // after every `merge` units (TILES_ST_H2D_MERGE): with D2H running, each
+  // copy costs a ~40 us gap on the H2D side (profiles/r01/pcie_gap.json), and
+  // H2D is the bottleneck of the steady state. With offset cuts
+  // (TILES_ST_OFFSET=1; default 0) a copy ending after unit v also carries
+  // the first T planes of unit v+1 (same tile layer), the top of unit v's
+  // halo, so unit v's sweeps and D2H can start when that copy lands; with
+  // 16-plane units in 64-plane layers this only moves one unit per layer and
+  // lengthens that copy (C2: no gain measured). The thin end
+  // units stay separate.
+  static const int offset = [] {
+    const char* e = getenv("TILES_ST_OFFSET");
+    return e ? atoi(e) : 0;
+  }();
   const int merge = st_h2d_merge();
-  for (size_t i = 0; i < order.size();) {
-    const int64_t u = order[i];
-    size_t j = i + 1;
-    int64_t np = np_of(u);
-    if (i >= 3 && np == sp.unit)
-      while (j < order.size() && (int)(j - i) < merge && order[j] == order[j - 1] + 1 &&
-             layer_of(order[j]) == layer_of(u) && np_of(order[j]) == sp.unit)
-        np += np_of(order[j++]);
-    r = X.h2d_part(d, layer_of(u) * lt, lt, cur_slot(u), p0_of(u), np, is);
-    if (r.bad()) return r;
-    for (; i < j; ++i) {
-      r = X.record(d, ev_in(d, order[i]), is);
-      if (r.bad()) return r;
+  const int64_t nzl = G.l[2];
+  struct Copy {
+    int64_t layer, p0, np;
+  };
+  std::vector<Copy> cps;
+  std::vector<int> cp_of((size_t)nzl, 0);  // plane -> index of the copy that uploads it
+  auto plan_copies = [&](bool off) {
+    cps.clear();
+    auto add = [&](int64_t zlo, int64_t zhi) {  // planes [zlo, zhi), one copy per tile layer
+      while (zlo < zhi) {
+        const int64_t L = zlo / tz, e = std::min(zhi, (L + 1) * tz);
+        for (int64_t z = zlo; z < e; ++z) cp_of[(size_t)z] = (int)cps.size();
+        cps.push_back({L, zlo - L * tz, e - zlo});
+        zlo = e;
+      }
+    };
+    const int64_t zend = z0_of(U - 1);
+    add(zend, zend + np_of(U - 1));
+    int64_t f = 0;
+    int since = 0;
+    for (int64_t v = 0; v + 1 < U; ++v) {
+      ++since;
+      const bool last = v + 2 >= U;
+      const bool regular = np_of(v) == sp.unit && !last && np_of(v + 1) == sp.unit && layer_of(v + 1) == layer_of(v);
+      if (!(v < 2 || !regular || since >= merge)) continue;
+      int64_t e = last ? zend : z0_of(v + 1);
+      if (off && !last && layer_of(v + 1) == layer_of(v)) e = std::min(zend, e + T);
+      if (e > f) add(f, e);
+      f = std::max(f, e);
+      since = 0;
     }
+  };
+  plan_copies(offset != 0);
+  if ((int64_t)cps.size() > G.ntiles) plan_copies(false);  // one ev_in event per copy
+  for (size_t k = 0; k < cps.size(); ++k) {
+    const Copy& c = cps[k];
+    const int is = P.in(0);
+    r = X.h2d_part(d, c.layer * lt, lt, bit ? (int)(G.ntiles + c.layer * lt) : (int)(c.layer * lt), c.p0, c.np, is);
+    if (r.bad()) return r;
+    r = X.record(d, ev_in(d, (int64_t)k), is);
+    if (r.bad()) return r;
   }
+  // the copy a set of planes waits for: the latest one (one stream, in order)
+  auto need = [&](int64_t zlo, int64_t zhi) {
+    int k = 0;
+    for (int64_t z = zlo; z < zhi; ++z) k = std::max(k, cp_of[(size_t)(((z % nzl) + nzl) % nzl)]);
+    return (int64_t)k;
+  };
   if (multi) {  // my slab-end planes of initial data to the neighbours, on the halo stream
     for (int side : {1, 0}) {
-      r = X.wait(d, ev_in(d, side ? U - 1 : 0), hs);
+      r = X.wait(d, ev_in(d, side ? need(nzl - T, nzl) : need(0, T)), hs);
       if (r.bad()) return r;
       r = X.st_halo(d, 0, side, T, hs);
       if (r.bad()) return r;
@@ -965,10 +1005,8 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
     if (r.bad()) return r;
   }
   for (int64_t u = 0; u < U; ++u) {
-    for (int64_t du : {(int64_t)-1, (int64_t)0, (int64_t)1}) {
-      r = X.wait(d, ev_in(d, (u + du + U) % U), cs);
-      if (r.bad()) return r;
-    }
+    r = X.wait(d, ev_in(d, need(z0_of(u) - T, z0_of(u) + np_of(u) + T)), cs);
+    if (r.bad()) return r;
     if (u >= 2) {  // the ring buffer u%2 was last read by unit u-2's D2H
       r = X.wait(d, ring_ev[u & 1], cs);
       if (r.bad()) return r;

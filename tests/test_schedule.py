@@ -11,6 +11,7 @@
 import os
 import re
 import subprocess
+import sys
 
 import numpy as np
 import pytest
@@ -329,6 +330,19 @@ def test_stream_through_schedule_replays_to_oracle(dims, td, T, ns):
     assert d.get_info()["resident"]
     # then a resident continuation and a second stream-through
     _run_and_replay(dims, td, [T, T], ns, seeds=(3,), wavefront=-1)
+
+
+@pytest.mark.parametrize("env", ["TILES_ST_OFFSET=1", "TILES_ST_H2D_MERGE=3", "TILES_ST_THIN=0"])
+def test_stream_through_copy_plans_replay_to_oracle(env):
+    """The stream-through's other H2D copy plans (copies cut T planes into the
+    next unit; three units per copy; uniform units): the replays above in a
+    fresh process with the knob set (the library reads it once)."""
+    k, v = env.split("=")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-p", "no:cacheprovider", "-x",
+                        "tests/test_schedule.py::test_stream_through_schedule_replays_to_oracle"],
+                       cwd=root, env={**os.environ, k: v}, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
 
 
 @pytest.mark.parametrize("dims,td,nslots,runs,ns", [
