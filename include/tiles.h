@@ -168,7 +168,10 @@ typedef struct {
                                    steps per pass in the streaming schedule
                                    (halves host-link bytes per step), single
                                    steps when resident; 1 = two steps in every
-                                   schedule; -1 = never */
+                                   schedule; -1 = never. Any ghost: resident
+                                   periodic single-rank domains 512 cells wide
+                                   with 64-wide tiles run two steps per kernel
+                                   (heat2_band) unless -1 */
   int32_t wavefront;            /* HEAT7 run starting from a fresh upload
                                    (periodic, single rank, resident, 2T planes
                                    of scratch fit): time-skewed march over
@@ -234,7 +237,9 @@ typedef struct {
                              whole-domain steps), 2 stream-through (fresh
                              upload), 3 out-of-core per-tile stream, 4
                              out-of-core stream-through, 5 synchronous (one
-                             stream), 6 wavefront (fresh upload) */
+                             stream), 6 wavefront (fresh upload), 7 resident,
+                             two steps per kernel (heat2_band: periodic,
+                             single rank, 512 cells wide, 64-wide tiles) */
   double sweep_link_ratio; /* the cost model's ratio in use (see tile_options) */
 } tile_info;
 
@@ -301,7 +306,10 @@ typedef enum {
                             [lo, hi) (c = lo | hi << 32, signed halves) from view a, written to
                             view b only at planes hi-2, hi-1 (its planes lo-2, lo-1 are read
                             from b); d = scratch layers. Views coded as for TILE_OP_WSWEEP */
-  TILE_OP_WSWEEP2_DST = 30/* the same kernel: level s+1 on [lo-1, hi-1) into view a */
+  TILE_OP_WSWEEP2_DST = 30,/* the same kernel: level s+1 on [lo-1, hi-1) into view a */
+  TILE_OP_BAND2 = 31     /* two steps of the whole resident periodic grid in one kernel
+                            (heat2_band): view a (the resident array, coded as for
+                            TILE_OP_WSWEEP) -> view b; c = 0 | nz << 32 */
 } tile_op_kind;
 
 typedef struct {

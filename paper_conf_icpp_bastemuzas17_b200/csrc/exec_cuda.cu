@@ -453,6 +453,35 @@ struct CudaExec final : Exec {
     d.stats.n_kernels++;
     return Status::ok();
   }
+  Band2Maps bmaps[2];
+  int bmaps_state = 0;  // 0 not tried, 1 encoded, -1 not available
+  bool band2_ok(Domain& d) override {
+    if (bmaps_state == 0) {
+      const Geometry& G = d.G;
+      bmaps_state = -1;
+      if (d.nslots >= 2 * G.ntiles &&
+          band2_maps_encode(&bmaps[0], d.slot_ptr(0), (int)G.t[0], (int)G.t[1], (int)G.t[2], (int)G.n[0],
+                            (int)G.n[1], (int)G.n[2]) &&
+          band2_maps_encode(&bmaps[1], d.slot_ptr((int)G.ntiles), (int)G.t[0], (int)G.t[1], (int)G.t[2],
+                            (int)G.n[0], (int)G.n[1], (int)G.n[2]))
+        bmaps_state = 1;
+    }
+    return bmaps_state == 1;
+  }
+  Status band2(Domain& d, int sbit, int dbit, int st) override {
+    INJECT(FAULT_KERNEL, st);
+    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
+    if (!band2_ok(d)) return make_err(TILE_ESTATE, "internal: heat2_band without its tensor maps");
+    const Geometry& G = d.G;
+    next_cells = d.kernel_timing ? (uint64_t)(G.l[0] * G.l[1] * G.l[2]) : 0;  // one pass over the cells
+    Status r = timed(d, st, [&] {
+      return launch_heat2_band(bmaps[sbit], d.slot_ptr(dbit ? (int)G.ntiles : 0), (int)G.t[1], (int)G.t[2],
+                               (int)G.n[1], (int)G.n[2], d.kernel_alpha, S(st));
+    });
+    if (r.bad()) return r;
+    d.stats.n_kernels++;
+    return Status::ok();
+  }
   Status slab_sweep2(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, int a, int b,
                      int st) override {
     INJECT(FAULT_KERNEL, st);

@@ -120,6 +120,13 @@ struct DryExec final : Exec {
         src.kind == SlabRef::RESIDENT ? src.zbase : 0);
     return Status::ok();
   }
+  bool band2_ok(Domain&) override { return true; }
+  Status band2(Domain& d, int sbit, int dbit, int st) override {
+    if (Status f_ = inject(d, FAULT_KERNEL); f_.bad()) return f_;
+    d.stats.n_kernels++;
+    put(d, TILE_OP_BAND2, st, (int64_t)sbit << 1, (int64_t)dbit << 1, d.G.l[2] << 32, 0);
+    return Status::ok();
+  }
   Status slab_sweep2(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, int a, int b,
                      int st) override {
     if (Status f_ = inject(d, FAULT_KERNEL); f_.bad()) return f_;

@@ -205,6 +205,18 @@ int sweep_tile_band();  // box rows (band) of the tile-column sweep kernel
 // cudaErrorNotSupported when the shapes do not fit.
 cudaError_t launch_slab_sweep2(const SlabView& src, const SlabView& mid, const SlabView& dst, int nx, int ny, int a,
                                int b, double alpha, int sms, cudaStream_t s, const SweepMaps* maps);
+// Two steps per pass over a resident periodic grid 512 cells wide
+// (heat2_band, kernels_band2.cu): 5-D tensor maps over one resident array
+// (boxes of 4 and 2 rows x 64 x 8 tile columns).
+struct Band2Maps {
+  TensorMapBlob m4, m2;
+};
+bool band2_shape_ok(int64_t nx, int64_t ny, int tx, int ty);
+bool band2_maps_encode(Band2Maps* m, const double* base, int tx, int ty, int tz, int ntx, int nty, int ntz);
+// u^{s+2} of the whole grid into dst (the resident array layout) from the
+// array the maps were encoded over
+cudaError_t launch_heat2_band(const Band2Maps& maps, double* dst, int ty, int tz, int nty, int ntz, double alpha,
+                              cudaStream_t s);
 // device -> mapped pinned host rows copied by the SMs (pitches, len in doubles;
 // len and pitches even)
 cudaError_t launch_push_rows(const double* src, int64_t src_pitch, double* dst, int64_t dst_pitch, int64_t rows,

@@ -1,0 +1,255 @@
+// kernels_band2.cu — two Jacobi steps per pass over a resident periodic grid
+// 512 cells wide (heat2_band). Each step is the update of
+// P:L35–L37 (reading R1, heat_update), so one pass gives exactly two single
+// steps; the point is the traffic: u^s is read and u^{s+2} written once per
+// pass, 16 B per cell for two steps instead of 32 B.
+//
+// A CTA owns one band of BY = 4 rows across the full width (8 tile columns of
+// 64, so x is periodic inside the CTA and no column outside it is ever needed)
+// and marches z over the whole periodic ring. Per plane thread 0 stages u^s
+// rows y0-2 .. y0+5 with three 5-D TMA boxes (2 / 4 / 2 rows x 64 x 8 tile
+// columns; the resident array seen as x, y, tile column, z, tile
+// row-and-layer). Consumer warp w owns tile column w, lane l the column pair
+// x = 2l: u^{s+1} on rows y0-1 .. y0+4 at plane z and u^{s+2} on rows
+// y0 .. y0+3 at plane z-1, both marching z in registers (u^s at z-1, z, z+1;
+// u^{s+1} at z-2, z-1, z), y neighbours from the thread's own registers, x
+// neighbours by shuffle; only the warps' edge columns cross warps — u^s's
+// from the stage, u^{s+1}'s through a three-slot edge ring with one named
+// barrier per plane. Grid = ny / 4 CTAs, one per SM, all marching z together,
+// so a band's y-halo rows were just read by its neighbour band (L2 hits).
+#include <cuda.h>
+
+#include "kernels.cuh"
+#include "ptx.cuh"
+
+namespace tiles {
+
+namespace b2 {
+constexpr int NW = 8, TX = 64, NT = NW * 32, BY = 4, S = 6;
+constexpr int OFF_A = 0, OFF_B = NW * 2 * TX, OFF_C = OFF_B + NW * 4 * TX;  // rows y0-2.. | y0.. | y0+4..
+constexpr int STAGE = NW * 8 * TX;                                             // doubles
+constexpr uint32_t BYTES = (uint32_t)STAGE * 8;
+constexpr int ER = 6;                   // u^{s+1} rows y0-1 .. y0+4
+constexpr int ESLOT = NW * 2 * ER;      // [tile column][side][row]
+constexpr size_t SMEM = (size_t)S * STAGE * 8 + (size_t)3 * ESLOT * 8 + (size_t)2 * S * 8;
+// staged row i (y0-2+i) of tile column w, relative to a stage
+__device__ __forceinline__ int srow(int i, int w) {
+  return i < 2 ? OFF_A + (w * 2 + i) * TX : i < 6 ? OFF_B + (w * 4 + i - 2) * TX : OFF_C + (w * 2 + i - 6) * TX;
+}
+}  // namespace b2
+
+static __device__ __forceinline__ void tma_5d(void* dst, const TensorMapBlob* map, int c0, int c1, int c2, int c3,
+                                              int c4, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.5d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5, %6}], "
+      "[%7];" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4), "r"(smem_u32(bar))
+      : "memory");
+}
+
+static __device__ __forceinline__ void bar_consumers_b2() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
+
+
+__global__ void __launch_bounds__(b2::NT, 1)
+    heat2_band(const __grid_constant__ Band2Maps maps, double* __restrict__ dst, const int ty, const int tz,
+               const int nty, const int nz, const int64_t te, const double alpha) {
+  using namespace b2;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double* stage = reinterpret_cast<double*>(smem_raw);
+  double* edge = stage + (size_t)S * STAGE;
+  uint64_t* full = reinterpret_cast<uint64_t*>(edge + 3 * ESLOT);
+  uint64_t* empty = full + S;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], NT);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  const int ny = nty * ty;
+  const int y0 = (int)blockIdx.x * BY;
+  const int nq = nz + 4;  // u^s planes -2 .. nz+1
+  // the producer is thread 0 (eight warps in all: two per scheduler leave
+  // 255 registers per thread, a ninth producer warp would cap them at 168)
+  const int ya = (y0 - 2 + ny) % ny, yc = (y0 + 4) % ny;
+  const int ta = ya / ty, la = ya % ty, tb = y0 / ty, lb = y0 % ty, tc = yc / ty, lc = yc % ty;
+  auto issue = [&](int q) {  // stage u^s plane q - 2 (wrapped) into slot q % S
+    const int st = q % S;
+    mbar_wait(&empty[st], ((q / S) & 1) ^ 1);
+    const int z = (q - 2 + nz) % nz, zl = z % tz, zt = z / tz;
+    double* d = stage + (size_t)st * STAGE;
+    fence_proxy_async();
+    mbar_expect_tx(&full[st], BYTES);
+    tma_5d(d + OFF_A, &maps.m2, 0, la, 0, zl, zt * nty + ta, &full[st]);
+    tma_5d(d + OFF_B, &maps.m4, 0, lb, 0, zl, zt * nty + tb, &full[st]);
+    tma_5d(d + OFF_C, &maps.m2, 0, lc, 0, zl, zt * nty + tc, &full[st]);
+  };
+  int issued = 0;  // thread 0: planes staged so far
+  if (threadIdx.x == 0) {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    for (; issued < S && issued < nq; ++issued) issue(issued);
+  }
+
+  // ------------------------------------------------------- consumer warps
+  const int t = (int)threadIdx.x, lane = t & 31, w = t >> 5;
+  const int x = 2 * lane;
+  // this lane's x-edge source: lane 0 the left tile column's x = 63, lane 31
+  // the right one's x = 0 (the other lanes load lane 0's: a broadcast)
+  const bool right = lane == 31;
+  const int we = right ? (w + 1) % NW : (w + NW - 1) % NW, xe = right ? 0 : TX - 1;
+  // u^{s+1} edge ring: [slot][tile column][side 0: x = 0, 1: x = 63][row]
+  const int e_mine = right ? (w * 2 + 1) * ER : w * 2 * ER;           // written by lanes 0 / 31
+  const int e_nbr = right ? ((w + 1) % NW) * 2 * ER : (((w + NW - 1) % NW) * 2 + 1) * ER;
+  const bool writer = lane == 0 || right;
+  const int yl0 = y0 % ty;
+  const int64_t obase = (int64_t)((y0 / ty) * NW + w) * te + (int64_t)yl0 * TX + x;  // + layer, plane
+  const int64_t oplane = (int64_t)ty * TX;
+
+  auto wait_q = [&](int q) { mbar_wait(&full[q % S], (q / S) & 1); };
+  auto release_q = [&](int q) { mbar_arrive(&empty[q % S]); };
+  auto ld2 = [&](const double* s, int i) { return *reinterpret_cast<const double2*>(s + srow(i, w) + x); };
+
+  double2 a0[6], a1[8], b0[4], b1[6];
+  wait_q(0);
+  {
+    const double* s0 = stage;
+#pragma unroll
+    for (int i = 0; i < 6; ++i) a0[i] = ld2(s0, i + 1);
+  }
+  release_q(0);
+  wait_q(1);
+  {
+    const double* s1 = stage + (size_t)STAGE;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) a1[i] = ld2(s1, i);
+  }
+#pragma unroll
+  for (int j = 0; j < 6; ++j) b1[j] = make_double2(0.0, 0.0);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) b0[j] = make_double2(0.0, 0.0);
+  int p = 0, pl = 0, pt = 0;  // level-2 output plane (z - 1), its in-tile plane and tile layer
+  for (int it = 0; it < nz + 2; ++it) {  // u^{s+1} at z = it - 1
+    const int q = it + 2;                 // u^s plane z + 1
+    wait_q(q);
+    const double* sz = stage + (size_t)((q - 1) % S) * STAGE;
+    const double* sp = stage + (size_t)(q % S) * STAGE;
+    double2 a2[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) a2[i] = ld2(sp, i);
+    double2 b2v[6];
+#pragma unroll
+    for (int r = 0; r < 6; ++r) {
+      const double2 c = a1[r + 1];
+      const double e = sz[srow(r + 1, we) + xe];
+      double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+      double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+      if (lane == 0) xm = e;
+      if (right) xp = e;
+      b2v[r].x = heat_update(c.x, xm, c.y, a1[r].x, a1[r + 2].x, a0[r].x, a2[r + 1].x, alpha);
+      b2v[r].y = heat_update(c.y, c.x, xp, a1[r].y, a1[r + 2].y, a0[r].y, a2[r + 1].y, alpha);
+    }
+    release_q(q - 1);
+    double* ez = edge + (size_t)(it % 3) * ESLOT;
+    if (writer) {
+#pragma unroll
+      for (int r = 0; r < 6; ++r) ez[e_mine + r] = right ? b2v[r].y : b2v[r].x;
+    }
+    bar_consumers_b2();  // u^{s+1} edges of plane z complete (read at it + 1)
+    // every thread has released the slots of planes <= z: refill them
+    if (t == 0)
+      for (; issued < nq && issued <= q - 1 + S; ++issued) issue(issued);
+    if (it >= 2) {        // u^{s+2} at p = z - 1
+      const double* em = edge + (size_t)((it + 2) % 3) * ESLOT + e_nbr;  // slot of it - 1
+      double* o = dst + obase + (int64_t)((pt * nty) * NW) * te + (int64_t)pl * oplane;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const double2 c = b1[j + 1];
+        const double e = em[j + 1];
+        double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+        double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+        if (lane == 0) xm = e;
+        if (right) xp = e;
+        double2 v;
+        v.x = heat_update(c.x, xm, c.y, b1[j].x, b1[j + 2].x, b0[j].x, b2v[j + 1].x, alpha);
+        v.y = heat_update(c.y, c.x, xp, b1[j].y, b1[j + 2].y, b0[j].y, b2v[j + 1].y, alpha);
+        stg2_stream(o + j * TX, v);
+      }
+      ++p;
+      if (++pl == tz) pl = 0, ++pt;
+    }
+#pragma unroll
+    for (int i = 0; i < 6; ++i) a0[i] = a1[i + 1];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) a1[i] = a2[i];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) b0[j] = b1[j + 1];
+#pragma unroll
+    for (int j = 0; j < 6; ++j) b1[j] = b2v[j];
+  }
+  release_q(nq - 1);
+  (void)p;
+}
+
+// driver entry point for cuTensorMapEncodeTiled (no -lcuda link dependency)
+using EncodeTiledFn5 = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                    const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+bool band2_maps_encode(Band2Maps* m, const double* base, int tx, int ty, int tz, int ntx, int nty, int ntz) {
+  static EncodeTiledFn5 f = [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q{};
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess)
+      return (EncodeTiledFn5) nullptr;
+    return reinterpret_cast<EncodeTiledFn5>(p);
+  }();
+  static_assert(sizeof(CUtensorMap) == sizeof(TensorMapBlob), "CUtensorMap size");
+  if (!f || !base || (reinterpret_cast<uintptr_t>(base) & 15) || tx != b2::TX || ntx != b2::NW || ty % b2::BY)
+    return false;
+  const uint64_t te = (uint64_t)tx * ty * tz;
+  // x in the tile, y in the tile, tile column, z in the tile, tile row + layer (iz * nty + iy)
+  const cuuint64_t dims[5] = {(cuuint64_t)tx, (cuuint64_t)ty, (cuuint64_t)ntx, (cuuint64_t)tz,
+                              (cuuint64_t)nty * ntz};
+  const cuuint64_t strides[4] = {(cuuint64_t)tx * 8, te * 8, (cuuint64_t)tx * ty * 8, te * ntx * 8};
+  const cuuint32_t estr[5] = {1, 1, 1, 1, 1};
+  for (int k = 0; k < 2; ++k) {
+    const cuuint32_t box[5] = {(cuuint32_t)tx, k ? 2u : 4u, (cuuint32_t)ntx, 1, 1};
+    if (f(reinterpret_cast<CUtensorMap*>(k ? &m->m2 : &m->m4), CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 5,
+          const_cast<double*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+          CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) !=
+        CUDA_SUCCESS)
+      return false;
+  }
+  return true;
+}
+
+bool band2_shape_ok(int64_t nx, int64_t ny, int tx, int ty) {
+  return tx == b2::TX && nx == (int64_t)b2::NW * b2::TX && ty % b2::BY == 0 && ny % b2::BY == 0;
+}
+
+cudaError_t launch_heat2_band(const Band2Maps& maps, double* dst, int ty, int tz, int nty, int ntz, double alpha,
+                              cudaStream_t s) {
+  using namespace b2;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(heat2_band, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  const int ny = nty * ty, nz = ntz * tz;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(ny / BY));
+  cfg.blockDim = dim3(NT);
+  cfg.dynamicSmemBytes = SMEM;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, heat2_band, maps, dst, ty, tz, nty, nz, (int64_t)TX * ty * tz, alpha);
+}
+
+}  // namespace tiles

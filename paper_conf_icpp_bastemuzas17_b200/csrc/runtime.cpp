@@ -1553,8 +1553,55 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
   return Status::ok();
 }
 
+// Two steps per kernel over the resident periodic grid (heat2_band,
+// DESIGN.md §4): the whole grid is one kernel's work, so each pass reads u^s
+// and writes u^{s+2} once (16 B per cell for two steps) and needs no faces;
+// the faces go stale (re-extracted by the next face-reading run).
+// TILES_BAND2=0 turns it off.
+static bool band2_use(Domain& d, int steps, bool load, bool serial) {
+  static const int on = [] {
+    const char* e = getenv("TILES_BAND2");
+    return e ? atoi(e) : 1;
+  }();
+  const Geometry& G = d.G;
+  return on && !load && !serial && steps >= 2 && d.opt.two_step >= 0 && G.nranks == 1 &&
+         G.bc == TILE_BC_PERIODIC && d.mode == MODE_RESIDENT && !d.user_fn &&
+         band2_shape_ok(G.l[0], G.l[1], (int)G.t[0], (int)G.t[1]) && d.exec->band2_ok(d);
+}
+
+static Status run_band2(Domain& d, int steps, int S) {
+  Exec& X = *d.exec;
+  const Geometry& G = d.G;
+  int bit = d.res_bit;
+  for (int s = 0; s + 1 < steps; s += 2) {  // stream 0: every stream was joined into it (domain_run)
+    Status r = X.band2(d, bit, bit ^ 1, 0);
+    if (r.bad()) return r;
+    bit ^= 1;
+  }
+  const int ev = ev_layer(d, 0, 0);
+  Status r = X.record(d, ev, 0);
+  if (r.bad()) return r;
+  d.res_bit = bit;
+  d.resident_valid = true;
+  d.faces_valid = d.xfaces_valid = false;
+  for (int64_t k = 0; k < G.ntiles; ++k) {
+    d.tile_slot[k] = bit == 0 ? (int)k : (int)(G.ntiles + k);
+    d.tile_dirty[k] = 1;
+  }
+  d.last_batches.clear();
+  d.last_batches.push_back({0, G.n[2], 0, Pipes(S, false).out(0), ev});
+  return Status::ok();
+}
+
 static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool serial) {
   const bool load = !d.resident_valid;
+  if (band2_use(d, steps, load, serial)) {
+    Status r = run_band2(d, steps & ~1, S);
+    if (r.bad()) return r;
+    if (steps & 1) r = run_heat_resident(d, alpha, 1, S, serial);  // the odd step: face-ghost single step
+    d.last_schedule = 7;
+    return r;
+  }
   const int64_t nL = d.G.n[2];
   StreamPlan sp{};
   if (load && !serial) {  // fresh upload: stream-through, wavefront or the batched schedule

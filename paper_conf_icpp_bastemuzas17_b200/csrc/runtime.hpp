@@ -129,6 +129,11 @@ struct Exec {
   // a-1 are read), level s+1 on [a-1, b-1) into dst
   virtual Status slab_sweep2(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, int a, int b,
                              int stream) = 0;
+  // two steps of the whole resident periodic grid in one kernel (heat2_band):
+  // resident array src_bit -> dst_bit; band2_ok: the executor can run it for
+  // this domain (the caller has checked the shape, band2_shape_ok)
+  virtual bool band2_ok(Domain& d) = 0;
+  virtual Status band2(Domain& d, int src_bit, int dst_bit, int stream) = 0;
   // planes [p0, p0+np) of n tile slots: slots s0.. -> host tiles t0.. (the
   // same planes), and slots -> slots (wavefront)
   virtual Status d2h_planes(Domain& d, int64_t t0, int64_t n, int s0, int64_t p0, int64_t np, int stream) = 0;

@@ -407,6 +407,16 @@ class Replayer:
                 self.wave_set(mid, p, nlo, lev[p - lo])
             for p in range(lo - 1, hi - 1):
                 self.wave_set(a, p, nlo, lev2[p - lo + 1])
+        elif name == "band2":
+            # two steps of the whole periodic grid: u^{s+2} (view b) from u^s
+            # (view a), two resident arrays coded as for wsweep
+            nz = c >> 32
+            assert (a >> 1) & 1 != (b >> 1) & 1, "heat2_band reads and writes one array"
+            blk = np.stack([self.wave_get(a, p, 0) for p in range(-2, nz + 2)])
+            lev1 = self.sweep(blk, None, 1, nz + 3)      # planes -1 .. nz
+            lev2 = self.sweep(lev1, None, 2, nz + 2)     # planes 0 .. nz-1
+            for p in range(nz):
+                self.wave_set(b, p, 0, lev2[p + 2])
         elif name == "d2h_planes":
             p0, np_ = d & 0xffffffff, d >> 32
             for i in range(c):

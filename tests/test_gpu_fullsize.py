@@ -110,18 +110,21 @@ def test_c2_wavefront_fig5_path():
         _check_cone(d, gdims, td, 64, blocks)
 
 
-def test_c2_value_path_persistent_resident():
+@pytest.mark.parametrize("two_step", [0, -1])
+def test_c2_value_path_persistent_resident(two_step):
     """C2 512^3, 64^3 tiles, 4 streams: the first run after the upload is the
-    e2e (stream-through) path, the next two are bench.py's `value` path
-    (resident, persistent multi-step launch); 30 steps in all."""
+    e2e (stream-through) path, the next two are bench.py's `resident` path
+    (two steps per kernel, heat2_band; with two_step = -1 the persistent
+    single-step launch); 30 steps in all."""
     n, td = 512, (64, 64, 64)
     gdims = (n, n, n)
-    with T.Domain(gdims, td) as d:
+    with T.Domain(gdims, td, two_step=two_step) as d:
         _fill(d, gdims, td, 42)
         for _ in range(3):
             d.run(T.heat7(ALPHA), 10, 4)
         d.sync()
         st = d.stats()
+        assert d.get_info()["last_schedule"] == (7 if two_step == 0 else 1)
         _check_cone(d, gdims, td, 30, _seam_blocks(gdims, td, 6))
     assert st["n_kernels"] > 0
 

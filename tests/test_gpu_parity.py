@@ -438,6 +438,34 @@ def test_wavefront_bit_exact(dims, td, T, wave):
     assert st["bytes_h2d"] == nx * ny * nz * 8 and st["bytes_d2h"] == nx * ny * nz * 8
 
 
+@pytest.mark.parametrize("dims,td,runs", [((512, 64, 64), (64, 64, 32), [1, 2, 3, 8]),
+                                          ((512, 96, 48), (64, 32, 16), [2, 6, 1]),
+                                          ((512, 8, 40), (64, 4, 8), [3, 4]),
+                                          ((512, 512, 64), (64, 64, 64), [1, 10])])
+def test_band2_resident_bit_exact(dims, td, runs):
+    """Resident periodic runs 512 cells wide: two steps per kernel over the
+    whole grid (heat2_band — full-width bands, 5-D TMA boxes, both levels in
+    registers), the odd step on the face-ghost path, bit-exact to the oracle;
+    the kernel timing counts one 16-byte pass per cell per two steps."""
+    out, ref, info, st = _heat(dims, td, sum(runs), runs=runs)
+    assert np.array_equal(out, ref), np.abs(out - ref).max()
+    u0 = synth.uniform_grid(*dims, 3)
+    with T.Domain(dims, td) as d:
+        d.load(u0)
+        d.run(T.heat7(), 1, 2)
+        d.sync()
+        d.set_kernel_timing(True)
+        d.reset_stats()
+        d.run(T.heat7(), 4, 2)
+        d.sync()
+        st = d.stats()
+        assert d.get_info()["last_schedule"] == 7
+        out = d.store()
+    assert np.array_equal(out, oracle.heat_c(u0, ALPHA, 5))
+    assert st["n_kernels"] == 2 and st["sweep_timed"] == 2
+    assert st["sweep_cells"] == 2 * dims[0] * dims[1] * dims[2]
+
+
 @pytest.mark.parametrize("td,runs", [((32, 64, 8), [1, 4]), ((32, 128, 8), [2, 5])])
 def test_banded_round_robin_snake_bit_exact(td, runs):
     """Banded tiles (ty > band) with enough columns for the round-robin

@@ -139,6 +139,30 @@ def test_resident_multiple_runs_and_dirichlet():
     _run_and_replay((16, 8, 16), (8, 4, 4), [4], 2, bc="dirichlet")
 
 
+@pytest.mark.parametrize("dims,td,runs,ns", [((512, 8, 16), (64, 4, 8), [1, 4, 3, 2], 2),
+                                             ((512, 12, 12), (64, 4, 4), [2, 5], 3),
+                                             ((512, 4, 8), (64, 4, 8), [3, 6], 1)])
+def test_band2_resident_runs_replay_to_oracle(dims, td, runs, ns):
+    """Resident periodic runs 512 cells wide take two steps per kernel over the
+    whole grid (heat2_band, TILE_OP_BAND2; an odd step the face-ghost single
+    step): replayed in random valid orders, bit-exact to the oracle, with the
+    arrays alternating and every later run re-extracting the stale faces."""
+    d = _run_and_replay(dims, td, runs, ns, seeds=(0, 1))
+    assert d.get_info()["last_schedule"] == 7
+    for T_ in (4, 5):
+        d.clear_trace()
+        d.run(T.heat7(ALPHA), T_, ns)
+        d.sync()
+        ops = [op[0] for op in d.trace()]
+        assert ops.count("band2") == T_ // 2
+        assert ("kernel" in ops or "kerneld" in ops) == bool(T_ % 2) and ("extract" in ops) == bool(T_ % 2)
+        b2 = [op for op in d.trace() if op[0] == "band2"]
+        assert all((op[2] >> 1) & 1 != (op[3] >> 1) & 1 for op in b2)
+    # two_step = -1 keeps single steps
+    d2 = _run_and_replay(dims, td, runs[:2], ns, seeds=(2,), two_step=-1)
+    assert "band2" not in [op[0] for op in d2.trace()]
+
+
 @pytest.mark.parametrize("bc", ["periodic", "dirichlet"])
 @pytest.mark.parametrize("dims,td,ns", [((64, 16, 16), (32, 8, 8), 2), ((64, 32, 24), (32, 16, 4), 3),
                                         ((32, 8, 8), (32, 8, 8), 1), ((64, 16, 32), (64, 8, 4), 4)])
