@@ -19,6 +19,8 @@
 // so a band's y-halo rows were just read by its neighbour band (L2 hits).
 #include <cuda.h>
 
+#include <type_traits>
+
 #include "kernels.cuh"
 #include "ptx.cuh"
 
@@ -111,85 +113,86 @@ __global__ void __launch_bounds__(b2::NT, 1)
   auto release_q = [&](int q) { mbar_arrive(&empty[q % S]); };
   auto ld2 = [&](const double* s, int i) { return *reinterpret_cast<const double2*>(s + srow(i, w) + x); };
 
-  double2 a0[6], a1[8], b0[4], b1[6];
+  // register rings, period 3 (the loop below is unrolled by three, so no
+  // value moves between registers): u^s planes z-1, z, z+1 in a[(k)..(k+2)
+  // % 3], u^{s+1} planes z-2, z-1, z in b[(k)..(k+2) % 3] at phase k
+  double2 a[3][8], b[3][6];
   wait_q(0);
-  {
-    const double* s0 = stage;
 #pragma unroll
-    for (int i = 0; i < 6; ++i) a0[i] = ld2(s0, i + 1);
-  }
+  for (int i = 0; i < 8; ++i) a[0][i] = ld2(stage, i);
   release_q(0);
   wait_q(1);
-  {
-    const double* s1 = stage + (size_t)STAGE;
 #pragma unroll
-    for (int i = 0; i < 8; ++i) a1[i] = ld2(s1, i);
-  }
+  for (int i = 0; i < 8; ++i) a[1][i] = ld2(stage + (size_t)STAGE, i);
 #pragma unroll
-  for (int j = 0; j < 6; ++j) b1[j] = make_double2(0.0, 0.0);
+  for (int k = 0; k < 3; ++k)
 #pragma unroll
-  for (int j = 0; j < 4; ++j) b0[j] = make_double2(0.0, 0.0);
-  int p = 0, pl = 0, pt = 0;  // level-2 output plane (z - 1), its in-tile plane and tile layer
-  for (int it = 0; it < nz + 2; ++it) {  // u^{s+1} at z = it - 1
-    const int q = it + 2;                 // u^s plane z + 1
+    for (int j = 0; j < 6; ++j) b[k][j] = make_double2(0.0, 0.0);
+  int pl = 0, pt = 0;           // level-2 output plane (z - 1): in-tile plane and tile layer
+  int sq = 2 % S, sq1 = 1;      // slots of u^s planes z + 1 and z
+  int e0 = 0, e1 = 2;           // edge-ring slots of it and it - 1
+  auto step = [&](int it, auto kc) {
+    constexpr int K = decltype(kc)::value;
+    constexpr int P0 = K, P1 = (K + 1) % 3, P2 = (K + 2) % 3;  // z-1, z, z+1 | z-2, z-1, z
+    const int q = it + 2;  // u^s plane z + 1
     wait_q(q);
-    const double* sz = stage + (size_t)((q - 1) % S) * STAGE;
-    const double* sp = stage + (size_t)(q % S) * STAGE;
-    double2 a2[8];
+    const double* sz = stage + (size_t)sq1 * STAGE;
+    const double* sp = stage + (size_t)sq * STAGE;
 #pragma unroll
-    for (int i = 0; i < 8; ++i) a2[i] = ld2(sp, i);
-    double2 b2v[6];
+    for (int i = 0; i < 8; ++i) a[P2][i] = ld2(sp, i);
 #pragma unroll
-    for (int r = 0; r < 6; ++r) {
-      const double2 c = a1[r + 1];
+    for (int r = 0; r < 6; ++r) {  // u^{s+1} at z, row y0-1+r
+      const double2 c = a[P1][r + 1];
       const double e = sz[srow(r + 1, we) + xe];
       double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
       double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
       if (lane == 0) xm = e;
       if (right) xp = e;
-      b2v[r].x = heat_update(c.x, xm, c.y, a1[r].x, a1[r + 2].x, a0[r].x, a2[r + 1].x, alpha);
-      b2v[r].y = heat_update(c.y, c.x, xp, a1[r].y, a1[r + 2].y, a0[r].y, a2[r + 1].y, alpha);
+      b[P2][r].x = heat_update(c.x, xm, c.y, a[P1][r].x, a[P1][r + 2].x, a[P0][r + 1].x, a[P2][r + 1].x, alpha);
+      b[P2][r].y = heat_update(c.y, c.x, xp, a[P1][r].y, a[P1][r + 2].y, a[P0][r + 1].y, a[P2][r + 1].y, alpha);
     }
     release_q(q - 1);
-    double* ez = edge + (size_t)(it % 3) * ESLOT;
     if (writer) {
+      double* ez = edge + (size_t)e0 * ESLOT + e_mine;
 #pragma unroll
-      for (int r = 0; r < 6; ++r) ez[e_mine + r] = right ? b2v[r].y : b2v[r].x;
+      for (int r = 0; r < 6; ++r) ez[r] = right ? b[P2][r].y : b[P2][r].x;
     }
     bar_consumers_b2();  // u^{s+1} edges of plane z complete (read at it + 1)
     // every thread has released the slots of planes <= z: refill them
     if (t == 0)
       for (; issued < nq && issued <= q - 1 + S; ++issued) issue(issued);
-    if (it >= 2) {        // u^{s+2} at p = z - 1
-      const double* em = edge + (size_t)((it + 2) % 3) * ESLOT + e_nbr;  // slot of it - 1
+    if (it >= 2) {  // u^{s+2} at p = z - 1, rows y0 .. y0+3
+      const double* em = edge + (size_t)e1 * ESLOT + e_nbr;
       double* o = dst + obase + (int64_t)((pt * nty) * NW) * te + (int64_t)pl * oplane;
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
-        const double2 c = b1[j + 1];
+        const double2 c = b[P1][j + 1];
         const double e = em[j + 1];
         double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
         double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
         if (lane == 0) xm = e;
         if (right) xp = e;
         double2 v;
-        v.x = heat_update(c.x, xm, c.y, b1[j].x, b1[j + 2].x, b0[j].x, b2v[j + 1].x, alpha);
-        v.y = heat_update(c.y, c.x, xp, b1[j].y, b1[j + 2].y, b0[j].y, b2v[j + 1].y, alpha);
+        v.x = heat_update(c.x, xm, c.y, b[P1][j].x, b[P1][j + 2].x, b[P0][j + 1].x, b[P2][j + 1].x, alpha);
+        v.y = heat_update(c.y, c.x, xp, b[P1][j].y, b[P1][j + 2].y, b[P0][j + 1].y, b[P2][j + 1].y, alpha);
         stg2_stream(o + j * TX, v);
       }
-      ++p;
       if (++pl == tz) pl = 0, ++pt;
     }
-#pragma unroll
-    for (int i = 0; i < 6; ++i) a0[i] = a1[i + 1];
-#pragma unroll
-    for (int i = 0; i < 8; ++i) a1[i] = a2[i];
-#pragma unroll
-    for (int j = 0; j < 4; ++j) b0[j] = b1[j + 1];
-#pragma unroll
-    for (int j = 0; j < 6; ++j) b1[j] = b2v[j];
+    sq1 = sq;
+    sq = sq + 1 == S ? 0 : sq + 1;
+    e1 = e0;
+    e0 = e0 == 2 ? 0 : e0 + 1;
+  };
+  const int nit = nz + 2;  // u^{s+1} at z = it - 1 for it in [0, nit)
+  for (int it = 0; it < nit; it += 3) {
+    step(it, std::integral_constant<int, 0>{});
+    if (it + 1 >= nit) break;
+    step(it + 1, std::integral_constant<int, 1>{});
+    if (it + 2 >= nit) break;
+    step(it + 2, std::integral_constant<int, 2>{});
   }
   release_q(nq - 1);
-  (void)p;
 }
 
 // driver entry point for cuTensorMapEncodeTiled (no -lcuda link dependency)
