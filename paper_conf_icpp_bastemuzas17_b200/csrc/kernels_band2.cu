@@ -33,7 +33,7 @@ constexpr int STAGE = NW * 8 * TX;                                             /
 constexpr uint32_t BYTES = (uint32_t)STAGE * 8;
 constexpr int ER = 6;                   // u^{s+1} rows y0-1 .. y0+4
 constexpr int ESLOT = NW * 2 * ER;      // [tile column][side][row]
-constexpr size_t SMEM = (size_t)S * STAGE * 8 + (size_t)3 * ESLOT * 8 + (size_t)2 * S * 8;
+constexpr size_t SMEM = (size_t)S * STAGE * 8 + (size_t)3 * ESLOT * 8 + (size_t)S * 8;
 // staged row i (y0-2+i) of tile column w, relative to a stage
 __device__ __forceinline__ int srow(int i, int w) {
   return i < 2 ? OFF_A + (w * 2 + i) * TX : i < 6 ? OFF_B + (w * 4 + i - 2) * TX : OFF_C + (w * 2 + i - 6) * TX;
@@ -60,12 +60,8 @@ __global__ void __launch_bounds__(b2::NT, 1)
   double* stage = reinterpret_cast<double*>(smem_raw);
   double* edge = stage + (size_t)S * STAGE;
   uint64_t* full = reinterpret_cast<uint64_t*>(edge + 3 * ESLOT);
-  uint64_t* empty = full + S;
   if (threadIdx.x == 0) {
-    for (int s = 0; s < S; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&empty[s], NT);
-    }
+    for (int s = 0; s < S; ++s) mbar_init(&full[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
@@ -77,21 +73,26 @@ __global__ void __launch_bounds__(b2::NT, 1)
   // 255 registers per thread, a ninth producer warp would cap them at 168)
   const int ya = (y0 - 2 + ny) % ny, yc = (y0 + 4) % ny;
   const int ta = ya / ty, la = ya % ty, tb = y0 / ty, lb = y0 % ty, tc = yc / ty, lc = yc % ty;
-  auto issue = [&](int q) {  // stage u^s plane q - 2 (wrapped) into slot q % S
-    const int st = q % S;
-    mbar_wait(&empty[st], ((q / S) & 1) ^ 1);
-    const int z = (q - 2 + nz) % nz, zl = z % tz, zt = z / tz;
-    double* d = stage + (size_t)st * STAGE;
+  // thread 0 stages u^s plane q - 2 (wrapped) into slot q % S. A slot is
+  // refilled only after the block barrier that follows every thread's last
+  // read of it, so no empty-slot mbarrier is needed (the barrier orders those
+  // reads before this thread's async-proxy writes, fence.proxy.async below)
+  int qz = nz - 2, qzl = qz % tz, qzt = qz / tz, qs = 0;  // next plane: z, in-tile z, layer, slot
+  auto issue = [&]() {
+    double* d = stage + (size_t)qs * STAGE;
     fence_proxy_async();
-    mbar_expect_tx(&full[st], BYTES);
-    tma_5d(d + OFF_A, &maps.m2, 0, la, 0, zl, zt * nty + ta, &full[st]);
-    tma_5d(d + OFF_B, &maps.m4, 0, lb, 0, zl, zt * nty + tb, &full[st]);
-    tma_5d(d + OFF_C, &maps.m2, 0, lc, 0, zl, zt * nty + tc, &full[st]);
+    mbar_expect_tx(&full[qs], BYTES);
+    tma_5d(d + OFF_A, &maps.m2, 0, la, 0, qzl, qzt * nty + ta, &full[qs]);
+    tma_5d(d + OFF_B, &maps.m4, 0, lb, 0, qzl, qzt * nty + tb, &full[qs]);
+    tma_5d(d + OFF_C, &maps.m2, 0, lc, 0, qzl, qzt * nty + tc, &full[qs]);
+    if (++qz == nz) qz = 0, qzl = 0, qzt = 0;
+    else if (++qzl == tz) qzl = 0, ++qzt;
+    qs = qs + 1 == S ? 0 : qs + 1;
   };
   int issued = 0;  // thread 0: planes staged so far
   if (threadIdx.x == 0) {
     asm volatile("griddepcontrol.wait;" ::: "memory");
-    for (; issued < S && issued < nq; ++issued) issue(issued);
+    for (; issued < S && issued < nq; ++issued) issue();
   }
 
   // ------------------------------------------------------- consumer warps
@@ -110,7 +111,6 @@ __global__ void __launch_bounds__(b2::NT, 1)
   const int64_t oplane = (int64_t)ty * TX;
 
   auto wait_q = [&](int q) { mbar_wait(&full[q % S], (q / S) & 1); };
-  auto release_q = [&](int q) { mbar_arrive(&empty[q % S]); };
   auto ld2 = [&](const double* s, int i) { return *reinterpret_cast<const double2*>(s + srow(i, w) + x); };
 
   // register rings, period 3 (the loop below is unrolled by three, so no
@@ -120,7 +120,6 @@ __global__ void __launch_bounds__(b2::NT, 1)
   wait_q(0);
 #pragma unroll
   for (int i = 0; i < 8; ++i) a[0][i] = ld2(stage, i);
-  release_q(0);
   wait_q(1);
 #pragma unroll
   for (int i = 0; i < 8; ++i) a[1][i] = ld2(stage + (size_t)STAGE, i);
@@ -151,7 +150,6 @@ __global__ void __launch_bounds__(b2::NT, 1)
       b[P2][r].x = heat_update(c.x, xm, c.y, a[P1][r].x, a[P1][r + 2].x, a[P0][r + 1].x, a[P2][r + 1].x, alpha);
       b[P2][r].y = heat_update(c.y, c.x, xp, a[P1][r].y, a[P1][r + 2].y, a[P0][r + 1].y, a[P2][r + 1].y, alpha);
     }
-    release_q(q - 1);
     if (writer) {
       double* ez = edge + (size_t)e0 * ESLOT + e_mine;
 #pragma unroll
@@ -160,7 +158,7 @@ __global__ void __launch_bounds__(b2::NT, 1)
     bar_consumers_b2();  // u^{s+1} edges of plane z complete (read at it + 1)
     // every thread has released the slots of planes <= z: refill them
     if (t == 0)
-      for (; issued < nq && issued <= q - 1 + S; ++issued) issue(issued);
+      for (; issued < nq && issued <= q - 1 + S; ++issued) issue();
     if (it >= 2) {  // u^{s+2} at p = z - 1, rows y0 .. y0+3
       const double* em = edge + (size_t)e1 * ESLOT + e_nbr;
       double* o = dst + obase + (int64_t)((pt * nty) * NW) * te + (int64_t)pl * oplane;
@@ -192,7 +190,6 @@ __global__ void __launch_bounds__(b2::NT, 1)
     if (it + 2 >= nit) break;
     step(it + 2, std::integral_constant<int, 2>{});
   }
-  release_q(nq - 1);
 }
 
 // driver entry point for cuTensorMapEncodeTiled (no -lcuda link dependency)
