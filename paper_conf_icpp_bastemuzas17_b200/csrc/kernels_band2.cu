@@ -150,16 +150,10 @@ __global__ void __launch_bounds__(b2::NT, 1)
       b[P2][r].x = heat_update(c.x, xm, c.y, a[P1][r].x, a[P1][r + 2].x, a[P0][r + 1].x, a[P2][r + 1].x, alpha);
       b[P2][r].y = heat_update(c.y, c.x, xp, a[P1][r].y, a[P1][r + 2].y, a[P0][r + 1].y, a[P2][r + 1].y, alpha);
     }
-    if (writer) {
-      double* ez = edge + (size_t)e0 * ESLOT + e_mine;
-#pragma unroll
-      for (int r = 0; r < 6; ++r) ez[r] = right ? b[P2][r].y : b[P2][r].x;
-    }
-    bar_consumers_b2();  // u^{s+1} edges of plane z complete (read at it + 1)
-    // every thread has released the slots of planes <= z: refill them
-    if (t == 0)
-      for (; issued < nq && issued <= q - 1 + S; ++issued) issue();
-    if (it >= 2) {  // u^{s+2} at p = z - 1, rows y0 .. y0+3
+    // u^{s+2} at p = z - 1, rows y0 .. y0+3: own registers and the edges of
+    // plane z - 1 (complete since the last barrier), so no barrier between the
+    // two levels and the compiler interleaves them
+    if (it >= 2) {
       const double* em = edge + (size_t)e1 * ESLOT + e_nbr;
       double* o = dst + obase + (int64_t)((pt * nty) * NW) * te + (int64_t)pl * oplane;
 #pragma unroll
@@ -177,6 +171,15 @@ __global__ void __launch_bounds__(b2::NT, 1)
       }
       if (++pl == tz) pl = 0, ++pt;
     }
+    if (writer) {
+      double* ez = edge + (size_t)e0 * ESLOT + e_mine;
+#pragma unroll
+      for (int r = 0; r < 6; ++r) ez[r] = right ? b[P2][r].y : b[P2][r].x;
+    }
+    bar_consumers_b2();  // u^{s+1} edges of plane z complete (read at it + 1)
+    // every thread has released the slots of planes <= z: refill them
+    if (t == 0)
+      for (; issued < nq && issued <= q - 1 + S; ++issued) issue();
     sq1 = sq;
     sq = sq + 1 == S ? 0 : sq + 1;
     e1 = e0;
