@@ -49,6 +49,18 @@ static __device__ __forceinline__ void tma_5d(void* dst, const TensorMapBlob* ma
       : "memory");
 }
 
+// v = [addr] in the lanes where pred != 0, unchanged elsewhere (a predicated
+// shared load: no branch, no select)
+static __device__ __forceinline__ void lds_if(double& v, uint32_t addr, uint32_t pred) {
+  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p ld.shared.f64 %0, [%1];\n}" : "+d"(v)
+               : "r"(addr), "r"(pred));
+}
+static __device__ __forceinline__ void sts_if(uint32_t addr, double v, uint32_t pred) {
+  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.shared.f64 [%0], %1;\n}" ::"r"(addr), "d"(v),
+               "r"(pred)
+               : "memory");
+}
+
 static __device__ __forceinline__ void bar_consumers_b2() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
 
 
@@ -105,7 +117,7 @@ __global__ void __launch_bounds__(b2::NT, 1)
   // u^{s+1} edge ring: [slot][tile column][side 0: x = 0, 1: x = 63][row]
   const int e_mine = right ? (w * 2 + 1) * ER : w * 2 * ER;           // written by lanes 0 / 31
   const int e_nbr = right ? ((w + 1) % NW) * 2 * ER : (((w + NW - 1) % NW) * 2 + 1) * ER;
-  const bool writer = lane == 0 || right;
+  const uint32_t is_left = lane == 0, is_right = right;
   const int yl0 = y0 % ty;
   const int64_t obase = (int64_t)((y0 / ty) * NW + w) * te + (int64_t)yl0 * TX + x;  // + layer, plane
   const int64_t oplane = (int64_t)ty * TX;
@@ -142,11 +154,11 @@ __global__ void __launch_bounds__(b2::NT, 1)
 #pragma unroll
     for (int r = 0; r < 6; ++r) {  // u^{s+1} at z, row y0-1+r
       const double2 c = a[P1][r + 1];
-      const double e = sz[srow(r + 1, we) + xe];
       double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
       double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
-      if (lane == 0) xm = e;
-      if (right) xp = e;
+      const uint32_t ea = smem_u32(sz + srow(r + 1, we) + xe);
+      lds_if(xm, ea, is_left);
+      lds_if(xp, ea, is_right);
       b[P2][r].x = heat_update(c.x, xm, c.y, a[P1][r].x, a[P1][r + 2].x, a[P0][r + 1].x, a[P2][r + 1].x, alpha);
       b[P2][r].y = heat_update(c.y, c.x, xp, a[P1][r].y, a[P1][r + 2].y, a[P0][r + 1].y, a[P2][r + 1].y, alpha);
     }
@@ -159,11 +171,10 @@ __global__ void __launch_bounds__(b2::NT, 1)
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
         const double2 c = b[P1][j + 1];
-        const double e = em[j + 1];
         double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
         double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
-        if (lane == 0) xm = e;
-        if (right) xp = e;
+        lds_if(xm, smem_u32(em + j + 1), is_left);
+        lds_if(xp, smem_u32(em + j + 1), is_right);
         double2 v;
         v.x = heat_update(c.x, xm, c.y, b[P1][j].x, b[P1][j + 2].x, b[P0][j + 1].x, b[P2][j + 1].x, alpha);
         v.y = heat_update(c.y, c.x, xp, b[P1][j].y, b[P1][j + 2].y, b[P0][j + 1].y, b[P2][j + 1].y, alpha);
@@ -171,10 +182,13 @@ __global__ void __launch_bounds__(b2::NT, 1)
       }
       if (++pl == tz) pl = 0, ++pt;
     }
-    if (writer) {
-      double* ez = edge + (size_t)e0 * ESLOT + e_mine;
+    {
+      const uint32_t ez = smem_u32(edge + (size_t)e0 * ESLOT + e_mine);
 #pragma unroll
-      for (int r = 0; r < 6; ++r) ez[r] = right ? b[P2][r].y : b[P2][r].x;
+      for (int r = 0; r < 6; ++r) {
+        sts_if(ez + 8 * r, b[P2][r].x, is_left);
+        sts_if(ez + 8 * r, b[P2][r].y, is_right);
+      }
     }
     bar_consumers_b2();  // u^{s+1} edges of plane z complete (read at it + 1)
     // every thread has released the slots of planes <= z: refill them
