@@ -1142,18 +1142,23 @@ def run_main_leg(args):
     res_value = ws * cells * T * args.steps / (ms_res / 1e3) / 1e9
     rs_ms, rs_cells, rs_n = st_res["sweep_ms"], st_res["sweep_cells"], max(1, st_res["sweep_timed"])
     r_ach = 16.0 * rs_cells / (rs_ms / 1e3) / 1e9 if rs_ms > 0 else None
-    tps = traffic_from_profile(args.config) if spp == 1 else None
-    steps_per_launch = rs_cells / rs_n / cells
+    res_sched = dom.get_info().get("last_schedule", 1)
+    band2 = res_sched == 7   # heat2_band: one launch = one pass = two steps
+    tps = traffic_from_profile("band2" if band2 else args.config) if (spp == 1 or band2) else None
+    steps_per_launch = rs_cells / rs_n / cells * (2 if band2 else 1)
     resident = {"value": res_value, "unit": "Gcell-updates/s", "ms_per_step": ms_res / args.steps,
                 "def": "grid resident in HBM; tile_run(T) per step, no host transfers",
                 "gpu_launches": st_res["n_kernels"],
                 "roofline": {"bound": "hbm", "achieved": r_ach, "peak": peak, "unit": "GB/s",
                              "frac": r_ach / peak if r_ach else None,
                              "traffic": tps * steps_per_launch if tps else None, "traffic_per_step": tps,
-                             "kernel": "heat7_fixed" if spp == 1 else "heat7x2 (2 steps per pass)",
-                             "algorithmic_bytes_per_cell_update": 16.0 / spp,
+                             "kernel": "heat2_band (2 steps per pass)" if band2 else
+                                       "heat7_fixed" if spp == 1 else "heat7x2 (2 steps per pass)",
+                             "schedule": SCHED_NAMES.get(res_sched, str(res_sched)),
+                             "algorithmic_bytes_per_cell_update": 8.0 if band2 else 16.0 / spp,
                              "algorithmic_bytes_per_launch": 16.0 * rs_cells / rs_n,
-                             "steps_per_launch": steps_per_launch * spp, "avg_launch_ms": rs_ms / rs_n,
+                             "steps_per_launch": steps_per_launch * (1 if band2 else spp),
+                             "avg_launch_ms": rs_ms / rs_n,
                              "peak_source": peak_src},
                 "clocks": clk_res.summary()}
 

@@ -1558,15 +1558,18 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
 // and writes u^{s+2} once (16 B per cell for two steps) and needs no faces;
 // the faces go stale (re-extracted by the next face-reading run).
 // TILES_BAND2=0 turns it off.
-static bool band2_use(Domain& d, int steps, bool load, bool serial) {
+static bool band2_fits(Domain& d, bool serial) {
   static const int on = [] {
     const char* e = getenv("TILES_BAND2");
     return e ? atoi(e) : 1;
   }();
   const Geometry& G = d.G;
-  return on && !load && !serial && steps >= 2 && d.opt.two_step >= 0 && G.nranks == 1 &&
-         G.bc == TILE_BC_PERIODIC && d.mode == MODE_RESIDENT && !d.user_fn &&
-         band2_shape_ok(G.l[0], G.l[1], (int)G.t[0], (int)G.t[1]) && d.exec->band2_ok(d);
+  return on && !serial && d.opt.two_step >= 0 && G.nranks == 1 && G.bc == TILE_BC_PERIODIC &&
+         d.mode == MODE_RESIDENT && !d.user_fn && band2_shape_ok(G.l[0], G.l[1], (int)G.t[0], (int)G.t[1]) &&
+         d.exec->band2_ok(d);
+}
+static bool band2_use(Domain& d, int steps, bool load, bool serial) {
+  return !load && steps >= 2 && band2_fits(d, serial);
 }
 
 static Status run_band2(Domain& d, int steps, int S) {
@@ -1614,7 +1617,10 @@ static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool 
     // whole-domain steps partly overlapped (0.52 r per plane-step: the
     // persistent heat7 step per plane over the duplex link-plane time, fitted
     // with r on the Fig. 5 sweep)
-    const double est_batched = 2.0 * nz + 0.52 * d.r_sweep * nz * steps;
+    // (0.6 r when the middle steps run two per kernel on heat2_band, fitted
+    // on the Fig. 5 sweep with heat2_band: T = 100 58.8 ms, T = 1000 257 ms;
+    // the wavefront's 53.4 ms wins at T = 100)
+    const double est_batched = 2.0 * nz + (band2_fits(d, serial) ? 0.6 : 0.52) * d.r_sweep * nz * steps;
     bool take_wf = wf && (d.opt.wavefront > 0 || (d.opt.stream_through <= 0 && wp.est < est_batched &&
                                                   (!st || wp.est < est_st)));
     bool take_st = !take_wf && st && (d.opt.stream_through > 0 || est_st < est_batched);
@@ -1633,18 +1639,26 @@ static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool 
   struct Phase {
     int steps;
     bool layered;
+    bool band2;  // whole-domain steps two per kernel (heat2_band, stream 0)
   };
   std::vector<Phase> ph;
   if (serial || !load) {
-    ph.push_back({T, false});
+    ph.push_back({T, false, false});
   } else {
     const int k1 = (int)std::min<int64_t>(T, nL / 2 + 1);
+    const int mid = T - k1 - 1;
+    const bool all1 = std::find(kp.begin(), kp.end(), 2) == kp.end();
     if (T <= k1 + 1) {
-      ph.push_back({T, true});
+      ph.push_back({T, true, false});
+    } else if (mid >= 2 && all1 && band2_fits(d, serial)) {
+      // the middle steps in pairs on heat2_band, an odd one with the last step
+      ph.push_back({k1, true, false});
+      ph.push_back({mid & ~1, false, true});
+      ph.push_back({1 + (mid & 1), true, false});
     } else {
-      ph.push_back({k1, true});
-      ph.push_back({T - k1 - 1, false});
-      ph.push_back({1, true});
+      ph.push_back({k1, true, false});
+      ph.push_back({mid, false, false});
+      ph.push_back({1, true, false});
     }
   }
   int bit = d.res_bit, fp = d.face_parity;
@@ -1653,13 +1667,25 @@ static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool 
   std::vector<std::pair<Batch, int>> last;  // batches of the last phase + final event
   size_t pass0 = 0;
   for (size_t pi = 0; pi < ph.size(); ++pi) {
+    if (ph[pi].band2) {  // after the join below (stream 0 waited for every batch)
+      for (int s = 0; s + 1 < ph[pi].steps; s += 2) {
+        Status r = d.exec->band2(d, bit, bit ^ 1, 0);
+        if (r.bad()) return r;
+        bit ^= 1;
+      }
+      pass0 += (size_t)ph[pi].steps;
+      d.faces_valid = d.xfaces_valid = false;  // the next phase re-extracts them
+      Status r = d.exec->record(d, ev_phase(d), 0);
+      if (r.bad()) return r;
+      continue;
+    }
     ResidentRun R(d);
     R.alpha = alpha;
     R.T = ph[pi].steps;
     R.kpass.assign(kp.begin() + (long)pass0, kp.begin() + (long)(pass0 + (size_t)R.T));
     pass0 += (size_t)R.T;
     R.need_load = pi == 0 && load;
-    R.need_extract = pi == 0 && !(any_x2 || !d.direct_ok ? d.faces_valid : d.xfaces_valid);
+    R.need_extract = (pi == 0 || ph[pi - 1].band2) && !(any_x2 || !d.direct_ok ? d.faces_valid : d.xfaces_valid);
     R.multi = d.G.nranks > 1;
     R.entry_wait = pi > 0;
     R.bit0 = bit;

@@ -466,6 +466,15 @@ def test_band2_resident_bit_exact(dims, td, runs):
     assert st["sweep_cells"] == 2 * dims[0] * dims[1] * dims[2]
 
 
+@pytest.mark.parametrize("T_", [7, 9, 12, 40])
+def test_band2_middle_of_batched_fresh_upload_bit_exact(T_):
+    """Fresh upload on the batched schedule: the load-overlapping layer steps,
+    the middle steps in pairs on heat2_band, the layered last step(s)."""
+    dims, td = (512, 64, 128), (64, 64, 16)
+    out, ref, info, st = _heat(dims, td, T_, wavefront=-1, stream_through=-1)
+    assert np.array_equal(out, ref), np.abs(out - ref).max()
+
+
 @pytest.mark.parametrize("td,runs", [((32, 64, 8), [1, 4]), ((32, 128, 8), [2, 5])])
 def test_banded_round_robin_snake_bit_exact(td, runs):
     """Banded tiles (ty > band) with enough columns for the round-robin

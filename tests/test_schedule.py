@@ -163,6 +163,21 @@ def test_band2_resident_runs_replay_to_oracle(dims, td, runs, ns):
     assert "band2" not in [op[0] for op in d2.trace()]
 
 
+@pytest.mark.parametrize("T_", [9, 12, 7])
+def test_band2_middle_of_batched_fresh_upload_replays(T_):
+    """A fresh upload on the batched schedule (layer batches overlapping the
+    load, whole-domain middle steps, a layered last step): the middle steps
+    run in pairs on heat2_band once the load phase is joined, an odd one
+    joins the last phase, which re-extracts the stale faces; replayed in
+    random orders, bit-exact."""
+    dims, td = (512, 8, 64), (64, 4, 8)   # 8 tile layers: load phase of 5 steps
+    d = _run_and_replay(dims, td, [T_], 2, seeds=(0, 1, 2), wavefront=-1, stream_through=-1)
+    ops = [op[0] for op in d.trace()]
+    mid = T_ - 5 - 1
+    assert ops.count("band2") == (mid // 2 if mid >= 2 else 0)
+    assert d.get_info()["last_schedule"] == 1
+
+
 @pytest.mark.parametrize("bc", ["periodic", "dirichlet"])
 @pytest.mark.parametrize("dims,td,ns", [((64, 16, 16), (32, 8, 8), 2), ((64, 32, 24), (32, 16, 4), 3),
                                         ((32, 8, 8), (32, 8, 8), 1), ((64, 16, 32), (64, 8, 4), 4)])
