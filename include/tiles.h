@@ -184,12 +184,15 @@ typedef struct {
                                    the periodic seam. -1 =
                                    never, 0 (default) = when the cost model
                                    prefers it to stream-through and the
-                                   batched schedule, 1 = whenever feasible,
-                                   2 = whenever feasible, two levels per pass
-                                   through a third level buffer when the
-                                   budget holds it (one kernel per pass,
-                                   slab_sweep2_tile; measured slower than two
-                                   single-level passes on B200) */
+                                   batched schedule, 1 = whenever feasible.
+                                   Grids 512 wide with 64-wide tiles take two
+                                   levels per pass (heat2_band_slab, through a
+                                   third level buffer when the budget holds
+                                   it); 2 = whenever feasible, two levels per
+                                   pass at any shape (slab_sweep2_tile off the
+                                   band shape: slower than two single-level
+                                   passes); 3 = whenever
+                                   feasible, one level per pass */
   double sweep_link_ratio;      /* cost model of the fresh-upload schedules
                                    (DESIGN.md §5): time of one stencil sweep
                                    per plane over one plane's duplex host-link

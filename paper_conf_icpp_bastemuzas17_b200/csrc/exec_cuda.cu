@@ -455,6 +455,65 @@ struct CudaExec final : Exec {
   }
   Band2Maps bmaps[2];
   int bmaps_state = 0;  // 0 not tried, 1 encoded, -1 not available
+  // tensor maps of other tile-blocked regions (wavefront level arrays and
+  // scratch layers), by base pointer and tile layers
+  struct MapEntry {
+    const double* base;
+    int layers;
+    bool ok;
+    Band2Maps m;
+  };
+  std::vector<MapEntry> band_maps;
+  const Band2Maps* band_maps_for(Domain& d, const double* base, int layers) {
+    for (auto& e : band_maps)
+      if (e.base == base && e.layers == layers) return e.ok ? &e.m : nullptr;
+    const Geometry& G = d.G;
+    MapEntry e{base, layers, false, {}};
+    e.ok = band2_maps_encode(&e.m, base, (int)G.t[0], (int)G.t[1], (int)G.t[2], (int)G.n[0], (int)G.n[1], layers);
+    band_maps.push_back(e);
+    return e.ok ? &band_maps.back().m : nullptr;
+  }
+  // the views of a two-level pass as heat2_band_slab descriptors (RESIDENT:
+  // wrapped array; WAVE: array + scratch layers); false if any does not fit
+  bool band2_slab_views(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, Band2View* bv,
+                        Band2Out* bo) {
+    static const int on = [] {
+      const char* e = getenv("TILES_BAND2_SLAB");
+      return e ? atoi(e) : 1;
+    }();
+    const Geometry& G = d.G;
+    if (!on || G.nranks != 1 || !band2_shape_ok(G.l[0], G.l[1], (int)G.t[0], (int)G.t[1])) return false;
+    auto in = [&](const SlabRef& r, Band2View* v) {
+      const Band2Maps* mm = nullptr;
+      v->nlo = 0;
+      v->wrap = r.kind == SlabRef::RESIDENT;
+      // (each map is copied out before the next lookup: the cache may grow)
+      if (r.kind == SlabRef::RESIDENT) {
+        mm = band_maps_for(d, d.slot_ptr(r.slot ? (int)G.ntiles : 0), (int)G.n[2]);
+        if (!mm) return false;
+        v->main = *mm;
+      } else if (r.kind == SlabRef::WAVE) {
+        mm = band_maps_for(d, d.slot_ptr(r.slot), (int)G.n[2]);
+        if (!mm) return false;
+        v->main = *mm;
+        mm = band_maps_for(d, d.slot_ptr(r.ring[0]), (int)r.un);
+        if (!mm) return false;
+        v->scr = *mm;
+        v->nlo = (int)r.un;
+      } else {
+        return false;
+      }
+      return true;
+    };
+    auto out = [&](const SlabRef& r, Band2Out* o) {
+      if (r.kind != SlabRef::WAVE) return false;
+      o->base = d.slot_ptr(r.slot);
+      o->hlo = d.slot_ptr(r.ring[0]);
+      o->nlo = (int)r.un;
+      return true;
+    };
+    return in(src, &bv[0]) && in(mid, &bv[1]) && out(mid, &bo[0]) && out(dst, &bo[1]);
+  }
   bool band2_ok(Domain& d) override {
     if (bmaps_state == 0) {
       const Geometry& G = d.G;
@@ -490,9 +549,17 @@ struct CudaExec final : Exec {
     const SlabView s = slab_view(d, src, a), m = slab_view(d, mid, a), t = slab_view(d, dst, a);
     bool fused = true;
     next_cells = d.kernel_timing ? (uint64_t)(b - a) * d.G.l[0] * d.G.l[1] : 0;  // one pass over the cells
+    // the band layout (heat2_band_slab) when the grid is 512 wide and every
+    // view has its tensor maps; else the tile-column kernel
+    Band2View bv[2];
+    Band2Out bo[2];
+    const bool band = band2_slab_views(d, src, mid, dst, bv, bo);
     Status r = timed(d, st, [&] {
-      const cudaError_t e = launch_slab_sweep2(s, m, t, (int)d.G.l[0], (int)d.G.l[1], a, b, d.kernel_alpha, sms,
-                                               S(st), &maps);
+      const Geometry& G = d.G;
+      const cudaError_t e =
+          band ? launch_heat2_band_slab(bv[0], bv[1], bo[0], bo[1], (int)G.t[1], (int)G.t[2], (int)G.n[1],
+                                        (int)G.l[2], a, b, d.kernel_alpha, S(st))
+               : launch_slab_sweep2(s, m, t, (int)G.l[0], (int)G.l[1], a, b, d.kernel_alpha, sms, S(st), &maps);
       if (e == cudaErrorNotSupported) {
         fused = false;
         cudaGetLastError();

@@ -217,6 +217,21 @@ bool band2_maps_encode(Band2Maps* m, const double* base, int tx, int ty, int tz,
 // array the maps were encoded over
 cudaError_t launch_heat2_band(const Band2Maps& maps, double* dst, int ty, int tz, int nty, int ntz, double alpha,
                               cudaStream_t s);
+// the wavefront's two-level pass (slab_sweep2 semantics) on the band layout:
+// views read through TMA (a tile-blocked array, planes mod nz when wrap, and
+// nlo scratch tile layers for planes < 0) and written directly
+struct Band2View {
+  Band2Maps main, scr;
+  int nlo, wrap;
+};
+struct Band2Out {
+  double* base;
+  double* hlo;
+  int nlo;
+};
+cudaError_t launch_heat2_band_slab(const Band2View& src, const Band2View& mid, const Band2Out& mido,
+                                   const Band2Out& dsto, int ty, int tz, int nty, int nz, int a, int b, double alpha,
+                                   cudaStream_t s);
 // device -> mapped pinned host rows copied by the SMs (pitches, len in doubles;
 // len and pitches even)
 cudaError_t launch_push_rows(const double* src, int64_t src_pitch, double* dst, int64_t dst_pitch, int64_t rows,

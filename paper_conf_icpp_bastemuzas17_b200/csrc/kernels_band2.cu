@@ -209,6 +209,203 @@ __global__ void __launch_bounds__(b2::NT, 1)
   }
 }
 
+// ---- the wavefront's two-level pass on the same band layout (heat2_band_slab):
+// level s on planes [a, b) from view src (level s-1), only its top two
+// planes b-2, b-1 written to view mid, whose planes a-2, a-1 it reads; level
+// s+1 on [a-1, b-1) into view dst (the semantics of slab_sweep2, DESIGN.md
+// §5). Staged planes, in order: mid a-2, mid a-1 (level s, rows y0-1 ..
+// y0+4 go straight to the level-s registers), then src a-1 .. b. Views are a
+// tile-blocked array (planes mod nz when wrapped: the resident level 0) plus
+// nlo scratch tile layers holding planes [-nlo*tz, 0).
+static __device__ __forceinline__ void b2_coords(const Band2View& v, int z, int tz, int nz, const TensorMapBlob*& m4,
+                                                 const TensorMapBlob*& m2, int& zl, int& zt) {
+  if (z < 0 && v.nlo > 0) {
+    const int q = z + v.nlo * tz;
+    m4 = &v.scr.m4, m2 = &v.scr.m2, zl = q % tz, zt = q / tz;
+  } else {
+    if (v.wrap) z = ((z % nz) + nz) % nz;
+    m4 = &v.main.m4, m2 = &v.main.m2, zl = z % tz, zt = z / tz;
+  }
+}
+static __device__ __forceinline__ double* b2_plane(const Band2Out& o, int z, int tz, int nty, int64_t te) {
+  // first element of plane z of tile layer/row 0, tile column 0
+  if (z < 0) {
+    const int q = z + o.nlo * tz;
+    return o.hlo + (int64_t)(q / tz) * nty * b2::NW * te + (int64_t)(q % tz) * (te / tz);
+  }
+  return o.base + (int64_t)(z / tz) * nty * b2::NW * te + (int64_t)(z % tz) * (te / tz);
+}
+
+__global__ void __launch_bounds__(b2::NT, 1)
+    heat2_band_slab(const __grid_constant__ Band2View src, const __grid_constant__ Band2View mid, const Band2Out mido,
+                    const Band2Out dsto, const int ty, const int tz, const int nty, const int nz, const int64_t te,
+                    const int a, const int b, const double alpha) {
+  using namespace b2;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double* stage = reinterpret_cast<double*>(smem_raw);
+  double* edge = stage + (size_t)S * STAGE;
+  uint64_t* full = reinterpret_cast<uint64_t*>(edge + 3 * ESLOT);
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) mbar_init(&full[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  const int ny = nty * ty;
+  const int y0 = (int)blockIdx.x * BY;
+  const int nq = b - a + 4;  // staged planes: mid a-2, a-1, src a-1 .. b
+  const int ya = (y0 - 2 + ny) % ny, yc = (y0 + 4) % ny;
+  const int ta = ya / ty, la = ya % ty, tb = y0 / ty, lb = y0 % ty, tc = yc / ty, lc = yc % ty;
+  int qn = 0, qs = 0;  // thread 0: next staged index, its slot
+  auto issue = [&]() {
+    const bool m = qn < 2;
+    const int z = m ? a - 2 + qn : a - 1 + (qn - 2);
+    const TensorMapBlob *m4, *m2;
+    int zl, zt;
+    b2_coords(m ? mid : src, z, tz, nz, m4, m2, zl, zt);
+    double* d = stage + (size_t)qs * STAGE;
+    fence_proxy_async();
+    mbar_expect_tx(&full[qs], BYTES);
+    tma_5d(d + OFF_A, m2, 0, la, 0, zl, zt * nty + ta, &full[qs]);
+    tma_5d(d + OFF_B, m4, 0, lb, 0, zl, zt * nty + tb, &full[qs]);
+    tma_5d(d + OFF_C, m2, 0, lc, 0, zl, zt * nty + tc, &full[qs]);
+    ++qn;
+    qs = qs + 1 == S ? 0 : qs + 1;
+  };
+  if (threadIdx.x == 0) {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    while (qn < S && qn < nq) issue();
+  }
+
+  const int t = (int)threadIdx.x, lane = t & 31, w = t >> 5;
+  const int x = 2 * lane;
+  const bool right = lane == 31;
+  const int we = right ? (w + 1) % NW : (w + NW - 1) % NW, xe = right ? 0 : TX - 1;
+  const int e_mine = right ? (w * 2 + 1) * ER : w * 2 * ER;
+  const int e_nbr = right ? ((w + 1) % NW) * 2 * ER : (((w + NW - 1) % NW) * 2 + 1) * ER;
+  const uint32_t is_left = lane == 0, is_right = right;
+  const int64_t oxy = (int64_t)(tb * NW + w) * te + (int64_t)lb * TX + x;  // band row y0, this lane's x, in a plane
+  auto wait_q = [&](int q) { mbar_wait(&full[q % S], (q / S) & 1); };
+  auto ld2 = [&](const double* st, int i) { return *reinterpret_cast<const double2*>(st + srow(i, w) + x); };
+
+  double2 a_[3][8], b_[3][6];
+  wait_q(0);
+#pragma unroll
+  for (int r = 0; r < 6; ++r) b_[0][r] = ld2(stage, r + 1);   // level s, plane a-2
+  wait_q(1);
+#pragma unroll
+  for (int r = 0; r < 6; ++r) b_[1][r] = ld2(stage + (size_t)STAGE, r + 1);  // level s, plane a-1
+  {
+    const uint32_t ez = smem_u32(edge + (size_t)2 * ESLOT + e_mine);  // its edges: slot of it - 1 at it = 0
+#pragma unroll
+    for (int r = 0; r < 6; ++r) {
+      sts_if(ez + 8 * r, b_[1][r].x, is_left);
+      sts_if(ez + 8 * r, b_[1][r].y, is_right);
+    }
+  }
+  wait_q(2);
+#pragma unroll
+  for (int i = 0; i < 8; ++i) a_[0][i] = ld2(stage + (size_t)(2 % S) * STAGE, i);  // src a-1
+  wait_q(3);
+#pragma unroll
+  for (int i = 0; i < 8; ++i) a_[1][i] = ld2(stage + (size_t)(3 % S) * STAGE, i);  // src a
+  bar_consumers_b2();  // plane a-1's edges written; staged 0..2 consumed
+  if (t == 0)
+    while (qn < nq && qn <= 2 + S) issue();
+  int sq = 4 % S, sq1 = 3 % S;  // slots of staged q = it + 4 (src p+1) and q - 1 (src p)
+  int e0 = 0, e1 = 2;
+  auto step = [&](int it, auto kc) {
+    constexpr int K = decltype(kc)::value;
+    constexpr int P0 = K, P1 = (K + 1) % 3, P2 = (K + 2) % 3;
+    const int p = a + it, q = it + 4;
+    wait_q(q);
+    const double* sz = stage + (size_t)sq1 * STAGE;
+    const double* sp = stage + (size_t)sq * STAGE;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) a_[P2][i] = ld2(sp, i);
+#pragma unroll
+    for (int r = 0; r < 6; ++r) {  // level s at p, row y0-1+r
+      const double2 c = a_[P1][r + 1];
+      double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+      double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+      const uint32_t ea = smem_u32(sz + srow(r + 1, we) + xe);
+      lds_if(xm, ea, is_left);
+      lds_if(xp, ea, is_right);
+      b_[P2][r].x = heat_update(c.x, xm, c.y, a_[P1][r].x, a_[P1][r + 2].x, a_[P0][r + 1].x, a_[P2][r + 1].x, alpha);
+      b_[P2][r].y = heat_update(c.y, c.x, xp, a_[P1][r].y, a_[P1][r + 2].y, a_[P0][r + 1].y, a_[P2][r + 1].y, alpha);
+    }
+    {  // level s+1 at p - 1, rows y0 .. y0+3
+      const double* em = edge + (size_t)e1 * ESLOT + e_nbr;
+      double* o = b2_plane(dsto, p - 1, tz, nty, te) + oxy;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const double2 c = b_[P1][j + 1];
+        double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+        double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+        lds_if(xm, smem_u32(em + j + 1), is_left);
+        lds_if(xp, smem_u32(em + j + 1), is_right);
+        double2 v;
+        v.x = heat_update(c.x, xm, c.y, b_[P1][j].x, b_[P1][j + 2].x, b_[P0][j + 1].x, b_[P2][j + 1].x, alpha);
+        v.y = heat_update(c.y, c.x, xp, b_[P1][j].y, b_[P1][j + 2].y, b_[P0][j + 1].y, b_[P2][j + 1].y, alpha);
+        *reinterpret_cast<double2*>(o + j * TX) = v;
+      }
+    }
+    if (p >= b - 2) {  // level s's top two planes, this band's rows, to mid
+      double* o = b2_plane(mido, p, tz, nty, te) + oxy;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) *reinterpret_cast<double2*>(o + j * TX) = b_[P2][j + 1];
+    }
+    {
+      const uint32_t ez = smem_u32(edge + (size_t)e0 * ESLOT + e_mine);
+#pragma unroll
+      for (int r = 0; r < 6; ++r) {
+        sts_if(ez + 8 * r, b_[P2][r].x, is_left);
+        sts_if(ez + 8 * r, b_[P2][r].y, is_right);
+      }
+    }
+    bar_consumers_b2();
+    if (t == 0)
+      while (qn < nq && qn <= q - 1 + S) issue();
+    sq1 = sq;
+    sq = sq + 1 == S ? 0 : sq + 1;
+    e1 = e0;
+    e0 = e0 == 2 ? 0 : e0 + 1;
+  };
+  const int nit = b - a;
+  for (int it = 0; it < nit; it += 3) {
+    step(it, std::integral_constant<int, 0>{});
+    if (it + 1 >= nit) break;
+    step(it + 1, std::integral_constant<int, 1>{});
+    if (it + 2 >= nit) break;
+    step(it + 2, std::integral_constant<int, 2>{});
+  }
+}
+
+cudaError_t launch_heat2_band_slab(const Band2View& src, const Band2View& mid, const Band2Out& mido,
+                                   const Band2Out& dsto, int ty, int tz, int nty, int nz, int a, int b, double alpha,
+                                   cudaStream_t s) {
+  using namespace b2;
+  if (b - a < 2) return cudaErrorNotSupported;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(heat2_band_slab, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(nty * ty / BY));
+  cfg.blockDim = dim3(NT);
+  cfg.dynamicSmemBytes = SMEM;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, heat2_band_slab, src, mid, mido, dsto, ty, tz, nty, nz, (int64_t)TX * ty * tz, a,
+                            b, alpha);
+}
+
 // driver entry point for cuTensorMapEncodeTiled (no -lcuda link dependency)
 using EncodeTiledFn5 = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                     const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,

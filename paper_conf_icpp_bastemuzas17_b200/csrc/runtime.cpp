@@ -1315,11 +1315,14 @@ static bool wavefront_ok(const Domain& d, int T, WavePlan* wp) {
   const int64_t B = (2 * (int64_t)T + c - 1) / c * c;
   if (B + c > nz) return false;  // the seam's cone would cover the ring
   const int64_t nlo = (2 * (int64_t)T + tz - 1) / tz;
-  // two levels per pass (wavefront = 2) take a third level array (ntiles
-  // slots) and three scratch parities, when the budget has them
+  // two levels per pass take a third level array (ntiles slots) and three
+  // scratch parities, when the budget has them: by default where the band
+  // kernel runs them (heat2_band_slab: grids 512 wide), with wavefront = 2
+  // everywhere (slab_sweep2_tile elsewhere), never with wavefront = 3
   const uint64_t avail = d.budget_left + (uint64_t)d.wave_slots * G.tile_elems * 8;
   const int64_t slots3 = G.ntiles + 3 * nlo * G.layer_tiles, slots2 = 2 * nlo * G.layer_tiles;
-  wp->fused = d.opt.wavefront == 2 && T >= 2 &&
+  const bool band = band2_shape_ok(G.l[0], G.l[1], (int)G.t[0], (int)G.t[1]) && d.exec->band2_ok(const_cast<Domain&>(d));
+  wp->fused = (d.opt.wavefront == 2 || (d.opt.wavefront != 3 && band)) && T >= 2 &&
               (d.wave_slots >= slots3 || (uint64_t)slots3 * G.tile_elems * 8 <= avail);
   const int64_t need_slots = wp->fused ? slots3 : slots2;
   if (d.wave_slots < need_slots && (uint64_t)need_slots * G.tile_elems * 8 > avail) return false;
@@ -1332,7 +1335,7 @@ static bool wavefront_ok(const Domain& d, int T, WavePlan* wp) {
   // by its T sweeps per plane; one chunk of fill/drain
   // (the bootstrap's sweeps are thick, about 0.7 of a chunk sweep's cost per
   // plane, fitted on the Fig. 5 sweep at T = 64 and 100)
-  const double rm = wp->fused ? 0.6 * r : r;  // two levels per pass: ~0.6 of the sweep time per level
+  const double rm = wp->fused ? 0.6 * r : r;  // two levels per pass: ~0.6 of the sweep time per level (C2: 0.6)
   wp->est = (double)B + 0.7 * r * Td * Td + std::max(n, rm * n * Td) + (double)c * (1.0 + rm * Td);
   return true;
 }

@@ -408,16 +408,20 @@ def test_stream_through_bit_exact(dims, td, T):
 
 @pytest.mark.parametrize("dims,td,T", [((64, 32, 128), (32, 16, 16), 20), ((128, 64, 256), (64, 64, 32), 48),
                                        ((64, 64, 64), (32, 32, 8), 7), ((96, 64, 160), (32, 32, 32), 1),
-                                       ((64, 32, 512), (32, 32, 64), 100), ((512, 64, 128), (64, 64, 64), 16)])
-@pytest.mark.parametrize("wave", [1, 2])
+                                       ((64, 32, 512), (32, 32, 64), 100), ((512, 64, 128), (64, 64, 64), 16),
+                                       ((512, 32, 256), (64, 32, 32), 20), ((512, 64, 384), (64, 64, 64), 48),
+                                       ((512, 16, 512), (64, 16, 64), 100)])
+@pytest.mark.parametrize("wave", [1, 2, 3])
 def test_wavefront_bit_exact(dims, td, T, wave):
     """Fresh-upload runs on the time-skewed wavefront (forced): chunks of
     planes, level s of chunk i on planes [c*i - s, c*i + c - s), the seam's
     bootstrap trapezoid in the scratch layers, each chunk's final planes
     back to the host as soon as it ends; the host result, the kept device
     copy (a following resident run) and a second wavefront run are exact,
-    and every cell crossed the link once per direction. wave = 1: one level
-    per pass (slab_sweep_tile); 2: two levels per pass (slab_sweep2_tile)."""
+    and every cell crossed the link once per direction. wave = 1: the default
+    (two levels per pass on grids 512 wide, heat2_band_slab); 2: two levels
+    per pass everywhere (slab_sweep2_tile off the band shape); 3: one level
+    per pass (slab_sweep_tile)."""
     nx, ny, nz = dims
     u0 = synth.uniform_grid(nx, ny, nz, 42)
     with T_.Domain(dims, td, wavefront=wave) as d:

@@ -589,6 +589,19 @@ def test_wavefront_schedule_replays_to_oracle(dims, td, T, ns, runs_after):
     assert planes3 == planes
 
 
+@pytest.mark.parametrize("T_", [5, 20])
+def test_wavefront_512_wide_default_two_levels(T_):
+    """On grids 512 wide with 64-wide tiles the wavefront runs two levels per
+    pass by default (heat2_band_slab on the GPU); wavefront = 3 keeps one
+    level per pass. Both replay to the oracle bit-exactly."""
+    dims, td = (512, 8, 128), (64, 4, 16)
+    d = _run_and_replay(dims, td, [T_, 2], 2, seeds=(0, 1), wavefront=1)
+    d1 = T_run_dry(dims, td, T_, 2, wavefront=1)
+    assert "wsweep2" in [op[0] for op in d1.trace()]
+    d3 = _run_and_replay(dims, td, [T_], 2, seeds=(2,), wavefront=3)
+    assert "wsweep2" not in [op[0] for op in d3.trace()] and d3.get_info()["last_schedule"] == 6
+
+
 def T_run_dry(dims, td, steps, ns, **kw):
     d = T.Domain(dims, td, dry_run=True, **kw)
     d.load(np.zeros(dims[::-1]))
@@ -622,10 +635,13 @@ def test_cost_model_ratio_option_and_report():
     d = T.Domain(dims, td, dry_run=True)
     assert abs(d.get_info()["sweep_link_ratio"] - 0.021) < 1e-12
     got = {}
-    for r in (0.005, 0.021, 0.5):
+    # (at C2's shape both the wavefront and the batched middle steps run two
+    # levels per kernel, so only a much slower sweep tips T = 32 to batched:
+    # the wavefront's T^2 seam bootstrap then dominates)
+    for r in (0.005, 0.021, 5.0):
         d = T.Domain(dims, td, dry_run=True, sweep_link_ratio=r)
         assert d.get_info()["sweep_link_ratio"] == r
         d.invalidate()
         d.run(T.heat7(ALPHA), 32, 4)
         got[r] = d.get_info()["last_schedule"]
-    assert got[0.005] in (2, 6) and got[0.021] == 6 and got[0.5] == 1
+    assert got[0.005] in (2, 6) and got[0.021] == 6 and got[5.0] == 1
