@@ -694,7 +694,12 @@ def run_fig5_leg(args):
         r["speedup_sync_vs_sync_pageable"] = r["sync_pageable"]["ms"] / r["sync"]["ms"]
         t_dep = cells * 8 / (bw["h2d"] * 1e9) + cells * 8 / (bw["d2h"] * 1e9)
         t_duplex = max(cells * 8 / (bw["h2d"] * 1e9), cells * 8 / (bw["d2h"] * 1e9), 2 * cells * 8 / (bidir * 1e9))
-        t_hbm = int(T) * 16 * cells / (hbm * 1e9)
+        # HBM at the schedule's algorithmic bytes: 8 B per cell-step where two
+        # steps run per pass (heat2_band / heat2_band_slab, grids 512 wide),
+        # else 16 B (the one-step figure is reported beside it)
+        two_level = n == 512 and td[0] == 64 and int(T) >= 2
+        t_hbm1 = int(T) * 16 * cells / (hbm * 1e9)
+        t_hbm = t_hbm1 / 2 if two_level else t_hbm1
         # a cell after T steps depends on the initial planes within T of it, so
         # no schedule returns a final plane before 2T+1 planes have crossed
         # H2D (solo rate), and the whole grid must then still cross D2H
@@ -702,7 +707,9 @@ def run_fig5_leg(args):
         t_cone = min(2 * int(T) + 1, n) * plane_b / (bw["h2d"] * 1e9)
         t_causal = t_cone + cells * 8 / (bw["d2h"] * 1e9)
         r["roofline_ms"] = {"t_link_dependency": t_dep * 1e3, "t_link_duplex": t_duplex * 1e3,
-                            "t_hbm": t_hbm * 1e3, "bound_ms": max(t_duplex, t_hbm) * 1e3,
+                            "t_hbm": t_hbm * 1e3, "t_hbm_one_step_per_pass": t_hbm1 * 1e3,
+                            "hbm_bytes_per_cell_step": 8 if two_level else 16,
+                            "bound_ms": max(t_duplex, t_hbm) * 1e3,
                             "t_cone_then_d2h": t_causal * 1e3,
                             "bound_causal_ms": max(t_duplex, t_hbm, t_causal) * 1e3,
                             "serial_ms": (t_dep + t_hbm) * 1e3}
