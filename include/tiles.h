@@ -310,9 +310,12 @@ typedef enum {
                             view b only at planes hi-2, hi-1 (its planes lo-2, lo-1 are read
                             from b); d = scratch layers. Views coded as for TILE_OP_WSWEEP */
   TILE_OP_WSWEEP2_DST = 30,/* the same kernel: level s+1 on [lo-1, hi-1) into view a */
-  TILE_OP_BAND2 = 31     /* two steps of the whole resident periodic grid in one kernel
+  TILE_OP_BAND2 = 31,    /* two steps of the whole resident periodic grid in one kernel
                             (heat2_band): view a (the resident array, coded as for
                             TILE_OP_WSWEEP) -> view b; c = 0 | nz << 32 */
+  TILE_OP_SWEEP2S = 32   /* stream-through, two sweeps in one kernel (heat2_band_slab):
+                            operands as TILE_OP_SWEEP; level 1 on [lo, hi) stays on
+                            chip, level 2 on [lo+1, hi-1) is written to b */
 } tile_op_kind;
 
 typedef struct {

@@ -456,63 +456,97 @@ struct CudaExec final : Exec {
   Band2Maps bmaps[2];
   int bmaps_state = 0;  // 0 not tried, 1 encoded, -1 not available
   // tensor maps of other tile-blocked regions (wavefront level arrays and
-  // scratch layers), by base pointer and tile layers
+  // scratch layers, stream-through slabs), by base pointer, tile depth and
+  // tile layers
   struct MapEntry {
     const double* base;
-    int layers;
+    int tz, layers;
     bool ok;
     Band2Maps m;
   };
   std::vector<MapEntry> band_maps;
-  const Band2Maps* band_maps_for(Domain& d, const double* base, int layers) {
+  bool band_maps_for(Domain& d, const double* base, int tz, int layers, Band2Maps* out) {
     for (auto& e : band_maps)
-      if (e.base == base && e.layers == layers) return e.ok ? &e.m : nullptr;
+      if (e.base == base && e.tz == tz && e.layers == layers) {
+        if (e.ok) *out = e.m;
+        return e.ok;
+      }
     const Geometry& G = d.G;
-    MapEntry e{base, layers, false, {}};
-    e.ok = band2_maps_encode(&e.m, base, (int)G.t[0], (int)G.t[1], (int)G.t[2], (int)G.n[0], (int)G.n[1], layers);
+    MapEntry e{base, tz, layers, false, {}};
+    e.ok = band2_maps_encode(&e.m, base, (int)G.t[0], (int)G.t[1], tz, (int)G.n[0], (int)G.n[1], layers);
     band_maps.push_back(e);
-    return e.ok ? &band_maps.back().m : nullptr;
+    if (e.ok) *out = e.m;
+    return e.ok;
   }
-  // the views of a two-level pass as heat2_band_slab descriptors (RESIDENT:
-  // wrapped array; WAVE: array + scratch layers); false if any does not fit
-  bool band2_slab_views(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, Band2View* bv,
-                        Band2Out* bo) {
+  bool band2_slab_on(Domain& d) {
     static const int on = [] {
       const char* e = getenv("TILES_BAND2_SLAB");
       return e ? atoi(e) : 1;
     }();
     const Geometry& G = d.G;
-    if (!on || G.nranks != 1 || !band2_shape_ok(G.l[0], G.l[1], (int)G.t[0], (int)G.t[1])) return false;
-    auto in = [&](const SlabRef& r, Band2View* v) {
-      const Band2Maps* mm = nullptr;
-      v->nlo = 0;
-      v->wrap = r.kind == SlabRef::RESIDENT;
-      // (each map is copied out before the next lookup: the cache may grow)
-      if (r.kind == SlabRef::RESIDENT) {
-        mm = band_maps_for(d, d.slot_ptr(r.slot ? (int)G.ntiles : 0), (int)G.n[2]);
-        if (!mm) return false;
-        v->main = *mm;
-      } else if (r.kind == SlabRef::WAVE) {
-        mm = band_maps_for(d, d.slot_ptr(r.slot), (int)G.n[2]);
-        if (!mm) return false;
-        v->main = *mm;
-        mm = band_maps_for(d, d.slot_ptr(r.ring[0]), (int)r.un);
-        if (!mm) return false;
-        v->scr = *mm;
-        v->nlo = (int)r.un;
-      } else {
-        return false;
-      }
-      return true;
-    };
-    auto out = [&](const SlabRef& r, Band2Out* o) {
-      if (r.kind != SlabRef::WAVE) return false;
-      o->base = d.slot_ptr(r.slot);
+    return on && G.nranks == 1 && band2_shape_ok(G.l[0], G.l[1], (int)G.t[0], (int)G.t[1]);
+  }
+  // a view read by heat2_band_slab: RESIDENT (wrapped, plane offset zbase),
+  // WAVE (level array + scratch layers), DENSE (one layer of slab_depth)
+  bool band2_in(Domain& d, const SlabRef& r, Band2View* v) {
+    const Geometry& G = d.G;
+    v->nlo = 0;
+    v->wrap = r.kind == SlabRef::RESIDENT;
+    v->zbase = 0;
+    v->nz = (int)G.l[2];
+    v->tz = (int)G.t[2];
+    if (r.kind == SlabRef::RESIDENT) {
+      v->zbase = (int)r.zbase;
+      return band_maps_for(d, d.slot_ptr(r.slot ? (int)G.ntiles : 0), v->tz, (int)G.n[2], &v->main);
+    }
+    if (r.kind == SlabRef::WAVE) {
+      v->nlo = (int)r.un;
+      return band_maps_for(d, d.slot_ptr(r.slot), v->tz, (int)G.n[2], &v->main) &&
+             band_maps_for(d, d.slot_ptr(r.ring[0]), v->tz, (int)r.un, &v->scr);
+    }
+    if (r.kind == SlabRef::DENSE) {
+      v->tz = (int)d.slab_depth;
+      return band_maps_for(d, d.slot_ptr(r.slot), v->tz, 1, &v->main);
+    }
+    return false;
+  }
+  // a view written by heat2_band_slab; SUB: plane `first` -> sub-tile plane 0
+  bool band2_out(Domain& d, const SlabRef& r, int first, Band2Out* o) {
+    const Geometry& G = d.G;
+    o->base = d.slot_ptr(r.slot);
+    o->hlo = nullptr;
+    o->nlo = 0;
+    o->zbase = 0;
+    if (r.kind == SlabRef::WAVE) {
       o->hlo = d.slot_ptr(r.ring[0]);
       o->nlo = (int)r.un;
-      return true;
-    };
-    return in(src, &bv[0]) && in(mid, &bv[1]) && out(mid, &bo[0]) && out(dst, &bo[1]);
+      o->tz = (int)G.t[2];
+    } else if (r.kind == SlabRef::DENSE) {
+      o->tz = (int)d.slab_depth;
+    } else if (r.kind == SlabRef::SUB) {
+      o->tz = (int)d.st_unit;
+      o->zbase = -first;
+    } else {
+      return false;
+    }
+    o->te = (int64_t)o->tz * G.t[0] * G.t[1];
+    return true;
+  }
+  bool sweep2s_ok(Domain& d) override { return band2_slab_on(d); }
+  Status slab_sweep2s(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi, int st) override {
+    INJECT(FAULT_KERNEL, st);
+    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
+    Band2View bv;
+    Band2Out bo;
+    if (!band2_in(d, src, &bv) || !band2_out(d, dst, lo + 1, &bo))
+      return make_err(TILE_ESTATE, "internal: two-sweep pass on views without band maps");
+    next_cells = d.kernel_timing ? (uint64_t)(hi - lo) * d.G.l[0] * d.G.l[1] : 0;  // one pass over the cells
+    Status r = timed(d, st, [&] {
+      return launch_heat2_band_slab(0, bv, bv, bo, bo, (int)d.G.t[1], (int)d.G.n[1], lo, hi, d.kernel_alpha, S(st));
+    });
+    if (r.bad()) return r;
+    d.stats.n_kernels++;
+    return Status::ok();
   }
   bool band2_ok(Domain& d) override {
     if (bmaps_state == 0) {
@@ -553,12 +587,13 @@ struct CudaExec final : Exec {
     // view has its tensor maps; else the tile-column kernel
     Band2View bv[2];
     Band2Out bo[2];
-    const bool band = band2_slab_views(d, src, mid, dst, bv, bo);
+    const bool band = band2_slab_on(d) && band2_in(d, src, &bv[0]) && band2_in(d, mid, &bv[1]) &&
+                      band2_out(d, mid, 0, &bo[0]) && band2_out(d, dst, 0, &bo[1]);
     Status r = timed(d, st, [&] {
       const Geometry& G = d.G;
       const cudaError_t e =
-          band ? launch_heat2_band_slab(bv[0], bv[1], bo[0], bo[1], (int)G.t[1], (int)G.t[2], (int)G.n[1],
-                                        (int)G.l[2], a, b, d.kernel_alpha, S(st))
+          band ? launch_heat2_band_slab(1, bv[0], bv[1], bo[0], bo[1], (int)G.t[1], (int)G.n[1], a, b,
+                                        d.kernel_alpha, S(st))
                : launch_slab_sweep2(s, m, t, (int)G.l[0], (int)G.l[1], a, b, d.kernel_alpha, sms, S(st), &maps);
       if (e == cudaErrorNotSupported) {
         fused = false;

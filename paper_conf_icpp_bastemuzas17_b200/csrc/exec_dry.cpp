@@ -121,6 +121,21 @@ struct DryExec final : Exec {
     return Status::ok();
   }
   bool band2_ok(Domain&) override { return true; }
+  bool sweep2s_ok(Domain& d) override {
+    const Geometry& G = d.G;
+    return G.nranks == 1 && band2_shape_ok(G.l[0], G.l[1], (int)G.t[0], (int)G.t[1]);
+  }
+  Status slab_sweep2s(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi, int st) override {
+    if (Status f_ = inject(d, FAULT_KERNEL); f_.bad()) return f_;
+    d.stats.n_kernels++;
+    // codes as TILE_OP_SWEEP: a slab slot or -1-bit (resident, slab plane 0
+    // at z = d); b slab slot or -1-slot (packed sub-tiles from plane lo+1)
+    const int64_t a = src.kind == SlabRef::DENSE ? src.slot : -1 - (int64_t)src.slot;
+    const int64_t b = dst.kind == SlabRef::DENSE ? dst.slot : -1 - (int64_t)dst.slot;
+    put(d, TILE_OP_SWEEP2S, st, a, b, (int64_t)lo | ((int64_t)hi << 32),
+        src.kind == SlabRef::RESIDENT ? src.zbase : 0);
+    return Status::ok();
+  }
   Status band2(Domain& d, int sbit, int dbit, int st) override {
     if (Status f_ = inject(d, FAULT_KERNEL); f_.bad()) return f_;
     d.stats.n_kernels++;

@@ -217,20 +217,27 @@ bool band2_maps_encode(Band2Maps* m, const double* base, int tx, int ty, int tz,
 // array the maps were encoded over
 cudaError_t launch_heat2_band(const Band2Maps& maps, double* dst, int ty, int tz, int nty, int ntz, double alpha,
                               cudaStream_t s);
-// the wavefront's two-level pass (slab_sweep2 semantics) on the band layout:
-// views read through TMA (a tile-blocked array, planes mod nz when wrap, and
-// nlo scratch tile layers for planes < 0) and written directly
+// two-level passes on the band layout over general views (heat2_band_slab):
+// a view is a tile-blocked region (tiles of tz planes, `layers` tile layers;
+// plane z of the view is region plane z + zbase, taken mod nz when wrap)
+// plus nlo scratch tile layers for region planes < 0. Inputs go through TMA
+// (maps encoded over the region / the scratch), outputs are written directly.
 struct Band2View {
   Band2Maps main, scr;
-  int nlo, wrap;
+  int nlo, wrap, tz, zbase, nz;
 };
 struct Band2Out {
   double* base;
   double* hlo;
-  int nlo;
+  int64_t te;  // elements per tile
+  int nlo, tz, zbase;
 };
-cudaError_t launch_heat2_band_slab(const Band2View& src, const Band2View& mid, const Band2Out& mido,
-                                   const Band2Out& dsto, int ty, int tz, int nty, int nz, int a, int b, double alpha,
+// mid = 1 (the wavefront, slab_sweep2 semantics): level s on [a, b) from
+// src, its planes b-2, b-1 written to mid (whose planes a-2, a-1 it reads),
+// level s+1 on [a-1, b-1) into dst. mid = 0 (stream-through): level s on
+// [a, b) from src kept on chip, level s+1 on [a+1, b-1) into dst.
+cudaError_t launch_heat2_band_slab(int mid_mode, const Band2View& src, const Band2View& mid, const Band2Out& mido,
+                                   const Band2Out& dsto, int ty, int nty, int a, int b, double alpha,
                                    cudaStream_t s);
 // device -> mapped pinned host rows copied by the SMs (pitches, len in doubles;
 // len and pitches even)

@@ -209,37 +209,38 @@ __global__ void __launch_bounds__(b2::NT, 1)
   }
 }
 
-// ---- the wavefront's two-level pass on the same band layout (heat2_band_slab):
-// level s on planes [a, b) from view src (level s-1), only its top two
-// planes b-2, b-1 written to view mid, whose planes a-2, a-1 it reads; level
-// s+1 on [a-1, b-1) into view dst (the semantics of slab_sweep2, DESIGN.md
-// §5). Staged planes, in order: mid a-2, mid a-1 (level s, rows y0-1 ..
-// y0+4 go straight to the level-s registers), then src a-1 .. b. Views are a
-// tile-blocked array (planes mod nz when wrapped: the resident level 0) plus
-// nlo scratch tile layers holding planes [-nlo*tz, 0).
-static __device__ __forceinline__ void b2_coords(const Band2View& v, int z, int tz, int nz, const TensorMapBlob*& m4,
+// ---- two-level passes over general views on the same band layout
+// (heat2_band_slab). MID (the wavefront, slab_sweep2 semantics): level s on
+// planes [a, b) from view src (level s-1), only its top two planes b-2, b-1
+// written to view mid, whose planes a-2, a-1 it reads; level s+1 on
+// [a-1, b-1) into view dst. Staged planes, in order: mid a-2, mid a-1 (rows
+// y0-1 .. y0+4 go straight to the level-s registers), then src a-1 .. b.
+// SHRINK (two sweeps of the stream-through): level s on [a, b) from src,
+// kept on chip; level s+1 on [a+1, b-1) into dst; staged src a-1 .. b.
+static __device__ __forceinline__ void b2_coords(const Band2View& v, int z, const TensorMapBlob*& m4,
                                                  const TensorMapBlob*& m2, int& zl, int& zt) {
+  z += v.zbase;
   if (z < 0 && v.nlo > 0) {
-    const int q = z + v.nlo * tz;
-    m4 = &v.scr.m4, m2 = &v.scr.m2, zl = q % tz, zt = q / tz;
+    const int q = z + v.nlo * v.tz;
+    m4 = &v.scr.m4, m2 = &v.scr.m2, zl = q % v.tz, zt = q / v.tz;
   } else {
-    if (v.wrap) z = ((z % nz) + nz) % nz;
-    m4 = &v.main.m4, m2 = &v.main.m2, zl = z % tz, zt = z / tz;
+    if (v.wrap) z = ((z % v.nz) + v.nz) % v.nz;
+    m4 = &v.main.m4, m2 = &v.main.m2, zl = z % v.tz, zt = z / v.tz;
   }
 }
-static __device__ __forceinline__ double* b2_plane(const Band2Out& o, int z, int tz, int nty, int64_t te) {
-  // first element of plane z of tile layer/row 0, tile column 0
-  if (z < 0) {
-    const int q = z + o.nlo * tz;
-    return o.hlo + (int64_t)(q / tz) * nty * b2::NW * te + (int64_t)(q % tz) * (te / tz);
-  }
-  return o.base + (int64_t)(z / tz) * nty * b2::NW * te + (int64_t)(z % tz) * (te / tz);
+// first element of view plane z in tile (tile row ty_i, tile column w)
+static __device__ __forceinline__ double* b2_plane(const Band2Out& o, int z, int nty, int tyi, int w, int ty) {
+  z += o.zbase;
+  double* base = o.base;
+  if (z < 0) base = o.hlo, z += o.nlo * o.tz;
+  return base + ((int64_t)(z / o.tz) * nty * b2::NW + (int64_t)tyi * b2::NW + w) * o.te +
+         (int64_t)(z % o.tz) * ty * b2::TX;
 }
 
+template <bool MID>
 __global__ void __launch_bounds__(b2::NT, 1)
     heat2_band_slab(const __grid_constant__ Band2View src, const __grid_constant__ Band2View mid, const Band2Out mido,
-                    const Band2Out dsto, const int ty, const int tz, const int nty, const int nz, const int64_t te,
-                    const int a, const int b, const double alpha) {
+                    const Band2Out dsto, const int ty, const int nty, const int a, const int b, const double alpha) {
   using namespace b2;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   double* stage = reinterpret_cast<double*>(smem_raw);
@@ -253,16 +254,17 @@ __global__ void __launch_bounds__(b2::NT, 1)
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   const int ny = nty * ty;
   const int y0 = (int)blockIdx.x * BY;
-  const int nq = b - a + 4;  // staged planes: mid a-2, a-1, src a-1 .. b
+  constexpr int NM = MID ? 2 : 0;  // staged mid planes
+  const int nq = NM + b - a + 2;   // staged planes: [mid a-2, a-1,] src a-1 .. b
   const int ya = (y0 - 2 + ny) % ny, yc = (y0 + 4) % ny;
   const int ta = ya / ty, la = ya % ty, tb = y0 / ty, lb = y0 % ty, tc = yc / ty, lc = yc % ty;
   int qn = 0, qs = 0;  // thread 0: next staged index, its slot
   auto issue = [&]() {
-    const bool m = qn < 2;
-    const int z = m ? a - 2 + qn : a - 1 + (qn - 2);
+    const bool m = qn < NM;
+    const int z = m ? a - 2 + qn : a - 1 + (qn - NM);
     const TensorMapBlob *m4, *m2;
     int zl, zt;
-    b2_coords(m ? mid : src, z, tz, nz, m4, m2, zl, zt);
+    b2_coords(m ? mid : src, z, m4, m2, zl, zt);
     double* d = stage + (size_t)qs * STAGE;
     fence_proxy_async();
     mbar_expect_tx(&full[qs], BYTES);
@@ -284,40 +286,45 @@ __global__ void __launch_bounds__(b2::NT, 1)
   const int e_mine = right ? (w * 2 + 1) * ER : w * 2 * ER;
   const int e_nbr = right ? ((w + 1) % NW) * 2 * ER : (((w + NW - 1) % NW) * 2 + 1) * ER;
   const uint32_t is_left = lane == 0, is_right = right;
-  const int64_t oxy = (int64_t)(tb * NW + w) * te + (int64_t)lb * TX + x;  // band row y0, this lane's x, in a plane
+  const int oyx = lb * TX + x;  // this lane's first output cell in a tile plane
   auto wait_q = [&](int q) { mbar_wait(&full[q % S], (q / S) & 1); };
   auto ld2 = [&](const double* st, int i) { return *reinterpret_cast<const double2*>(st + srow(i, w) + x); };
 
   double2 a_[3][8], b_[3][6];
-  wait_q(0);
+  if (MID) {
+    wait_q(0);
 #pragma unroll
-  for (int r = 0; r < 6; ++r) b_[0][r] = ld2(stage, r + 1);   // level s, plane a-2
-  wait_q(1);
+    for (int r = 0; r < 6; ++r) b_[0][r] = ld2(stage, r + 1);   // level s, plane a-2
+    wait_q(1);
 #pragma unroll
-  for (int r = 0; r < 6; ++r) b_[1][r] = ld2(stage + (size_t)STAGE, r + 1);  // level s, plane a-1
-  {
+    for (int r = 0; r < 6; ++r) b_[1][r] = ld2(stage + (size_t)STAGE, r + 1);  // level s, plane a-1
     const uint32_t ez = smem_u32(edge + (size_t)2 * ESLOT + e_mine);  // its edges: slot of it - 1 at it = 0
 #pragma unroll
     for (int r = 0; r < 6; ++r) {
       sts_if(ez + 8 * r, b_[1][r].x, is_left);
       sts_if(ez + 8 * r, b_[1][r].y, is_right);
     }
+  } else {
+#pragma unroll
+    for (int k = 0; k < 2; ++k)
+#pragma unroll
+      for (int r = 0; r < 6; ++r) b_[k][r] = make_double2(0.0, 0.0);
   }
-  wait_q(2);
+  wait_q(NM);
 #pragma unroll
-  for (int i = 0; i < 8; ++i) a_[0][i] = ld2(stage + (size_t)(2 % S) * STAGE, i);  // src a-1
-  wait_q(3);
+  for (int i = 0; i < 8; ++i) a_[0][i] = ld2(stage + (size_t)(NM % S) * STAGE, i);  // src a-1
+  wait_q(NM + 1);
 #pragma unroll
-  for (int i = 0; i < 8; ++i) a_[1][i] = ld2(stage + (size_t)(3 % S) * STAGE, i);  // src a
-  bar_consumers_b2();  // plane a-1's edges written; staged 0..2 consumed
+  for (int i = 0; i < 8; ++i) a_[1][i] = ld2(stage + (size_t)((NM + 1) % S) * STAGE, i);  // src a
+  bar_consumers_b2();  // (MID: plane a-1's edges written); staged 0 .. NM consumed
   if (t == 0)
-    while (qn < nq && qn <= 2 + S) issue();
-  int sq = 4 % S, sq1 = 3 % S;  // slots of staged q = it + 4 (src p+1) and q - 1 (src p)
+    while (qn < nq && qn <= NM + S) issue();
+  int sq = (NM + 2) % S, sq1 = (NM + 1) % S;  // slots of staged src p+1 and src p
   int e0 = 0, e1 = 2;
   auto step = [&](int it, auto kc) {
     constexpr int K = decltype(kc)::value;
     constexpr int P0 = K, P1 = (K + 1) % 3, P2 = (K + 2) % 3;
-    const int p = a + it, q = it + 4;
+    const int p = a + it, q = it + NM + 2;
     wait_q(q);
     const double* sz = stage + (size_t)sq1 * STAGE;
     const double* sp = stage + (size_t)sq * STAGE;
@@ -334,9 +341,9 @@ __global__ void __launch_bounds__(b2::NT, 1)
       b_[P2][r].x = heat_update(c.x, xm, c.y, a_[P1][r].x, a_[P1][r + 2].x, a_[P0][r + 1].x, a_[P2][r + 1].x, alpha);
       b_[P2][r].y = heat_update(c.y, c.x, xp, a_[P1][r].y, a_[P1][r + 2].y, a_[P0][r + 1].y, a_[P2][r + 1].y, alpha);
     }
-    {  // level s+1 at p - 1, rows y0 .. y0+3
+    if (MID || it >= 2) {  // level s+1 at p - 1, rows y0 .. y0+3
       const double* em = edge + (size_t)e1 * ESLOT + e_nbr;
-      double* o = b2_plane(dsto, p - 1, tz, nty, te) + oxy;
+      double* o = b2_plane(dsto, p - 1, nty, tb, w, ty) + oyx;
 #pragma unroll
       for (int j = 0; j < 4; ++j) {
         const double2 c = b_[P1][j + 1];
@@ -350,8 +357,8 @@ __global__ void __launch_bounds__(b2::NT, 1)
         *reinterpret_cast<double2*>(o + j * TX) = v;
       }
     }
-    if (p >= b - 2) {  // level s's top two planes, this band's rows, to mid
-      double* o = b2_plane(mido, p, tz, nty, te) + oxy;
+    if (MID && p >= b - 2) {  // level s's top two planes, this band's rows, to mid
+      double* o = b2_plane(mido, p, nty, tb, w, ty) + oyx;
 #pragma unroll
       for (int j = 0; j < 4; ++j) *reinterpret_cast<double2*>(o + j * TX) = b_[P2][j + 1];
     }
@@ -381,16 +388,17 @@ __global__ void __launch_bounds__(b2::NT, 1)
   }
 }
 
-cudaError_t launch_heat2_band_slab(const Band2View& src, const Band2View& mid, const Band2Out& mido,
-                                   const Band2Out& dsto, int ty, int tz, int nty, int nz, int a, int b, double alpha,
+cudaError_t launch_heat2_band_slab(int mid_mode, const Band2View& src, const Band2View& mid, const Band2Out& mido,
+                                   const Band2Out& dsto, int ty, int nty, int a, int b, double alpha,
                                    cudaStream_t s) {
   using namespace b2;
-  if (b - a < 2) return cudaErrorNotSupported;
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(heat2_band_slab, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+  if (b - a < (mid_mode ? 2 : 3)) return cudaErrorNotSupported;
+  auto kern = mid_mode ? heat2_band_slab<true> : heat2_band_slab<false>;
+  static bool attr[2] = {false, false};
+  if (!attr[mid_mode ? 1 : 0]) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
     if (e != cudaSuccess) return e;
-    attr = true;
+    attr[mid_mode ? 1 : 0] = true;
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)(nty * ty / BY));
@@ -402,8 +410,7 @@ cudaError_t launch_heat2_band_slab(const Band2View& src, const Band2View& mid, c
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, heat2_band_slab, src, mid, mido, dsto, ty, tz, nty, nz, (int64_t)TX * ty * tz, a,
-                            b, alpha);
+  return cudaLaunchKernelEx(&cfg, kern, src, mid, mido, dsto, ty, nty, a, b, alpha);
 }
 
 // driver entry point for cuTensorMapEncodeTiled (no -lcuda link dependency)

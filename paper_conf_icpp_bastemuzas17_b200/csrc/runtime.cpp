@@ -925,6 +925,11 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
   const int ring_ev[2] = {d.ev_misc_base + 4 + d.halo_stream + 1, d.ev_misc_base + 5 + d.halo_stream + 1};
   const int cs = P.comp(0), os = P.out(0);
   const bool multi = G.nranks > 1;  // z-slab ranks: halo layers replace the periodic wrap
+  static const int two_env = [] {
+    const char* e = getenv("TILES_ST_TWO");
+    return e ? atoi(e) : 1;
+  }();
+  const bool two = two_env && !multi && d.opt.two_step >= 0 && X.sweep2s_ok(d);  // two sweeps per kernel
   const int hs = d.halo_stream;
   const int ev_push = d.ev_misc_base + 6 + d.halo_stream + 1;
   if (multi) ++d.st_epoch;
@@ -1019,13 +1024,18 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
         }
     // sweep i reads planes [i-1, n+2T-i+1) and writes [i, n+2T-i); the
     // first reads the resident array directly (gather fused), the last writes
-    // the unit's packed sub-tiles (scatter fused)
-    for (int i = 1; i <= T; ++i) {
-      const SlabRef src = i == 1 ? SlabRef{SlabRef::RESIDENT, bit, z0_of(u) - T}
-                                 : SlabRef{SlabRef::DENSE, slab[(i - 1) & 1], 0};
-      const SlabRef dst = i == T ? SlabRef{SlabRef::SUB, res_of(u), 0} : SlabRef{SlabRef::DENSE, slab[i & 1], 0};
+    // the unit's packed sub-tiles (scatter fused). On grids 512 wide two
+    // sweeps run per kernel (heat2_band_slab, level i kept on chip).
+    int cur = -1;  // dense slab holding the last level written (-1: the resident array)
+    for (int i = 1; i <= T;) {
+      const bool pair = two && i + 1 <= T;
+      const int last = pair ? i + 1 : i;  // the level this kernel writes
+      const int out = cur == 0 ? 1 : 0;
+      const SlabRef src = i == 1 ? SlabRef{SlabRef::RESIDENT, bit, z0_of(u) - T} : SlabRef{SlabRef::DENSE, slab[cur], 0};
+      const SlabRef dst = last == T ? SlabRef{SlabRef::SUB, res_of(u), 0} : SlabRef{SlabRef::DENSE, slab[out], 0};
       d.st_unit = np_of(u);  // packed sub-tile depth of the last sweep
-      r = X.slab_sweep(d, src, dst, i, (int)(np_of(u) + 2 * T - i), cs);
+      const int hi = (int)(np_of(u) + 2 * T - i);
+      r = pair ? X.slab_sweep2s(d, src, dst, i, hi, cs) : X.slab_sweep(d, src, dst, i, hi, cs);
       if (r.bad()) return r;
       if (i == 1 && u >= 2) {  // unit u-1's initial data has no reader left
         r = X.copy_part(d, res_of(u - 1), cur_slot(u - 1), lt, p0_of(u - 1), np_of(u - 1), cs);
@@ -1037,6 +1047,8 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
             r = X.st_halo(d, 2, side, T, cs);
             if (r.bad()) return r;
           }
+      cur = out;
+      i = last + 1;
     }
     r = X.record(d, ev_unit_done(u), cs);
     if (r.bad()) return r;

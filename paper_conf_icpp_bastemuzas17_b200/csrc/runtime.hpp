@@ -129,6 +129,11 @@ struct Exec {
   // a-1 are read), level s+1 on [a-1, b-1) into dst
   virtual Status slab_sweep2(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, int a, int b,
                              int stream) = 0;
+  // stream-through, two sweeps in one kernel (heat2_band_slab, shrink mode):
+  // level 1 on [lo, hi) from src kept on chip, level 2 on [lo+1, hi-1) into
+  // dst; sweep2s_ok: the executor runs it for this domain's shape
+  virtual bool sweep2s_ok(Domain& d) = 0;
+  virtual Status slab_sweep2s(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi, int stream) = 0;
   // two steps of the whole resident periodic grid in one kernel (heat2_band):
   // resident array src_bit -> dst_bit; band2_ok: the executor can run it for
   // this domain (the caller has checked the shape, band2_shape_ok)

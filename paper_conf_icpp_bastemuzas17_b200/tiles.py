@@ -36,7 +36,8 @@ OP_NAMES = {1: "h2d", 2: "d2h", 3: "kernel", 4: "record", 5: "wait", 6: "faces_h
             13: "gather", 14: "sweep", 15: "scatter", 16: "copy", 17: "h2d_part", 18: "d2h_part",
             19: "copy_part", 20: "h2d_pack", 21: "sweep_u", 22: "kerneld", 23: "halo_signal",
             24: "st_halo", 25: "sync", 26: "wsweep", 27: "d2h_planes", 28: "copy_planes",
-            29: "wsweep2", 30: "wsweep2_dst", 31: "band2"}
+            29: "wsweep2", 30: "wsweep2_dst", 31: "band2",
+            32: "sweep2s"}
 SCHEDS = {"auto": 0, "resident": 1, "stream": 2, "sync": 3}
 BCS = {"periodic": 0, "dirichlet": 1}
 

@@ -348,6 +348,23 @@ class Replayer:
                 for i in range(G.n[0] * G.n[1]):
                     ix, iy = i % G.n[0], i // G.n[0]
                     self.sub[(-b - 1, i)] = new[lo:hi, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx].copy()
+        elif name == "sweep2s":
+            # two sweeps in one kernel: level 1 on [lo, hi) (not stored),
+            # level 2 on [lo+1, hi-1) into b (codes as for "sweep")
+            lo, hi = c & 0xffffffff, c >> 32
+            src = self.slabs[a] if a >= 0 else self.gather(hi + 1, d)
+            assert a < 0 or a != b, "two-sweep kernel writes the slab it reads"
+            lev1 = self.sweep(src, None, lo, hi)
+            lo2, hi2 = lo + 1, hi - 1
+            if b >= 0:
+                self.slabs[b] = self.sweep(lev1, self.slabs.get(b), lo2, hi2)
+            else:
+                new = self.sweep(lev1, None, lo2, hi2)
+                G = self.G
+                tx, ty, tz = G.t
+                for i in range(G.n[0] * G.n[1]):
+                    ix, iy = i % G.n[0], i // G.n[0]
+                    self.sub[(-b - 1, i)] = new[lo2:hi2, iy * ty:(iy + 1) * ty, ix * tx:(ix + 1) * tx].copy()
         elif name == "sweep_u":
             # source: units u-1, u, u+1 as packed sub-tiles (slots in b);
             # a: destination code as for "sweep"

@@ -1,7 +1,6 @@
 python -c "import __graft_entry__ as g; g.build()" || exit 1
-timeout 600 python -m pytest tests/test_gpu_parity.py -x -q -m gpu -k "band2 or wavefront" 2>&1 | tail -4
-for wf in 1 2; do
-timeout 900 python bench.py --config fig5 --steps 3 --warmup 3 --wavefront $wf 2>/dev/null | tail -1 > gpurun_out/fig5_b2s_wf$wf.json
+for c in 32 64 128 16; do
+TILES_WAVE_C=$c timeout 900 python bench.py --config fig5 --steps 3 --warmup 3 --sweep 32,64,100,200 2>/dev/null | tail -1 > gpurun_out/fig5_c$c.json
 python -c "
-import json;d=json.load(open('gpurun_out/fig5_b2s_wf$wf.json'));print('wf=$wf', {T:(round(v['tiled']['ms'],1), v['tiled']['schedule'][:12]) for T,v in d['sweep'].items()})"
+import json;d=json.load(open('gpurun_out/fig5_c$c.json'));print('c=$c', {T:(round(v['tiled']['ms'],1), v['tiled']['schedule'][:12]) for T,v in d['sweep'].items()})"
 done

@@ -3,7 +3,8 @@ synccheck / initcheck): resident heat (layered + whole-domain phases),
 streaming heat with a tiny budget, Dirichlet, sincos, the generic kernel, the
 persistent multi-step launch (direct ghosts, grid counter, snake order; banded tiles in round-robin order), a ranged NVRTC user kernel, a user stencil and
 the stream-through schedule, the wavefront (tile-column TMA sweeps with
-tensor-map x halos) and the in-process multi-rank transport."""
+tensor-map x halos), the band kernels (heat2_band, heat2_band_slab) and the
+in-process multi-rank transport."""
 import os
 import sys
 import threading
@@ -72,6 +73,12 @@ with T.Domain((128, 64, 256), (64, 64, 32), wavefront=1) as d:   # tile-column T
     d.invalidate(); d.run(T.heat7(), 7, 3); d.store()
 with T.Domain((128, 64, 256), (64, 64, 32), stream_through=1, wavefront=-1) as d:  # stream-through, tile kernel
     d.load(uw); d.run(T.heat7(), 12, 2); d.store()
+ub2 = synth.uniform_grid(512, 16, 32, 14)                # heat2_band (resident, 512 wide, two steps per kernel)
+with T.Domain((512, 16, 32), (64, 16, 16)) as d:
+    d.load(ub2); d.run(T.heat7(), 1, 2); d.sync(); d.run(T.heat7(), 4, 2); d.store(); d.run(T.heat7(), 3, 2); d.store()
+uw2 = synth.uniform_grid(512, 16, 128, 15)               # wavefront, two-level band passes (heat2_band_slab)
+with T.Domain((512, 16, 128), (64, 16, 16), wavefront=1) as d:
+    d.load(uw2); d.run(T.heat7(), 12, 2); d.store()
 g = T.LocalGroup(2)
 def rank(r):
     with T.Domain((64, 32, 64), (32, 16, 16), nranks=2, rank=r, local_group=g) as d:

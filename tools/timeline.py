@@ -48,8 +48,8 @@ def main():
         n, td, kern, steps, kw = 512, (64, 64, 64), T.sincos(32), 10, {}
     elif cfg == "c2":
         n, td, kern, steps, kw = 512, (64, 64, 64), T.heat7(), 10, {}
-    elif cfg == "wave":   # C2 shape, fresh upload at T = 64: the wavefront schedule
-        n, td, kern, steps, kw = 512, (64, 64, 64), T.heat7(), 64, {}
+    elif cfg == "wave":   # C2 shape, fresh upload at T = 64 (env T): the wavefront schedule
+        n, td, kern, steps, kw = 512, (64, 64, 64), T.heat7(), int(os.environ.get("T", "64")), {}
     else:  # small out-of-core heat, budget for 8 tiles
         n, td, kern, steps, kw = 512, (128, 128, 128), T.heat7(), 2, {"sched": "stream",
                                                                         "device_budget_bytes": 1200 << 20}
