@@ -470,6 +470,27 @@ def test_band2_resident_bit_exact(dims, td, runs):
     assert st["sweep_cells"] == 2 * dims[0] * dims[1] * dims[2]
 
 
+@pytest.mark.parametrize("dims,td,T_", [((512, 64, 256), (64, 64, 32), 10), ((512, 32, 192), (64, 32, 16), 5),
+                                         ((512, 64, 128), (64, 64, 64), 2), ((512, 128, 256), (64, 64, 64), 13)])
+def test_stream_through_two_sweeps_bit_exact(dims, td, T_):
+    """Fresh-upload stream-through on grids 512 wide: two sweeps per kernel
+    (heat2_band_slab shrink mode: resident array / dense slabs / packed
+    sub-tiles as views), an odd T's last sweep alone; bit-exact, then a
+    resident continuation."""
+    nx, ny, nz = dims
+    u0 = synth.uniform_grid(nx, ny, nz, 8)
+    with T.Domain(dims, td, stream_through=1, wavefront=-1) as d:
+        d.load(u0)
+        d.run(T.heat7(), T_, 3)
+        out1 = d.store()
+        sched = d.get_info()["last_schedule"]
+        d.run(T.heat7(), 2, 2)
+        out2 = d.store()
+    assert sched == 2
+    assert np.array_equal(out1, oracle.heat_c(u0, ALPHA, T_))
+    assert np.array_equal(out2, oracle.heat_c(u0, ALPHA, T_ + 2))
+
+
 @pytest.mark.parametrize("T_", [7, 9, 12, 40])
 def test_band2_middle_of_batched_fresh_upload_bit_exact(T_):
     """Fresh upload on the batched schedule: the load-overlapping layer steps,
