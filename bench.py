@@ -1028,8 +1028,7 @@ SWEEP_KERNEL = {1: "heat7_fixed", 2: "slab_sweep_tile", 4: "slab_sweep_tile", 5:
 def n_two_level(gdims, td, T, args):
     """The stream-through / wavefront sweeps run two levels per kernel
     (heat2_band_slab) on single-rank grids 512 wide with 64-wide tiles."""
-    return gdims[0] == 512 and td[0] == 64 and T >= 2 and args.two_step >= 0 and \
-        int(os.environ.get("TILES_ST_TWO", "1")) != 0
+    return gdims[0] == 512 and td[0] == 64 and T >= 2 and args.two_step >= 0
 
 
 def run_main_leg(args):
@@ -1117,7 +1116,7 @@ def run_main_leg(args):
     sw_ms, sw_cells, sw_n = stk["sweep_ms"], stk["sweep_cells"], max(1, stk["sweep_timed"])
     achieved = 16.0 * sw_cells / (sw_ms / 1e3) / 1e9 if sw_ms > 0 else None
     kname = SWEEP_KERNEL.get(sched, "stencil sweeps")
-    if sched in (2, 6) and ws == 1 and n_two_level(gdims, td, T, args):
+    if (sched == 6 or (sched == 2 and args.two_step > 0)) and ws == 1 and n_two_level(gdims, td, T, args):
         kname = "heat2_band_slab"   # two sweeps / levels per kernel on grids 512 wide
     prof = traffic_per_cell(kname)
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

@@ -171,7 +171,9 @@ typedef struct {
                                    schedule; -1 = never. Any ghost: resident
                                    periodic single-rank domains 512 cells wide
                                    with 64-wide tiles run two steps per kernel
-                                   (heat2_band) unless -1 */
+                                   (heat2_band) unless -1, and with 1 their
+                                   stream-through runs two sweeps per kernel
+                                   (heat2_band_slab) */
   int32_t wavefront;            /* HEAT7 run starting from a fresh upload
                                    (periodic, single rank, resident, 2T planes
                                    of scratch fit): time-skewed march over

@@ -925,11 +925,12 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
   const int ring_ev[2] = {d.ev_misc_base + 4 + d.halo_stream + 1, d.ev_misc_base + 5 + d.halo_stream + 1};
   const int cs = P.comp(0), os = P.out(0);
   const bool multi = G.nranks > 1;  // z-slab ranks: halo layers replace the periodic wrap
-  static const int two_env = [] {
-    const char* e = getenv("TILES_ST_TWO");
-    return e ? atoi(e) : 1;
-  }();
-  const bool two = two_env && !multi && d.opt.two_step >= 0 && X.sweep2s_ok(d);  // two sweeps per kernel
+  // two sweeps per kernel (heat2_band_slab shrink mode) with two_step = 1:
+  // half the HBM traffic of the unit sweeps, but the C2 step is link-bound
+  // and measured the same (24.82 vs 24.84 ms, four alternating pairs), while
+  // the short two-level launches reach 0.53 of HBM against the single
+  // sweeps' 0.67-0.76 — single sweeps by default
+  const bool two = d.opt.two_step > 0 && !multi && X.sweep2s_ok(d);
   const int hs = d.halo_stream;
   const int ev_push = d.ev_misc_base + 6 + d.halo_stream + 1;
   if (multi) ++d.st_epoch;

@@ -473,13 +473,13 @@ def test_band2_resident_bit_exact(dims, td, runs):
 @pytest.mark.parametrize("dims,td,T_", [((512, 64, 256), (64, 64, 32), 10), ((512, 32, 192), (64, 32, 16), 5),
                                          ((512, 64, 128), (64, 64, 64), 2), ((512, 128, 256), (64, 64, 64), 13)])
 def test_stream_through_two_sweeps_bit_exact(dims, td, T_):
-    """Fresh-upload stream-through on grids 512 wide: two sweeps per kernel
+    """Fresh-upload stream-through on grids 512 wide with two_step = 1: two sweeps per kernel
     (heat2_band_slab shrink mode: resident array / dense slabs / packed
     sub-tiles as views), an odd T's last sweep alone; bit-exact, then a
     resident continuation."""
     nx, ny, nz = dims
     u0 = synth.uniform_grid(nx, ny, nz, 8)
-    with T.Domain(dims, td, stream_through=1, wavefront=-1) as d:
+    with T.Domain(dims, td, stream_through=1, wavefront=-1, two_step=1) as d:
         d.load(u0)
         d.run(T.heat7(), T_, 3)
         out1 = d.store()

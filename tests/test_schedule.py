@@ -374,18 +374,18 @@ def test_stream_through_schedule_replays_to_oracle(dims, td, T, ns):
 @pytest.mark.parametrize("dims,td,T_,ns", [((512, 8, 128), (64, 4, 8), 4, 2), ((512, 8, 192), (64, 8, 16), 5, 3),
                                             ((512, 4, 256), (64, 4, 32), 10, 2), ((512, 8, 128), (64, 4, 8), 1, 2)])
 def test_stream_through_two_sweeps_per_kernel_replays(dims, td, T_, ns):
-    """Stream-through on grids 512 wide: two sweeps per kernel (heat2_band_slab
-    shrink mode, TILE_OP_SWEEP2S; an odd T's last sweep alone), first from the
+    """Stream-through on grids 512 wide with two_step = 1: two sweeps per kernel
+    (heat2_band_slab shrink mode, TILE_OP_SWEEP2S; an odd T's last sweep alone), first from the
     resident array, the last into the packed sub-tiles; the intermediate
     level never leaves the chip. Random valid orders give the oracle."""
-    d = _run_and_replay(dims, td, [T_, 2], ns, seeds=(0, 1, 2), wavefront=-1, stream_through=1)
-    d1 = T_run_dry(dims, td, T_, ns, wavefront=-1, stream_through=1)
+    d = _run_and_replay(dims, td, [T_, 2], ns, seeds=(0, 1, 2), wavefront=-1, stream_through=1, two_step=1)
+    d1 = T_run_dry(dims, td, T_, ns, wavefront=-1, stream_through=1, two_step=1)
     ops = [op[0] for op in d1.trace()]
     assert d1.get_info()["last_schedule"] == 2
     units = ops.count("d2h_part")
     assert ops.count("sweep2s") == units * (T_ // 2) and ops.count("sweep") == units * (T_ % 2)
-    # two_step = -1: single sweeps
-    d3 = T_run_dry(dims, td, T_, ns, wavefront=-1, stream_through=1, two_step=-1)
+    # the default (two_step = 0): single sweeps
+    d3 = T_run_dry(dims, td, T_, ns, wavefront=-1, stream_through=1)
     assert "sweep2s" not in [op[0] for op in d3.trace()]
 
 
