@@ -79,6 +79,8 @@ with T.Domain((512, 16, 32), (64, 16, 16)) as d:
 uw2 = synth.uniform_grid(512, 16, 128, 15)               # wavefront, two-level band passes (heat2_band_slab)
 with T.Domain((512, 16, 128), (64, 16, 16), wavefront=1) as d:
     d.load(uw2); d.run(T.heat7(), 12, 2); d.store()
+with T.Domain((512, 8, 128), (64, 4, 8), stream_through=1, wavefront=-1, two_step=1) as d:  # two sweeps per kernel
+    d.load(synth.uniform_grid(512, 8, 128, 16)); d.run(T.heat7(), 5, 2); d.store()
 g = T.LocalGroup(2)
 def rank(r):
     with T.Domain((64, 32, 64), (32, 16, 16), nranks=2, rank=r, local_group=g) as d:
