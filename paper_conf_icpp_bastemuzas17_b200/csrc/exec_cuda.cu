@@ -533,6 +533,44 @@ struct CudaExec final : Exec {
     return true;
   }
   bool sweep2s_ok(Domain& d) override { return band2_slab_on(d); }
+  unsigned long long* iter_flags = nullptr;
+  unsigned long long iter_epoch = 0;
+  bool wave_iter_ok(Domain& d) override {
+    static const int on = [] {
+      const char* e = getenv("TILES_WAVE_ITER");
+      return e ? atoi(e) : 1;
+    }();
+    return on && band2_slab_on(d) && d.G.l[1] / 4 <= sms;
+  }
+  Status wave_iteration(Domain& d, const SlabRef* lv, int64_t ci, int c, int s0, int P, int st) override {
+    INJECT(FAULT_KERNEL, st);
+    if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
+    const Geometry& G = d.G;
+    Band2Iter p{};
+    for (int k = 0; k < 4; ++k)
+      if (!band2_in(d, lv[k], &p.v[k])) return make_err(TILE_ESTATE, "internal: wavefront views without band maps");
+    for (int k = 0; k < 3; ++k)
+      if (!band2_out(d, lv[k], 0, &p.o[k])) return make_err(TILE_ESTATE, "internal: wavefront views without band maps");
+    if (!iter_flags) {
+      const size_t nb = (size_t)(G.l[1] / 4);
+      CK(cudaMalloc(reinterpret_cast<void**>(&iter_flags), nb * sizeof(unsigned long long)));
+      CK(cudaMemset(iter_flags, 0, nb * sizeof(unsigned long long)));
+    }
+    p.flags = iter_flags;
+    p.epoch = ++iter_epoch;
+    p.ty = (int)G.t[1];
+    p.nty = (int)G.n[1];
+    p.ci = (int)ci;
+    p.c = c;
+    p.s0 = s0;
+    p.P = P;
+    p.alpha = d.kernel_alpha;
+    next_cells = d.kernel_timing ? (uint64_t)P * c * G.l[0] * G.l[1] : 0;  // one pass over each level pair's cells
+    Status r = timed(d, st, [&] { return launch_heat2_band_iter(p, S(st)); });
+    if (r.bad()) return r;
+    d.stats.n_kernels++;
+    return Status::ok();
+  }
   Status slab_sweep2s(Domain& d, const SlabRef& src, const SlabRef& dst, int lo, int hi, int st) override {
     INJECT(FAULT_KERNEL, st);
     if (d.measure == TILE_MEASURE_XFER_ONLY) return Status::ok();
@@ -1028,6 +1066,8 @@ struct CudaExec final : Exec {
       if (own_stream[i] && streams[i]) cudaStreamDestroy(streams[i]);
     events.clear();
     streams.clear();
+    if (iter_flags) cudaFree(iter_flags);
+    iter_flags = nullptr;
   }
 };
 

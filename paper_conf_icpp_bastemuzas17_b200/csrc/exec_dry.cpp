@@ -121,6 +121,16 @@ struct DryExec final : Exec {
     return Status::ok();
   }
   bool band2_ok(Domain&) override { return true; }
+  bool wave_iter_ok(Domain& d) override { return sweep2s_ok(d); }
+  Status wave_iteration(Domain& d, const SlabRef* lv, int64_t ci, int c, int s0, int P, int st) override {
+    for (int k = 0; k < P; ++k) {
+      const int s = s0 + 2 * k;
+      const SlabRef& src = s - 1 == 0 ? lv[3] : lv[(s - 1) % 3];
+      Status r = slab_sweep2(d, src, lv[s % 3], lv[(s + 1) % 3], (int)(ci - s), (int)(ci - s + c), st);
+      if (r.bad()) return r;
+    }
+    return Status::ok();
+  }
   bool sweep2s_ok(Domain& d) override {
     const Geometry& G = d.G;
     return G.nranks == 1 && band2_shape_ok(G.l[0], G.l[1], (int)G.t[0], (int)G.t[1]);

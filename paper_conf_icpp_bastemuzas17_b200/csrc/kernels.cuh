@@ -239,6 +239,20 @@ struct Band2Out {
 cudaError_t launch_heat2_band_slab(int mid_mode, const Band2View& src, const Band2View& mid, const Band2Out& mido,
                                    const Band2Out& dsto, int ty, int nty, int a, int b, double alpha,
                                    cudaStream_t s);
+// all two-level passes of one wavefront iteration (heat2_band_iter): level
+// views v[k] = lvl(s) for s % 3 == k (s >= 1), v[3] = lvl(0) (the resident
+// array); o[k] the level arrays as outputs; pass k runs levels s0 + 2k and
+// s0 + 2k + 1 on planes [ci - s, ci - s + c); bands synchronise through
+// per-band progress flags (nbands u64, epoch in the high half)
+struct Band2Iter {
+  Band2View v[4];
+  Band2Out o[3];
+  unsigned long long* flags;
+  unsigned long long epoch;
+  int ty, nty, ci, c, s0, P;
+  double alpha;
+};
+cudaError_t launch_heat2_band_iter(const Band2Iter& p, cudaStream_t s);
 // device -> mapped pinned host rows copied by the SMs (pitches, len in doubles;
 // len and pitches even)
 cudaError_t launch_push_rows(const double* src, int64_t src_pitch, double* dst, int64_t dst_pitch, int64_t rows,

@@ -413,6 +413,218 @@ cudaError_t launch_heat2_band_slab(int mid_mode, const Band2View& src, const Ban
   return cudaLaunchKernelEx(&cfg, kern, src, mid, mido, dsto, ty, nty, a, b, alpha);
 }
 
+// ---- all two-level passes of one wavefront iteration in one launch
+// (heat2_band_iter). Pass k (levels s, s+1 with s = s0 + 2k) has the
+// heat2_band_slab<MID> semantics over the level views lvl(s-1), lvl(s),
+// lvl(s+1). A band runs its passes back to back; between passes it needs
+// nothing but its two neighbour bands' progress: the source planes of pass k
+// that pass k-1 wrote (rows y0-2 .. y0+5 come from bands b-1, b, b+1) are
+// staged only once both neighbours have published that pass k-1 iteration
+// (per-band 64-bit flags: epoch << 32 | pass << 16 | iterations done,
+// published by thread 0 after the block barrier with a GPU-scope fence, read
+// with ld.acquire and followed by a proxy fence before the TMA). Every
+// other hazard between consecutive passes is ordered by that wait (DESIGN.md
+// §4). The producer's staging runs across pass boundaries, so a pass starts
+// with its first planes already on chip. All CTAs must be co-resident (one
+// band per SM, grid = ny/4 <= SMs); no programmatic early launch of the next
+// kernel (it could take the SMs of CTAs this one waits on).
+static __device__ __forceinline__ void st_relaxed_gpu_u64(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__global__ void __launch_bounds__(b2::NT, 1) heat2_band_iter(const __grid_constant__ Band2Iter it_) {
+  using namespace b2;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  double* stage = reinterpret_cast<double*>(smem_raw);
+  double* edge = stage + (size_t)S * STAGE;
+  uint64_t* full = reinterpret_cast<uint64_t*>(edge + 3 * ESLOT);
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) mbar_init(&full[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  const int ty = it_.ty, nty = it_.nty, ny = nty * ty;
+  const int band = (int)blockIdx.x, nb = (int)gridDim.x;
+  const int y0 = band * BY;
+  const int ya = (y0 - 2 + ny) % ny, yc = (y0 + 4) % ny;
+  const int ta = ya / ty, la = ya % ty, tb = y0 / ty, lb = y0 % ty, tc = yc / ty, lc = yc % ty;
+  unsigned long long* const fl_me = it_.flags + band;
+  const unsigned long long* const fl_lo = it_.flags + (band + nb - 1) % nb;
+  const unsigned long long* const fl_hi = it_.flags + (band + 1) % nb;
+  const unsigned long long ep = it_.epoch << 32;
+  auto src_of = [&](int k) -> const Band2View& {
+    const int s = it_.s0 + 2 * k;
+    return s - 1 == 0 ? it_.v[3] : it_.v[(s - 1) % 3];
+  };
+  // thread 0: staging cursor (pass, staged index within the pass, ring slot)
+  int ik = 0, iq = 0, qs = 0;
+  const int nqp = 2 + it_.c + 2;  // staged planes per pass: mid a-2, a-1, src a-1 .. b
+  auto issue = [&]() {
+    const int k = ik, s = it_.s0 + 2 * k, a = it_.ci - s;
+    const bool m = iq < 2;
+    const int z = m ? a - 2 + iq : a - 1 + (iq - 2);
+    if (!m && k > 0) {  // a plane pass k-1 wrote: wait for the neighbour bands
+      const int a1 = a + 2;       // pass k-1's a
+      if (z >= a1 - 1) {
+        const unsigned long long need = ep | ((unsigned long long)(k - 1) << 16) | (unsigned)(z - a1 + 2);
+        long long spin = 0;
+        while (ld_acquire_gpu(fl_lo) < need || ld_acquire_gpu(fl_hi) < need)
+          if (++spin > (1ll << 28)) asm volatile("trap;");
+        fence_proxy_async_all();
+      }
+    }
+    const TensorMapBlob *m4, *m2;
+    int zl, zt;
+    b2_coords(m ? it_.v[s % 3] : src_of(k), z, m4, m2, zl, zt);
+    double* d = stage + (size_t)qs * STAGE;
+    fence_proxy_async();
+    mbar_expect_tx(&full[qs], BYTES);
+    tma_5d(d + OFF_A, m2, 0, la, 0, zl, zt * nty + ta, &full[qs]);
+    tma_5d(d + OFF_B, m4, 0, lb, 0, zl, zt * nty + tb, &full[qs]);
+    tma_5d(d + OFF_C, m2, 0, lc, 0, zl, zt * nty + tc, &full[qs]);
+    qs = qs + 1 == S ? 0 : qs + 1;
+    if (++iq == nqp) iq = 0, ++ik;
+  };
+  const int ntot = it_.P * nqp;  // staged planes of the launch
+  int issued = 0;                // thread 0: global staged index
+  if (threadIdx.x == 0) {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    for (; issued < S && issued < ntot; ++issued) issue();
+  }
+
+  const int t = (int)threadIdx.x, lane = t & 31, w = t >> 5;
+  const int x = 2 * lane;
+  const bool right = lane == 31;
+  const int we = right ? (w + 1) % NW : (w + NW - 1) % NW, xe = right ? 0 : TX - 1;
+  const int e_mine = right ? (w * 2 + 1) * ER : w * 2 * ER;
+  const int e_nbr = right ? ((w + 1) % NW) * 2 * ER : (((w + NW - 1) % NW) * 2 + 1) * ER;
+  const uint32_t is_left = lane == 0, is_right = right;
+  const int oyx = lb * TX + x;
+  auto wait_g = [&](int g) { mbar_wait(&full[g % S], (g / S) & 1); };
+  auto ld2 = [&](const double* st, int i) { return *reinterpret_cast<const double2*>(st + srow(i, w) + x); };
+
+  double2 a_[3][8], b_[3][6];
+  int g0 = 0;  // global staged index of this pass's first plane
+  for (int k = 0; k < it_.P; ++k, g0 += nqp) {
+    const int s = it_.s0 + 2 * k, a = it_.ci - s, b = a + it_.c;
+    const Band2Out& mido = it_.o[s % 3];
+    const Band2Out& dsto = it_.o[(s + 1) % 3];
+    wait_g(g0);
+#pragma unroll
+    for (int r = 0; r < 6; ++r) b_[0][r] = ld2(stage + (size_t)(g0 % S) * STAGE, r + 1);
+    wait_g(g0 + 1);
+#pragma unroll
+    for (int r = 0; r < 6; ++r) b_[1][r] = ld2(stage + (size_t)((g0 + 1) % S) * STAGE, r + 1);
+    {
+      const uint32_t ez = smem_u32(edge + (size_t)2 * ESLOT + e_mine);
+#pragma unroll
+      for (int r = 0; r < 6; ++r) {
+        sts_if(ez + 8 * r, b_[1][r].x, is_left);
+        sts_if(ez + 8 * r, b_[1][r].y, is_right);
+      }
+    }
+    wait_g(g0 + 2);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) a_[0][i] = ld2(stage + (size_t)((g0 + 2) % S) * STAGE, i);
+    wait_g(g0 + 3);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) a_[1][i] = ld2(stage + (size_t)((g0 + 3) % S) * STAGE, i);
+    bar_consumers_b2();
+    if (t == 0)
+      for (; issued < ntot && issued <= g0 + 2 + S; ++issued) issue();
+    int sq = (g0 + 4) % S, sq1 = (g0 + 3) % S;
+    int e0 = 0, e1 = 2;
+    auto step = [&](int it, auto kc) {
+      constexpr int K = decltype(kc)::value;
+      constexpr int P0 = K, P1 = (K + 1) % 3, P2 = (K + 2) % 3;
+      const int p = a + it, g = g0 + it + 4;
+      wait_g(g);
+      const double* sz = stage + (size_t)sq1 * STAGE;
+      const double* sp = stage + (size_t)sq * STAGE;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) a_[P2][i] = ld2(sp, i);
+#pragma unroll
+      for (int r = 0; r < 6; ++r) {
+        const double2 c = a_[P1][r + 1];
+        double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+        double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+        const uint32_t ea = smem_u32(sz + srow(r + 1, we) + xe);
+        lds_if(xm, ea, is_left);
+        lds_if(xp, ea, is_right);
+        b_[P2][r].x = heat_update(c.x, xm, c.y, a_[P1][r].x, a_[P1][r + 2].x, a_[P0][r + 1].x, a_[P2][r + 1].x, it_.alpha);
+        b_[P2][r].y = heat_update(c.y, c.x, xp, a_[P1][r].y, a_[P1][r + 2].y, a_[P0][r + 1].y, a_[P2][r + 1].y, it_.alpha);
+      }
+      {
+        const double* em = edge + (size_t)e1 * ESLOT + e_nbr;
+        double* o = b2_plane(dsto, p - 1, nty, tb, w, ty) + oyx;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const double2 c = b_[P1][j + 1];
+          double xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+          double xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+          lds_if(xm, smem_u32(em + j + 1), is_left);
+          lds_if(xp, smem_u32(em + j + 1), is_right);
+          double2 v;
+          v.x = heat_update(c.x, xm, c.y, b_[P1][j].x, b_[P1][j + 2].x, b_[P0][j + 1].x, b_[P2][j + 1].x, it_.alpha);
+          v.y = heat_update(c.y, c.x, xp, b_[P1][j].y, b_[P1][j + 2].y, b_[P0][j + 1].y, b_[P2][j + 1].y, it_.alpha);
+          *reinterpret_cast<double2*>(o + j * TX) = v;
+        }
+      }
+      if (p >= b - 2) {
+        double* o = b2_plane(mido, p, nty, tb, w, ty) + oyx;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) *reinterpret_cast<double2*>(o + j * TX) = b_[P2][j + 1];
+      }
+      {
+        const uint32_t ez = smem_u32(edge + (size_t)e0 * ESLOT + e_mine);
+#pragma unroll
+        for (int r = 0; r < 6; ++r) {
+          sts_if(ez + 8 * r, b_[P2][r].x, is_left);
+          sts_if(ez + 8 * r, b_[P2][r].y, is_right);
+        }
+      }
+      bar_consumers_b2();
+      if (t == 0) {
+        // this band's level s+1 planes up to p - 1 are written: publish
+        fence_acq_rel_gpu();
+        st_relaxed_gpu_u64(fl_me, ep | ((unsigned long long)k << 16) | (unsigned)(it + 1));
+        for (; issued < ntot && issued <= g - 1 + S; ++issued) issue();
+      }
+      sq1 = sq;
+      sq = sq + 1 == S ? 0 : sq + 1;
+      e1 = e0;
+      e0 = e0 == 2 ? 0 : e0 + 1;
+    };
+    const int nit = b - a;
+    for (int it = 0; it < nit; it += 3) {
+      step(it, std::integral_constant<int, 0>{});
+      if (it + 1 >= nit) break;
+      step(it + 1, std::integral_constant<int, 1>{});
+      if (it + 2 >= nit) break;
+      step(it + 2, std::integral_constant<int, 2>{});
+    }
+  }
+}
+
+cudaError_t launch_heat2_band_iter(const Band2Iter& p, cudaStream_t s) {
+  using namespace b2;
+  if (p.c < 2 || p.P < 1) return cudaErrorNotSupported;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(heat2_band_iter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  int dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int grid = p.nty * p.ty / BY;
+  if (grid > sms) return cudaErrorNotSupported;  // every band co-resident
+  // a plain launch: waits for the previous kernel, lets nothing start early
+  heat2_band_iter<<<grid, NT, SMEM, s>>>(p);
+  return cudaGetLastError();
+}
+
 // driver entry point for cuTensorMapEncodeTiled (no -lcuda link dependency)
 using EncodeTiledFn5 = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                     const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,

@@ -1517,7 +1517,14 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
         r = X.wait(d, ev_in(d, i), cs);
         if (r.bad()) return r;
       }
-      for (int s = 1; s <= T;) {
+      int s = 1;
+      if (wp.fused && T >= 2 && X.wave_iter_ok(d)) {  // every pair of levels in one launch
+        const SlabRef lv[4] = {lvl(3), lvl(1), lvl(2), lvl(0)};
+        r = X.wave_iteration(d, lv, c * i, (int)c, 1, T / 2, cs);
+        if (r.bad()) return r;
+        s = 2 * (T / 2) + 1;
+      }
+      while (s <= T) {
         int done = 0;
         r = pass_of_iteration(i, s, &done);
         if (r.bad()) return r;

@@ -129,6 +129,12 @@ struct Exec {
   // a-1 are read), level s+1 on [a-1, b-1) into dst
   virtual Status slab_sweep2(Domain& d, const SlabRef& src, const SlabRef& mid, const SlabRef& dst, int a, int b,
                              int stream) = 0;
+  // the wavefront: passes k = 0..P-1 of iteration ci/c (levels s0+2k,
+  // s0+2k+1 on [ci - s, ci - s + c)) in one launch (heat2_band_iter); lv[k]
+  // the view of the levels s with s % 3 == k, lv[3] level 0; the trace
+  // records the passes as separate TILE_OP_WSWEEP2 ops
+  virtual bool wave_iter_ok(Domain& d) = 0;
+  virtual Status wave_iteration(Domain& d, const SlabRef* lv, int64_t ci, int c, int s0, int P, int stream) = 0;
   // stream-through, two sweeps in one kernel (heat2_band_slab, shrink mode):
   // level 1 on [lo, hi) from src kept on chip, level 2 on [lo+1, hi-1) into
   // dst; sweep2s_ok: the executor runs it for this domain's shape
