@@ -428,6 +428,7 @@ cudaError_t launch_heat2_band_slab(int mid_mode, const Band2View& src, const Ban
 // with its first planes already on chip. All CTAs must be co-resident (one
 // band per SM, grid = ny/4 <= SMs); no programmatic early launch of the next
 // kernel (it could take the SMs of CTAs this one waits on).
+constexpr int kIterPub = 8;  // progress published every 8 planes (and at each pass's end)
 static __device__ __forceinline__ void st_relaxed_gpu_u64(unsigned long long* p, unsigned long long v) {
   asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
@@ -458,6 +459,7 @@ __global__ void __launch_bounds__(b2::NT, 1) heat2_band_iter(const __grid_consta
   };
   // thread 0: staging cursor (pass, staged index within the pass, ring slot)
   int ik = 0, iq = 0, qs = 0;
+  unsigned long long seen_lo = 0, seen_hi = 0;  // thread 0: neighbour progress last observed
   const int nqp = 2 + it_.c + 2;  // staged planes per pass: mid a-2, a-1, src a-1 .. b
   auto issue = [&]() {
     const int k = ik, s = it_.s0 + 2 * k, a = it_.ci - s;
@@ -466,11 +468,15 @@ __global__ void __launch_bounds__(b2::NT, 1) heat2_band_iter(const __grid_consta
     if (!m && k > 0) {  // a plane pass k-1 wrote: wait for the neighbour bands
       const int a1 = a + 2;       // pass k-1's a
       if (z >= a1 - 1) {
+        // the neighbours are usually a pass ahead: the progress last seen
+        // answers most checks without a GPU-scope load
         const unsigned long long need = ep | ((unsigned long long)(k - 1) << 16) | (unsigned)(z - a1 + 2);
-        long long spin = 0;
-        while (ld_acquire_gpu(fl_lo) < need || ld_acquire_gpu(fl_hi) < need)
-          if (++spin > (1ll << 28)) asm volatile("trap;");
-        fence_proxy_async_all();
+        if (seen_lo < need || seen_hi < need) {
+          long long spin = 0;
+          while ((seen_lo = ld_acquire_gpu(fl_lo)) < need || (seen_hi = ld_acquire_gpu(fl_hi)) < need)
+            if (++spin > (1ll << 28)) asm volatile("trap;");
+          fence_proxy_async_all();
+        }
       }
     }
     const TensorMapBlob *m4, *m2;
@@ -585,9 +591,13 @@ __global__ void __launch_bounds__(b2::NT, 1) heat2_band_iter(const __grid_consta
       }
       bar_consumers_b2();
       if (t == 0) {
-        // this band's level s+1 planes up to p - 1 are written: publish
-        fence_acq_rel_gpu();
-        st_relaxed_gpu_u64(fl_me, ep | ((unsigned long long)k << 16) | (unsigned)(it + 1));
+        // this band's level s+1 planes up to p - 1 are written: publish every
+        // PUB iterations and at the pass's end (a GPU-scope fence costs about
+        // a plane's time; the neighbours read a pass's flags a pass later)
+        if ((it + 1) % kIterPub == 0 || it + 1 == b - a) {
+          fence_acq_rel_gpu();
+          st_relaxed_gpu_u64(fl_me, ep | ((unsigned long long)k << 16) | (unsigned)(it + 1));
+        }
         for (; issued < ntot && issued <= g - 1 + S; ++issued) issue();
       }
       sq1 = sq;
