@@ -491,6 +491,23 @@ def test_stream_through_two_sweeps_bit_exact(dims, td, T_):
     assert np.array_equal(out2, oracle.heat_c(u0, ALPHA, T_ + 2))
 
 
+def test_wavefront_one_launch_per_iteration_bit_exact():
+    """The opt-in one-launch-per-iteration wavefront (heat2_band_iter,
+    TILES_WAVE_ITER=1: bands synchronised by progress flags) on the 512-wide
+    wavefront parity cases, in a fresh process (the knob is read once)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    ids = [f"tests/test_gpu_parity.py::test_wavefront_bit_exact[1-dims{k}-td{k}-{t}]"
+           for k, t in ((5, 16), (6, 20), (7, 48), (8, 100))]   # the 512-wide cases
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-p", "no:cacheprovider", *ids],
+                       cwd=root, env={**os.environ, "TILES_WAVE_ITER": "1"}, capture_output=True, text=True,
+                       timeout=900)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
+    assert " passed" in r.stdout
+
+
 @pytest.mark.parametrize("T_", [7, 9, 12, 40])
 def test_band2_middle_of_batched_fresh_upload_bit_exact(T_):
     """Fresh upload on the batched schedule: the load-overlapping layer steps,
