@@ -1020,9 +1020,10 @@ def main():
 SCHED_NAMES = {0: "none", 1: "resident batched (layer batches + whole-domain steps)",
                2: "stream-through (fresh upload, T <= tz)", 3: "out-of-core per-tile stream",
                4: "out-of-core stream-through", 5: "synchronous (one stream)", 6: "wavefront (fresh upload)",
-               7: "resident, two steps per kernel (heat2_band)"}
+               7: "resident, two steps per kernel (heat2_band)",
+               8: "wavefront (upload) + resident two-step passes + wavefront (download)"}
 SWEEP_KERNEL = {1: "heat7_fixed", 2: "slab_sweep_tile", 4: "slab_sweep_tile", 5: "heat7_fixed",
-                6: "slab_sweep_tile", 7: "heat2_band"}
+                6: "slab_sweep_tile", 7: "heat2_band", 8: "heat2_band"}
 
 
 def n_two_level(gdims, td, T, args):

@@ -244,7 +244,10 @@ typedef struct {
                              out-of-core stream-through, 5 synchronous (one
                              stream), 6 wavefront (fresh upload), 7 resident,
                              two steps per kernel (heat2_band: periodic,
-                             single rank, 512 cells wide, 64-wide tiles) */
+                             single rank, 512 cells wide, 64-wide tiles),
+                             8 fresh upload at large T: wavefront during the
+                             upload, resident two-step passes, wavefront
+                             during the download */
   double sweep_link_ratio; /* the cost model's ratio in use (see tile_options) */
 } tile_info;
 

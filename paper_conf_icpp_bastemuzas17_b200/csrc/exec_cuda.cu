@@ -378,6 +378,7 @@ struct CudaExec final : Exec {
   SweepMaps maps{};
   bool maps_tried = false;
   const double* maps_wave = nullptr;
+  int64_t maps_wave_slots = 0;
   // tensor maps of the slot pool and the wavefront scratch (x halos of the
   // tile-column sweep), encoded once per allocation
   void ensure_maps(Domain& d) {
@@ -386,8 +387,12 @@ struct CudaExec final : Exec {
       sweep_map_encode(&maps, 0, d.slot_base, (uint64_t)d.nslots * d.G.tile_elems * 8, (int)d.G.t[0],
                        sweep_tile_band());
     }
-    if (d.wave_base && maps_wave != d.wave_base) {
+    // (re-encoded when the scratch moves or grows: a reallocation may return
+    // the same address with more slots, which a stale map would read as
+    // out-of-bounds zeros)
+    if (d.wave_base && (maps_wave != d.wave_base || maps_wave_slots != d.wave_slots)) {
       maps_wave = d.wave_base;
+      maps_wave_slots = d.wave_slots;
       sweep_map_encode(&maps, 1, d.wave_base, (uint64_t)d.wave_slots * d.G.tile_elems * 8, (int)d.G.t[0],
                        sweep_tile_band());
     }

@@ -1385,7 +1385,12 @@ static Status ensure_wave_scratch(Domain& d, int64_t slots) {
   return Status::ok();
 }
 
-static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
+// h2d = false: level 0 is already in the resident array (no uploads; the
+// upload events are still recorded); d2h = false: the chunks' level-T planes
+// stay on the device (no D2H; the tiles are left dirty for tile_sync). The
+// large-T fresh-upload schedule runs the wavefront twice this way around the
+// resident two-step passes (run_heat_resident).
+static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp, bool h2d = true, bool d2h = true) {
   Exec& X = *d.exec;
   const Geometry& G = d.G;
   const int64_t nz = G.l[2], tz = G.t[2], lt = G.layer_tiles, c = wp.c, B = wp.B, nlo = wp.nlo;
@@ -1419,6 +1424,7 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
     return Status::ok();
   };
   auto upload = [&](int64_t z0, int64_t z1) {
+    if (!h2d) return Status::ok();
     return pieces(z0, z1, [&](int64_t L, int64_t lz, int64_t np) {
       return X.h2d_part(d, L * lt, lt, arr0(bit, L), lz, np, is);
     });
@@ -1531,6 +1537,7 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
         s += done;
       }
     }
+    if (!d2h) continue;
     r = X.record(d, ev_host(d, i), cs);
     if (r.bad()) return r;
     r = X.wait(d, ev_host(d, i), os);
@@ -1567,12 +1574,18 @@ static Status run_wavefront(Domain& d, int T, int S, const WavePlan& wp) {
   }
   d.res_bit = fin;
   for (int64_t k = 0; k < G.ntiles; ++k) {
-    d.tile_dirty[k] = 0;  // the host received u^T through the D2H above
+    d.tile_dirty[k] = d2h ? 0 : 1;  // with d2h the host received u^T through the D2H above
     d.tile_slot[k] = fin ? (int)(G.ntiles + k) : (int)k;
   }
   d.resident_valid = true;
   d.faces_valid = d.xfaces_valid = false;  // faces are re-extracted by the next resident run
   d.last_batches.clear();
+  if (!d2h) {  // tile_sync copies the whole grid back after this run's last kernel
+    const int ev = ev_layer(d, 0, 0);
+    r = X.record(d, ev, cs);
+    if (r.bad()) return r;
+    d.last_batches.push_back({0, G.n[2], cs, os, ev});
+  }
   return Status::ok();
 }
 
@@ -1654,6 +1667,31 @@ static Status run_heat_resident(Domain& d, double alpha, int steps, int S, bool 
     if (take_st) {
       d.last_schedule = 2;
       return run_streamthrough(d, alpha, steps, S, sp);
+    }
+    // large T (the batched schedule's range): a wavefront of Tw levels while
+    // the grid uploads (nothing downloaded), the middle steps two per kernel
+    // on the resident grid, and a wavefront of the last Tw (+1) levels while
+    // it downloads (nothing uploaded) — both link directions overlap compute
+    // instead of bracketing it (TILES_WAVE_SPLIT=0: the batched schedule)
+    static const int split = [] {
+      const char* e = getenv("TILES_WAVE_SPLIT");
+      return e ? atoi(e) : 1;
+    }();
+    if (split && d.opt.wavefront >= 0 && band2_fits(d, serial)) {
+      int Tw = 64;
+      WavePlan w0;
+      while (Tw >= 8 && !wavefront_ok(d, Tw, &w0)) Tw /= 2;
+      const int mid = steps - 2 * Tw;
+      WavePlan w1;
+      if (Tw >= 8 && mid >= 2 && wavefront_ok(d, Tw + (mid & 1), &w1)) {
+        Status r = run_wavefront(d, Tw, S, w0, true, false);
+        if (r.bad()) return r;
+        r = run_band2(d, mid & ~1, S);
+        if (r.bad()) return r;
+        r = run_wavefront(d, Tw + (mid & 1), S, w1, false, true);
+        d.last_schedule = 8;
+        return r;
+      }
     }
   }
   d.last_schedule = serial ? 5 : 1;

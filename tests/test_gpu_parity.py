@@ -410,7 +410,7 @@ def test_stream_through_bit_exact(dims, td, T):
                                        ((64, 64, 64), (32, 32, 8), 7), ((96, 64, 160), (32, 32, 32), 1),
                                        ((64, 32, 512), (32, 32, 64), 100), ((512, 64, 128), (64, 64, 64), 16),
                                        ((512, 32, 256), (64, 32, 32), 20), ((512, 64, 384), (64, 64, 64), 48),
-                                       ((512, 16, 512), (64, 16, 64), 100)])
+                                       ((512, 16, 512), (64, 16, 64), 100), ((512, 32, 256), (64, 32, 32), 21)])
 @pytest.mark.parametrize("wave", [1, 2, 3])
 def test_wavefront_bit_exact(dims, td, T, wave):
     """Fresh-upload runs on the time-skewed wavefront (forced): chunks of
@@ -509,6 +509,27 @@ def test_wavefront_one_launch_per_iteration_bit_exact():
                        timeout=900)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
     assert " passed" in r.stdout
+
+
+@pytest.mark.parametrize("T_", [70, 73])
+def test_large_T_split_wavefront_bit_exact(T_):
+    """Fresh upload at large T: wavefront during the upload, two-step passes,
+    wavefront during the download (last_schedule 8); bit-exact, then a
+    resident continuation."""
+    dims, td = (512, 64, 128), (64, 64, 16)
+    u0 = synth.uniform_grid(*dims, 21)
+    with T.Domain(dims, td) as d:
+        d.load(u0)
+        d.run(T.heat7(), T_, 4)
+        out1 = d.store()
+        sched = d.get_info()["last_schedule"]
+        st = d.stats()
+        d.run(T.heat7(), 3, 2)
+        out2 = d.store()
+    assert sched == 8
+    assert np.array_equal(out1, oracle.heat_c(u0, ALPHA, T_))
+    assert np.array_equal(out2, oracle.heat_c(u0, ALPHA, T_ + 3))
+    assert st["bytes_h2d"] == u0.nbytes and st["bytes_d2h"] == u0.nbytes
 
 
 @pytest.mark.parametrize("T_", [7, 9, 12, 40])

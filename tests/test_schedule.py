@@ -620,6 +620,24 @@ def test_wavefront_512_wide_default_two_levels(T_):
     assert "wsweep2" not in [op[0] for op in d3.trace()] and d3.get_info()["last_schedule"] == 6
 
 
+@pytest.mark.parametrize("T_", [70, 71])
+def test_large_T_split_wavefront_replays(T_):
+    """A fresh upload at large T on a grid 512 wide: a wavefront of Tw levels
+    during the upload (no D2H), the middle steps in pairs on heat2_band, a
+    wavefront of the last Tw (+1) levels during the download (no H2D): every
+    cell crosses the link once per direction, and random valid orders give
+    the oracle bit-exactly."""
+    dims, td = (512, 8, 128), (64, 4, 16)   # wavefront up to T = 56 here: Tw = 32
+    d = _run_and_replay(dims, td, [T_, 2], 2, seeds=(0, 1))
+    d1 = T_run_dry(dims, td, T_, 2)
+    ops = [op[0] for op in d1.trace()]
+    assert d1.get_info()["last_schedule"] == 8
+    assert ops.count("band2") == (T_ - 64) // 2
+    st = d1.stats()
+    cells = dims[0] * dims[1] * dims[2]
+    assert st["bytes_h2d"] == cells * 8 and st["bytes_d2h"] == cells * 8
+
+
 def T_run_dry(dims, td, steps, ns, **kw):
     d = T.Domain(dims, td, dry_run=True, **kw)
     d.load(np.zeros(dims[::-1]))
@@ -641,7 +659,7 @@ def test_wavefront_cost_model_choice():
         sched[steps] = d.get_info()["last_schedule"]
         d.free()
     assert sched[10] == 2 and sched[32] == 6 and sched[64] == 6 and sched[100] == 6
-    assert sched[300] == 1
+    assert sched[300] == 8   # wavefront (upload) + two-step passes + wavefront (download)
 
 
 def test_cost_model_ratio_option_and_report():
