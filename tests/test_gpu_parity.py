@@ -511,6 +511,23 @@ def test_wavefront_one_launch_per_iteration_bit_exact():
     assert " passed" in r.stdout
 
 
+@pytest.mark.parametrize("wave", [1, 3])
+def test_wavefront_growing_T_on_one_domain_bit_exact(wave):
+    """Fresh-upload wavefront runs of growing T on one domain (the Fig. 5
+    sweep's pattern): the scratch grows in place between runs and every
+    tensor map over it must follow (a stale map read the new part as
+    out-of-bounds zeros)."""
+    dims, td = (512, 32, 256), (64, 32, 32)
+    u0 = synth.uniform_grid(*dims, 31)
+    with T.Domain(dims, td, wavefront=wave) as d:
+        for T_ in (5, 20, 47, 64):
+            d.load(u0)   # the host store holds the previous run's result after store()
+            d.run(T.heat7(), T_, 3)
+            out = d.store()
+            assert d.get_info()["last_schedule"] == 6
+            assert np.array_equal(out, oracle.heat_c(u0, ALPHA, T_)), T_
+
+
 @pytest.mark.parametrize("T_", [70, 73])
 def test_large_T_split_wavefront_bit_exact(T_):
     """Fresh upload at large T: wavefront during the upload, two-step passes,
