@@ -3,7 +3,7 @@
 # sanitizers, the default bench line, the ncu launch list of the same
 # command, per-kernel DRAM traffic, --set full captures of the band kernels,
 # the Fig. 5 sweep and CUPTI timelines.
-O=gpurun_out/r2f
+O=gpurun_out/r2f3
 mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" || exit 1
 timeout 2400 python -m pytest tests -m gpu -q 2>&1 | tail -3 > $O/gputests.txt; cat $O/gputests.txt
@@ -36,6 +36,6 @@ ncu -i $O/heat2_band_full.ncu-rep --page raw --csv > $O/heat2_band_full.raw.csv 
 SCHED=wave T=64 timeout 900 ncu --set full --clock-control none --import-source on -k regex:heat2_band_slab -s 200 -c 1 -o $O/heat2_band_slab_full python tools/prof_sweep.py > /dev/null 2>&1
 ncu -i $O/heat2_band_slab_full.ncu-rep --page raw --csv > $O/heat2_band_slab_full.raw.csv 2>/dev/null
 rm -f $O/*.ncu-rep
-timeout 900 python bench.py --config fig5 --steps 3 --warmup 3 > $O/fig5.json 2>/dev/null
+timeout 1200 python bench.py --config fig5 --steps 3 --warmup 3 --sweep 1,10,32,48,64,100,200,1000 > $O/fig5.json 2>/dev/null
 for c in c2 wave; do T=64 python tools/timeline.py $c $O/timeline_$c > /dev/null 2>&1; rm -f $O/timeline_$c.trace.json; done
 ls $O
