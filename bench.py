@@ -1224,6 +1224,15 @@ def run_main_leg(args):
                                    "t_link_dependency_form_ms": t_dep * 1e3, "t_hbm_ms": t_hbm * 1e3,
                                    "frac": R / (wall / 1e3), "achieved_gbs": (h2d_b + d2h_b) / (wall / 1e3) / 1e9,
                                    "peak_gbs": bidir, "pcie_gbs": {**bw, "bidir": bidir}}
+        # the stencil's own constraint on top of the duplex form: no output
+        # plane before its 2T+1-plane cone has arrived (H2D alone), and the
+        # last upload's cone returns alone (D2H alone); between, both ways
+        cone = min(2 * T + 1, nzl) * nx * ny * 8
+        t_causal = cone / (bw["h2d"] * 1e9) + cone / (bw["d2h"] * 1e9) + 2 * max(0, B - cone) / (bidir * 1e9)
+        extras["roofline_link"].update({
+            "t_causal_duplex_ms": t_causal * 1e3, "frac_causal_duplex": t_causal / (wall / 1e3),
+            "causal_duplex_def": "(2T+1) planes H2D alone + (2T+1) planes D2H alone + the rest both ways "
+                                 "at the bidirectional rate"})
         if ws == 1:
             dom.free()
             sdom = Tl.Domain(gdims, td, ghost=args.ghost, device=lr, sched="sync")
