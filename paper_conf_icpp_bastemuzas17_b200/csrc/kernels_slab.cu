@@ -868,9 +868,10 @@ cudaError_t launch_slab_sweep(const SlabView& src, const SlabView& dst, int nx, 
   if (use_tma && maps && maps->valid[0] && maps->band == tb && !src.ring && src.tx == 64 && dst.tx == 64 &&
       src.ty % tb == 0 && dst.ty % tb == 0 && nx % 64 == 0 && ny % tb == 0 && !src.hhi &&
       (!src.hlo || (maps->valid[1] && src.hlo >= maps->base[1] && src.hlo < maps->end[1])))
-    // band 32, 4 rows per consumer thread, 4 stages, 2 CTAs per SM (band 16 or 64, 3 CTAs per SM
-    // and 6 stages measured slower: profiles/r02/bench_sweep_cfg*.json)
-    return launch_tile_cfg<32, 8, 4, 2>(to_dev(src), to_dev(dst), *maps, nx, ny, lo, hi, alpha, sms, s);
+    // band 32, 4 rows per consumer thread, 5 stages, 2 CTAs per SM (band 16 or 64, 3 CTAs per SM
+    // measured slower: profiles/r02/bench_sweep_cfg*.json; 4 / 5 / 6 stages at 2 CTAs per SM:
+    // 0.757 / 0.768 / 0.765 of HBM on the C2 e2e step, three alternating runs)
+    return launch_tile_cfg<32, 8, 5, 2>(to_dev(src), to_dev(dst), *maps, nx, ny, lo, hi, alpha, sms, s);
   const int npairs = nx / 2;
   const int gx = (npairs + 127) / 128;
   // rows per thread: must divide every view's ty (the dense slab's is ny,
