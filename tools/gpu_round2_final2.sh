@@ -3,7 +3,7 @@
 # sanitizers, the default bench line, the ncu launch list of the same
 # command, per-kernel DRAM traffic, --set full captures of the band kernels,
 # the Fig. 5 sweep and CUPTI timelines.
-O=gpurun_out/r2f3
+O=gpurun_out/r2f4
 mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" || exit 1
 timeout 2400 python -m pytest tests -m gpu -q 2>&1 | tail -3 > $O/gputests.txt; cat $O/gputests.txt
