@@ -110,6 +110,25 @@ def test_c2_wavefront_fig5_path():
         _check_cone(d, gdims, td, 64, blocks)
 
 
+@pytest.mark.parametrize("T_", [130, 131])
+def test_split_large_T_schedule_full_plane_bit_exact(T_):
+    """A fresh upload at T beyond the wavefront's reach on a 512 x 64 x 512
+    grid (64^3 tiles): wavefront of 64 levels during the
+    upload, the middle steps two per kernel, a wavefront of the last 64 (65)
+    levels during the download (last_schedule 8); every cell against the
+    OpenMP twin of the oracle, bit-exact."""
+    import os
+    dims, td = (512, 64, 512), (64, 64, 64)
+    u0 = synth.uniform_grid(*dims, 41)
+    with T.Domain(dims, td) as d:
+        d.load(u0)
+        d.run(T.heat7(ALPHA), T_, 4)
+        out = d.store()
+        assert d.get_info()["last_schedule"] == 8
+    ref = oracle.heat_c(u0, ALPHA, T_, threads=max(1, min(16, os.cpu_count() or 1)))
+    assert np.array_equal(out, ref)
+
+
 @pytest.mark.parametrize("two_step", [0, -1])
 def test_c2_value_path_persistent_resident(two_step):
     """C2 512^3, 64^3 tiles, 4 streams: the first run after the upload is the
