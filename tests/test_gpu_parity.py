@@ -528,6 +528,16 @@ def test_wavefront_growing_T_on_one_domain_bit_exact(wave):
             assert np.array_equal(out, oracle.heat_c(u0, ALPHA, T_)), T_
 
 
+@pytest.mark.parametrize("two_step", [0, 1])
+def test_band2_with_ghost2_domains_bit_exact(two_step):
+    """Ghost-2 domains 512 wide: resident runs take heat2_band (faces left
+    stale), the next face-reading run (the layered first phase, heat7x2
+    passes with two_step = 1, the odd step) re-extracts depth-2 faces."""
+    dims, td = (512, 64, 64), (64, 32, 16)
+    out, ref, info, st = _heat(dims, td, 12, runs=[3, 4, 5], ghost=2, two_step=two_step)
+    assert np.array_equal(out, ref), np.abs(out - ref).max()
+
+
 @pytest.mark.parametrize("T_", [70, 73])
 def test_large_T_split_wavefront_bit_exact(T_):
     """Fresh upload at large T: wavefront during the upload, two-step passes,
