@@ -89,7 +89,7 @@ __global__ void __launch_bounds__(b2::NT, 1)
   // refilled only after the block barrier that follows every thread's last
   // read of it, so no empty-slot mbarrier is needed (the barrier orders those
   // reads before this thread's async-proxy writes, fence.proxy.async below)
-  int qz = nz - 2, qzl = qz % tz, qzt = qz / tz, qs = 0;  // next plane: z, in-tile z, layer, slot
+  int qz = ((-2 % nz) + nz) % nz, qzl = qz % tz, qzt = qz / tz, qs = 0;  // next plane (z, in-tile z, layer), slot
   auto issue = [&]() {
     double* d = stage + (size_t)qs * STAGE;
     fence_proxy_async();

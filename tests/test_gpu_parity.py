@@ -448,7 +448,9 @@ def test_wavefront_bit_exact(dims, td, T, wave):
                                           ((512, 512, 64), (64, 64, 64), [1, 10]),
                                           ((512, 20, 16), (64, 20, 4), [2, 5]),     # one tile row, thin layers
                                           ((512, 12, 6), (64, 4, 3), [4]),          # bands = tile rows, nz = 6
-                                          ((512, 40, 9), (64, 8, 9), [1, 6])])      # 5 tile rows, one layer
+                                          ((512, 40, 9), (64, 8, 9), [1, 6]),       # 5 tile rows, one layer
+                                          ((512, 4, 2), (64, 4, 1), [2, 3]),        # one band, nz = 2
+                                          ((512, 8, 1), (64, 8, 1), [1, 4])])       # nz = 1 (z neighbours = self)
 def test_band2_resident_bit_exact(dims, td, runs):
     """Resident periodic runs 512 cells wide: two steps per kernel over the
     whole grid (heat2_band — full-width bands, 5-D TMA boxes, both levels in
