@@ -141,7 +141,8 @@ def test_resident_multiple_runs_and_dirichlet():
 
 @pytest.mark.parametrize("dims,td,runs,ns", [((512, 8, 16), (64, 4, 8), [1, 4, 3, 2], 2),
                                              ((512, 12, 12), (64, 4, 4), [2, 5], 3),
-                                             ((512, 4, 8), (64, 4, 8), [3, 6], 1)])
+                                             ((512, 4, 8), (64, 4, 8), [3, 6], 1),
+                                             ((512, 4, 1), (64, 4, 1), [1, 4], 2)])   # nz = 1
 def test_band2_resident_runs_replay_to_oracle(dims, td, runs, ns):
     """Resident periodic runs 512 cells wide take two steps per kernel over the
     whole grid (heat2_band, TILE_OP_BAND2; an odd step the face-ghost single
