@@ -410,7 +410,8 @@ def test_stream_through_bit_exact(dims, td, T):
                                        ((64, 64, 64), (32, 32, 8), 7), ((96, 64, 160), (32, 32, 32), 1),
                                        ((64, 32, 512), (32, 32, 64), 100), ((512, 64, 128), (64, 64, 64), 16),
                                        ((512, 32, 256), (64, 32, 32), 20), ((512, 64, 384), (64, 64, 64), 48),
-                                       ((512, 16, 512), (64, 16, 64), 100), ((512, 32, 256), (64, 32, 32), 21)])
+                                       ((512, 16, 512), (64, 16, 64), 100), ((512, 32, 256), (64, 32, 32), 21),
+                                       ((512, 4, 128), (64, 4, 16), 10), ((512, 12, 192), (64, 4, 32), 33)])
 @pytest.mark.parametrize("wave", [1, 2, 3])
 def test_wavefront_bit_exact(dims, td, T, wave):
     """Fresh-upload runs on the time-skewed wavefront (forced): chunks of
@@ -476,6 +477,7 @@ def test_band2_resident_bit_exact(dims, td, runs):
 
 
 @pytest.mark.parametrize("dims,td,T_", [((512, 64, 256), (64, 64, 32), 10), ((512, 32, 192), (64, 32, 16), 5),
+                                         ((512, 4, 128), (64, 4, 16), 7),
                                          ((512, 64, 128), (64, 64, 64), 2), ((512, 128, 256), (64, 64, 64), 13)])
 def test_stream_through_two_sweeps_bit_exact(dims, td, T_):
     """Fresh-upload stream-through on grids 512 wide with two_step = 1: two sweeps per kernel
