@@ -532,6 +532,34 @@ def test_wavefront_growing_T_on_one_domain_bit_exact(wave):
             assert np.array_equal(out, oracle.heat_c(u0, ALPHA, T_)), T_
 
 
+@pytest.mark.parametrize("case", range(40))
+def test_band_kernels_random_shapes_bit_exact(case):
+    """Seeded random 512-wide shapes and run sequences through the default
+    schedules (fresh uploads: stream-through / two-level wavefront / split
+    large-T; resident: heat2_band, odd steps on the face-ghost path), every
+    stored grid against the oracle, bit-exact."""
+    import random
+    rng = random.Random(1000 + case)
+    ny = rng.choice([4, 8, 12, 16, 24, 32, 64])
+    ty = rng.choice([t for t in range(4, ny + 1, 4) if ny % t == 0])
+    nz = rng.choice([1, 2, 3, 8, 24, 48, 96, 128, 192])
+    tz = rng.choice([t for t in range(1, nz + 1) if nz % t == 0 and t <= 64])
+    dims, td = (512, ny, nz), (64, ty, tz)
+    u = synth.uniform_grid(*dims, case)
+    total = 0
+    with T.Domain(dims, td) as d:
+        d.load(u)
+        for k in range(3):
+            steps = rng.choice([1, 2, 3, 5, 8, 13, 21, 34, 40, 70])
+            d.run(T.heat7(), steps, rng.choice([1, 2, 4]))
+            total += steps
+            sched = d.get_info()["last_schedule"]
+            out = d.store()
+            assert np.array_equal(out, oracle.heat_c(u, ALPHA, total)), (dims, td, total, sched)
+            if rng.random() < 0.5:   # the next run starts from the host store again
+                d.invalidate()
+
+
 @pytest.mark.parametrize("two_step", [0, 1])
 def test_band2_with_ghost2_domains_bit_exact(two_step):
     """Ghost-2 domains 512 wide: resident runs take heat2_band (faces left
