@@ -639,6 +639,37 @@ def test_large_T_split_wavefront_replays(T_):
     assert st["bytes_h2d"] == cells * 8 and st["bytes_d2h"] == cells * 8
 
 
+@pytest.mark.parametrize("case", range(80))
+def test_random_shapes_and_options_replay_to_oracle(case):
+    """Seeded random small shapes, ghost widths, boundary conditions, device
+    budgets and schedule options; the dry-run traces of a few runs replayed
+    in random valid orders give the oracle bit-exactly."""
+    import random
+    rng = random.Random(700 + case)
+    def dim():
+        n = rng.choice([8, 16, 24, 32])
+        return n, rng.choice([t for t in (4, 8, 16) if n % t == 0])
+    (nx, tx), (ny, ty), (nz, tz) = dim(), dim(), dim()
+    dims, td = (nx, ny, nz), (tx, ty, tz)
+    bc = rng.choice(["periodic", "periodic", "dirichlet"])
+    ghost = rng.choice([1, 1, 2])
+    kw = {"wavefront": rng.choice([-1, 0, 1, 2, 3]), "stream_through": rng.choice([-1, 0, 1]),
+          "two_step": rng.choice([-1, 0, 1])}
+    if rng.random() < 0.4:
+        kw["sched"] = "stream"
+        try:
+            kw["device_budget_bytes"] = _budget_for(dims, td, rng.choice([3, 4, 6]), sched="stream", bc=bc,
+                                                    ghost=ghost)
+        except Exception:
+            pytest.skip("no stream budget for this shape")
+    runs = [rng.choice([1, 2, 3, 5]) for _ in range(rng.choice([1, 2, 3]))]
+    try:
+        T.Domain(dims, td, dry_run=True, bc=bc, ghost=ghost, **kw).free()
+    except T.TileError:
+        pytest.skip("shape not accepted")
+    _run_and_replay(dims, td, runs, rng.choice([1, 2, 3]), seeds=(case,), bc=bc, ghost=ghost, **kw)
+
+
 def T_run_dry(dims, td, steps, ns, **kw):
     d = T.Domain(dims, td, dry_run=True, **kw)
     d.load(np.zeros(dims[::-1]))
