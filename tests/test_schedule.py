@@ -670,6 +670,28 @@ def test_random_shapes_and_options_replay_to_oracle(case):
     _run_and_replay(dims, td, runs, rng.choice([1, 2, 3]), seeds=(case,), bc=bc, ghost=ghost, **kw)
 
 
+@pytest.mark.parametrize("case", range(16))
+def test_random_band_shapes_replay_to_oracle(case):
+    """Seeded random 512-wide shapes (the band kernels' domain: heat2_band,
+    the two-level wavefront, the split large-T schedule, two sweeps per
+    stream-through kernel with two_step = 1) and run sequences, replayed."""
+    import random
+    rng = random.Random(900 + case)
+    ny = rng.choice([4, 8, 12])
+    ty = rng.choice([t for t in (4, 8, 12) if ny % t == 0])
+    nz = rng.choice([8, 16, 32, 64, 96, 128])
+    tz = rng.choice([t for t in (2, 4, 8, 16, 32) if nz % t == 0])
+    dims, td = (512, ny, nz), (64, ty, tz)
+    kw = {"two_step": rng.choice([0, 0, 1])}
+    runs = [rng.choice([1, 2, 3, 5, 8, 20, 40, 70]) for _ in range(rng.choice([1, 2]))]
+    try:
+        T.Domain(dims, td, dry_run=True, **kw).free()
+    except T.TileError:
+        pytest.skip("shape not accepted")
+    d = _run_and_replay(dims, td, runs, rng.choice([1, 2, 4]), seeds=(case,), **kw)
+    assert d.get_info()["last_schedule"] in (1, 2, 6, 7, 8)
+
+
 def T_run_dry(dims, td, steps, ns, **kw):
     d = T.Domain(dims, td, dry_run=True, **kw)
     d.load(np.zeros(dims[::-1]))
