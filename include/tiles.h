@@ -379,6 +379,35 @@ tile_status tile_host_region(tile_domain* dom, int64_t tile_id, int32_t mode, do
  * shell reaches another rank. */
 tile_status tile_host_ghosts(tile_domain* dom, int64_t tile_id, double* out, int64_t out_len);
 
+/* GPU-disabled iteration (§IV.B.5: the paper's compute(tile, lambda)
+ * with the tile iterator's GPU flag off, "no change in the source code for
+ * both CPU and GPU executions"; the regions' newest data comes to the
+ * host first, waited for as P:L86 requires; ghost cells of regions on
+ * the host are updated on the host). For each tile id in ids[0..n) (ids
+ * NULL: every rank-local tile in id order) the library calls, on the calling
+ * thread,
+ *   fn(ctx, tile_id, tile, shell, tile_dims, origin, ghost)
+ * tile      = the tile's interior in the pinned host store ([tz][ty][tx], x
+ *             fastest), writable when mode == TILE_HOST_WRITE;
+ * shell     = with ghosted != 0, the tile and its g-deep shell as
+ *             tile_host_ghosts fills it ((tz+2g)(ty+2g)(tx+2g), library-owned,
+ *             valid during the call); every listed tile's shell is gathered
+ *             before the first call, so an update written in place reads only
+ *             old values through the shells (Jacobi order); NULL otherwise;
+ * tile_dims = (tx, ty, tz); origin = the global (x, y, z) of tile[0].
+ * The library runs no arithmetic on the cells itself: fn is the caller's CPU
+ * code (the paper's lambda); every library cell update stays on the GPU.
+ * READ leaves the device copies valid; WRITE hands the host the newest data
+ * (device copies are dropped, as tile_mark_host_dirty; the next tile_run
+ * re-uploads). Errors: TILE_EINVAL (null fn, a bad id or mode, n < 0; no
+ * side effects), TILE_ENOMEM_HOST (the shells), TILE_EINVAL from the gather
+ * of a z-slab rank's end tiles (their shells live on another rank, checked
+ * before any call), CUDA errors of the write-back poison the handle. */
+typedef void (*tile_host_fn)(void* ctx, int64_t tile_id, double* tile, const double* shell,
+                             const int64_t tile_dims[3], const int64_t origin[3], int32_t ghost);
+tile_status tile_host_compute(tile_domain* dom, const int64_t* ids, int64_t n, int32_t mode,
+                              int32_t ghosted, tile_host_fn fn, void* ctx);
+
 /* Enqueue `steps` steps of kernel k over every tile (no sync
  * after issue). nstreams in [1, 64] streams carry transfers and kernels
  * (P:L81-L84). Returns once all work is enqueued; may block only for

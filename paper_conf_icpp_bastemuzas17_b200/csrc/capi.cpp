@@ -82,6 +82,25 @@ tile_status tile_host_ghosts(tile_domain* h, int64_t tile_id, double* out, int64
   return finish(h, tiles::domain_host_ghosts(*h->d, tile_id, out));
 }
 
+tile_status tile_host_compute(tile_domain* h, const int64_t* ids, int64_t n, int32_t mode, int32_t ghosted,
+                              tile_host_fn fn, void* ctx) {
+  CHECK_DOM(h);
+  const tiles::Geometry& G = h->d->G;
+  if (!fn || n < 0 || (n > 0 && !ids)) return fail(TILE_EINVAL, "null fn, n < 0 or null ids");
+  if (mode != TILE_HOST_READ && mode != TILE_HOST_WRITE) return fail(TILE_EINVAL, "bad host mode");
+  for (int64_t i = 0; ids && i < n; ++i)
+    if (ids[i] < 0 || ids[i] >= G.ntiles) return fail(TILE_EINVAL, "bad tile id");
+  if (ghosted && G.nranks > 1)
+    for (int64_t i = 0; i < (ids ? n : G.ntiles); ++i) {
+      int64_t c[3];
+      G.tile_coords(ids ? ids[i] : i, &c[0], &c[1], &c[2]);
+      const bool lo = c[2] == 0 && (G.bc == TILE_BC_PERIODIC || G.rank > 0);
+      const bool hi = c[2] == G.n[2] - 1 && (G.bc == TILE_BC_PERIODIC || G.rank < G.nranks - 1);
+      if (lo || hi) return fail(TILE_EINVAL, "ghost cells of a listed tile live on another rank");
+    }
+  return finish(h, tiles::domain_host_compute(*h->d, ids, ids ? n : G.ntiles, mode, ghosted, fn, ctx));
+}
+
 tile_status tile_mark_host_dirty(tile_domain* h) {
   CHECK_DOM(h);
   Domain& d = *h->d;

@@ -2267,6 +2267,56 @@ Status domain_host_ghosts(Domain& d, int64_t t, double* out) {
   return Status::ok();
 }
 
+// GPU-disabled iteration (§IV.B.5: compute(tile, lambda) with the
+// iterator's GPU flag off; the regions' newest data is brought to the
+// host first; their ghost cells are updated on the host). The
+// library only moves data and calls the caller's function: no cell update of
+// its own runs on the CPU. With `ghosted`, every listed tile's shell is
+// gathered before the first call, so an update that writes its tile in
+// place still reads only old values through the shells (Jacobi order, as
+// the paper's separate old/new tile arrays give). WRITE hands the host store
+// the newest data: device copies are dropped (as tile_mark_host_dirty).
+Status domain_host_compute(Domain& d, const int64_t* ids, int64_t n, int mode, int ghosted, tile_host_fn fn,
+                           void* ctx) {
+  const Geometry& G = d.G;
+  std::vector<int64_t> list;
+  if (ids) list.assign(ids, ids + n);
+  else for (int64_t k = 0; k < G.ntiles; ++k) list.push_back(k);
+  bool dirty = d.host_pending || d.in_flight;
+  for (int64_t k = 0; k < G.ntiles && !dirty; ++k) dirty = d.tile_dirty[k] && d.tile_slot[k] >= 0;
+  if (dirty) {
+    Status r = domain_sync(d);
+    if (r.bad()) return r;
+  }
+  const int64_t g = G.ghost;
+  const int64_t box = (G.t[0] + 2 * g) * (G.t[1] + 2 * g) * (G.t[2] + 2 * g);
+  std::vector<double> shells;
+  if (ghosted) {
+    try {
+      shells.resize((size_t)(box * (int64_t)list.size()));
+    } catch (const std::bad_alloc&) {
+      return make_err(TILE_ENOMEM_HOST, "host ghost shells for the listed tiles");
+    }
+    for (size_t i = 0; i < list.size(); ++i) {
+      Status r = domain_host_ghosts(d, list[i], shells.data() + i * (size_t)box);
+      if (r.bad()) return r;
+    }
+  }
+  for (size_t i = 0; i < list.size(); ++i) {
+    int64_t c[3];
+    G.tile_coords(list[i], &c[0], &c[1], &c[2]);
+    const int64_t origin[3] = {c[0] * G.t[0], c[1] * G.t[1], c[2] * G.t[2] + G.zoff};
+    fn(ctx, list[i], d.host_tile(list[i]), ghosted ? shells.data() + i * (size_t)box : nullptr, G.t, origin,
+       (int32_t)g);
+  }
+  if (mode == TILE_HOST_WRITE) {
+    d.host_faces_valid = false;
+    for (auto& x : d.tile_dirty) x = 0;
+    return domain_invalidate(d);
+  }
+  return Status::ok();
+}
+
 Status domain_load(Domain& d, const double* src) {
   if (d.in_flight) {
     Status r = domain_sync(d);

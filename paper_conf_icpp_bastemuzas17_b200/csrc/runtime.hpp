@@ -358,6 +358,8 @@ Status domain_store(Domain& d, double* dst);
 Status domain_invalidate(Domain& d);
 Status domain_host_region(Domain& d, int64_t tile, int mode, double** ptr);
 Status domain_host_ghosts(Domain& d, int64_t tile, double* out);
+Status domain_host_compute(Domain& d, const int64_t* ids, int64_t n, int mode, int ghosted, tile_host_fn fn,
+                           void* ctx);
 Status domain_free(Domain* d);
 Status domain_setup(Domain& d);
 void host_extract_faces(const Geometry& G, const double* host, double* const faces[6]);

@@ -102,6 +102,7 @@ _sig = {
     "tile_mark_host_dirty": ([_P], ctypes.c_int),
     "tile_host_region": ([_P, ctypes.c_int64, ctypes.c_int32, ctypes.POINTER(_P)], ctypes.c_int),
     "tile_host_ghosts": ([_P, ctypes.c_int64, _P, ctypes.c_int64], ctypes.c_int),
+    "tile_host_compute": ([_P, _I64P, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, _P, _P], ctypes.c_int),
     "tile_run": ([_P, ctypes.POINTER(TileKernel), ctypes.c_int32, ctypes.c_int32], ctypes.c_int),
     "tile_sync": ([_P], ctypes.c_int),
     "tile_store": ([_P, _P], ctypes.c_int),
@@ -130,6 +131,9 @@ _sig = {
     "tile_user_stencil_create": ([ctypes.c_char_p, ctypes.c_char_p, ctypes.POINTER(_P)], ctypes.c_int),
 }
 EXPORTED = tuple(_sig)
+# tile_host_fn(ctx, tile_id, tile, shell, tile_dims, origin, ghost)
+HOST_FN = ctypes.CFUNCTYPE(None, _P, ctypes.c_int64, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double),
+                           _I64P, _I64P, ctypes.c_int32)
 for _name, (_args, _res) in _sig.items():
     _f = getattr(_lib, _name)
     _f.argtypes = _args
@@ -348,6 +352,41 @@ class Domain:
         out = np.empty((tz + 2 * g, ty + 2 * g, tx + 2 * g))
         _check(tile_host_ghosts(self._h, tile_id, out.ctypes.data, out.size), "tile_host_ghosts")
         return out
+
+    def host_compute(self, fn, tiles=None, write=False, ghosted=False):
+        """GPU-disabled iteration (P:L92 compute(tile, lambda) on the CPU;
+        P:L90): calls fn(tile_id, tile, shell, origin) for each tile
+        (default: all) with `tile` a NumPy view (tz, ty, tx) of the tile in the
+        pinned host store (writable with write=True) and `shell` the tile plus
+        its ghost shell gathered on the host before the first call
+        (ghosted=True; else None). fn is the caller's CPU code: the library
+        itself only moves data."""
+        err = []
+
+        def tramp(_ctx, tid, tp, sp, dims, origin, g):
+            try:
+                tx, ty, tz = dims[0], dims[1], dims[2]
+                tile = np.ctypeslib.as_array(tp, shape=(tz, ty, tx))
+                if not write:
+                    tile = tile.view()
+                    tile.flags.writeable = False
+                shell = None
+                if sp:
+                    shell = np.ctypeslib.as_array(sp, shape=(tz + 2 * g, ty + 2 * g, tx + 2 * g)).view()
+                    shell.flags.writeable = False
+                fn(tid, tile, shell, (origin[0], origin[1], origin[2]))
+            except BaseException as e:  # noqa: BLE001  (re-raised after the C call returns)
+                if not err:
+                    err.append(e)
+
+        cb = HOST_FN(tramp)
+        ids = None if tiles is None else np.ascontiguousarray(tiles, dtype=np.int64)
+        n = 0 if ids is None else ids.size
+        ptr = None if ids is None else ids.ctypes.data_as(_I64P)
+        _check(tile_host_compute(self._h, ptr, n, 1 if write else 0, 1 if ghosted else 0,
+                                 ctypes.cast(cb, _P), None), "tile_host_compute")
+        if err:
+            raise err[0]
 
     def run(self, kernel, steps, nstreams=4):
         _check(tile_run(self._h, ctypes.byref(kernel), steps, nstreams), "tile_run")

@@ -124,3 +124,105 @@ def test_host_region_and_ghosts_gpu(sched):
         d.run(T.heat7(ALPHA), 2, 2)
         out = d.store()
     assert np.array_equal(out, oracle.heat_c(mod, ALPHA, 2))
+
+
+def _cpu_heat_step(alpha):
+    """The caller's CPU code (the paper's lambda in a GPU-disabled iteration,
+    P:L92): one 7-point Jacobi update of a tile from its host shell, written
+    in place, in the oracle's order of operations (heat_np)."""
+    def fn(tid, tile, shell, origin):
+        g = (shell.shape[0] - tile.shape[0]) // 2
+        c = shell[g:-g, g:-g, g:-g]
+        xm, xp = shell[g:-g, g:-g, g - 1:-g - 1], shell[g:-g, g:-g, g + 1:shell.shape[2] - g + 1]
+        ym, yp = shell[g:-g, g - 1:-g - 1, g:-g], shell[g:-g, g + 1:shell.shape[1] - g + 1, g:-g]
+        zm, zp = shell[g - 1:-g - 1, g:-g, g:-g], shell[g + 1:shell.shape[0] - g + 1, g:-g, g:-g]
+        s = ((xm + xp) + (ym + yp)) + (zm + zp)
+        tile[:] = c + alpha * (s - 6.0 * c)
+    return fn
+
+
+@pytest.mark.parametrize("dims,td,g", [((16, 8, 12), (8, 4, 4), 1), ((12, 8, 8), (4, 4, 4), 2)])
+def test_host_compute_jacobi_step_equals_the_oracle_dry(dims, td, g):
+    """GPU-disabled iteration over every tile with ghosted shells: the shells
+    are gathered before the first call, so a CPU update written in place
+    still reads only old values — the result is the oracle's heat step
+    (P:L92 compute on the CPU, P:L96 host ghost update)."""
+    u = synth.uniform_grid(*dims, 5)
+    d = T.Domain(dims, td, ghost=g, dry_run=True)
+    d.load(u)
+    d.host_compute(_cpu_heat_step(ALPHA), write=True, ghosted=True)
+    assert np.array_equal(d.store(), oracle.heat_c(u, ALPHA, 1))
+
+
+def test_host_compute_jacobi_step_dirichlet_dry():
+    """Dirichlet: the shells carry the fixed boundary faces."""
+    dims, td = (16, 8, 8), (8, 4, 4)
+    ext = synth.uniform_grid(18, 10, 10, 7)
+    d = T.Domain(dims, td, bc="dirichlet", dry_run=True)
+    d.load(ext)
+    d.host_compute(_cpu_heat_step(ALPHA), write=True, ghosted=True)
+    ref = oracle.heat_c(ext, ALPHA, 1, oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+    assert np.array_equal(d.store()[1:-1, 1:-1, 1:-1], ref)
+
+
+def test_host_compute_calls_origins_subset_and_read_only_dry():
+    dims, td = (16, 8, 12), (8, 4, 4)
+    u = synth.uniform_grid(*dims, 6)
+    d = T.Domain(dims, td, dry_run=True)
+    d.load(u)
+    seen = []
+
+    def look(tid, tile, shell, origin):
+        x, y, z = origin
+        assert np.array_equal(tile, u[z:z + 4, y:y + 4, x:x + 8])
+        assert shell is None and not tile.flags.writeable
+        seen.append((tid, origin))
+
+    d.host_compute(look, tiles=[5, 2])
+    assert [s[0] for s in seen] == [5, 2]
+    assert seen[0][1] == (8, 0, 4) and seen[1][1] == (0, 4, 0)
+
+    def add_one(tid, tile, shell, origin):
+        tile += 1.0
+
+    d.host_compute(add_one, tiles=[1], write=True)
+    exp = u.copy()
+    exp[0:4, 0:4, 8:16] += 1.0
+    assert np.array_equal(d.store(), exp)
+
+
+def test_host_compute_errors_dry():
+    d = T.Domain((16, 8, 12), (8, 4, 4), dry_run=True)
+    d.load(np.zeros((12, 8, 16)))
+    with pytest.raises(T.TileError) as e:
+        d.host_compute(lambda *a: None, tiles=[99])
+    assert e.value.code == 1  # TILE_EINVAL
+    with pytest.raises(ZeroDivisionError):  # the caller's exception comes back
+        d.host_compute(lambda *a: 1 / 0, tiles=[0])
+    calls = []
+    with pytest.raises(T.TileError):
+        d.host_compute(lambda *a: calls.append(a), tiles=[0, -1])
+    assert calls == []  # EINVAL has no side effects
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("sched", ["resident", "stream"])
+def test_host_compute_interleaved_with_gpu_steps(sched):
+    """The uniform API's two sides in one run: T1 steps on the GPU, one step
+    by the caller's CPU code in a GPU-disabled iteration (newest data
+    brought to the host first; ghosts on the host), T2 more on
+    the GPU — bit-exact against the oracle's T1 + 1 + T2 steps."""
+    if not cuda_available():
+        pytest.skip("no CUDA device")
+    dims, td = (64, 32, 48), (32, 16, 16)
+    u = synth.uniform_grid(*dims, 43)
+    kw = {"stream_through": -1}
+    if sched == "stream":
+        kw.update(sched="stream", device_budget_bytes=_budget_for(dims, td, 5, sched="stream", stream_through=-1))
+    with T.Domain(dims, td, **kw) as d:
+        d.load(u)
+        d.run(T.heat7(ALPHA), 3, 2)
+        d.host_compute(_cpu_heat_step(ALPHA), write=True, ghosted=True)
+        d.run(T.heat7(ALPHA), 2, 2)
+        out = d.store()
+    assert np.array_equal(out, oracle.heat_c(u, ALPHA, 6))

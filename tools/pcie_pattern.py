@@ -73,6 +73,19 @@ def main(out):
                 "gbs_best": gb / (min(spans) / 1e3), "gbs_median": gb / (statistics.median(spans) / 1e3)}
 
     res = {}
+    if len(sys.argv) > 2 and sys.argv[2] == "rows":
+        # 2-D duplex by row size (chunk = 64 rows), rounds interleaved so that
+        # drift of the link rate hits every variant alike
+        cases = [(64 * MB, 32 * MB), (16 * MB, 16 * MB), (8 * MB, 8 * MB), (4 * MB, 4 * MB), (2 * MB, 2 * MB),
+                 (8 * MB, 32 * MB), (64 * MB, 8 * MB)]
+        for rnd in range(4):
+            for ch_in, ch_out in cases:
+                key = f"2d_rows_in{ch_in // NT // 1024}k_out{ch_out // NT // 1024}k"
+                res.setdefault(key, []).append(timed(("h2d", "d2h"), "2d", ch_in, ch_out, reps=3)["gbs_median"])
+        for k, v in res.items():
+            print(k, [round(x, 1) for x in v], "median", round(statistics.median(v), 1), flush=True)
+        json.dump(res, open(out, "w"), indent=1)
+        return
     for pattern in ("1d", "2d"):
         for ch_in, ch_out in ((64 * MB, 32 * MB), (32 * MB, 32 * MB), (8 * MB, 8 * MB)):
             key = f"{pattern}_in{ch_in // MB}_out{ch_out // MB}"
