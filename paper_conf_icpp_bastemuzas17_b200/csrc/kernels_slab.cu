@@ -352,6 +352,10 @@ __global__ void __launch_bounds__(TileCfg<BY, RPP, S>::NT + 32, MB)
     // before the first load (consumers write only after consuming a stage,
     // so this also orders their stores after the previous grid's reads)
     asm volatile("griddepcontrol.wait;" ::: "memory");
+    // L2 policy of the staged loads (st_mode >> 4, TILES_SWEEP_LD): 0 none,
+    // 1 evict_first (a level's input is dead after the sweep), 2 evict_last
+    const int ldm = st_mode >> 4;
+    const uint64_t lpol = ldm == 2 ? policy_evict_last() : policy_evict_first();
     uint32_t g = 0;
     for (int64_t pp = pb; pp < pe;) {
       const int64_t col = pp / np;
@@ -372,9 +376,15 @@ __global__ void __launch_bounds__(TileCfg<BY, RPP, S>::NT + 32, MB)
         const double* pz = Sv.P(z);
         fence_proxy_async();
         mbar_expect_tx(&full[st], C::BYTES);
-        bulk_g2s(dst + TX, pz + oband, (uint32_t)BY * TX * 8, &full[st]);
-        bulk_g2s(dst, pz + om, TX * 8, &full[st]);
-        bulk_g2s(dst + (BY + 1) * TX, pz + op, TX * 8, &full[st]);
+        if (ldm) {
+          bulk_g2s_hint(dst + TX, pz + oband, (uint32_t)BY * TX * 8, &full[st], lpol);
+          bulk_g2s_hint(dst, pz + om, TX * 8, &full[st], lpol);
+          bulk_g2s_hint(dst + (BY + 1) * TX, pz + op, TX * 8, &full[st], lpol);
+        } else {
+          bulk_g2s(dst + TX, pz + oband, (uint32_t)BY * TX * 8, &full[st]);
+          bulk_g2s(dst, pz + om, TX * 8, &full[st]);
+          bulk_g2s(dst + (BY + 1) * TX, pz + op, TX * 8, &full[st]);
+        }
         const double* a = pz + oxl;
         const double* b = pz + oxr;
         const int ka = (a >= maps.base[1] && a < maps.end[1]) ? 1 : 0;
@@ -392,7 +402,8 @@ __global__ void __launch_bounds__(TileCfg<BY, RPP, S>::NT + 32, MB)
   const bool xl_edge = c2 == 0, xr_edge = c2 == C::HALF - 1;
   // output stores: streaming (evict-first; 0) or kept in L2 for the next
   // sweep's reads (1 evict_normal, 2 evict_last)
-  const uint64_t spol = st_mode == 2 ? policy_evict_last() : policy_evict_normal();
+  const int stm = st_mode & 15;
+  const uint64_t spol = stm == 2 ? policy_evict_last() : policy_evict_normal();
   // the x-halo cell of this thread's rows: left box column 1 (x = 63 of the
   // left tile), right box column 0 (x = 0 of the right tile)
   const int hoff = xl_edge ? C::XH + 2 * r0 + 1 : C::XH + 2 * BY + 2 * r0;
@@ -444,7 +455,7 @@ __global__ void __launch_bounds__(TileCfg<BY, RPP, S>::NT + 32, MB)
         double2 v;
         v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm[j].x, zp.x, alpha);
         v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm[j].y, zp.y, alpha);
-        if (st_mode == 0) stg2_stream(od + j * ostep, v);
+        if (stm == 0) stg2_stream(od + j * ostep, v);
         else st2_hint(od + j * ostep, v, spol);
         zm[j] = c;
         zc[j] = zp;
@@ -479,7 +490,8 @@ static cudaError_t launch_tile_cfg(const ViewDev& Sv, const ViewDev& Dv, const S
   const int64_t grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * occ, P / 6));
   static const int st_mode = [] {
     const char* e = getenv("TILES_SWEEP_ST");
-    return e ? atoi(e) : 0;
+    const char* l = getenv("TILES_SWEEP_LD");
+    return (e ? atoi(e) : 0) | ((l ? atoi(l) : 0) << 4);
   }();
   static const int pdl = [] {
     const char* e = getenv("TILES_SWEEP_PDL");
