@@ -226,3 +226,24 @@ def test_host_compute_interleaved_with_gpu_steps(sched):
         d.run(T.heat7(ALPHA), 2, 2)
         out = d.store()
     assert np.array_equal(out, oracle.heat_c(u, ALPHA, 6))
+
+
+def test_host_compute_z_slab_rank_shells_dry():
+    """z-slab ranks: ghosted host compute of a middle tile layer works (its
+    shell is inside the rank's slab: the oracle's step there); an end layer's
+    shell lives on another rank — TILE_EINVAL before any call."""
+    G, dims, td = 2, (16, 8, 24), (8, 4, 4)
+    u = synth.uniform_grid(*dims, 11)
+    nzl = dims[2] // G
+    d = T.Domain(dims, td, nranks=G, rank=1, dry_run=True)
+    d.load(u[nzl:])
+    mid = [k for k in range(d.info["ntiles"]) if 0 < k // 4 < nzl // 4 - 1]
+    d.host_compute(_cpu_heat_step(ALPHA), tiles=mid, write=True, ghosted=True)
+    ref = oracle.heat_c(u, ALPHA, 1)[nzl:]
+    got = d.store()
+    assert np.array_equal(got[4:8], ref[4:8])          # the middle layer updated
+    assert np.array_equal(got[:4], u[nzl:][:4])        # the end layers untouched
+    calls = []
+    with pytest.raises(T.TileError) as e:
+        d.host_compute(lambda *a: calls.append(a), tiles=[0], ghosted=True)
+    assert e.value.code == 1 and calls == []
