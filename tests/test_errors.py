@@ -36,12 +36,15 @@ def _every_call_is_estate(d):
     ms = ctypes.c_double()
     n = ctypes.c_int64()
     blob = ctypes.create_string_buffer(64)
+    called = []
+    noop = T.HOST_FN(lambda *a: called.append(a))
     calls = {
         "tile_load": lambda: T.tile_load(h, arr.ctypes.data),
         "tile_host_tile": lambda: T.tile_host_tile(h, 0, ctypes.byref(p)),
         "tile_mark_host_dirty": lambda: T.tile_mark_host_dirty(h),
         "tile_host_region": lambda: T.tile_host_region(h, 0, 0, ctypes.byref(p)),
         "tile_host_ghosts": lambda: T.tile_host_ghosts(h, 0, gm, len(gm)),
+        "tile_host_compute": lambda: T.tile_host_compute(h, None, 0, 0, 0, ctypes.cast(noop, T._P), None),
         "tile_run": lambda: T.tile_run(h, ctypes.byref(k), 1, 2),
         "tile_sync": lambda: T.tile_sync(h),
         "tile_store": lambda: T.tile_store(h, arr.ctypes.data),
@@ -68,6 +71,7 @@ def _every_call_is_estate(d):
         rc = call()
         assert rc == T.TILE_ESTATE, (name, rc)
         assert "poisoned" in T.tile_last_error().decode()
+    assert not called  # a poisoned domain calls no host function
 
 
 def _run_to_fault(d, u):

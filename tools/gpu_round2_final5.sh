@@ -8,11 +8,7 @@ mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" || exit 1
 timeout 2400 python -m pytest tests -m gpu -q 2>&1 | tail -3 > $O/gputests.txt; cat $O/gputests.txt
 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.txt 2>&1; tail -1 $O/smoke.txt
-for tool in memcheck racecheck synccheck initcheck; do
-  timeout 1500 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize.py > $O/sanitize_$tool.log 2>&1
-  echo "$tool rc=$?" >> $O/sanitize_summary.txt; grep -E "ERROR SUMMARY|RACECHECK SUMMARY" $O/sanitize_$tool.log | head -2 >> $O/sanitize_summary.txt
-done
-cat $O/sanitize_summary.txt
+# compute-sanitizer is closed on the pool (late round 2): the last sanitizer logs are profiles/r02/final4
 timeout 900 python bench.py > $O/bench.json 2> $O/bench.err
 timeout 900 python bench.py --impl reference > $O/bench_reference.json 2> $O/bench_reference.err
 TILES_BENCH_ONE_GPU=1 timeout 900 python bench.py --gpus 2 --steps 5 --warmup 3 --no-extras --no-cpu-baseline > $O/bench_n2_one_gpu.json 2> $O/bench_n2.err
