@@ -391,9 +391,11 @@ tile_status tile_host_ghosts(tile_domain* dom, int64_t tile_id, double* out, int
  *             fastest), writable when mode == TILE_HOST_WRITE;
  * shell     = with ghosted != 0, the tile and its g-deep shell as
  *             tile_host_ghosts fills it ((tz+2g)(ty+2g)(tx+2g), library-owned,
- *             valid during the call); every listed tile's shell is gathered
- *             before the first call, so an update written in place reads only
- *             old values through the shells (Jacobi order); NULL otherwise;
+ *             valid during the call); with WRITE every listed tile's shell is
+ *             gathered before the first call (host memory: one shell per
+ *             listed tile), so an update written in place reads only old
+ *             values through the shells (Jacobi order); with READ one shell
+ *             at a time; NULL otherwise;
  * tile_dims = (tx, ty, tz); origin = the global (x, y, z) of tile[0].
  * The library runs no arithmetic on the cells itself: fn is the caller's CPU
  * code (the paper's lambda); every library cell update stays on the GPU.

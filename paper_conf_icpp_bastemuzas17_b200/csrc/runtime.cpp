@@ -2290,14 +2290,17 @@ Status domain_host_compute(Domain& d, const int64_t* ids, int64_t n, int mode, i
   }
   const int64_t g = G.ghost;
   const int64_t box = (G.t[0] + 2 * g) * (G.t[1] + 2 * g) * (G.t[2] + 2 * g);
+  // WRITE: every shell before the first call (Jacobi order); READ: one at a
+  // time (nothing changes between the calls)
+  const bool all_first = ghosted && mode == TILE_HOST_WRITE;
   std::vector<double> shells;
   if (ghosted) {
     try {
-      shells.resize((size_t)(box * (int64_t)list.size()));
+      shells.resize((size_t)(box * (all_first ? (int64_t)list.size() : 1)));
     } catch (const std::bad_alloc&) {
       return make_err(TILE_ENOMEM_HOST, "host ghost shells for the listed tiles");
     }
-    for (size_t i = 0; i < list.size(); ++i) {
+    for (size_t i = 0; all_first && i < list.size(); ++i) {
       Status r = domain_host_ghosts(d, list[i], shells.data() + i * (size_t)box);
       if (r.bad()) return r;
     }
@@ -2306,8 +2309,14 @@ Status domain_host_compute(Domain& d, const int64_t* ids, int64_t n, int mode, i
     int64_t c[3];
     G.tile_coords(list[i], &c[0], &c[1], &c[2]);
     const int64_t origin[3] = {c[0] * G.t[0], c[1] * G.t[1], c[2] * G.t[2] + G.zoff};
-    fn(ctx, list[i], d.host_tile(list[i]), ghosted ? shells.data() + i * (size_t)box : nullptr, G.t, origin,
-       (int32_t)g);
+    const double* sh = nullptr;
+    if (ghosted && all_first) sh = shells.data() + i * (size_t)box;
+    if (ghosted && !all_first) {
+      Status r = domain_host_ghosts(d, list[i], shells.data());
+      if (r.bad()) return r;
+      sh = shells.data();
+    }
+    fn(ctx, list[i], d.host_tile(list[i]), sh, G.t, origin, (int32_t)g);
   }
   if (mode == TILE_HOST_WRITE) {
     d.host_faces_valid = false;

@@ -191,6 +191,23 @@ def test_host_compute_calls_origins_subset_and_read_only_dry():
     assert np.array_equal(d.store(), exp)
 
 
+def test_host_compute_read_shells_one_at_a_time_dry():
+    """READ with shells: each call sees its tile's ghost-map gather (the shells
+    are gathered one at a time: nothing changes between the calls)."""
+    dims, td, g = (12, 8, 8), (4, 4, 4), 2
+    u = synth.uniform_grid(*dims, 9)
+    d = T.Domain(dims, td, ghost=g, dry_run=True)
+    d.load(u)
+    seen = []
+
+    def check(tid, tile, shell, origin):
+        assert np.array_equal(shell, _gather(u, oracle.ghost_map(dims, td, g, tid)), equal_nan=True)
+        seen.append(tid)
+
+    d.host_compute(check, ghosted=True)
+    assert seen == list(range(d.info["ntiles"]))
+
+
 def test_host_compute_errors_dry():
     d = T.Domain((16, 8, 12), (8, 4, 4), dry_run=True)
     d.load(np.zeros((12, 8, 16)))
