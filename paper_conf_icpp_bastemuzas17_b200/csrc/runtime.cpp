@@ -952,6 +952,12 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
     return e ? atoi(e) : 0;
   }();
   const int merge = st_h2d_merge();
+  // units uploaded one per copy at the head (TILES_ST_HEAD, default 2: the
+  // fill's units 0 and 1; more lets the first D2Hs follow unit by unit)
+  static const int head = [] {
+    const char* e = getenv("TILES_ST_HEAD");
+    return e ? std::max(0, atoi(e)) : 2;
+  }();
   const int64_t nzl = G.l[2];
   struct Copy {
     int64_t layer, p0, np;
@@ -976,7 +982,7 @@ static Status run_streamthrough(Domain& d, double alpha, int T, int S, const Str
       ++since;
       const bool last = v + 2 >= U;
       const bool regular = np_of(v) == sp.unit && !last && np_of(v + 1) == sp.unit && layer_of(v + 1) == layer_of(v);
-      if (!(v < 2 || !regular || since >= merge)) continue;
+      if (!(v < head || !regular || since >= merge)) continue;
       int64_t e = last ? zend : z0_of(v + 1);
       if (off && !last && layer_of(v + 1) == layer_of(v)) e = std::min(zend, e + T);
       if (e > f) add(f, e);

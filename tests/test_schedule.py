@@ -390,7 +390,7 @@ def test_stream_through_two_sweeps_per_kernel_replays(dims, td, T_, ns):
     assert "sweep2s" not in [op[0] for op in d3.trace()]
 
 
-@pytest.mark.parametrize("env", ["TILES_ST_OFFSET=1", "TILES_ST_H2D_MERGE=3", "TILES_ST_THIN=0"])
+@pytest.mark.parametrize("env", ["TILES_ST_OFFSET=1", "TILES_ST_H2D_MERGE=3", "TILES_ST_THIN=0", "TILES_ST_HEAD=4"])
 def test_stream_through_copy_plans_replay_to_oracle(env):
     """The stream-through's other H2D copy plans (copies cut T planes into the
     next unit; three units per copy; uniform units): the replays above in a
