@@ -1,4 +1,5 @@
 #!/bin/bash
+# (experiment script: the knob it sets was measured and reverted; kept as the record of the A/B)
 # Chained tile-column sweeps: parity (stream-through / wavefront / random shapes / full size),
 # repeated to shake out races, then A/B chain on/off on the C2 e2e step.
 O=gpurun_out/s2i

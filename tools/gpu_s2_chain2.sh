@@ -1,4 +1,5 @@
 #!/bin/bash
+# (experiment script: the knob it sets was measured and reverted; kept as the record of the A/B)
 O=gpurun_out/s2k
 mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" > $O/build.txt 2>&1 || { tail -20 $O/build.txt; exit 1; }

@@ -1,4 +1,5 @@
 #!/bin/bash
+# (experiment script: the knob it sets was measured and reverted; kept as the record of the A/B)
 # heat2_band with the split (mbarrier arrive / wait) barrier: band-kernel parity, then A/B on the resident leg.
 O=gpurun_out/s2q
 mkdir -p $O

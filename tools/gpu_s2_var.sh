@@ -1,4 +1,5 @@
 #!/bin/bash
+# (experiment script: the knob it sets was measured and reverted; kept as the record of the A/B)
 # A/B of tile-column sweep variants (TILES_SWEEP_VAR) on the C2 e2e step, alternating rounds.
 O=gpurun_out/s2h
 mkdir -p $O
