@@ -800,10 +800,19 @@ def multi_domain(Tl, dist, ws, rk, transport, *args, **kw):
 
 
 def run_c5_leg(args):
+    """C5 line on rank 0 (c5_line)."""
+    line = c5_line(args)
+    if line is not None:
+        print(json.dumps(line), flush=True)
+    return 0
+
+
+def c5_line(args):
     """C5: heat 4096^3 fp64 slab-decomposed over N GPUs (z-slabs, NCCL halo
     exchange), each rank streaming its own tiles from pinned host memory.
     With N = 1 this runs the per-GPU slab of the 8-GPU decomposition
-    (4096 x 4096 x 512) alone (z-periodic), i.e. one rank's work."""
+    (4096 x 4096 x 512) alone (z-periodic), i.e. one rank's work. Returns
+    the JSON line on rank 0, None on the others."""
     import torch
     import torch.distributed as dist
     from paper_conf_icpp_bastemuzas17_b200 import tiles as Tl
@@ -903,10 +912,9 @@ def run_c5_leg(args):
                              "unit": "GB/s", "frac": 16 * per_launch / (avg / 1e3) / 1e9 / peak, "traffic": None,
                              "kernel": f"heat7_fixed (tiles {td[0]}x{td[1]}x{td[2]})", "peak_source": src},
                 "halo_bytes_per_step": st["bytes_halo"] // max(1, args.steps), "clocks": clk.summary()}
-        print(json.dumps(line), flush=True)
     if ws > 1:
         dist.destroy_process_group()
-    return 0
+    return line if rk == 0 else None
 
 
 
@@ -1269,12 +1277,17 @@ def run_main_leg(args):
         for key, fn, kw in (("c3", c3_line, dict(n=None, T=None, nstreams=None, budget_gb=None, ghost=1,
                                                   stream_through=0, steps=2, warmup=1)),
                             ("c4", c4_line, dict(n=None, T=None, nstreams=None, K=args.K, sweep="1,2,4,8",
+                                                  steps=2, warmup=1)),
+                            # C5's per-GPU slab of the 8-GPU decomposition (4096 x 4096 x 512)
+                            ("c5", c5_line, dict(n=None, T=None, nstreams=None, tile=None, transport=args.transport,
                                                   steps=2, warmup=1))):
             try:
                 ln = fn(_ap.Namespace(**kw))
                 extras[key] = {kk: ln[kk] for kk in ("value", "unit", "ms_per_step", "config", "e2e", "overlap",
                                                       "roofline", "clocks", "stream_sweep_e2e")
                                if kk in ln}
+                if key == "c5":
+                    extras[key]["value_def"] = "per-GPU slab resident in HBM (heat7_fixed); e2e: with H2D/D2H"
             except Exception as e:  # e.g. not enough host RAM for C3's pinned store
                 extras[key] = {"error": str(e)[:300]}
 
