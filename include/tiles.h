@@ -401,7 +401,8 @@ tile_status tile_host_ghosts(tile_domain* dom, int64_t tile_id, double* out, int
  * code (the paper's lambda); every library cell update stays on the GPU.
  * READ leaves the device copies valid; WRITE hands the host the newest data
  * (device copies are dropped, as tile_mark_host_dirty; the next tile_run
- * re-uploads). Errors: TILE_EINVAL (null fn, a bad id or mode, n < 0; no
+ * re-uploads). fn must not call the library on the same domain (the
+ * iteration is in progress). Errors: TILE_EINVAL (null fn, a bad id or mode, n < 0; no
  * side effects), TILE_ENOMEM_HOST (the shells), TILE_EINVAL from the gather
  * of a z-slab rank's end tiles (their shells live on another rank, checked
  * before any call), CUDA errors of the write-back poison the handle. */
