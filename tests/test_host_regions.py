@@ -224,7 +224,8 @@ def test_host_compute_errors_dry():
 
 @pytest.mark.gpu
 @pytest.mark.parametrize("sched", ["resident", "stream"])
-def test_host_compute_interleaved_with_gpu_steps(sched):
+@pytest.mark.parametrize("bc", ["periodic", "dirichlet"])
+def test_host_compute_interleaved_with_gpu_steps(sched, bc):
     """The uniform API's two sides in one run: T1 steps on the GPU, one step
     by the caller's CPU code in a GPU-disabled iteration (newest data
     brought to the host first; ghosts on the host), T2 more on
@@ -232,17 +233,23 @@ def test_host_compute_interleaved_with_gpu_steps(sched):
     if not cuda_available():
         pytest.skip("no CUDA device")
     dims, td = (64, 32, 48), (32, 16, 16)
-    u = synth.uniform_grid(*dims, 43)
-    kw = {"stream_through": -1}
+    ext = bc == "dirichlet"
+    u = synth.uniform_grid(*((66, 34, 50) if ext else dims), 43)
+    kw = {"stream_through": -1, "bc": bc}
     if sched == "stream":
-        kw.update(sched="stream", device_budget_bytes=_budget_for(dims, td, 5, sched="stream", stream_through=-1))
+        kw.update(sched="stream",
+                  device_budget_bytes=_budget_for(dims, td, 5, sched="stream", stream_through=-1, bc=bc))
     with T.Domain(dims, td, **kw) as d:
         d.load(u)
         d.run(T.heat7(ALPHA), 3, 2)
         d.host_compute(_cpu_heat_step(ALPHA), write=True, ghosted=True)
         d.run(T.heat7(ALPHA), 2, 2)
         out = d.store()
-    assert np.array_equal(out, oracle.heat_c(u, ALPHA, 6))
+    if ext:
+        ref = oracle.heat_c(u, ALPHA, 6, oracle.BC_DIRICHLET)[1:-1, 1:-1, 1:-1]
+        assert np.array_equal(out[1:-1, 1:-1, 1:-1], ref)
+    else:
+        assert np.array_equal(out, oracle.heat_c(u, ALPHA, 6))
 
 
 def test_host_compute_z_slab_rank_shells_dry():
