@@ -319,7 +319,11 @@ static __device__ __forceinline__ void tma_2d(void* dst, const TensorMapBlob* ma
       : "memory");
 }
 
-template <int BY, int RPP, int S, int MB>
+// CS: a consumer thread's NR rows are consecutive (y neighbours of its inner
+// rows from its own registers) instead of RPP rows apart
+// XS: x neighbours by warp shuffle (a warp holds one 64-wide row) instead
+// of shared-memory loads
+template <int BY, int RPP, int S, int MB, bool CS = false, bool XS = false>
 __global__ void __launch_bounds__(TileCfg<BY, RPP, S>::NT + 32, MB)
     slab_sweep_tile(const ViewDev Sv, const ViewDev Dv, const __grid_constant__ SweepMaps maps, const int ny,
                     const int lo, const int hi, const double alpha, const int st_mode) {
@@ -398,6 +402,8 @@ __global__ void __launch_bounds__(TileCfg<BY, RPP, S>::NT + 32, MB)
 
   // ------------------------------------------------------- consumer warps
   const int c2 = (int)threadIdx.x % C::HALF, r0 = (int)threadIdx.x / C::HALF;
+  constexpr int RS = CS ? 1 : RPP;          // row step between a thread's rows
+  const int rb = CS ? r0 * C::NR : r0;      // its first row in the band
   const int x = 2 * c2;
   const bool xl_edge = c2 == 0, xr_edge = c2 == C::HALF - 1;
   // output stores: streaming (evict-first; 0) or kept in L2 for the next
@@ -406,7 +412,7 @@ __global__ void __launch_bounds__(TileCfg<BY, RPP, S>::NT + 32, MB)
   const uint64_t spol = stm == 2 ? policy_evict_last() : policy_evict_normal();
   // the x-halo cell of this thread's rows: left box column 1 (x = 63 of the
   // left tile), right box column 0 (x = 0 of the right tile)
-  const int hoff = xl_edge ? C::XH + 2 * r0 + 1 : C::XH + 2 * BY + 2 * r0;
+  const int hoff = xl_edge ? C::XH + 2 * rb + 1 : C::XH + 2 * BY + 2 * rb;
   uint32_t seq = 0;
   auto wait_g = [&](uint32_t g) { mbar_wait(&full[g % S], (g / S) & 1u); };
   auto release_g = [&](uint32_t g) { mbar_arrive(&empty[g % S]); };
@@ -417,18 +423,18 @@ __global__ void __launch_bounds__(TileCfg<BY, RPP, S>::NT + 32, MB)
     const int n = (int)(left < inrun ? left : inrun);
     pp += n;
     const int cx = (int)(col % ntx), y0 = (int)(col / ntx) * BY;
-    const int64_t orow = Dv.Y(y0 + r0) + Dv.X(cx * TX + x);
-    const int64_t ostep = Dv.Y(y0 + r0 + RPP) - Dv.Y(y0 + r0);  // rows of a band share a tile
+    const int64_t orow = Dv.Y(y0 + rb) + Dv.X(cx * TX + x);
+    const int64_t ostep = Dv.Y(y0 + rb + RS) - Dv.Y(y0 + rb);  // rows of a band share a tile
     double2 zm[C::NR], zc[C::NR];
     wait_g(seq);
     wait_g(seq + 1);
     {
-      const double* s0 = stage + (size_t)(seq % S) * C::STAGE + (r0 + 1) * TX + x;
-      const double* s1 = stage + (size_t)((seq + 1) % S) * C::STAGE + (r0 + 1) * TX + x;
+      const double* s0 = stage + (size_t)(seq % S) * C::STAGE + (rb + 1) * TX + x;
+      const double* s1 = stage + (size_t)((seq + 1) % S) * C::STAGE + (rb + 1) * TX + x;
 #pragma unroll
       for (int j = 0; j < C::NR; ++j) {
-        zm[j] = *reinterpret_cast<const double2*>(s0 + j * RPP * TX);
-        zc[j] = *reinterpret_cast<const double2*>(s1 + j * RPP * TX);
+        zm[j] = *reinterpret_cast<const double2*>(s0 + j * RS * TX);
+        zc[j] = *reinterpret_cast<const double2*>(s1 + j * RS * TX);
       }
     }
     release_g(seq);
@@ -438,27 +444,39 @@ __global__ void __launch_bounds__(TileCfg<BY, RPP, S>::NT + 32, MB)
     for (int i = 0; i < n; ++i) {
       wait_g(seq + i + 2);
       const double* cur = stage + (size_t)((seq + i + 1) % S) * C::STAGE;
-      const double* nxt = stage + (size_t)((seq + i + 2) % S) * C::STAGE + (r0 + 1) * TX + x;
-      const double* cc = cur + (r0 + 1) * TX + x;
+      const double* nxt = stage + (size_t)((seq + i + 2) % S) * C::STAGE + (rb + 1) * TX + x;
+      const double* cc = cur + (rb + 1) * TX + x;
+      double2 zpn[C::NR];
 #pragma unroll
       for (int j = 0; j < C::NR; ++j) {
-        const int jo = j * RPP * TX;
+        const int jo = j * RS * TX;
         const double2 zp = *reinterpret_cast<const double2*>(nxt + jo);
-        const double2 ym = *reinterpret_cast<const double2*>(cc + jo - TX);
-        const double2 yp = *reinterpret_cast<const double2*>(cc + jo + TX);
-        double xm = cc[jo - 1];
-        double xp = cc[jo + 2];
-        const double hv = cur[hoff + 2 * j * RPP];
+        zpn[j] = zp;
+        const double2 ym = CS && j > 0 ? zc[j > 0 ? j - 1 : 0] : *reinterpret_cast<const double2*>(cc + jo - TX);
+        const double2 yp =
+            CS && j < C::NR - 1 ? zc[j < C::NR - 1 ? j + 1 : 0] : *reinterpret_cast<const double2*>(cc + jo + TX);
+        const double2 c = zc[j];
+        double xm, xp;
+        if (XS) {
+          xm = __shfl_up_sync(0xffffffffu, c.y, 1);
+          xp = __shfl_down_sync(0xffffffffu, c.x, 1);
+        } else {
+          xm = cc[jo - 1];
+          xp = cc[jo + 2];
+        }
+        const double hv = cur[hoff + 2 * j * RS];
         if (xl_edge) xm = hv;
         if (xr_edge) xp = hv;
-        const double2 c = zc[j];
         double2 v;
         v.x = heat_update(c.x, xm, c.y, ym.x, yp.x, zm[j].x, zp.x, alpha);
         v.y = heat_update(c.y, c.x, xp, ym.y, yp.y, zm[j].y, zp.y, alpha);
         if (stm == 0) stg2_stream(od + j * ostep, v);
         else st2_hint(od + j * ostep, v, spol);
-        zm[j] = c;
-        zc[j] = zp;
+      }
+#pragma unroll
+      for (int j = 0; j < C::NR; ++j) {  // after the row loop: rows j+-1 read zc of this plane
+        zm[j] = zc[j];
+        zc[j] = zpn[j];
       }
       release_g(seq + i + 1);
       if (++lz == Dv.tz) {  // next tile layer (or the wrap): recompute
@@ -473,17 +491,17 @@ __global__ void __launch_bounds__(TileCfg<BY, RPP, S>::NT + 32, MB)
   }
 }
 
-template <int BY, int RPP, int S, int MB>
+template <int BY, int RPP, int S, int MB, bool CS = false, bool XS = false>
 static cudaError_t launch_tile_cfg(const ViewDev& Sv, const ViewDev& Dv, const SweepMaps& m, int nx, int ny,
                                    int lo, int hi, double alpha, int sms, cudaStream_t s) {
   using C = TileCfg<BY, RPP, S>;
   static int occ = 0;
   if (!occ) {
-    cudaError_t e = cudaFuncSetAttribute(slab_sweep_tile<BY, RPP, S, MB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(slab_sweep_tile<BY, RPP, S, MB, CS, XS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)C::SMEM);
     if (e != cudaSuccess) return e;
     int o = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, slab_sweep_tile<BY, RPP, S, MB>, C::NT + 32, C::SMEM);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, slab_sweep_tile<BY, RPP, S, MB, CS, XS>, C::NT + 32, C::SMEM);
     occ = o < 1 ? 1 : o;
   }
   const int64_t P = (int64_t)(nx / 64) * (ny / BY) * (hi - lo);
@@ -510,7 +528,7 @@ static cudaError_t launch_tile_cfg(const ViewDev& Sv, const ViewDev& Dv, const S
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = pdl ? 1 : 0;
-  return cudaLaunchKernelEx(&cfg, slab_sweep_tile<BY, RPP, S, MB>, Sv, Dv, m, ny, lo, hi, alpha, st_mode);
+  return cudaLaunchKernelEx(&cfg, slab_sweep_tile<BY, RPP, S, MB, CS, XS>, Sv, Dv, m, ny, lo, hi, alpha, st_mode);
 }
 
 // driver entry point for cuTensorMapEncodeTiled (no -lcuda link dependency)
@@ -886,7 +904,19 @@ cudaError_t launch_slab_sweep(const SlabView& src, const SlabView& dst, int nx, 
     // band 32, 4 rows per consumer thread, 5 stages, 2 CTAs per SM (band 16 or 64, 3 CTAs per SM
     // measured slower: profiles/r02/bench_sweep_cfg*.json; 4 / 5 / 6 stages at 2 CTAs per SM:
     // 0.757 / 0.768 / 0.765 of HBM on the C2 e2e step, three alternating runs)
+  {
+    // consumers: 128 threads, each one x pair of 8 consecutive rows (y
+    // neighbours of the inner rows from its registers, x neighbours by warp
+    // shuffle): 0.839 of HBM per launch against 0.791-0.795 for 256 threads
+    // of 4 rows 8 apart with shared-memory neighbours (TILES_SWEEP_CS=0),
+    // three alternating rounds
+    static const int cs = [] {
+      const char* e = getenv("TILES_SWEEP_CS");
+      return e ? atoi(e) : 1;
+    }();
+    if (cs) return launch_tile_cfg<32, 4, 5, 2, true, true>(to_dev(src), to_dev(dst), *maps, nx, ny, lo, hi, alpha, sms, s);
     return launch_tile_cfg<32, 8, 5, 2>(to_dev(src), to_dev(dst), *maps, nx, ny, lo, hi, alpha, sms, s);
+  }
   const int npairs = nx / 2;
   const int gx = (npairs + 127) / 128;
   // rows per thread: must divide every view's ty (the dense slab's is ny,
